@@ -1,0 +1,109 @@
+"""Seeded synthetic inputs for window attention — shared by tests, bench and smoke.
+
+This module holds NO arithmetic of the method (no scores, softmax or gradients):
+it only draws the random inputs and rounds them to the storage dtype.  Both the
+fp64 oracle (`oracle/`) and the CUDA path (`paper_conf_pldi_tangzwjzyz22_b200`)
+consume what it returns; neither imports the other.
+
+Recipe:
+  * numpy ``Generator(PCG64(seed))`` draws q, k, v, dout in that order, each
+    i.i.d. U(-1, 1) in fp64, shape [B, H, L, d] ("We use random
+    input for the test").
+  * The draws are rounded to the storage dtype (fp32 by numpy, bf16 by torch's
+    round-to-nearest-even), and the oracle reads the ROUNDED values upcast
+    exactly to fp64, so parity measures kernel error, not input quantisation.
+  * ``q_scale`` multiplies q before rounding (the x16 "overflow probe").
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+__all__ = ["WinAttnShape", "CONFIGS", "make_inputs", "round_to", "TORCH_DTYPES"]
+
+
+@dataclass(frozen=True)
+class WinAttnShape:
+    batch: int
+    heads: int
+    seq_len: int
+    d: int
+    w: int
+    dilation: int = 1
+
+    @property
+    def units(self) -> int:
+        return self.batch * self.heads
+
+    @property
+    def rows(self) -> int:
+        return self.batch * self.heads * self.seq_len
+
+
+# Named configurations (BASELINE.json "configs").
+CONFIGS = {
+    # configs[0]: tiny, oracle fwd+bwd + finite differences in seconds.
+    "C1": WinAttnShape(1, 1, 64, 16, 4, 1),
+    # configs[1]/[2]: Longformer-shaped, reading A14(a) of the FreeTensor artefact
+    # (n_heads=8, seq_len=10000, feat_len=512, w=32).
+    "C2a": WinAttnShape(1, 8, 10000, 512, 32, 1),
+    # the artefact's dilated heads (heads 0-1 use dilation 4), run as its own call.
+    "C2a_dil": WinAttnShape(1, 2, 10000, 512, 32, 4),
+    # Longformer-base shape, reading A14(b).
+    "C2b": WinAttnShape(1, 12, 4096, 64, 256, 1),
+    # configs[3]: dilated, large window, 16K tokens.
+    "C4d2": WinAttnShape(1, 12, 16384, 64, 256, 2),
+    "C4d4": WinAttnShape(1, 12, 16384, 64, 256, 4),
+    # configs[4]: sweep corners (H in {8..64}, L in {4K..32K}, w in {32, 256}).
+    "C5_small_w32": WinAttnShape(1, 8, 4096, 64, 32, 1),
+    "C5_big_w32": WinAttnShape(1, 64, 32768, 64, 32, 1),
+    "C5_big_w256": WinAttnShape(1, 64, 32768, 64, 256, 1),
+}
+
+
+def _torch():
+    import torch  # local import: the oracle tests must not need CUDA
+
+    return torch
+
+
+TORCH_DTYPES = ("f32", "bf16")
+
+
+def round_to(x: np.ndarray, dtype: str):
+    """Round fp64 ``x`` to the storage dtype.
+
+    Returns ``(torch_tensor_in_dtype, fp64_numpy_of_the_rounded_values)``.
+    The fp64 copy is exact (both f32 and bf16 embed in fp64).
+    """
+    torch = _torch()
+    t64 = torch.from_numpy(np.ascontiguousarray(x))
+    if dtype == "f32":
+        t = t64.to(torch.float32)
+    elif dtype == "bf16":
+        t = t64.to(torch.bfloat16)  # round-to-nearest-even
+    else:
+        raise ValueError(f"unknown dtype {dtype!r}")
+    return t.contiguous(), t.to(torch.float64).numpy()
+
+
+def make_inputs(shape: WinAttnShape, seed: int, dtype: str = "f32", q_scale: float = 1.0,
+                with_dout: bool = True):
+    """Draw q, k, v (and dout) for ``shape``.
+
+    Returns a dict with torch tensors (CPU, storage dtype) under 'q','k','v','dout'
+    and their exact fp64 numpy copies under 'q64','k64','v64','dout64'.
+    """
+    rng = np.random.Generator(np.random.PCG64(seed))
+    dims = (shape.batch, shape.heads, shape.seq_len, shape.d)
+    out = {}
+    names = ["q", "k", "v"] + (["dout"] if with_dout else [])
+    for name in names:
+        x = rng.uniform(-1.0, 1.0, size=dims)
+        if name == "q" and q_scale != 1.0:
+            x = x * q_scale
+        t, x64 = round_to(x, dtype)
+        out[name] = t
+        out[name + "64"] = x64
+    return out
