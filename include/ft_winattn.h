@@ -1,0 +1,114 @@
+/* include/ft_winattn.h -- C ABI of the B200 (sm_100a) banded window-attention library.
+ *
+ * The operation is the hot path of FreeTensor's Longformer workload (PAPER.md:58
+ * "computes correlations for pairs of nearby tokens that have a distance no greater
+ * than a threshold"; Fig. 5 caption PAPER.md:172 "The range j-w to j+w marks the
+ * sliding window"; the inlined program Fig. 8).  Each query row i
+ * of every (batch, head) unit attends to the window
+ *
+ *     N(i) = { j = i + k*dilation : |k| <= w, 0 <= j < seq_len }
+ *
+ * (inclusive window, reading A1; out-of-sequence keys excluded, reading A2;
+ * dilation as in Longformer [8], reading A4).  No logit scale is applied
+ * (Fig. 8 "dot[k+w] += Q[j,p] * K[j+k,p]", reading A3): callers pre-scale q.
+ *
+ *   forward:
+ *     s_ij  = sum_p q_ip k_jp,  lse_i = log sum_{j in N(i)} exp(s_ij),
+ *     out_i = sum_{j in N(i)} exp(s_ij - lse_i) v_j
+ *   backward  (the gradient program of PAPER.md:447-453, P recomputed from lse as in
+ *              PAPER.md:489-497 "selective materialization", reading A6):
+ *     D_i = dout_i . out_i,  P_ij = exp(s_ij - lse_i),  dS_ij = P_ij (dout_i . v_j - D_i)
+ *     dq_i = sum_j dS_ij k_j,  dk_j = sum_i dS_ij q_i,  dv_j = sum_i P_ij dout_i
+ *
+ * Layout (reading A9): q, k, v, out, dout, dq, dk, dv are contiguous row-major
+ * [batch, heads, seq_len, d] in the storage dtype; lse is contiguous fp32
+ * [batch, heads, seq_len] (natural log).  All pointers are DEVICE pointers.
+ *
+ * Ownership: the caller owns every buffer (including the workspace).  The library
+ * never allocates, frees, synchronises or copies host<->device.  Outputs are fully
+ * overwritten, never accumulated into.
+ *
+ * Async: work is enqueued on `stream` (a cudaStream_t passed as void*; NULL = legacy
+ * default stream) and the call returns immediately.
+ *
+ * Errors: all argument checks run before any launch; on failure nothing is launched
+ * and the outputs are untouched.
+ *   FT_ERR_INVALID_VALUE  null pointer; batch, heads, seq_len or d < 1; w < 0;
+ *                         dilation < 1; an output buffer overlapping an input or
+ *                         another output; workspace smaller than required.
+ *   FT_ERR_MISALIGNED     a tensor pointer not 16-byte aligned.
+ *   FT_ERR_NOT_SUPPORTED  d not a multiple of 16 or d > 512; unknown dtype;
+ *                         seq_len * d or batch * heads too large for 31-bit tiling.
+ *   FT_ERR_CUDA           a CUDA launch failed (cudaGetLastError after the launch).
+ * Domain: any w >= 0 (w >= seq_len is full attention), any dilation >= 1.
+ * Thread safety: stateless; safe to call concurrently from several host threads.
+ */
+#ifndef FT_WINATTN_H
+#define FT_WINATTN_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FT_WINATTN_ABI_VERSION 1
+
+typedef enum {
+    FT_OK = 0,
+    FT_ERR_INVALID_VALUE = 1,
+    FT_ERR_NOT_SUPPORTED = 2,
+    FT_ERR_MISALIGNED = 3,
+    FT_ERR_CUDA = 4
+} ft_status;
+
+typedef enum { FT_F32 = 0, FT_BF16 = 1 } ft_dtype;
+
+/* Kernel family chosen for a call (reported by ft_winattn_plan; tests may force one
+ * through the environment variable FT_WINATTN_PATH=simt|tc). */
+typedef enum {
+    FT_PATH_SIMT = 0,   /* CUDA-core FMA kernels (fp32 math), any dtype / d / w      */
+    FT_PATH_TC = 1      /* tcgen05/TMEM tensor-core kernels, bf16 only               */
+} ft_path;
+
+/* Forward.  q, k, v: [B,H,L,d] dtype (inputs).  out: [B,H,L,d] dtype, lse: [B,H,L]
+ * fp32 (outputs).  w: one-sided window (keys per side), dilation: key stride. */
+ft_status ft_winattn_fwd(const void* q, const void* k, const void* v,
+                         void* out, float* lse,
+                         int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                         int64_t w, int64_t dilation, ft_dtype dtype, void* stream);
+
+/* Backward.  q, k, v, out (the forward's output), lse (the forward's lse) and dout
+ * are inputs; dq, dk, dv ([B,H,L,d] dtype) are overwritten.  workspace must hold at
+ * least ft_winattn_bwd_workspace_bytes(...) bytes of device memory (16-byte aligned;
+ * may be NULL when that size is 0); its contents on entry are ignored. */
+ft_status ft_winattn_bwd(const void* q, const void* k, const void* v,
+                         const void* out, const float* lse, const void* dout,
+                         void* dq, void* dk, void* dv,
+                         int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                         int64_t w, int64_t dilation, ft_dtype dtype,
+                         void* workspace, size_t workspace_bytes, void* stream);
+
+/* Device workspace the backward needs (the per-row D_i = dout_i . out_i, fp32). */
+size_t ft_winattn_bwd_workspace_bytes(int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                                      int64_t w, int64_t dilation, ft_dtype dtype);
+
+/* Describe what a call would launch, without launching: the kernel family and the
+ * number of kernel launches of the forward (is_bwd = 0) or backward (is_bwd = 1).
+ * Returns the same validation status the real call would for its scalar arguments. */
+ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                          int64_t w, int64_t dilation, ft_dtype dtype,
+                          int* path, int* num_launches);
+
+/* Human-readable text for a status (static storage, never NULL).  For FT_ERR_CUDA it
+ * includes the CUDA error string of the last failure on the calling thread. */
+const char* ft_status_str(ft_status s);
+
+/* ABI version of the loaded library (FT_WINATTN_ABI_VERSION it was built with). */
+int ft_winattn_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FT_WINATTN_H */

@@ -1,0 +1,178 @@
+"""B200-native banded (dilated) sliding-window attention — Python binding of ft_winattn.
+
+The compute lives in ``libft_winattn.so`` (hand-written sm_100a CUDA kernels behind the
+C ABI of ``include/ft_winattn.h``).  This module only marshals arguments: it checks
+dtype / device / contiguity, allocates outputs with PyTorch and calls the C entry points
+through ctypes on ``torch.cuda.current_stream()``.  There is no CPU or PyTorch fallback:
+if the library is missing or a call fails, it raises.
+
+Operation (Fig. 5/8, lines 167-231): for each (batch, head) and
+query row i, attend to keys j = i + k*dilation with |k| <= w and 0 <= j < L, unscaled
+logits q_i.k_j, row softmax with saved log-sum-exp, weighted sum over V; the backward
+recomputes P from lse and returns dq, dk, dv.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+__all__ = ["fwd", "bwd", "plan", "WinAttn", "win_attn", "lib_path", "load_library",
+           "FT_F32", "FT_BF16", "PATH_SIMT", "PATH_TC", "FtError"]
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+_LIB_NAME = "libft_winattn.so"
+
+FT_F32, FT_BF16 = 0, 1
+PATH_SIMT, PATH_TC = 0, 1
+_STATUS = {0: "FT_OK", 1: "FT_ERR_INVALID_VALUE", 2: "FT_ERR_NOT_SUPPORTED",
+           3: "FT_ERR_MISALIGNED", 4: "FT_ERR_CUDA"}
+
+_lib = None
+
+
+class FtError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(msg)
+        self.status = status
+
+
+def lib_path() -> str:
+    return os.path.join(_PKG, _LIB_NAME)
+
+
+def load_library(build_if_missing: bool = False):
+    """Load (optionally build) the in-tree shared library and declare its C signatures."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    path = lib_path()
+    if not os.path.exists(path):
+        if not build_if_missing:
+            raise RuntimeError(f"{path} is missing: build it with "
+                               "`python -m paper_conf_pldi_tangzwjzyz22_b200.build`")
+        from . import build as _build
+        _build.build()
+    lib = ctypes.CDLL(path)
+    i64, vp, sz = ctypes.c_int64, ctypes.c_void_p, ctypes.c_size_t
+    fp = ctypes.c_void_p
+    lib.ft_winattn_fwd.argtypes = [vp, vp, vp, vp, fp] + [i64] * 6 + [ctypes.c_int, vp]
+    lib.ft_winattn_fwd.restype = ctypes.c_int
+    lib.ft_winattn_bwd.argtypes = [vp] * 9 + [i64] * 6 + [ctypes.c_int, vp, sz, vp]
+    lib.ft_winattn_bwd.restype = ctypes.c_int
+    lib.ft_winattn_bwd_workspace_bytes.argtypes = [i64] * 6 + [ctypes.c_int]
+    lib.ft_winattn_bwd_workspace_bytes.restype = sz
+    lib.ft_winattn_plan.argtypes = [ctypes.c_int] + [i64] * 6 + [ctypes.c_int,
+                                                                 ctypes.POINTER(ctypes.c_int),
+                                                                 ctypes.POINTER(ctypes.c_int)]
+    lib.ft_winattn_plan.restype = ctypes.c_int
+    lib.ft_status_str.argtypes = [ctypes.c_int]
+    lib.ft_status_str.restype = ctypes.c_char_p
+    lib.ft_winattn_abi_version.restype = ctypes.c_int
+    _lib = lib
+    return lib
+
+
+def _dtype_code(t: torch.Tensor) -> int:
+    if t.dtype == torch.float32:
+        return FT_F32
+    if t.dtype == torch.bfloat16:
+        return FT_BF16
+    raise TypeError(f"unsupported dtype {t.dtype} (expected float32 or bfloat16)")
+
+
+def _check(status: int):
+    if status != 0:
+        msg = load_library().ft_status_str(status).decode()
+        raise FtError(status, msg)
+
+
+def _check_inputs(*ts: torch.Tensor):
+    ref = ts[0]
+    if ref.dim() != 4:
+        raise ValueError("expected [batch, heads, seq_len, d] tensors")
+    for t in ts:
+        if not t.is_cuda:
+            raise ValueError("ft_winattn tensors must be CUDA tensors")
+        if t.shape != ref.shape or t.dtype != ref.dtype or t.device != ref.device:
+            raise ValueError("q, k, v (and out, dout) must share shape, dtype and device")
+        if not t.is_contiguous():
+            raise ValueError("ft_winattn tensors must be contiguous")
+
+
+def _stream(device) -> int:
+    return torch.cuda.current_stream(device).cuda_stream
+
+
+def plan(is_bwd: bool, batch: int, heads: int, seq_len: int, d: int, w: int, dilation: int,
+         dtype) -> tuple[int, int]:
+    """(path, number of kernel launches) a call with these arguments would make."""
+    code = dtype if isinstance(dtype, int) else (FT_F32 if dtype == torch.float32 else FT_BF16)
+    path, n = ctypes.c_int(0), ctypes.c_int(0)
+    _check(load_library().ft_winattn_plan(int(is_bwd), batch, heads, seq_len, d, w, dilation,
+                                          code, ctypes.byref(path), ctypes.byref(n)))
+    return path.value, n.value
+
+
+def fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, w: int, dilation: int = 1,
+        out: torch.Tensor | None = None, lse: torch.Tensor | None = None):
+    """Forward: returns (out [B,H,L,d] in q.dtype, lse [B,H,L] fp32)."""
+    _check_inputs(q, k, v)
+    B, H, L, d = q.shape
+    if out is None:
+        out = torch.empty_like(q)
+    if lse is None:
+        lse = torch.empty((B, H, L), dtype=torch.float32, device=q.device)
+    _check(load_library().ft_winattn_fwd(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(),
+                                         lse.data_ptr(), B, H, L, d, int(w), int(dilation),
+                                         _dtype_code(q), _stream(q.device)))
+    return out, lse
+
+
+def workspace_bytes(q: torch.Tensor, w: int, dilation: int = 1) -> int:
+    B, H, L, d = q.shape
+    return int(load_library().ft_winattn_bwd_workspace_bytes(B, H, L, d, int(w), int(dilation),
+                                                             _dtype_code(q)))
+
+
+def bwd(q, k, v, out, lse, dout, w: int, dilation: int = 1, dq=None, dk=None, dv=None,
+        workspace: torch.Tensor | None = None):
+    """Backward: returns (dq, dk, dv) in q.dtype."""
+    _check_inputs(q, k, v, out, dout)
+    B, H, L, d = q.shape
+    if lse.dtype != torch.float32 or not lse.is_contiguous() or lse.shape != (B, H, L):
+        raise ValueError("lse must be a contiguous fp32 [B, H, L] tensor")
+    dq = torch.empty_like(q) if dq is None else dq
+    dk = torch.empty_like(q) if dk is None else dk
+    dv = torch.empty_like(q) if dv is None else dv
+    wsb = workspace_bytes(q, w, dilation)
+    if workspace is None or workspace.numel() * workspace.element_size() < wsb:
+        workspace = torch.empty(max(wsb, 16), dtype=torch.uint8, device=q.device)
+    _check(load_library().ft_winattn_bwd(
+        q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), lse.data_ptr(), dout.data_ptr(),
+        dq.data_ptr(), dk.data_ptr(), dv.data_ptr(), B, H, L, d, int(w), int(dilation),
+        _dtype_code(q), workspace.data_ptr(), workspace.numel() * workspace.element_size(),
+        _stream(q.device)))
+    return dq, dk, dv
+
+
+class WinAttn(torch.autograd.Function):
+    """autograd wrapper: saves (q, k, v, out, lse); backward recomputes P from lse."""
+
+    @staticmethod
+    def forward(ctx, q, k, v, w: int, dilation: int = 1):
+        out, lse = fwd(q.contiguous(), k.contiguous(), v.contiguous(), w, dilation)
+        ctx.save_for_backward(q, k, v, out, lse)
+        ctx.w, ctx.dilation = w, dilation
+        return out
+
+    @staticmethod
+    def backward(ctx, dout):
+        q, k, v, out, lse = ctx.saved_tensors
+        dq, dk, dv = bwd(q, k, v, out, lse, dout.contiguous(), ctx.w, ctx.dilation)
+        return dq, dk, dv, None, None
+
+
+def win_attn(q, k, v, w: int, dilation: int = 1):
+    return WinAttn.apply(q, k, v, w, dilation)

@@ -1,0 +1,194 @@
+// api.cu -- the extern "C" boundary of ft_winattn (declared and documented in
+// include/ft_winattn.h): argument validation, kernel-family selection, dispatch.
+//
+// The library is stateless: it never allocates, frees, synchronises or copies between
+// host and device.  Every check runs before the first launch, so a failing call leaves
+// the outputs untouched.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include "ft_winattn.h"
+#include "internal.h"
+
+namespace {
+
+thread_local char g_cuda_msg[256] = "CUDA error";
+
+ft_status cuda_fail(cudaError_t e) {
+    snprintf(g_cuda_msg, sizeof(g_cuda_msg), "FT_ERR_CUDA: %s (%s)", cudaGetErrorName(e),
+             cudaGetErrorString(e));
+    return FT_ERR_CUDA;
+}
+
+size_t elt_size(ft_dtype dt) { return dt == FT_F32 ? 4 : 2; }
+
+ft_status check_scalars(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                        ft_dtype dt) {
+    if (B < 1 || H < 1 || L < 1 || d < 1 || w < 0 || dil < 1) return FT_ERR_INVALID_VALUE;
+    if (dt != FT_F32 && dt != FT_BF16) return FT_ERR_NOT_SUPPORTED;
+    if (d % 16 != 0 || d > 512) return FT_ERR_NOT_SUPPORTED;
+    // Tiling uses 31-bit row indices inside a (unit, residue) and a 1-D grid of CTAs.
+    if (L > (int64_t)1 << 30 || B * H > (int64_t)1 << 30) return FT_ERR_NOT_SUPPORTED;
+    const int64_t nres = dil < L ? dil : L;
+    const int64_t tiles = ftw::ceil_div(ftw::ceil_div(L, dil), 32);
+    if ((double)B * H * nres * tiles > 2147483647.0) return FT_ERR_NOT_SUPPORTED;
+    return FT_OK;
+}
+
+bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+struct Span {
+    uintptr_t lo, hi;
+};
+bool overlap(Span a, Span b) { return a.lo < b.hi && b.lo < a.hi; }
+
+// 0 = auto, 1 = force SIMT, 2 = force tensor cores (test-only override).
+int forced_path() {
+    const char* s = getenv("FT_WINATTN_PATH");
+    if (!s || !*s) return 0;
+    if (!strcmp(s, "simt")) return 1;
+    if (!strcmp(s, "tc")) return 2;
+    return 0;
+}
+
+ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil, ft_dtype dt,
+                      int* path) {
+    const bool tc_ok = dt == FT_BF16 && (is_bwd ? ftw::tc_bwd_supported(units, L, d, w, dil)
+                                                : ftw::tc_fwd_supported(units, L, d, w, dil));
+    const int f = forced_path();
+    if (f == 1) { *path = FT_PATH_SIMT; return FT_OK; }
+    if (f == 2) {
+        if (!tc_ok) return FT_ERR_NOT_SUPPORTED;
+        *path = FT_PATH_TC;
+        return FT_OK;
+    }
+    *path = tc_ok ? FT_PATH_TC : FT_PATH_SIMT;
+    return FT_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int ft_winattn_abi_version(void) { return FT_WINATTN_ABI_VERSION; }
+
+const char* ft_status_str(ft_status s) {
+    switch (s) {
+        case FT_OK: return "FT_OK";
+        case FT_ERR_INVALID_VALUE: return "FT_ERR_INVALID_VALUE: invalid argument";
+        case FT_ERR_NOT_SUPPORTED: return "FT_ERR_NOT_SUPPORTED: unsupported dtype / head dim / size";
+        case FT_ERR_MISALIGNED: return "FT_ERR_MISALIGNED: tensor pointer not 16-byte aligned";
+        case FT_ERR_CUDA: return g_cuda_msg;
+    }
+    return "unknown ft_status";
+}
+
+size_t ft_winattn_bwd_workspace_bytes(int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                                      int64_t w, int64_t dilation, ft_dtype dtype) {
+    if (check_scalars(batch, heads, seq_len, d, w, dilation, dtype) != FT_OK) return 0;
+    // D_i = dout_i . out_i for every row, fp32, rounded up to 256 bytes.
+    const size_t rows = (size_t)(batch * heads * seq_len);
+    return ((rows * sizeof(float) + 255) / 256) * 256;
+}
+
+ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                          int64_t w, int64_t dilation, ft_dtype dtype, int* path,
+                          int* num_launches) {
+    ft_status s = check_scalars(batch, heads, seq_len, d, w, dilation, dtype);
+    if (s != FT_OK) return s;
+    int p = 0;
+    s = choose_path(is_bwd, batch * heads, seq_len, d, w, dilation, dtype, &p);
+    if (s != FT_OK) return s;
+    int n;
+    if (p == FT_PATH_TC)
+        n = is_bwd ? ftw::tc_bwd_launches(seq_len, d, w, dilation)
+                   : ftw::tc_fwd_launches(seq_len, d, w, dilation);
+    else
+        n = is_bwd ? ftw::simt_bwd_launches() : ftw::simt_fwd_launches();
+    if (path) *path = p;
+    if (num_launches) *num_launches = n;
+    return FT_OK;
+}
+
+ft_status ft_winattn_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
+                         int64_t batch, int64_t heads, int64_t seq_len, int64_t d, int64_t w,
+                         int64_t dilation, ft_dtype dtype, void* stream) {
+    if (!q || !k || !v || !out || !lse) return FT_ERR_INVALID_VALUE;
+    ft_status s = check_scalars(batch, heads, seq_len, d, w, dilation, dtype);
+    if (s != FT_OK) return s;
+    if (!aligned16(q) || !aligned16(k) || !aligned16(v) || !aligned16(out) || !aligned16(lse))
+        return FT_ERR_MISALIGNED;
+    const size_t nb = (size_t)(batch * heads * seq_len * d) * elt_size(dtype);
+    const size_t lb = (size_t)(batch * heads * seq_len) * sizeof(float);
+    const Span in[3] = {{(uintptr_t)q, (uintptr_t)q + nb}, {(uintptr_t)k, (uintptr_t)k + nb},
+                        {(uintptr_t)v, (uintptr_t)v + nb}};
+    const Span so = {(uintptr_t)out, (uintptr_t)out + nb}, sl = {(uintptr_t)lse, (uintptr_t)lse + lb};
+    if (overlap(so, sl)) return FT_ERR_INVALID_VALUE;
+    for (const Span& x : in)
+        if (overlap(x, so) || overlap(x, sl)) return FT_ERR_INVALID_VALUE;
+    int path = 0;
+    s = choose_path(0, batch * heads, seq_len, d, w, dilation, dtype, &path);
+    if (s != FT_OK) return s;
+
+    cudaStream_t st = (cudaStream_t)stream;
+    cudaError_t e;
+    if (path == FT_PATH_TC) {
+        int n = 0;
+        e = ftw::tc_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, st, &n);
+    } else {
+        e = ftw::simt_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype, st);
+    }
+    return e == cudaSuccess ? FT_OK : cuda_fail(e);
+}
+
+ft_status ft_winattn_bwd(const void* q, const void* k, const void* v, const void* out,
+                         const float* lse, const void* dout, void* dq, void* dk, void* dv,
+                         int64_t batch, int64_t heads, int64_t seq_len, int64_t d, int64_t w,
+                         int64_t dilation, ft_dtype dtype, void* workspace,
+                         size_t workspace_bytes, void* stream) {
+    if (!q || !k || !v || !out || !lse || !dout || !dq || !dk || !dv) return FT_ERR_INVALID_VALUE;
+    ft_status s = check_scalars(batch, heads, seq_len, d, w, dilation, dtype);
+    if (s != FT_OK) return s;
+    const size_t need = ft_winattn_bwd_workspace_bytes(batch, heads, seq_len, d, w, dilation, dtype);
+    if (workspace_bytes < need || (need > 0 && !workspace)) return FT_ERR_INVALID_VALUE;
+    const void* ptrs[] = {q, k, v, out, lse, dout, dq, dk, dv, workspace};
+    for (const void* p : ptrs)
+        if (p && !aligned16(p)) return FT_ERR_MISALIGNED;
+    const size_t nb = (size_t)(batch * heads * seq_len * d) * elt_size(dtype);
+    const size_t lb = (size_t)(batch * heads * seq_len) * sizeof(float);
+    const Span ins[6] = {{(uintptr_t)q, (uintptr_t)q + nb},     {(uintptr_t)k, (uintptr_t)k + nb},
+                         {(uintptr_t)v, (uintptr_t)v + nb},     {(uintptr_t)out, (uintptr_t)out + nb},
+                         {(uintptr_t)lse, (uintptr_t)lse + lb}, {(uintptr_t)dout, (uintptr_t)dout + nb}};
+    const Span outs[4] = {{(uintptr_t)dq, (uintptr_t)dq + nb},
+                          {(uintptr_t)dk, (uintptr_t)dk + nb},
+                          {(uintptr_t)dv, (uintptr_t)dv + nb},
+                          {(uintptr_t)workspace, (uintptr_t)workspace + need}};
+    for (int a = 0; a < 4; ++a) {
+        if (outs[a].hi == outs[a].lo) continue;
+        for (const Span& x : ins)
+            if (overlap(outs[a], x)) return FT_ERR_INVALID_VALUE;
+        for (int b = a + 1; b < 4; ++b)
+            if (outs[b].hi != outs[b].lo && overlap(outs[a], outs[b])) return FT_ERR_INVALID_VALUE;
+    }
+    int path = 0;
+    s = choose_path(1, batch * heads, seq_len, d, w, dilation, dtype, &path);
+    if (s != FT_OK) return s;
+
+    cudaStream_t st = (cudaStream_t)stream;
+    float* Dws = (float*)workspace;
+    cudaError_t e;
+    if (path == FT_PATH_TC) {
+        int n = 0;
+        e = ftw::tc_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w,
+                        dilation, st, &n);
+    } else {
+        e = ftw::simt_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w,
+                          dilation, dtype, st);
+    }
+    return e == cudaSuccess ? FT_OK : cuda_fail(e);
+}
+
+}  // extern "C"

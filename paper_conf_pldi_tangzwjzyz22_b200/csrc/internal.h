@@ -1,0 +1,72 @@
+// internal.h -- shared launch-side declarations of the ft_winattn library (not part of the ABI).
+//
+// Geometry: every (batch, head) unit u and dilation residue r (0 <= r < min(dilation, L))
+// forms an independent dilation-1 band problem on the strided rows i = r + m*dilation,
+// m in [0, Lr), Lr = ceil((L - r) / dilation)  (reading A4; the oracle pins the
+// equivalence in tests/test_oracle.py::test_dilation_is_residue_decomposition).
+// Kernels tile m ("residue space"), so dilation costs only an address stride.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "ft_winattn.h"
+
+namespace ftw {
+
+struct Geo {
+    int64_t L;        // seq_len
+    int64_t d;        // head dim
+    int64_t w;        // one-sided window, clamped to L (|k| >= L never hits the sequence)
+    int64_t dil;      // dilation
+    int64_t units;    // batch * heads
+    int64_t nres;     // min(dil, L) non-empty residues
+    int64_t tiles;    // tiles per residue = ceil(ceil(L / dil) / T)
+    int T;            // rows per tile
+};
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+inline Geo make_geo(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, int T) {
+    Geo g;
+    g.L = L;
+    g.d = d;
+    g.w = w < L ? w : L;
+    g.dil = dil;
+    g.units = B * H;
+    g.nres = dil < L ? dil : L;
+    g.tiles = ceil_div(ceil_div(L, dil), T);
+    g.T = T;
+    return g;
+}
+
+inline int64_t geo_blocks(const Geo& g) { return g.units * g.nres * g.tiles; }
+
+// SIMT (CUDA-core) kernels -- simt.cu
+cudaError_t simt_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
+                     int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                     ft_dtype dt, cudaStream_t st);
+cudaError_t simt_bwd(const void* q, const void* k, const void* v, const void* out,
+                     const float* lse, const void* dout, void* dq, void* dk, void* dv,
+                     float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
+                     int64_t dil, ft_dtype dt, cudaStream_t st);
+int simt_fwd_launches();
+int simt_bwd_launches();
+
+// tcgen05 / TMEM kernels -- tc_fwd.cu, tc_bwd.cu (bf16 only)
+bool tc_fwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+bool tc_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
+                   int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                   cudaStream_t st, int* launches);
+cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
+                   const float* lse, const void* dout, void* dq, void* dk, void* dv,
+                   float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
+                   int64_t dil, cudaStream_t st, int* launches);
+int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
+int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
+
+// D_i = dout_i . out_i pre-pass shared by both backward families -- simt.cu
+cudaError_t launch_rowdot(const void* dout, const void* out, float* D, int64_t rows, int64_t d,
+                          ft_dtype dt, cudaStream_t st);
+
+}  // namespace ftw

@@ -1,0 +1,586 @@
+// simt.cu -- CUDA-core (FMA) window-attention kernels for sm_100a: fp32 math for fp32 or
+// bf16 storage, any d (multiple of 16, <= 512), any w, any dilation.
+//
+// Tiling follows the paper's redundancy-free formulation (keys are
+// indexed directly as j+k, never copied (2w+1)-fold).  A CTA owns a tile of T rows of one
+// (unit, residue) band problem and streams only the key chunks that intersect its band
+// [m0 - w, m0 + T - 1 + w]: the "cache a[i:i+m]" of PAPER.md Fig. 14 (lines 402-423) is the
+// per-chunk K/V staging in shared memory.  Scores and the running row max are produced in
+// one pass (the dot/max fusion of Fig. 10); the normalisation uses the
+// online-softmax rewrite so the dot_max dependence does not force a second
+// sweep.  The backward recomputes P from the saved lse (selective materialization,
+// PAPER.md:489-497) and writes dq (query-major kernel) and dk/dv (key-major kernel) each
+// from exactly one CTA: no atomics, deterministic (the Fig. 13(d) parallel-reduction
+// choice rather than Fig. 13(e) atomics).
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <mutex>
+
+#include "internal.h"
+
+namespace ftw {
+namespace {
+
+constexpr int NT = 256;      // threads per CTA (16 x 16 thread grid)
+constexpr int C = 64;        // key (or query) chunk per step
+constexpr int DS = 32;       // d-slice staged per step
+constexpr int SP = DS + 1;   // padded slice row (bank-conflict free column reads)
+constexpr float LOG2E = 1.4426950408889634f;
+constexpr float LN2 = 0.6931471805599453f;
+
+template <typename T> struct Vec;
+template <> struct Vec<float> {
+    static constexpr int N = 4;
+    __device__ static void load(const float* p, float* o) {
+        float4 x = __ldg(reinterpret_cast<const float4*>(p));
+        o[0] = x.x; o[1] = x.y; o[2] = x.z; o[3] = x.w;
+    }
+    __device__ static void store1(float* p, float x) { *p = x; }
+    __device__ static float to_f(float x) { return x; }
+};
+template <> struct Vec<__nv_bfloat16> {
+    static constexpr int N = 8;
+    __device__ static void load(const __nv_bfloat16* p, float* o) {
+        uint4 x = __ldg(reinterpret_cast<const uint4*>(p));
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&x);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+            float2 f = __bfloat1622float2(h[e]);
+            o[2 * e] = f.x; o[2 * e + 1] = f.y;
+        }
+    }
+    __device__ static void store1(__nv_bfloat16* p, float x) { *p = __float2bfloat16_rn(x); }
+    __device__ static float to_f(__nv_bfloat16 x) { return __bfloat162float(x); }
+};
+
+// Stage rows [mbase, mbase+R) x cols [col0, col0+DS) of a strided band view into dst[R][SP].
+// Rows outside [0, Lr) and columns >= d read as zero.
+template <typename Tin, int R>
+__device__ __forceinline__ void load_slice(float (*dst)[SP], const Tin* __restrict__ base,
+                                           int64_t rstride, int mbase, int Lr, int col0, int d) {
+    constexpr int V = Vec<Tin>::N;
+    constexpr int NV = DS / V;
+    for (int idx = threadIdx.x; idx < R * NV; idx += NT) {
+        const int row = idx / NV, cv = idx % NV;
+        const int m = mbase + row, c = col0 + cv * V;
+        float vals[V];
+        if (m >= 0 && m < Lr && c < d) {
+            Vec<Tin>::load(base + (int64_t)m * rstride + c, vals);
+        } else {
+#pragma unroll
+            for (int e = 0; e < V; ++e) vals[e] = 0.f;
+        }
+#pragma unroll
+        for (int e = 0; e < V; ++e) dst[row][cv * V + e] = vals[e];
+    }
+}
+
+struct TileCoord {
+    int64_t u, r;
+    int Lr, m0;
+    int64_t off;       // element offset of row m=0 of this (unit, residue)
+    int64_t rstride;   // element stride between consecutive m
+    int64_t row0;      // flat row id (u*L + r) of m=0; flat(m) = row0 + m*dil
+};
+
+__device__ __forceinline__ bool decode(const Geo& g, TileCoord& c) {
+    int64_t b = blockIdx.x;
+    const int64_t t = b % g.tiles;
+    b /= g.tiles;
+    c.r = b % g.nres;
+    c.u = b / g.nres;
+    c.Lr = (int)((g.L - c.r + g.dil - 1) / g.dil);
+    c.m0 = (int)t * g.T;
+    c.off = (c.u * g.L + c.r) * g.d;
+    c.rstride = g.dil * g.d;
+    c.row0 = c.u * g.L + c.r;
+    return c.m0 < c.Lr;
+}
+
+__device__ __forceinline__ float hmax16(float x) {
+#pragma unroll
+    for (int o = 8; o >= 1; o >>= 1) x = fmaxf(x, __shfl_xor_sync(0xffffffffu, x, o));
+    return x;
+}
+__device__ __forceinline__ float hsum16(float x) {
+#pragma unroll
+    for (int o = 8; o >= 1; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+    return x;
+}
+
+// ------------------------------------------------------------------------------ forward
+template <typename Tin>
+__global__ void __launch_bounds__(NT) simt_fwd_kernel(const Tin* __restrict__ q,
+                                                      const Tin* __restrict__ k,
+                                                      const Tin* __restrict__ v,
+                                                      Tin* __restrict__ out, float* __restrict__ lse,
+                                                      Geo g) {
+    constexpr int T = 64, RA = T / 16;
+    extern __shared__ float smem[];
+    float(*Qs)[SP] = reinterpret_cast<float(*)[SP]>(smem);
+    float(*Ks)[SP] = Qs + T;                                   // K slice, then V slice
+    float(*Ps)[C + 1] = reinterpret_cast<float(*)[C + 1]>(Ks + C);
+    float* Os = reinterpret_cast<float*>(Ps + T);              // T x d accumulator
+    float* rowM = Os + T * g.d;
+    float* rowL = rowM + T;
+
+    TileCoord tc;
+    if (!decode(g, tc)) return;
+    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
+    const Tin* Qb = q + tc.off;
+    const Tin* Kb = k + tc.off;
+    const Tin* Vb = v + tc.off;
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+
+    for (int i = threadIdx.x; i < T * d; i += NT) Os[i] = 0.f;
+    float mrow[RA], lrow[RA];
+#pragma unroll
+    for (int a = 0; a < RA; ++a) { mrow[a] = -INFINITY; lrow[a] = 0.f; }
+
+    const int kbeg = max(0, m0 - w);
+    const int kend = min(Lr, m0 + T + w);
+    for (int c0 = kbeg; c0 < kend; c0 += C) {
+        float s[RA][4];
+#pragma unroll
+        for (int a = 0; a < RA; ++a)
+#pragma unroll
+            for (int b = 0; b < 4; ++b) s[a][b] = 0.f;
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            load_slice<Tin, T>(Qs, Qb, tc.rstride, m0, Lr, col0, d);
+            load_slice<Tin, C>(Ks, Kb, tc.rstride, c0, kend, col0, d);
+            __syncthreads();
+#pragma unroll 8
+            for (int p = 0; p < DS; ++p) {
+                float qa[RA], kb[4];
+#pragma unroll
+                for (int a = 0; a < RA; ++a) qa[a] = Qs[ty + 16 * a][p];
+#pragma unroll
+                for (int b = 0; b < 4; ++b) kb[b] = Ks[tx + 16 * b][p];
+#pragma unroll
+                for (int a = 0; a < RA; ++a)
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) s[a][b] = fmaf(qa[a], kb[b], s[a][b]);
+            }
+        }
+        // band mask + online softmax (log2 domain)
+        float alpha[RA];
+#pragma unroll
+        for (int a = 0; a < RA; ++a) {
+            const int mq = m0 + ty + 16 * a;
+            float cmax = -INFINITY;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int mk = c0 + tx + 16 * b;
+                const bool ok = (mk < kend) && (abs(mk - mq) <= w);
+                s[a][b] = ok ? s[a][b] * LOG2E : -INFINITY;
+                cmax = fmaxf(cmax, s[a][b]);
+            }
+            cmax = hmax16(cmax);
+            const float mnew = fmaxf(mrow[a], cmax);
+            alpha[a] = (mnew == -INFINITY) ? 1.f : exp2f(mrow[a] - mnew);
+            float sum = 0.f;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const float p = (s[a][b] == -INFINITY) ? 0.f : exp2f(s[a][b] - mnew);
+                Ps[ty + 16 * a][tx + 16 * b] = p;
+                sum += p;
+            }
+            sum = hsum16(sum);
+            lrow[a] = lrow[a] * alpha[a] + sum;
+            mrow[a] = mnew;
+        }
+        // O = alpha * O + P V
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            load_slice<Tin, C>(Ks, Vb, tc.rstride, c0, kend, col0, d);
+            __syncthreads();
+            float acc[RA][2];
+#pragma unroll
+            for (int a = 0; a < RA; ++a) { acc[a][0] = 0.f; acc[a][1] = 0.f; }
+#pragma unroll 8
+            for (int kk = 0; kk < C; ++kk) {
+                const float v0 = Ks[kk][tx], v1 = Ks[kk][tx + 16];
+#pragma unroll
+                for (int a = 0; a < RA; ++a) {
+                    const float p = Ps[ty + 16 * a][kk];
+                    acc[a][0] = fmaf(p, v0, acc[a][0]);
+                    acc[a][1] = fmaf(p, v1, acc[a][1]);
+                }
+            }
+#pragma unroll
+            for (int a = 0; a < RA; ++a)
+#pragma unroll
+                for (int b = 0; b < 2; ++b) {
+                    const int col = col0 + tx + 16 * b;
+                    if (col < d) {
+                        float* o = &Os[(ty + 16 * a) * d + col];
+                        *o = *o * alpha[a] + acc[a][b];
+                    }
+                }
+        }
+    }
+    if (tx == 0) {
+#pragma unroll
+        for (int a = 0; a < RA; ++a) { rowM[ty + 16 * a] = mrow[a]; rowL[ty + 16 * a] = lrow[a]; }
+    }
+    __syncthreads();
+    const int nrows = min(T, Lr - m0);
+    for (int i = threadIdx.x; i < nrows * d; i += NT) {
+        const int row = i / d, col = i % d;
+        Vec<Tin>::store1(out + tc.off + (int64_t)(m0 + row) * tc.rstride + col, Os[i] / rowL[row]);
+    }
+    for (int row = threadIdx.x; row < nrows; row += NT)
+        lse[tc.row0 + (int64_t)(m0 + row) * g.dil] = (rowM[row] + log2f(rowL[row])) * LN2;
+}
+
+// ------------------------------------------------------------------------------ backward: dq
+// Query-major: for owned query rows, dq_i = sum_j dS_ij k_j over the band.
+template <typename Tin>
+__global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
+                                                     const Tin* __restrict__ k,
+                                                     const Tin* __restrict__ v,
+                                                     const Tin* __restrict__ dout,
+                                                     const float* __restrict__ lse,
+                                                     const float* __restrict__ Dws,
+                                                     Tin* __restrict__ dq, Geo g) {
+    constexpr int T = 64, RA = T / 16;
+    extern __shared__ float smem[];
+    float(*Qs)[SP] = reinterpret_cast<float(*)[SP]>(smem);
+    float(*Gs)[SP] = Qs + T;   // dout rows
+    float(*Ks)[SP] = Gs + T;
+    float(*Vs)[SP] = Ks + C;
+    float(*Ps)[C + 1] = reinterpret_cast<float(*)[C + 1]>(Vs + C);
+    float* Os = reinterpret_cast<float*>(Ps + T);
+
+    TileCoord tc;
+    if (!decode(g, tc)) return;
+    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+    for (int i = threadIdx.x; i < T * d; i += NT) Os[i] = 0.f;
+
+    float lse2[RA], Drow[RA];
+#pragma unroll
+    for (int a = 0; a < RA; ++a) {
+        const int mq = m0 + ty + 16 * a;
+        const int64_t fr = tc.row0 + (int64_t)mq * g.dil;
+        lse2[a] = mq < Lr ? lse[fr] * LOG2E : 0.f;
+        Drow[a] = mq < Lr ? Dws[fr] : 0.f;
+    }
+    const int kbeg = max(0, m0 - w);
+    const int kend = min(Lr, m0 + T + w);
+    for (int c0 = kbeg; c0 < kend; c0 += C) {
+        float s[RA][4], dp[RA][4];
+#pragma unroll
+        for (int a = 0; a < RA; ++a)
+#pragma unroll
+            for (int b = 0; b < 4; ++b) { s[a][b] = 0.f; dp[a][b] = 0.f; }
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            load_slice<Tin, T>(Qs, q + tc.off, tc.rstride, m0, Lr, col0, d);
+            load_slice<Tin, T>(Gs, dout + tc.off, tc.rstride, m0, Lr, col0, d);
+            load_slice<Tin, C>(Ks, k + tc.off, tc.rstride, c0, kend, col0, d);
+            load_slice<Tin, C>(Vs, v + tc.off, tc.rstride, c0, kend, col0, d);
+            __syncthreads();
+#pragma unroll 4
+            for (int p = 0; p < DS; ++p) {
+                float qa[RA], ga[RA], kb[4], vb[4];
+#pragma unroll
+                for (int a = 0; a < RA; ++a) { qa[a] = Qs[ty + 16 * a][p]; ga[a] = Gs[ty + 16 * a][p]; }
+#pragma unroll
+                for (int b = 0; b < 4; ++b) { kb[b] = Ks[tx + 16 * b][p]; vb[b] = Vs[tx + 16 * b][p]; }
+#pragma unroll
+                for (int a = 0; a < RA; ++a)
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) {
+                        s[a][b] = fmaf(qa[a], kb[b], s[a][b]);
+                        dp[a][b] = fmaf(ga[a], vb[b], dp[a][b]);
+                    }
+            }
+        }
+#pragma unroll
+        for (int a = 0; a < RA; ++a) {
+            const int mq = m0 + ty + 16 * a;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int mk = c0 + tx + 16 * b;
+                const bool ok = (mk < kend) && (abs(mk - mq) <= w);
+                const float p = ok ? exp2f(s[a][b] * LOG2E - lse2[a]) : 0.f;
+                Ps[ty + 16 * a][tx + 16 * b] = p * (dp[a][b] - Drow[a]);
+            }
+        }
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            load_slice<Tin, C>(Ks, k + tc.off, tc.rstride, c0, kend, col0, d);
+            __syncthreads();
+            float acc[RA][2];
+#pragma unroll
+            for (int a = 0; a < RA; ++a) { acc[a][0] = 0.f; acc[a][1] = 0.f; }
+#pragma unroll 8
+            for (int kk = 0; kk < C; ++kk) {
+                const float k0 = Ks[kk][tx], k1 = Ks[kk][tx + 16];
+#pragma unroll
+                for (int a = 0; a < RA; ++a) {
+                    const float ds = Ps[ty + 16 * a][kk];
+                    acc[a][0] = fmaf(ds, k0, acc[a][0]);
+                    acc[a][1] = fmaf(ds, k1, acc[a][1]);
+                }
+            }
+#pragma unroll
+            for (int a = 0; a < RA; ++a)
+#pragma unroll
+                for (int b = 0; b < 2; ++b) {
+                    const int col = col0 + tx + 16 * b;
+                    if (col < d) Os[(ty + 16 * a) * d + col] += acc[a][b];
+                }
+        }
+    }
+    __syncthreads();
+    const int nrows = min(T, Lr - m0);
+    for (int i = threadIdx.x; i < nrows * d; i += NT) {
+        const int row = i / d, col = i % d;
+        Vec<Tin>::store1(dq + tc.off + (int64_t)(m0 + row) * tc.rstride + col, Os[i]);
+    }
+}
+
+// ------------------------------------------------------------------------------ backward: dk, dv
+// Key-major: for owned key rows j, dk_j = sum_i dS_ij q_i and dv_j = sum_i P_ij dout_i over
+// the queries i whose window contains j (the band is symmetric: |m_i - m_j| <= w).
+template <typename Tin, int T>
+__global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q,
+                                                       const Tin* __restrict__ k,
+                                                       const Tin* __restrict__ v,
+                                                       const Tin* __restrict__ dout,
+                                                       const float* __restrict__ lse,
+                                                       const float* __restrict__ Dws,
+                                                       Tin* __restrict__ dk, Tin* __restrict__ dv,
+                                                       Geo g) {
+    constexpr int RA = T / 16;
+    extern __shared__ float smem[];
+    float(*Ks)[SP] = reinterpret_cast<float(*)[SP]>(smem);
+    float(*Vs)[SP] = Ks + T;
+    float(*Qs)[SP] = Vs + T;   // query rows of the chunk
+    float(*Gs)[SP] = Qs + C;   // dout rows of the chunk
+    float(*Ps)[C + 1] = reinterpret_cast<float(*)[C + 1]>(Gs + C);
+    float(*DSs)[C + 1] = Ps + T;
+    float* qlse = reinterpret_cast<float*>(DSs + T);
+    float* qD = qlse + C;
+    float* OsK = qD + C;
+    float* OsV = OsK + T * g.d;
+
+    TileCoord tc;
+    if (!decode(g, tc)) return;
+    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+    for (int i = threadIdx.x; i < T * d; i += NT) { OsK[i] = 0.f; OsV[i] = 0.f; }
+
+    const int qbeg = max(0, m0 - w);
+    const int qend = min(Lr, m0 + T + w);
+    for (int c0 = qbeg; c0 < qend; c0 += C) {
+        float s[RA][4], dp[RA][4];
+#pragma unroll
+        for (int a = 0; a < RA; ++a)
+#pragma unroll
+            for (int b = 0; b < 4; ++b) { s[a][b] = 0.f; dp[a][b] = 0.f; }
+        __syncthreads();
+        for (int i = threadIdx.x; i < C; i += NT) {
+            const int mq = c0 + i;
+            const int64_t fr = tc.row0 + (int64_t)mq * g.dil;
+            qlse[i] = mq < qend ? lse[fr] * LOG2E : 0.f;
+            qD[i] = mq < qend ? Dws[fr] : 0.f;
+        }
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            load_slice<Tin, T>(Ks, k + tc.off, tc.rstride, m0, Lr, col0, d);
+            load_slice<Tin, T>(Vs, v + tc.off, tc.rstride, m0, Lr, col0, d);
+            load_slice<Tin, C>(Qs, q + tc.off, tc.rstride, c0, qend, col0, d);
+            load_slice<Tin, C>(Gs, dout + tc.off, tc.rstride, c0, qend, col0, d);
+            __syncthreads();
+#pragma unroll 4
+            for (int p = 0; p < DS; ++p) {
+                float ka[RA], va[RA], qb[4], gb[4];
+#pragma unroll
+                for (int a = 0; a < RA; ++a) { ka[a] = Ks[ty + 16 * a][p]; va[a] = Vs[ty + 16 * a][p]; }
+#pragma unroll
+                for (int b = 0; b < 4; ++b) { qb[b] = Qs[tx + 16 * b][p]; gb[b] = Gs[tx + 16 * b][p]; }
+#pragma unroll
+                for (int a = 0; a < RA; ++a)
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) {
+                        s[a][b] = fmaf(ka[a], qb[b], s[a][b]);
+                        dp[a][b] = fmaf(va[a], gb[b], dp[a][b]);
+                    }
+            }
+        }
+#pragma unroll
+        for (int a = 0; a < RA; ++a) {
+            const int mk = m0 + ty + 16 * a;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int qi = tx + 16 * b;
+                const int mq = c0 + qi;
+                const bool ok = (mq < qend) && (abs(mq - mk) <= w);
+                const float p = ok ? exp2f(s[a][b] * LOG2E - qlse[qi]) : 0.f;
+                Ps[ty + 16 * a][qi] = p;
+                DSs[ty + 16 * a][qi] = p * (dp[a][b] - qD[qi]);
+            }
+        }
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            load_slice<Tin, C>(Qs, q + tc.off, tc.rstride, c0, qend, col0, d);
+            load_slice<Tin, C>(Gs, dout + tc.off, tc.rstride, c0, qend, col0, d);
+            __syncthreads();
+            float ak[RA][2], av[RA][2];
+#pragma unroll
+            for (int a = 0; a < RA; ++a) { ak[a][0] = ak[a][1] = av[a][0] = av[a][1] = 0.f; }
+#pragma unroll 4
+            for (int qi = 0; qi < C; ++qi) {
+                const float q0 = Qs[qi][tx], q1 = Qs[qi][tx + 16];
+                const float g0 = Gs[qi][tx], g1 = Gs[qi][tx + 16];
+#pragma unroll
+                for (int a = 0; a < RA; ++a) {
+                    const float ds = DSs[ty + 16 * a][qi], p = Ps[ty + 16 * a][qi];
+                    ak[a][0] = fmaf(ds, q0, ak[a][0]);
+                    ak[a][1] = fmaf(ds, q1, ak[a][1]);
+                    av[a][0] = fmaf(p, g0, av[a][0]);
+                    av[a][1] = fmaf(p, g1, av[a][1]);
+                }
+            }
+#pragma unroll
+            for (int a = 0; a < RA; ++a)
+#pragma unroll
+                for (int b = 0; b < 2; ++b) {
+                    const int col = col0 + tx + 16 * b;
+                    if (col < d) {
+                        OsK[(ty + 16 * a) * d + col] += ak[a][b];
+                        OsV[(ty + 16 * a) * d + col] += av[a][b];
+                    }
+                }
+        }
+    }
+    __syncthreads();
+    const int nrows = min(T, Lr - m0);
+    for (int i = threadIdx.x; i < nrows * d; i += NT) {
+        const int row = i / d, col = i % d;
+        const int64_t o = tc.off + (int64_t)(m0 + row) * tc.rstride + col;
+        Vec<Tin>::store1(dk + o, OsK[i]);
+        Vec<Tin>::store1(dv + o, OsV[i]);
+    }
+}
+
+// ------------------------------------------------------------------------------ D_i pre-pass
+// D_i = sum_p dout_ip out_ip, one warp per row, fp32 accumulation.
+template <typename Tin>
+__global__ void __launch_bounds__(NT) rowdot_kernel(const Tin* __restrict__ a,
+                                                    const Tin* __restrict__ b,
+                                                    float* __restrict__ D, int64_t rows, int d) {
+    constexpr int V = Vec<Tin>::N;
+    const int64_t row = (int64_t)blockIdx.x * (NT / 32) + threadIdx.x / 32;
+    const int lane = threadIdx.x % 32;
+    if (row >= rows) return;
+    const Tin* pa = a + row * d;
+    const Tin* pb = b + row * d;
+    float acc = 0.f;
+    for (int c = lane * V; c < d; c += 32 * V) {
+        float x[V], y[V];
+        Vec<Tin>::load(pa + c, x);
+        Vec<Tin>::load(pb + c, y);
+#pragma unroll
+        for (int e = 0; e < V; ++e) acc = fmaf(x[e], y[e], acc);
+    }
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) D[row] = acc;
+}
+
+size_t fwd_smem(int64_t d) { return sizeof(float) * (64 * SP + C * SP + 64 * (C + 1) + 64 * d + 128); }
+size_t dq_smem(int64_t d) { return sizeof(float) * (2 * 64 * SP + 2 * C * SP + 64 * (C + 1) + 64 * d); }
+size_t dkdv_smem(int T, int64_t d) {
+    return sizeof(float) * (2 * T * SP + 2 * C * SP + 2 * T * (C + 1) + 2 * C + 2 * T * d);
+}
+
+template <typename F>
+void set_smem_once(F* f, size_t bytes, std::once_flag& flag) {
+    std::call_once(flag, [&] {
+        cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(227 * 1024));
+    });
+    (void)bytes;
+}
+
+template <typename Tin>
+cudaError_t fwd_impl(const void* q, const void* k, const void* v, void* out, float* lse,
+                     int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                     cudaStream_t st) {
+    static std::once_flag once;
+    Geo g = make_geo(B, H, L, d, w, dil, 64);
+    set_smem_once(simt_fwd_kernel<Tin>, fwd_smem(d), once);
+    simt_fwd_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_smem(d), st>>>(
+        (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, g);
+    return cudaGetLastError();
+}
+
+template <typename Tin>
+cudaError_t bwd_impl(const void* q, const void* k, const void* v, const void* out,
+                     const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
+                     int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                     cudaStream_t st) {
+    static std::once_flag o1, o2, o3;
+    cudaError_t e = launch_rowdot(dout, out, Dws, B * H * L, d,
+                                  sizeof(Tin) == 4 ? FT_F32 : FT_BF16, st);
+    if (e != cudaSuccess) return e;
+    Geo g = make_geo(B, H, L, d, w, dil, 64);
+    set_smem_once(simt_dq_kernel<Tin>, dq_smem(d), o1);
+    simt_dq_kernel<Tin><<<(unsigned)geo_blocks(g), NT, dq_smem(d), st>>>(
+        (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dq, g);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    if (d <= 256) {
+        Geo g2 = make_geo(B, H, L, d, w, dil, 64);
+        set_smem_once(simt_dkdv_kernel<Tin, 64>, dkdv_smem(64, d), o2);
+        simt_dkdv_kernel<Tin, 64><<<(unsigned)geo_blocks(g2), NT, dkdv_smem(64, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dk,
+            (Tin*)dv, g2);
+    } else {
+        Geo g2 = make_geo(B, H, L, d, w, dil, 32);
+        set_smem_once(simt_dkdv_kernel<Tin, 32>, dkdv_smem(32, d), o3);
+        simt_dkdv_kernel<Tin, 32><<<(unsigned)geo_blocks(g2), NT, dkdv_smem(32, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dk,
+            (Tin*)dv, g2);
+    }
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_rowdot(const void* dout, const void* out, float* D, int64_t rows, int64_t d,
+                          ft_dtype dt, cudaStream_t st) {
+    const unsigned blocks = (unsigned)ceil_div(rows, NT / 32);
+    if (dt == FT_F32)
+        rowdot_kernel<float><<<blocks, NT, 0, st>>>((const float*)dout, (const float*)out, D, rows, (int)d);
+    else
+        rowdot_kernel<__nv_bfloat16><<<blocks, NT, 0, st>>>(
+            (const __nv_bfloat16*)dout, (const __nv_bfloat16*)out, D, rows, (int)d);
+    return cudaGetLastError();
+}
+
+cudaError_t simt_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
+                     int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                     ft_dtype dt, cudaStream_t st) {
+    if (dt == FT_F32) return fwd_impl<float>(q, k, v, out, lse, B, H, L, d, w, dil, st);
+    return fwd_impl<__nv_bfloat16>(q, k, v, out, lse, B, H, L, d, w, dil, st);
+}
+
+cudaError_t simt_bwd(const void* q, const void* k, const void* v, const void* out,
+                     const float* lse, const void* dout, void* dq, void* dk, void* dv,
+                     float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
+                     int64_t dil, ft_dtype dt, cudaStream_t st) {
+    if (dt == FT_F32)
+        return bwd_impl<float>(q, k, v, out, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st);
+    return bwd_impl<__nv_bfloat16>(q, k, v, out, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st);
+}
+
+int simt_fwd_launches() { return 1; }
+int simt_bwd_launches() { return 3; }
+
+}  // namespace ftw

@@ -1,0 +1,125 @@
+"""C-ABI checks that need no GPU: the library builds for sm_100a, loads, exports every
+symbol include/ft_winattn.h declares, and argument validation returns the documented
+status codes before any launch (fake device pointers are never dereferenced)."""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+import subprocess
+
+import pytest
+
+import paper_conf_pldi_tangzwjzyz22_b200 as ft
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "ft_winattn.h")
+
+OK, INVALID, NOTSUP, MISALIGNED = 0, 1, 2, 3
+
+
+@pytest.fixture(scope="module")
+def lib():
+    return ft.load_library(build_if_missing=True)
+
+
+def declared_symbols():
+    src = open(HEADER).read()
+    return sorted(set(re.findall(r"^\S[^;()]*?\b(ft_\w+)\s*\(", src, flags=re.M)))
+
+
+def test_header_declares_the_boundary():
+    syms = declared_symbols()
+    for s in ("ft_winattn_fwd", "ft_winattn_bwd", "ft_winattn_bwd_workspace_bytes",
+              "ft_winattn_plan", "ft_status_str", "ft_winattn_abi_version"):
+        assert s in syms
+
+
+def test_library_exports_every_declared_symbol(lib):
+    out = subprocess.run(["nm", "-D", "--defined-only", ft.lib_path()], capture_output=True,
+                         text=True, check=True).stdout
+    exported = set(re.findall(r"\bT\s+(\w+)", out))
+    missing = [s for s in declared_symbols() if s not in exported]
+    assert not missing, missing
+    assert lib.ft_winattn_abi_version() == 1
+
+
+def test_library_is_sm100a(lib):
+    out = subprocess.run(["cuobjdump", "--list-elf", ft.lib_path()], capture_output=True,
+                         text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_library_has_tcgen05_and_tma(lib):
+    sass = subprocess.run(["cuobjdump", "-sass", ft.lib_path()], capture_output=True,
+                          text=True).stdout
+    assert "UTCHMMA" in sass          # tcgen05.mma
+    assert "UTMALDG" in sass          # TMA load
+    assert "LDTM" in sass             # tcgen05.ld
+
+
+# fake, 16-byte aligned "device" pointers in disjoint ranges (never dereferenced)
+def P(i, off=0):
+    return ctypes.c_void_p(0x10000000000 + i * 0x100000000 + off)
+
+
+def fwd_call(lib, q=None, k=None, v=None, out=None, lse=None, B=1, H=1, L=64, d=64, w=4, dil=1,
+             dt=1, alias=None):
+    given = [q, k, v, out, lse]
+    args = [P(i) if a is None else a for i, a in enumerate(given)]
+    if alias:
+        args[alias[0]] = args[alias[1]]
+    return lib.ft_winattn_fwd(*args, B, H, L, d, w, dil, dt, None)
+
+
+def test_fwd_validation(lib):
+    assert fwd_call(lib, q=ctypes.c_void_p(0)) == INVALID
+    assert fwd_call(lib, B=0) == INVALID
+    assert fwd_call(lib, L=0) == INVALID
+    assert fwd_call(lib, w=-1) == INVALID
+    assert fwd_call(lib, dil=0) == INVALID
+    assert fwd_call(lib, d=24) == NOTSUP
+    assert fwd_call(lib, d=528) == NOTSUP
+    assert fwd_call(lib, dt=7) == NOTSUP
+    assert fwd_call(lib, q=P(0, 8)) == MISALIGNED
+    assert fwd_call(lib, alias=(3, 0)) == INVALID     # out aliases q
+    assert fwd_call(lib, alias=(4, 3)) == INVALID     # lse aliases out
+
+
+def bwd_call(lib, ws_bytes=None, ws=None, alias=None, **kw):
+    B, H, L, d, w, dil, dt = (kw.get(n, dv) for n, dv in
+                              (("B", 1), ("H", 1), ("L", 64), ("d", 64), ("w", 4), ("dil", 1), ("dt", 1)))
+    need = lib.ft_winattn_bwd_workspace_bytes(B, H, L, d, w, dil, dt)
+    args = [P(i) for i in range(9)]
+    if alias:
+        args[alias[0]] = args[alias[1]]
+    return lib.ft_winattn_bwd(*args, B, H, L, d, w, dil, dt, ws or P(9),
+                              need if ws_bytes is None else ws_bytes, None)
+
+
+def test_bwd_validation(lib):
+    assert bwd_call(lib, w=-2) == INVALID
+    assert bwd_call(lib, ws_bytes=0) == INVALID          # workspace too small
+    assert bwd_call(lib, ws=P(9, 4)) == MISALIGNED
+    assert bwd_call(lib, alias=(6, 0)) == INVALID        # dq aliases q
+    assert bwd_call(lib, alias=(7, 6)) == INVALID        # dk aliases dq
+    assert bwd_call(lib, d=8) == NOTSUP
+
+
+def test_workspace_and_plan(lib):
+    assert lib.ft_winattn_bwd_workspace_bytes(2, 3, 100, 64, 4, 1, 1) >= 2 * 3 * 100 * 4
+    assert lib.ft_winattn_bwd_workspace_bytes(0, 3, 100, 64, 4, 1, 1) == 0
+    path, n = ft.plan(False, 1, 8, 10000, 512, 32, 1, ft.FT_BF16)
+    assert path == ft.PATH_TC and n == 1
+    path, n = ft.plan(False, 1, 8, 10000, 512, 32, 1, ft.FT_F32)
+    assert path == ft.PATH_SIMT and n >= 1
+    path, n = ft.plan(True, 1, 1, 64, 16, 4, 1, ft.FT_F32)
+    assert path == ft.PATH_SIMT and n >= 1
+    with pytest.raises(ft.FtError):
+        ft.plan(False, 1, 1, 64, 24, 4, 1, ft.FT_F32)
+
+
+def test_status_strings(lib):
+    for s in range(5):
+        assert lib.ft_status_str(s)
+    assert b"INVALID" in lib.ft_status_str(1)

@@ -1,0 +1,224 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle on the same
+seeded inputs.  Run on a B200 with ``pytest -m gpu``.
+
+* element-by-element at sizes the oracle finishes in seconds, spanning several tiles and a
+  ragged tail, for both kernel families (FT_WINATTN_PATH=simt|tc forces one);
+* sampled rows at BASELINE.json's full sizes (C2a, C2b, C4), in the launch configuration
+  bench.py times, against the oracle's per-row entry points;
+* edge cases: L=1, w=0, w >= L, dilation >= L, ragged tails, x16 logits.
+"""
+from __future__ import annotations
+
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth import CONFIGS, WinAttnShape, make_inputs
+from tests._util import compare
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ft():
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    import paper_conf_pldi_tangzwjzyz22_b200 as ft
+
+    ft.load_library(build_if_missing=True)
+    return ft
+
+
+class forced_path:
+    def __init__(self, path):
+        self.path = path
+
+    def __enter__(self):
+        self.old = os.environ.get("FT_WINATTN_PATH")
+        if self.path:
+            os.environ["FT_WINATTN_PATH"] = self.path
+        else:
+            os.environ.pop("FT_WINATTN_PATH", None)
+
+    def __exit__(self, *a):
+        if self.old is None:
+            os.environ.pop("FT_WINATTN_PATH", None)
+        else:
+            os.environ["FT_WINATTN_PATH"] = self.old
+
+
+def _dtype_code(dtype):
+    return 0 if dtype == "f32" else 1
+
+
+def run_case(ft, shape: WinAttnShape, dtype: str, path: str | None, seed: int = 0,
+             q_scale: float = 1.0, check_bwd: bool = True):
+    x = make_inputs(shape, seed, dtype, q_scale=q_scale)
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    with forced_path(path):
+        if path == "tc":
+            p, _ = ft.plan(False, shape.batch, shape.heads, shape.seq_len, shape.d, shape.w,
+                           shape.dilation, _dtype_code(dtype))
+            assert p == ft.PATH_TC
+        out, lse = ft.fwd(q, k, v, shape.w, shape.dilation)
+        if check_bwd:
+            dq, dk, dv = ft.bwd(q, k, v, out, lse, g, shape.w, shape.dilation)
+    torch.cuda.synchronize()
+    ro, rl = oracle.fwd(x["q64"], x["k64"], x["v64"], shape.w, shape.dilation)
+    compare("out", out.double().cpu().numpy(), ro, dtype)
+    compare("lse", lse.double().cpu().numpy(), rl, dtype)
+    if check_bwd:
+        rdq, rdk, rdv = oracle.bwd(x["q64"], x["k64"], x["v64"], ro, rl, x["dout64"], shape.w,
+                                   shape.dilation)
+        compare("dq", dq.double().cpu().numpy(), rdq, dtype)
+        compare("dk", dk.double().cpu().numpy(), rdk, dtype)
+        compare("dv", dv.double().cpu().numpy(), rdv, dtype)
+
+
+# (B, H, L, d, w, dil): several tiles of 64/128 rows, ragged tails, dilation, edges.
+SMALL = [
+    (1, 1, 64, 16, 4, 1),        # C1
+    (1, 2, 300, 64, 32, 1),
+    (1, 2, 300, 64, 32, 3),
+    (2, 1, 257, 128, 17, 2),
+    (1, 1, 200, 512, 32, 1),
+    (1, 1, 130, 64, 64, 1),
+    (1, 1, 100, 64, 0, 1),
+    (1, 1, 50, 64, 100, 1),      # w >= L: full attention
+    (1, 1, 1, 64, 3, 1),         # L = 1
+    (1, 1, 40, 64, 4, 50),       # dilation >= L
+    (1, 2, 333, 48, 9, 4),
+]
+SIMT_ONLY = [
+    (1, 1, 300, 64, 100, 1),     # w > 64
+    (1, 1, 520, 32, 200, 2),
+]
+
+
+@pytest.mark.parametrize("shape", SMALL + SIMT_ONLY, ids=lambda s: "x".join(map(str, s)))
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+def test_simt_parity(ft, shape, dtype):
+    run_case(ft, WinAttnShape(*shape), dtype, "simt", seed=1)
+
+
+def _tc_ok(ft, shape, bwd=False):
+    B, H, L, d, w, dil = shape
+    os.environ["FT_WINATTN_PATH"] = "tc"
+    try:
+        ft.plan(bwd, B, H, L, d, w, dil, 1)
+        return True
+    except ft.FtError:
+        return False
+    finally:
+        os.environ.pop("FT_WINATTN_PATH", None)
+
+
+@pytest.mark.parametrize("shape", SMALL, ids=lambda s: "x".join(map(str, s)))
+def test_tc_fwd_parity(ft, shape):
+    if not _tc_ok(ft, shape):
+        pytest.skip("shape not on the tensor-core path")
+    run_case(ft, WinAttnShape(*shape), "bf16", "tc", seed=2, check_bwd=False)
+
+
+@pytest.mark.parametrize("shape", SMALL, ids=lambda s: "x".join(map(str, s)))
+def test_tc_bwd_parity(ft, shape):
+    if not _tc_ok(ft, shape, bwd=True):
+        pytest.skip("shape not on the tensor-core backward path")
+    run_case(ft, WinAttnShape(*shape), "bf16", "tc", seed=3)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_default_path_seeds(ft, seed):
+    run_case(ft, WinAttnShape(1, 2, 384, 64, 32, 1), "bf16", None, seed=seed)
+    run_case(ft, WinAttnShape(1, 1, 192, 64, 8, 1), "f32", None, seed=seed)
+
+
+def test_overflow_probe(ft):
+    """q x16: logits of std ~ 43; max subtraction must keep everything finite and exact."""
+    for dt in ("f32", "bf16"):
+        run_case(ft, WinAttnShape(1, 1, 256, 64, 16, 1), dt, None, seed=4, q_scale=16.0)
+
+
+def test_dout_ones(ft):
+    """the gradient seed of JAX/Julia is sum(outputs) -> dout = 1."""
+    shape = WinAttnShape(1, 1, 200, 64, 8, 2)
+    x = make_inputs(shape, 5, "f32")
+    dev = torch.device("cuda:0")
+    q, k, v = (x[n].to(dev) for n in ("q", "k", "v"))
+    g = torch.ones_like(q)
+    out, lse = ft.fwd(q, k, v, shape.w, shape.dilation)
+    dq, dk, dv = ft.bwd(q, k, v, out, lse, g, shape.w, shape.dilation)
+    ro, rl = oracle.fwd(x["q64"], x["k64"], x["v64"], shape.w, shape.dilation)
+    r = oracle.bwd(x["q64"], x["k64"], x["v64"], ro, rl, np.ones_like(ro), shape.w, shape.dilation)
+    for n, a, b in zip(("dq", "dk", "dv"), (dq, dk, dv), r):
+        compare(n, a.double().cpu().numpy(), b, "f32")
+
+
+def test_determinism(ft):
+    """No atomics: two runs are bit-identical."""
+    shape = WinAttnShape(1, 2, 500, 64, 32, 1)
+    x = make_inputs(shape, 6, "bf16")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    a = ft.fwd(q, k, v, 32) + ft.bwd(q, k, v, *ft.fwd(q, k, v, 32), g, 32)
+    b = ft.fwd(q, k, v, 32) + ft.bwd(q, k, v, *ft.fwd(q, k, v, 32), g, 32)
+    for x1, x2 in zip(a, b):
+        assert torch.equal(x1, x2)
+
+
+def test_autograd_function(ft):
+    shape = WinAttnShape(1, 2, 130, 64, 5, 1)
+    x = make_inputs(shape, 7, "f32")
+    dev = torch.device("cuda:0")
+    q, k, v = (x[n].to(dev).requires_grad_() for n in ("q", "k", "v"))
+    g = x["dout"].to(dev)
+    out = ft.win_attn(q, k, v, 5, 1)
+    out.backward(g)
+    ro, rl = oracle.fwd(x["q64"], x["k64"], x["v64"], 5, 1)
+    r = oracle.bwd(x["q64"], x["k64"], x["v64"], ro, rl, x["dout64"], 5, 1)
+    compare("out", out.detach().double().cpu().numpy(), ro, "f32")
+    for n, t, b in zip(("dq", "dk", "dv"), (q, k, v), r):
+        compare(n, t.grad.double().cpu().numpy(), b, "f32")
+
+
+# ------------------------------------------------------------------ full-size sampled checks
+def _sample_rows(shape: WinAttnShape, n_mid: int, seed: int):
+    L, U = shape.seq_len, shape.units
+    rng = np.random.default_rng(seed)
+    rows = set()
+    for u in {0, U - 1}:
+        for i in list(range(0, 3)) + list(range(L - 3, L)) + [shape.w, L - 1 - shape.w, 127, 128]:
+            if 0 <= i < L:
+                rows.add(u * L + i)
+    rows.update(int(r) for r in rng.integers(0, U * L, size=n_mid))
+    return np.array(sorted(rows), dtype=np.int64)
+
+
+@pytest.mark.parametrize("name,dtype", [("C2a", "bf16"), ("C2a", "f32"), ("C2a_dil", "bf16"),
+                                        ("C2b", "bf16"), ("C4d2", "bf16"), ("C4d4", "bf16")])
+def test_full_size_sampled(ft, name, dtype):
+    shape = CONFIGS[name]
+    x = make_inputs(shape, 0, dtype)
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    out, lse = ft.fwd(q, k, v, shape.w, shape.dilation)
+    dq, dk, dv = ft.bwd(q, k, v, out, lse, g, shape.w, shape.dilation)
+    torch.cuda.synchronize()
+    rows = _sample_rows(shape, 48, seed=1)
+    d = shape.d
+    ro, rl = oracle.fwd_rows(x["q64"], x["k64"], x["v64"], shape.w, shape.dilation, rows)
+    compare("out", out.reshape(-1, d)[torch.from_numpy(rows).to(dev)].double().cpu().numpy(), ro, dtype)
+    compare("lse", lse.reshape(-1)[torch.from_numpy(rows).to(dev)].double().cpu().numpy(), rl, dtype)
+    rq, rk, rv = oracle.bwd_rows(x["q64"], x["k64"], x["v64"], x["dout64"], shape.w,
+                                 shape.dilation, rows)
+    idx = torch.from_numpy(rows).to(dev)
+    compare("dq", dq.reshape(-1, d)[idx].double().cpu().numpy(), rq, dtype)
+    compare("dk", dk.reshape(-1, d)[idx].double().cpu().numpy(), rk, dtype)
+    compare("dv", dv.reshape(-1, d)[idx].double().cpu().numpy(), rv, dtype)
+    # properties at any size: everything finite
+    for t in (out, lse, dq, dk, dv):
+        assert torch.isfinite(t).all()
