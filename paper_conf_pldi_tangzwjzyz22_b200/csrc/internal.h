@@ -65,8 +65,4 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
 int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
 int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
 
-// D_i = dout_i . out_i pre-pass shared by both backward families -- simt.cu
-cudaError_t launch_rowdot(const void* dout, const void* out, float* D, int64_t rows, int64_t d,
-                          ft_dtype dt, cudaStream_t st);
-
 }  // namespace ftw

@@ -237,37 +237,45 @@ __global__ void __launch_bounds__(NT) simt_fwd_kernel(const Tin* __restrict__ q,
 }
 
 // ------------------------------------------------------------------------------ backward: dq
-// Query-major: for owned query rows, dq_i = sum_j dS_ij k_j over the band.
-template <typename Tin>
+// Query-major: for owned query rows i,
+//     D_i  = sum_j P_ij dP_ij                 (= dout_i . o_i exactly, without reading the
+//                                              stored, possibly bf16-rounded, out)
+//     dq_i = sum_j P_ij (dP_ij - D_i) k_j  =  sum_j (P_ij dP_ij) k_j  -  D_i sum_j P_ij k_j
+// so one sweep over the band accumulates A_i = sum (P dP) k, B_i = sum P k and D_i, and
+// dq_i = A_i - D_i B_i at the end.  D is also written to the workspace for the key-major
+// kernel.
+template <typename Tin, int T>
 __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
                                                      const Tin* __restrict__ k,
                                                      const Tin* __restrict__ v,
                                                      const Tin* __restrict__ dout,
                                                      const float* __restrict__ lse,
-                                                     const float* __restrict__ Dws,
+                                                     float* __restrict__ Dws,
                                                      Tin* __restrict__ dq, Geo g) {
-    constexpr int T = 64, RA = T / 16;
+    constexpr int RA = T / 16;
     extern __shared__ float smem[];
     float(*Qs)[SP] = reinterpret_cast<float(*)[SP]>(smem);
     float(*Gs)[SP] = Qs + T;   // dout rows
     float(*Ks)[SP] = Gs + T;
     float(*Vs)[SP] = Ks + C;
-    float(*Ps)[C + 1] = reinterpret_cast<float(*)[C + 1]>(Vs + C);
-    float* Os = reinterpret_cast<float*>(Ps + T);
+    float(*PDs)[C + 1] = reinterpret_cast<float(*)[C + 1]>(Vs + C);   // P * dP
+    float(*Ps)[C + 1] = PDs + T;                                        // P
+    float* rowD = reinterpret_cast<float*>(Ps + T);
+    float* OsA = rowD + T;
+    float* OsB = OsA + T * g.d;
 
     TileCoord tc;
     if (!decode(g, tc)) return;
     const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
     const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
-    for (int i = threadIdx.x; i < T * d; i += NT) Os[i] = 0.f;
+    for (int i = threadIdx.x; i < T * d; i += NT) { OsA[i] = 0.f; OsB[i] = 0.f; }
 
-    float lse2[RA], Drow[RA];
+    float lse2[RA], Dacc[RA];
 #pragma unroll
     for (int a = 0; a < RA; ++a) {
         const int mq = m0 + ty + 16 * a;
-        const int64_t fr = tc.row0 + (int64_t)mq * g.dil;
-        lse2[a] = mq < Lr ? lse[fr] * LOG2E : 0.f;
-        Drow[a] = mq < Lr ? Dws[fr] : 0.f;
+        lse2[a] = mq < Lr ? lse[tc.row0 + (int64_t)mq * g.dil] * LOG2E : 0.f;
+        Dacc[a] = 0.f;
     }
     const int kbeg = max(0, m0 - w);
     const int kend = min(Lr, m0 + T + w);
@@ -308,24 +316,29 @@ __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
                 const int mk = c0 + tx + 16 * b;
                 const bool ok = (mk < kend) && (abs(mk - mq) <= w);
                 const float p = ok ? exp2f(s[a][b] * LOG2E - lse2[a]) : 0.f;
-                Ps[ty + 16 * a][tx + 16 * b] = p * (dp[a][b] - Drow[a]);
+                const float pd = p * dp[a][b];
+                Dacc[a] += pd;
+                PDs[ty + 16 * a][tx + 16 * b] = pd;
+                Ps[ty + 16 * a][tx + 16 * b] = p;
             }
         }
         for (int col0 = 0; col0 < d; col0 += DS) {
             __syncthreads();
             load_slice<Tin, C>(Ks, k + tc.off, tc.rstride, c0, kend, col0, d);
             __syncthreads();
-            float acc[RA][2];
+            float aA[RA][2], aB[RA][2];
 #pragma unroll
-            for (int a = 0; a < RA; ++a) { acc[a][0] = 0.f; acc[a][1] = 0.f; }
-#pragma unroll 8
+            for (int a = 0; a < RA; ++a) { aA[a][0] = aA[a][1] = aB[a][0] = aB[a][1] = 0.f; }
+#pragma unroll 4
             for (int kk = 0; kk < C; ++kk) {
                 const float k0 = Ks[kk][tx], k1 = Ks[kk][tx + 16];
 #pragma unroll
                 for (int a = 0; a < RA; ++a) {
-                    const float ds = Ps[ty + 16 * a][kk];
-                    acc[a][0] = fmaf(ds, k0, acc[a][0]);
-                    acc[a][1] = fmaf(ds, k1, acc[a][1]);
+                    const float pd = PDs[ty + 16 * a][kk], p = Ps[ty + 16 * a][kk];
+                    aA[a][0] = fmaf(pd, k0, aA[a][0]);
+                    aA[a][1] = fmaf(pd, k1, aA[a][1]);
+                    aB[a][0] = fmaf(p, k0, aB[a][0]);
+                    aB[a][1] = fmaf(p, k1, aB[a][1]);
                 }
             }
 #pragma unroll
@@ -333,16 +346,27 @@ __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
 #pragma unroll
                 for (int b = 0; b < 2; ++b) {
                     const int col = col0 + tx + 16 * b;
-                    if (col < d) Os[(ty + 16 * a) * d + col] += acc[a][b];
+                    if (col < d) {
+                        OsA[(ty + 16 * a) * d + col] += aA[a][b];
+                        OsB[(ty + 16 * a) * d + col] += aB[a][b];
+                    }
                 }
         }
+    }
+#pragma unroll
+    for (int a = 0; a < RA; ++a) {
+        const float D = hsum16(Dacc[a]);
+        if (tx == 0) rowD[ty + 16 * a] = D;
     }
     __syncthreads();
     const int nrows = min(T, Lr - m0);
     for (int i = threadIdx.x; i < nrows * d; i += NT) {
         const int row = i / d, col = i % d;
-        Vec<Tin>::store1(dq + tc.off + (int64_t)(m0 + row) * tc.rstride + col, Os[i]);
+        Vec<Tin>::store1(dq + tc.off + (int64_t)(m0 + row) * tc.rstride + col,
+                         OsA[i] - rowD[row] * OsB[i]);
     }
+    for (int row = threadIdx.x; row < nrows; row += NT)
+        Dws[tc.row0 + (int64_t)(m0 + row) * g.dil] = rowD[row];
 }
 
 // ------------------------------------------------------------------------------ backward: dk, dv
@@ -470,33 +494,8 @@ __global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q
     }
 }
 
-// ------------------------------------------------------------------------------ D_i pre-pass
-// D_i = sum_p dout_ip out_ip, one warp per row, fp32 accumulation.
-template <typename Tin>
-__global__ void __launch_bounds__(NT) rowdot_kernel(const Tin* __restrict__ a,
-                                                    const Tin* __restrict__ b,
-                                                    float* __restrict__ D, int64_t rows, int d) {
-    constexpr int V = Vec<Tin>::N;
-    const int64_t row = (int64_t)blockIdx.x * (NT / 32) + threadIdx.x / 32;
-    const int lane = threadIdx.x % 32;
-    if (row >= rows) return;
-    const Tin* pa = a + row * d;
-    const Tin* pb = b + row * d;
-    float acc = 0.f;
-    for (int c = lane * V; c < d; c += 32 * V) {
-        float x[V], y[V];
-        Vec<Tin>::load(pa + c, x);
-        Vec<Tin>::load(pb + c, y);
-#pragma unroll
-        for (int e = 0; e < V; ++e) acc = fmaf(x[e], y[e], acc);
-    }
-#pragma unroll
-    for (int o = 16; o >= 1; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if (lane == 0) D[row] = acc;
-}
-
 size_t fwd_smem(int64_t d) { return sizeof(float) * (64 * SP + C * SP + 64 * (C + 1) + 64 * d + 128); }
-size_t dq_smem(int64_t d) { return sizeof(float) * (2 * 64 * SP + 2 * C * SP + 64 * (C + 1) + 64 * d); }
+size_t dq_smem(int T, int64_t d) { return sizeof(float) * (2 * T * SP + 2 * C * SP + 2 * T * (C + 1) + T + 2 * T * d); }
 size_t dkdv_smem(int T, int64_t d) {
     return sizeof(float) * (2 * T * SP + 2 * C * SP + 2 * T * (C + 1) + 2 * C + 2 * T * d);
 }
@@ -526,43 +525,36 @@ cudaError_t bwd_impl(const void* q, const void* k, const void* v, const void* ou
                      const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
                      int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                      cudaStream_t st) {
-    static std::once_flag o1, o2, o3;
-    cudaError_t e = launch_rowdot(dout, out, Dws, B * H * L, d,
-                                  sizeof(Tin) == 4 ? FT_F32 : FT_BF16, st);
-    if (e != cudaSuccess) return e;
-    Geo g = make_geo(B, H, L, d, w, dil, 64);
-    set_smem_once(simt_dq_kernel<Tin>, dq_smem(d), o1);
-    simt_dq_kernel<Tin><<<(unsigned)geo_blocks(g), NT, dq_smem(d), st>>>(
-        (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dq, g);
-    if ((e = cudaGetLastError()) != cudaSuccess) return e;
-    if (d <= 256) {
-        Geo g2 = make_geo(B, H, L, d, w, dil, 64);
-        set_smem_once(simt_dkdv_kernel<Tin, 64>, dkdv_smem(64, d), o2);
-        simt_dkdv_kernel<Tin, 64><<<(unsigned)geo_blocks(g2), NT, dkdv_smem(64, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dk,
-            (Tin*)dv, g2);
+    (void)out;   // D_i is recomputed exactly as sum_j P_ij dP_ij (see simt_dq_kernel)
+    static std::once_flag o1, o2, o3, o4;
+    cudaError_t e;
+    const int T = d <= 256 ? 64 : 32;
+    Geo g = make_geo(B, H, L, d, w, dil, T);
+    if (T == 64) {
+        set_smem_once(simt_dq_kernel<Tin, 64>, dq_smem(64, d), o1);
+        simt_dq_kernel<Tin, 64><<<(unsigned)geo_blocks(g), NT, dq_smem(64, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dq, g);
     } else {
-        Geo g2 = make_geo(B, H, L, d, w, dil, 32);
-        set_smem_once(simt_dkdv_kernel<Tin, 32>, dkdv_smem(32, d), o3);
-        simt_dkdv_kernel<Tin, 32><<<(unsigned)geo_blocks(g2), NT, dkdv_smem(32, d), st>>>(
+        set_smem_once(simt_dq_kernel<Tin, 32>, dq_smem(32, d), o2);
+        simt_dq_kernel<Tin, 32><<<(unsigned)geo_blocks(g), NT, dq_smem(32, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dq, g);
+    }
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    if (T == 64) {
+        set_smem_once(simt_dkdv_kernel<Tin, 64>, dkdv_smem(64, d), o3);
+        simt_dkdv_kernel<Tin, 64><<<(unsigned)geo_blocks(g), NT, dkdv_smem(64, d), st>>>(
             (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dk,
-            (Tin*)dv, g2);
+            (Tin*)dv, g);
+    } else {
+        set_smem_once(simt_dkdv_kernel<Tin, 32>, dkdv_smem(32, d), o4);
+        simt_dkdv_kernel<Tin, 32><<<(unsigned)geo_blocks(g), NT, dkdv_smem(32, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dk,
+            (Tin*)dv, g);
     }
     return cudaGetLastError();
 }
 
 }  // namespace
-
-cudaError_t launch_rowdot(const void* dout, const void* out, float* D, int64_t rows, int64_t d,
-                          ft_dtype dt, cudaStream_t st) {
-    const unsigned blocks = (unsigned)ceil_div(rows, NT / 32);
-    if (dt == FT_F32)
-        rowdot_kernel<float><<<blocks, NT, 0, st>>>((const float*)dout, (const float*)out, D, rows, (int)d);
-    else
-        rowdot_kernel<__nv_bfloat16><<<blocks, NT, 0, st>>>(
-            (const __nv_bfloat16*)dout, (const __nv_bfloat16*)out, D, rows, (int)d);
-    return cudaGetLastError();
-}
 
 cudaError_t simt_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
                      int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
@@ -581,6 +573,6 @@ cudaError_t simt_bwd(const void* q, const void* k, const void* v, const void* ou
 }
 
 int simt_fwd_launches() { return 1; }
-int simt_bwd_launches() { return 3; }
+int simt_bwd_launches() { return 2; }
 
 }  // namespace ftw

@@ -17,7 +17,7 @@ import torch
 
 import oracle
 from synth import CONFIGS, WinAttnShape, make_inputs
-from tests._util import compare
+from _util import compare
 
 pytestmark = pytest.mark.gpu
 
