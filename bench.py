@@ -1,0 +1,412 @@
+#!/usr/bin/env python
+"""bench.py -- fwd+bwd banded window-attention throughput on B200 (one JSON line).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2a] [--dtype bf16]
+    python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N
+    python bench.py --impl reference ...      # the fp64 CPU oracle as the reference arm
+
+A step is one pass of the whole hot path (SURVEY.md §8(a) F0-F6 + B0-B5): ft_winattn_fwd
+then ft_winattn_bwd over one batch of synthetic inputs resident in HBM.  Default workload
+is BASELINE.json configs[2] "same shape forward+backward" at reading A14(a) of the
+paper's Longformer shape: B=1, H=8, L=10000, d=512, w=32 (C2a), bf16.
+
+Multi-GPU: (batch, head) units are independent, so the job is sharded
+with NO collective on the data path: every rank runs its own batch element (weak scaling,
+global_batch = N), timed between a barrier + synchronize on both sides, and the elapsed
+time is the max over ranks.
+
+Keys beyond the base contract: "roofline" (dominant kernel, CUDA events on the launching
+stream via the ft_winattn_profile_events hook), "hbm_step" (whole step vs SURVEY.md §8(d)
+algorithmic bytes), "cpu_baseline" (the fp64 oracle on a bounded sample, rank 0, N=1),
+"e2e" (pinned host buffers, H2D + fwd + bwd + D2H inside the timed region), "clocks"
+(NVML samples during the timed region) and "gpu_launches".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # name: (batch per rank, heads, seq_len, d, w, dilation, description)
+    "C2a": (1, 8, 10000, 512, 32, 1, "BASELINE configs[2]: Longformer-shaped fwd+bwd, reading A14(a)"),
+    "C2a_dil": (1, 2, 10000, 512, 32, 4, "C2a's dilated heads (artefact heads 0-1, dilation 4)"),
+    "C2b": (1, 12, 4096, 64, 256, 1, "Longformer-base shape, reading A14(b)"),
+    "C4d2": (1, 12, 16384, 64, 256, 2, "BASELINE configs[3]: dilated w=256, 16K tokens"),
+    "C4d4": (1, 12, 16384, 64, 256, 4, "BASELINE configs[3]: dilated w=256, 16K tokens"),
+    "C5_w32": (1, 64, 32768, 64, 32, 1, "BASELINE configs[4] sweep corner, HBM-bound"),
+    "C5_w256": (1, 64, 32768, 64, 256, 1, "BASELINE configs[4] sweep corner, ridge"),
+    "C5_small": (1, 8, 4096, 64, 32, 1, "BASELINE configs[4] sweep corner, small"),
+}
+
+METRIC = "window-attn fwd+bwd tokens/s per GPU and % HBM roofline at 1/2/4/8 B200"
+L2_BYTES = 126 * 1024 * 1024
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), float(p["bf16_tflops"]), float(p.get("sm_max_mhz", 1965.0)), "measured"
+    except Exception:
+        return 6650.0, 1590.0, 1965.0, "fallback"
+
+
+# ----------------------------------------------------------------------------- algorithmic work
+def rows_of(B, H, L):
+    return B * H * L
+
+
+def window_sizes(L, w, dil):
+    """n_i = |N(i)| for every row (SURVEY.md §8 closed form, pinned by the oracle tests)."""
+    import numpy as np
+    i = np.arange(L)
+    return np.minimum(w, i // dil) + np.minimum(w, (L - 1 - i) // dil) + 1
+
+
+def kernel_bytes_per_row(kind: str, d: int, e: int) -> int:
+    """Minimal HBM bytes one row of each kernel must move.
+    fwd : read q, k, v ; write o (dtype) and lse (fp32)                 = 4de + 4
+    bwdA: read q, k, v, dout, lse ; write dq, D                          = 5de + 8
+    bwdB: read q, k, v, dout, lse, D ; write dk, dv                      = 6de + 8"""
+    return {"fwd": 4 * d * e + 4, "bwdA": 5 * d * e + 8, "bwdB": 6 * d * e + 8}[kind]
+
+
+def step_bytes_per_row(d: int, e: int) -> int:
+    """fwd 4de+4 plus bwd 8de+4 (the bwd figure counts reading o)."""
+    return (4 * d * e + 4) + (8 * d * e + 4)
+
+
+# ----------------------------------------------------------------------------- clocks (NVML)
+class ClockSampler:
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+        0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+        0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, index: int, period_s: float = 0.005):
+        self.index, self.period = index, period_s
+        self.samples, self.reasons = [], set()
+        self._stop = threading.Event()
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.max_mhz = None
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                    "samples": len(self.samples)}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ----------------------------------------------------------------------------- CPU oracle legs
+def oracle_sample(shape, units: int, rows_cap: int, seed: int = 0):
+    """Time the fp64 oracle fwd+bwd on `units` (batch, head) units of the workload, each
+    truncated to its first rows_cap rows (its own band problem; per-row work equals the
+    full problem's away from the two sequence edges).  Returns (seconds, units, rows)."""
+    import numpy as np
+    import oracle
+    B, H, L, d, w, dil = shape
+    Ls = min(L, rows_cap)
+    rng = np.random.Generator(np.random.PCG64(seed))
+    x = [rng.uniform(-1.0, 1.0, size=(1, units, Ls, d)) for _ in range(4)]
+    oracle.fwd(x[0][:, :1, :8], x[1][:, :1, :8], x[2][:, :1, :8], w, dil)   # load / warm
+    t0 = time.perf_counter()
+    o, lse = oracle.fwd(x[0], x[1], x[2], w, dil)
+    oracle.bwd(x[0], x[1], x[2], o, lse, x[3], w, dil)
+    return time.perf_counter() - t0, units, Ls
+
+
+def cpu_baseline(shape, budget_s: float = 15.0):
+    """The oracle as it stands, on as many whole (batch, head) units of the workload as fit
+    in ~budget_s seconds of CPU work (at least one unit), extrapolated per unit."""
+    import oracle
+    B, H, L, d, w, dil = shape
+    s1, _, Ls = oracle_sample(shape, 1, L)
+    n = int(max(1, min(B * H, budget_s // max(s1, 1e-3))))
+    secs, n, Ls = oracle_sample(shape, n, L, seed=1) if n > 1 else (s1, 1, Ls)
+    value = (n * Ls / secs) / (B * H) * B
+    return {"value": value, "unit": "tokens/s", "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"fp64 oracle fwd+bwd on {n} of {B * H} (batch, head) units at full length "
+                      f"{Ls}; {secs:.2f} s of CPU work; tokens/s extrapolated linearly per unit",
+            "seconds": secs}
+
+
+def run_reference(args, shape, cfg):
+    """--impl reference: the fp64 CPU oracle as it stands, rank 0 only."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    B, H, L, d, w, dil = shape
+    rows_cap = args.ref_rows if args.ref_rows > 0 else L
+    for _ in range(args.warmup):
+        oracle_sample(shape, 1, rows_cap)
+    times = []
+    Ls = rows_cap
+    for _ in range(args.steps):
+        s, _, Ls = oracle_sample(shape, 1, rows_cap)
+        times.append(s)
+    mean = sum(times) / len(times)
+    value = (Ls / mean) / (B * H) * B
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "tokens/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": mean * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic", "config": cfg,
+        "cpu_baseline": {"value": value, "unit": "tokens/s", "kind": "oracle",
+                         "cores": oracle.num_threads(),
+                                  "sample": f"each step: fp64 oracle fwd+bwd on 1 of {B * H} (batch, head) "
+                                   f"units, {Ls} of {L} rows, tokens/s extrapolated per unit"},
+        "e2e": {"value": value, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- GPU arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="C2a", choices=sorted(WORKLOADS))
+    ap.add_argument("--dtype", default="bf16", choices=["bf16", "f32"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work (cpu_baseline)")
+    ap.add_argument("--ref-rows", type=int, default=0, help="oracle rows per reference step (0 = full L)")
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    B, H, L, d, w, dil, desc = WORKLOADS[args.workload]
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    shape = (B, H, L, d, w, dil)
+    e = 2 if args.dtype == "bf16" else 4
+    in_bytes = 4 * B * H * L * d * e
+    cfg = {"workload": args.workload, "desc": desc, "batch_per_rank": B, "heads": H, "seq_len": L,
+           "d": d, "w": w, "dilation": dil, "global_batch": B * world,
+           "parallelism": f"dp{world} over (batch, head) units, no collective on the data path",
+           "l2": ("inputs larger than L2" if in_bytes > L2_BYTES else "L2 flushed between steps") +
+                 f" ({in_bytes / 2**20:.0f} MiB of q/k/v/dout vs {L2_BYTES / 2**20:.0f} MiB L2)"}
+    if args.impl == "reference":
+        run_reference(args, shape, cfg)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_pldi_tangzwjzyz22_b200 as ft
+
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    ft.load_library()
+    tdt = torch.bfloat16 if args.dtype == "bf16" else torch.float32
+    code = ft.FT_BF16 if args.dtype == "bf16" else ft.FT_F32
+    path_f, nf = ft.plan(False, B, H, L, d, w, dil, code)
+    path_b, nb = ft.plan(True, B, H, L, d, w, dil, code)
+
+    gen = torch.Generator(device=dev)
+    gen.manual_seed(1234 + rank)
+    def rnd():
+        return (torch.rand((B, H, L, d), device=dev, generator=gen, dtype=torch.float32) * 2 - 1).to(tdt)
+    q, k, v, g = rnd(), rnd(), rnd(), rnd()
+    out, dq, dk, dv = (torch.empty_like(q) for _ in range(4))
+    lse = torch.empty((B, H, L), device=dev, dtype=torch.float32)
+    ws = torch.empty(max(ft.workspace_bytes(q, w, dil), 16), device=dev, dtype=torch.uint8)
+    flush = None
+    if in_bytes <= L2_BYTES:
+        flush = torch.empty(2 * L2_BYTES, device=dev, dtype=torch.uint8)
+
+    def step():
+        ft.fwd(q, k, v, w, dil, out=out, lse=lse)
+        ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # ---------------------------------------------------------------- timed region
+    stream = torch.cuda.current_stream(dev)
+    ev = lambda: torch.cuda.Event(enable_timing=True)
+    starts, fevs, bevs, ends = [], [], [], []
+    sampler = ClockSampler(dev.index if dev.index is not None else 0)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with sampler:
+        for _ in range(args.steps):
+            if flush is not None:
+                flush.zero_()   # outside the events: evicts q/k/v/dout from L2
+            s0, fe, be, s1 = ev(), [ev() for _ in range(nf)], [ev() for _ in range(nb)], ev()
+            s0.record(stream)
+            with ft.profile_events(fe):
+                ft.fwd(q, k, v, w, dil, out=out, lse=lse)
+            with ft.profile_events(be):
+                ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws)
+            s1.record(stream)
+            starts.append(s0); fevs.append(fe); bevs.append(be); ends.append(s1)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in zip(starts, ends)]
+    elapsed_ms = sum(step_ms)
+    # per-kernel durations (each launch timed from the previous event on the same stream)
+    names = [f"fwd{i}" for i in range(nf)] + [f"bwd{i}" for i in range(nb)]
+    kdur = {n: [] for n in names}
+    for s0, fe, be in zip(starts, fevs, bevs):
+        prev = s0
+        for n, e1 in zip(names, fe + be):
+            kdur[n].append(prev.elapsed_time(e1))
+            prev = e1
+    if world > 1:
+        t = torch.tensor([elapsed_ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        elapsed_ms = float(t.item())
+
+    tokens = B * L * world * args.steps
+    value = tokens / (elapsed_ms / 1e3)
+    hbm_peak, bf16_peak, sm_max, peak_src = load_peaks()
+    rows = rows_of(B, H, L)
+
+    # dominant kernel roofline
+    kinds = {}
+    if path_f == ft.PATH_TC or path_f == ft.PATH_SIMT:
+        for i in range(nf):
+            kinds[f"fwd{i}"] = "fwd"
+    kinds.update({f"bwd{i}": ("bwdA" if i == 0 else "bwdB") for i in range(nb)})
+    mean_k = {n: sum(x) / len(x) for n, x in kdur.items()}
+    dom = max(mean_k, key=mean_k.get)
+    # rows processed per launch: all rows (fwd launches are per residue group)
+    rows_per_launch = rows if not dom.startswith("fwd") or nf == 1 else rows / nf
+    if args.dtype == "bf16":
+        by = kernel_bytes_per_row(kinds[dom], d, e) * rows_per_launch
+        ach = by / (mean_k[dom] / 1e3) / 1e9
+        roof = {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
+                "frac": ach / hbm_peak, "traffic": None, "kernel": dom,
+                "kernel_kind": kinds[dom], "ms_per_launch": mean_k[dom],
+                "algorithmic_bytes_per_launch": by, "peak_source": peak_src}
+    else:
+        nsum = float(window_sizes(L, w, dil).sum()) * B * H
+        fl = {"fwd": 4, "bwdA": 6, "bwdB": 8}[kinds[dom]] * d * nsum
+        ach = fl / (mean_k[dom] / 1e3) / 1e12
+        fma_peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12
+        roof = {"bound": "alu", "achieved": ach, "peak": fma_peak, "unit": "TFLOP/s",
+                "frac": ach / fma_peak, "traffic": None, "kernel": dom, "kernel_kind": kinds[dom],
+                "ms_per_launch": mean_k[dom],
+                "peak_source": "derived: 148 SM x 128 FP32 lanes x 2 flop x sm_max_mhz"}
+    tr_path = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tr_path):
+        try:
+            tr = json.load(open(tr_path)).get(f"{args.workload}/{args.dtype}/{kinds[dom]}")
+            if tr:
+                roof["traffic"] = tr["bytes_per_launch"]
+                roof["traffic_source"] = tr.get("source")
+        except Exception:
+            pass
+    step_alg = step_bytes_per_row(d, e) * rows * world
+    hbm_step = {"algorithmic_bytes_per_step": step_alg,
+                "achieved_gbs": step_alg / (elapsed_ms / args.steps / 1e3) / 1e9 / world,
+                "peak": hbm_peak, "frac": step_alg / (elapsed_ms / args.steps / 1e3) / 1e9 / world / hbm_peak}
+
+    # ---------------------------------------------------------------- e2e (pinned host buffers)
+    e2e = None
+    if rank == 0 or world > 1:
+        hq, hk, hv, hg = (x.cpu().pin_memory() for x in (q, k, v, g))
+        ho, hdq, hdk, hdv = (torch.empty_like(hq).pin_memory() for _ in range(4))
+        hl = torch.empty(lse.shape, dtype=torch.float32).pin_memory()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        e0, e1 = ev(), ev()
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            for dst, src in ((q, hq), (k, hk), (v, hv), (g, hg)):
+                dst.copy_(src, non_blocking=True)
+            step()
+            for dst, src in ((ho, out), (hl, lse), (hdq, dq), (hdk, dk), (hdv, dv)):
+                dst.copy_(src, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1)
+        if world > 1:
+            t = torch.tensor([ems], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": B * L * world * args.e2e_steps / (ems / 1e3), "unit": "tokens/s",
+               "h2d_bytes_per_step": 4 * q.numel() * e,
+               "d2h_bytes_per_step": 4 * q.numel() * e + lse.numel() * 4,
+               "steps": args.e2e_steps}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(shape, args.cpu_budget)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": args.dtype, "data": "synthetic: U(-1,1) q/k/v/dout generated on device",
+            "config": cfg,
+            "per_gpu_tokens_per_s": value / world,
+            "paths": {"fwd": "tc" if path_f == ft.PATH_TC else "simt",
+                      "bwd": "tc" if path_b == ft.PATH_TC else "simt"},
+            "kernel_ms": {n: sum(x) / len(x) for n, x in kdur.items()},
+            "roofline": roof, "hbm_step": hbm_step,
+            "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": args.steps * (nf + nb),
+            "clocks": sampler.summary(),
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

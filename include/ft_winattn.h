@@ -101,6 +101,13 @@ ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_
                           int64_t w, int64_t dilation, ft_dtype dtype,
                           int* path, int* num_launches);
 
+/* Profiling hook (off by default).  After ft_winattn_profile_events(evs, n) with n > 0,
+ * every subsequent fwd/bwd call on the calling host thread records evs[i] (cudaEvent_t
+ * handles passed as void*, created by the caller) on its stream right after its i-th
+ * kernel launch, for i < n, so a caller can time each kernel on the launching stream.
+ * ft_winattn_profile_events(NULL, 0) turns it off.  Always returns FT_OK. */
+ft_status ft_winattn_profile_events(void* const* events, int n);
+
 /* Human-readable text for a status (static storage, never NULL).  For FT_ERR_CUDA it
  * includes the CUDA error string of the last failure on the calling thread. */
 const char* ft_status_str(ft_status s);

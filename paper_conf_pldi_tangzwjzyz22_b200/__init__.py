@@ -18,7 +18,7 @@ import os
 
 import torch
 
-__all__ = ["fwd", "bwd", "plan", "WinAttn", "win_attn", "lib_path", "load_library",
+__all__ = ["fwd", "bwd", "plan", "profile_events", "WinAttn", "win_attn", "lib_path", "load_library",
            "FT_F32", "FT_BF16", "PATH_SIMT", "PATH_TC", "FtError"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -70,6 +70,8 @@ def load_library(build_if_missing: bool = False):
     lib.ft_status_str.argtypes = [ctypes.c_int]
     lib.ft_status_str.restype = ctypes.c_char_p
     lib.ft_winattn_abi_version.restype = ctypes.c_int
+    lib.ft_winattn_profile_events.argtypes = [ctypes.c_void_p, ctypes.c_int]
+    lib.ft_winattn_profile_events.restype = ctypes.c_int
     _lib = lib
     return lib
 
@@ -103,6 +105,25 @@ def _check_inputs(*ts: torch.Tensor):
 
 def _stream(device) -> int:
     return torch.cuda.current_stream(device).cuda_stream
+
+
+class profile_events:
+    """Context manager: record ``events[i]`` (torch.cuda.Event, timing enabled) right after
+    the i-th kernel launch of every fwd/bwd call made inside the block (C ABI
+    ft_winattn_profile_events).  Use a fresh list per call to time each launch."""
+
+    def __init__(self, events):
+        self.events = list(events)
+        self._arr = (ctypes.c_void_p * max(1, len(self.events)))(
+            *[ctypes.c_void_p(e.cuda_event) for e in self.events])
+
+    def __enter__(self):
+        load_library().ft_winattn_profile_events(ctypes.cast(self._arr, ctypes.c_void_p),
+                                                 len(self.events))
+        return self
+
+    def __exit__(self, *a):
+        load_library().ft_winattn_profile_events(None, 0)
 
 
 def plan(is_bwd: bool, batch: int, heads: int, seq_len: int, d: int, w: int, dilation: int,

@@ -16,6 +16,9 @@
 namespace {
 
 thread_local char g_cuda_msg[256] = "CUDA error";
+thread_local void* const* g_prof_events = nullptr;
+thread_local int g_prof_n = 0;
+thread_local int g_prof_i = 0;
 
 ft_status cuda_fail(cudaError_t e) {
     snprintf(g_cuda_msg, sizeof(g_cuda_msg), "FT_ERR_CUDA: %s (%s)", cudaGetErrorName(e),
@@ -71,7 +74,23 @@ ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w
 
 }  // namespace
 
+namespace ftw {
+void prof_reset() { g_prof_i = 0; }
+void prof_mark(cudaStream_t st) {
+    if (g_prof_events && g_prof_i < g_prof_n)
+        cudaEventRecord(static_cast<cudaEvent_t>(g_prof_events[g_prof_i]), st);
+    ++g_prof_i;
+}
+}  // namespace ftw
+
 extern "C" {
+
+ft_status ft_winattn_profile_events(void* const* events, int n) {
+    g_prof_events = n > 0 ? events : nullptr;
+    g_prof_n = n > 0 ? n : 0;
+    g_prof_i = 0;
+    return FT_OK;
+}
 
 int ft_winattn_abi_version(void) { return FT_WINATTN_ABI_VERSION; }
 
@@ -135,6 +154,7 @@ ft_status ft_winattn_fwd(const void* q, const void* k, const void* v, void* out,
 
     cudaStream_t st = (cudaStream_t)stream;
     cudaError_t e;
+    ftw::prof_reset();
     if (path == FT_PATH_TC) {
         int n = 0;
         e = ftw::tc_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, st, &n);
@@ -180,6 +200,7 @@ ft_status ft_winattn_bwd(const void* q, const void* k, const void* v, const void
     cudaStream_t st = (cudaStream_t)stream;
     float* Dws = (float*)workspace;
     cudaError_t e;
+    ftw::prof_reset();
     if (path == FT_PATH_TC) {
         int n = 0;
         e = ftw::tc_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w,

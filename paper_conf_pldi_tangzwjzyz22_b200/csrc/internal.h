@@ -65,4 +65,8 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
 int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
 int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
 
+// Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
+void prof_reset();
+void prof_mark(cudaStream_t st);
+
 }  // namespace ftw

@@ -517,6 +517,7 @@ cudaError_t fwd_impl(const void* q, const void* k, const void* v, void* out, flo
     set_smem_once(simt_fwd_kernel<Tin>, fwd_smem(d), once);
     simt_fwd_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_smem(d), st>>>(
         (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, g);
+    prof_mark(st);
     return cudaGetLastError();
 }
 
@@ -539,6 +540,7 @@ cudaError_t bwd_impl(const void* q, const void* k, const void* v, const void* ou
         simt_dq_kernel<Tin, 32><<<(unsigned)geo_blocks(g), NT, dq_smem(32, d), st>>>(
             (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dq, g);
     }
+    prof_mark(st);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
     if (T == 64) {
         set_smem_once(simt_dkdv_kernel<Tin, 64>, dkdv_smem(64, d), o3);
@@ -551,6 +553,7 @@ cudaError_t bwd_impl(const void* q, const void* k, const void* v, const void* ou
             (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dk,
             (Tin*)dv, g);
     }
+    prof_mark(st);
     return cudaGetLastError();
 }
 

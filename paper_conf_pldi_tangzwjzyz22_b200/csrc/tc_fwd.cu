@@ -296,6 +296,7 @@ cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float
         const int64_t Lr0 = ceil_div(L - r0, dil);   // longest residue of this group
         dim3 grid((unsigned)ceil_div(Lr0, BM), (unsigned)nr, (unsigned)units);
         tc_fwd_band_kernel<<<grid, NTHREADS, smem, st>>>(p);
+        prof_mark(st);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
         ++n;
