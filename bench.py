@@ -273,7 +273,10 @@ def main():
 
     # ---------------------------------------------------------------- timed region
     stream = torch.cuda.current_stream(dev)
-    ev = lambda: torch.cuda.Event(enable_timing=True)
+    def ev():
+        e_ = torch.cuda.Event(enable_timing=True)
+        e_.record(stream)   # materialise the CUDA event so its handle can go through the ABI
+        return e_
     starts, fevs, bevs, ends = [], [], [], []
     sampler = ClockSampler(dev.index if dev.index is not None else 0)
     if world > 1:

@@ -1,0 +1,501 @@
+// tc_band.cu -- tcgen05/TMEM tensor-core kernels of banded window attention for sm_100a
+// (bf16 storage; fp32 scores, softmax statistics and accumulators).
+//
+// One kernel template, three modes.  A CTA owns BM = 128 rows m0..m0+127 of one
+// (unit, residue) band problem and the NK = round_up(128 + 2w, 32) <= 256-row halo
+// m0-w .. m0+127+w of the other operand: the cached a[i:i+m] window of PAPER.md Fig. 14
+// (lines 402-423), staged by TMA instead of the (2w+1)-fold as_strided copy of Q that the
+// operator baseline makes (Fig. 1c).
+//
+//   FWD   rows = queries.  S = Q K_h^T -> row max, exp, row sum (the fused dot/max of
+//         Fig. 10 and dot_norm/softmax of Fig. 8), lse -> HBM,
+//         P (bf16) -> TMEM;  O_n = P V_h,n  (n = 64-column d-slices), scaled by 1/l.
+//   BWDQ  rows = queries.  S = Q K_h^T, dP = dO V_h^T;  P = exp(S - lse) (recomputed from the
+//         saved lse: selective materialization);  D = sum_j P dP (exact,
+//         written to the workspace);  dS = P (dP - D) (bf16) -> TMEM;  dQ_n = dS K_h,n.
+//   BWDKV rows = keys (tile ownership: each dk/dv row has exactly one writer, no atomics;
+//         the parallel-reduction choice of PAPER.md Fig. 13(d) over 13(e)).  S^T = K Q_h^T,
+//         dP^T = V dO_h^T;  P^T = exp(S^T - lse_col), dS^T = P^T (dP^T - D_col);
+//         dV_n = P^T dO_h,n,  dK_n = dS^T Q_h,n.
+//
+// Roles (192 threads): warps 0-3 softmax + epilogue (thread t <-> row m0+t <-> TMEM lane t),
+// warp 4 TMA producer + TMEM allocator, warp 5 MMA issuer (one elected thread).
+// The band geometry: column n of the halo is residue row m0 - w + n, and
+// |m_col - m_row| <= w  <=>  0 <= n - t <= 2w, so one mask serves all three modes.
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <mutex>
+
+#include "internal.h"
+#include "tc_common.cuh"
+#include "tmap.h"
+
+namespace ftw {
+namespace {
+
+using namespace tc;
+
+enum { FWD = 0, BWDQ = 1, BWDKV = 2 };
+
+constexpr int BM = 128;
+constexpr int NST = 2;           // smem pipeline stages
+constexpr int NTHREADS = 192;    // 4 softmax/epilogue warps + producer + MMA
+constexpr int RES_PER_LAUNCH = 4;
+constexpr uint32_t ABYTES = BM * 128;   // one 128-row x 64-col bf16 slice (SW128)
+constexpr uint32_t OSTG = BM * 128;     // one output staging slice
+constexpr float LOG2E = 1.4426950408889634f;
+constexpr float LN2 = 0.6931471805599453f;
+
+template <int MODE> struct Cfg {
+    static constexpr int NA = MODE == FWD ? 1 : 2;       // score GEMMs (S, and dP)
+    static constexpr int NO = MODE == BWDKV ? 2 : 1;     // output GEMMs per d-slice
+    static constexpr int NSTG = MODE == BWDKV ? 1 : 2;   // output staging buffers
+    static constexpr uint32_t TCOLS = MODE == FWD ? 256 : 512;
+};
+
+// a1/b1: first score GEMM (A rows m0.., B halo rows m0-w..), a2/b2: second (or, in FWD,
+// b2 = V for the output GEMM); o1/o2: outputs.
+struct Maps {
+    CUtensorMap a1, b1, a2, b2, o1, o2;
+};
+struct Params {
+    Maps maps[RES_PER_LAUNCH];
+    float* lse;   // FWD: written; BWD: read
+    float* D;     // BWDQ: written; BWDKV: read
+    int64_t L;
+    int d, w, dil, r0, NK, nsl;
+};
+
+template <int MODE>
+__host__ __device__ inline uint32_t stage_bytes(int NK) {
+    return Cfg<MODE>::NA * (ABYTES + (uint32_t)NK * 128u);
+}
+template <int MODE>
+inline size_t smem_bytes(int NK) {
+    return 1024 + NST * (size_t)stage_bytes<MODE>(NK) + Cfg<MODE>::NSTG * OSTG +
+           (MODE == BWDKV ? 2 * 256 * sizeof(float) : 0) + 256;
+}
+
+__device__ __forceinline__ bool band_ok(int n, int t, int w, int mcol, int Lr) {
+    return (unsigned)(n - t) <= (unsigned)(2 * w) && mcol >= 0 && mcol < Lr;
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_constant__ Params p) {
+    using C = Cfg<MODE>;
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t raw_u32 = smem_u32(smem_raw);
+    uint8_t* smem = smem_raw + (((raw_u32 + 1023u) & ~1023u) - raw_u32);
+
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    const int rl = blockIdx.y, u = blockIdx.z;
+    const int r = p.r0 + rl;
+    const int Lr = (int)((p.L - r + p.dil - 1) / p.dil);
+    const int m0 = blockIdx.x * BM;
+    if (m0 >= Lr) return;
+    const Maps& mp = p.maps[rl];
+    const int NK = p.NK, nsl = p.nsl, w = p.w;
+    const uint32_t SB = stage_bytes<MODE>(NK);
+    const uint32_t HB = (uint32_t)NK * 128u;   // one halo slice
+
+    uint8_t* ostg = smem + NST * SB;
+    float* colLse = reinterpret_cast<float*>(ostg + C::NSTG * OSTG);   // BWDKV only
+    float* colD = colLse + 256;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(ostg + C::NSTG * OSTG +
+                                                 (MODE == BWDKV ? 2 * 256 * sizeof(float) : 0));
+    uint64_t* full = bars;
+    uint64_t* empty = bars + NST;
+    uint64_t* s_full = bars + 2 * NST;
+    uint64_t* p_full = s_full + 1;
+    uint64_t* o_full = s_full + 2;    // [2]
+    uint64_t* o_empty = s_full + 4;   // [2]
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 6);
+
+    if (warp == 4) {
+        if (lane == 0) {
+            for (int i = 0; i < NST; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+            mbar_init(s_full, 1);
+            mbar_init(p_full, 128);
+            for (int i = 0; i < 2; ++i) { mbar_init(&o_full[i], 1); mbar_init(&o_empty[i], 128); }
+            fence_barrier_init();
+            tma_prefetch(&mp.a1); tma_prefetch(&mp.b1); tma_prefetch(&mp.b2); tma_prefetch(&mp.o1);
+            if (C::NA == 2) tma_prefetch(&mp.a2);
+            if (C::NO == 2) tma_prefetch(&mp.o2);
+        }
+        __syncwarp();
+        tmem_alloc(tmem_holder, C::TCOLS);
+        tmem_relinquish();
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tbase = *tmem_holder;
+
+    if (warp == 4) {
+        if (lane == 0) {   // ------------------------------------------------ TMA producer
+            int st = 0;
+            uint32_t ph = 0;
+            for (int s = 0; s < nsl; ++s) {
+                mbar_wait(&empty[st], ph ^ 1u);
+                uint8_t* sp = smem + st * SB;
+                mbar_arrive_expect_tx(&full[st], SB);
+                tma_load_3d(sp, &mp.a1, &full[st], s * 64, m0, u);
+                tma_load_3d(sp + ABYTES, &mp.b1, &full[st], s * 64, m0 - w, u);
+                if (C::NA == 2) {
+                    tma_load_3d(sp + ABYTES + HB, &mp.a2, &full[st], s * 64, m0, u);
+                    tma_load_3d(sp + 2 * ABYTES + HB, &mp.b2, &full[st], s * 64, m0 - w, u);
+                }
+                if (++st == NST) { st = 0; ph ^= 1u; }
+            }
+            for (int n = 0; n < nsl; ++n) {
+                mbar_wait(&empty[st], ph ^ 1u);
+                uint8_t* sp = smem + st * SB;
+                mbar_arrive_expect_tx(&full[st], C::NO * HB);
+                // output-GEMM B operands: FWD V (b2), BWDQ K (b1), BWDKV dO (b2) then Q (b1)
+                const CUtensorMap* m_first = MODE == BWDQ ? &mp.b1 : &mp.b2;
+                tma_load_3d(sp, m_first, &full[st], n * 64, m0 - w, u);
+                if (C::NO == 2) tma_load_3d(sp + HB, &mp.b1, &full[st], n * 64, m0 - w, u);
+                if (++st == NST) { st = 0; ph ^= 1u; }
+            }
+        }
+    } else if (warp == 5) {
+        if (lane == 0) {   // ------------------------------------------------ MMA issuer
+            const uint32_t idS = idesc_bf16(128, NK, false, false);
+            const uint32_t idO = idesc_bf16(128, 64, false, true);
+            int st = 0;
+            uint32_t ph = 0;
+            for (int s = 0; s < nsl; ++s) {
+                mbar_wait(&full[st], ph);
+                tc_fence_after();
+                const uint32_t a1 = smem_u32(smem + st * SB), b1 = a1 + ABYTES;
+#pragma unroll
+                for (int kk = 0; kk < 4; ++kk)
+                    mma_ss(tbase, sdesc_sw128(a1 + kk * 32, 16, 1024),
+                           sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
+                if (C::NA == 2) {
+                    const uint32_t a2 = b1 + HB, b2 = a2 + ABYTES;
+#pragma unroll
+                    for (int kk = 0; kk < 4; ++kk)
+                        mma_ss(tbase + 256, sdesc_sw128(a2 + kk * 32, 16, 1024),
+                               sdesc_sw128(b2 + kk * 32, 16, 1024), idS, (s | kk) != 0);
+                }
+                mma_commit(&empty[st]);
+                if (++st == NST) { st = 0; ph ^= 1u; }
+            }
+            mma_commit(s_full);
+            mbar_wait(p_full, 0);
+            tc_fence_after();
+            for (int n = 0; n < nsl; ++n) {
+                const int buf = n & 1;
+                if (n >= 2) {
+                    mbar_wait(&o_empty[buf], ((n >> 1) - 1) & 1);
+                    tc_fence_after();
+                }
+                mbar_wait(&full[st], ph);
+                tc_fence_after();
+                const uint32_t bb = smem_u32(smem + st * SB);
+#pragma unroll
+                for (int o = 0; o < C::NO; ++o) {
+                    // A operand in TMEM: P / dS / P^T at column 0, dS^T at column 256
+                    const uint32_t tA = tbase + (o == 1 ? 256u : 0u);
+                    const uint32_t tD = tbase + (o == 1 ? 384u : 128u) + 64u * buf;
+                    for (int kk = 0; kk < NK / 16; ++kk)
+                        mma_ts(tD, tA + kk * 8, sdesc_sw128(bb + o * HB + kk * 2048, HB, 1024), idO,
+                               kk != 0);
+                }
+                mma_commit(&empty[st]);
+                mma_commit(&o_full[buf]);
+                if (++st == NST) { st = 0; ph ^= 1u; }
+            }
+        }
+    } else {   // --------------------------------------------------------- softmax + epilogue
+        const int t = warp * 32 + lane;
+        const uint32_t trow = tbase + ((uint32_t)(warp * 32) << 16);
+        const int mrow = m0 + t;
+        const int kb = m0 - w;   // residue index of halo column 0
+        const int nch = NK / 32;
+        const int64_t rowbase = (int64_t)u * p.L + r;   // flat row of m = 0
+        float scale = 1.f;
+
+        if (MODE == BWDKV) {
+            for (int n = t; n < NK; n += 128) {
+                const int mc = kb + n;
+                const bool ok = mc >= 0 && mc < Lr;
+                colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
+                colD[n] = ok ? p.D[rowbase + (int64_t)mc * p.dil] : 0.f;
+            }
+            named_bar_sync(1, 128);
+        }
+        mbar_wait(s_full, 0);
+        tc_fence_after();
+
+        if (MODE == FWD) {
+            float mx = -INFINITY;
+            for (int c = 0; c < nch; ++c) {
+                uint32_t rr[32];
+                tmem_ld32(trow + c * 32, rr);
+                tmem_wait_ld();
+#pragma unroll
+                for (int e = 0; e < 32; ++e) {
+                    const int n = c * 32 + e;
+                    if (band_ok(n, t, w, kb + n, Lr)) mx = fmaxf(mx, __uint_as_float(rr[e]));
+                }
+            }
+            if (mx == -INFINITY) mx = 0.f;   // only rows beyond the sequence (never stored)
+            const float mxs = mx * LOG2E;
+            float sum = 0.f;
+            for (int c = 0; c < nch; ++c) {
+                uint32_t rr[32], pk[16];
+                tmem_ld32(trow + c * 32, rr);
+                tmem_wait_ld();
+#pragma unroll
+                for (int e = 0; e < 32; e += 2) {
+                    float pv[2];
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        const int n = c * 32 + e + h;
+                        pv[h] = band_ok(n, t, w, kb + n, Lr)
+                                    ? exp2f(fmaf(__uint_as_float(rr[e + h]), LOG2E, -mxs))
+                                    : 0.f;
+                        sum += pv[h];
+                    }
+                    pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
+                }
+                tmem_st16(trow + c * 16, pk);
+            }
+            tmem_wait_st();
+            tc_fence_before();
+            mbar_arrive(p_full);
+            if (mrow < Lr) p.lse[rowbase + (int64_t)mrow * p.dil] = (mxs + log2f(sum)) * LN2;
+            scale = 1.f / sum;
+        } else if (MODE == BWDQ) {
+            const float lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
+            float D = 0.f;
+            for (int c = 0; c < nch; ++c) {   // pass 1: D = sum_j P_ij dP_ij
+                uint32_t rs[32], rd[32];
+                tmem_ld32(trow + c * 32, rs);
+                tmem_ld32(trow + 256 + c * 32, rd);
+                tmem_wait_ld();
+#pragma unroll
+                for (int e = 0; e < 32; ++e) {
+                    const int n = c * 32 + e;
+                    const float pv = band_ok(n, t, w, kb + n, Lr)
+                                         ? exp2f(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2))
+                                         : 0.f;
+                    D = fmaf(pv, __uint_as_float(rd[e]), D);
+                }
+            }
+            for (int c = 0; c < nch; ++c) {   // pass 2: dS = P (dP - D) -> TMEM (bf16)
+                uint32_t rs[32], rd[32], pk[16];
+                tmem_ld32(trow + c * 32, rs);
+                tmem_ld32(trow + 256 + c * 32, rd);
+                tmem_wait_ld();
+#pragma unroll
+                for (int e = 0; e < 32; e += 2) {
+                    float dv[2];
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        const int n = c * 32 + e + h;
+                        const float pv = band_ok(n, t, w, kb + n, Lr)
+                                             ? exp2f(fmaf(__uint_as_float(rs[e + h]), LOG2E, -lse2))
+                                             : 0.f;
+                        dv[h] = pv * (__uint_as_float(rd[e + h]) - D);
+                    }
+                    pk[e / 2] = pack_bf16x2(dv[0], dv[1]);
+                }
+                tmem_st16(trow + c * 16, pk);
+            }
+            tmem_wait_st();
+            tc_fence_before();
+            mbar_arrive(p_full);
+            if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
+        } else {   // BWDKV: rows are keys, columns are halo queries
+            for (int c = 0; c < nch; ++c) {
+                uint32_t rs[32], rd[32], pk[16], dk[16];
+                tmem_ld32(trow + c * 32, rs);
+                tmem_ld32(trow + 256 + c * 32, rd);
+                tmem_wait_ld();
+#pragma unroll
+                for (int e = 0; e < 32; e += 2) {
+                    float pv[2], dv[2];
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        const int n = c * 32 + e + h;
+                        pv[h] = band_ok(n, t, w, kb + n, Lr)
+                                    ? exp2f(fmaf(__uint_as_float(rs[e + h]), LOG2E, -colLse[n]))
+                                    : 0.f;
+                        dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
+                    }
+                    pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
+                    dk[e / 2] = pack_bf16x2(dv[0], dv[1]);
+                }
+                tmem_st16(trow + c * 16, pk);
+                tmem_st16(trow + 256 + c * 16, dk);
+            }
+            tmem_wait_st();
+            tc_fence_before();
+            mbar_arrive(p_full);
+        }
+
+        // ----------------------------------------------------------- epilogue: d-slices
+        int sidx = 0;   // output slices issued (staging ring position)
+        for (int n = 0; n < nsl; ++n) {
+            const int buf = n & 1;
+            mbar_wait(&o_full[buf], (n >> 1) & 1);
+            tc_fence_after();
+#pragma unroll
+            for (int o = 0; o < C::NO; ++o) {
+                uint32_t ov[64];
+                const uint32_t tcol = (o == 1 ? 384u : 128u) + 64u * buf;
+                tmem_ld32(trow + tcol, *reinterpret_cast<uint32_t(*)[32]>(&ov[0]));
+                tmem_ld32(trow + tcol + 32, *reinterpret_cast<uint32_t(*)[32]>(&ov[32]));
+                tmem_wait_ld();
+                if (o == C::NO - 1) {
+                    tc_fence_before();
+                    mbar_arrive(&o_empty[buf]);
+                }
+                uint8_t* stg = ostg + (sidx % C::NSTG) * OSTG;
+                if (t == 0 && sidx >= C::NSTG) tma_store_wait_read<C::NSTG - 1>();
+                named_bar_sync(1, 128);
+#pragma unroll
+                for (int c = 0; c < 8; ++c) {
+                    uint4 val;
+                    val.x = pack_bf16x2(__uint_as_float(ov[8 * c + 0]) * scale, __uint_as_float(ov[8 * c + 1]) * scale);
+                    val.y = pack_bf16x2(__uint_as_float(ov[8 * c + 2]) * scale, __uint_as_float(ov[8 * c + 3]) * scale);
+                    val.z = pack_bf16x2(__uint_as_float(ov[8 * c + 4]) * scale, __uint_as_float(ov[8 * c + 5]) * scale);
+                    val.w = pack_bf16x2(__uint_as_float(ov[8 * c + 6]) * scale, __uint_as_float(ov[8 * c + 7]) * scale);
+                    *reinterpret_cast<uint4*>(stg + t * 128 + ((c ^ (t & 7)) * 16)) = val;
+                }
+                fence_proxy_async_smem();
+                named_bar_sync(1, 128);
+                if (t == 0) {
+                    tma_store_3d(o == 1 ? &mp.o2 : &mp.o1, stg, n * 64, m0, u);
+                    tma_store_commit();
+                }
+                ++sidx;
+            }
+        }
+        if (t == 0) tma_store_wait_all<0>();
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 4) {
+        tc_fence_after();
+        tmem_dealloc(tbase, C::TCOLS);
+    }
+}
+
+template <int MODE>
+void set_attr_once() {
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaFuncSetAttribute(tc_band_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             227 * 1024);
+    });
+}
+
+int halo_rows(int64_t L, int64_t w) {
+    const int64_t wc = w < L ? w : L;
+    return (int)(((BM + 2 * wc) + 31) / 32 * 32);
+}
+
+// maps: per residue, (a1, b1, a2, b2, o1, o2) tensors; box rows BM for a/o, NK for b.
+template <int MODE>
+cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b2, void* o1,
+                   void* o2, float* lse, float* D, int64_t B, int64_t H, int64_t L, int64_t d,
+                   int64_t w, int64_t dil, cudaStream_t st, int* launches) {
+    const int64_t wc = w < L ? w : L;
+    const int NK = halo_rows(L, w);
+    const int64_t units = B * H;
+    const int64_t nres = dil < L ? dil : L;
+    set_attr_once<MODE>();
+    int n = 0;
+    for (int64_t r0 = 0; r0 < nres; r0 += RES_PER_LAUNCH) {
+        Params p;
+        memset(&p, 0, sizeof(p));
+        const int nr = (int)(nres - r0 < RES_PER_LAUNCH ? nres - r0 : RES_PER_LAUNCH);
+        for (int i = 0; i < nr; ++i) {
+            const int64_t r = r0 + i;
+            Maps& m = p.maps[i];
+            bool ok = make_residue_map(&m.a1, a1, L, d, units, dil, r, BM) &&
+                      make_residue_map(&m.b1, b1, L, d, units, dil, r, NK) &&
+                      make_residue_map(&m.b2, b2, L, d, units, dil, r, NK) &&
+                      make_residue_map(&m.o1, o1, L, d, units, dil, r, BM);
+            if (ok && a2) ok = make_residue_map(&m.a2, a2, L, d, units, dil, r, BM);
+            if (ok && o2) ok = make_residue_map(&m.o2, o2, L, d, units, dil, r, BM);
+            if (!ok) return cudaErrorInvalidValue;
+        }
+        p.lse = lse;
+        p.D = D;
+        p.L = L;
+        p.d = (int)d;
+        p.w = (int)wc;
+        p.dil = (int)dil;
+        p.r0 = (int)r0;
+        p.NK = NK;
+        p.nsl = (int)(d / 64);
+        const int64_t Lr0 = ceil_div(L - r0, dil);   // longest residue of this group
+        dim3 grid((unsigned)ceil_div(Lr0, BM), (unsigned)nr, (unsigned)units);
+        tc_band_kernel<MODE><<<grid, NTHREADS, smem_bytes<MODE>(NK), st>>>(p);
+        prof_mark(st);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        ++n;
+    }
+    if (launches) *launches += n;
+    return cudaSuccess;
+}
+
+bool band_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    const int64_t wc = w < L ? w : L;
+    return d % 64 == 0 && d <= 512 && wc <= 64 && dil <= 256 && units <= 65535;
+}
+
+int band_launches(int64_t L, int64_t dil) {
+    const int64_t nres = dil < L ? dil : L;
+    return (int)ceil_div(nres, RES_PER_LAUNCH);
+}
+
+}  // namespace
+
+bool tc_fwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    return band_supported(units, L, d, w, dil);
+}
+bool tc_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    return band_supported(units, L, d, w, dil);
+}
+int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
+    (void)d; (void)w;
+    return band_launches(L, dil);
+}
+int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
+    (void)d; (void)w;
+    return 2 * band_launches(L, dil);
+}
+
+cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B,
+                   int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
+                   int* launches) {
+    if (launches) *launches = 0;
+    return launch<FWD>(q, k, nullptr, v, out, nullptr, lse, nullptr, B, H, L, d, w, dil, st,
+                       launches);
+}
+
+cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
+                   const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
+                   int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                   cudaStream_t st, int* launches) {
+    (void)out;   // D_i is recomputed exactly as sum_j P_ij dP_ij by the BWDQ kernel
+    if (launches) *launches = 0;
+    cudaError_t e = launch<BWDQ>(q, k, dout, v, dq, nullptr, const_cast<float*>(lse), Dws, B, H,
+                                 L, d, w, dil, st, launches);
+    if (e != cudaSuccess) return e;
+    return launch<BWDKV>(k, q, v, dout, dv, dk, const_cast<float*>(lse), Dws, B, H, L, d, w, dil,
+                         st, launches);
+}
+
+}  // namespace ftw
