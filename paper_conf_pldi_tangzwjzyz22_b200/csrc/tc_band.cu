@@ -50,12 +50,33 @@ constexpr uint32_t OSTG = BM * 128;     // one output staging slice
 constexpr float LOG2E = 1.4426950408889634f;
 constexpr float LN2 = 0.6931471805599453f;
 
+// TMEM layout (columns).  Score accumulators: S at 0, dP at 256.  The bf16 A operands of
+// the output GEMMs overwrite them as they are consumed: "compact" = 16 columns per 32-column
+// score chunk at 16c; "split" = hi/lo bf16 pair (x = hi + lo, lo = bf16(x - hi)) in place of
+// chunk c: hi at 32c, lo at 32c+16.  dS is split because at large d its entries reach O(10)
+// and a single bf16 rounding (2^-9) of them would dominate the dq/dk error budget.
 template <int MODE> struct Cfg {
     static constexpr int NA = MODE == FWD ? 1 : 2;       // score GEMMs (S, and dP)
     static constexpr int NO = MODE == BWDKV ? 2 : 1;     // output GEMMs per d-slice
     static constexpr int NSTG = MODE == BWDKV ? 1 : 2;   // output staging buffers
     static constexpr uint32_t TCOLS = MODE == FWD ? 256 : 512;
+    static constexpr bool SPLIT0 = MODE == BWDQ;         // A of output GEMM 0 split?
+    static constexpr bool SPLIT1 = MODE == BWDKV;        // A of output GEMM 1 split?
+    static constexpr uint32_t A0 = 0, A1 = 256;          // A operand bases
+    static constexpr uint32_t OUT0 = MODE == BWDQ ? 256 : 128;   // output accumulators
+    static constexpr uint32_t OUT1 = 192;
+    static constexpr int OBUFS = MODE == BWDKV ? 1 : 2;  // TMEM output buffers per output
 };
+
+__device__ __forceinline__ uint32_t a_col(bool split, int kk) {
+    return split ? 32u * (kk >> 1) + 8u * (kk & 1) : 8u * kk;
+}
+__device__ __forceinline__ void split_bf16x2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(x0, x1);
+    const float2 hf = __bfloat1622float2(h);
+    hi = *reinterpret_cast<uint32_t*>(&h);
+    lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
+}
 
 // a1/b1: first score GEMM (A rows m0.., B halo rows m0-w..), a2/b2: second (or, in FWD,
 // b2 = V for the output GEMM); o1/o2: outputs.
@@ -190,9 +211,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             mbar_wait(p_full, 0);
             tc_fence_after();
             for (int n = 0; n < nsl; ++n) {
-                const int buf = n & 1;
-                if (n >= 2) {
-                    mbar_wait(&o_empty[buf], ((n >> 1) - 1) & 1);
+                const int buf = n % C::OBUFS;
+                if (n >= C::OBUFS) {
+                    mbar_wait(&o_empty[buf], ((n / C::OBUFS) - 1) & 1);
                     tc_fence_after();
                 }
                 mbar_wait(&full[st], ph);
@@ -200,12 +221,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 const uint32_t bb = smem_u32(smem + st * SB);
 #pragma unroll
                 for (int o = 0; o < C::NO; ++o) {
-                    // A operand in TMEM: P / dS / P^T at column 0, dS^T at column 256
-                    const uint32_t tA = tbase + (o == 1 ? 256u : 0u);
-                    const uint32_t tD = tbase + (o == 1 ? 384u : 128u) + 64u * buf;
-                    for (int kk = 0; kk < NK / 16; ++kk)
-                        mma_ts(tD, tA + kk * 8, sdesc_sw128(bb + o * HB + kk * 2048, HB, 1024), idO,
-                               kk != 0);
+                    const bool split = o == 0 ? C::SPLIT0 : C::SPLIT1;
+                    const uint32_t tA = tbase + (o == 0 ? C::A0 : C::A1);
+                    const uint32_t tD = tbase + (o == 0 ? C::OUT0 : C::OUT1) + 64u * buf;
+                    for (int kk = 0; kk < NK / 16; ++kk) {
+                        const uint64_t bd = sdesc_sw128(bb + o * HB + kk * 2048, HB, 1024);
+                        mma_ts(tD, tA + a_col(split, kk), bd, idO, kk != 0);
+                        if (split) mma_ts(tD, tA + a_col(split, kk) + 16, bd, idO, 1);
+                    }
                 }
                 mma_commit(&empty[st]);
                 mma_commit(&o_full[buf]);
@@ -289,8 +312,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     D = fmaf(pv, __uint_as_float(rd[e]), D);
                 }
             }
-            for (int c = 0; c < nch; ++c) {   // pass 2: dS = P (dP - D) -> TMEM (bf16)
-                uint32_t rs[32], rd[32], pk[16];
+            for (int c = 0; c < nch; ++c) {   // pass 2: dS = P (dP - D) -> TMEM (bf16 hi/lo)
+                uint32_t rs[32], rd[32], pk[16], pl[16];
                 tmem_ld32(trow + c * 32, rs);
                 tmem_ld32(trow + 256 + c * 32, rd);
                 tmem_wait_ld();
@@ -305,9 +328,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                                              : 0.f;
                         dv[h] = pv * (__uint_as_float(rd[e + h]) - D);
                     }
-                    pk[e / 2] = pack_bf16x2(dv[0], dv[1]);
+                    split_bf16x2(dv[0], dv[1], pk[e / 2], pl[e / 2]);
                 }
-                tmem_st16(trow + c * 16, pk);
+                tmem_st16(trow + C::A0 + c * 32, pk);
+                tmem_st16(trow + C::A0 + c * 32 + 16, pl);
             }
             tmem_wait_st();
             tc_fence_before();
@@ -315,7 +339,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
         } else {   // BWDKV: rows are keys, columns are halo queries
             for (int c = 0; c < nch; ++c) {
-                uint32_t rs[32], rd[32], pk[16], dk[16];
+                uint32_t rs[32], rd[32], pk[16], dk[16], dl[16];
                 tmem_ld32(trow + c * 32, rs);
                 tmem_ld32(trow + 256 + c * 32, rd);
                 tmem_wait_ld();
@@ -331,10 +355,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
                     }
                     pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
-                    dk[e / 2] = pack_bf16x2(dv[0], dv[1]);
+                    split_bf16x2(dv[0], dv[1], dk[e / 2], dl[e / 2]);
                 }
-                tmem_st16(trow + c * 16, pk);
-                tmem_st16(trow + 256 + c * 16, dk);
+                tmem_st16(trow + C::A0 + c * 16, pk);
+                tmem_st16(trow + C::A1 + c * 32, dk);
+                tmem_st16(trow + C::A1 + c * 32 + 16, dl);
             }
             tmem_wait_st();
             tc_fence_before();
@@ -344,13 +369,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
         // ----------------------------------------------------------- epilogue: d-slices
         int sidx = 0;   // output slices issued (staging ring position)
         for (int n = 0; n < nsl; ++n) {
-            const int buf = n & 1;
-            mbar_wait(&o_full[buf], (n >> 1) & 1);
+            const int buf = n % C::OBUFS;
+            mbar_wait(&o_full[buf], (n / C::OBUFS) & 1);
             tc_fence_after();
 #pragma unroll
             for (int o = 0; o < C::NO; ++o) {
                 uint32_t ov[64];
-                const uint32_t tcol = (o == 1 ? 384u : 128u) + 64u * buf;
+                const uint32_t tcol = (o == 0 ? C::OUT0 : C::OUT1) + 64u * buf;
                 tmem_ld32(trow + tcol, *reinterpret_cast<uint32_t(*)[32]>(&ov[0]));
                 tmem_ld32(trow + tcol + 32, *reinterpret_cast<uint32_t(*)[32]>(&ov[32]));
                 tmem_wait_ld();
