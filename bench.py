@@ -359,7 +359,7 @@ def main():
 
     # ---------------------------------------------------------------- e2e (pinned host buffers)
     e2e = None
-    if rank == 0 or world > 1:
+    if args.e2e_steps > 0:
         hq, hk, hv, hg = (x.cpu().pin_memory() for x in (q, k, v, g))
         ho, hdq, hdk, hdv = (torch.empty_like(hq).pin_memory() for _ in range(4))
         hl = torch.empty(lse.shape, dtype=torch.float32).pin_memory()
