@@ -108,6 +108,13 @@ ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_
  * ft_winattn_profile_events(NULL, 0) turns it off.  Always returns FT_OK. */
 ft_status ft_winattn_profile_events(void* const* events, int n);
 
+/* Debug trace (off by default): while device_buffer is non-NULL, tensor-core kernels of
+ * the given mode (0 = forward, 1 = backward dq, 2 = backward dk/dv) launched from the
+ * calling host thread write globaltimer stamps of their pipeline phases into it:
+ * uint64 [gridDim.x][8 tiles][10 events] (layout documented in csrc/tc_band.cu).  The
+ * buffer must hold 148*8*10*8 bytes per SM-sized grid.  Profiling only. */
+ft_status ft_winattn_debug_trace(int kernel_mode, void* device_buffer);
+
 /* Human-readable text for a status (static storage, never NULL).  For FT_ERR_CUDA it
  * includes the CUDA error string of the last failure on the calling thread. */
 const char* ft_status_str(ft_status s);

@@ -19,6 +19,7 @@ thread_local char g_cuda_msg[256] = "CUDA error";
 thread_local void* const* g_prof_events = nullptr;
 thread_local int g_prof_n = 0;
 thread_local int g_prof_i = 0;
+thread_local void* g_trace[3] = {nullptr, nullptr, nullptr};
 
 ft_status cuda_fail(cudaError_t e) {
     snprintf(g_cuda_msg, sizeof(g_cuda_msg), "FT_ERR_CUDA: %s (%s)", cudaGetErrorName(e),
@@ -76,6 +77,7 @@ ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w
 
 namespace ftw {
 void prof_reset() { g_prof_i = 0; }
+void* trace_buffer(int mode) { return (mode >= 0 && mode < 3) ? g_trace[mode] : nullptr; }
 void prof_mark(cudaStream_t st) {
     if (g_prof_events && g_prof_i < g_prof_n)
         cudaEventRecord(static_cast<cudaEvent_t>(g_prof_events[g_prof_i]), st);
@@ -84,6 +86,12 @@ void prof_mark(cudaStream_t st) {
 }  // namespace ftw
 
 extern "C" {
+
+ft_status ft_winattn_debug_trace(int kernel_mode, void* device_buffer) {
+    if (kernel_mode < 0 || kernel_mode > 2) return FT_ERR_INVALID_VALUE;
+    g_trace[kernel_mode] = device_buffer;
+    return FT_OK;
+}
 
 ft_status ft_winattn_profile_events(void* const* events, int n) {
     g_prof_events = n > 0 ? events : nullptr;

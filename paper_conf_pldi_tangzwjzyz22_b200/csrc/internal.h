@@ -67,6 +67,7 @@ int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
 
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();
+void* trace_buffer(int kernel_mode);   // ft_winattn_debug_trace target for a kernel mode, or null
 void prof_mark(cudaStream_t st);
 
 }  // namespace ftw

@@ -1,0 +1,159 @@
+// tools/mma_microbench.cu -- cycles per tcgen05.mma (kind::f16, M=128, K=16) for the operand
+// shapes the band kernels use.  Profiling aid, not part of the library.
+//   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -I paper_conf_pldi_tangzwjzyz22_b200/csrc \
+//        tools/mma_microbench.cu -o /tmp/mma_mb && /tmp/mma_mb
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "tc_common.cuh"
+
+using namespace ftw::tc;
+
+// whole-warp variants: all 32 lanes execute, one elected lane issues
+__device__ __forceinline__ void mma_ss_w(uint32_t d, uint64_t a, uint64_t b, uint32_t id, uint32_t acc) {
+    asm volatile("{\n\t.reg .pred p, e;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+                 :: "r"(d), "l"(a), "l"(b), "r"(id), "r"(acc) : "memory");
+}
+__device__ __forceinline__ void mma_ts_w(uint32_t d, uint32_t a, uint64_t b, uint32_t id, uint32_t acc) {
+    asm volatile("{\n\t.reg .pred p, e;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}"
+                 :: "r"(d), "r"(a), "l"(b), "r"(id), "r"(acc) : "memory");
+}
+__device__ __forceinline__ void commit_w(uint64_t* bar) {
+    asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+                 "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}"
+                 :: "r"(smem_u32(bar)) : "memory");
+}
+
+__global__ void bench_w(int mode, int N, int nacc, int iters, unsigned long long* out) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    __shared__ uint32_t holder;
+    __shared__ uint64_t bar;
+    const int warp = threadIdx.x / 32;
+    for (int i = threadIdx.x; i < 64 * 1024 / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(smem)[i] = 0;
+    if (warp == 0) { tmem_alloc(&holder, 512); tmem_relinquish(); }
+    if (threadIdx.x == 32) { mbar_init(&bar, 1); fence_barrier_init(); }
+    fence_proxy_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tb = holder;
+    if (warp == 1) {
+        const uint32_t sa = smem_u32(smem), sb = sa + 16384;
+        const uint32_t id = idesc_bf16(128, N, false, mode == 1);
+        for (int i = 0; i < 16; ++i)
+            for (int a = 0; a < nacc; ++a) {
+                const uint32_t d = mode == 0 ? tb + (nacc > 2 ? 128 : 256) * a : tb + 128 + 128 * a;
+                if (mode == 0) mma_ss_w(d, sdesc_sw128(sa, 16, 1024), sdesc_sw128(sb, 16, 1024), id, 1);
+                else mma_ts_w(d, tb, sdesc_sw128(sb, 8192, 1024), id, 1);
+            }
+        commit_w(&bar);
+        mbar_wait(&bar, 0);
+        unsigned long long t0 = clock64();
+        for (int i = 0; i < iters; ++i)
+            for (int a = 0; a < nacc; ++a) {
+                const uint32_t d = mode == 0 ? tb + (nacc > 2 ? 128 : 256) * a : tb + 128 + 128 * a;
+                const int kk = i & 3;
+                if (mode == 0)
+                    mma_ss_w(d, sdesc_sw128(sa + kk * 32, 16, 1024), sdesc_sw128(sb + kk * 32, 16, 1024), id, 1);
+                else
+                    mma_ts_w(d, tb + kk * 8, sdesc_sw128(sb + kk * 2048, 8192, 1024), id, 1);
+            }
+        commit_w(&bar);
+        mbar_wait(&bar, 1);
+        unsigned long long t1 = clock64();
+        if (threadIdx.x == 32) out[blockIdx.x] = t1 - t0;
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) { tc_fence_after(); tmem_dealloc(tb, 512); }
+}
+
+// mode 0: SS (A K-major smem, B K-major smem), mode 1: TS (A tmem, B MN-major smem)
+__global__ void bench(int mode, int N, int nacc, int iters, unsigned long long* out, int M = 128) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    __shared__ uint32_t holder;
+    __shared__ uint64_t bar;
+    const int warp = threadIdx.x / 32;
+    for (int i = threadIdx.x; i < 64 * 1024 / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(smem)[i] = 0;
+    if (warp == 0) { tmem_alloc(&holder, 512); tmem_relinquish(); }
+    if (threadIdx.x == 32) { mbar_init(&bar, 1); fence_barrier_init(); }
+    fence_proxy_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tb = holder;
+    if (threadIdx.x == 32) {
+        const uint32_t sa = smem_u32(smem), sb = sa + 16384;
+        const uint32_t id = idesc_bf16(M, N, false, mode == 1);
+        // warm up
+        for (int i = 0; i < 16; ++i)
+            for (int a = 0; a < nacc; ++a) {
+                const uint32_t d = mode == 0 ? tb + (nacc > 2 ? 128 : 256) * a : tb + 128 + 128 * a;
+                if (mode == 0) mma_ss(d, sdesc_sw128(sa, 16, 1024), sdesc_sw128(sb, 16, 1024), id, 1);
+                else mma_ts(d, tb, sdesc_sw128(sb, 8192, 1024), id, 1);
+            }
+        mma_commit(&bar);
+        mbar_wait(&bar, 0);
+        unsigned long long t0 = clock64();
+        for (int i = 0; i < iters; ++i)
+            for (int a = 0; a < nacc; ++a) {
+                const uint32_t d = mode == 0 ? tb + (nacc > 2 ? 128 : 256) * a : tb + 128 + 128 * a;
+                const int kk = i & 3;
+                if (mode == 0)
+                    mma_ss(d, sdesc_sw128(sa + kk * 32, 16, 1024), sdesc_sw128(sb + kk * 32, 16, 1024), id, 1);
+                else
+                    mma_ts(d, tb + kk * 8, sdesc_sw128(sb + kk * 2048, 8192, 1024), id, 1);
+            }
+        mma_commit(&bar);
+        mbar_wait(&bar, 1);
+        unsigned long long t1 = clock64();
+        out[blockIdx.x] = t1 - t0;
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) { tc_fence_after(); tmem_dealloc(tb, 512); }
+}
+
+int main() {
+    unsigned long long* d;
+    cudaMalloc(&d, 8 * 148);
+    cudaFuncSetAttribute(bench, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+    cudaFuncSetAttribute(bench_w, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+    const int iters = 2048;
+    for (int N : {64, 128, 256})
+        for (int nacc : {1, 2, 4}) {
+            if (N == 256 && nacc == 4) continue;
+            bench<<<148, 128, 96 * 1024>>>(0, N, nacc, iters, d, 64);
+            unsigned long long h[148] = {0};
+            cudaMemcpy(h, d, 8 * 148, cudaMemcpyDeviceToHost);
+            double mx = 0;
+            for (int i = 0; i < 148; ++i) mx = h[i] > mx ? h[i] : mx;
+            const double per = mx / (iters * nacc);
+            printf("lane0 SS M= 64 N=%3d acc=%d grid=148: %6.1f clk/MMA  %5.0f MAC/clk/SM\n", N, nacc, per,
+                   64.0 * N * 16 / per);
+        }
+    struct Cfg { int variant, mode, N, nacc, grid; };
+    Cfg cfgs[] = {
+        {0, 0, 64, 1, 1}, {0, 0, 64, 4, 1}, {0, 0, 128, 1, 1}, {0, 0, 128, 4, 1},
+        {0, 0, 256, 1, 1}, {0, 0, 256, 1, 148}, {0, 0, 128, 4, 148}, {0, 0, 64, 4, 148},
+        {1, 0, 256, 1, 148}, {1, 0, 128, 4, 148}, {0, 1, 64, 2, 148}, {0, 1, 128, 2, 148},
+        {0, 1, 256, 1, 148},
+    };
+    for (const Cfg& c : cfgs) {
+        if (c.variant == 0) bench<<<c.grid, 128, 96 * 1024>>>(c.mode, c.N, c.nacc, iters, d);
+        else bench_w<<<c.grid, 128, 96 * 1024>>>(c.mode, c.N, c.nacc, iters, d);
+        unsigned long long h[148] = {0};
+        cudaError_t e = cudaMemcpy(h, d, 8 * c.grid, cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) { printf("err %s\n", cudaGetErrorString(e)); return 1; }
+        double mx = 0;
+        for (int i = 0; i < c.grid; ++i) mx = h[i] > mx ? h[i] : mx;
+        const double per = mx / (iters * c.nacc);
+        printf("%s %s M=128 N=%3d acc=%d grid=%3d: %6.1f clk/MMA (floor %3d) %5.0f MAC/clk/SM\n",
+               c.variant == 0 ? "lane0" : "warp ", c.mode == 0 ? "SS" : "TS", c.N, c.nacc, c.grid,
+               per, 128 * c.N / 256, 128.0 * c.N * 16 / per);
+    }
+    return 0;
+}

@@ -1,0 +1,75 @@
+"""Phase timeline of the tensor-core kernels from ft_winattn_debug_trace (profiling aid).
+
+    python tools/trace_phases.py [--workload C2a]
+
+Prints, per kernel mode, the median over CTAs/tiles of each pipeline phase (microseconds).
+"""
+import argparse
+import ctypes
+import os
+import sys
+
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import bench  # noqa: E402
+import paper_conf_pldi_tangzwjzyz22_b200 as ft  # noqa: E402
+
+EV = ["prod_g1_start", "prod_out_end", "mma_g1_ready", "mma_s_commit", "mma_p_seen",
+      "mma_out_end", "sm_s_seen", "sm_p_arrive", "epi_first", "epi_done"]
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="C2a")
+    a = ap.parse_args()
+    B, H, L, d, w, dil, _ = bench.WORKLOADS[a.workload]
+    lib = ft.load_library()
+    lib.ft_winattn_debug_trace.argtypes = [ctypes.c_int, ctypes.c_void_p]
+    dev = torch.device("cuda:0")
+    x = [(torch.rand(B, H, L, d, device=dev) * 2 - 1).to(torch.bfloat16) for _ in range(4)]
+    q, k, v, g = x
+    out, lse = ft.fwd(q, k, v, w, dil)
+    ft.bwd(q, k, v, out, lse, g, w, dil)
+    torch.cuda.synchronize()
+    bufs = [torch.zeros(148 * 8 * 48, dtype=torch.int64, device=dev) for _ in range(3)]
+    for m in range(3):
+        lib.ft_winattn_debug_trace(m, bufs[m].data_ptr())
+    out, lse = ft.fwd(q, k, v, w, dil)
+    ft.bwd(q, k, v, out, lse, g, w, dil)
+    torch.cuda.synchronize()
+    for m in range(3):
+        lib.ft_winattn_debug_trace(m, None)
+    for m, name in enumerate(["FWD", "BWDQ", "BWDKV"]):
+        t = bufs[m].view(148, 8, 48).cpu().double()
+        valid = (t[:, :, :10] > 0).all(dim=2)
+        t0 = t[:, 0, 0][t[:, 0, 0] > 0].min()
+        t = (t - t0) / 1e3
+        print(f"== {name}: kernel span {t[valid].max():.1f} us, tiles traced {int(valid.sum())}")
+        def med(x):
+            return float(x[valid].median())
+        print(f"  GEMM1 (mma ready -> s commit)     {med(t[:,:,3]-t[:,:,2]):7.2f} us")
+        print(f"  s commit -> softmax start         {med(t[:,:,6]-t[:,:,3]):7.2f}")
+        print(f"  softmax (s seen -> p arrive)      {med(t[:,:,7]-t[:,:,6]):7.2f}")
+        print(f"  p arrive -> mma sees p            {med(t[:,:,4]-t[:,:,7]):7.2f}")
+        print(f"  output MMAs issued (p -> out end) {med(t[:,:,5]-t[:,:,4]):7.2f}")
+        print(f"  epilogue (first o_full -> done)   {med(t[:,:,9]-t[:,:,8]):7.2f}")
+        print(f"  tile period (g1 ready j -> j+1)   {float((t[:,1:,2]-t[:,:-1,2])[valid[:,1:] & valid[:,:-1]].median()):7.2f}")
+        print(f"  producer span per tile            {med(t[:,:,1]-t[:,:,0]):7.2f}")
+        print(f"  first tile start (median over CTAs) {float(t[:,0,2][valid[:,0]].median()):7.2f}")
+        # per-slice detail for local tile 1 (steady state), relative to its p_full seen by MMA
+        jj = 1
+        v1 = valid[:, jj]
+        base = t[:, jj, 4]
+        rows = []
+        for n in range(8):
+            f = lambda e: float((t[:, jj, e] - base)[v1].median())
+            rows.append(f"    slice {n}: mma o_empty {f(18+n):6.2f}  mma stage-full {f(10+n):6.2f}  "
+                        f"epi o_full {f(26+n):6.2f}  epi stored {f(34+n):6.2f}")
+        print("  per-slice (tile 1, us after MMA saw p_full):")
+        print("\n".join(rows))
+
+
+if __name__ == "__main__":
+    main()
