@@ -65,6 +65,17 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
 int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
 int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
 
+// wide-window tensor-core kernels -- tc_chunk.cu (used when 128 + 2w > 256)
+bool tc_chunk_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+cudaError_t tc_chunk_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
+                         int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                         cudaStream_t st, int* launches);
+cudaError_t tc_chunk_bwd(const void* q, const void* k, const void* v, const float* lse,
+                         const void* dout, void* dq, void* dk, void* dv, float* Dws, int64_t B,
+                         int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
+                         int* launches);
+int tc_chunk_launches(int64_t L, int64_t dil);
+
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();
 void* trace_buffer(int kernel_mode);   // ft_winattn_debug_trace target for a kernel mode, or null

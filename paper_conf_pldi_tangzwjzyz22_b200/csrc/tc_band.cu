@@ -690,24 +690,26 @@ int band_launches(int64_t L, int64_t dil) {
 }  // namespace
 
 bool tc_fwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
-    return band_supported(units, L, d, w, dil);
+    return halo_rows(L, w) <= 256 ? band_supported(units, L, d, w, dil)
+                                  : tc_chunk_supported(units, L, d, w, dil);
 }
 bool tc_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
-    return band_supported(units, L, d, w, dil);
+    return tc_fwd_supported(units, L, d, w, dil);
 }
 int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
-    (void)d; (void)w;
-    return band_launches(L, dil);
+    (void)d;
+    return halo_rows(L, w) <= 256 ? band_launches(L, dil) : tc_chunk_launches(L, dil);
 }
 int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
-    (void)d; (void)w;
-    return 2 * band_launches(L, dil);
+    return 2 * tc_fwd_launches(L, d, w, dil);
 }
 
 cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B,
                    int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
                    int* launches) {
     if (launches) *launches = 0;
+    if (halo_rows(L, w) > 256)
+        return tc_chunk_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
     return launch<FWD>(q, k, nullptr, v, out, nullptr, lse, nullptr, B, H, L, d, w, dil, st,
                        launches);
 }
@@ -718,6 +720,8 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
                    cudaStream_t st, int* launches) {
     (void)out;   // D_i is recomputed exactly as sum_j P_ij dP_ij by the BWDQ kernel
     if (launches) *launches = 0;
+    if (halo_rows(L, w) > 256)
+        return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     cudaError_t e = launch<BWDQ>(q, k, dout, v, dq, nullptr, const_cast<float*>(lse), Dws, B, H,
                                  L, d, w, dil, st, launches);
     if (e != cudaSuccess) return e;

@@ -97,6 +97,15 @@ SIMT_ONLY = [
     (1, 1, 300, 64, 100, 1),     # w > 64
     (1, 1, 520, 32, 200, 2),
 ]
+# windows wider than one 256-row halo: the chunked tensor-core kernels (d in {64, 128})
+WIDE = [
+    (1, 2, 700, 64, 100, 1),
+    (1, 1, 520, 64, 200, 2),
+    (2, 1, 300, 128, 130, 1),
+    (1, 1, 90, 64, 100, 1),      # w >= L
+    (1, 2, 1100, 64, 256, 3),    # ragged residues, 5 key chunks
+    (1, 1, 257, 64, 65, 1),      # smallest wide window
+]
 
 
 @pytest.mark.parametrize("shape", SMALL + SIMT_ONLY, ids=lambda s: "x".join(map(str, s)))
@@ -117,14 +126,14 @@ def _tc_ok(ft, shape, bwd=False):
         os.environ.pop("FT_WINATTN_PATH", None)
 
 
-@pytest.mark.parametrize("shape", SMALL, ids=lambda s: "x".join(map(str, s)))
+@pytest.mark.parametrize("shape", SMALL + WIDE, ids=lambda s: "x".join(map(str, s)))
 def test_tc_fwd_parity(ft, shape):
     if not _tc_ok(ft, shape):
         pytest.skip("shape not on the tensor-core path")
     run_case(ft, WinAttnShape(*shape), "bf16", "tc", seed=2, check_bwd=False)
 
 
-@pytest.mark.parametrize("shape", SMALL, ids=lambda s: "x".join(map(str, s)))
+@pytest.mark.parametrize("shape", SMALL + WIDE, ids=lambda s: "x".join(map(str, s)))
 def test_tc_bwd_parity(ft, shape):
     if not _tc_ok(ft, shape, bwd=True):
         pytest.skip("shape not on the tensor-core backward path")
