@@ -1,27 +1,37 @@
 // tc_band.cu -- tcgen05/TMEM tensor-core kernels of banded window attention for sm_100a
-// (bf16 storage; fp32 scores, softmax statistics and accumulators).
+// (bf16 storage; fp32 scores, softmax statistics and accumulators), windows with
+// 128 + 2w <= 256 halo rows (w <= 64).  Wider windows: tc_chunk.cu.
 //
-// One kernel template, three modes.  A CTA owns BM = 128 rows m0..m0+127 of one
-// (unit, residue) band problem and the NK = round_up(128 + 2w, 32) <= 256-row halo
-// m0-w .. m0+127+w of the other operand: the cached a[i:i+m] window of PAPER.md Fig. 14
+// One persistent kernel template, three modes.  A CTA owns BM = 128 rows m0..m0+127 of one
+// (unit, residue) band problem at a time, and the NK = round_up(128 + 2w, 64) <= 256-row
+// halo m0-w .. of the other operand: the cached a[i:i+m] window of PAPER.md Fig. 14
 // (lines 402-423), staged by TMA instead of the (2w+1)-fold as_strided copy of Q that the
 // operator baseline makes (Fig. 1c).
 //
 //   FWD   rows = queries.  S = Q K_h^T -> row max, exp, row sum (the fused dot/max of
 //         Fig. 10 and dot_norm/softmax of Fig. 8), lse -> HBM,
-//         P (bf16) -> TMEM;  O_n = P V_h,n  (n = 64-column d-slices), scaled by 1/l.
+//         P (bf16) -> smem;  O_c = P V_h,c  (c = 256-column output chunks), scaled by 1/l.
 //   BWDQ  rows = queries.  S = Q K_h^T, dP = dO V_h^T;  P = exp(S - lse) (recomputed from the
 //         saved lse: selective materialization);  D = sum_j P dP (exact,
-//         written to the workspace);  dS = P (dP - D) (bf16) -> TMEM;  dQ_n = dS K_h,n.
+//         written to the workspace);  dS = P (dP - D) (bf16 hi/lo) -> TMEM;  dQ_c = dS K_h,c.
 //   BWDKV rows = keys (tile ownership: each dk/dv row has exactly one writer, no atomics;
 //         the parallel-reduction choice of PAPER.md Fig. 13(d) over 13(e)).  S^T = K Q_h^T,
-//         dP^T = V dO_h^T;  P^T = exp(S^T - lse_col), dS^T = P^T (dP^T - D_col);
-//         dV_n = P^T dO_h,n,  dK_n = dS^T Q_h,n.
+//         dP^T = V dO_h^T;  P^T = exp(S^T - lse_col) -> smem, dS^T = P^T (dP^T - D_col)
+//         (bf16 hi/lo) -> TMEM;  dV_c = P^T dO_h,c,  dK_c = dS^T Q_h,c.
 //
-// Roles (192 threads): warps 0-3 softmax + epilogue (thread t <-> row m0+t <-> TMEM lane t),
-// warp 4 TMA producer + TMEM allocator, warp 5 MMA issuer (one elected thread).
-// The band geometry: column n of the halo is residue row m0 - w + n, and
+// Instruction economy (profiles/README.md, tools/mma_microbench.cu): a 1-SM tcgen05.mma
+// costs ~150-300 cycles whatever its N, so output GEMMs use N = 256-column chunks whose B
+// operand (V, K, dO or Q of the halo) is streamed in 64-row key blocks, and FWD issues the
+// next tile's QK^T right after this tile's first output chunk.
+//
+// Roles (320 threads): warps 0-3 softmax (thread t <-> row m0+t <-> TMEM lane t), warps 4-7
+// epilogue (TMEM -> bf16 -> smem -> warp-local TMA store), warp 8 TMA producer + TMEM
+// allocator, warp 9 MMA issuer.  Halo column n is residue row m0 - w + n, and
 // |m_col - m_row| <= w  <=>  0 <= n - t <= 2w, so one mask serves all three modes.
+//
+// TMEM (512 columns): S (or S^T) at [0, NK), dP (dP^T) at [256, 256+NK); dS / dS^T bf16
+// hi/lo overwrite S in place; the output accumulator is [256, 256 + chunk) once the
+// scores are consumed.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -42,59 +52,28 @@ using namespace tc;
 enum { FWD = 0, BWDQ = 1, BWDKV = 2 };
 
 constexpr int BM = 128;
-
-constexpr int RES_PER_LAUNCH = 4;
-constexpr uint32_t ABYTES = BM * 128;   // one 128-row x 64-col bf16 slice (SW128)
+constexpr int KB = 64;                   // key-block rows of an output-GEMM B operand
+constexpr int RES_PER_LAUNCH = 3;        // residues per launch (8 tensor maps each)
+constexpr uint32_t ABYTES = BM * 128;    // one 128-row x 64-col bf16 slice (SW128)
+constexpr uint32_t OBOX = KB * 128;      // one 64-row x 64-col bf16 box
+constexpr uint32_t STG = 32 * 128;       // one warp's 32-row x 64-col staging slice
+constexpr int NSTG = 2;                  // staging slices per epilogue warp
+constexpr int NTHREADS = 320;
+constexpr int MAX_NST = 8;
+constexpr size_t SMEM_LIMIT = 227 * 1024;
 constexpr float LOG2E = 1.4426950408889634f;
 constexpr float LN2 = 0.6931471805599453f;
 
-// TMEM layout (columns).  Score accumulators: S at 0 and dP at 256 (FWD: S of tile j in
-// region 256*(j&1), so the next tile's QK^T runs while this tile's softmax + epilogue do).
-// The bf16 A operands of the output GEMMs overwrite the scores as they are consumed:
-// "compact" = 16 columns per 32-column score chunk, at 16c; "split" = hi/lo bf16 pair
-// (x = hi + lo, lo = bf16(x - hi)) in place of chunk c: hi at 32c, lo at 32c+16.  dS is
-// split because at large d its entries reach O(10) and one bf16 rounding (2^-9) of them
-// would dominate the dq/dk error budget.  Output accumulators (64-column slices) sit outside
-// the score regions when NK <= 192 ("out-of-region"), so the next tile's score GEMMs can
-// run while the epilogue drains them; otherwise inside, and the next tile waits (tile_done).
 template <int MODE> struct Cfg {
-    static constexpr int NA = MODE == FWD ? 1 : 2;       // score GEMMs (S, and dP)
-    static constexpr int NO = MODE == BWDKV ? 2 : 1;     // output GEMMs per d-slice
-    static constexpr int NR = MODE == FWD ? 2 : 1;       // TMEM score regions
-    static constexpr int LA = MODE == FWD ? 1 : 0;       // score-GEMM tile lookahead
-    static constexpr uint32_t TCOLS = 512;
-    static constexpr bool SPLIT0 = MODE == BWDQ;         // A of output GEMM 0 split?
-    static constexpr bool SPLIT1 = MODE == BWDKV;        // A of output GEMM 1 split?
-    static constexpr int OBUFS = MODE == BWDKV ? 1 : 2;  // TMEM output buffers per output
+    static constexpr int NA = MODE == FWD ? 1 : 2;       // score GEMMs; also slots per G slice
+    static constexpr int NOUT = MODE == BWDKV ? 2 : 1;   // output tensors per chunk
+    static constexpr bool PSMEM = MODE != BWDQ;          // P / P^T staged in smem
 };
 
-// Column of output accumulator `o`, buffer `b`, for a tile in score region R.
-template <int MODE>
-__device__ __forceinline__ uint32_t out_col(int o, int b, int R, bool outside) {
-    if (MODE == FWD) return 256u * R + 128u + 64u * b;
-    if (MODE == BWDQ) return outside ? (b == 0 ? 192u : 448u) : 256u + 64u * b;
-    return outside ? (o == 0 ? 192u : 448u) : (o == 0 ? 128u : 192u);   // BWDKV
-}
-
-__device__ __forceinline__ uint32_t a_col(bool split, int kk) {
-    return split ? 32u * (kk >> 1) + 8u * (kk & 1) : 8u * kk;
-}
-__device__ __forceinline__ void split_bf16x2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
-    __nv_bfloat162 h = __floats2bfloat162_rn(x0, x1);
-    const float2 hf = __bfloat1622float2(h);
-    hi = *reinterpret_cast<uint32_t*>(&h);
-    lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
-}
-__device__ __forceinline__ float fast_exp2(float x) {
-    float y;
-    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
-    return y;
-}
-
-// a1/b1: first score GEMM (A rows m0.., B halo rows m0-w..), a2/b2: second (or, in FWD,
-// b2 = V for the output GEMM); o1/o2: outputs (TMA boxes of 32 rows: one per epilogue warp).
+// a1/b1, a2/b2: score-GEMM operands (A: rows m0.., box 128; B: halo rows m0-w.., box NK);
+// ob1/ob2: output-GEMM B operands (halo, box 64 rows); o1/o2: outputs (box 32 rows).
 struct Maps {
-    CUtensorMap a1, b1, a2, b2, o1, o2;
+    CUtensorMap a1, b1, a2, b2, ob1, ob2, o1, o2;
 };
 struct Params {
     Maps maps[RES_PER_LAUNCH];
@@ -102,17 +81,14 @@ struct Params {
     float* D;     // BWDQ: written; BWDKV: read
     int64_t L;
     int d, w, dil, r0, nr, NK, nsl, nst, units, tiles;
-    unsigned long long* trace;   // optional: [grid][TRACE_TILES][TRACE_EV] globaltimer stamps
+    unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace)
 };
 
-// Optional phase trace (ft_winattn_debug_trace): per CTA and local tile j < TRACE_TILES,
-// globaltimer stamps of: 0 producer first score-GEMM load, 1 producer last output load,
-// 2 MMA score GEMM first stage ready, 3 MMA s_full commit, 4 MMA p_full seen,
-// 5 MMA last output MMA issued, 6 softmax s_full seen, 7 softmax p_full arrive,
-// 8 epilogue first o_full seen, 9 epilogue done.
+// Phase trace: per CTA and local tile j < TRACE_TILES, globaltimer stamps of
+// 0 producer first score-GEMM load, 1 producer last output load, 2 MMA score GEMM first
+// stage ready, 3 MMA s_full commit, 4 MMA p_full seen, 5 MMA last output MMA issued,
+// 6 softmax s_full seen, 7 softmax p_full arrive, 8 epilogue first o_full, 9 epilogue done.
 constexpr int TRACE_TILES = 8, TRACE_EV = 48;
-// per-slice (n < 8): 10+n MMA stage-full seen, 18+n MMA o_empty seen, 26+n epilogue o_full
-// seen, 34+n epilogue store issued (epilogue warp 0)
 __device__ __forceinline__ void trace_ev(const Params& p, int j, int ev) {
     if (p.trace && j < TRACE_TILES) {
         unsigned long long t;
@@ -121,37 +97,46 @@ __device__ __forceinline__ void trace_ev(const Params& p, int j, int ev) {
     }
 }
 
-constexpr int NTHREADS = 320;    // warps 0-3 softmax, 4-7 epilogue, 8 producer, 9 MMA
-constexpr uint32_t STG = 32 * 128;   // one warp's 32-row x 64-col bf16 staging slice
-constexpr int NSTG = 2;              // staging slices per epilogue warp
-
-template <int MODE>
-__host__ __device__ inline uint32_t stage_bytes(int NK) {
-    return Cfg<MODE>::NA * (ABYTES + (uint32_t)NK * 128u);
+__device__ __forceinline__ float fast_exp2(float x) {
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
 }
-template <int MODE>
-inline size_t fixed_smem_bytes() {
-    return 1024 + 4 * NSTG * STG + 2 * 256 * sizeof(float) + 2 * 128 * sizeof(float) + 512;
+__device__ __forceinline__ void split_bf16x2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(x0, x1);
+    const float2 hf = __bfloat1622float2(h);
+    hi = *reinterpret_cast<uint32_t*>(&h);
+    lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
 }
-constexpr int MAX_NST = 8;
-constexpr size_t SMEM_LIMIT = 227 * 1024;
-
-template <int MODE>
-inline int pick_nst(int NK) {
-    const size_t avail = SMEM_LIMIT - fixed_smem_bytes<MODE>();
-    int n = (int)(avail / stage_bytes<MODE>(NK));
-    return n < MAX_NST ? n : MAX_NST;
-}
-
 __device__ __forceinline__ bool band_ok(int n, int t, int w, int mcol, int Lr) {
     return (unsigned)(n - t) <= (unsigned)(2 * w) && mcol >= 0 && mcol < Lr;
+}
+
+__host__ __device__ inline int chunk_w(int d, int c) { return d - 256 * c < 256 ? d - 256 * c : 256; }
+
+__host__ __device__ inline uint32_t slot_bytes(int NK) {
+    const uint32_t g = ABYTES + (uint32_t)NK * 128u;
+    const uint32_t o = 4u * OBOX;
+    return g > o ? g : o;
+}
+template <int MODE>
+inline size_t fixed_smem_bytes(int NK) {
+    return 1024 + 4 * NSTG * STG + (Cfg<MODE>::PSMEM ? (size_t)NK * 256 : 0) +
+           2 * 256 * sizeof(float) + 2 * 128 * sizeof(float) + 512;
+}
+template <int MODE>
+inline int pick_nst(int NK) {
+    const size_t fixed = fixed_smem_bytes<MODE>(NK);
+    if (fixed >= SMEM_LIMIT) return 0;
+    int n = (int)((SMEM_LIMIT - fixed) / slot_bytes(NK));
+    return n < MAX_NST ? n : MAX_NST;
 }
 
 struct Tile {
     int u, rl, r, Lr, m0;
 };
-// Tile tau -> (unit, residue, row block); t fastest so concurrently running CTAs work on
-// neighbouring row blocks and share their K/V halos through L2.
+// Tile tau -> (unit, residue, row block); row block fastest so concurrently running CTAs
+// work on neighbouring row blocks and share their halos through L2.
 __device__ __forceinline__ bool decode_tile(const Params& p, int tau, Tile& T) {
     const int t = tau % p.tiles;
     const int rest = tau / p.tiles;
@@ -162,8 +147,7 @@ __device__ __forceinline__ bool decode_tile(const Params& p, int tau, Tile& T) {
     T.m0 = t * BM;
     return T.m0 < T.Lr;
 }
-// Iterates this CTA's valid tiles in order (static round robin over the grid).
-struct TileCursor {
+struct TileCursor {   // this CTA's valid tiles, static round robin over the grid
     int tau;
     __device__ explicit TileCursor(int start) : tau(start - (int)gridDim.x) {}
     __device__ bool next(const Params& p, int total, Tile& T) {
@@ -173,6 +157,19 @@ struct TileCursor {
     }
 };
 
+// P / P^T in smem as the K-major SWIZZLE_128B A operand: 64-column atoms of 16 KB, row t at
+// t*128, 16-byte granule g at ((g ^ (t & 7)) * 16).  Thread t writes its row's 32-column
+// chunk c (16 packed words).
+__device__ __forceinline__ void st_p_chunk(uint8_t* P, int t, int c, const uint32_t (&pk)[16]) {
+    uint8_t* row = P + (c >> 1) * (BM * 128) + t * 128;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const int g = (c & 1) * 4 + q;
+        *reinterpret_cast<uint4*>(row + ((g ^ (t & 7)) * 16)) =
+            make_uint4(pk[4 * q], pk[4 * q + 1], pk[4 * q + 2], pk[4 * q + 3]);
+    }
+}
+
 template <int MODE>
 __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_constant__ Params p) {
     using C = Cfg<MODE>;
@@ -181,47 +178,48 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     uint8_t* smem = smem_raw + (((raw_u32 + 1023u) & ~1023u) - raw_u32);
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    const int NK = p.NK, nsl = p.nsl, w = p.w, NST = p.nst;
+    const int NK = p.NK, nsl = p.nsl, w = p.w, NST = p.nst, d = p.d;
+    const int nkb = NK / KB;
+    const int ncw = (d + 255) / 256;            // output chunks
+    const int nacc = ncw * C::NOUT;             // accumulations per tile
     const int total = p.units * p.nr * p.tiles;
-    const uint32_t SB = stage_bytes<MODE>(NK);
-    const uint32_t HB = (uint32_t)NK * 128u;   // one halo slice
-    const bool outside = MODE != FWD && NK <= 192;
-    const bool wait_region = !outside;          // next score GEMM must wait for the epilogue
+    const uint32_t SLOT = slot_bytes(NK);
+    const uint32_t HB = (uint32_t)NK * 128u;
 
-    uint8_t* ostg = smem + NST * SB;                                       // [4 warps][NSTG]
-    float* colLse = reinterpret_cast<float*>(ostg + 4 * NSTG * STG);       // BWDKV
+    uint8_t* sslots = smem;                                          // NST slots
+    uint8_t* sP = smem + (size_t)NST * SLOT;                         // P / P^T (PSMEM)
+    uint8_t* ostg = sP + (C::PSMEM ? (size_t)NK * 256 : 0);          // [4 warps][NSTG]
+    float* colLse = reinterpret_cast<float*>(ostg + 4 * NSTG * STG); // BWDKV
     float* colD = colLse + 256;
-    float* rowScale = colD + 256;                                          // FWD [2][128]
+    float* rowScale = colD + 256;                                    // FWD [2][128]
     uint64_t* bars = reinterpret_cast<uint64_t*>(rowScale + 256);
     uint64_t* full = bars;
     uint64_t* empty = bars + MAX_NST;
-    uint64_t* s_full = bars + 2 * MAX_NST;   // [NR]
-    uint64_t* p_full = s_full + 2;           // [NR]
-    uint64_t* o_full = s_full + 4;           // [2]
-    uint64_t* o_empty = s_full + 6;          // [2]
-    uint64_t* tile_done = s_full + 8;        // [NR]
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 10);
+    uint64_t* s_full = bars + 2 * MAX_NST;
+    uint64_t* p_full = s_full + 1;
+    uint64_t* o_full = s_full + 2;
+    uint64_t* o_empty = s_full + 3;
+    uint64_t* p_free = s_full + 4;   // P smem consumed by the tile's output MMAs
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 6);
 
     if (warp == 8) {
         if (lane == 0) {
             for (int i = 0; i < NST; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
-            for (int i = 0; i < 2; ++i) {
-                mbar_init(&s_full[i], 1);
-                mbar_init(&p_full[i], 128);
-                mbar_init(&o_full[i], 1);
-                mbar_init(&o_empty[i], 128);
-                mbar_init(&tile_done[i], 128);
-            }
+            mbar_init(s_full, 1);
+            mbar_init(p_full, 128);
+            mbar_init(o_full, 1);
+            mbar_init(o_empty, 128);
+            mbar_init(p_free, 1);
             fence_barrier_init();
             for (int i = 0; i < p.nr; ++i) {
                 const Maps& mp = p.maps[i];
-                tma_prefetch(&mp.a1); tma_prefetch(&mp.b1); tma_prefetch(&mp.b2); tma_prefetch(&mp.o1);
-                if (C::NA == 2) tma_prefetch(&mp.a2);
-                if (C::NO == 2) tma_prefetch(&mp.o2);
+                tma_prefetch(&mp.a1); tma_prefetch(&mp.b1); tma_prefetch(&mp.ob1); tma_prefetch(&mp.o1);
+                if (C::NA == 2) { tma_prefetch(&mp.a2); tma_prefetch(&mp.b2); }
+                if (C::NOUT == 2) { tma_prefetch(&mp.ob2); tma_prefetch(&mp.o2); }
             }
         }
         __syncwarp();
-        tmem_alloc(tmem_holder, C::TCOLS);
+        tmem_alloc(tmem_holder, 512);
         tmem_relinquish();
     }
     tc_fence_before();
@@ -231,161 +229,176 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 
     if (warp == 8) {
         if (lane == 0) {   // ------------------------------------------------ TMA producer
-            // Load order = MMA consumption order: G(0..LA-1), then per step i: G(i+LA), O(i).
+            // Slot order = MMA consumption order.  FWD: G(0), then per tile j:
+            // O_0(j), G(j+1), O_1(j) .. O_last(j).  BWD: per tile: G(j), O_0(j) .. O_last(j).
             int st = 0;
             uint32_t ph = 0;
-            TileCursor cg(blockIdx.x), co(blockIdx.x);
-            Tile Tg, To;
-            bool hg = cg.next(p, total, Tg), ho = co.next(p, total, To);
-            int jg = 0, jo = 0;
-            auto load_g = [&](const Tile& T) {
+            auto take = [&]() -> uint8_t* {
+                mbar_wait(&empty[st], ph ^ 1u);
+                return sslots + (size_t)st * SLOT;
+            };
+            auto adv = [&]() { if (++st == NST) { st = 0; ph ^= 1u; } };
+            auto load_g = [&](const Tile& T, int j) {
                 const Maps& mp = p.maps[T.rl];
                 for (int s = 0; s < nsl; ++s) {
-                    mbar_wait(&empty[st], ph ^ 1u);
-                    if (s == 0) trace_ev(p, jg, 0);
-                    uint8_t* sp = smem + st * SB;
-                    mbar_arrive_expect_tx(&full[st], SB);
+                    uint8_t* sp = take();
+                    if (s == 0) trace_ev(p, j, 0);
+                    mbar_arrive_expect_tx(&full[st], ABYTES + HB);
                     tma_load_3d(sp, &mp.a1, &full[st], s * 64, T.m0, T.u);
                     tma_load_3d(sp + ABYTES, &mp.b1, &full[st], s * 64, T.m0 - w, T.u);
+                    adv();
                     if (C::NA == 2) {
-                        tma_load_3d(sp + ABYTES + HB, &mp.a2, &full[st], s * 64, T.m0, T.u);
-                        tma_load_3d(sp + 2 * ABYTES + HB, &mp.b2, &full[st], s * 64, T.m0 - w, T.u);
+                        sp = take();
+                        mbar_arrive_expect_tx(&full[st], ABYTES + HB);
+                        tma_load_3d(sp, &mp.a2, &full[st], s * 64, T.m0, T.u);
+                        tma_load_3d(sp + ABYTES, &mp.b2, &full[st], s * 64, T.m0 - w, T.u);
+                        adv();
                     }
-                    if (++st == NST) { st = 0; ph ^= 1u; }
                 }
             };
-            auto load_o = [&](const Tile& T) {
+            auto load_o = [&](const Tile& T, int a) {   // key blocks of accumulation a
                 const Maps& mp = p.maps[T.rl];
-                for (int n = 0; n < nsl; ++n) {
-                    mbar_wait(&empty[st], ph ^ 1u);
-                    uint8_t* sp = smem + st * SB;
-                    mbar_arrive_expect_tx(&full[st], C::NO * HB);
-                    // output-GEMM B operands: FWD V (b2), BWDQ K (b1), BWDKV dO (b2) then Q (b1)
-                    const CUtensorMap* m_first = MODE == BWDQ ? &mp.b1 : &mp.b2;
-                    tma_load_3d(sp, m_first, &full[st], n * 64, T.m0 - w, T.u);
-                    if (C::NO == 2) tma_load_3d(sp + HB, &mp.b1, &full[st], n * 64, T.m0 - w, T.u);
-                    if (++st == NST) { st = 0; ph ^= 1u; }
+                const int c = a / C::NOUT;
+                const CUtensorMap* m = (C::NOUT == 2 && (a & 1)) ? &mp.ob2 : &mp.ob1;
+                const int nbox = chunk_w(d, c) / 64;
+                for (int kb = 0; kb < nkb; ++kb) {
+                    uint8_t* sp = take();
+                    mbar_arrive_expect_tx(&full[st], nbox * OBOX);
+                    for (int b = 0; b < nbox; ++b)
+                        tma_load_3d(sp + b * OBOX, m, &full[st], 256 * c + 64 * b, T.m0 - w + kb * KB, T.u);
+                    adv();
+                }
+            };
+            TileCursor cg(blockIdx.x), co(blockIdx.x);
+            Tile Tg, To;
+            bool hg = cg.next(p, total, Tg);
+            int jg = 0, jo = 0;
+            if (MODE == FWD && hg) { load_g(Tg, jg++); hg = cg.next(p, total, Tg); }
+            while (co.next(p, total, To)) {
+                if (MODE != FWD) { load_g(Tg, jg++); hg = cg.next(p, total, Tg); }
+                for (int a = 0; a < nacc; ++a) {
+                    load_o(To, a);
+                    if (MODE == FWD && a == 0 && hg) { load_g(Tg, jg++); hg = cg.next(p, total, Tg); }
                 }
                 trace_ev(p, jo, 1);
-            };
-            for (int la = 0; la < C::LA && hg; ++la) { load_g(Tg); ++jg; hg = cg.next(p, total, Tg); }
-            while (ho) {
-                if (hg) { load_g(Tg); ++jg; hg = cg.next(p, total, Tg); }
-                load_o(To); ++jo; ho = co.next(p, total, To);
+                ++jo;
             }
         }
     } else if (warp == 9) {
         if (lane == 0) {   // ------------------------------------------------ MMA issuer
             const uint32_t idS = idesc_bf16(128, NK, false, false);
-            const uint32_t idO = idesc_bf16(128, 64, false, true);
-            int st = 0, g = 0;
+            int st = 0, ga = 0;   // ga: global accumulation counter (o_full / o_empty phase)
             uint32_t ph = 0;
-            TileCursor cg(blockIdx.x), co(blockIdx.x);
-            Tile Tg, To;
-            bool hg = cg.next(p, total, Tg), ho = co.next(p, total, To);
-            int jg = 0, jo = 0;
-            auto mma_g = [&]() {   // score GEMM(s) of local tile jg into its region
-                const int R = jg % C::NR;
-                const uint32_t tR = tbase + 256u * R;
-                if (wait_region && jg >= C::NR) {
-                    mbar_wait(&tile_done[R], ((jg / C::NR) - 1) & 1);
+            auto wait_full = [&]() -> uint32_t {
+                mbar_wait(&full[st], ph);
+                tc_fence_after();
+                return smem_u32(sslots + (size_t)st * SLOT);
+            };
+            auto release = [&]() { mma_commit(&empty[st]); if (++st == NST) { st = 0; ph ^= 1u; } };
+            auto mma_g = [&](int j) {
+                // BWD: the score GEMMs write dP into the accumulator columns: the epilogue
+                // must have drained the previous tile's last accumulation.
+                if (MODE != FWD && ga > 0) {
+                    mbar_wait(o_empty, (ga - 1) & 1);
                     tc_fence_after();
                 }
                 for (int s = 0; s < nsl; ++s) {
-                    mbar_wait(&full[st], ph);
-                    tc_fence_after();
-                    if (s == 0) trace_ev(p, jg, 2);
-                    const uint32_t a1 = smem_u32(smem + st * SB), b1 = a1 + ABYTES;
-                    const uint32_t a2 = b1 + HB, b2 = a2 + ABYTES;
-                    // S and dP are independent accumulators: interleave their K-steps so the
-                    // tensor core always has two chains in flight
+                    const uint32_t a1 = wait_full();
+                    if (s == 0) trace_ev(p, j, 2);
+                    const uint32_t b1 = a1 + ABYTES;
+                    if (C::NA == 1) {
 #pragma unroll
-                    for (int kk = 0; kk < 4; ++kk) {
-                        mma_ss(tR, sdesc_sw128(a1 + kk * 32, 16, 1024),
-                               sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
-                        if (C::NA == 2)
+                        for (int kk = 0; kk < 4; ++kk)
+                            mma_ss(tbase, sdesc_sw128(a1 + kk * 32, 16, 1024),
+                                   sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
+                        release();
+                    } else {
+                        const int stA = st;
+                        if (++st == NST) { st = 0; ph ^= 1u; }
+                        const uint32_t a2 = wait_full(), b2 = a2 + ABYTES;
+                        // S and dP are independent accumulators: interleave their K-steps
+#pragma unroll
+                        for (int kk = 0; kk < 4; ++kk) {
+                            mma_ss(tbase, sdesc_sw128(a1 + kk * 32, 16, 1024),
+                                   sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
                             mma_ss(tbase + 256, sdesc_sw128(a2 + kk * 32, 16, 1024),
                                    sdesc_sw128(b2 + kk * 32, 16, 1024), idS, (s | kk) != 0);
+                        }
+                        mma_commit(&empty[stA]);
+                        release();
                     }
-                    mma_commit(&empty[st]);
-                    if (++st == NST) { st = 0; ph ^= 1u; }
                 }
-                mma_commit(&s_full[R]);
-                trace_ev(p, jg, 3);
+                mma_commit(s_full);
+                trace_ev(p, j, 3);
             };
-            auto mma_o = [&]() {   // output GEMMs of local tile jo, 64-column slices
-                const int R = jo % C::NR;
-                const uint32_t tR = tbase + 256u * R;
-                mbar_wait(&p_full[R], (jo / C::NR) & 1);
+            auto mma_o = [&](int a) {   // accumulation a of the current tile into [256, 256+cw)
+                const int c = a / C::NOUT;
+                const int cw = chunk_w(d, c);
+                const uint32_t idO = idesc_bf16(128, cw, false, true);
+                const bool smemA = C::PSMEM && (C::NOUT == 1 || (a & 1) == 0);   // P / P^T
+                const uint32_t sPa = smem_u32(sP);
+                if (ga > 0) {
+                    mbar_wait(o_empty, (ga - 1) & 1);
+                    tc_fence_after();
+                }
+                for (int kb = 0; kb < nkb; ++kb) {
+                    const uint32_t bb = wait_full();
+#pragma unroll
+                    for (int k4 = 0; k4 < 4; ++k4) {
+                        const int kk = kb * 4 + k4;   // 16-key step over the halo
+                        const uint64_t bd = sdesc_sw128(bb + k4 * 2048, OBOX, 1024);
+                        const uint32_t acc = (kk != 0);
+                        if (smemA) {
+                            const uint64_t ad = sdesc_sw128(sPa + (kk >> 2) * (BM * 128) + (kk & 3) * 32, 16, 1024);
+                            mma_ss(tbase + 256, ad, bd, idO, acc);
+                        } else {   // dS / dS^T hi/lo in TMEM over the S region
+                            const uint32_t tA = tbase + 32u * (kk >> 1) + 8u * (kk & 1);
+                            mma_ts(tbase + 256, tA, bd, idO, acc);
+                            mma_ts(tbase + 256, tA + 16, bd, idO, 1);
+                        }
+                    }
+                    release();
+                }
+                mma_commit(o_full);
+                ++ga;
+            };
+            TileCursor cg(blockIdx.x), co(blockIdx.x);
+            Tile Tg, To;
+            bool hg = cg.next(p, total, Tg);
+            int jg = 0, jo = 0;
+            if (MODE == FWD && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
+            while (co.next(p, total, To)) {
+                if (MODE != FWD) { mma_g(jg++); hg = cg.next(p, total, Tg); }
+                mbar_wait(p_full, jo & 1);
                 tc_fence_after();
                 trace_ev(p, jo, 4);
-                // Slices are issued in pairs (n, n+1) when both TMEM buffers exist, with
-                // their K-steps interleaved: consecutive MMAs then target independent
-                // accumulators instead of serialising on one (BWDKV interleaves dV / dK).
-                const int pair = C::OBUFS == 2 ? 2 : 1;
-                for (int n = 0; n < nsl; n += pair) {
-                    const int cnt = min(pair, nsl - n);
-                    uint32_t bbs[2], tDs[2][2];
-                    int sts[2];
-                    for (int q = 0; q < cnt; ++q) {
-                        const int gq = g + q, buf = gq % C::OBUFS;
-                        if (gq >= C::OBUFS) {
-                            mbar_wait(&o_empty[buf], ((gq / C::OBUFS) - 1) & 1);
-                            tc_fence_after();
-                        }
-                        if (n + q < 8) trace_ev(p, jo, 18 + n + q);
-                        mbar_wait(&full[st], ph);
-                        tc_fence_after();
-                        if (n + q < 8) trace_ev(p, jo, 10 + n + q);
-                        bbs[q] = smem_u32(smem + st * SB);
-                        sts[q] = st;
-                        for (int o = 0; o < C::NO; ++o) tDs[q][o] = tbase + out_col<MODE>(o, buf, R, outside);
-                        if (++st == NST) { st = 0; ph ^= 1u; }
-                    }
-                    for (int kk = 0; kk < NK / 16; ++kk) {
-                        for (int q = 0; q < cnt; ++q) {
-#pragma unroll
-                            for (int o = 0; o < C::NO; ++o) {
-                                const bool split = o == 0 ? C::SPLIT0 : C::SPLIT1;
-                                const uint32_t tA = tR + (o == 0 ? 0u : 256u) + a_col(split, kk);
-                                const uint64_t bd = sdesc_sw128(bbs[q] + o * HB + kk * 2048, HB, 1024);
-                                mma_ts(tDs[q][o], tA, bd, idO, kk != 0);
-                                if (split) mma_ts(tDs[q][o], tA + 16, bd, idO, 1);
-                            }
-                        }
-                    }
-                    for (int q = 0; q < cnt; ++q) {
-                        mma_commit(&empty[sts[q]]);
-                        mma_commit(&o_full[(g + q) % C::OBUFS]);
-                    }
-                    g += cnt;
+                for (int a = 0; a < nacc; ++a) {
+                    mma_o(a);
+                    if (MODE == FWD && a == 0 && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
                 }
+                if (C::PSMEM) mma_commit(p_free);
                 trace_ev(p, jo, 5);
-            };
-            for (int la = 0; la < C::LA && hg; ++la) { mma_g(); ++jg; hg = cg.next(p, total, Tg); }
-            while (ho) {
-                if (hg) { mma_g(); ++jg; hg = cg.next(p, total, Tg); }
-                mma_o(); ++jo; ho = co.next(p, total, To);
+                ++jo;
             }
         }
     } else if (warp < 4) {   // ------------------------------------------- softmax warps
         const int t = warp * 32 + lane;
-        const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+        const uint32_t trow = tbase + ((uint32_t)(warp * 32) << 16);
         const int nch = NK / 32;
-        // chunks holding any column of this warp's band rows (warp-uniform): rows
-        // 32*warp..32*warp+31 need columns [32*warp, 32*warp + 31 + 2w]
+        // chunks holding any band column of this warp's rows (warp-uniform):
+        // rows 32*warp .. 32*warp+31 need columns [32*warp, 32*warp + 31 + 2w]
         const int c_lo = warp, c_hi = min(nch - 1, (32 * warp + 31 + 2 * w) / 32);
         TileCursor cur(blockIdx.x);
         Tile T;
         int j = 0;
+        uint32_t zero16[16];
+#pragma unroll
+        for (int e = 0; e < 16; ++e) zero16[e] = 0u;
         while (cur.next(p, total, T)) {
-            const int R = j % C::NR;
-            const uint32_t trow = tbase + lane_off + 256u * R;   // score region of this tile
-            const uint32_t trow0 = tbase + lane_off;
             const int Lr = T.Lr, m0 = T.m0;
             const int mrow = m0 + t;
             const int kb = m0 - w;   // residue index of halo column 0
-            const int64_t rowbase = (int64_t)T.u * p.L + T.r;   // flat row of m = 0
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
 
             if (MODE == BWDKV) {
                 named_bar_sync(1, 128);   // everyone is done with the previous tile's columns
@@ -397,12 +410,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 }
                 named_bar_sync(1, 128);
             }
-            mbar_wait(&s_full[R], (j / C::NR) & 1);
+            mbar_wait(s_full, j & 1);
             tc_fence_after();
             if (t == 0) trace_ev(p, j, 6);
-            uint32_t zero16[16];
-#pragma unroll
-            for (int e = 0; e < 16; ++e) zero16[e] = 0u;
 
             if (MODE == FWD) {
                 float mx = -INFINITY;
@@ -418,9 +428,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 }
                 if (mx == -INFINITY) mx = 0.f;   // only rows beyond the sequence (never stored)
                 const float mxs = mx * LOG2E;
+                if (j > 0) mbar_wait(p_free, (j - 1) & 1);   // P smem of the previous tile consumed
                 float sum = 0.f;
                 for (int c = 0; c < nch; ++c) {
-                    if (c < c_lo || c > c_hi) { tmem_st16(trow + c * 16, zero16); continue; }
+                    if (c < c_lo || c > c_hi) { st_p_chunk(sP, t, c, zero16); continue; }
                     uint32_t rr[32], pk[16];
                     tmem_ld32(trow + c * 32, rr);
                     tmem_wait_ld();
@@ -437,12 +448,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         }
                         pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
                     }
-                    tmem_st16(trow + c * 16, pk);
+                    st_p_chunk(sP, t, c, pk);
                 }
-                rowScale[R * 128 + t] = 1.f / sum;
-                tmem_wait_st();
+                rowScale[(j & 1) * 128 + t] = 1.f / sum;
+                fence_proxy_async_smem();   // P (generic-proxy stores) -> tensor core (async proxy)
                 tc_fence_before();
-                mbar_arrive(&p_full[R]);
+                mbar_arrive(p_full);
                 if (mrow < Lr) p.lse[rowbase + (int64_t)mrow * p.dil] = (mxs + log2f(sum)) * LN2;
             } else if (MODE == BWDQ) {
                 const float lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
@@ -450,7 +461,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 for (int c = c_lo; c <= c_hi; ++c) {   // pass 1: D = sum_j P_ij dP_ij
                     uint32_t rs[32], rd[32];
                     tmem_ld32(trow + c * 32, rs);
-                    tmem_ld32(trow0 + 256 + c * 32, rd);
+                    tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
 #pragma unroll
                     for (int e = 0; e < 32; ++e) {
@@ -469,7 +480,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     }
                     uint32_t rs[32], rd[32], pk[16], pl[16];
                     tmem_ld32(trow + c * 32, rs);
-                    tmem_ld32(trow0 + 256 + c * 32, rd);
+                    tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
 #pragma unroll
                     for (int e = 0; e < 32; e += 2) {
@@ -489,19 +500,20 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 }
                 tmem_wait_st();
                 tc_fence_before();
-                mbar_arrive(&p_full[R]);
+                mbar_arrive(p_full);
                 if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
             } else {   // BWDKV: rows are keys, columns are halo queries
+                if (j > 0) mbar_wait(p_free, (j - 1) & 1);
                 for (int c = 0; c < nch; ++c) {
                     if (c < c_lo || c > c_hi) {
-                        tmem_st16(trow + c * 16, zero16);
-                        tmem_st16(trow0 + 256 + c * 32, zero16);
-                        tmem_st16(trow0 + 256 + c * 32 + 16, zero16);
+                        st_p_chunk(sP, t, c, zero16);
+                        tmem_st16(trow + c * 32, zero16);
+                        tmem_st16(trow + c * 32 + 16, zero16);
                         continue;
                     }
                     uint32_t rs[32], rd[32], pk[16], dk[16], dl[16];
                     tmem_ld32(trow + c * 32, rs);
-                    tmem_ld32(trow0 + 256 + c * 32, rd);
+                    tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
 #pragma unroll
                     for (int e = 0; e < 32; e += 2) {
@@ -517,68 +529,66 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
                         split_bf16x2(dv[0], dv[1], dk[e / 2], dl[e / 2]);
                     }
-                    tmem_st16(trow + c * 16, pk);
-                    tmem_st16(trow0 + 256 + c * 32, dk);
-                    tmem_st16(trow0 + 256 + c * 32 + 16, dl);
+                    st_p_chunk(sP, t, c, pk);
+                    tmem_st16(trow + c * 32, dk);
+                    tmem_st16(trow + c * 32 + 16, dl);
                 }
+                fence_proxy_async_smem();
                 tmem_wait_st();
                 tc_fence_before();
-                mbar_arrive(&p_full[R]);
+                mbar_arrive(p_full);
             }
             if (t == 0) trace_ev(p, j, 7);
             ++j;
         }
     } else if (warp < 8) {   // ------------------------------------------ epilogue warps
         const int ew = warp - 4;   // TMEM lanes 32*ew .. 32*ew+31  (warp % 4 == ew)
-        const uint32_t trow0 = tbase + ((uint32_t)(ew * 32) << 16);
+        const uint32_t trow = tbase + ((uint32_t)(ew * 32) << 16);
         uint8_t* mystg = ostg + ew * NSTG * STG;
         TileCursor cur(blockIdx.x);
         Tile T;
-        int j = 0, g = 0, sidx = 0;
+        int j = 0, ga = 0, sidx = 0;
         while (cur.next(p, total, T)) {
             const Maps& mp = p.maps[T.rl];
-            const int R = j % C::NR;
             float scale = 1.f;
             if (MODE == FWD) {   // 1/l of this row, published before p_full
-                mbar_wait(&p_full[R], (j / C::NR) & 1);
-                scale = rowScale[R * 128 + ew * 32 + lane];
+                mbar_wait(p_full, j & 1);
+                scale = rowScale[(j & 1) * 128 + ew * 32 + lane];
             }
-            for (int n = 0; n < nsl; ++n, ++g) {
-                const int buf = g % C::OBUFS;
-                mbar_wait(&o_full[buf], (g / C::OBUFS) & 1);
+            for (int a = 0; a < nacc; ++a, ++ga) {
+                const int c = a / C::NOUT;
+                const int nsl_c = chunk_w(d, c) / 64;
+                const CUtensorMap* om = (C::NOUT == 2 && (a & 1)) ? &mp.o2 : &mp.o1;
+                mbar_wait(o_full, ga & 1);
                 tc_fence_after();
-                if (lane == 0 && ew == 0 && n == 0) trace_ev(p, j, 8);
-                if (lane == 0 && ew == 0 && n < 8) trace_ev(p, j, 26 + n);
-#pragma unroll
-                for (int o = 0; o < C::NO; ++o) {
+                if (lane == 0 && ew == 0 && a == 0) trace_ev(p, j, 8);
+                for (int s = 0; s < nsl_c; ++s) {
                     uint32_t ov[64];
-                    const uint32_t tcol = out_col<MODE>(o, buf, R, outside);
-                    tmem_ld32(trow0 + tcol, *reinterpret_cast<uint32_t(*)[32]>(&ov[0]));
-                    tmem_ld32(trow0 + tcol + 32, *reinterpret_cast<uint32_t(*)[32]>(&ov[32]));
+                    const uint32_t tcol = 256u + 64u * s;
+                    tmem_ld32(trow + tcol, *reinterpret_cast<uint32_t(*)[32]>(&ov[0]));
+                    tmem_ld32(trow + tcol + 32, *reinterpret_cast<uint32_t(*)[32]>(&ov[32]));
                     tmem_wait_ld();
-                    if (o == C::NO - 1) {
+                    if (s == nsl_c - 1) {
                         tc_fence_before();
-                        mbar_arrive(&o_empty[buf]);
-                        if (n == nsl - 1) mbar_arrive(&tile_done[R]);
+                        mbar_arrive(o_empty);
                     }
                     uint8_t* stg = mystg + (sidx % NSTG) * STG;
                     if (lane == 0 && sidx >= NSTG) tma_store_wait_read<NSTG - 1>();
                     __syncwarp();
 #pragma unroll
-                    for (int c = 0; c < 8; ++c) {
+                    for (int q = 0; q < 8; ++q) {
                         uint4 val;
-                        val.x = pack_bf16x2(__uint_as_float(ov[8 * c + 0]) * scale, __uint_as_float(ov[8 * c + 1]) * scale);
-                        val.y = pack_bf16x2(__uint_as_float(ov[8 * c + 2]) * scale, __uint_as_float(ov[8 * c + 3]) * scale);
-                        val.z = pack_bf16x2(__uint_as_float(ov[8 * c + 4]) * scale, __uint_as_float(ov[8 * c + 5]) * scale);
-                        val.w = pack_bf16x2(__uint_as_float(ov[8 * c + 6]) * scale, __uint_as_float(ov[8 * c + 7]) * scale);
-                        *reinterpret_cast<uint4*>(stg + lane * 128 + ((c ^ (lane & 7)) * 16)) = val;
+                        val.x = pack_bf16x2(__uint_as_float(ov[8 * q + 0]) * scale, __uint_as_float(ov[8 * q + 1]) * scale);
+                        val.y = pack_bf16x2(__uint_as_float(ov[8 * q + 2]) * scale, __uint_as_float(ov[8 * q + 3]) * scale);
+                        val.z = pack_bf16x2(__uint_as_float(ov[8 * q + 4]) * scale, __uint_as_float(ov[8 * q + 5]) * scale);
+                        val.w = pack_bf16x2(__uint_as_float(ov[8 * q + 6]) * scale, __uint_as_float(ov[8 * q + 7]) * scale);
+                        *reinterpret_cast<uint4*>(stg + lane * 128 + ((q ^ (lane & 7)) * 16)) = val;
                     }
                     fence_proxy_async_smem();
                     __syncwarp();
                     if (lane == 0) {
-                        tma_store_3d(o == 1 ? &mp.o2 : &mp.o1, stg, n * 64, T.m0 + 32 * ew, T.u);
+                        tma_store_3d(om, stg, 256 * c + 64 * s, T.m0 + 32 * ew, T.u);
                         tma_store_commit();
-                        if (ew == 0 && n < 8 && o == C::NO - 1) trace_ev(p, j, 34 + n);
                     }
                     ++sidx;
                 }
@@ -592,7 +602,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     __syncthreads();
     if (warp == 8) {
         tc_fence_after();
-        tmem_dealloc(tbase, C::TCOLS);
+        tmem_dealloc(tbase, 512);
     }
 }
 
@@ -619,18 +629,21 @@ int num_sms() {
 
 int halo_rows(int64_t L, int64_t w) {
     const int64_t wc = w < L ? w : L;
-    return (int)(((BM + 2 * wc) + 31) / 32 * 32);
+    return (int)(((BM + 2 * wc) + 63) / 64 * 64);
 }
 
-// maps: per residue, (a1, b1, a2, b2, o1, o2) tensors; box rows BM for a/o, NK for b.
+// Tensors per mode: a1, b1 (score GEMM 1), a2, b2 (score GEMM 2), ob1, ob2 (output-GEMM
+// B operands), o1, o2 (outputs).
 template <int MODE>
-cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b2, void* o1,
-                   void* o2, float* lse, float* D, int64_t B, int64_t H, int64_t L, int64_t d,
-                   int64_t w, int64_t dil, cudaStream_t st, int* launches) {
+cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b2, const void* ob1,
+                   const void* ob2, void* o1, void* o2, float* lse, float* D, int64_t B, int64_t H,
+                   int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
     const int64_t wc = w < L ? w : L;
     const int NK = halo_rows(L, w);
     const int64_t units = B * H;
     const int64_t nres = dil < L ? dil : L;
+    const int nst = pick_nst<MODE>(NK);
+    if (nst < 2) return cudaErrorInvalidConfiguration;
     set_attr_once<MODE>();
     int n = 0;
     for (int64_t r0 = 0; r0 < nres; r0 += RES_PER_LAUNCH) {
@@ -642,9 +655,11 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
             Maps& m = p.maps[i];
             bool ok = make_residue_map(&m.a1, a1, L, d, units, dil, r, BM) &&
                       make_residue_map(&m.b1, b1, L, d, units, dil, r, NK) &&
-                      make_residue_map(&m.b2, b2, L, d, units, dil, r, NK) &&
+                      make_residue_map(&m.ob1, ob1, L, d, units, dil, r, KB) &&
                       make_residue_map(&m.o1, o1, L, d, units, dil, r, 32);
             if (ok && a2) ok = make_residue_map(&m.a2, a2, L, d, units, dil, r, BM);
+            if (ok && b2) ok = make_residue_map(&m.b2, b2, L, d, units, dil, r, NK);
+            if (ok && ob2) ok = make_residue_map(&m.ob2, ob2, L, d, units, dil, r, KB);
             if (ok && o2) ok = make_residue_map(&m.o2, o2, L, d, units, dil, r, 32);
             if (!ok) return cudaErrorInvalidValue;
         }
@@ -657,6 +672,7 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         p.r0 = (int)r0;
         p.NK = NK;
         p.nsl = (int)(d / 64);
+        p.nst = nst;
         const int64_t Lr0 = ceil_div(L - r0, dil);   // longest residue of this group
         p.nr = nr;
         p.trace = (unsigned long long*)trace_buffer(MODE);
@@ -664,9 +680,7 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         p.tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = (int64_t)p.units * p.nr * p.tiles;
         dim3 grid((unsigned)(total < num_sms() ? total : num_sms()));
-        const int nst = pick_nst<MODE>(NK);
-        p.nst = nst;
-        const size_t smem = fixed_smem_bytes<MODE>() + (size_t)nst * stage_bytes<MODE>(NK);
+        const size_t smem = fixed_smem_bytes<MODE>(NK) + (size_t)nst * slot_bytes(NK);
         tc_band_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
         prof_mark(st);
         cudaError_t e = cudaGetLastError();
@@ -679,7 +693,10 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
 
 bool band_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
     const int64_t wc = w < L ? w : L;
-    return d % 64 == 0 && d <= 512 && wc <= 64 && dil <= 256 && units * ((L + 127) / 128) < (1 << 30);
+    const int NK = halo_rows(L, w);
+    return d % 64 == 0 && d <= 512 && wc <= 64 && dil <= 256 &&
+           units * ((L + 127) / 128) < (1 << 30) && pick_nst<BWDKV>(NK) >= 2 &&
+           pick_nst<FWD>(NK) >= 2 && pick_nst<BWDQ>(NK) >= 2;
 }
 
 int band_launches(int64_t L, int64_t dil) {
@@ -710,8 +727,8 @@ cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float
     if (launches) *launches = 0;
     if (halo_rows(L, w) > 256)
         return tc_chunk_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
-    return launch<FWD>(q, k, nullptr, v, out, nullptr, lse, nullptr, B, H, L, d, w, dil, st,
-                       launches);
+    return launch<FWD>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, B, H, L,
+                       d, w, dil, st, launches);
 }
 
 cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
@@ -722,11 +739,12 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
     if (launches) *launches = 0;
     if (halo_rows(L, w) > 256)
         return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
-    cudaError_t e = launch<BWDQ>(q, k, dout, v, dq, nullptr, const_cast<float*>(lse), Dws, B, H,
-                                 L, d, w, dil, st, launches);
+    cudaError_t e = launch<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse),
+                                 Dws, B, H, L, d, w, dil, st, launches);
     if (e != cudaSuccess) return e;
-    return launch<BWDKV>(k, q, v, dout, dv, dk, const_cast<float*>(lse), Dws, B, H, L, d, w, dil,
-                         st, launches);
+    // BWDKV accumulation order per chunk: dV (P^T dO, ob1 = dout) then dK (dS^T Q, ob2 = q)
+    return launch<BWDKV>(k, q, v, dout, dout, q, dv, dk, const_cast<float*>(lse), Dws, B, H, L,
+                         d, w, dil, st, launches);
 }
 
 }  // namespace ftw

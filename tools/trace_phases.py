@@ -58,17 +58,7 @@ def main():
         print(f"  tile period (g1 ready j -> j+1)   {float((t[:,1:,2]-t[:,:-1,2])[valid[:,1:] & valid[:,:-1]].median()):7.2f}")
         print(f"  producer span per tile            {med(t[:,:,1]-t[:,:,0]):7.2f}")
         print(f"  first tile start (median over CTAs) {float(t[:,0,2][valid[:,0]].median()):7.2f}")
-        # per-slice detail for local tile 1 (steady state), relative to its p_full seen by MMA
-        jj = 1
-        v1 = valid[:, jj]
-        base = t[:, jj, 4]
-        rows = []
-        for n in range(8):
-            f = lambda e: float((t[:, jj, e] - base)[v1].median())
-            rows.append(f"    slice {n}: mma o_empty {f(18+n):6.2f}  mma stage-full {f(10+n):6.2f}  "
-                        f"epi o_full {f(26+n):6.2f}  epi stored {f(34+n):6.2f}")
-        print("  per-slice (tile 1, us after MMA saw p_full):")
-        print("\n".join(rows))
+
 
 
 if __name__ == "__main__":
