@@ -36,6 +36,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <mutex>
@@ -82,6 +83,7 @@ struct Params {
     int64_t L;
     int d, w, dil, r0, nr, NK, nsl, nst, units, tiles;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace)
+    int prefetch;                // L2-prefetch the next tile's score operands
 };
 
 // Phase trace: per CTA and local tile j < TRACE_TILES, globaltimer stamps of
@@ -256,6 +258,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     }
                 }
             };
+            // Warm L2 with a future tile's score-GEMM operands so HBM keeps streaming while
+            // this tile's softmax and output phases run (they barely touch DRAM).
+            auto prefetch_g = [&](const Tile& T) {
+                const Maps& mp = p.maps[T.rl];
+                for (int s = 0; s < nsl; ++s) {
+                    tma_prefetch_l2_3d(&mp.a1, s * 64, T.m0, T.u);
+                    if (p.prefetch != 3) tma_prefetch_l2_3d(&mp.b1, s * 64, T.m0 - w, T.u);
+                    if (C::NA == 2) {
+                        tma_prefetch_l2_3d(&mp.a2, s * 64, T.m0, T.u);
+                        if (p.prefetch != 3) tma_prefetch_l2_3d(&mp.b2, s * 64, T.m0 - w, T.u);
+                    }
+                }
+            };
             auto load_o = [&](const Tile& T, int a) {   // key blocks of accumulation a
                 const Maps& mp = p.maps[T.rl];
                 const int c = a / C::NOUT;
@@ -273,12 +288,25 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             Tile Tg, To;
             bool hg = cg.next(p, total, Tg);
             int jg = 0, jo = 0;
-            if (MODE == FWD && hg) { load_g(Tg, jg++); hg = cg.next(p, total, Tg); }
+            if (MODE == FWD && hg) {
+                load_g(Tg, jg++);
+                hg = cg.next(p, total, Tg);
+                if (hg && p.prefetch == 1) prefetch_g(Tg);
+            }
             while (co.next(p, total, To)) {
-                if (MODE != FWD) { load_g(Tg, jg++); hg = cg.next(p, total, Tg); }
+                if (MODE != FWD) {
+                    load_g(Tg, jg++);
+                    hg = cg.next(p, total, Tg);
+                    if (hg && p.prefetch == 1) prefetch_g(Tg);
+                }
                 for (int a = 0; a < nacc; ++a) {
+                    if (a == nacc - 1 && hg && p.prefetch >= 2) prefetch_g(Tg);
                     load_o(To, a);
-                    if (MODE == FWD && a == 0 && hg) { load_g(Tg, jg++); hg = cg.next(p, total, Tg); }
+                    if (MODE == FWD && a == 0 && hg) {
+                        load_g(Tg, jg++);
+                        hg = cg.next(p, total, Tg);
+                        if (hg && p.prefetch == 1) prefetch_g(Tg);
+                    }
                 }
                 trace_ev(p, jo, 1);
                 ++jo;
@@ -676,6 +704,10 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         const int64_t Lr0 = ceil_div(L - r0, dil);   // longest residue of this group
         p.nr = nr;
         p.trace = (unsigned long long*)trace_buffer(MODE);
+        {
+            const char* pf = getenv("FT_WINATTN_L2PF");   // tuning knob: 0 disables prefetch
+            p.prefetch = pf ? atoi(pf) : 0;
+        }
         p.units = (int)units;
         p.tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = (int64_t)p.units * p.nr * p.tiles;

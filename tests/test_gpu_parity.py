@@ -92,6 +92,9 @@ SMALL = [
     (1, 1, 1, 64, 3, 1),         # L = 1
     (1, 1, 40, 64, 4, 50),       # dilation >= L
     (1, 2, 333, 48, 9, 4),
+    (1, 1, 260, 192, 20, 1),     # one 192-column output chunk
+    (1, 1, 300, 320, 32, 2),     # chunks of 256 + 64 columns
+    (1, 1, 140, 448, 64, 1),     # 256 + 192 columns, widest band (NK = 256)
 ]
 SIMT_ONLY = [
     (1, 1, 300, 64, 100, 1),     # w > 64
