@@ -58,7 +58,7 @@ constexpr int RES_PER_LAUNCH = 3;        // residues per launch (8 tensor maps e
 constexpr uint32_t ABYTES = BM * 128;    // one 128-row x 64-col bf16 slice (SW128)
 constexpr uint32_t OBOX = KB * 128;      // one 64-row x 64-col bf16 box
 constexpr uint32_t STG = 32 * 128;       // one warp's 32-row x 64-col staging slice
-constexpr int NSTG = 2;                  // staging slices per epilogue warp
+constexpr int NSTG = 1;                  // staging slices per epilogue warp
 constexpr int NTHREADS = 320;
 constexpr int MAX_NST = 8;
 constexpr size_t SMEM_LIMIT = 227 * 1024;
@@ -121,10 +121,18 @@ __host__ __device__ inline uint32_t slot_bytes(int NK) {
     const uint32_t o = 4u * OBOX;
     return g > o ? g : o;
 }
+// Fixed shared memory besides the slot ring, carved tightly so that one more 40 KB slot
+// fits: alignment slack, P / P^T, epilogue staging, per-mode scratch (BWDKV column lse/D,
+// FWD row scales), barriers.
+constexpr size_t BAR_BYTES = 256;
+template <int MODE>
+__host__ __device__ inline size_t scratch_bytes(int NK) {
+    return MODE == BWDKV ? 2 * (size_t)NK * sizeof(float) : (MODE == FWD ? 2 * 128 * sizeof(float) : 0);
+}
 template <int MODE>
 inline size_t fixed_smem_bytes(int NK) {
-    return 1024 + 4 * NSTG * STG + (Cfg<MODE>::PSMEM ? (size_t)NK * 256 : 0) +
-           2 * 256 * sizeof(float) + 2 * 128 * sizeof(float) + 512;
+    return 1024 + (Cfg<MODE>::PSMEM ? (size_t)NK * 256 : 0) + 4 * NSTG * STG +
+           scratch_bytes<MODE>(NK) + BAR_BYTES;
 }
 template <int MODE>
 inline int pick_nst(int NK) {
@@ -191,10 +199,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     uint8_t* sslots = smem;                                          // NST slots
     uint8_t* sP = smem + (size_t)NST * SLOT;                         // P / P^T (PSMEM)
     uint8_t* ostg = sP + (C::PSMEM ? (size_t)NK * 256 : 0);          // [4 warps][NSTG]
-    float* colLse = reinterpret_cast<float*>(ostg + 4 * NSTG * STG); // BWDKV
-    float* colD = colLse + 256;
-    float* rowScale = colD + 256;                                    // FWD [2][128]
-    uint64_t* bars = reinterpret_cast<uint64_t*>(rowScale + 256);
+    float* scratch = reinterpret_cast<float*>(ostg + 4 * NSTG * STG);
+    float* colLse = scratch;                                         // BWDKV [NK]
+    float* colD = scratch + NK;                                      // BWDKV [NK]
+    float* rowScale = scratch;                                       // FWD [2][128]
+    uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(scratch) +
+                                                 scratch_bytes<MODE>(NK));
     uint64_t* full = bars;
     uint64_t* empty = bars + MAX_NST;
     uint64_t* s_full = bars + 2 * MAX_NST;
@@ -590,35 +600,49 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 mbar_wait(o_full, ga & 1);
                 tc_fence_after();
                 if (lane == 0 && ew == 0 && a == 0) trace_ev(p, j, 8);
-                for (int s = 0; s < nsl_c; ++s) {
-                    uint32_t ov[64];
-                    const uint32_t tcol = 256u + 64u * s;
-                    tmem_ld32(trow + tcol, *reinterpret_cast<uint32_t(*)[32]>(&ov[0]));
-                    tmem_ld32(trow + tcol + 32, *reinterpret_cast<uint32_t(*)[32]>(&ov[32]));
+                // Drain the accumulator 128 columns at a time: both 64-column halves are
+                // loaded before the wait, and o_empty is released as soon as every column is
+                // in registers, so the next accumulation's MMAs start before the stores.
+                for (int s0 = 0; s0 < nsl_c; s0 += 2) {
+                    const int ns = min(2, nsl_c - s0);
+                    uint32_t ov[2][64];
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        if (h < ns) {
+                            const uint32_t tcol = 256u + 64u * (s0 + h);
+                            tmem_ld32(trow + tcol, *reinterpret_cast<uint32_t(*)[32]>(&ov[h][0]));
+                            tmem_ld32(trow + tcol + 32, *reinterpret_cast<uint32_t(*)[32]>(&ov[h][32]));
+                        }
+                    }
                     tmem_wait_ld();
-                    if (s == nsl_c - 1) {
+                    if (s0 + ns == nsl_c) {
                         tc_fence_before();
                         mbar_arrive(o_empty);
                     }
-                    uint8_t* stg = mystg + (sidx % NSTG) * STG;
-                    if (lane == 0 && sidx >= NSTG) tma_store_wait_read<NSTG - 1>();
-                    __syncwarp();
 #pragma unroll
-                    for (int q = 0; q < 8; ++q) {
-                        uint4 val;
-                        val.x = pack_bf16x2(__uint_as_float(ov[8 * q + 0]) * scale, __uint_as_float(ov[8 * q + 1]) * scale);
-                        val.y = pack_bf16x2(__uint_as_float(ov[8 * q + 2]) * scale, __uint_as_float(ov[8 * q + 3]) * scale);
-                        val.z = pack_bf16x2(__uint_as_float(ov[8 * q + 4]) * scale, __uint_as_float(ov[8 * q + 5]) * scale);
-                        val.w = pack_bf16x2(__uint_as_float(ov[8 * q + 6]) * scale, __uint_as_float(ov[8 * q + 7]) * scale);
-                        *reinterpret_cast<uint4*>(stg + lane * 128 + ((q ^ (lane & 7)) * 16)) = val;
+                    for (int h = 0; h < 2; ++h) {
+                        if (h >= ns) break;
+                        const int s = s0 + h;
+                        uint8_t* stg = mystg + (sidx % NSTG) * STG;
+                        if (lane == 0 && sidx >= NSTG) tma_store_wait_read<NSTG - 1>();
+                        __syncwarp();
+#pragma unroll
+                        for (int q = 0; q < 8; ++q) {
+                            uint4 val;
+                            val.x = pack_bf16x2(__uint_as_float(ov[h][8 * q + 0]) * scale, __uint_as_float(ov[h][8 * q + 1]) * scale);
+                            val.y = pack_bf16x2(__uint_as_float(ov[h][8 * q + 2]) * scale, __uint_as_float(ov[h][8 * q + 3]) * scale);
+                            val.z = pack_bf16x2(__uint_as_float(ov[h][8 * q + 4]) * scale, __uint_as_float(ov[h][8 * q + 5]) * scale);
+                            val.w = pack_bf16x2(__uint_as_float(ov[h][8 * q + 6]) * scale, __uint_as_float(ov[h][8 * q + 7]) * scale);
+                            *reinterpret_cast<uint4*>(stg + lane * 128 + ((q ^ (lane & 7)) * 16)) = val;
+                        }
+                        fence_proxy_async_smem();
+                        __syncwarp();
+                        if (lane == 0) {
+                            tma_store_3d(om, stg, 256 * c + 64 * s, T.m0 + 32 * ew, T.u);
+                            tma_store_commit();
+                        }
+                        ++sidx;
                     }
-                    fence_proxy_async_smem();
-                    __syncwarp();
-                    if (lane == 0) {
-                        tma_store_3d(om, stg, 256 * c + 64 * s, T.m0 + 32 * ew, T.u);
-                        tma_store_commit();
-                    }
-                    ++sidx;
                 }
             }
             if (lane == 0 && ew == 0) trace_ev(p, j, 9);
