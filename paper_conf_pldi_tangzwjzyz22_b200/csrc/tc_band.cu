@@ -84,6 +84,7 @@ struct Params {
     int d, w, dil, r0, nr, NK, nsl, nst, units, tiles;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace)
     int prefetch;                // L2-prefetch the next tile's score operands
+    int g_first;                 // FWD: issue G(j+1) before (1) or after (0) O_0(j)
 };
 
 // Phase trace: per CTA and local tile j < TRACE_TILES, globaltimer stamps of
@@ -127,7 +128,7 @@ __host__ __device__ inline uint32_t slot_bytes(int NK) {
 constexpr size_t BAR_BYTES = 256;
 template <int MODE>
 __host__ __device__ inline size_t scratch_bytes(int NK) {
-    return MODE == BWDKV ? 2 * (size_t)NK * sizeof(float) : (MODE == FWD ? 2 * 128 * sizeof(float) : 0);
+    return MODE == BWDKV ? 2 * (size_t)NK * sizeof(float) : (MODE == FWD ? 3 * 128 * sizeof(float) : 0);
 }
 template <int MODE>
 inline size_t fixed_smem_bytes(int NK) {
@@ -191,7 +192,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     const int NK = p.NK, nsl = p.nsl, w = p.w, NST = p.nst, d = p.d;
     const int nkb = NK / KB;
     const int ncw = (d + 255) / 256;            // output chunks
-    const int nacc = ncw * C::NOUT;             // accumulations per tile
+    // BWDKV with d <= 128: dV and dK accumulate side by side ([256, 256+d) and
+    // [256+d, 256+2d)) with interleaved MMAs; otherwise one output per accumulation.
+    const bool dual = MODE == BWDKV && 2 * d <= 256;
+    const int nacc = dual ? ncw : ncw * C::NOUT;   // accumulations per tile
     const int total = p.units * p.nr * p.tiles;
     const uint32_t SLOT = slot_bytes(NK);
     const uint32_t HB = (uint32_t)NK * 128u;
@@ -202,7 +206,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     float* scratch = reinterpret_cast<float*>(ostg + 4 * NSTG * STG);
     float* colLse = scratch;                                         // BWDKV [NK]
     float* colD = scratch + NK;                                      // BWDKV [NK]
-    float* rowScale = scratch;                                       // FWD [2][128]
+    float* rowScale = scratch;                                       // FWD [3][128]
     uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(scratch) +
                                                  scratch_bytes<MODE>(NK));
     uint64_t* full = bars;
@@ -283,14 +287,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             };
             auto load_o = [&](const Tile& T, int a) {   // key blocks of accumulation a
                 const Maps& mp = p.maps[T.rl];
-                const int c = a / C::NOUT;
-                const CUtensorMap* m = (C::NOUT == 2 && (a & 1)) ? &mp.ob2 : &mp.ob1;
+                const int c = dual ? a : a / C::NOUT;
+                const CUtensorMap* m = (C::NOUT == 2 && !dual && (a & 1)) ? &mp.ob2 : &mp.ob1;
                 const int nbox = chunk_w(d, c) / 64;
                 for (int kb = 0; kb < nkb; ++kb) {
                     uint8_t* sp = take();
-                    mbar_arrive_expect_tx(&full[st], nbox * OBOX);
-                    for (int b = 0; b < nbox; ++b)
+                    mbar_arrive_expect_tx(&full[st], (dual ? 2 : 1) * nbox * OBOX);
+                    for (int b = 0; b < nbox; ++b) {
                         tma_load_3d(sp + b * OBOX, m, &full[st], 256 * c + 64 * b, T.m0 - w + kb * KB, T.u);
+                        if (dual)
+                            tma_load_3d(sp + (nbox + b) * OBOX, &mp.ob2, &full[st], 256 * c + 64 * b,
+                                        T.m0 - w + kb * KB, T.u);
+                    }
                     adv();
                 }
             };
@@ -304,7 +312,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 if (hg && p.prefetch == 1) prefetch_g(Tg);
             }
             while (co.next(p, total, To)) {
-                if (MODE != FWD) {
+                // FWD: G(j+1) precedes O(j) (P is in smem, so S can be overwritten as soon
+                // as softmax(j) is done); BWD: G(j) then O(j) (dS lives in the S columns).
+                if (hg && (MODE != FWD || p.g_first)) {
                     load_g(Tg, jg++);
                     hg = cg.next(p, total, Tg);
                     if (hg && p.prefetch == 1) prefetch_g(Tg);
@@ -312,10 +322,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 for (int a = 0; a < nacc; ++a) {
                     if (a == nacc - 1 && hg && p.prefetch >= 2) prefetch_g(Tg);
                     load_o(To, a);
-                    if (MODE == FWD && a == 0 && hg) {
+                    if (MODE == FWD && !p.g_first && a == 0 && hg) {
                         load_g(Tg, jg++);
                         hg = cg.next(p, total, Tg);
-                        if (hg && p.prefetch == 1) prefetch_g(Tg);
                     }
                 }
                 trace_ev(p, jo, 1);
@@ -370,11 +379,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 trace_ev(p, j, 3);
             };
             auto mma_o = [&](int a) {   // accumulation a of the current tile into [256, 256+cw)
-                const int c = a / C::NOUT;
+                const int c = dual ? a : a / C::NOUT;
                 const int cw = chunk_w(d, c);
                 const uint32_t idO = idesc_bf16(128, cw, false, true);
-                const bool smemA = C::PSMEM && (C::NOUT == 1 || (a & 1) == 0);   // P / P^T
+                const bool smemA = C::PSMEM && (C::NOUT == 1 || dual || (a & 1) == 0);   // P / P^T
+                const bool tmemA = MODE == BWDQ || (MODE == BWDKV && (dual || (a & 1) == 1));   // dS / dS^T
                 const uint32_t sPa = smem_u32(sP);
+                const uint32_t tD0 = tbase + 256, tD1 = tbase + 256 + (dual ? cw : 0);
+                const uint32_t boff = dual ? (uint32_t)(cw / 64) * OBOX : 0u;   // dK's B boxes
                 if (ga > 0) {
                     mbar_wait(o_empty, (ga - 1) & 1);
                     tc_fence_after();
@@ -384,15 +396,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 #pragma unroll
                     for (int k4 = 0; k4 < 4; ++k4) {
                         const int kk = kb * 4 + k4;   // 16-key step over the halo
-                        const uint64_t bd = sdesc_sw128(bb + k4 * 2048, OBOX, 1024);
                         const uint32_t acc = (kk != 0);
-                        if (smemA) {
+                        if (smemA) {   // P (FWD) or P^T (BWDKV dV) from smem
+                            const uint64_t bd = sdesc_sw128(bb + k4 * 2048, OBOX, 1024);
                             const uint64_t ad = sdesc_sw128(sPa + (kk >> 2) * (BM * 128) + (kk & 3) * 32, 16, 1024);
-                            mma_ss(tbase + 256, ad, bd, idO, acc);
-                        } else {   // dS / dS^T hi/lo in TMEM over the S region
+                            mma_ss(tD0, ad, bd, idO, acc);
+                        }
+                        if (tmemA) {   // dS (BWDQ) or dS^T (BWDKV dK), hi/lo in TMEM over S
+                            const uint64_t bd = sdesc_sw128(bb + boff + k4 * 2048, OBOX, 1024);
                             const uint32_t tA = tbase + 32u * (kk >> 1) + 8u * (kk & 1);
-                            mma_ts(tbase + 256, tA, bd, idO, acc);
-                            mma_ts(tbase + 256, tA + 16, bd, idO, 1);
+                            mma_ts(tD1, tA, bd, idO, acc);
+                            mma_ts(tD1, tA + 16, bd, idO, 1);
                         }
                     }
                     release();
@@ -404,15 +418,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             Tile Tg, To;
             bool hg = cg.next(p, total, Tg);
             int jg = 0, jo = 0;
-            if (MODE == FWD && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
+            if (MODE == FWD && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }   // G(0)
             while (co.next(p, total, To)) {
                 if (MODE != FWD) { mma_g(jg++); hg = cg.next(p, total, Tg); }
                 mbar_wait(p_full, jo & 1);
                 tc_fence_after();
                 trace_ev(p, jo, 4);
+                if (MODE == FWD && p.g_first && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
                 for (int a = 0; a < nacc; ++a) {
                     mma_o(a);
-                    if (MODE == FWD && a == 0 && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
+                    if (MODE == FWD && !p.g_first && a == 0 && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
                 }
                 if (C::PSMEM) mma_commit(p_free);
                 trace_ev(p, jo, 5);
@@ -488,7 +503,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     }
                     st_p_chunk(sP, t, c, pk);
                 }
-                rowScale[(j & 1) * 128 + t] = 1.f / sum;
+                rowScale[(j % 3) * 128 + t] = 1.f / sum;
                 fence_proxy_async_smem();   // P (generic-proxy stores) -> tensor core (async proxy)
                 tc_fence_before();
                 mbar_arrive(p_full);
@@ -591,12 +606,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             float scale = 1.f;
             if (MODE == FWD) {   // 1/l of this row, published before p_full
                 mbar_wait(p_full, j & 1);
-                scale = rowScale[(j & 1) * 128 + ew * 32 + lane];
+                scale = rowScale[(j % 3) * 128 + ew * 32 + lane];
             }
             for (int a = 0; a < nacc; ++a, ++ga) {
-                const int c = a / C::NOUT;
-                const int nsl_c = chunk_w(d, c) / 64;
-                const CUtensorMap* om = (C::NOUT == 2 && (a & 1)) ? &mp.o2 : &mp.o1;
+                const int c = dual ? a : a / C::NOUT;
+                const int cw = chunk_w(d, c);
+                // dual: slices 0..cw/64-1 are dV (o1), the next cw/64 are dK (o2)
+                const int nsl_c = (dual ? 2 : 1) * cw / 64;
                 mbar_wait(o_full, ga & 1);
                 tc_fence_after();
                 if (lane == 0 && ew == 0 && a == 0) trace_ev(p, j, 8);
@@ -637,8 +653,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         }
                         fence_proxy_async_smem();
                         __syncwarp();
+                        const bool second = dual ? (64 * s >= cw) : (C::NOUT == 2 && (a & 1));
+                        const CUtensorMap* om = second ? &mp.o2 : &mp.o1;
+                        const int col = 256 * c + (dual && second ? 64 * s - cw : 64 * s);
                         if (lane == 0) {
-                            tma_store_3d(om, stg, 256 * c + 64 * s, T.m0 + 32 * ew, T.u);
+                            tma_store_3d(om, stg, col, T.m0 + 32 * ew, T.u);
                             tma_store_commit();
                         }
                         ++sidx;
@@ -731,6 +750,10 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         {
             const char* pf = getenv("FT_WINATTN_L2PF");   // tuning knob: 0 disables prefetch
             p.prefetch = pf ? atoi(pf) : 0;
+            const char* gf = getenv("FT_WINATTN_GFIRST");
+            // measured (profiles/README.md): G(j+1) before O(j) wins when the output is
+            // one chunk (d <= 256); at d = 512 issuing it between the two chunks wins.
+            p.g_first = gf ? atoi(gf) : (d <= 256 ? 1 : 0);
         }
         p.units = (int)units;
         p.tiles = (int)ceil_div(Lr0, BM);
