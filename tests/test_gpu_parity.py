@@ -95,6 +95,8 @@ SMALL = [
     (1, 1, 260, 192, 20, 1),     # one 192-column output chunk
     (1, 1, 300, 320, 32, 2),     # chunks of 256 + 64 columns
     (1, 1, 140, 448, 64, 1),     # 256 + 192 columns, widest band (NK = 256)
+    (1, 2, 700, 64, 20, 5),      # 5 residues -> two launch groups
+    (2, 1, 900, 128, 3, 7),      # 7 residues, short windows
 ]
 SIMT_ONLY = [
     (1, 1, 300, 64, 100, 1),     # w > 64
@@ -108,6 +110,7 @@ WIDE = [
     (1, 1, 90, 64, 100, 1),      # w >= L
     (1, 2, 1100, 64, 256, 3),    # ragged residues, 5 key chunks
     (1, 1, 257, 64, 65, 1),      # smallest wide window
+    (1, 1, 1500, 64, 100, 5),    # wide window over 5 residues (two launch groups)
 ]
 
 
@@ -180,6 +183,33 @@ def test_determinism(ft):
     b = ft.fwd(q, k, v, 32) + ft.bwd(q, k, v, *ft.fwd(q, k, v, 32), g, 32)
     for x1, x2 in zip(a, b):
         assert torch.equal(x1, x2)
+
+
+def test_binding_rejects_bad_inputs(ft):
+    dev = torch.device("cuda:0")
+    q = torch.zeros(1, 1, 64, 64, device=dev, dtype=torch.bfloat16)
+    with pytest.raises(ValueError):
+        ft.fwd(q, q.transpose(2, 3), q, 4)                  # non-contiguous / wrong shape
+    with pytest.raises(ValueError):
+        ft.fwd(q, q.float(), q, 4)                          # dtype mismatch
+    with pytest.raises(TypeError):
+        ft.fwd(q.half(), q.half(), q.half(), 4)             # unsupported dtype
+    with pytest.raises(ft.FtError):
+        ft.fwd(q, q, q, -1)                                 # w < 0 -> FT_ERR_INVALID_VALUE
+    with pytest.raises(ValueError):
+        ft.fwd(q.cpu(), q.cpu(), q.cpu(), 4)                # not CUDA
+
+
+def test_outputs_untouched_on_error(ft):
+    """Argument checks run before any launch: a failing call leaves the outputs as they were."""
+    dev = torch.device("cuda:0")
+    q = torch.randn(1, 1, 64, 64, device=dev).to(torch.bfloat16)
+    out = torch.full_like(q, 7.0)
+    lse = torch.full((1, 1, 64), 3.0, device=dev)
+    with pytest.raises(ft.FtError):
+        ft.fwd(q, q, q, 4, dilation=0, out=out, lse=lse)
+    torch.cuda.synchronize()
+    assert bool((out == 7.0).all()) and bool((lse == 3.0).all())
 
 
 def test_autograd_function(ft):

@@ -1,0 +1,24 @@
+#!/bin/bash
+# compute-sanitizer passes over small shapes of every kernel family (run under gpurun).
+set -u
+cd "$(dirname "$0")/.."
+cat > /tmp/san_case.py <<'PY'
+import sys, torch
+sys.path.insert(0, ".")
+import paper_conf_pldi_tangzwjzyz22_b200 as ft
+from synth import WinAttnShape, make_inputs
+dev = torch.device("cuda:0")
+for shape, dt in [((1, 2, 300, 64, 32, 3), "bf16"), ((1, 1, 200, 512, 32, 1), "bf16"),
+                  ((1, 1, 600, 64, 100, 2), "bf16"), ((1, 1, 130, 64, 8, 1), "f32")]:
+    s = WinAttnShape(*shape)
+    x = make_inputs(s, 0, dt)
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    o, l = ft.fwd(q, k, v, s.w, s.dilation)
+    ft.bwd(q, k, v, o, l, g, s.w, s.dilation)
+torch.cuda.synchronize()
+print("cases ok")
+PY
+for tool in memcheck racecheck synccheck initcheck; do
+  echo "== $tool"
+  timeout 600 compute-sanitizer --tool $tool --kernel-name kns=tc_ --kernel-name kns=simt --print-limit 10 python /tmp/san_case.py 2>&1 | tail -4
+done
