@@ -181,6 +181,36 @@ __device__ __forceinline__ void st_p_chunk(uint8_t* P, int t, int c, const uint3
     }
 }
 
+// Masked max of one 32-column score chunk (columns n0 .. n0+31 of the halo).
+__device__ __forceinline__ float chunk_max(const uint32_t (&rr)[32], int n0, int t, int w, int kb,
+                                           int Lr, float mx) {
+#pragma unroll
+    for (int e = 0; e < 32; ++e)
+        if (band_ok(n0 + e, t, w, kb + n0 + e, Lr)) mx = fmaxf(mx, __uint_as_float(rr[e]));
+    return mx;
+}
+// P = exp2(S*log2e - mxs) on one chunk (masked), packed to bf16 into the smem P operand;
+// returns the chunk's contribution to the row sum.
+__device__ __forceinline__ float chunk_exp_store(uint8_t* sP, const uint32_t (&rr)[32], int c,
+                                                 int t, int w, int kb, int Lr, float mxs) {
+    uint32_t pk[16];
+    float sum = 0.f;
+#pragma unroll
+    for (int e = 0; e < 32; e += 2) {
+        float pv[2];
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int n = c * 32 + e + h;
+            pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rr[e + h]), LOG2E, -mxs))
+                                                 : 0.f;
+            sum += pv[h];
+        }
+        pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
+    }
+    st_p_chunk(sP, t, c, pk);
+    return sum;
+}
+
 template <int MODE>
 __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_constant__ Params p) {
     using C = Cfg<MODE>;
@@ -468,40 +498,28 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             if (t == 0) trace_ev(p, j, 6);
 
             if (MODE == FWD) {
+                // Band-empty chunks of P never change: zero them once per CTA.
+                if (j == 0)
+                    for (int c = 0; c < nch; ++c)
+                        if (c < c_lo || c > c_hi) st_p_chunk(sP, t, c, zero16);
                 float mx = -INFINITY;
                 for (int c = c_lo; c <= c_hi; ++c) {
                     uint32_t rr[32];
                     tmem_ld32(trow + c * 32, rr);
                     tmem_wait_ld();
-#pragma unroll
-                    for (int e = 0; e < 32; ++e) {
-                        const int n = c * 32 + e;
-                        if (band_ok(n, t, w, kb + n, Lr)) mx = fmaxf(mx, __uint_as_float(rr[e]));
-                    }
+                    mx = chunk_max(rr, c * 32, t, w, kb, Lr, mx);
                 }
                 if (mx == -INFINITY) mx = 0.f;   // only rows beyond the sequence (never stored)
                 const float mxs = mx * LOG2E;
+                if (t == 0) trace_ev(p, j, 10);
                 if (j > 0) mbar_wait(p_free, (j - 1) & 1);   // P smem of the previous tile consumed
+                if (t == 0) trace_ev(p, j, 11);
                 float sum = 0.f;
-                for (int c = 0; c < nch; ++c) {
-                    if (c < c_lo || c > c_hi) { st_p_chunk(sP, t, c, zero16); continue; }
-                    uint32_t rr[32], pk[16];
+                for (int c = c_lo; c <= c_hi; ++c) {
+                    uint32_t rr[32];
                     tmem_ld32(trow + c * 32, rr);
                     tmem_wait_ld();
-#pragma unroll
-                    for (int e = 0; e < 32; e += 2) {
-                        float pv[2];
-#pragma unroll
-                        for (int h = 0; h < 2; ++h) {
-                            const int n = c * 32 + e + h;
-                            pv[h] = band_ok(n, t, w, kb + n, Lr)
-                                        ? fast_exp2(fmaf(__uint_as_float(rr[e + h]), LOG2E, -mxs))
-                                        : 0.f;
-                            sum += pv[h];
-                        }
-                        pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
-                    }
-                    st_p_chunk(sP, t, c, pk);
+                    sum += chunk_exp_store(sP, rr, c, t, w, kb, Lr, mxs);
                 }
                 rowScale[(j % 3) * 128 + t] = 1.f / sum;
                 fence_proxy_async_smem();   // P (generic-proxy stores) -> tensor core (async proxy)
@@ -559,7 +577,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 if (j > 0) mbar_wait(p_free, (j - 1) & 1);
                 for (int c = 0; c < nch; ++c) {
                     if (c < c_lo || c > c_hi) {
-                        st_p_chunk(sP, t, c, zero16);
+                        if (j == 0) st_p_chunk(sP, t, c, zero16);   // P^T zeros persist
                         tmem_st16(trow + c * 32, zero16);
                         tmem_st16(trow + c * 32 + 16, zero16);
                         continue;

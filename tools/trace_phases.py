@@ -52,6 +52,10 @@ def main():
         print(f"  GEMM1 (mma ready -> s commit)     {med(t[:,:,3]-t[:,:,2]):7.2f} us")
         print(f"  s commit -> softmax start         {med(t[:,:,6]-t[:,:,3]):7.2f}")
         print(f"  softmax (s seen -> p arrive)      {med(t[:,:,7]-t[:,:,6]):7.2f}")
+        if name == "FWD":
+            print(f"    pass 1 (max)                    {med(t[:,:,10]-t[:,:,6]):7.2f}")
+            print(f"    wait P buffer free              {med(t[:,:,11]-t[:,:,10]):7.2f}")
+            print(f"    pass 2 (exp, P -> smem)         {med(t[:,:,7]-t[:,:,11]):7.2f}")
         print(f"  p arrive -> mma sees p            {med(t[:,:,4]-t[:,:,7]):7.2f}")
         print(f"  output MMAs issued (p -> out end) {med(t[:,:,5]-t[:,:,4]):7.2f}")
         print(f"  epilogue (first o_full -> done)   {med(t[:,:,9]-t[:,:,8]):7.2f}")
