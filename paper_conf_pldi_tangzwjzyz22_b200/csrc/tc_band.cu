@@ -225,6 +225,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     // BWDKV with d <= 128: dV and dK accumulate side by side ([256, 256+d) and
     // [256+d, 256+2d)) with interleaved MMAs; otherwise one output per accumulation.
     const bool dual = MODE == BWDKV && 2 * d <= 256;
+    // BWDQ with NK + d <= 256 (d = 64, w <= 32): the dQ accumulator fits beside both score
+    // regions at [256 + NK, 256 + NK + d), so dS can be handed to the MMA per 64-key block
+    // while the softmax is still reading dP, and the next tile's score GEMMs need not wait
+    // for the epilogue drain.
+    const bool early = MODE == BWDQ && NK + d <= 256;
+    const uint32_t acc0 = early ? 256u + (uint32_t)NK : 256u;   // accumulator base column
     const int nacc = dual ? ncw : ncw * C::NOUT;   // accumulations per tile
     const int total = p.units * p.nr * p.tiles;
     const uint32_t SLOT = slot_bytes(NK);
@@ -246,7 +252,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     uint64_t* o_full = s_full + 2;
     uint64_t* o_empty = s_full + 3;
     uint64_t* p_free = s_full + 4;   // P smem consumed by the tile's output MMAs
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 6);
+    uint64_t* p_blk = s_full + 5;    // [4] BWD: dS of 64-key block b written (per-block handoff)
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 9);
 
     if (warp == 8) {
         if (lane == 0) {
@@ -256,6 +263,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             mbar_init(o_full, 1);
             mbar_init(o_empty, 128);
             mbar_init(p_free, 1);
+            for (int i = 0; i < 4; ++i) mbar_init(&p_blk[i], 128);
             fence_barrier_init();
             for (int i = 0; i < p.nr; ++i) {
                 const Maps& mp = p.maps[i];
@@ -365,6 +373,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
         if (lane == 0) {   // ------------------------------------------------ MMA issuer
             const uint32_t idS = idesc_bf16(128, NK, false, false);
             int st = 0, ga = 0;   // ga: global accumulation counter (o_full / o_empty phase)
+            int jo_cur = 0;       // local index of the tile whose outputs are being issued
             uint32_t ph = 0;
             auto wait_full = [&]() -> uint32_t {
                 mbar_wait(&full[st], ph);
@@ -375,7 +384,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             auto mma_g = [&](int j) {
                 // BWD: the score GEMMs write dP into the accumulator columns: the epilogue
                 // must have drained the previous tile's last accumulation.
-                if (MODE != FWD && ga > 0) {
+                if (MODE != FWD && !early && ga > 0) {
                     mbar_wait(o_empty, (ga - 1) & 1);
                     tc_fence_after();
                 }
@@ -415,13 +424,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 const bool smemA = C::PSMEM && (C::NOUT == 1 || dual || (a & 1) == 0);   // P / P^T
                 const bool tmemA = MODE == BWDQ || (MODE == BWDKV && (dual || (a & 1) == 1));   // dS / dS^T
                 const uint32_t sPa = smem_u32(sP);
-                const uint32_t tD0 = tbase + 256, tD1 = tbase + 256 + (dual ? cw : 0);
+                const uint32_t tD0 = tbase + acc0, tD1 = tbase + acc0 + (dual ? cw : 0);
                 const uint32_t boff = dual ? (uint32_t)(cw / 64) * OBOX : 0u;   // dK's B boxes
                 if (ga > 0) {
                     mbar_wait(o_empty, (ga - 1) & 1);
                     tc_fence_after();
                 }
                 for (int kb = 0; kb < nkb; ++kb) {
+                    if (early && a == 0) {   // dS of this 64-key block written?
+                        mbar_wait(&p_blk[kb], jo_cur & 1);
+                        tc_fence_after();
+                    }
                     const uint32_t bb = wait_full();
 #pragma unroll
                     for (int k4 = 0; k4 < 4; ++k4) {
@@ -451,8 +464,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             if (MODE == FWD && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }   // G(0)
             while (co.next(p, total, To)) {
                 if (MODE != FWD) { mma_g(jg++); hg = cg.next(p, total, Tg); }
-                mbar_wait(p_full, jo & 1);
-                tc_fence_after();
+                jo_cur = jo;
+                if (!early) {   // early BWDQ waits per key block inside mma_o
+                    mbar_wait(p_full, jo & 1);
+                    tc_fence_after();
+                }
                 trace_ev(p, jo, 4);
                 if (MODE == FWD && p.g_first && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
                 for (int a = 0; a < nacc; ++a) {
@@ -543,10 +559,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         D = fmaf(pv, __uint_as_float(rd[e]), D);
                     }
                 }
+                auto block_done = [&](int c) {   // early: hand block c/2 to the MMA
+                    if (early && (c & 1)) {
+                        tmem_wait_st();
+                        tc_fence_before();
+                        mbar_arrive(&p_blk[c >> 1]);
+                    }
+                };
                 for (int c = 0; c < nch; ++c) {   // pass 2: dS = P (dP - D) -> TMEM (bf16 hi/lo)
                     if (c < c_lo || c > c_hi) {
                         tmem_st16(trow + c * 32, zero16);
                         tmem_st16(trow + c * 32 + 16, zero16);
+                        block_done(c);
                         continue;
                     }
                     uint32_t rs[32], rd[32], pk[16], pl[16];
@@ -568,6 +592,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     }
                     tmem_st16(trow + c * 32, pk);
                     tmem_st16(trow + c * 32 + 16, pl);
+                    block_done(c);
                 }
                 tmem_wait_st();
                 tc_fence_before();
@@ -643,7 +668,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 #pragma unroll
                     for (int h = 0; h < 2; ++h) {
                         if (h < ns) {
-                            const uint32_t tcol = 256u + 64u * (s0 + h);
+                            const uint32_t tcol = acc0 + 64u * (s0 + h);
                             tmem_ld32(trow + tcol, *reinterpret_cast<uint32_t(*)[32]>(&ov[h][0]));
                             tmem_ld32(trow + tcol + 32, *reinterpret_cast<uint32_t(*)[32]>(&ov[h][32]));
                         }
