@@ -39,7 +39,8 @@ class FtError(RuntimeError):
 
 
 def lib_path() -> str:
-    return os.path.join(_PKG, _LIB_NAME)
+    """The in-tree library; FT_WINATTN_LIB names another build of it (A/B timing aid)."""
+    return os.environ.get("FT_WINATTN_LIB") or os.path.join(_PKG, _LIB_NAME)
 
 
 def load_library(build_if_missing: bool = False):

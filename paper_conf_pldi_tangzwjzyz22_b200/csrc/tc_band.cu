@@ -59,7 +59,7 @@ constexpr uint32_t ABYTES = BM * 128;    // one 128-row x 64-col bf16 slice (SW1
 constexpr uint32_t OBOX = KB * 128;      // one 64-row x 64-col bf16 box
 constexpr uint32_t STG = 32 * 128;       // one warp's 32-row x 64-col staging slice
 constexpr int NSTG = 1;                  // staging slices per epilogue warp
-constexpr int NTHREADS = 320;
+constexpr int NTHREADS = 352;
 constexpr int MAX_NST = 8;
 constexpr size_t SMEM_LIMIT = 227 * 1024;
 constexpr float LOG2E = 1.4426950408889634f;
@@ -83,8 +83,7 @@ struct Params {
     int64_t L;
     int d, w, dil, r0, nr, NK, nsl, nst, units, tiles;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace)
-    int prefetch;                // L2-prefetch the next tile's score operands
-    int g_first;                 // FWD: issue G(j+1) before (1) or after (0) O_0(j)
+    int two;                     // 1: two MMA issuers (warps 9, 10); 0: warp 9 issues all
 };
 
 // Phase trace: per CTA and local tile j < TRACE_TILES, globaltimer stamps of
@@ -257,10 +256,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 
     if (warp == 8) {
         if (lane == 0) {
-            for (int i = 0; i < NST; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
-            mbar_init(s_full, 1);
+            // Arrival counts: both MMA issuers pass every slot; s_full / o_full are committed
+            // by the issuers owning a chain of that GEMM (see the MMA issuers below).
+            for (int i = 0; i < NST; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], p.two ? 2 : 1); }
+            mbar_init(s_full, MODE != FWD && p.two ? 2 : 1);
             mbar_init(p_full, 128);
-            mbar_init(o_full, 1);
+            mbar_init(o_full, dual && p.two ? 2 : 1);
             mbar_init(o_empty, 128);
             mbar_init(p_free, 1);
             for (int i = 0; i < 4; ++i) mbar_init(&p_blk[i], 128);
@@ -292,86 +293,82 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 return sslots + (size_t)st * SLOT;
             };
             auto adv = [&]() { if (++st == NST) { st = 0; ph ^= 1u; } };
-            auto load_g = [&](const Tile& T, int j) {
+            auto load_g_slice = [&](const Tile& T, int j, int s) {
                 const Maps& mp = p.maps[T.rl];
-                for (int s = 0; s < nsl; ++s) {
-                    uint8_t* sp = take();
-                    if (s == 0) trace_ev(p, j, 0);
+                uint8_t* sp = take();
+                if (s == 0) trace_ev(p, j, 0);
+                mbar_arrive_expect_tx(&full[st], ABYTES + HB);
+                tma_load_3d(sp, &mp.a1, &full[st], s * 64, T.m0, T.u);
+                tma_load_3d(sp + ABYTES, &mp.b1, &full[st], s * 64, T.m0 - w, T.u);
+                adv();
+                if (C::NA == 2) {
+                    sp = take();
                     mbar_arrive_expect_tx(&full[st], ABYTES + HB);
-                    tma_load_3d(sp, &mp.a1, &full[st], s * 64, T.m0, T.u);
-                    tma_load_3d(sp + ABYTES, &mp.b1, &full[st], s * 64, T.m0 - w, T.u);
+                    tma_load_3d(sp, &mp.a2, &full[st], s * 64, T.m0, T.u);
+                    tma_load_3d(sp + ABYTES, &mp.b2, &full[st], s * 64, T.m0 - w, T.u);
                     adv();
-                    if (C::NA == 2) {
-                        sp = take();
-                        mbar_arrive_expect_tx(&full[st], ABYTES + HB);
-                        tma_load_3d(sp, &mp.a2, &full[st], s * 64, T.m0, T.u);
-                        tma_load_3d(sp + ABYTES, &mp.b2, &full[st], s * 64, T.m0 - w, T.u);
-                        adv();
-                    }
                 }
             };
-            // Warm L2 with a future tile's score-GEMM operands so HBM keeps streaming while
-            // this tile's softmax and output phases run (they barely touch DRAM).
-            auto prefetch_g = [&](const Tile& T) {
-                const Maps& mp = p.maps[T.rl];
-                for (int s = 0; s < nsl; ++s) {
-                    tma_prefetch_l2_3d(&mp.a1, s * 64, T.m0, T.u);
-                    if (p.prefetch != 3) tma_prefetch_l2_3d(&mp.b1, s * 64, T.m0 - w, T.u);
-                    if (C::NA == 2) {
-                        tma_prefetch_l2_3d(&mp.a2, s * 64, T.m0, T.u);
-                        if (p.prefetch != 3) tma_prefetch_l2_3d(&mp.b2, s * 64, T.m0 - w, T.u);
-                    }
-                }
-            };
-            auto load_o = [&](const Tile& T, int a) {   // key blocks of accumulation a
+            auto load_o_block = [&](const Tile& T, int a, int kb) {   // key block kb of accumulation a
                 const Maps& mp = p.maps[T.rl];
                 const int c = dual ? a : a / C::NOUT;
                 const CUtensorMap* m = (C::NOUT == 2 && !dual && (a & 1)) ? &mp.ob2 : &mp.ob1;
                 const int nbox = chunk_w(d, c) / 64;
-                for (int kb = 0; kb < nkb; ++kb) {
-                    uint8_t* sp = take();
-                    mbar_arrive_expect_tx(&full[st], (dual ? 2 : 1) * nbox * OBOX);
-                    for (int b = 0; b < nbox; ++b) {
-                        tma_load_3d(sp + b * OBOX, m, &full[st], 256 * c + 64 * b, T.m0 - w + kb * KB, T.u);
-                        if (dual)
-                            tma_load_3d(sp + (nbox + b) * OBOX, &mp.ob2, &full[st], 256 * c + 64 * b,
-                                        T.m0 - w + kb * KB, T.u);
-                    }
-                    adv();
+                uint8_t* sp = take();
+                mbar_arrive_expect_tx(&full[st], (dual ? 2 : 1) * nbox * OBOX);
+                for (int b = 0; b < nbox; ++b) {
+                    tma_load_3d(sp + b * OBOX, m, &full[st], 256 * c + 64 * b, T.m0 - w + kb * KB, T.u);
+                    if (dual)
+                        tma_load_3d(sp + (nbox + b) * OBOX, &mp.ob2, &full[st], 256 * c + 64 * b,
+                                    T.m0 - w + kb * KB, T.u);
                 }
+                adv();
             };
             TileCursor cg(blockIdx.x), co(blockIdx.x);
             Tile Tg, To;
             bool hg = cg.next(p, total, Tg);
             int jg = 0, jo = 0;
             if (MODE == FWD && hg) {
-                load_g(Tg, jg++);
+                for (int s = 0; s < nsl; ++s) load_g_slice(Tg, jg, s);
+                ++jg;
                 hg = cg.next(p, total, Tg);
-                if (hg && p.prefetch == 1) prefetch_g(Tg);
             }
             while (co.next(p, total, To)) {
-                // FWD: G(j+1) precedes O(j) (P is in smem, so S can be overwritten as soon
-                // as softmax(j) is done); BWD: G(j) then O(j) (dS lives in the S columns).
-                if (hg && (MODE != FWD || p.g_first)) {
-                    load_g(Tg, jg++);
-                    hg = cg.next(p, total, Tg);
-                    if (hg && p.prefetch == 1) prefetch_g(Tg);
-                }
-                for (int a = 0; a < nacc; ++a) {
-                    if (a == nacc - 1 && hg && p.prefetch >= 2) prefetch_g(Tg);
-                    load_o(To, a);
-                    if (MODE == FWD && !p.g_first && a == 0 && hg) {
-                        load_g(Tg, jg++);
-                        hg = cg.next(p, total, Tg);
+                if (MODE == FWD) {
+                    // G(j+1) slices and O(j) key blocks alternate, the order in which the
+                    // two issuers consume them concurrently (one issuer: G(j+1) first).
+                    const int nG = hg ? nsl : 0, nO = nacc * nkb;
+                    for (int gi = 0, oi = 0; gi < nG || oi < nO;) {
+                        if (gi < nG) load_g_slice(Tg, jg, gi++);
+                        if (oi < nO && (p.two || gi == nG)) { load_o_block(To, oi / nkb, oi % nkb); ++oi; }
                     }
+                    if (hg) { ++jg; hg = cg.next(p, total, Tg); }
+                } else {   // BWD: G(j) then O(j) (dS lives in the S columns)
+                    for (int s = 0; s < nsl; ++s) load_g_slice(To, jo, s);
+                    for (int a = 0; a < nacc; ++a)
+                        for (int kb = 0; kb < nkb; ++kb) load_o_block(To, a, kb);
                 }
                 trace_ev(p, jo, 1);
                 ++jo;
             }
         }
-    } else if (warp == 9) {
-        if (lane == 0) {   // ------------------------------------------------ MMA issuer
+    } else if (warp == 9 || warp == 10) {
+        if (lane == 0 && (warp == 9 || p.two)) {   // ------------------------------ MMA issuers
+            // A dependent tcgen05.mma chain advances one instruction per ~350 cycles
+            // whatever its N, and one issuing thread sustains ~115-150 cycles per
+            // instruction (tools/mma_microbench.cu): independent chains go to different
+            // issuers.  Issuer 0: S / S^T, and the BWD outputs (BWDKV dual: dV); issuer 1:
+            // dP / dP^T, the FWD outputs O(j) (concurrent with issuer 0's G(j+1)), and
+            // BWDKV dual dK.  Both walk every ring slot in order (full wait, then commit or
+            // plain arrive on empty, count 2), so slot phases stay consistent.
+            // With p.two == 0 warp 9 owns every chain.
+            const int h = warp - 9;
+            const bool one = !p.two;
             const uint32_t idS = idesc_bf16(128, NK, false, false);
+            const bool ownS = one || h == 0, ownDP = one || h == 1;
+            const bool ownSmemA = one || (MODE == FWD ? h == 1 : h == 0);   // P / P^T operand
+            const bool ownTmemA = one || (dual ? h == 1 : h == 0);           // dS / dS^T operand
+            const int otr = MODE == FWD && !one ? 1 : 0;                     // issuer tracing outputs
             int st = 0, ga = 0;   // ga: global accumulation counter (o_full / o_empty phase)
             int jo_cur = 0;       // local index of the tile whose outputs are being issued
             uint32_t ph = 0;
@@ -380,103 +377,126 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 tc_fence_after();
                 return smem_u32(sslots + (size_t)st * SLOT);
             };
-            auto release = [&]() { mma_commit(&empty[st]); if (++st == NST) { st = 0; ph ^= 1u; } };
-            auto mma_g = [&](int j) {
-                // BWD: the score GEMMs write dP into the accumulator columns: the epilogue
-                // must have drained the previous tile's last accumulation.
-                if (MODE != FWD && !early && ga > 0) {
-                    mbar_wait(o_empty, (ga - 1) & 1);
-                    tc_fence_after();
-                }
-                for (int s = 0; s < nsl; ++s) {
-                    const uint32_t a1 = wait_full();
-                    if (s == 0) trace_ev(p, j, 2);
+            auto release = [&](bool used) {
+                if (used) mma_commit(&empty[st]);
+                else mbar_arrive(&empty[st]);
+                if (++st == NST) { st = 0; ph ^= 1u; }
+            };
+            auto g_slice = [&](int j, int s) {
+                const uint32_t a1 = wait_full();
+                if (s == 0 && h == 0) trace_ev(p, j, 2);
+                if (ownS) {
                     const uint32_t b1 = a1 + ABYTES;
-                    if (C::NA == 1) {
+#pragma unroll
+                    for (int kk = 0; kk < 4; ++kk)
+                        mma_ss(tbase, sdesc_sw128(a1 + kk * 32, 16, 1024),
+                               sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
+                }
+                release(ownS);
+                if (C::NA == 2) {
+                    const uint32_t a2 = wait_full();
+                    if (ownDP) {
+                        const uint32_t b2 = a2 + ABYTES;
 #pragma unroll
                         for (int kk = 0; kk < 4; ++kk)
-                            mma_ss(tbase, sdesc_sw128(a1 + kk * 32, 16, 1024),
-                                   sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
-                        release();
-                    } else {
-                        const int stA = st;
-                        if (++st == NST) { st = 0; ph ^= 1u; }
-                        const uint32_t a2 = wait_full(), b2 = a2 + ABYTES;
-                        // S and dP are independent accumulators: interleave their K-steps
-#pragma unroll
-                        for (int kk = 0; kk < 4; ++kk) {
-                            mma_ss(tbase, sdesc_sw128(a1 + kk * 32, 16, 1024),
-                                   sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
                             mma_ss(tbase + 256, sdesc_sw128(a2 + kk * 32, 16, 1024),
                                    sdesc_sw128(b2 + kk * 32, 16, 1024), idS, (s | kk) != 0);
-                        }
-                        mma_commit(&empty[stA]);
-                        release();
                     }
+                    release(ownDP);
                 }
-                mma_commit(s_full);
-                trace_ev(p, j, 3);
+                if (s == nsl - 1) {
+                    if ((MODE != FWD && !one) || ownS) mma_commit(s_full);
+                    if (h == 0) trace_ev(p, j, 3);
+                    if (h == 0 && MODE == FWD && j > 0) trace_ev(p, j - 1, 14);   // G(j) issued during tile j-1
+                }
             };
-            auto mma_o = [&](int a) {   // accumulation a of the current tile into [256, 256+cw)
+            auto o_block = [&](int a, int kb) {   // key block kb of accumulation a -> [acc0, acc0+cw)
                 const int c = dual ? a : a / C::NOUT;
                 const int cw = chunk_w(d, c);
                 const uint32_t idO = idesc_bf16(128, cw, false, true);
-                const bool smemA = C::PSMEM && (C::NOUT == 1 || dual || (a & 1) == 0);   // P / P^T
-                const bool tmemA = MODE == BWDQ || (MODE == BWDKV && (dual || (a & 1) == 1));   // dS / dS^T
+                const bool smemA = ownSmemA && C::PSMEM && (C::NOUT == 1 || dual || (a & 1) == 0);
+                const bool tmemA = ownTmemA && (MODE == BWDQ || (MODE == BWDKV && (dual || (a & 1) == 1)));
+                const bool own = smemA || tmemA;
                 const uint32_t sPa = smem_u32(sP);
                 const uint32_t tD0 = tbase + acc0, tD1 = tbase + acc0 + (dual ? cw : 0);
                 const uint32_t boff = dual ? (uint32_t)(cw / 64) * OBOX : 0u;   // dK's B boxes
-                if (ga > 0) {
+                // the epilogue drained the accumulator.  In BWD the other issuer waits too:
+                // it waits on o_empty again before the next score GEMMs, and a parity wait
+                // is only unambiguous while the waiter is at most one phase ahead.
+                if ((own || MODE != FWD) && kb == 0 && ga > 0) {
                     mbar_wait(o_empty, (ga - 1) & 1);
                     tc_fence_after();
                 }
-                for (int kb = 0; kb < nkb; ++kb) {
-                    if (early && a == 0) {   // dS of this 64-key block written?
-                        mbar_wait(&p_blk[kb], jo_cur & 1);
-                        tc_fence_after();
-                    }
-                    const uint32_t bb = wait_full();
-#pragma unroll
-                    for (int k4 = 0; k4 < 4; ++k4) {
-                        const int kk = kb * 4 + k4;   // 16-key step over the halo
-                        const uint32_t acc = (kk != 0);
-                        if (smemA) {   // P (FWD) or P^T (BWDKV dV) from smem
-                            const uint64_t bd = sdesc_sw128(bb + k4 * 2048, OBOX, 1024);
-                            const uint64_t ad = sdesc_sw128(sPa + (kk >> 2) * (BM * 128) + (kk & 3) * 32, 16, 1024);
-                            mma_ss(tD0, ad, bd, idO, acc);
-                        }
-                        if (tmemA) {   // dS (BWDQ) or dS^T (BWDKV dK), hi/lo in TMEM over S
-                            const uint64_t bd = sdesc_sw128(bb + boff + k4 * 2048, OBOX, 1024);
-                            const uint32_t tA = tbase + 32u * (kk >> 1) + 8u * (kk & 1);
-                            mma_ts(tD1, tA, bd, idO, acc);
-                            mma_ts(tD1, tA + 16, bd, idO, 1);
-                        }
-                    }
-                    release();
+                if (own && a == 0 && kb == 0) trace_ev(p, jo_cur, 12);
+                if (own && early && a == 0) {   // dS of this 64-key block written?
+                    mbar_wait(&p_blk[kb], jo_cur & 1);
+                    tc_fence_after();
                 }
-                mma_commit(o_full);
-                ++ga;
+                const uint32_t bb = wait_full();
+                if (own && a == 0 && kb == 0) trace_ev(p, jo_cur, 13);
+#pragma unroll
+                for (int k4 = 0; k4 < 4; ++k4) {
+                    const int kk = kb * 4 + k4;   // 16-key step over the halo
+                    const uint32_t acc = (kk != 0);
+                    if (smemA) {   // P (FWD) or P^T (BWDKV dV) from smem
+                        const uint64_t bd = sdesc_sw128(bb + k4 * 2048, OBOX, 1024);
+                        const uint64_t ad = sdesc_sw128(sPa + (kk >> 2) * (BM * 128) + (kk & 3) * 32, 16, 1024);
+                        mma_ss(tD0, ad, bd, idO, acc);
+                    }
+                    if (tmemA) {   // dS (BWDQ) or dS^T (BWDKV dK), hi/lo in TMEM over S
+                        const uint64_t bd = sdesc_sw128(bb + boff + k4 * 2048, OBOX, 1024);
+                        const uint32_t tA = tbase + 32u * (kk >> 1) + 8u * (kk & 1);
+                        mma_ts(tD1, tA, bd, idO, acc);
+                        mma_ts(tD1, tA + 16, bd, idO, 1);
+                    }
+                }
+                release(own);
+                if (kb == nkb - 1) {
+                    if (own) mma_commit(o_full);
+                    ++ga;
+                }
             };
             TileCursor cg(blockIdx.x), co(blockIdx.x);
             Tile Tg, To;
             bool hg = cg.next(p, total, Tg);
             int jg = 0, jo = 0;
-            if (MODE == FWD && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }   // G(0)
+            if (MODE == FWD && hg) {   // G(0)
+                for (int s = 0; s < nsl; ++s) g_slice(jg, s);
+                ++jg;
+                hg = cg.next(p, total, Tg);
+            }
             while (co.next(p, total, To)) {
-                if (MODE != FWD) { mma_g(jg++); hg = cg.next(p, total, Tg); }
                 jo_cur = jo;
-                if (!early) {   // early BWDQ waits per key block inside mma_o
+                if (MODE != FWD) {
+                    // the score GEMMs write dP into the accumulator columns (unless early):
+                    // the epilogue must have drained the previous tile's last accumulation
+                    if (!early && ga > 0) {
+                        mbar_wait(o_empty, (ga - 1) & 1);
+                        tc_fence_after();
+                    }
+                    for (int s = 0; s < nsl; ++s) g_slice(jo, s);
+                }
+                // FWD: S(j) consumed (G(j+1) may overwrite it) and P(j) in smem.  BWD: dS
+                // written; early BWDQ hands dS to issuer 0 per key block instead, and issuer
+                // 1 waits here so that dP(j+1) does not overwrite dP(j) under the softmax.
+                if (!(early && h == 0)) {
                     mbar_wait(p_full, jo & 1);
                     tc_fence_after();
                 }
-                trace_ev(p, jo, 4);
-                if (MODE == FWD && p.g_first && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
-                for (int a = 0; a < nacc; ++a) {
-                    mma_o(a);
-                    if (MODE == FWD && !p.g_first && a == 0 && hg) { mma_g(jg++); hg = cg.next(p, total, Tg); }
+                if (h == otr) trace_ev(p, jo, 4);
+                if (MODE == FWD) {
+                    const int nG = hg ? nsl : 0, nO = nacc * nkb;
+                    for (int gi = 0, oi = 0; gi < nG || oi < nO;) {
+                        if (gi < nG) g_slice(jg, gi++);
+                        if (oi < nO && (p.two || gi == nG)) { o_block(oi / nkb, oi % nkb); ++oi; }
+                    }
+                    if (hg) { ++jg; hg = cg.next(p, total, Tg); }
+                } else {
+                    for (int a = 0; a < nacc; ++a)
+                        for (int kb = 0; kb < nkb; ++kb) o_block(a, kb);
                 }
-                if (C::PSMEM) mma_commit(p_free);
-                trace_ev(p, jo, 5);
+                if (C::PSMEM && ownSmemA) mma_commit(p_free);
+                if (h == otr) trace_ev(p, jo, 5);
                 ++jo;
             }
         }
@@ -791,12 +811,10 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         p.nr = nr;
         p.trace = (unsigned long long*)trace_buffer(MODE);
         {
-            const char* pf = getenv("FT_WINATTN_L2PF");   // tuning knob: 0 disables prefetch
-            p.prefetch = pf ? atoi(pf) : 0;
-            const char* gf = getenv("FT_WINATTN_GFIRST");
-            // measured (profiles/README.md): G(j+1) before O(j) wins when the output is
-            // one chunk (d <= 256); at d = 512 issuing it between the two chunks wins.
-            p.g_first = gf ? atoi(gf) : (d <= 256 ? 1 : 0);
+            // Two issuers (measured faster for every mode and d, profiles/README.md);
+            // FT_WINATTN_ISSUERS=1 restores the single-issuer schedule for A/B timing.
+            const char* e = getenv("FT_WINATTN_ISSUERS");
+            p.two = !(e && atoi(e) == 1);
         }
         p.units = (int)units;
         p.tiles = (int)ceil_div(Lr0, BM);

@@ -35,14 +35,19 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
                  "r"(bytes)
                  : "memory");
 }
+// try_wait suspends the waiting thread until the phase completes or the hint (ns) elapses,
+// so warps parked on a barrier do not take issue slots from the working warps.
+#ifndef FT_MBAR_SUSPEND_NS
+#define FT_MBAR_SUSPEND_NS 0x989680u
+#endif
 __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
     uint32_t ok;
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
         "selp.u32 %0, 1, 0, p;\n\t}"
         : "=r"(ok)
-        : "r"(smem_u32(bar)), "r"(parity)
+        : "r"(smem_u32(bar)), "r"(parity), "r"(FT_MBAR_SUSPEND_NS)
         : "memory");
     return ok != 0;
 }

@@ -117,7 +117,71 @@ __global__ void bench(int mode, int N, int nacc, int iters, unsigned long long* 
     if (warp == 0) { tc_fence_after(); tmem_dealloc(tb, 512); }
 }
 
+__global__ void bench_multi(int N, int nacc, int issuers, int iters, unsigned long long* out, int wstride = 1) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    __shared__ uint32_t holder;
+    __shared__ uint64_t bar[4];
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    for (int i = threadIdx.x; i < 64 * 1024 / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(smem)[i] = 0;
+    if (warp == 0) { tmem_alloc(&holder, 512); tmem_relinquish(); }
+    if (threadIdx.x == 0) { for (int i = 0; i < 4; ++i) mbar_init(&bar[i], 1); fence_barrier_init(); }
+    fence_proxy_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tb = holder;
+    unsigned long long t0 = clock64();
+    if (warp % wstride == 0 && warp / wstride < issuers && lane == 0) {
+        const uint32_t sa = smem_u32(smem), sb = sa + 16384;
+        const uint32_t id = idesc_bf16(128, N, false, false);
+        for (int i = 0; i < iters; ++i)
+            for (int a = 0; a < nacc; ++a) {
+                const uint32_t d = tb + (uint32_t)(((warp / wstride) * nacc + a) * N);
+                const int kk = i & 3;
+                mma_ss(d, sdesc_sw128(sa + kk * 32, 16, 1024), sdesc_sw128(sb + kk * 32, 16, 1024), id, 1);
+            }
+        mma_commit(&bar[warp / wstride]);
+        mbar_wait(&bar[warp / wstride], 0);
+    }
+    __syncthreads();
+    unsigned long long t1 = clock64();
+    if (threadIdx.x == 0) out[blockIdx.x] = t1 - t0;
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) { tc_fence_after(); tmem_dealloc(tb, 512); }
+}
+
 int main() {
+    {
+        unsigned long long* dd;
+        cudaMalloc(&dd, 8 * 148);
+        cudaFuncSetAttribute(bench_multi, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+        const int iters = 2048;
+        struct M { int N, nacc, issuers; };
+        for (int rep = 0; rep < 2; ++rep)
+        for (M m : {M{128, 1, 1}, M{128, 2, 1}, M{128, 4, 1}, M{128, 1, 2}, M{128, 2, 2}, M{128, 1, 3},
+                    M{256, 1, 1}, M{256, 1, 2}, M{256, 2, 2}, M{64, 1, 1}, M{64, 1, 2}, M{64, 1, 4}}) {
+            bench_multi<<<148, 128, 96 * 1024>>>(m.N, m.nacc, m.issuers, iters, dd);
+            unsigned long long h[148] = {0};
+            cudaMemcpy(h, dd, 8 * 148, cudaMemcpyDeviceToHost);
+            double mx = 0;
+            for (int i = 0; i < 148; ++i) mx = h[i] > mx ? h[i] : mx;
+            const double total = (double)iters * m.nacc * m.issuers;
+            printf("multi-issuer SS M=128 N=%3d chains/issuer=%d issuers=%d: %6.1f clk/MMA per issuer, %5.0f MAC/clk/SM\n",
+                   m.N, m.nacc, m.issuers, mx / (total / m.issuers), 128.0 * m.N * 16 * total / mx);
+        }
+        for (M m : {M{64, 2, 2}, M{128, 2, 2}}) {   // issuers on warps 0 and 4: same SM sub-partition
+            bench_multi<<<148, 256, 96 * 1024>>>(m.N, m.nacc, m.issuers, iters, dd, 4);
+            unsigned long long h[148] = {0};
+            cudaMemcpy(h, dd, 8 * 148, cudaMemcpyDeviceToHost);
+            double mx = 0;
+            for (int i = 0; i < 148; ++i) mx = h[i] > mx ? h[i] : mx;
+            const double total = (double)iters * m.nacc * m.issuers;
+            printf("multi-issuer same-SMSP N=%3d acc/issuer=%d issuers=%d: %6.1f clk per MMA, %5.0f MAC/clk/SM\n",
+                   m.N, m.nacc, m.issuers, mx / total, 128.0 * m.N * 16 * total / mx);
+        }
+    }
+
     unsigned long long* d;
     cudaMalloc(&d, 8 * 148);
     cudaFuncSetAttribute(bench, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);

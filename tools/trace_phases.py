@@ -43,7 +43,7 @@ def main():
         lib.ft_winattn_debug_trace(m, None)
     for m, name in enumerate(["FWD", "BWDQ", "BWDKV"]):
         t = bufs[m].view(148, 8, 48).cpu().double()
-        valid = (t[:, :, :10] > 0).all(dim=2)
+        valid = (t[:, :, :10] > 0).all(dim=2) & (t[:, :, 12] > 0) & (t[:, :, 13] > 0)
         t0 = t[:, 0, 0][t[:, 0, 0] > 0].min()
         t = (t - t0) / 1e3
         print(f"== {name}: kernel span {t[valid].max():.1f} us, tiles traced {int(valid.sum())}")
@@ -58,6 +58,10 @@ def main():
             print(f"    pass 2 (exp, P -> smem)         {med(t[:,:,7]-t[:,:,11]):7.2f}")
         print(f"  p arrive -> mma sees p            {med(t[:,:,4]-t[:,:,7]):7.2f}")
         print(f"  output MMAs issued (p -> out end) {med(t[:,:,5]-t[:,:,4]):7.2f}")
+        print(f"    p seen -> o_empty passed        {med(t[:,:,12]-t[:,:,4]):7.2f}")
+        print(f"    o_empty -> first O block full   {med(t[:,:,13]-t[:,:,12]):7.2f}")
+        if name == "FWD":
+            print(f"    p seen -> G(j+1) issued         {med(t[:,:,14]-t[:,:,4]):7.2f}")
         print(f"  epilogue (first o_full -> done)   {med(t[:,:,9]-t[:,:,8]):7.2f}")
         print(f"  tile period (g1 ready j -> j+1)   {float((t[:,1:,2]-t[:,:-1,2])[valid[:,1:] & valid[:,:-1]].median()):7.2f}")
         print(f"  producer span per tile            {med(t[:,:,1]-t[:,:,0]):7.2f}")
