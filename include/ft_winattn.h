@@ -111,8 +111,9 @@ ft_status ft_winattn_profile_events(void* const* events, int n);
 /* Debug trace (off by default): while device_buffer is non-NULL, tensor-core kernels of
  * the given mode (0 = forward, 1 = backward dq, 2 = backward dk/dv) launched from the
  * calling host thread write globaltimer stamps of their pipeline phases into it:
- * uint64 [gridDim.x][8 tiles][10 events] (layout documented in csrc/tc_band.cu).  The
- * buffer must hold 148*8*10*8 bytes per SM-sized grid.  Profiling only. */
+ * uint64 [gridDim.x][8 tiles][48 slots] (slot meanings documented in csrc/tc_band.cu and
+ * csrc/tc_wide.cu).  The buffer must hold 148*8*48*8 bytes per SM-sized grid.  Profiling
+ * only. */
 ft_status ft_winattn_debug_trace(int kernel_mode, void* device_buffer);
 
 /* Human-readable text for a status (static storage, never NULL).  For FT_ERR_CUDA it

@@ -76,6 +76,13 @@ cudaError_t tc_chunk_bwd(const void* q, const void* k, const void* v, const floa
                          int* launches);
 int tc_chunk_launches(int64_t L, int64_t dil);
 
+// wide-window forward, two-pass with partial accumulators -- tc_wide.cu
+bool tc_wide_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+cudaError_t tc_wide_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
+                        int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                        cudaStream_t st, int* launches);
+int tc_wide_launches(int64_t L, int64_t dil);
+
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();
 void* trace_buffer(int kernel_mode);   // ft_winattn_debug_trace target for a kernel mode, or null

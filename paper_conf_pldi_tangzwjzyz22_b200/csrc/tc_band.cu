@@ -865,8 +865,12 @@ cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float
                    int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
                    int* launches) {
     if (launches) *launches = 0;
-    if (halo_rows(L, w) > 256)
-        return tc_chunk_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
+    if (halo_rows(L, w) > 256) {
+        const char* v1 = getenv("FT_WINATTN_WIDE_V1");   // A/B timing: previous chunk kernel
+        if ((v1 && atoi(v1) == 1) || !tc_wide_supported(B * H, L, d, w, dil))
+            return tc_chunk_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
+        return tc_wide_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
+    }
     return launch<FWD>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, B, H, L,
                        d, w, dil, st, launches);
 }
