@@ -158,6 +158,33 @@ def test_overflow_probe(ft):
         run_case(ft, WinAttnShape(1, 1, 256, 64, 16, 1), dt, None, seed=4, q_scale=16.0)
 
 
+@pytest.mark.parametrize("d,sign", [(64, 1.0), (128, 1.0), (64, -1.0)])
+def test_wide_lazy_rescale(ft, d, sign):
+    """Wide-window forward (csrc/tc_wide.cu) with scores that grow along the keys: q = 1,
+    k_j = sign * 0.002 * j (+ noise), so s_ij = sign * 0.002 * d * j and every later chunk's max
+    exceeds the running one by more than the 2^20 lazy-rescale threshold -- the rescale and
+    redo path that random inputs never reach.  sign = -1: the max sits in the first chunks."""
+    L, w = 1000, 100
+    shape = WinAttnShape(1, 2, L, d, w, 1)
+    x = make_inputs(shape, 9, "bf16")
+    j = torch.arange(L, dtype=torch.float64).view(1, 1, L, 1)
+    q64 = torch.ones(1, 2, L, d, dtype=torch.float64)
+    k64 = sign * 0.002 * j + 0.01 * torch.from_numpy(x["k64"])
+    q = q64.to(torch.bfloat16)
+    k = k64.to(torch.bfloat16)
+    qn, kn = q.double().numpy(), k.double().numpy()
+    dev = torch.device("cuda:0")
+    v, g = x["v"].to(dev), x["dout"].to(dev)
+    out, lse = ft.fwd(q.to(dev), k.to(dev), v, w, 1)
+    ro, rl = oracle.fwd(qn, kn, x["v64"], w, 1)
+    compare("out", out.double().cpu().numpy(), ro, "bf16")
+    compare("lse", lse.double().cpu().numpy(), rl, "bf16")
+    dq, dk, dv = ft.bwd(q.to(dev), k.to(dev), v, out, lse, g, w, 1)
+    r = oracle.bwd(qn, kn, x["v64"], ro, rl, x["dout64"], w, 1)
+    for n, a, b in zip(("dq", "dk", "dv"), (dq, dk, dv), r):
+        compare(n, a.double().cpu().numpy(), b, "bf16")
+
+
 def test_dout_ones(ft):
     """the gradient seed of JAX/Julia is sum(outputs) -> dout = 1."""
     shape = WinAttnShape(1, 1, 200, 64, 8, 2)
