@@ -82,6 +82,12 @@ cudaError_t tc_wide_fwd(const void* q, const void* k, const void* v, void* out, 
                         int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                         cudaStream_t st, int* launches);
 int tc_wide_launches(int64_t L, int64_t dil);
+// wide-window backward, TMEM region rotation, three MMA issuers -- tc_wide_bwd.cu
+bool tc_wide_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+cudaError_t tc_wide_bwd(const void* q, const void* k, const void* v, const float* lse,
+                        const void* dout, void* dq, void* dk, void* dv, float* Dws, int64_t B,
+                        int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
+                        int* launches);
 
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();

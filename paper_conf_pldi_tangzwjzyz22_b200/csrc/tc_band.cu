@@ -881,8 +881,12 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
                    cudaStream_t st, int* launches) {
     (void)out;   // D_i is recomputed exactly as sum_j P_ij dP_ij by the BWDQ kernel
     if (launches) *launches = 0;
-    if (halo_rows(L, w) > 256)
-        return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
+    if (halo_rows(L, w) > 256) {
+        const char* v1 = getenv("FT_WINATTN_WIDE_V1");   // A/B timing: previous chunk kernels
+        if ((v1 && atoi(v1) == 1) || !tc_wide_bwd_supported(B * H, L, d, w, dil))
+            return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
+        return tc_wide_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
+    }
     cudaError_t e = launch<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse),
                                  Dws, B, H, L, d, w, dil, st, launches);
     if (e != cudaSuccess) return e;
