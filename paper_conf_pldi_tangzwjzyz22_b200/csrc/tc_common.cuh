@@ -231,6 +231,16 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
 }
 
 __device__ __forceinline__ uint32_t elect_lane0() { return (threadIdx.x & 31u) == 0u; }
+// One lane of a converged warp (elect.sync).  Whole-warp MMA issuers run their loop on all
+// 32 lanes -- descriptors stay warp-uniform (uniform registers) -- and issue through the
+// elected lane: ~1.5x the MMA issue rate of a lane-0-only issuer when several accumulator
+// chains are in flight (tools/mma_microbench.cu).
+__device__ __forceinline__ uint32_t elect_one() {
+    uint32_t e;
+    asm volatile("{\n\t.reg .pred p;\n\telect.sync _|p, 0xffffffff;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                 : "=r"(e));
+    return e;
+}
 
 }  // namespace tc
 }  // namespace ftw

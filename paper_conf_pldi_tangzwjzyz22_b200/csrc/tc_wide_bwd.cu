@@ -69,7 +69,21 @@ struct BParams {
     int64_t L;
     int d, w, dil, r0, nr, nkc, units, tiles;
     int na, n1, n2;   // row-operand buffers, ring-1 / ring-2 slots
+    unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, mode 1 / 2)
 };
+
+// Phase trace, per CTA and local tile j < 8, 48 uint64 slots (ns sums over the tile):
+// softmax warp 0: 0 tile start, 1 S/dP wait, 2 compute, 6 tile end; issuer A: 10 region
+// wait, 11 ring wait; issuer B: 14 region wait, 15 ring wait; issuer C: 20 p_full wait,
+// 21 o_empty wait; epilogue: 30 o_full seen, 31 done.
+__device__ __forceinline__ unsigned long long gtime() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ void trace_put(const BParams& p, int j, int slot, unsigned long long v) {
+    if (p.trace && j < 8) p.trace[((size_t)blockIdx.x * 8 + j) * 48 + slot] = v;
+}
 
 struct Tile {
     int u, rl, r, Lr, m0;
@@ -262,12 +276,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 mbar_wait(&a_full[ab], (j / p.na) & 1);
                 tc_fence_after();
                 const uint32_t sa = smem_u32(sA + (size_t)ab * 2 * RB + (isA ? 0 : RB));
+                const bool tr = p.trace && j < 8;
+                unsigned long long wr = 0, wf = 0, t0 = 0;
                 for (int k = 0; k < nsteps; ++k, ++gk) {
                     const int m = 2 * gk + (isA ? 0 : 1);
+                    if (tr) t0 = gtime();
                     wait_region(m);
+                    if (tr) { wr += gtime() - t0; t0 = gtime(); }
                     uint64_t* fullb = isA ? r1_full : r2_full;
                     mbar_wait(&fullb[rr.s], rr.ph);
                     tc_fence_after();
+                    if (tr) wf += gtime() - t0;
                     const uint32_t sb = smem_u32((isA ? sR1 : sR2) + (size_t)rr.s * SB);
                     const uint32_t td = tbase + region_col(m);
                     for (int s = 0; s < nds; ++s) {
@@ -286,6 +305,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     }
                 }
                 mma_commit(&a_empty[ab]);
+                if (tr) { trace_put(p, j, isA ? 10 : 14, wr); trace_put(p, j, isA ? 11 : 15, wf); }
                 if (MODE == WKV && !isA) {   // the tile's last dV
                     if (nsteps == 1 && j > 0) { mbar_wait(o_empty, (j - 1) & 1); tc_fence_after(); }
                     issue_dv(gk - 1, nsteps == 1);
@@ -307,9 +327,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             const uint32_t acc_lo = d == 64 ? acc_hi + (uint32_t)d : acc_hi;
             while (cur.next(p, total, T)) {
                 int outk = 0;   // output steps issued in this tile
+                const bool tr = p.trace && j < 8;
+                unsigned long long wp = 0, wo = 0, t0 = 0;
                 for (int k = 0; k < nsteps; ++k, ++gk) {
+                    if (tr) t0 = gtime();
                     mbar_wait(&p_full[gk & 3], (gk >> 2) & 1);
                     tc_fence_after();
+                    if (tr) wp += gtime() - t0;
                     const bool out = MODE == WKV || k >= nkc;
                     const int mS = 2 * gk, mD = 2 * gk + 1;
                     if (!out) {   // WQ pass 1: the softmax only read S and dP
@@ -319,7 +343,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                         r1.adv(p.n1);
                         continue;
                     }
+                    if (tr) t0 = gtime();
                     if (outk == 0 && j > 0) { mbar_wait(o_empty, (j - 1) & 1); tc_fence_after(); }
+                    if (tr) wo += gtime() - t0;
                     const uint32_t xa = region_col(MODE == WQ ? mS : mD);   // dS (hi/lo) region
                     const uint32_t sb = smem_u32(sR1 + (size_t)r1.s * SB);
 #pragma unroll
@@ -337,6 +363,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     ++outk;
                 }
                 mma_commit(o_full);
+                if (tr) { trace_put(p, j, 20, wp); trace_put(p, j, 21, wo); }
                 ++j;
             }
         }
@@ -364,6 +391,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             } else {
                 lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
             }
+            const bool tr = p.trace && j < 8 && warp == 0 && lane == 0;
+            unsigned long long ws = 0, wc = 0, t0 = 0, t1 = 0;
+            if (tr) trace_put(p, j, 0, gtime());
             for (int k = 0; k < nsteps; ++k, ++gk) {
                 const int c = k % nkc;
                 const bool pass2 = MODE == WQ && k >= nkc;
@@ -375,9 +405,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 }
                 const uint32_t xs = tbase + lrow + region_col(2 * gk) + 32u * hf;
                 const uint32_t xd = tbase + lrow + region_col(2 * gk + 1) + 32u * hf;
+                if (tr) t0 = gtime();
                 mbar_wait(&s_full[gk & 3], (gk >> 2) & 1);
                 mbar_wait(&dp_full[gk & 3], (gk >> 2) & 1);
                 tc_fence_after();
+                if (tr) { t1 = gtime(); ws += t1 - t0; t0 = t1; }
                 const int h0 = c * KC + 32 * hf;   // first halo column of my 32
                 uint32_t rs[32], rd[32];
                 tmem_ld32(xs, rs);
@@ -433,7 +465,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 if (MODE == WKV || pass2) tmem_wait_st();
                 tc_fence_before();
                 mbar_arrive(&p_full[gk & 3]);
+                if (tr) wc += gtime() - t0;
             }
+            if (tr) { trace_put(p, j, 1, ws); trace_put(p, j, 2, wc); trace_put(p, j, 6, gtime()); }
             ++j;
         }
     } else if (warp < 12) {   // ----------------------------------------- epilogue warps
@@ -447,6 +481,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             const BMaps& mp = p.maps[T.rl];
             mbar_wait(o_full, j & 1);
             tc_fence_after();
+            if (ew == 0 && lane == 0) trace_put(p, j, 30, gtime());
             if (lane == 0) tma_store_wait_read<0>();   // staging of the previous tile read
             __syncwarp();
             // WQ: dQ = [0, d) (+ [d, 2d) for d = 64);  WKV: dV = [0, d), dK = [d, 2d) (+ [2d, 3d))
@@ -494,6 +529,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     }
                 }
             }
+            if (ew == 0 && lane == 0) trace_put(p, j, 31, gtime());
             ++j;
         }
         if (lane == 0) tma_store_wait_all<0>();
@@ -584,6 +620,7 @@ cudaError_t launch(const void* a1, const void* a2, const void* b1, const void* b
         p.na = na;
         p.n1 = n1;
         p.n2 = n2;
+        p.trace = (unsigned long long*)trace_buffer(MODE == WQ ? 1 : 2);
         const int64_t Lr0 = ceil_div(L - r0, dil);
         p.tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = (int64_t)p.units * p.nr * p.tiles;

@@ -9,6 +9,12 @@
 #include "tc_common.cuh"
 
 using namespace ftw::tc;
+__device__ __forceinline__ uint32_t elect_one() {
+    uint32_t e;
+    asm volatile("{\n\t.reg .pred p;\n\telect.sync _|p, 0xffffffff;\n\tselp.u32 %0, 1, 0, p;\n\t}" : "=r"(e));
+    return e;
+}
+
 
 // whole-warp variants: all 32 lanes execute, one elected lane issues
 __device__ __forceinline__ void mma_ss_w(uint32_t d, uint64_t a, uint64_t b, uint32_t id, uint32_t acc) {
@@ -117,7 +123,8 @@ __global__ void bench(int mode, int N, int nacc, int iters, unsigned long long* 
     if (warp == 0) { tc_fence_after(); tmem_dealloc(tb, 512); }
 }
 
-__global__ void bench_multi(int N, int nacc, int issuers, int iters, unsigned long long* out, int wstride = 1) {
+template <bool WW>
+__global__ void bench_multi_t(int N, int nacc, int issuers, int iters, unsigned long long* out, int wstride = 1) {
     extern __shared__ __align__(1024) uint8_t smem[];
     __shared__ uint32_t holder;
     __shared__ uint64_t bar[4];
@@ -131,17 +138,61 @@ __global__ void bench_multi(int N, int nacc, int issuers, int iters, unsigned lo
     tc_fence_after();
     const uint32_t tb = holder;
     unsigned long long t0 = clock64();
-    if (warp % wstride == 0 && warp / wstride < issuers && lane == 0) {
+    if (warp % wstride == 0 && warp / wstride < issuers && (WW || lane == 0)) {
         const uint32_t sa = smem_u32(smem), sb = sa + 16384;
         const uint32_t id = idesc_bf16(128, N, false, false);
         for (int i = 0; i < iters; ++i)
             for (int a = 0; a < nacc; ++a) {
                 const uint32_t d = tb + (uint32_t)(((warp / wstride) * nacc + a) * N);
                 const int kk = i & 3;
-                mma_ss(d, sdesc_sw128(sa + kk * 32, 16, 1024), sdesc_sw128(sb + kk * 32, 16, 1024), id, 1);
+                if (WW) { if (elect_one()) mma_ss(d, sdesc_sw128(sa + kk * 32, 16, 1024), sdesc_sw128(sb + kk * 32, 16, 1024), id, 1); }
+                else mma_ss(d, sdesc_sw128(sa + kk * 32, 16, 1024), sdesc_sw128(sb + kk * 32, 16, 1024), id, 1);
             }
-        mma_commit(&bar[warp / wstride]);
+        if (WW) { if (elect_one()) mma_commit(&bar[warp / wstride]); }
+        else mma_commit(&bar[warp / wstride]);
         mbar_wait(&bar[warp / wstride], 0);
+    }
+    __syncthreads();
+    unsigned long long t1 = clock64();
+    if (threadIdx.x == 0) out[blockIdx.x] = t1 - t0;
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) { tc_fence_after(); tmem_dealloc(tb, 512); }
+}
+
+// Whole-warp issuer: all 32 lanes run the loop (descriptors warp-uniform, so they can
+// live in uniform registers); one elected lane issues each MMA (elect.sync).
+__device__ __forceinline__ void mma_ss_elect(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
+                                             uint32_t idesc, uint32_t accumulate) {
+    if (elect_one()) mma_ss(d_tmem, adesc, bdesc, idesc, accumulate);
+}
+__device__ __forceinline__ void commit_elect(uint64_t* bar) {
+    if (elect_one()) mma_commit(bar);
+}
+__global__ void bench_warp(int N, int nacc, int iters, unsigned long long* out) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    __shared__ uint32_t holder;
+    __shared__ uint64_t bar;
+    const int warp = threadIdx.x / 32;
+    for (int i = threadIdx.x; i < 64 * 1024 / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(smem)[i] = 0;
+    if (warp == 0) { tmem_alloc(&holder, 512); tmem_relinquish(); }
+    if (threadIdx.x == 0) { mbar_init(&bar, 1); fence_barrier_init(); }
+    fence_proxy_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tb = holder;
+    unsigned long long t0 = clock64();
+    if (warp == 1) {   // whole warp
+        const uint32_t sa = smem_u32(smem), sb = sa + 16384;
+        const uint32_t id = idesc_bf16(128, N, false, false);
+        for (int i = 0; i < iters; ++i)
+            for (int a = 0; a < nacc; ++a) {
+                const int kk = i & 3;
+                mma_ss_elect(tb + (uint32_t)(a * N), sdesc_sw128(sa + kk * 32, 16, 1024), sdesc_sw128(sb + kk * 32, 16, 1024), id, 1);
+            }
+        commit_elect(&bar);
+        mbar_wait(&bar, 0);
     }
     __syncthreads();
     unsigned long long t1 = clock64();
@@ -155,13 +206,45 @@ int main() {
     {
         unsigned long long* dd;
         cudaMalloc(&dd, 8 * 148);
-        cudaFuncSetAttribute(bench_multi, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+        cudaFuncSetAttribute(bench_warp, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+        const int iters = 2048;
+        for (int rep = 0; rep < 2; ++rep)
+        for (int nacc : {1, 2, 4}) for (int N : {64, 128}) {
+            bench_warp<<<148, 128, 96 * 1024>>>(N, nacc, iters, dd);
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) { printf("launch err %s\n", cudaGetErrorString(e)); return 1; }
+            e = cudaDeviceSynchronize();
+            if (e != cudaSuccess) { printf("err %s\n", cudaGetErrorString(e)); return 1; }
+            unsigned long long h[148] = {0};
+            cudaMemcpy(h, dd, 8 * 148, cudaMemcpyDeviceToHost);
+            double mx = 0;
+            for (int i = 0; i < 148; ++i) mx = h[i] > mx ? h[i] : mx;
+            printf("whole-warp issuer (elect.sync) N=%3d chains=%d: %6.1f clk/MMA\n", N, nacc, mx / ((double)iters * nacc));
+        }
+    }
+
+    {
+        unsigned long long* dd;
+        cudaMalloc(&dd, 8 * 148);
+        cudaFuncSetAttribute(bench_multi_t<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
         const int iters = 2048;
         struct M { int N, nacc, issuers; };
-        for (int rep = 0; rep < 2; ++rep)
+        cudaFuncSetAttribute(bench_multi_t<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+        for (M m : {M{128, 1, 1}, M{128, 2, 1}, M{128, 4, 1}, M{64, 2, 1}, M{128, 2, 2}}) {
+            bench_multi_t<true><<<148, 128, 96 * 1024>>>(m.N, m.nacc, m.issuers, iters, dd);
+            cudaDeviceSynchronize();
+            unsigned long long h[148] = {0};
+            cudaMemcpy(h, dd, 8 * 148, cudaMemcpyDeviceToHost);
+            double mx = 0;
+            for (int i = 0; i < 148; ++i) mx = h[i] > mx ? h[i] : mx;
+            const double total = (double)iters * m.nacc * m.issuers;
+            printf("WHOLE-WARP issuer N=%3d chains/issuer=%d issuers=%d: %6.1f clk/MMA per issuer\n",
+                   m.N, m.nacc, m.issuers, mx / (total / m.issuers));
+        }
+        for (int rep = 0; rep < 1; ++rep)
         for (M m : {M{128, 1, 1}, M{128, 2, 1}, M{128, 4, 1}, M{128, 1, 2}, M{128, 2, 2}, M{128, 1, 3},
                     M{256, 1, 1}, M{256, 1, 2}, M{256, 2, 2}, M{64, 1, 1}, M{64, 1, 2}, M{64, 1, 4}}) {
-            bench_multi<<<148, 128, 96 * 1024>>>(m.N, m.nacc, m.issuers, iters, dd);
+            bench_multi_t<false><<<148, 128, 96 * 1024>>>(m.N, m.nacc, m.issuers, iters, dd);
             unsigned long long h[148] = {0};
             cudaMemcpy(h, dd, 8 * 148, cudaMemcpyDeviceToHost);
             double mx = 0;
@@ -171,7 +254,7 @@ int main() {
                    m.N, m.nacc, m.issuers, mx / (total / m.issuers), 128.0 * m.N * 16 * total / mx);
         }
         for (M m : {M{64, 2, 2}, M{128, 2, 2}}) {   // issuers on warps 0 and 4: same SM sub-partition
-            bench_multi<<<148, 256, 96 * 1024>>>(m.N, m.nacc, m.issuers, iters, dd, 4);
+            bench_multi_t<false><<<148, 256, 96 * 1024>>>(m.N, m.nacc, m.issuers, iters, dd, 4);
             unsigned long long h[148] = {0};
             cudaMemcpy(h, dd, 8 * 148, cudaMemcpyDeviceToHost);
             double mx = 0;
