@@ -89,6 +89,13 @@ cudaError_t tc_wide_bwd(const void* q, const void* k, const void* v, const float
                         int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
                         int* launches);
 
+// d = 64, w <= 32 forward with two ping-pong softmax warpgroups -- tc_narrow.cu
+bool tc_narrow_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+cudaError_t tc_narrow_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
+                          int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                          cudaStream_t st, int* launches);
+int tc_narrow_launches(int64_t L, int64_t dil);
+
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();
 void* trace_buffer(int kernel_mode);   // ft_winattn_debug_trace target for a kernel mode, or null

@@ -854,11 +854,12 @@ bool tc_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t di
     return tc_fwd_supported(units, L, d, w, dil);
 }
 int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
-    (void)d;
+    if (tc_narrow_supported(1, L, d, w, dil)) return tc_narrow_launches(L, dil);
     return halo_rows(L, w) <= 256 ? band_launches(L, dil) : tc_chunk_launches(L, dil);
 }
 int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
-    return 2 * tc_fwd_launches(L, d, w, dil);
+    (void)d;
+    return 2 * (halo_rows(L, w) <= 256 ? band_launches(L, dil) : tc_chunk_launches(L, dil));
 }
 
 cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B,
@@ -871,6 +872,8 @@ cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float
             return tc_chunk_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
         return tc_wide_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
     }
+    if (tc_narrow_supported(B * H, L, d, w, dil))
+        return tc_narrow_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
     return launch<FWD>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, B, H, L,
                        d, w, dil, st, launches);
 }
