@@ -95,6 +95,11 @@ cudaError_t tc_narrow_fwd(const void* q, const void* k, const void* v, void* out
                           int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                           cudaStream_t st, int* launches);
 int tc_narrow_launches(int64_t L, int64_t dil);
+bool tc_narrow_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+cudaError_t tc_narrow_bwd(const void* q, const void* k, const void* v, const float* lse,
+                          const void* dout, void* dq, void* dk, void* dv, float* Dws, int64_t B,
+                          int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
+                          int* launches);
 
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();

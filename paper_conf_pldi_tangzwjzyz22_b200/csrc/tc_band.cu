@@ -858,7 +858,7 @@ int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
     return halo_rows(L, w) <= 256 ? band_launches(L, dil) : tc_chunk_launches(L, dil);
 }
 int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
-    (void)d;
+    if (tc_narrow_bwd_supported(1, L, d, w, dil)) return 2 * tc_narrow_launches(L, dil);
     return 2 * (halo_rows(L, w) <= 256 ? band_launches(L, dil) : tc_chunk_launches(L, dil));
 }
 
@@ -890,6 +890,8 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
             return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
         return tc_wide_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     }
+    if (tc_narrow_bwd_supported(B * H, L, d, w, dil))
+        return tc_narrow_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     cudaError_t e = launch<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse),
                                  Dws, B, H, L, d, w, dil, st, launches);
     if (e != cudaSuccess) return e;

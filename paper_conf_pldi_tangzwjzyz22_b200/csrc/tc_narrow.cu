@@ -322,6 +322,12 @@ bool tc_narrow_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t
     return d == D && wc <= 32 && dil <= 256 && units * ((L + BM - 1) / BM) < (1 << 30);
 }
 
+bool tc_narrow_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    const char* e = getenv("FT_WINATTN_NARROW_BWD");   // A/B timing: 0 falls back to tc_band
+    if (e && atoi(e) == 0) return false;
+    return tc_narrow_supported(units, L, d, w, dil);
+}
+
 int tc_narrow_launches(int64_t L, int64_t dil) {
     const int64_t nres = dil < L ? dil : L;
     return (int)ceil_div(nres, RES_PER_LAUNCH);

@@ -152,17 +152,18 @@ def test_default_path_seeds(ft, seed):
     run_case(ft, WinAttnShape(1, 1, 192, 64, 8, 1), "f32", None, seed=seed)
 
 
-# d = 64, w <= 32 forward (tc_narrow.cu): enough tiles per CTA that the 3-stage TMA ring and
+# d = 64, w <= 32 (tc_narrow.cu, tc_narrow_bwd.cu): enough tiles per CTA that the 3-stage TMA ring and
 # both ping-pong softmax groups wrap their barrier phases several times; with dilation,
 # ragged residues and a tile count that does not divide the grid.
 @pytest.mark.parametrize("shape", [(1, 16, 8192, 64, 32, 1), (1, 6, 5000, 64, 7, 3),
                                    (2, 5, 2001, 64, 32, 2), (1, 3, 129, 64, 31, 1)],
                          ids=lambda s: "x".join(map(str, s)))
-def test_narrow_fwd_many_tiles(ft, shape):
+def test_narrow_many_tiles(ft, shape):
     sh = WinAttnShape(*shape)
-    p, _ = ft.plan(False, sh.batch, sh.heads, sh.seq_len, sh.d, sh.w, sh.dilation, 1)
-    assert p == ft.PATH_TC
-    run_case(ft, sh, "bf16", None, seed=5, check_bwd=False)
+    for bwd in (False, True):
+        p, _ = ft.plan(bwd, sh.batch, sh.heads, sh.seq_len, sh.d, sh.w, sh.dilation, 1)
+        assert p == ft.PATH_TC
+    run_case(ft, sh, "bf16", None, seed=5)
 
 
 def test_overflow_probe(ft):
