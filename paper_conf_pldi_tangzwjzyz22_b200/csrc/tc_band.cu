@@ -43,6 +43,7 @@
 
 #include "internal.h"
 #include "tc_common.cuh"
+#include "tile_sched.cuh"
 #include "tmap.h"
 
 namespace ftw {
@@ -81,21 +82,20 @@ struct Params {
     float* lse;   // FWD: written; BWD: read
     float* D;     // BWDQ: written; BWDKV: read
     int64_t L;
-    int d, w, dil, r0, nr, NK, nsl, nst, units, tiles;
+    int d, w, dil, NK, nsl, nst;
+    SchedParams sc;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace)
     int two;                     // 1: two MMA issuers (warps 9, 10); 0: warp 9 issues all
 };
 
-// Phase trace: per CTA and local tile j < TRACE_TILES, globaltimer stamps of
+// Phase trace: per CTA and local tile j < TRACE_TILES, clock64 stamps (SM cycles) of
 // 0 producer first score-GEMM load, 1 producer last output load, 2 MMA score GEMM first
 // stage ready, 3 MMA s_full commit, 4 MMA p_full seen, 5 MMA last output MMA issued,
 // 6 softmax s_full seen, 7 softmax p_full arrive, 8 epilogue first o_full, 9 epilogue done.
 constexpr int TRACE_TILES = 8, TRACE_EV = 48;
 __device__ __forceinline__ void trace_ev(const Params& p, int j, int ev) {
     if (p.trace && j < TRACE_TILES) {
-        unsigned long long t;
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-        p.trace[((size_t)blockIdx.x * TRACE_TILES + j) * TRACE_EV + ev] = t;
+        p.trace[((size_t)blockIdx.x * TRACE_TILES + j) * TRACE_EV + ev] = clock64();   // SM cycles
     }
 }
 
@@ -142,30 +142,8 @@ inline int pick_nst(int NK) {
     return n < MAX_NST ? n : MAX_NST;
 }
 
-struct Tile {
-    int u, rl, r, Lr, m0;
-};
-// Tile tau -> (unit, residue, row block); row block fastest so concurrently running CTAs
-// work on neighbouring row blocks and share their halos through L2.
-__device__ __forceinline__ bool decode_tile(const Params& p, int tau, Tile& T) {
-    const int t = tau % p.tiles;
-    const int rest = tau / p.tiles;
-    T.rl = rest % p.nr;
-    T.u = rest / p.nr;
-    T.r = p.r0 + T.rl;
-    T.Lr = (int)((p.L - T.r + p.dil - 1) / p.dil);
-    T.m0 = t * BM;
-    return T.m0 < T.Lr;
-}
-struct TileCursor {   // this CTA's valid tiles, static round robin over the grid
-    int tau;
-    __device__ explicit TileCursor(int start) : tau(start - (int)gridDim.x) {}
-    __device__ bool next(const Params& p, int total, Tile& T) {
-        for (tau += gridDim.x; tau < total; tau += gridDim.x)
-            if (decode_tile(p, tau, T)) return true;
-        return false;
-    }
-};
+using Tile = SchedTile;
+using TileCursor = SchedCursor<BM>;
 
 // P / P^T in smem as the K-major SWIZZLE_128B A operand: 64-column atoms of 16 KB, row t at
 // t*128, 16-byte granule g at ((g ^ (t & 7)) * 16).  Thread t writes its row's 32-column
@@ -231,7 +209,6 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     const bool early = MODE == BWDQ && NK + d <= 256;
     const uint32_t acc0 = early ? 256u + (uint32_t)NK : 256u;   // accumulator base column
     const int nacc = dual ? ncw : ncw * C::NOUT;   // accumulations per tile
-    const int total = p.units * p.nr * p.tiles;
     const uint32_t SLOT = slot_bytes(NK);
     const uint32_t HB = (uint32_t)NK * 128u;
 
@@ -266,7 +243,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             mbar_init(p_free, 1);
             for (int i = 0; i < 4; ++i) mbar_init(&p_blk[i], 128);
             fence_barrier_init();
-            for (int i = 0; i < p.nr; ++i) {
+            for (int i = 0; i < p.sc.nr; ++i) {
                 const Maps& mp = p.maps[i];
                 tma_prefetch(&mp.a1); tma_prefetch(&mp.b1); tma_prefetch(&mp.ob1); tma_prefetch(&mp.o1);
                 if (C::NA == 2) { tma_prefetch(&mp.a2); tma_prefetch(&mp.b2); }
@@ -324,16 +301,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 }
                 adv();
             };
-            TileCursor cg(blockIdx.x), co(blockIdx.x);
+            TileCursor cg(p.sc), co(p.sc);
             Tile Tg, To;
-            bool hg = cg.next(p, total, Tg);
+            bool hg = cg.next(p.sc, Tg);
             int jg = 0, jo = 0;
             if (MODE == FWD && hg) {
                 for (int s = 0; s < nsl; ++s) load_g_slice(Tg, jg, s);
                 ++jg;
-                hg = cg.next(p, total, Tg);
+                hg = cg.next(p.sc, Tg);
             }
-            while (co.next(p, total, To)) {
+            while (co.next(p.sc, To)) {
                 if (MODE == FWD) {
                     // G(j+1) slices and O(j) key blocks alternate, the order in which the
                     // two issuers consume them concurrently (one issuer: G(j+1) first).
@@ -342,7 +319,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         if (gi < nG) load_g_slice(Tg, jg, gi++);
                         if (oi < nO && (p.two || gi == nG)) { load_o_block(To, oi / nkb, oi % nkb); ++oi; }
                     }
-                    if (hg) { ++jg; hg = cg.next(p, total, Tg); }
+                    if (hg) { ++jg; hg = cg.next(p.sc, Tg); }
                 } else {   // BWD: G(j) then O(j) (dS lives in the S columns)
                     for (int s = 0; s < nsl; ++s) load_g_slice(To, jo, s);
                     for (int a = 0; a < nacc; ++a)
@@ -456,16 +433,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     ++ga;
                 }
             };
-            TileCursor cg(blockIdx.x), co(blockIdx.x);
+            TileCursor cg(p.sc), co(p.sc);
             Tile Tg, To;
-            bool hg = cg.next(p, total, Tg);
+            bool hg = cg.next(p.sc, Tg);
             int jg = 0, jo = 0;
             if (MODE == FWD && hg) {   // G(0)
                 for (int s = 0; s < nsl; ++s) g_slice(jg, s);
                 ++jg;
-                hg = cg.next(p, total, Tg);
+                hg = cg.next(p.sc, Tg);
             }
-            while (co.next(p, total, To)) {
+            while (co.next(p.sc, To)) {
                 jo_cur = jo;
                 if (MODE != FWD) {
                     // the score GEMMs write dP into the accumulator columns (unless early):
@@ -490,7 +467,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         if (gi < nG) g_slice(jg, gi++);
                         if (oi < nO && (p.two || gi == nG)) { o_block(oi / nkb, oi % nkb); ++oi; }
                     }
-                    if (hg) { ++jg; hg = cg.next(p, total, Tg); }
+                    if (hg) { ++jg; hg = cg.next(p.sc, Tg); }
                 } else {
                     for (int a = 0; a < nacc; ++a)
                         for (int kb = 0; kb < nkb; ++kb) o_block(a, kb);
@@ -507,13 +484,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
         // chunks holding any band column of this warp's rows (warp-uniform):
         // rows 32*warp .. 32*warp+31 need columns [32*warp, 32*warp + 31 + 2w]
         const int c_lo = warp, c_hi = min(nch - 1, (32 * warp + 31 + 2 * w) / 32);
-        TileCursor cur(blockIdx.x);
+        TileCursor cur(p.sc);
         Tile T;
         int j = 0;
         uint32_t zero16[16];
 #pragma unroll
         for (int e = 0; e < 16; ++e) zero16[e] = 0u;
-        while (cur.next(p, total, T)) {
+        while (cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0;
             const int mrow = m0 + t;
             const int kb = m0 - w;   // residue index of halo column 0
@@ -661,10 +638,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
         const int ew = warp - 4;   // TMEM lanes 32*ew .. 32*ew+31  (warp % 4 == ew)
         const uint32_t trow = tbase + ((uint32_t)(ew * 32) << 16);
         uint8_t* mystg = ostg + ew * NSTG * STG;
-        TileCursor cur(blockIdx.x);
+        TileCursor cur(p.sc);
         Tile T;
         int j = 0, ga = 0, sidx = 0;
-        while (cur.next(p, total, T)) {
+        while (cur.next(p.sc, T)) {
             const Maps& mp = p.maps[T.rl];
             float scale = 1.f;
             if (MODE == FWD) {   // 1/l of this row, published before p_full
@@ -803,12 +780,10 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         p.d = (int)d;
         p.w = (int)wc;
         p.dil = (int)dil;
-        p.r0 = (int)r0;
         p.NK = NK;
         p.nsl = (int)(d / 64);
         p.nst = nst;
         const int64_t Lr0 = ceil_div(L - r0, dil);   // longest residue of this group
-        p.nr = nr;
         p.trace = (unsigned long long*)trace_buffer(MODE);
         {
             // Two issuers (measured faster for every mode and d, profiles/README.md);
@@ -816,10 +791,10 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
             const char* e = getenv("FT_WINATTN_ISSUERS");
             p.two = !(e && atoi(e) == 1);
         }
-        p.units = (int)units;
-        p.tiles = (int)ceil_div(Lr0, BM);
-        const int64_t total = (int64_t)p.units * p.nr * p.tiles;
+        const int tiles = (int)ceil_div(Lr0, BM);
+        const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms() ? total : num_sms()));
+        sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_smem_bytes<MODE>(NK) + (size_t)nst * slot_bytes(NK);
         tc_band_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
         prof_mark(st);

@@ -30,7 +30,11 @@
 #include <mutex>
 
 #include "internal.h"
+#ifndef FT_MBAR_SUSPEND_NS
+#define FT_MBAR_SUSPEND_NS 0   // latency-critical handoffs: no suspend-time hint
+#endif
 #include "tc_common.cuh"
+#include "tile_sched.cuh"
 #include "tmap.h"
 
 namespace ftw {
@@ -60,31 +64,12 @@ struct NParams {
     NMaps maps[RES_PER_LAUNCH];
     float* lse;
     int64_t L;
-    int w, dil, r0, nr, units, tiles;
+    int w, dil;
+    SchedParams sc;
 };
 
-struct Tile {
-    int u, rl, r, Lr, m0;
-};
-__device__ __forceinline__ bool decode_tile(const NParams& p, int tau, Tile& T) {
-    const int t = tau % p.tiles;
-    const int rest = tau / p.tiles;
-    T.rl = rest % p.nr;
-    T.u = rest / p.nr;
-    T.r = p.r0 + T.rl;
-    T.Lr = (int)((p.L - T.r + p.dil - 1) / p.dil);
-    T.m0 = t * BM;
-    return T.m0 < T.Lr;
-}
-struct TileCursor {   // this CTA's valid tiles, static round robin over the grid
-    int tau;
-    __device__ explicit TileCursor(int start) : tau(start - (int)gridDim.x) {}
-    __device__ bool next(const NParams& p, int total, Tile& T) {
-        for (tau += gridDim.x; tau < total; tau += gridDim.x)
-            if (decode_tile(p, tau, T)) return true;
-        return false;
-    }
-};
+using Tile = SchedTile;
+using TileCursor = SchedCursor<BM>;
 
 __device__ __forceinline__ float fast_exp2(float x) {
     float y;
@@ -110,7 +95,6 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int w = p.w;
-    const int total = p.units * p.nr * p.tiles;
 
     if (warp == 8) {
         if (lane == 0) {
@@ -126,7 +110,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
                 mbar_init(&o_free[b], 128);
             }
             fence_barrier_init();
-            for (int i = 0; i < p.nr; ++i) {
+            for (int i = 0; i < p.sc.nr; ++i) {
                 tma_prefetch(&p.maps[i].q); tma_prefetch(&p.maps[i].k);
                 tma_prefetch(&p.maps[i].v); tma_prefetch(&p.maps[i].o);
             }
@@ -142,9 +126,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
 
     if (warp == 8) {
         if (lane == 0) {   // ---------------------------------------------------- TMA producer
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
-            for (int j = 0; cur.next(p, total, T); ++j) {
+            for (int j = 0; cur.next(p.sc, T); ++j) {
                 const int s = j % NSTAGE;
                 if (j >= NSTAGE) mbar_wait(&empty[s], ((j / NSTAGE) - 1) & 1);
                 uint8_t* st = stages + (size_t)s * STAGE;
@@ -176,10 +160,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
                 mma_commit(&o_full[b]);
                 mma_commit(&empty[s]);
             };
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
             int j = 0;
-            for (; cur.next(p, total, T); ++j) {
+            for (; cur.next(p.sc, T); ++j) {
                 const int b = j & 1, s = j % NSTAGE;
                 mbar_wait(&qk_full[s], (j / NSTAGE) & 1);
                 // S[b] held P(j-2), read by O(j-2): wait for it to complete
@@ -203,11 +187,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
         uint32_t zero16[16];
 #pragma unroll
         for (int e = 0; e < 16; ++e) zero16[e] = 0u;
-        TileCursor cur(blockIdx.x);
+        TileCursor cur(p.sc);
         Tile T;
         int jl = 0;   // local tile index
         int k = 0;    // this group's tile count
-        for (; cur.next(p, total, T); ++jl) {
+        for (; cur.next(p.sc, T); ++jl) {
             if ((jl & 1) != g) continue;
             const int ph = k & 1;
             ++k;
@@ -362,13 +346,12 @@ cudaError_t tc_narrow_fwd(const void* q, const void* k, const void* v, void* out
         p.L = L;
         p.w = (int)wc;
         p.dil = (int)dil;
-        p.r0 = (int)r0;
-        p.nr = nr;
-        p.units = (int)units;
+
         const int64_t Lr0 = ceil_div(L - r0, dil);
-        p.tiles = (int)ceil_div(Lr0, BM);
-        const int64_t total = (int64_t)p.units * p.nr * p.tiles;
+        const int tiles = (int)ceil_div(Lr0, BM);
+        const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms_n() ? total : num_sms_n()));
+        sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         tc_narrow_fwd_kernel<<<grid, NTHREADS, SMEM_BYTES, st>>>(p);
         prof_mark(st);
         cudaError_t e = cudaGetLastError();

@@ -20,10 +20,13 @@
 // (tcgen05.mma executes in issue order).  Per tile the tensor pipe runs S(j+1), out(j),
 // dP(j+1) while the softmax warps drain tile j's accumulator.
 //
-// dS enters the output MMAs as a bf16 hi + lo pair (reading A10): a single bf16 dS put dq
-// 1.1e-2 off at one element of 8.4M in the 16 x 8192 parity case.  TMEM: NQ writes dS_hi |
-// dS_lo over S; NKV writes P^T | dS^T_hi over S^T and dS^T_lo over the first 96 columns of
-// dP^T, so its output MMAs are issued before the next tile's S^T (which reuses that region).
+// dS enters its output MMA as fp16, with the bf16 halo it multiplies (K_h for dQ, Q_h for
+// dK) converted to fp16 in shared memory once the score GEMM has read it (exact for bf16
+// values of magnitude 6.1e-5 .. 65504).  A single bf16 dS put dq 1.1e-2 off at one element of
+// 8.4M in the 16 x 8192 parity case; fp16's 11-bit significand is 8x finer, and unlike a bf16
+// hi + lo pair it costs one operand: NQ writes dS over S, NKV writes P^T (bf16) | dS^T (fp16)
+// over S^T, and the dP region is free as soon as the softmax holds dP in registers
+// (reading A10).
 //
 // Roles (320 threads): warps 0-7 softmax -- warp w reads TMEM lanes 32*(w%4).. (thread <->
 // row) and column half h = w/4 of the row's 96-column band range; warp 8 TMA producer +
@@ -39,7 +42,11 @@
 #include <mutex>
 
 #include "internal.h"
+#ifndef FT_MBAR_SUSPEND_NS
+#define FT_MBAR_SUSPEND_NS 0   // latency-critical handoffs: no suspend-time hint
+#endif
 #include "tc_common.cuh"
+#include "tile_sched.cuh"
 #include "tmap.h"
 
 namespace ftw {
@@ -53,13 +60,16 @@ constexpr int BM = 128;
 constexpr int D = 64;
 constexpr int NK = 192;
 constexpr int NSTAGE = 2;
-constexpr int NTHREADS = 320;
+constexpr int NTHREADS = 352;
 constexpr int RES_PER_LAUNCH = 3;
 constexpr uint32_t ABYTES = BM * D * 2;      // 16 KB: a 128-row tile
 constexpr uint32_t HBYTES = NK * D * 2;      // 24 KB: a 192-row halo
 constexpr uint32_t STAGE = 2 * ABYTES + 2 * HBYTES;   // {A1, A2, B1, B2}
 constexpr uint32_t STG = 32 * 128;
-constexpr size_t SMEM_BYTES = 1024 + (size_t)NSTAGE * STAGE + 8 * STG + 2 * 2 * NK * 4 + 2 * 2 * BM * 4 + 256;
+constexpr uint32_t XBYTES = 3 * 16384;      // NQ: dS operand (fp16, 128 x 192); NKV: 8 x STG staging
+// per-tile scratch: NKV [2][2][NK] column lse / D; NQ [2][2][BM] D halves + [2][256] row lse
+constexpr int SCRATCH_FLOATS = 2 * 2 * BM + 2 * 256 > 2 * 2 * NK ? 2 * 2 * BM + 2 * 256 : 2 * 2 * NK;
+constexpr size_t SMEM_BYTES = 1024 + (size_t)NSTAGE * STAGE + XBYTES + SCRATCH_FLOATS * 4 + 256;
 constexpr float LOG2E = 1.4426950408889634f;
 constexpr uint32_t TACC = 384;
 
@@ -70,44 +80,30 @@ struct BMaps {
 struct BParams {
     BMaps maps[RES_PER_LAUNCH];
     const float* lse;
-    float* D;   // NQ: written; NKV: read
+    float* D;      // NQ: written; NKV: read
+    uint16_t* o1;  // NQ: dq (written with direct 16-byte stores)
     int64_t L;
-    int w, dil, r0, nr, units, tiles;
+    int w, dil;
+    SchedParams sc;
+    unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, modes 1 / 2)
 };
 
-struct Tile {
-    int u, rl, r, Lr, m0;
-};
-__device__ __forceinline__ bool decode_tile(const BParams& p, int tau, Tile& T) {
-    const int t = tau % p.tiles;
-    const int rest = tau / p.tiles;
-    T.rl = rest % p.nr;
-    T.u = rest / p.nr;
-    T.r = p.r0 + T.rl;
-    T.Lr = (int)((p.L - T.r + p.dil - 1) / p.dil);
-    T.m0 = t * BM;
-    return T.m0 < T.Lr;
+// Phase trace: per CTA and local tile j < 8, clock64 stamps (tools/trace_narrow.py).
+// MMA: 0 iteration start, 1 S(j) issued, 2 out(j-1) issued, 3 dP(j) issued.  Softmax warp 0:
+// 4 s_full seen, 5 S/dP loaded, 6 operand buffer free, 7 pair barrier passed, 8 p_done
+// arrived, 9 accumulator seen, 10 drained.  Producer: 11 loads of tile j issued.
+// Converter: 12 halo converted.
+__device__ __forceinline__ void trace_ev(const BParams& p, int j, int ev) {
+    if (p.trace && j >= 0 && j < 8) p.trace[((size_t)blockIdx.x * 8 + j) * 48 + ev] = clock64();
 }
-struct TileCursor {
-    int tau;
-    __device__ explicit TileCursor(int start) : tau(start - (int)gridDim.x) {}
-    __device__ bool next(const BParams& p, int total, Tile& T) {
-        for (tau += gridDim.x; tau < total; tau += gridDim.x)
-            if (decode_tile(p, tau, T)) return true;
-        return false;
-    }
-};
+
+using Tile = SchedTile;
+using TileCursor = SchedCursor<BM>;
 
 __device__ __forceinline__ float fast_exp2(float x) {
     float y;
     asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
-}
-__device__ __forceinline__ void split_bf16x2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
-    __nv_bfloat162 hb = __floats2bfloat162_rn(x0, x1);
-    const float2 hf = __bfloat1622float2(hb);
-    hi = *reinterpret_cast<uint32_t*>(&hb);
-    lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
 }
 
 // rows 32*wq .. +31 of a 64-column accumulator -> bf16 -> this warp's staging -> TMA store
@@ -146,23 +142,22 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
     const uint32_t raw_u32 = smem_u32(smem_raw);
     uint8_t* smem = smem_raw + (((raw_u32 + 1023u) & ~1023u) - raw_u32);
     uint8_t* stages = smem;                                        // [NSTAGE] {A1, A2, B1, B2}
-    uint8_t* ostg = smem + (size_t)NSTAGE * STAGE;                 // [8 warps] 4 KB
-    float* colv = reinterpret_cast<float*>(ostg + 8 * STG);        // NKV [2][2][NK]: lse*log2e, D
-    float* dx = colv + 2 * 2 * NK;                                 // NQ [2][2][BM]: D halves
-    uint64_t* bars = reinterpret_cast<uint64_t*>(dx + 2 * 2 * BM);
+    uint8_t* xbuf = smem + (size_t)NSTAGE * STAGE;                 // NQ: dS operand; NKV: staging
+    float* colv = reinterpret_cast<float*>(xbuf + XBYTES);         // NKV [2][2][NK]: lse, D of columns
+    float* dx = colv;                                              // NQ [2][2][BM]: D halves, then [2][256] lse
+    uint64_t* bars = reinterpret_cast<uint64_t*>(colv + SCRATCH_FLOATS);
     uint64_t* full1 = bars;                 // [NSTAGE] A1 + B1
     uint64_t* full2 = bars + NSTAGE;        // [NSTAGE] A2 + B2
     uint64_t* empty = bars + 2 * NSTAGE;    // [NSTAGE]
     uint64_t* s_full = bars + 3 * NSTAGE;   // S and dP of the tile done
-    uint64_t* p_done = s_full + 1;          // softmax read dP and wrote the operand
-    uint64_t* acc_full = s_full + 2;
-    uint64_t* acc_free = s_full + 3;
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 4);
+    uint64_t* dp_free = s_full + 1;         // softmax holds S and dP in registers
+    uint64_t* p_done = s_full + 2;          // operands written and the dS halo converted
+    uint64_t* acc_full = s_full + 3;        // [2]
+    uint64_t* acc_free = s_full + 5;        // [2]
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 7);
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int w = p.w;
-    const int total = p.units * p.nr * p.tiles;
-    constexpr int NDRAIN = MODE == NQ ? 128 : 256;
 
     if (warp == 8) {
         if (lane == 0) {
@@ -172,15 +167,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 mbar_init(&empty[i], 1);
             }
             mbar_init(s_full, 1);
-            mbar_init(p_done, 256);
-            mbar_init(acc_full, 1);
-            mbar_init(acc_free, NDRAIN);
+            mbar_init(dp_free, 256);
+            mbar_init(p_done, 256 + 32);
+            for (int b = 0; b < 2; ++b) {
+                mbar_init(&acc_full[b], 1);
+                mbar_init(&acc_free[b], 256);
+            }
             fence_barrier_init();
-            for (int i = 0; i < p.nr; ++i) {
+            for (int i = 0; i < p.sc.nr; ++i) {
                 const BMaps& m = p.maps[i];
                 tma_prefetch(&m.a1); tma_prefetch(&m.a2); tma_prefetch(&m.b1); tma_prefetch(&m.b2);
-                tma_prefetch(&m.o1);
-                if (MODE == NKV) tma_prefetch(&m.o2);
+                if (MODE == NKV) { tma_prefetch(&m.o1); tma_prefetch(&m.o2); }
             }
         }
         __syncwarp();
@@ -194,13 +191,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
 
     if (warp == 8) {
         if (lane == 0) {   // ---------------------------------------------------- TMA producer
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
-            for (int j = 0; cur.next(p, total, T); ++j) {
+            for (int j = 0; cur.next(p.sc, T); ++j) {
                 const int s = j % NSTAGE;
                 if (j >= NSTAGE) mbar_wait(&empty[s], ((j / NSTAGE) - 1) & 1);
                 uint8_t* st = stages + (size_t)s * STAGE;
                 const BMaps& mp = p.maps[T.rl];
+                trace_ev(p, j, 11);
                 mbar_arrive_expect_tx(&full1[s], ABYTES + HBYTES);
                 tma_load_3d(st, &mp.a1, &full1[s], 0, T.m0, T.u);
                 tma_load_3d(st + 2 * ABYTES, &mp.b1, &full1[s], 0, T.m0 - w, T.u);
@@ -209,78 +207,109 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 tma_load_3d(st + 2 * ABYTES + HBYTES, &mp.b2, &full2[s], 0, T.m0 - w, T.u);
             }
         }
+    } else if (warp == 10) {   // ------------------------------------------ halo converter
+        // the halo of the dS GEMM (NQ: K_h, NKV: Q_h) to fp16 in place, once the score GEMM
+        // has read it as bf16 (s_full); the output MMAs read it after p_done
+        TileCursor cur(p.sc);
+        Tile T;
+        for (int j = 0; cur.next(p.sc, T); ++j) {
+            mbar_wait(s_full, j & 1);
+            if (lane == 0) trace_ev(p, j, 14);
+            uint4* hb = reinterpret_cast<uint4*>(stages + (size_t)(j % NSTAGE) * STAGE + 2 * ABYTES);
+#pragma unroll 4
+            for (int i = lane; i < (int)(HBYTES / 16); i += 32) {
+                uint4 v4 = hb[i];
+                uint32_t* wv = reinterpret_cast<uint32_t*>(&v4);
+#pragma unroll
+                for (int x = 0; x < 4; ++x) {
+                    const float2 f = __bfloat1622float2(*reinterpret_cast<__nv_bfloat162*>(&wv[x]));
+                    wv[x] = pack_f16x2(f.x, f.y);
+                }
+                hb[i] = v4;
+            }
+            fence_proxy_async_smem();
+            mbar_arrive(p_done);
+            if (lane == 0) trace_ev(p, j, 12);
+        }
     } else if (warp == 9) {
         if (lane == 0) {   // ------------------------------------------------------ MMA issuer
             constexpr uint32_t idS = idesc_bf16(BM, NK, false, false);
             constexpr uint32_t idO = idesc_bf16(BM, D, false, true);
-            // output MMAs of tile i: A = bf16 operand packed in region i&1 (8 columns per
-            // 16-key step), B = a halo as MN-major SW128 (2048 B per step)
+            constexpr uint32_t idH = idesc_f16(BM, D, false, true);
+            // output MMAs of tile i (B = a halo as MN-major SW128, 2048 B per 16-key step):
+            //   NQ:  dQ = dS K_h, A = dS in smem (K-major SW128: 64-key atoms of 16 KB), -> acc[i&1]
+            //   NKV: dV = P^T dO_h, dK = dS^T Q_h, A = packed operands over S^T in TMEM region
+            //        i&1 (8 columns per step) -> acc (dV at 384, dK at 448)
             auto out = [&](int i) {
-                const int s = i % NSTAGE;
+                const int s = i % NSTAGE, b = MODE == NQ ? (i & 1) : 0;
                 const uint32_t st = smem_u32(stages + (size_t)s * STAGE);
-                const uint32_t tR = tbase + 192u * (i & 1), tR2 = tbase + 192u * ((i + 1) & 1);
-                if (i >= 1) mbar_wait(acc_free, (i - 1) & 1);
+                mbar_wait(p_done, i & 1);
+                if (MODE == NQ ? i >= 2 : i >= 1)
+                    mbar_wait(&acc_free[b], (MODE == NQ ? (i - 2) >> 1 : i - 1) & 1);
                 tc_fence_after();
-                if (MODE == NQ) {   // dQ = (dS_hi + dS_lo) K_h
-                    const uint32_t sb = st + 2 * ABYTES;
+                if (MODE == NQ) {
+                    const uint32_t sb = st + 2 * ABYTES, sa = smem_u32(xbuf);
 #pragma unroll
-                    for (int g = 0; g < 3; ++g) {
-                        const uint64_t bd = sdesc_sw128(sb + 8192u * g, 8192, 1024);
-                        mma_ts_x4<8, 128>(tbase + TACC, tR + 32u * g, bd, idO, g);
-                        mma_ts_x4<8, 128>(tbase + TACC, tR + 96u + 32u * g, bd, idO, 1);
-                    }
-                } else {            // dV = P^T dO_h, dK = (dS^T_hi + dS^T_lo) Q_h
+                    for (int g = 0; g < 3; ++g)
+                        mma_ss_x4<2, 128>(tbase + TACC + 64u * b, sdesc_sw128(sa + 16384u * g, 16, 1024),
+                                          sdesc_sw128(sb + 8192u * g, 8192, 1024), idH, g);
+                } else {
+                    const uint32_t tR = tbase + 192u * (i & 1);
                     const uint32_t sq = st + 2 * ABYTES, sdo = sq + HBYTES;
 #pragma unroll
                     for (int g = 0; g < 3; ++g) {
-                        const uint64_t bq = sdesc_sw128(sq + 8192u * g, 8192, 1024);
                         mma_ts_x4<8, 128>(tbase + TACC, tR + 32u * g, sdesc_sw128(sdo + 8192u * g, 8192, 1024), idO, g);
-                        mma_ts_x4<8, 128>(tbase + TACC + 64, tR + 96u + 32u * g, bq, idO, g);
-                        mma_ts_x4<8, 128>(tbase + TACC + 64, tR2 + 32u * g, bq, idO, 1);
+                        mma_ts_x4<8, 128>(tbase + TACC + 64, tR + 96u + 32u * g, sdesc_sw128(sq + 8192u * g, 8192, 1024), idH, g);
                     }
                 }
-                mma_commit(acc_full);
+                mma_commit(&acc_full[b]);
                 mma_commit(&empty[s]);
             };
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
             int j = 0;
-            for (; cur.next(p, total, T); ++j) {
+            for (; cur.next(p.sc, T); ++j) {
                 const int s = j % NSTAGE, ph = (j / NSTAGE) & 1;
                 const uint32_t st = smem_u32(stages + (size_t)s * STAGE);
-                const uint32_t rS = tbase + 192u * (j & 1), rP = tbase + 192u * ((j + 1) & 1);
-                // region j&1 held dP(j-1) (NKV: and dS^T_lo(j-1)); region (j+1)&1 the operands
-                // of j-1.  out(j-1) is issued first; the MMAs below run after it in issue order.
-                if (j >= 1) {
-                    mbar_wait(p_done, (j - 1) & 1);
-                    out(j - 1);
-                }
+                // NQ: S in [0,192), dP in [192,384) every tile (the dS operand is in smem), so
+                // both score GEMMs of j run while the softmax of j-1 computes.
+                // NKV: S(j) in region j&1 (which held dP(j-1)), dP(j) in region (j+1)&1 (the
+                // operands of j-1, read by out(j-1) first: tcgen05.mma executes in issue order)
+                const uint32_t rS = MODE == NQ ? tbase : tbase + 192u * (j & 1);
+                const uint32_t rP = MODE == NQ ? tbase + 192u : tbase + 192u * ((j + 1) & 1);
+                trace_ev(p, j, 0);
+                if (j >= 1) mbar_wait(dp_free, (j - 1) & 1);
                 mbar_wait(&full1[s], ph);
                 tc_fence_after();
                 mma_ss_x4<2, 2>(rS, sdesc_sw128(st, 16, 1024), sdesc_sw128(st + 2 * ABYTES, 16, 1024), idS, 0);
+                trace_ev(p, j, 1);
+                if (MODE == NKV && j >= 1) out(j - 1);
                 mbar_wait(&full2[s], ph);
                 tc_fence_after();
                 mma_ss_x4<2, 2>(rP, sdesc_sw128(st + ABYTES, 16, 1024),
                                 sdesc_sw128(st + 2 * ABYTES + HBYTES, 16, 1024), idS, 0);
                 mma_commit(s_full);
+                trace_ev(p, j, 3);
+                if (p.trace && j < 8) {   // debug only: when did the score GEMMs complete?
+                    mbar_wait(s_full, j & 1);
+                    trace_ev(p, j, 13);
+                }
+                if (MODE == NQ && j >= 1) out(j - 1);
+                trace_ev(p, j, 2);
             }
-            if (j >= 1) {
-                mbar_wait(p_done, (j - 1) & 1);
-                out(j - 1);
-            }
+            if (j >= 1) out(j - 1);
         }
-    } else {   // ------------------------------------------------------------ softmax warps
+    } else if (warp < 8) {   // ------------------------------------------------- softmax warps
         const int wq = warp & 3, h = warp >> 2;
         const int t = wq * 32 + lane;
         const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
         const int c0 = 32 * wq + 48 * h;         // first of this warp's 48 score columns
-        const uint32_t pc = 16u * wq + 24u * h;  // its packed bf16 operand columns
-        uint8_t* mystg = ostg + warp * STG;
+        const uint32_t pc = 16u * wq + 24u * h;  // NKV: its packed operand columns
         uint32_t zero16[16];
 #pragma unroll
         for (int e = 0; e < 16; ++e) zero16[e] = 0u;
-        // 48 packed columns of an operand at base (+ zeros on the columns outside every band
-        // column of this row: h = 0 writes the ones before, h = 1 the ones after)
+        // NKV: 48 packed columns of an operand at TMEM base (+ zeros on the columns outside
+        // every band column of this row: h = 0 writes the ones before, h = 1 the ones after)
         auto st_operand = [&](uint32_t base, const uint32_t (&pk)[24]) {
             tmem_st16(base + pc, *reinterpret_cast<const uint32_t(*)[16]>(&pk[0]));
             tmem_st8(base + pc + 16, &pk[16]);
@@ -290,50 +319,112 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 for (int c = wq + 3; c < NK / 32; ++c) tmem_st16(base + 16u * c, zero16);
             }
         };
-        // per-tile values from HBM are loaded one tile ahead (NQ: this row's lse; NKV: lse and
-        // D of halo column threadIdx.x), so their latency hides behind the previous tile
-        TileCursor cur(blockIdx.x), nxt(blockIdx.x);
+        // NQ: dS row t in smem (K-major SW128, 64-key atoms of 128 rows x 128 B): keys
+        // c .. c+7 are 16-byte granule ((c % 64) / 8) ^ (t % 8) of row t in atom c / 64
+        auto ds_granule = [&](int c) -> uint4* {
+            return reinterpret_cast<uint4*>(xbuf + (c >> 6) * 16384 + t * 128 + ((((c & 63) >> 3) ^ (t & 7)) << 4));
+        };
+        if (MODE == NQ) {   // keys outside every band column of this row stay zero
+            const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+            if (h == 0) for (int c = 0; c < 32 * wq; c += 8) *ds_granule(c) = z;
+            else for (int c = 32 * wq + 96; c < NK; c += 8) *ds_granule(c) = z;
+        }
+        // per-tile values from HBM are copied one tile ahead into shared memory with cp.async
+        // (NQ: this row's lse -> lpre[b][threadIdx.x]; NKV: lse and D of halo column
+        // threadIdx.x -> colv[b]), so their latency hides behind the previous tile
+        float* lpre = colv + (MODE == NQ ? 2 * 2 * BM : 0);   // NQ [2][256]
+        TileCursor cur(p.sc), nxt(p.sc);
         Tile T, Tn;
-        bool hn = nxt.next(p, total, Tn);
-        float pre_l = 0.f, pre_d = 0.f;
-        auto prefetch = [&](const Tile& X) {
+        bool hn = nxt.next(p.sc, Tn);
+        auto prefetch = [&](const Tile& X, int jx) {
             const int64_t rb = (int64_t)X.u * p.L + X.r;
             if (MODE == NKV) {
-                const int mc = X.m0 - w + (int)threadIdx.x;
-                const bool ok = threadIdx.x < NK && mc >= 0 && mc < X.Lr;
-                pre_l = ok ? p.lse[rb + (int64_t)mc * p.dil] : 0.f;
-                pre_d = ok ? p.D[rb + (int64_t)mc * p.dil] : 0.f;
-            } else {
-                const int mrow = X.m0 + t;
-                pre_l = mrow < X.Lr ? p.lse[rb + (int64_t)mrow * p.dil] : 0.f;
-            }
-        };
-        if (hn) prefetch(Tn);
-        for (int j = 0; cur.next(p, total, T); ++j) {
-            const int Lr = T.Lr, m0 = T.m0, kb = m0 - w;
-            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
-            const uint32_t tS = tbase + lane_off + 192u * (j & 1);
-            const uint32_t tP = tbase + lane_off + 192u * ((j + 1) & 1);
-            float* cl = colv + (j & 1) * 2 * NK;   // NKV: this tile's column lse*log2e and D
-            float lse2 = 0.f;
-            if (MODE == NKV) {
                 if (threadIdx.x < NK) {
-                    cl[threadIdx.x] = pre_l * LOG2E;
-                    cl[NK + threadIdx.x] = pre_d;
+                    const int mc = X.m0 - w + (int)threadIdx.x;
+                    const bool ok = mc >= 0 && mc < X.Lr;
+                    const int64_t off = ok ? rb + (int64_t)mc * p.dil : 0;
+                    float* cl = colv + (jx & 1) * 2 * NK;
+                    cp_async4(cl + threadIdx.x, p.lse + off, ok ? 4u : 0u);
+                    cp_async4(cl + NK + threadIdx.x, p.D + off, ok ? 4u : 0u);
                 }
             } else {
-                lse2 = pre_l * LOG2E;
+                const int mrow = X.m0 + t;
+                const bool ok = mrow < X.Lr;
+                cp_async4(lpre + (jx & 1) * 256 + threadIdx.x, p.lse + (ok ? rb + (int64_t)mrow * p.dil : 0),
+                          ok ? 4u : 0u);
             }
-            hn = nxt.next(p, total, Tn);
-            if (hn) prefetch(Tn);
-            if (MODE == NKV) named_bar_sync(5, 256);
+            cp_async_commit();
+        };
+        if (hn) prefetch(Tn, 0);
+        // per-tile state, set up for tile j+1 as soon as tile j's operands are written
+        struct St {
+            int Lr, m0, kb, u, rl;
+            int64_t rowbase;
+            float lse2;
+            uint64_t bits;
+        };
+        auto setup = [&](const Tile& X, int jx) -> St {
+            St c;
+            c.Lr = X.Lr; c.m0 = X.m0; c.kb = X.m0 - w; c.u = X.u; c.rl = X.rl;
+            c.rowbase = (int64_t)X.u * p.L + X.r;
+            cp_async_wait_all();   // this tile's values (copied a tile ago)
+            c.lse2 = MODE == NQ ? lpre[(jx & 1) * 256 + threadIdx.x] * LOG2E : 0.f;
+            if (MODE == NKV) named_bar_sync(5, 256);   // every thread's columns landed
+            hn = nxt.next(p.sc, Tn);
+            if (hn) prefetch(Tn, jx + 1);
             // band columns of this row: n in [t, t+2w] within the sequence
-            const int lo = max(t, -kb) - c0, hi = min(t + 2 * w, Lr - 1 - kb) - c0;
+            const int lo = max(t, -c.kb) - c0, hi = min(t + 2 * w, c.Lr - 1 - c.kb) - c0;
             const int l0 = max(lo, 0), h0 = min(hi, 47);
-            const uint64_t bits = h0 < l0 ? 0ull : ((~0ull >> (63 - h0)) & (~0ull << l0));
-
+            c.bits = h0 < l0 ? 0ull : ((~0ull >> (63 - h0)) & (~0ull << l0));
+            return c;
+        };
+        // NQ: drain dQ of tile i (columns 32h .. 32h+31 of this row) with direct 16-byte
+        // stores; NKV: dV (h = 0) or dK (h = 1) of tile i through staging + TMA store
+        auto drain = [&](int i, const St& c) {
+            const int b = MODE == NQ ? (i & 1) : 0;
+            mbar_wait(&acc_full[b], MODE == NQ ? (i >> 1) & 1 : i & 1);
+            tc_fence_after();
+            if (threadIdx.x == 0) trace_ev(p, i, 9);
+            if (MODE == NQ) {
+                uint32_t ov[32];
+                tmem_ld32(tbase + lane_off + TACC + 64u * b + 32u * h, ov);
+                tmem_wait_ld();
+                if (threadIdx.x == 0) trace_ev(p, i, 16);
+                tc_fence_before();
+                mbar_arrive(&acc_free[b]);
+                const int mrow = c.m0 + t;
+                if (mrow < c.Lr) {
+                    uint4* dst = reinterpret_cast<uint4*>(p.o1 + (c.rowbase + (int64_t)mrow * p.dil) * D + 32 * h);
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        dst[q] = make_uint4(pack_bf16x2(__uint_as_float(ov[8 * q]), __uint_as_float(ov[8 * q + 1])),
+                                            pack_bf16x2(__uint_as_float(ov[8 * q + 2]), __uint_as_float(ov[8 * q + 3])),
+                                            pack_bf16x2(__uint_as_float(ov[8 * q + 4]), __uint_as_float(ov[8 * q + 5])),
+                                            pack_bf16x2(__uint_as_float(ov[8 * q + 6]), __uint_as_float(ov[8 * q + 7])));
+                }
+            } else {
+                const BMaps& mp = p.maps[c.rl];
+                drain_store(tbase + lane_off + TACC + 64u * h, xbuf + warp * STG, h == 0 ? &mp.o1 : &mp.o2,
+                            c.m0 + 32 * wq, c.u, lane, &acc_free[0]);
+            }
+            if (threadIdx.x == 0) trace_ev(p, i, 10);
+        };
+        bool have = cur.next(p.sc, T);
+        St cs = have ? setup(T, 0) : St{};
+        St prev = cs;
+        int j = 0;
+        for (; have; ++j) {
+            const int Lr = cs.Lr, m0 = cs.m0;
+            const int64_t rowbase = cs.rowbase;
+            const float lse2 = cs.lse2;
+            const uint64_t bits = cs.bits;
+            const uint32_t tS = MODE == NQ ? tbase + lane_off : tbase + lane_off + 192u * (j & 1);
+            const uint32_t tP = MODE == NQ ? tbase + lane_off + 192u : tbase + lane_off + 192u * ((j + 1) & 1);
+            const float* cl = colv + (j & 1) * 2 * NK;   // NKV: this tile's column lse*log2e and D
+            const bool tr = threadIdx.x == 0;
             mbar_wait(s_full, j & 1);
             tc_fence_after();
+            if (tr) trace_ev(p, j, 4);
             uint32_t rs[48], rd[48];
             tmem_ld16(tS + c0, *reinterpret_cast<uint32_t(*)[16]>(&rs[0]));
             tmem_ld16(tS + c0 + 16, *reinterpret_cast<uint32_t(*)[16]>(&rs[16]));
@@ -342,7 +433,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             tmem_ld16(tP + c0 + 16, *reinterpret_cast<uint32_t(*)[16]>(&rd[16]));
             tmem_ld16(tP + c0 + 32, *reinterpret_cast<uint32_t(*)[16]>(&rd[32]));
             tmem_wait_ld();
-            uint32_t pk[24], pk2[24], pk3[24];
+            tc_fence_before();
+            mbar_arrive(dp_free);
+            if (tr) trace_ev(p, j, 5);
+            uint32_t pk[24], pk2[24];
             if (MODE == NQ) {
                 float dpart[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
@@ -353,54 +447,69 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 }
                 float* dxb = dx + (j & 1) * 2 * BM;
                 dxb[h * BM + t] = (dpart[0] + dpart[1]) + (dpart[2] + dpart[3]);
-                named_bar_sync(1 + wq, 64);   // both halves read S/dP and posted their D part
+                named_bar_sync(1 + wq, 64);   // both halves posted their D part
+                if (tr) trace_ev(p, j, 7);
                 const float Dv = dxb[t] + dxb[BM + t];
 #pragma unroll
                 for (int e = 0; e < 48; e += 2) {
                     const float d0 = __uint_as_float(rs[e]) * (__uint_as_float(rd[e]) - Dv);
                     const float d1 = __uint_as_float(rs[e + 1]) * (__uint_as_float(rd[e + 1]) - Dv);
-                    split_bf16x2(d0, d1, pk[e / 2], pk2[e / 2]);
+                    pk[e / 2] = pack_f16x2(d0, d1);
                 }
-                // dS_hi | dS_lo packed over S (keys 2c, 2c+1 -> column c of each half)
-                st_operand(tS, pk);
-                st_operand(tS + 96, pk2);
+                // the dS buffer is free once out(j-1) completed
+                if (j >= 1) mbar_wait(&acc_full[(j - 1) & 1], ((j - 1) >> 1) & 1);
+                if (tr) trace_ev(p, j, 6);
+#pragma unroll
+                for (int g = 0; g < 6; ++g)
+                    *ds_granule(c0 + 8 * g) = make_uint4(pk[4 * g], pk[4 * g + 1], pk[4 * g + 2], pk[4 * g + 3]);
+                fence_proxy_async_smem();
                 const int mrow = m0 + t;
                 if (h == 0 && mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = Dv;
             } else {
-                const float* cL = cl + c0;
-                const float* cD = cl + NK + c0;
+                const float4* cL = reinterpret_cast<const float4*>(cl + c0);
+                const float4* cD = reinterpret_cast<const float4*>(cl + NK + c0);
 #pragma unroll
-                for (int e = 0; e < 48; e += 2) {
-                    float pv[2], dv[2];
+                for (int e4 = 0; e4 < 12; ++e4) {
+                    const float4 l4 = cL[e4], d4 = cD[e4];
+                    const float lv[4] = {l4.x * LOG2E, l4.y * LOG2E, l4.z * LOG2E, l4.w * LOG2E};
+                    const float dvv[4] = {d4.x, d4.y, d4.z, d4.w};
+                    float pv[4], dv[4];
 #pragma unroll
-                    for (int x = 0; x < 2; ++x) {
-                        pv[x] = ((bits >> (e + x)) & 1ull) ? fast_exp2(fmaf(__uint_as_float(rs[e + x]), LOG2E, -cL[e + x])) : 0.f;
-                        dv[x] = pv[x] * (__uint_as_float(rd[e + x]) - cD[e + x]);
+                    for (int x = 0; x < 4; ++x) {
+                        const int e = 4 * e4 + x;
+                        pv[x] = ((bits >> e) & 1ull) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lv[x])) : 0.f;
+                        dv[x] = pv[x] * (__uint_as_float(rd[e]) - dvv[x]);
                     }
-                    pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
-                    split_bf16x2(dv[0], dv[1], pk2[e / 2], pk3[e / 2]);
+                    pk[2 * e4] = pack_bf16x2(pv[0], pv[1]);
+                    pk[2 * e4 + 1] = pack_bf16x2(pv[2], pv[3]);
+                    pk2[2 * e4] = pack_f16x2(dv[0], dv[1]);
+                    pk2[2 * e4 + 1] = pack_f16x2(dv[2], dv[3]);
                 }
                 named_bar_sync(1 + wq, 64);   // both halves read S^T / dP^T
-                // P^T | dS^T_hi over S^T, dS^T_lo over dP^T
+                if (tr) trace_ev(p, j, 7);
+                // P^T (bf16) | dS^T (fp16) over S^T
                 st_operand(tS, pk);
                 st_operand(tS + 96, pk2);
-                st_operand(tP, pk3);
+                tmem_wait_st();
             }
-            tmem_wait_st();
             tc_fence_before();
             mbar_arrive(p_done);
-
-            // epilogue: drain the accumulator of this tile (NQ: dQ by the h = 0 warps; NKV: dV
-            // by h = 0, dK by h = 1) once its output MMAs completed
-            if (MODE == NKV || h == 0) {
-                mbar_wait(acc_full, j & 1);
-                tc_fence_after();
-                const BMaps& mp = p.maps[T.rl];
-                drain_store(tbase + lane_off + TACC + 64u * h, mystg, h == 0 ? &mp.o1 : &mp.o2,
-                            m0 + 32 * wq, T.u, lane, acc_free);
+            if (tr) trace_ev(p, j, 8);
+            const St done = cs;
+            have = cur.next(p.sc, T);
+            if (have) cs = setup(T, j + 1);
+            if (tr) trace_ev(p, j, 15);
+            // NQ: the accumulator of the previous tile (out(j-1) completed before dS(j) was
+            // written); NKV: this tile's, once out(j) completed
+            if (MODE == NQ) {
+                if (j >= 1) drain(j - 1, prev);
+            } else {
+                drain(j, done);
             }
+            prev = done;
         }
-        if (lane == 0) tma_store_wait_all<0>();
+        if (MODE == NQ && j >= 1) drain(j - 1, prev);
+        if (MODE == NKV && lane == 0) tma_store_wait_all<0>();
     }
     tc_fence_before();
     __syncthreads();
@@ -452,16 +561,17 @@ cudaError_t launch_nb(const void* a1, const void* a2, const void* b1, const void
         }
         p.lse = lse;
         p.D = Dws;
+        p.o1 = static_cast<uint16_t*>(o1);
         p.L = L;
         p.w = (int)wc;
         p.dil = (int)dil;
-        p.r0 = (int)r0;
-        p.nr = nr;
-        p.units = (int)units;
+
+        p.trace = (unsigned long long*)trace_buffer(MODE == NQ ? 1 : 2);
         const int64_t Lr0 = ceil_div(L - r0, dil);
-        p.tiles = (int)ceil_div(Lr0, BM);
-        const int64_t total = (int64_t)p.units * p.nr * p.tiles;
+        const int tiles = (int)ceil_div(Lr0, BM);
+        const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms_nb() ? total : num_sms_nb()));
+        sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         tc_narrow_bwd_kernel<MODE><<<grid, NTHREADS, SMEM_BYTES, st>>>(p);
         prof_mark(st);
         cudaError_t e = cudaGetLastError();

@@ -74,6 +74,20 @@ __global__ void bench(int outer, unsigned long long* out, float* val) {
                 mma_ss_x4(tb + (i % NACC) * N, sdesc_sw128(sa + ks * 8192, 16, 1024),
                           sdesc_sw128(sb + ks * 8192, 16, 1024), id, i != 0);
             }
+        } else if (STYLE == 4) {   // TS: A from TMEM (cols 256..), B MN-major (LBO 8192)
+            constexpr uint32_t idT = idesc_bf16(M, N, false, true);
+#pragma unroll 1
+            for (int i = 0; i < outer * 4; ++i) {
+                const int ks = i & 3;
+                mma_ts_x4<8, 128>(tb + (i % NACC) * N, tb + 256 + 32 * ks, sdesc_sw128(sb + ks * 8192, 8192, 1024), idT, i != 0);
+            }
+        } else if (STYLE == 5) {   // latency: 4 SS MMAs + commit + wait, repeated
+#pragma unroll 1
+            for (int i = 0; i < outer; ++i) {
+                mma_ss_x4<2, 2>(tb, da, db, id, 0);
+                mma_commit(&bar);
+                mbar_wait(&bar, i & 1);
+            }
         } else
         for (int o = 0; o < outer; ++o) {
 #pragma unroll
@@ -86,8 +100,10 @@ __global__ void bench(int outer, unsigned long long* out, float* val) {
                     else mma_ss(tb + a * N, da + off, db + off, id, acc);
                 }
         }
-        if (STYLE == 0) commit_el(&bar); else mma_commit(&bar);
-        mbar_wait(&bar, 0);
+        if (STYLE != 5) {
+            if (STYLE == 0) commit_el(&bar); else mma_commit(&bar);
+            mbar_wait(&bar, 0);
+        }
         const unsigned long long t1 = clock64();
         if (lane == 0) out[blockIdx.x] = t1 - t0;   // the issuing thread times itself
     }
@@ -123,10 +139,10 @@ void run(unsigned long long* d) {
         cudaMemcpy(h, d, 8 * 148, cudaMemcpyDeviceToHost);
         double mx = 0;
         for (int i = 0; i < 148; ++i) mx = h[i] > mx ? h[i] : mx;
-        const double n = (double)outer * 16 * NACC;
+        const double n = STYLE == 5 ? (double)outer : (double)outer * 16 * (STYLE >= 2 ? 1 : NACC);
         if (rep == 1)
             printf("[h0=%llu] %s M=%d N=%3d chains=%d: %6.1f clk/MMA  %6.0f MAC/clk/SM\n", h[0],
-                   STYLE == 0 ? "warp+elect" : STYLE == 1 ? "lane0     " : STYLE == 2 ? "lane0-rt  " : "lane0-x4  ", M, N, NACC, mx / n, (double)M * N * 16 * n / mx);
+                   STYLE == 0 ? "warp+elect" : STYLE == 1 ? "lane0     " : STYLE == 2 ? "lane0-rt  " : STYLE == 3 ? "lane0-x4  " : STYLE == 4 ? "TS-x4     " : "lat4+cmt  ", M, N, NACC, mx / n, (double)M * N * 16 * n / mx);
     }
 }
 
@@ -135,8 +151,8 @@ int main() {
     cudaMalloc(&d, 8 * 148);
     cudaMalloc(&g_val, 4);
     run<64, 1, 0>(d); run<128, 1, 0>(d); run<256, 1, 0>(d); run<192, 1, 0>(d);
-    run<64, 1, 2>(d); run<64, 2, 2>(d); run<128, 1, 2>(d); run<256, 1, 2>(d);
-    run<64, 1, 3>(d); run<64, 2, 3>(d); run<128, 1, 3>(d); run<256, 1, 3>(d);
-    run<64, 1, 0, 64>(d);
+    run<64, 1, 3>(d); run<128, 1, 3>(d); run<192, 1, 3>(d);
+    run<64, 1, 4>(d); run<128, 1, 4>(d); run<64, 2, 4>(d);
+    run<192, 1, 5>(d); run<64, 1, 5>(d);
     return 0;
 }
