@@ -51,6 +51,7 @@
 
 #include "internal.h"
 #include "tc_common.cuh"
+#include "tile_sched.cuh"
 #include "tmap.h"
 
 namespace ftw {
@@ -77,7 +78,8 @@ struct WParams {
     WMaps maps[RES_PER_LAUNCH];
     float* lse;
     int64_t L;
-    int d, w, dil, r0, nr, nkc, units, tiles;
+    int d, w, dil, nkc;
+    SchedParams sc;
     int nq, nks, nvs;   // Q buffers, K ring slots, V ring slots
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, mode 0)
     int dbg;                     // 0 unless built with FT_WIDE_DBG_KNOBS; timing experiments only
@@ -98,28 +100,8 @@ __device__ __forceinline__ void trace_put(const WParams& p, int j, int slot, uns
     if (p.trace && j < 8) p.trace[((size_t)blockIdx.x * 8 + j) * 48 + slot] = v;
 }
 
-struct Tile {
-    int u, rl, r, Lr, m0;
-};
-__device__ __forceinline__ bool decode_tile(const WParams& p, int tau, Tile& T) {
-    const int t = tau % p.tiles;
-    const int rest = tau / p.tiles;
-    T.rl = rest % p.nr;
-    T.u = rest / p.nr;
-    T.r = p.r0 + T.rl;
-    T.Lr = (int)((p.L - T.r + p.dil - 1) / p.dil);
-    T.m0 = t * BM;
-    return T.m0 < T.Lr;
-}
-struct TileCursor {
-    int tau;
-    __device__ explicit TileCursor(int start) : tau(start - (int)gridDim.x) {}
-    __device__ bool next(const WParams& p, int total, Tile& T) {
-        for (tau += gridDim.x; tau < total; tau += gridDim.x)
-            if (decode_tile(p, tau, T)) return true;
-        return false;
-    }
-};
+using Tile = SchedTile;
+using TileCursor = SchedCursor<BM>;
 
 __device__ __forceinline__ float fast_exp2(float x) {
     float y;
@@ -166,7 +148,6 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
     const int d = p.d, w = p.w, nkc = p.nkc, nds = d / 64;
     const int NOB = 128 / d;                          // O buffers (tiles in flight)
     const int mid = nkc / 2;                          // first chunk visited (in every band)
-    const int total = p.units * p.nr * p.tiles;
     const uint32_t TB = tile_bytes(d);
 
     uint8_t* sQ = smem;                               // [nq] Q tiles
@@ -214,7 +195,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                 mbar_init(&st_full[i], 128);
             }
             fence_barrier_init();
-            for (int i = 0; i < p.nr; ++i) {
+            for (int i = 0; i < p.sc.nr; ++i) {
                 tma_prefetch(&p.maps[i].q); tma_prefetch(&p.maps[i].k);
                 tma_prefetch(&p.maps[i].v); tma_prefetch(&p.maps[i].o);
             }
@@ -233,9 +214,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
             // Order = consumption order: Q(j), then K_c / V_c per chunk.
             Ring kr, vr;
             int j = 0;
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
-            while (cur.next(p, total, T)) {
+            while (cur.next(p.sc, T)) {
                 const WMaps& mp = p.maps[T.rl];
                 const int qb = j % p.nq;
                 if (j >= p.nq) mbar_wait(&q_empty[qb], ((j / p.nq) - 1) & 1);
@@ -271,9 +252,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
             const uint32_t idS = idesc_bf16(128, KC, false, false);
             Ring kr;
             int j = 0, gk = 0;   // gk: global chunk-step counter (S buffer gk & 1)
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
-            while (cur.next(p, total, T)) {
+            while (cur.next(p.sc, T)) {
                 const int qb = j % p.nq;
                 mbar_wait(&q_full[qb], (j / p.nq) & 1);
                 tc_fence_after();
@@ -316,9 +297,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
             const uint32_t idO = idesc_bf16(128, d, false, true);
             Ring vr;
             int j = 0, gk = 0;
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
-            while (cur.next(p, total, T)) {
+            while (cur.next(p.sc, T)) {
                 const bool tr = p.trace && j < 8;
                 unsigned long long w_p = 0, w_o = 0, w_v = 0, t0 = 0;
                 const int ob = j % NOB;
@@ -371,7 +352,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
         uint32_t zero16[16];
 #pragma unroll
         for (int e = 0; e < 16; ++e) zero16[e] = 0u;
-        TileCursor cur(blockIdx.x);
+        TileCursor cur(p.sc);
         Tile T;
         // warp-uniform band extent of rows 32*wq.. in halo columns
         const int hlo = 32 * wq, hhi = 32 * wq + 31 + 2 * w;
@@ -384,7 +365,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
             ++xc;
             return fmaxf(slot[t], slot[128 + t]);
         };
-        while (cur.next(p, total, T)) {
+        while (cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t, kb = m0 - w;
             const bool tr = p.trace && j < 8 && t == 0 && hf == 0;
             unsigned long long acc_t[4] = {0, 0, 0, 0}, t0 = 0, t1 = 0;
@@ -551,9 +532,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
         const uint32_t trow = tbase + ((uint32_t)(ew * 32) << 16);
         uint8_t* mystg = ostg + ew * nds * STG;
         int j = 0;
-        TileCursor cur(blockIdx.x);
+        TileCursor cur(p.sc);
         Tile T;
-        while (cur.next(p, total, T)) {
+        while (cur.next(p.sc, T)) {
             const WMaps& mp = p.maps[T.rl];
             const int ob = j % NOB;
             mbar_wait(&st_full[j & 1], (j >> 1) & 1);
@@ -690,10 +671,7 @@ cudaError_t tc_wide_fwd(const void* q, const void* k, const void* v, void* out, 
         p.d = (int)d;
         p.w = (int)wc;
         p.dil = (int)dil;
-        p.r0 = (int)r0;
-        p.nr = nr;
         p.nkc = nkc;
-        p.units = (int)units;
         p.nq = nq;
         p.nks = nks;
         p.nvs = nvs;
@@ -705,9 +683,10 @@ cudaError_t tc_wide_fwd(const void* q, const void* k, const void* v, void* out, 
         }
 #endif
         const int64_t Lr0 = ceil_div(L - r0, dil);
-        p.tiles = (int)ceil_div(Lr0, BM);
-        const int64_t total = (int64_t)p.units * p.nr * p.tiles;
+        const int tiles = (int)ceil_div(Lr0, BM);
+        const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms_w() ? total : num_sms_w()));
+        sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_bytes((int)d) + (size_t)(nq + nks + nvs) * tile_bytes((int)d);
         if (psm_for((int)d)) tc_wide_fwd_kernel<true><<<grid, NTHREADS, smem, st>>>(p);
         else tc_wide_fwd_kernel<false><<<grid, NTHREADS, smem, st>>>(p);

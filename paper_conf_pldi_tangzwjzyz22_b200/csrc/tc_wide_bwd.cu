@@ -38,6 +38,7 @@
 
 #include "internal.h"
 #include "tc_common.cuh"
+#include "tile_sched.cuh"
 #include "tmap.h"
 
 namespace ftw {
@@ -67,7 +68,8 @@ struct BParams {
     const float* lse;
     float* D;       // WQ: written; WKV: read
     int64_t L;
-    int d, w, dil, r0, nr, nkc, units, tiles;
+    int d, w, dil, nkc;
+    SchedParams sc;
     int na, n1, n2;   // row-operand buffers, ring-1 / ring-2 slots
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, mode 1 / 2)
 };
@@ -85,28 +87,8 @@ __device__ __forceinline__ void trace_put(const BParams& p, int j, int slot, uns
     if (p.trace && j < 8) p.trace[((size_t)blockIdx.x * 8 + j) * 48 + slot] = v;
 }
 
-struct Tile {
-    int u, rl, r, Lr, m0;
-};
-__device__ __forceinline__ bool decode_tile(const BParams& p, int tau, Tile& T) {
-    const int t = tau % p.tiles;
-    const int rest = tau / p.tiles;
-    T.rl = rest % p.nr;
-    T.u = rest / p.nr;
-    T.r = p.r0 + T.rl;
-    T.Lr = (int)((p.L - T.r + p.dil - 1) / p.dil);
-    T.m0 = t * BM;
-    return T.m0 < T.Lr;
-}
-struct TileCursor {
-    int tau;
-    __device__ explicit TileCursor(int start) : tau(start - (int)gridDim.x) {}
-    __device__ bool next(const BParams& p, int total, Tile& T) {
-        for (tau += gridDim.x; tau < total; tau += gridDim.x)
-            if (decode_tile(p, tau, T)) return true;
-        return false;
-    }
-};
+using Tile = SchedTile;
+using TileCursor = SchedCursor<BM>;
 struct Ring {
     int s = 0;
     uint32_t ph = 0;
@@ -146,7 +128,6 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
     const int d = p.d, w = p.w, nkc = p.nkc, nds = d / 64;
     const int ACC = acc_cols<MODE>(d), NREG = n_regions<MODE>(d);
     const int nsteps = (MODE == WQ ? 2 : 1) * nkc;   // steps per tile
-    const int total = p.units * p.nr * p.tiles;
     const uint32_t RB = row_bytes(d), SB = slot_bytes(d);
     const int NKt = nkc * KC;
 
@@ -190,7 +171,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             mbar_init(o_full, MODE == WKV ? 2 : 1);
             mbar_init(o_empty, 128);
             fence_barrier_init();
-            for (int i = 0; i < p.nr; ++i) {
+            for (int i = 0; i < p.sc.nr; ++i) {
                 const BMaps& m = p.maps[i];
                 tma_prefetch(&m.a1); tma_prefetch(&m.a2); tma_prefetch(&m.b1); tma_prefetch(&m.b2);
                 tma_prefetch(&m.o1);
@@ -221,9 +202,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
         if (lane == 0) {   // ------------------------------------------------ TMA producer
             Ring r1, r2;
             int j = 0;
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
-            while (cur.next(p, total, T)) {
+            while (cur.next(p.sc, T)) {
                 const BMaps& mp = p.maps[T.rl];
                 const int ab = j % p.na;
                 if (j >= p.na) mbar_wait(&a_empty[ab], ((j / p.na) - 1) & 1);
@@ -255,7 +236,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             Ring rr;   // ring 1 (A) or ring 2 (B)
             Ring rv;   // B, WKV: the ring-2 slot of the previous step (dV)
             int j = 0, gk = 0;
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
             // WKV, issuer B: dV(step g) = P^T(g) dO_c(g), P^T packed bf16 in g's S region
             auto issue_dv = [&](int g, bool first) {
@@ -271,7 +252,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 mma_commit(&r2_empty[rv.s]);
                 rv.adv(p.n2);
             };
-            while (cur.next(p, total, T)) {
+            while (cur.next(p.sc, T)) {
                 const int ab = j % p.na;
                 mbar_wait(&a_full[ab], (j / p.na) & 1);
                 tc_fence_after();
@@ -318,14 +299,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
         if (lane == 0) {   // ------------------------------------------------ issuer C: dQ / dK
             Ring r1;
             int j = 0, gk = 0;
-            TileCursor cur(blockIdx.x);
+            TileCursor cur(p.sc);
             Tile T;
             // dQ (WQ, dS hi/lo over S) or dK (WKV, dS^T hi/lo over dP^T): hi into column 0
             // (+ d for dK), lo into the next d columns for d = 64 (separate partial: two
             // 4-deep chains), into the same accumulator for d = 128.
             const uint32_t acc_hi = MODE == WQ ? 0u : (uint32_t)d;
             const uint32_t acc_lo = d == 64 ? acc_hi + (uint32_t)d : acc_hi;
-            while (cur.next(p, total, T)) {
+            while (cur.next(p.sc, T)) {
                 int outk = 0;   // output steps issued in this tile
                 const bool tr = p.trace && j < 8;
                 unsigned long long wp = 0, wo = 0, t0 = 0;
@@ -372,10 +353,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
         const int t = wq * 32 + lane;
         const uint32_t lrow = (uint32_t)(wq * 32) << 16;
         int j = 0, gk = 0;
-        TileCursor cur(blockIdx.x);
+        TileCursor cur(p.sc);
         Tile T;
         const int hlo = 32 * wq;   // warp-uniform band extent of rows 32*wq..: [hlo, hlo+31+2w]
-        while (cur.next(p, total, T)) {
+        while (cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t, kb = m0 - w;
             const int64_t rowbase = (int64_t)T.u * p.L + T.r;
             float lse2 = 0.f, D = 0.f;
@@ -475,9 +456,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
         const uint32_t trow = tbase + ((uint32_t)(ew * 32) << 16);
         uint8_t* mystg = ostg + ew * nds * STG;
         int j = 0;
-        TileCursor cur(blockIdx.x);
+        TileCursor cur(p.sc);
         Tile T;
-        while (cur.next(p, total, T)) {
+        while (cur.next(p.sc, T)) {
             const BMaps& mp = p.maps[T.rl];
             mbar_wait(o_full, j & 1);
             tc_fence_after();
@@ -613,18 +594,16 @@ cudaError_t launch(const void* a1, const void* a2, const void* b1, const void* b
         p.d = (int)d;
         p.w = (int)wc;
         p.dil = (int)dil;
-        p.r0 = (int)r0;
-        p.nr = nr;
         p.nkc = nkc;
-        p.units = (int)units;
         p.na = na;
         p.n1 = n1;
         p.n2 = n2;
         p.trace = (unsigned long long*)trace_buffer(MODE == WQ ? 1 : 2);
         const int64_t Lr0 = ceil_div(L - r0, dil);
-        p.tiles = (int)ceil_div(Lr0, BM);
-        const int64_t total = (int64_t)p.units * p.nr * p.tiles;
+        const int tiles = (int)ceil_div(Lr0, BM);
+        const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms_b() ? total : num_sms_b()));
+        sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_bytes<MODE>((int)d, nkc) + (size_t)na * 2 * row_bytes((int)d) +
                             (size_t)(n1 + n2) * slot_bytes((int)d);
         tc_wide_bwd_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
