@@ -76,8 +76,10 @@ def kernel_bytes_per_row(kind: str, d: int, e: int) -> int:
     """Minimal HBM bytes one row of each kernel must move.
     fwd : read q, k, v ; write o (dtype) and lse (fp32)                 = 4de + 4
     bwdA: read q, k, v, dout, lse ; write dq, D                          = 5de + 8
-    bwdB: read q, k, v, dout, lse, D ; write dk, dv                      = 6de + 8"""
-    return {"fwd": 4 * d * e + 4, "bwdA": 5 * d * e + 8, "bwdB": 6 * d * e + 8}[kind]
+    bwdB: read q, k, v, dout, lse, D ; write dk, dv                      = 6de + 8
+    rowdot (wide windows): read dout, o ; write D                        = 2de + 4"""
+    return {"fwd": 4 * d * e + 4, "bwdA": 5 * d * e + 8, "bwdB": 6 * d * e + 8,
+            "rowdot": 2 * d * e + 4}[kind]
 
 
 def step_bytes_per_row(d: int, e: int) -> int:
@@ -322,7 +324,11 @@ def main():
     if path_f == ft.PATH_TC or path_f == ft.PATH_SIMT:
         for i in range(nf):
             kinds[f"fwd{i}"] = "fwd"
-    kinds.update({f"bwd{i}": ("bwdA" if i == 0 else "bwdB") for i in range(nb)})
+    # backward launches: [rowdot,] bwdA x g, bwdB x g (g residue groups); the band and narrow
+    # kernels have no rowdot
+    pre = nb % 2
+    g = (nb - pre) // 2
+    kinds.update({f"bwd{i}": ("rowdot" if i < pre else "bwdA" if i < pre + g else "bwdB") for i in range(nb)})
     mean_k = {n: sum(x) / len(x) for n, x in kdur.items()}
     dom = max(mean_k, key=mean_k.get)
     # rows processed per launch: all rows (fwd launches are per residue group)

@@ -84,10 +84,10 @@ cudaError_t tc_wide_fwd(const void* q, const void* k, const void* v, void* out, 
 int tc_wide_launches(int64_t L, int64_t dil);
 // wide-window backward, TMEM region rotation, three MMA issuers -- tc_wide_bwd.cu
 bool tc_wide_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
-cudaError_t tc_wide_bwd(const void* q, const void* k, const void* v, const float* lse,
-                        const void* dout, void* dq, void* dk, void* dv, float* Dws, int64_t B,
-                        int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
-                        int* launches);
+cudaError_t tc_wide_bwd(const void* q, const void* k, const void* v, const void* out,
+                        const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
+                        int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                        cudaStream_t st, int* launches);
 
 // d = 64, w <= 32 forward with two ping-pong softmax warpgroups -- tc_narrow.cu
 bool tc_narrow_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
@@ -100,6 +100,8 @@ cudaError_t tc_narrow_bwd(const void* q, const void* k, const void* v, const flo
                           const void* dout, void* dq, void* dk, void* dv, float* Dws, int64_t B,
                           int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
                           int* launches);
+
+int tc_wide_bwd_pre_launches();   // 1 when the wide backward first runs rowdot_kernel (D)
 
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();

@@ -56,6 +56,7 @@ enum { FWD = 0, BWDQ = 1, BWDKV = 2 };
 constexpr int BM = 128;
 constexpr int KB = 64;                   // key-block rows of an output-GEMM B operand
 constexpr int RES_PER_LAUNCH = 3;        // residues per launch (8 tensor maps each)
+static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t ABYTES = BM * 128;    // one 128-row x 64-col bf16 slice (SW128)
 constexpr uint32_t OBOX = KB * 128;      // one 64-row x 64-col bf16 box
 constexpr uint32_t STG = 32 * 128;       // one warp's 32-row x 64-col staging slice
@@ -834,7 +835,10 @@ int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
 }
 int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
     if (tc_narrow_bwd_supported(1, L, d, w, dil)) return 2 * tc_narrow_launches(L, dil);
-    return 2 * (halo_rows(L, w) <= 256 ? band_launches(L, dil) : tc_chunk_launches(L, dil));
+    if (halo_rows(L, w) <= 256) return 2 * band_launches(L, dil);
+    const char* v1 = getenv("FT_WINATTN_WIDE_V1");
+    const bool wide = !(v1 && atoi(v1) == 1) && tc_wide_bwd_supported(1, L, d, w, dil);
+    return 2 * tc_chunk_launches(L, dil) + (wide ? tc_wide_bwd_pre_launches() : 0);
 }
 
 cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B,
@@ -857,13 +861,14 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
                    const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
                    int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                    cudaStream_t st, int* launches) {
-    (void)out;   // D_i is recomputed exactly as sum_j P_ij dP_ij by the BWDQ kernel
+    // band kernels: D_i is recomputed exactly as sum_j P_ij dP_ij by BWDQ (reading R1); the
+    // wide (d <= 128) kernels take D = rowsum(dout * out)
     if (launches) *launches = 0;
     if (halo_rows(L, w) > 256) {
         const char* v1 = getenv("FT_WINATTN_WIDE_V1");   // A/B timing: previous chunk kernels
         if ((v1 && atoi(v1) == 1) || !tc_wide_bwd_supported(B * H, L, d, w, dil))
             return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
-        return tc_wide_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
+        return tc_wide_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     }
     if (tc_narrow_bwd_supported(B * H, L, d, w, dil))
         return tc_narrow_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);

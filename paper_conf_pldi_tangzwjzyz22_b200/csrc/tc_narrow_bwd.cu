@@ -62,6 +62,7 @@ constexpr int NK = 192;
 constexpr int NSTAGE = 2;
 constexpr int NTHREADS = 352;
 constexpr int RES_PER_LAUNCH = 3;
+static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t ABYTES = BM * D * 2;      // 16 KB: a 128-row tile
 constexpr uint32_t HBYTES = NK * D * 2;      // 24 KB: a 192-row halo
 constexpr uint32_t STAGE = 2 * ABYTES + 2 * HBYTES;   // {A1, A2, B1, B2}

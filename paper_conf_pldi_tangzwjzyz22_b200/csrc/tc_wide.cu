@@ -63,6 +63,7 @@ constexpr int BM = 128;
 constexpr int KC = 128;
 constexpr int NTHREADS = 480;
 constexpr int RES_PER_LAUNCH = 4;
+static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr int MAX_RING = 8;
 constexpr uint32_t BOX = 128 * 128;   // one 128-row x 64-col bf16 box (SW128)
 constexpr uint32_t STG = 32 * 128;    // one epilogue warp's 32-row x 64-col staging slice
