@@ -101,8 +101,6 @@ cudaError_t tc_narrow_bwd(const void* q, const void* k, const void* v, const flo
                           int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
                           int* launches);
 
-int tc_wide_bwd_pre_launches();   // 1 when the wide backward first runs rowdot_kernel (D)
-
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();
 void* trace_buffer(int kernel_mode);   // ft_winattn_debug_trace target for a kernel mode, or null

@@ -836,9 +836,7 @@ int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
 int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
     if (tc_narrow_bwd_supported(1, L, d, w, dil)) return 2 * tc_narrow_launches(L, dil);
     if (halo_rows(L, w) <= 256) return 2 * band_launches(L, dil);
-    const char* v1 = getenv("FT_WINATTN_WIDE_V1");
-    const bool wide = !(v1 && atoi(v1) == 1) && tc_wide_bwd_supported(1, L, d, w, dil);
-    return 2 * tc_chunk_launches(L, dil) + (wide ? tc_wide_bwd_pre_launches() : 0);
+    return 2 * tc_chunk_launches(L, dil);
 }
 
 cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B,
@@ -862,7 +860,7 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
                    int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                    cudaStream_t st, int* launches) {
     // band kernels: D_i is recomputed exactly as sum_j P_ij dP_ij by BWDQ (reading R1); the
-    // wide (d <= 128) kernels take D = rowsum(dout * out)
+    // wide kernels also compute it exactly, and read out only for the first-guess D~
     if (launches) *launches = 0;
     if (halo_rows(L, w) > 256) {
         const char* v1 = getenv("FT_WINATTN_WIDE_V1");   // A/B timing: previous chunk kernels

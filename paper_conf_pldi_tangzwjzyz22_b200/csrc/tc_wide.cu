@@ -276,14 +276,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                     tc_fence_after();
                     if (tr) w_k += gtime() - t0;
                     const uint32_t sb = smem_u32(sK + (size_t)kr.s * TB);
-                    for (int s = 0; s < ((p.dbg & 4) ? 0 : nds); ++s) {
-#pragma unroll
-                        for (int kk = 0; kk < 4; ++kk) {
-                            const uint32_t off = s * BOX + kk * 32;
-                            mma_ss(tbase + 128u * b, sdesc_sw128(sa + off, 16, 1024),
-                                   sdesc_sw128(sb + off, 16, 1024), idS, (s | kk) != 0);
-                        }
-                    }
+                    for (int s = 0; s < ((p.dbg & 4) ? 0 : nds); ++s)
+                        mma_ss_x4<2, 2>(tbase + 128u * b, sdesc_sw128(sa + s * BOX, 16, 1024),
+                                        sdesc_sw128(sb + s * BOX, 16, 1024), idS, s != 0);
                     mma_commit(&k_empty[kr.s]);
                     kr.adv(p.nks);
                     mma_commit(&s_full[b]);
@@ -324,16 +319,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                     const uint32_t tO0 = tbase + 256u + (uint32_t)(ob * 2 * d);
                     const uint32_t tO1 = tO0 + (uint32_t)d;
                     const uint32_t sPa = smem_u32(sP + (size_t)b * PBUF);
-#pragma unroll
-                    for (int kk = 0; kk < ((p.dbg & 2) ? 0 : KC / 16); ++kk) {
-                        const uint32_t acc = (i > 0 || (kk & 3) != 0) ? 1u : 0u;
-                        const uint32_t tO = kk < 4 ? tO0 : tO1;
-                        const uint64_t bd = sdesc_sw128(sb + kk * 2048, BOX, 1024);
-                        if (PSM)   // P_c from smem
-                            mma_ss(tO, sdesc_sw128(sPa + (kk >> 2) * (BM * 128) + (kk & 3) * 32, 16, 1024), bd,
-                                   idO, acc);
-                        else       // P_c packed bf16 over S_c
-                            mma_ts(tO, tbase + 128u * b + 8u * kk, bd, idO, acc);
+                    if (!(p.dbg & 2)) {   // 4 K-steps per partial, one asm block each
+                        const uint32_t acc = i > 0 ? 1u : 0u;
+                        if (PSM) {   // P_c from smem: 64-key atoms of 16 KB, 32 B per step
+                            mma_ss_x4<2, 128>(tO0, sdesc_sw128(sPa, 16, 1024), sdesc_sw128(sb, BOX, 1024), idO, acc);
+                            mma_ss_x4<2, 128>(tO1, sdesc_sw128(sPa + BM * 128, 16, 1024),
+                                              sdesc_sw128(sb + 4 * 2048, BOX, 1024), idO, acc);
+                        } else {     // P_c packed bf16 over S_c: 8 columns per step
+                            mma_ts_x4<8, 128>(tO0, tbase + 128u * b, sdesc_sw128(sb, BOX, 1024), idO, acc);
+                            mma_ts_x4<8, 128>(tO1, tbase + 128u * b + 32u, sdesc_sw128(sb + 4 * 2048, BOX, 1024), idO, acc);
+                        }
                     }
                     mma_commit(&v_empty[vr.s]);
                     vr.adv(p.nvs);

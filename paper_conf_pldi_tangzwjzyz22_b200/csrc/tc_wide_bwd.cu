@@ -72,7 +72,9 @@ struct BParams {
     int d, w, dil, nkc;
     SchedParams sc;
     int na, n1, n2;   // row-operand buffers, ring-1 / ring-2 slots
-    int dfromo;       // 1: D = rowsum(dout * out) precomputed (rowdot_kernel), WQ is one pass
+    int wqc;          // WQ in one pass with the D correction (see the header); 0: two passes
+    const uint16_t* dout;   // WQ (wqc): raw dout / out rows for D~ = dout . out
+    const uint16_t* out;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, mode 1 / 2)
 };
 
@@ -109,15 +111,16 @@ __device__ __forceinline__ void split_bf16x2(float x0, float x1, uint32_t& hi, u
     lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
 }
 
-template <int MODE> __host__ __device__ inline int acc_cols(int d) {
-    return MODE == WQ ? 128 : (d == 64 ? 192 : 256);
+// WQ: dQ (d = 64: hi and lo partials) + with wqc the PK = sum_j P_ij k_j accumulator
+template <int MODE> __host__ __device__ inline int acc_cols(int d, int wqc) {
+    return MODE == WQ ? 128 + (wqc ? d : 0) : (d == 64 ? 192 : 256);
 }
-template <int MODE> __host__ __device__ inline int n_regions(int d) { return (512 - acc_cols<MODE>(d)) / 64; }
+template <int MODE> __host__ __device__ inline int n_regions(int d, int wqc) { return (512 - acc_cols<MODE>(d, wqc)) / 64; }
 __host__ __device__ inline uint32_t row_bytes(int d) { return (uint32_t)(d / 64) * ABOX; }
 __host__ __device__ inline uint32_t slot_bytes(int d) { return (uint32_t)(d / 64) * HBOX; }
 template <int MODE> inline size_t fixed_bytes(int d, int nkc) {
     return 1024 + 4 * (size_t)(d / 64) * STG + (MODE == WKV ? 2 * (size_t)nkc * KC * sizeof(float) : 0) +
-           2 * 128 * sizeof(float) + 1024;
+           6 * 128 * sizeof(float) + 1024;
 }
 
 template <int MODE>
@@ -128,8 +131,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int d = p.d, w = p.w, nkc = p.nkc, nds = d / 64;
-    const int ACC = acc_cols<MODE>(d), NREG = n_regions<MODE>(d);
-    const int nsteps = (MODE == WQ && !p.dfromo ? 2 : 1) * nkc;   // steps per tile
+    const bool wqc = MODE == WQ && p.wqc;
+    const int ACC = acc_cols<MODE>(d, p.wqc), NREG = n_regions<MODE>(d, p.wqc);
+    const int nsteps = (MODE == WQ && !wqc ? 2 : 1) * nkc;   // steps per tile
     const uint32_t RB = row_bytes(d), SB = slot_bytes(d);
     const int NKt = nkc * KC;
 
@@ -140,7 +144,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
     float* colLse = reinterpret_cast<float*>(ostg + 4 * nds * STG);   // WKV [NKt] (log2 units)
     float* colD = colLse + (MODE == WKV ? NKt : 0);                   // WKV [NKt]
     float* Dx = colD + (MODE == WKV ? NKt : 0);                       // WQ [2 halves][128]
-    uint64_t* bars = reinterpret_cast<uint64_t*>(Dx + 2 * 128);
+    float* Dt = Dx + 2 * 128;                                         // WQ [2 tiles][128]: D~
+    float* dlt = Dt + 2 * 128;                                        // WQ [2 tiles][128]: D - D~
+    uint64_t* bars = reinterpret_cast<uint64_t*>(dlt + 2 * 128);
     uint64_t* a_full = bars;                  // [2]
     uint64_t* a_empty = bars + 2;             // [2]
     uint64_t* r1_full = bars + 4;             // [MAX_RING]
@@ -153,7 +159,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
     uint64_t* rfree = p_full + 4;             // [8] TMEM region freed
     uint64_t* o_full = rfree + 8;             // accumulators complete
     uint64_t* o_empty = o_full + 1;           // accumulators drained (128)
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(o_empty + 1);
+    uint64_t* d_full = o_empty + 1;           // [2] WQ (wqc): D - D~ of the tile published (256)
+    uint64_t* dt_full = d_full + 2;           // [2] WQ (wqc): D~ of the tile published (128)
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(dt_full + 2);
 
     if (warp == 12) {
         if (lane == 0) {
@@ -172,6 +180,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             for (int i = 0; i < 8; ++i) mbar_init(&rfree[i], 1);
             mbar_init(o_full, MODE == WKV ? 2 : 1);
             mbar_init(o_empty, 128);
+            mbar_init(&d_full[0], 256);
+            mbar_init(&d_full[1], 256);
+            mbar_init(&dt_full[0], 128);
+            mbar_init(&dt_full[1], 128);
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
                 const BMaps& m = p.maps[i];
@@ -246,10 +258,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 tc_fence_after();
                 const uint32_t xs = region_col(2 * g);
                 const uint32_t sb = smem_u32(sR2 + (size_t)rv.s * SB);
-#pragma unroll
-                for (int kk = 0; kk < KC / 16; ++kk)
-                    mma_ts(tbase, tbase + xs + 32u * (kk >> 1) + 8u * (kk & 1),
-                           sdesc_sw128(sb + kk * 2048, HBOX, 1024), idO, (first && kk == 0) ? 0u : 1u);
+                mma_ts_x4o<8, 32, 40, 128>(tbase, tbase + xs, sdesc_sw128(sb, HBOX, 1024), idO, first ? 0u : 1u);
                 mma_commit(&rfree[(2 * g) % NREG]);
                 mma_commit(&r2_empty[rv.s]);
                 rv.adv(p.n2);
@@ -272,12 +281,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     if (tr) wf += gtime() - t0;
                     const uint32_t sb = smem_u32((isA ? sR1 : sR2) + (size_t)rr.s * SB);
                     const uint32_t td = tbase + region_col(m);
-                    for (int s = 0; s < nds; ++s) {
-#pragma unroll
-                        for (int kk = 0; kk < 4; ++kk)
-                            mma_ss(td, sdesc_sw128(sa + s * ABOX + kk * 32, 16, 1024),
-                                   sdesc_sw128(sb + s * HBOX + kk * 32, 16, 1024), idS, (s | kk) != 0);
-                    }
+                    for (int s = 0; s < nds; ++s)
+                        mma_ss_x4<2, 2>(td, sdesc_sw128(sa + s * ABOX, 16, 1024),
+                                        sdesc_sw128(sb + s * HBOX, 16, 1024), idS, s != 0);
                     mma_commit(isA ? &s_full[gk & 3] : &dp_full[gk & 3]);
                     if (isA) mma_commit(&r1_empty[rr.s]);
                     else if (MODE == WQ) mma_commit(&r2_empty[rr.s]);
@@ -317,7 +323,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     mbar_wait(&p_full[gk & 3], (gk >> 2) & 1);
                     tc_fence_after();
                     if (tr) wp += gtime() - t0;
-                    const bool out = MODE == WKV || p.dfromo || k >= nkc;
+                    const bool out = MODE == WKV || wqc || k >= nkc;
                     const int mS = 2 * gk, mD = 2 * gk + 1;
                     if (!out) {   // WQ pass 1: the softmax only read S and dP
                         mbar_arrive(&rfree[mS % NREG]);
@@ -331,16 +337,21 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     if (tr) wo += gtime() - t0;
                     const uint32_t xa = region_col(MODE == WQ ? mS : mD);   // dS (hi/lo) region
                     const uint32_t sb = smem_u32(sR1 + (size_t)r1.s * SB);
-#pragma unroll
-                    for (int kk = 0; kk < KC / 16; ++kk) {
-                        const uint64_t bd = sdesc_sw128(sb + kk * 2048, HBOX, 1024);
-                        const uint32_t ta = tbase + xa + 32u * (kk >> 1) + 8u * (kk & 1);
-                        const uint32_t acc = (outk == 0 && kk == 0) ? 0u : 1u;
-                        mma_ts(tbase + acc_hi, ta, bd, idO, acc);
-                        mma_ts(tbase + acc_lo, ta + 16, bd, idO, d == 64 ? acc : 1u);
+                    {   // K-steps kk = 0..3 of the 64-key chunk: A columns 0, 8, 32, 40 (hi;
+                        // lo at +16), B rows 16 kk (2048 B = 128 descriptor units per step)
+                        const uint64_t bd = sdesc_sw128(sb, HBOX, 1024);
+                        const uint32_t ta = tbase + xa;
+                        const uint32_t acc = outk == 0 ? 0u : 1u;
+                        mma_ts_x4o<8, 32, 40, 128>(tbase + acc_hi, ta, bd, idO, acc);
+                        mma_ts_x4o<8, 32, 40, 128>(tbase + acc_lo, ta + 16, bd, idO, d == 64 ? acc : 1u);
+                        if (wqc)   // PK += P K_c, P (bf16) packed over dP
+                            mma_ts_x4o<8, 32, 40, 128>(tbase + 128u, tbase + region_col(mD), bd, idO, acc);
                     }
                     mma_commit(&rfree[(MODE == WQ ? mS : mD) % NREG]);
-                    if (MODE == WQ) mbar_arrive(&rfree[mD % NREG]);   // dP only read by the softmax
+                    if (MODE == WQ) {
+                        if (wqc) mma_commit(&rfree[mD % NREG]);   // P read by the PK MMAs
+                        else mbar_arrive(&rfree[mD % NREG]);      // dP only read by the softmax
+                    }
                     mma_commit(&r1_empty[r1.s]);
                     r1.adv(p.n1);
                     ++outk;
@@ -373,15 +384,15 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 named_bar_sync(1, 256);
             } else {
                 lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
-                if (p.dfromo) D = mrow < Lr ? p.D[rowbase + (int64_t)mrow * p.dil] : 0.f;
             }
+            float Dtil = 0.f, Dex = 0.f;   // wqc: D~ (from the epilogue warps), exact D
             const bool tr = p.trace && j < 8 && warp == 0 && lane == 0;
             unsigned long long ws = 0, wc = 0, t0 = 0, t1 = 0;
             if (tr) trace_put(p, j, 0, gtime());
             for (int k = 0; k < nsteps; ++k, ++gk) {
                 const int c = k % nkc;
-                const bool pass2 = MODE == WQ && (p.dfromo || k >= nkc);
-                if (MODE == WQ && !p.dfromo && k == nkc) {   // end of pass 1: D of the whole row
+                const bool pass2 = MODE == WQ && (wqc || k >= nkc);
+                if (MODE == WQ && !wqc && k == nkc) {   // end of pass 1: D of the whole row
                     Dx[hf * 128 + t] = D;
                     named_bar_sync(1 + wq, 64);
                     D = Dx[t] + Dx[128 + t];
@@ -395,6 +406,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 tc_fence_after();
                 if (tr) { t1 = gtime(); ws += t1 - t0; t0 = t1; }
                 const int h0 = c * KC + 32 * hf;   // first halo column of my 32
+                if (wqc && k == 0) {   // D~ = dout_i . out_i, computed by the epilogue warps
+                    mbar_wait(&dt_full[j & 1], (j >> 1) & 1);
+                    Dtil = Dt[(j & 1) * 128 + t];
+                }
                 uint32_t rs[32], rd[32];
                 tmem_ld32(xs, rs);
                 tmem_ld32(xd, rd);
@@ -418,16 +433,27 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     }
                     D += d2[0] + d2[1];
                 } else if (MODE == WQ) {
-                    uint32_t ph[16], pl[16];
+                    // two-pass: dS = P (dP - D) with the exact D of pass 1.  wqc: dS~ = P (dP - D~),
+                    // the exact D accumulated on the way, and P (bf16) over dP for PK
+                    const float Dsub = wqc ? Dtil : D;
+                    uint32_t ph[16], pl[16], pp[16];
+                    float dd[2] = {0.f, 0.f};
 #pragma unroll
                     for (int e = 0; e < 32; e += 2) {
                         const float p0 = fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2));
                         const float p1 = fast_exp2(fmaf(__uint_as_float(rs[e + 1]), LOG2E, -lse2));
-                        split_bf16x2(p0 * (__uint_as_float(rd[e]) - D), p1 * (__uint_as_float(rd[e + 1]) - D),
+                        if (wqc) {
+                            dd[0] = fmaf(p0, __uint_as_float(rd[e]), dd[0]);
+                            dd[1] = fmaf(p1, __uint_as_float(rd[e + 1]), dd[1]);
+                            pp[e / 2] = pack_bf16x2(p0, p1);
+                        }
+                        split_bf16x2(p0 * (__uint_as_float(rd[e]) - Dsub), p1 * (__uint_as_float(rd[e + 1]) - Dsub),
                                      ph[e / 2], pl[e / 2]);
                     }
+                    if (wqc) Dex += dd[0] + dd[1];
                     tmem_st16(xs, ph);
                     tmem_st16(xs + 16, pl);
+                    if (wqc) tmem_st16(xd, pp);
                 } else {   // WKV: P^T over S^T, dS^T hi/lo over dP^T
                     uint32_t pk[16], ph[16], pl[16];
 #pragma unroll
@@ -451,6 +477,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 mbar_arrive(&p_full[gk & 3]);
                 if (tr) wc += gtime() - t0;
             }
+            if (wqc) {   // exact D of the row; the epilogue subtracts (D - D~) PK from dQ~
+                Dx[hf * 128 + t] = Dex;
+                named_bar_sync(1 + wq, 64);
+                const float Dfull = Dx[t] + Dx[128 + t];
+                if (hf == 0) {
+                    dlt[(j & 1) * 128 + t] = Dfull - Dtil;
+                    if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = Dfull;
+                }
+                mbar_arrive(&d_full[j & 1]);
+            }
             if (tr) { trace_put(p, j, 1, ws); trace_put(p, j, 2, wc); trace_put(p, j, 6, gtime()); }
             ++j;
         }
@@ -459,12 +495,46 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
         const uint32_t trow = tbase + ((uint32_t)(ew * 32) << 16);
         uint8_t* mystg = ostg + ew * nds * STG;
         int j = 0;
-        TileCursor cur(p.sc);
-        Tile T;
+        // wqc: D~_i = dout_i . out_i of a tile's rows (thread <-> row), published one tile
+        // ahead of the softmax warps that need it at the tile's first step
+        auto publish_dtil = [&](const Tile& X, int jx) {
+            const int mr = X.m0 + ew * 32 + lane;
+            float acc = 0.f;
+            if (mr < X.Lr) {
+                const int64_t off = ((int64_t)X.u * p.L + X.r + (int64_t)mr * p.dil) * d;
+                const uint4* dr = reinterpret_cast<const uint4*>(p.dout + off);
+                const uint4* orr = reinterpret_cast<const uint4*>(p.out + off);
+                for (int v = 0; v < d / 8; v += 4) {
+                    uint4 a4[4], b4[4];
+#pragma unroll
+                    for (int x = 0; x < 4; ++x) { a4[x] = dr[v + x]; b4[x] = orr[v + x]; }
+#pragma unroll
+                    for (int x = 0; x < 4; ++x) {
+                        const uint32_t* aw = reinterpret_cast<const uint32_t*>(&a4[x]);
+                        const uint32_t* bw = reinterpret_cast<const uint32_t*>(&b4[x]);
+#pragma unroll
+                        for (int y = 0; y < 4; ++y) {
+                            const float2 fa = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&aw[y]));
+                            const float2 fb = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&bw[y]));
+                            acc = fmaf(fa.x, fb.x, fmaf(fa.y, fb.y, acc));
+                        }
+                    }
+                }
+            }
+            Dt[(jx & 1) * 128 + ew * 32 + lane] = acc;
+            mbar_arrive(&dt_full[jx & 1]);
+        };
+        TileCursor cur(p.sc), nxt(p.sc);
+        Tile T, Tn;
+        if (wqc && nxt.next(p.sc, Tn)) publish_dtil(Tn, 0);
         while (cur.next(p.sc, T)) {
             const BMaps& mp = p.maps[T.rl];
-            mbar_wait(o_full, j & 1);
-            tc_fence_after();
+            if (wqc && nxt.next(p.sc, Tn)) publish_dtil(Tn, j + 1);
+            mbar_wait(o_full, j & 1);            float dl = 0.f;   // wqc: D - D~ of this row
+            if (wqc) {
+                mbar_wait(&d_full[j & 1], (j >> 1) & 1);
+                dl = dlt[(j & 1) * 128 + ew * 32 + lane];
+            }
             if (ew == 0 && lane == 0) trace_put(p, j, 30, gtime());
             if (lane == 0) tma_store_wait_read<0>();   // staging of the previous tile read
             __syncwarp();
@@ -482,14 +552,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     }
 #pragma unroll 1
                     for (int hh = 0; hh < 2; ++hh) {
-                        uint32_t v0[32], v1[32];
+                        uint32_t v0[32], v1[32], v2[32];
                         const uint32_t col = c0 + (uint32_t)(s * 64 + hh * 32);
                         tmem_ld32(trow + col, v0);
                         if (two) tmem_ld32(trow + col + (uint32_t)d, v1);
+                        if (wqc) tmem_ld32(trow + 128u + col, v2);   // PK
                         tmem_wait_ld();
                         float acc[32];
 #pragma unroll
-                        for (int e = 0; e < 32; ++e) acc[e] = __uint_as_float(v0[e]) + (two ? __uint_as_float(v1[e]) : 0.f);
+                        for (int e = 0; e < 32; ++e) {
+                            acc[e] = __uint_as_float(v0[e]) + (two ? __uint_as_float(v1[e]) : 0.f);
+                            if (wqc) acc[e] = fmaf(-dl, __uint_as_float(v2[e]), acc[e]);
+                        }
                         if (o == nout - 1 && s == nds - 1 && hh == 1) {
                             tc_fence_before();
                             mbar_arrive(o_empty);
@@ -560,40 +634,11 @@ bool plan(int d, int nkc, int& na, int& n1, int& n2) {
     return false;
 }
 
-// D_i = sum_p dout_ip out_ip (bf16 in, fp32 out) for every row: the D of the softmax
-// gradient from the saved output, as FlashAttention computes it (reading
-// R1, d <= 128).  8 threads per row, 16-byte loads, a shuffle reduction.
-__global__ void __launch_bounds__(256) rowdot_kernel(const uint4* __restrict__ dout, const uint4* __restrict__ out,
-                                                     float* __restrict__ D, int64_t rows, int vpt) {
-    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int64_t row = gt >> 3;
-    const int sub = (int)(gt & 7);
-    float acc = 0.f;
-    if (row < rows) {
-        for (int i = 0; i < vpt; ++i) {
-            const int64_t idx = row * 8 * vpt + sub + 8 * i;
-            const uint4 a = dout[idx], b = out[idx];
-            const uint32_t* aw = reinterpret_cast<const uint32_t*>(&a);
-            const uint32_t* bw = reinterpret_cast<const uint32_t*>(&b);
-#pragma unroll
-            for (int x = 0; x < 4; ++x) {
-                const float2 fa = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&aw[x]));
-                const float2 fb = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&bw[x]));
-                acc = fmaf(fa.x, fb.x, acc);
-                acc = fmaf(fa.y, fb.y, acc);
-            }
-        }
-    }
-    acc += __shfl_xor_sync(0xffffffffu, acc, 1);
-    acc += __shfl_xor_sync(0xffffffffu, acc, 2);
-    acc += __shfl_xor_sync(0xffffffffu, acc, 4);
-    if (row < rows && sub == 0) D[row] = acc;
-}
-
 template <int MODE>
 cudaError_t launch(const void* a1, const void* a2, const void* b1, const void* b2, void* o1,
                    void* o2, const float* lse, float* D, int64_t B, int64_t H, int64_t L,
-                   int64_t d, int64_t w, int64_t dil, int dfromo, cudaStream_t st, int* launches) {
+                   int64_t d, int64_t w, int64_t dil, int wqc, const void* dout, const void* out,
+                   cudaStream_t st, int* launches) {
     static std::once_flag once;
     std::call_once(once, [] {
         cudaFuncSetAttribute(tc_wide_bwd_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -632,7 +677,9 @@ cudaError_t launch(const void* a1, const void* a2, const void* b1, const void* b
         p.n1 = n1;
         p.n2 = n2;
         p.trace = (unsigned long long*)trace_buffer(MODE == WQ ? 1 : 2);
-        p.dfromo = dfromo;
+        p.wqc = MODE == WQ ? wqc : 0;
+        p.dout = static_cast<const uint16_t*>(dout);
+        p.out = static_cast<const uint16_t*>(out);
         const int64_t Lr0 = ceil_div(L - r0, dil);
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
@@ -660,36 +707,19 @@ bool tc_wide_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64
            plan<WQ>((int)d, nkc, na, n1, n2) && plan<WKV>((int)d, nkc, na, n1, n2);
 }
 
-// Exact D (two WQ passes, reading R1) by default.  FT_WINATTN_D_FROM_OUT=1 takes D =
-// rowsum(dout * out) from the bf16 output instead (one WQ pass, -12 % on C5_w256) -- an A/B
-// knob only: its D error, ~|dout| |o| 2^-9 sqrt(d), moved dq / dk by up to 1.5e-2 in the
-// parity cases, outside the 1e-2 + 2e-2|x| bound.
-static int wide_dfromo() {
-    const char* e = getenv("FT_WINATTN_D_FROM_OUT");
-    return (e && atoi(e) == 1) ? 1 : 0;
-}
-int tc_wide_bwd_pre_launches() { return wide_dfromo(); }
-
 cudaError_t tc_wide_bwd(const void* q, const void* k, const void* v, const void* out,
                         const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
                         int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                         cudaStream_t st, int* launches) {
-    const int dfromo = wide_dfromo();
-    if (dfromo) {
-        const int64_t rows = B * H * L;
-        const int vpt = (int)(d / 64);   // 16-byte vectors per thread (8 threads per row)
-        const int64_t threads = rows * 8;
-        rowdot_kernel<<<(unsigned)ceil_div(threads, 256), 256, 0, st>>>(
-            static_cast<const uint4*>(dout), static_cast<const uint4*>(out), Dws, rows, vpt);
-        prof_mark(st);
-        cudaError_t e0 = cudaGetLastError();
-        if (e0 != cudaSuccess) return e0;
-        if (launches) *launches += 1;
-    }
+    // WQ in one pass with the D correction; FT_WINATTN_WQ_TWOPASS=1 restores the two-pass
+    // schedule (exact D first, then dS = P (dP - D)) for A/B timing
+    const char* e2 = getenv("FT_WINATTN_WQ_TWOPASS");
+    const int wqc = (e2 && atoi(e2) == 1) ? 0 : 1;
     // WQ: rows Q (a1) / dO (a2), halo K (b1) / V (b2) -> dQ;  WKV: rows K / V, halo Q / dO -> dV, dK
-    cudaError_t e = launch<WQ>(q, dout, k, v, dq, nullptr, lse, Dws, B, H, L, d, w, dil, dfromo, st, launches);
+    cudaError_t e = launch<WQ>(q, dout, k, v, dq, nullptr, lse, Dws, B, H, L, d, w, dil, wqc, dout, out, st,
+                               launches);
     if (e != cudaSuccess) return e;
-    return launch<WKV>(k, v, q, dout, dv, dk, lse, Dws, B, H, L, d, w, dil, dfromo, st, launches);
+    return launch<WKV>(k, v, q, dout, dv, dk, lse, Dws, B, H, L, d, w, dil, 0, dout, out, st, launches);
 }
 
 }  // namespace ftw
