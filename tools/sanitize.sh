@@ -8,7 +8,8 @@ sys.path.insert(0, ".")
 import paper_conf_pldi_tangzwjzyz22_b200 as ft
 from synth import WinAttnShape, make_inputs
 dev = torch.device("cuda:0")
-for shape, dt in [((1, 2, 300, 64, 32, 3), "bf16"), ((1, 1, 200, 512, 32, 1), "bf16"),
+for shape, dt in [((1, 2, 300, 64, 32, 3), "bf16"), ((1, 4, 1500, 64, 32, 1), "bf16"),
+                  ((1, 2, 700, 64, 20, 5), "bf16"), ((1, 1, 200, 512, 32, 1), "bf16"),
                   ((1, 1, 600, 64, 100, 2), "bf16"), ((1, 1, 500, 128, 80, 1), "bf16"),
                   ((1, 1, 130, 64, 8, 1), "f32")]:
     s = WinAttnShape(*shape)
