@@ -530,7 +530,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
         while (cur.next(p.sc, T)) {
             const BMaps& mp = p.maps[T.rl];
             if (wqc && nxt.next(p.sc, Tn)) publish_dtil(Tn, j + 1);
-            mbar_wait(o_full, j & 1);            float dl = 0.f;   // wqc: D - D~ of this row
+            mbar_wait(o_full, j & 1);
+            tc_fence_after();
+            float dl = 0.f;   // wqc: D - D~ of this row
             if (wqc) {
                 mbar_wait(&d_full[j & 1], (j >> 1) & 1);
                 dl = dlt[(j & 1) * 128 + ew * 32 + lane];
