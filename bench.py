@@ -77,9 +77,10 @@ def kernel_bytes_per_row(kind: str, d: int, e: int) -> int:
     fwd : read q, k, v ; write o (dtype) and lse (fp32)                 = 4de + 4
     bwdA: read q, k, v, dout, lse ; write dq, D                          = 5de + 8
     bwdB: read q, k, v, dout, lse, D ; write dk, dv                      = 6de + 8
-    rowdot (wide windows): read dout, o ; write D                        = 2de + 4"""
+    rowdot (wide windows): read dout, o ; write D                        = 2de + 4
+    bwdF (d = 64, w <= 32, one kernel): read q, k, v, dout, lse ; write dq, dk, dv = 7de + 4"""
     return {"fwd": 4 * d * e + 4, "bwdA": 5 * d * e + 8, "bwdB": 6 * d * e + 8,
-            "rowdot": 2 * d * e + 4}[kind]
+            "rowdot": 2 * d * e + 4, "bwdF": 7 * d * e + 4}[kind]
 
 
 def step_bytes_per_row(d: int, e: int) -> int:
@@ -326,9 +327,14 @@ def main():
             kinds[f"fwd{i}"] = "fwd"
     # backward launches: [rowdot,] bwdA x g, bwdB x g (g residue groups); the band and narrow
     # kernels have no rowdot
-    pre = nb % 2
-    ngrp = (nb - pre) // 2
-    kinds.update({f"bwd{i}": ("rowdot" if i < pre else "bwdA" if i < pre + ngrp else "bwdB") for i in range(nb)})
+    # (the fused d = 64 backward, tc_narrow_fused.cu, is one launch per residue group)
+    groups = -(-min(dil, L) // 3)
+    if nb == groups and path_b == ft.PATH_TC and d == 64 and min(w, L) <= 32:
+        kinds.update({f"bwd{i}": "bwdF" for i in range(nb)})
+    else:
+        pre = nb % 2
+        ngrp = (nb - pre) // 2
+        kinds.update({f"bwd{i}": ("rowdot" if i < pre else "bwdA" if i < pre + ngrp else "bwdB") for i in range(nb)})
     mean_k = {n: sum(x) / len(x) for n, x in kdur.items()}
     dom = max(mean_k, key=mean_k.get)
     # rows processed per launch: all rows (fwd launches are per residue group)

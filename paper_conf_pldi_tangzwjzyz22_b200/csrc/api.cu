@@ -131,7 +131,7 @@ ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_
     if (s != FT_OK) return s;
     int n;
     if (p == FT_PATH_TC)
-        n = is_bwd ? ftw::tc_bwd_launches(seq_len, d, w, dilation)
+        n = is_bwd ? ftw::tc_bwd_launches(batch * heads, seq_len, d, w, dilation)
                    : ftw::tc_fwd_launches(seq_len, d, w, dilation);
     else
         n = is_bwd ? ftw::simt_bwd_launches() : ftw::simt_fwd_launches();

@@ -63,7 +63,7 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
                    float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
                    int64_t dil, cudaStream_t st, int* launches);
 int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
-int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
+int tc_bwd_launches(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
 
 // wide-window tensor-core kernels -- tc_chunk.cu (used when 128 + 2w > 256)
 bool tc_chunk_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
@@ -100,6 +100,14 @@ cudaError_t tc_narrow_bwd(const void* q, const void* k, const void* v, const flo
                           const void* dout, void* dq, void* dk, void* dv, float* Dws, int64_t B,
                           int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
                           int* launches);
+
+// d = 64, w <= 32 backward in ONE kernel (query-major strips, dK/dV key blocks in TMEM) --
+// tc_narrow_fused.cu.  Used instead of tc_narrow_bwd when there are >= ~4 tiles per SM.
+bool tc_narrow_fused_ok(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+int tc_narrow_fused_launches(int64_t L, int64_t dil);
+cudaError_t tc_narrow_fused_bwd(const void* q, const void* k, const void* v, const float* lse,
+                                const void* dout, void* dq, void* dk, void* dv, int64_t B, int64_t H,
+                                int64_t L, int64_t w, int64_t dil, cudaStream_t st, int* launches);
 
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();

@@ -833,7 +833,8 @@ int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
     if (tc_narrow_supported(1, L, d, w, dil)) return tc_narrow_launches(L, dil);
     return halo_rows(L, w) <= 256 ? band_launches(L, dil) : tc_chunk_launches(L, dil);
 }
-int tc_bwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
+int tc_bwd_launches(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    if (tc_narrow_fused_ok(units, L, d, w, dil)) return tc_narrow_fused_launches(L, dil);
     if (tc_narrow_bwd_supported(1, L, d, w, dil)) return 2 * tc_narrow_launches(L, dil);
     if (halo_rows(L, w) <= 256) return 2 * band_launches(L, dil);
     return 2 * tc_chunk_launches(L, dil);
@@ -868,6 +869,8 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
             return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
         return tc_wide_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     }
+    if (tc_narrow_fused_ok(B * H, L, d, w, dil))
+        return tc_narrow_fused_bwd(q, k, v, lse, dout, dq, dk, dv, B, H, L, w, dil, st, launches);
     if (tc_narrow_bwd_supported(B * H, L, d, w, dil))
         return tc_narrow_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     cudaError_t e = launch<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse),

@@ -306,3 +306,46 @@ def test_full_size_sampled(ft, name, dtype):
     # properties at any size: everything finite
     for t in (out, lse, dq, dk, dv):
         assert torch.isfinite(t).all()
+
+
+class _env:
+    def __init__(self, **kv):
+        self.kv = kv
+
+    def __enter__(self):
+        self.old = {k: os.environ.get(k) for k in self.kv}
+        os.environ.update(self.kv)
+
+    def __exit__(self, *a):
+        for k, v in self.old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+
+
+# d = 64, w <= 32 backward in one kernel (tc_narrow_fused.cu), forced even where the dispatcher
+# would pick the split kernels: strips of one tile (every CTA starts with a warm-up tile), strips
+# crossing (unit, residue) boundaries, tails of ragged residues, two launch groups, w = 0 and
+# w < 32, and enough tiles per CTA that the K (5-slot) and V (4-slot) rings wrap many times.
+FUSED = [
+    (1, 3, 129, 64, 31, 1),
+    (1, 2, 300, 64, 32, 3),
+    (1, 6, 5000, 64, 7, 3),
+    (2, 5, 2001, 64, 32, 2),
+    (1, 16, 8192, 64, 32, 1),
+    (1, 2, 700, 64, 20, 5),
+    (1, 1, 300, 64, 0, 1),
+    (1, 1, 1, 64, 3, 1),
+    (1, 64, 4096, 64, 32, 1),
+    (3, 1, 1000, 64, 16, 1),
+]
+
+
+@pytest.mark.parametrize("shape", FUSED, ids=lambda s: "x".join(map(str, s)))
+def test_narrow_fused_bwd(ft, shape):
+    sh = WinAttnShape(*shape)
+    with _env(FT_WINATTN_FUSED="2"):
+        p, n = ft.plan(True, sh.batch, sh.heads, sh.seq_len, sh.d, sh.w, sh.dilation, 1)
+        assert p == ft.PATH_TC and n == (min(sh.dilation, sh.seq_len) + 2) // 3
+        run_case(ft, sh, "bf16", None, seed=6)
