@@ -23,8 +23,9 @@
 //
 // Consecutive tiles share 64 halo rows, so K and V are staged by TMA in 64-row blocks through
 // rings (K: 5 slots, V: 4) and each tile loads two new blocks of each.  dS enters its MMAs as
-// fp16 (reading A10) and the bf16 operands it multiplies (Q_t, the K blocks) are converted to
-// fp16 in place by two converter warps after their last bf16 use (the score GEMM).
+// fp16 (reading A10), so the operands it multiplies (Q_t, the K blocks) are converted to fp16
+// in place by a converter warp as soon as they land, and the score GEMM S = Q K^T runs in fp16
+// too (dP = dO V^T stays bf16).
 //
 // P (bf16) and dS (fp16) go to shared memory (from registers: thread <-> query row) and serve
 // as MN-major A operands for the transposed products (M = keys).  Their 64-key atoms are
@@ -36,9 +37,14 @@
 // before dP is issued); dQ at [192,256); dK|dV blocks X[0] = [256,384), X[1] = [384,512);
 // tile j uses X[j&1] as A_t and X[(j+1)&1] as A_{t+1}.
 //
-// Roles (384 threads): warps 0-7 softmax + drains (warp w: TMEM lanes 32*(w%4).., column half
-// w/4 of the row's 96-column band window); warp 8 TMA producer + TMEM allocator; warp 9 MMA
-// issuer; warps 10-11 fp16 converters.
+// Measured (C5_w32, tools/trace_fused.py): ~9000 clk per tile, bound by the serial handoffs of
+// that chain (MMA issue at ~60-90 clk per N = 64 MMA, 36 output MMAs per tile; mbarrier
+// handoffs; the 48 KB drain), not by HBM (~5100 clk per tile at the measured peak).
+//
+// Roles (640 threads): warps 0-15 softmax + drains (warp w: TMEM lanes 32*(w%4).., columns
+// 24*(w/4).. of the row's 96-column band window); warp 16 TMA producer + TMEM allocator; warps
+// 17 and 19 MMA issuers (S, dP, dQ | dK, dV); warp 18 fp16 converter.  Per tile the MMA chain is
+// S(j) -> softmax -> dP(j) -> softmax -> out(j); the drain of tile j-1 runs while dP(j) does.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -62,7 +68,8 @@ constexpr int BM = 128;
 constexpr int D = 64;
 constexpr int KB = 64;                       // rows per K / V ring block
 constexpr int RK = 5, RV = 4;                // ring slots
-constexpr int NTHREADS = 384;
+constexpr int NTHREADS = 640;
+constexpr int NSM = 512;                     // softmax threads (warps 0-15)
 constexpr int RES_PER_LAUNCH = 3;
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table");
 constexpr uint32_t TILE = BM * D * 2;        // 16 KB
@@ -73,7 +80,7 @@ constexpr uint32_t O_DS0 = 0, O_Z = 8192, O_DS2 = 16384, O_DS1 = 24576;
 constexpr uint32_t O_P0 = 40960, O_P1 = 49152, O_P2 = 65536, O_ZB = 73728, OPS = 81920;
 constexpr uint32_t OFF_QO = 0, OFF_K = 2 * QO, OFF_V = OFF_K + RK * BLK, OFF_OPS = OFF_V + RV * BLK;
 constexpr uint32_t OFF_SCR = OFF_OPS + OPS;
-constexpr int SCR_FLOATS = 2 * 2 * BM + 2 * 256;   // D halves [2][2][BM], row lse [2][256]
+constexpr int SCR_FLOATS = 2 * 4 * BM + 2 * NSM;   // D parts [2][4][BM], row lse [2][NSM]
 constexpr uint32_t OFF_BAR = OFF_SCR + SCR_FLOATS * 4;
 constexpr int NBAR = 40;
 constexpr size_t SMEM_BYTES = 1024 + OFF_BAR + NBAR * 8 + 16;
@@ -169,41 +176,38 @@ __device__ __forceinline__ float fast_exp2(float x) {
     return y;
 }
 
-// A warp's 32 rows (lane = row row0 + lane) x 32 fp32 columns (this half h of d = 64) -> bf16 in
-// HBM.  Direct per-row stores (4 x 16 B per lane) put 32 different rows in every store
-// instruction, whose LSU transactions stalled the whole SM sub-partition (MMA issue and
-// mbarrier polls included; tools/trace_fused.py).  A 4 x 4 transpose of 16-byte chunks among
-// each quad of lanes (two shfl.xor butterfly stages) makes each of the 4 store instructions
-// cover 8 rows x 64 contiguous bytes instead.
-__device__ __forceinline__ void store_rows(uint16_t* t, int64_t rowbase, int dil, int row0, int Lr, int h,
-                                           int lane, const uint32_t (&v)[32]) {
-    uint32_t c[16];
+// A warp's 32 rows (lane = row row0 + lane) x 16 fp32 columns (part pq of d = 64) -> bf16 in HBM.
+// Lane pairs swap one 16-byte chunk (shfl.xor 1), so each of the two store instructions covers
+// 16 rows x 32 contiguous bytes instead of 32 rows x 16 B: per-row direct stores put so many LSU
+// transactions in flight that they stalled the whole SM sub-partition, MMA issue and mbarrier
+// polls included (tools/trace_fused.py).
+__device__ __forceinline__ void store_rows16(uint16_t* t, int64_t rowbase, int dil, int row0, int Lr, int pq,
+                                             int lane, const uint32_t (&v)[16]) {
+    uint32_t c[8];
 #pragma unroll
-    for (int i = 0; i < 16; ++i) c[i] = pack_bf16x2(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
+    for (int i = 0; i < 8; ++i) c[i] = pack_bf16x2(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
+    const bool hi = (lane & 1) != 0;
 #pragma unroll
-    for (int m = 1; m <= 2; m <<= 1) {
-        const bool hi = (lane & m) != 0;
-#pragma unroll
-        for (int k0 = 0; k0 < 4; ++k0) {
-            if (k0 & m) continue;
-            const int k1 = k0 | m;
-#pragma unroll
-            for (int x = 0; x < 4; ++x) {
-                const uint32_t send = hi ? c[4 * k0 + x] : c[4 * k1 + x];
-                const uint32_t recv = __shfl_xor_sync(0xffffffffu, send, m);
-                if (hi) c[4 * k0 + x] = recv;
-                else c[4 * k1 + x] = recv;
-            }
-        }
+    for (int x = 0; x < 4; ++x) {
+        const uint32_t send = hi ? c[x] : c[4 + x];
+        const uint32_t recv = __shfl_xor_sync(0xffffffffu, send, 1);
+        if (hi) c[x] = recv;
+        else c[4 + x] = recv;
     }
-    const int g = lane >> 2, ch = lane & 3;
+    const int pr = lane >> 1, ch = lane & 1;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const int row = row0 + 4 * g + q;
+    for (int q = 0; q < 2; ++q) {
+        const int row = row0 + 2 * pr + q;
         if (row >= 0 && row < Lr)
-            *reinterpret_cast<uint4*>(t + (rowbase + (int64_t)row * dil) * D + 32 * h + 8 * ch) =
+            *reinterpret_cast<uint4*>(t + (rowbase + (int64_t)row * dil) * D + 16 * pq + 8 * ch) =
                 make_uint4(c[4 * q], c[4 * q + 1], c[4 * q + 2], c[4 * q + 3]);
     }
+}
+
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t* r) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+                 : "r"(taddr));
 }
 
 // bf16 at src -> fp16 at dst (may alias), `bytes`, by the converter warp
@@ -256,7 +260,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
     for (int i = threadIdx.x; i < (int)(OPS / 16); i += NTHREADS)
         reinterpret_cast<uint4*>(ops)[i] = make_uint4(0u, 0u, 0u, 0u);
     fence_proxy_async_smem();
-    if (warp == 8) {
+    if (warp == 16) {
         if (lane == 0) {
             for (int i = 0; i < 2; ++i) {
                 mbar_init(&qo_full[i], 1);
@@ -264,16 +268,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 mbar_init(&s_full[i], 1);
                 mbar_init(&oq_full[i], 1);
                 mbar_init(&okv_full[i], 1);
-                mbar_init(&accfree[i], 256);
+                mbar_init(&accfree[i], NSM);
                 mbar_init(&convB[i], 32);
             }
             for (int i = 0; i < RK; ++i) { mbar_init(&kfull[i], 1); mbar_init(&kempty[i], 1); }
             for (int i = 0; i < RV; ++i) { mbar_init(&vfull[i], 1); mbar_init(&vempty[i], 1); }
-            mbar_init(s_free, 256);
+            mbar_init(s_free, NSM);
             mbar_init(dp_full, 1);
-            mbar_init(dp_free, 256);
-            mbar_init(p_done, 256);
-            mbar_init(dqfree, 256);
+            mbar_init(dp_free, NSM);
+            mbar_init(p_done, NSM);
+            mbar_init(dqfree, NSM);
             mbar_init(opfree, 2);
             fence_barrier_init();
             for (int i = 0; i < p.nr; ++i) {
@@ -290,7 +294,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
     tc_fence_after();
     const uint32_t tbase = *tmem_holder;
 
-    if (warp == 8) {
+    if (warp == 16) {
         if (lane == 0) {   // ---------------------------------------------------- TMA producer
             FCursor cur(p);
             FItem it;
@@ -318,7 +322,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 trace_ev(p, j, 10);
             }
         }
-    } else if (warp == 10) {   // ---------------------------------------------- fp16 converter
+    } else if (warp == 18) {   // ---------------------------------------------- fp16 converter
         // Q_t and the tile's new K blocks to fp16 in place as soon as they land: dS enters its
         // MMAs as fp16, so the operands it multiplies (Q for dK, K for dQ) and therefore the score
         // GEMM S = Q K^T run in fp16 (exact for bf16 values of magnitude 6.1e-5 .. 65504)
@@ -338,9 +342,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
             mbar_arrive(&convB[j & 1]);
             if (lane == 0) trace_ev(p, j, 13);
         }
-    } else if (warp == 9 || warp == 11) {
-        // Two MMA issuers.  Issuer 1 (warp 9): S(j), dP(j), then dQ(j) once the softmax wrote
-        // dS.  Issuer 2 (warp 11): the dK / dV products of tile j.  One thread cannot issue the
+    } else if (warp == 17 || warp == 19) {
+        // Two MMA issuers.  Issuer 1 (warp 17): S(j), dP(j), then dQ(j) once the softmax wrote
+        // dS.  Issuer 2 (warp 19): the dK / dV products of tile j.  One thread cannot issue the
         // ~50 MMAs of a tile (N = 64: ~48 clk each in the pipe, 60-90 clk each to issue) and wait
         // on their barriers fast enough (tools/trace_fused.py).
         constexpr uint32_t idS64 = idesc_f16(BM, 64, false, false);      // S: fp16 Q and K
@@ -358,7 +362,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
         FItem I, N;
         bool have = cur.next(p, I);
         nx.next(p, N);   // nx runs one item ahead of cur
-        if (warp == 9 && lane == 0) {   // ------------------------------------------ issuer 1
+        if (warp == 17 && lane == 0) {   // ----------------------------------------- issuer 1
             // C[0..192) = A (128 x 64, K-major) x three consecutive ring blocks (K-major), split
             // into contiguous runs of slots
             auto score = [&](uint32_t a_addr, uint32_t ring, int R, int s0, bool f16) {
@@ -417,7 +421,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 I = N;
                 have = hnext;
             }
-        } else if (warp == 11 && lane == 0) {   // ------------------------------------ issuer 2
+        } else if (warp == 19 && lane == 0) {   // ----------------------------------- issuer 2
             int x_req[2] = {0, 0}, x_wait[2] = {0, 0};
             auto wait_x = [&](int b) {
                 if (x_req[b] > x_wait[b]) {
@@ -467,13 +471,15 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 have = hnext;
             }
         }
-    } else {   // ------------------------------------------------------------ softmax warps 0-7
-        const int wq = warp & 3, h = warp >> 2;
+    } else {   // ----------------------------------------------------------- softmax warps 0-15
+        // warp w: TMEM lanes 32*(w%4).. (thread <-> query row t), columns 24*(w/4) .. +23 of the
+        // row's 96-column band window; four warps per row exchange their parts of D in smem
+        const int wq = warp & 3, pq = warp >> 2;
         const int t = wq * 32 + lane;
         const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
-        const int c0 = 32 * wq + 48 * h;   // first of this thread's 48 halo columns
-        float* dx = scr;                   // [2][2][BM]
-        float* lpre = scr + 2 * 2 * BM;    // [2][256]
+        const int c0 = 32 * wq + 24 * pq;  // first of this thread's 24 halo columns
+        float* dx = scr;                   // [2][4][BM]
+        float* lpre = scr + 2 * 4 * BM;    // [2][NSM]
         // 16-byte granule of row t, columns c .. c+7, in the compressed operand atoms
         auto gran = [&](uint32_t o0, uint32_t o1, uint32_t o2, int c) -> uint4* {
             const int a = c >> 6;
@@ -483,44 +489,45 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
         auto prefetch = [&](const FItem& X, int jx) {
             const int mrow = X.m0 + t;
             const bool ok = mrow < X.Lr;
-            cp_async4(lpre + (jx & 1) * 256 + threadIdx.x, p.lse + (ok ? X.rowbase + (int64_t)mrow * p.dil : 0),
+            cp_async4(lpre + (jx & 1) * NSM + threadIdx.x, p.lse + (ok ? X.rowbase + (int64_t)mrow * p.dil : 0),
                       ok ? 4u : 0u);
             cp_async_commit();
         };
+        // accumulators of tile i -> HBM: this warp's 32 rows x 16 columns of dQ, dK, dV
         auto drain = [&](int i, const FItem& X) {
-            uint32_t va[32], vb[32];
+            uint32_t va[16], vb[16];
             if (!X.warm) {
                 mbar_wait(&oq_full[i & 1], (i >> 1) & 1);
                 tc_fence_after();
-                tmem_ld32(tbase + lane_off + T_DQ + 32u * h, va);
+                tmem_ld16(tbase + lane_off + T_DQ + 16u * pq, va);
                 tmem_wait_ld();
                 tc_fence_before();
                 mbar_arrive(dqfree);
                 if (threadIdx.x == 0) trace_ev(p, i + 1, 21);
-                store_rows(p.dq, X.rowbase, p.dil, X.m0 + 32 * wq, X.Lr, h, lane, va);
+                store_rows16(p.dq, X.rowbase, p.dil, X.m0 + 32 * wq, X.Lr, pq, lane, va);
                 mbar_wait(&okv_full[i & 1], (i >> 1) & 1);
                 tc_fence_after();
                 const uint32_t xa = tbase + lane_off + T_X + 128u * (i & 1);
-                tmem_ld32(xa + 32u * h, va);
-                tmem_ld32(xa + 64u + 32u * h, vb);
+                tmem_ld16(xa + 16u * pq, va);
+                tmem_ld16(xa + 64u + 16u * pq, vb);
                 tmem_wait_ld();
                 tc_fence_before();
                 mbar_arrive(&accfree[i & 1]);
                 if (threadIdx.x == 0) trace_ev(p, i + 1, 22);
-                store_rows(p.dk, X.rowbase, p.dil, X.m0 - w + 32 * wq, X.Lr, h, lane, va);
-                store_rows(p.dv, X.rowbase, p.dil, X.m0 - w + 32 * wq, X.Lr, h, lane, vb);
+                store_rows16(p.dk, X.rowbase, p.dil, X.m0 - w + 32 * wq, X.Lr, pq, lane, va);
+                store_rows16(p.dv, X.rowbase, p.dil, X.m0 - w + 32 * wq, X.Lr, pq, lane, vb);
             }
             if (X.tail) {
                 mbar_wait(&okv_full[i & 1], (i >> 1) & 1);
                 tc_fence_after();
                 const uint32_t xb = tbase + lane_off + T_X + 128u * ((i + 1) & 1);
-                tmem_ld32(xb + 32u * h, va);
-                tmem_ld32(xb + 64u + 32u * h, vb);
+                tmem_ld16(xb + 16u * pq, va);
+                tmem_ld16(xb + 64u + 16u * pq, vb);
                 tmem_wait_ld();
                 tc_fence_before();
                 mbar_arrive(&accfree[(i + 1) & 1]);
-                store_rows(p.dk, X.rowbase, p.dil, X.m0 - w + BM + 32 * wq, X.Lr, h, lane, va);
-                store_rows(p.dv, X.rowbase, p.dil, X.m0 - w + BM + 32 * wq, X.Lr, h, lane, vb);
+                store_rows16(p.dk, X.rowbase, p.dil, X.m0 - w + BM + 32 * wq, X.Lr, pq, lane, va);
+                store_rows16(p.dv, X.rowbase, p.dil, X.m0 - w + BM + 32 * wq, X.Lr, pq, lane, vb);
             }
         };
         FCursor cur(p), nx(p);
@@ -530,32 +537,31 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
         int j = 0;
         for (; cur.next(p, I); ++j) {
             cp_async_wait_all();
-            const float lse2 = lpre[(j & 1) * 256 + threadIdx.x] * LOG2E;
+            const float lse2 = lpre[(j & 1) * NSM + threadIdx.x] * LOG2E;
             hn = nx.next(p, In);
             if (hn) prefetch(In, j + 1);
             // band columns of row t: n in [t, t+2w], keys inside the sequence, query inside too
             const int kb = I.m0 - w;
             const int lo = max(t, -kb) - c0;
             const int hi = (I.m0 + t < I.Lr) ? min(t + 2 * w, I.Lr - 1 - kb) - c0 : -1;
-            const int l0 = max(lo, 0), h0 = min(hi, 47);
-            const uint64_t bits = h0 < l0 ? 0ull : ((~0ull >> (63 - h0)) & (~0ull << l0));
+            const int l0 = max(lo, 0), h0 = min(hi, 23);
+            const uint32_t bits = h0 < l0 ? 0u : ((~0u >> (31 - h0)) & (~0u << l0));
 
             mbar_wait(&s_full[j & 1], (j >> 1) & 1);
             tc_fence_after();
             const bool tr = threadIdx.x == 0;
             if (tr) trace_ev(p, j, 4);
-            uint32_t rs[48], rd[48];
+            uint32_t rs[24], rd[24];
             tmem_ld16(tbase + lane_off + c0, *reinterpret_cast<uint32_t(*)[16]>(&rs[0]));
-            tmem_ld16(tbase + lane_off + c0 + 16, *reinterpret_cast<uint32_t(*)[16]>(&rs[16]));
-            tmem_ld16(tbase + lane_off + c0 + 32, *reinterpret_cast<uint32_t(*)[16]>(&rs[32]));
+            tmem_ld8(tbase + lane_off + c0 + 16, &rs[16]);
             tmem_wait_ld();
             tc_fence_before();
             mbar_arrive(s_free);
-            uint32_t pk[24];
+            uint32_t pk[12];
 #pragma unroll
-            for (int e = 0; e < 48; e += 2) {
-                const float p0 = ((bits >> e) & 1ull) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f;
-                const float p1 = ((bits >> (e + 1)) & 1ull) ? fast_exp2(fmaf(__uint_as_float(rs[e + 1]), LOG2E, -lse2)) : 0.f;
+            for (int e = 0; e < 24; e += 2) {
+                const float p0 = ((bits >> e) & 1u) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f;
+                const float p1 = ((bits >> (e + 1)) & 1u) ? fast_exp2(fmaf(__uint_as_float(rs[e + 1]), LOG2E, -lse2)) : 0.f;
                 rs[e] = __float_as_uint(p0);
                 rs[e + 1] = __float_as_uint(p1);
                 pk[e / 2] = pack_bf16x2(p0, p1);
@@ -564,7 +570,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
             // tile j-1's output MMAs completed
             if (j >= 1) mbar_wait(opfree, (j - 1) & 1);
 #pragma unroll
-            for (int g = 0; g < 6; ++g)
+            for (int g = 0; g < 3; ++g)
                 *gran(O_P0, O_P1, O_P2, c0 + 8 * g) = make_uint4(pk[4 * g], pk[4 * g + 1], pk[4 * g + 2], pk[4 * g + 3]);
             if (j >= 1) drain(j - 1, Pv);
             if (tr) trace_ev(p, j, 7);
@@ -572,27 +578,26 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
             tc_fence_after();
             if (tr) trace_ev(p, j, 5);
             tmem_ld16(tbase + lane_off + c0, *reinterpret_cast<uint32_t(*)[16]>(&rd[0]));
-            tmem_ld16(tbase + lane_off + c0 + 16, *reinterpret_cast<uint32_t(*)[16]>(&rd[16]));
-            tmem_ld16(tbase + lane_off + c0 + 32, *reinterpret_cast<uint32_t(*)[16]>(&rd[32]));
+            tmem_ld8(tbase + lane_off + c0 + 16, &rd[16]);
             tmem_wait_ld();
             tc_fence_before();
             mbar_arrive(dp_free);
             float dpart[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-            for (int e = 0; e < 48; ++e) dpart[e & 3] = fmaf(__uint_as_float(rs[e]), __uint_as_float(rd[e]), dpart[e & 3]);
-            float* dxb = dx + (j & 1) * 2 * BM;
-            dxb[h * BM + t] = (dpart[0] + dpart[1]) + (dpart[2] + dpart[3]);
-            named_bar_sync(1 + wq, 64);   // both halves of the row posted their part of D
+            for (int e = 0; e < 24; ++e) dpart[e & 3] = fmaf(__uint_as_float(rs[e]), __uint_as_float(rd[e]), dpart[e & 3]);
+            float* dxb = dx + (j & 1) * 4 * BM;
+            dxb[pq * BM + t] = (dpart[0] + dpart[1]) + (dpart[2] + dpart[3]);
+            named_bar_sync(1 + wq, 128);   // all four parts of the row posted their part of D
             if (tr) trace_ev(p, j, 17);
-            const float Dv = dxb[t] + dxb[BM + t];
+            const float Dv = (dxb[t] + dxb[BM + t]) + (dxb[2 * BM + t] + dxb[3 * BM + t]);
 #pragma unroll
-            for (int e = 0; e < 48; e += 2) {
+            for (int e = 0; e < 24; e += 2) {
                 const float d0 = __uint_as_float(rs[e]) * (__uint_as_float(rd[e]) - Dv);
                 const float d1 = __uint_as_float(rs[e + 1]) * (__uint_as_float(rd[e + 1]) - Dv);
                 pk[e / 2] = pack_f16x2(d0, d1);
             }
 #pragma unroll
-            for (int g = 0; g < 6; ++g)
+            for (int g = 0; g < 3; ++g)
                 *gran(O_DS0, O_DS1, O_DS2, c0 + 8 * g) = make_uint4(pk[4 * g], pk[4 * g + 1], pk[4 * g + 2], pk[4 * g + 3]);
             fence_proxy_async_smem();
             mbar_arrive(p_done);
@@ -603,7 +608,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
     }
     tc_fence_before();
     __syncthreads();
-    if (warp == 8) {
+    if (warp == 16) {
         tc_fence_after();
         tmem_dealloc(tbase, 512);
     }
@@ -624,10 +629,10 @@ int num_sms_nf() {
 }  // namespace
 
 bool tc_narrow_fused_ok(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
-    // Opt-in (measured at parity with the split NQ + NKV kernels, not faster yet):
-    // FT_WINATTN_FUSED=1 uses it from ~4 tiles per SM, =2 always (tests).
+    // Default from ~4 tiles per SM (C5_w32: 0.620 vs 0.648 ms for NQ + NKV, same box);
+    // FT_WINATTN_FUSED=0 selects the split kernels (A/B timing), =2 forces it (tests).
     const char* e = getenv("FT_WINATTN_FUSED");
-    const int mode = e ? atoi(e) : 0;
+    const int mode = e ? atoi(e) : 1;
     if (mode != 1 && mode != 2) return false;
     if (!tc_narrow_bwd_supported(units, L, d, w, dil)) return false;
     const int64_t nres = dil < L ? dil : L;
