@@ -45,6 +45,8 @@ WORKLOADS = {
     "C5_w32": (1, 64, 32768, 64, 32, 1, "BASELINE configs[4] sweep corner, HBM-bound"),
     "C5_w256": (1, 64, 32768, 64, 256, 1, "BASELINE configs[4] sweep corner, ridge"),
     "C5_small": (1, 8, 4096, 64, 32, 1, "BASELINE configs[4] sweep corner, small"),
+    # per-head dilation in one call (ft_winattn_*_mixed): heads 0-1 dilation 4, heads 2-7 dilation 1
+    "C2a_mix": (1, 8, 10000, 512, 32, 4, "C2a with the artefact's mixed heads (0-1 dilated x4), one call", 2),
 }
 
 METRIC = "window-attn fwd+bwd tokens/s per GPU and % HBM roofline at 1/2/4/8 B200"
@@ -86,6 +88,36 @@ def kernel_bytes_per_row(kind: str, d: int, e: int) -> int:
 def step_bytes_per_row(d: int, e: int) -> int:
     """fwd 4de+4 plus bwd 8de+4 (the bwd figure counts reading o)."""
     return (4 * d * e + 4) + (8 * d * e + 4)
+
+
+def launch_table(ft, B, H, L, d, w, dil, code):
+    """[(kind, rows)] of the forward and backward launches of one call, in launch order, with the
+    rows each launch processes (launches cover residue groups of 8 -- 4 for the wide-window
+    kernels -- of the min(dil, L) residues)."""
+    path_f, nf = ft.plan(False, B, H, L, d, w, dil, code)
+    path_b, nb = ft.plan(True, B, H, L, d, w, dil, code)
+    rows = rows_of(B, H, L)
+    nres = min(dil, L)
+
+    def split(n_launch, res_per):
+        sizes = [min(res_per, nres - i) for i in range(0, nres, res_per)]
+        if len(sizes) != n_launch:   # SIMT kernels and anything else: every launch sees all rows
+            return [rows] * n_launch
+        return [rows * sz / nres for sz in sizes]
+
+    res = 8 if min(w, L) <= 64 else 4
+    fwd = [("fwd", r) for r in (split(nf, res) if path_f == ft.PATH_TC else [rows] * nf)]
+    groups = -(-nres // res)
+    if path_b == ft.PATH_TC and nb == groups and d == 64 and min(w, L) <= 32:
+        bwd = [("bwdF", r) for r in split(nb, 8)]        # fused d = 64 backward (tc_narrow_fused.cu)
+    elif path_b == ft.PATH_TC:
+        pre = nb % 2                                     # wide windows: optional rowdot pre-pass
+        g = (nb - pre) // 2
+        per = split(g, res)
+        bwd = [("rowdot", rows)] * pre + [("bwdA", r) for r in per] + [("bwdB", r) for r in per]
+    else:
+        bwd = [("bwdA", rows)] + [("bwdB", rows)] * (nb - 1)
+    return path_f, path_b, fwd, bwd
 
 
 # ----------------------------------------------------------------------------- clocks (NVML)
@@ -223,13 +255,15 @@ def main():
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
-    B, H, L, d, w, dil, desc = WORKLOADS[args.workload]
+    B, H, L, d, w, dil, desc = WORKLOADS[args.workload][:7]
+    hd = WORKLOADS[args.workload][7] if len(WORKLOADS[args.workload]) > 7 else None
     world = int(os.environ.get("WORLD_SIZE", "1"))
     shape = (B, H, L, d, w, dil)
     e = 2 if args.dtype == "bf16" else 4
     in_bytes = 4 * B * H * L * d * e
     cfg = {"workload": args.workload, "desc": desc, "batch_per_rank": B, "heads": H, "seq_len": L,
            "d": d, "w": w, "dilation": dil, "global_batch": B * world,
+           **({"dilated_heads": hd} if hd is not None else {}),
            "parallelism": f"dp{world} over (batch, head) units, no collective on the data path",
            "l2": ("inputs larger than L2" if in_bytes > L2_BYTES else "L2 flushed between steps") +
                  f" ({in_bytes / 2**20:.0f} MiB of q/k/v/dout vs {L2_BYTES / 2**20:.0f} MiB L2)"}
@@ -251,8 +285,17 @@ def main():
     ft.load_library()
     tdt = torch.bfloat16 if args.dtype == "bf16" else torch.float32
     code = ft.FT_BF16 if args.dtype == "bf16" else ft.FT_F32
-    path_f, nf = ft.plan(False, B, H, L, d, w, dil, code)
-    path_b, nb = ft.plan(True, B, H, L, d, w, dil, code)
+    if hd is None:
+        path_f, path_b, ltf, ltb = launch_table(ft, B, H, L, d, w, dil, code)
+    else:   # B = 1: the dilated head slice, then the rest (ft_winattn_*_mixed launch order)
+        assert B == 1
+        ltf, ltb = [], []
+        for nh, dl in ((hd, dil), (H - hd, 1)):
+            if nh:
+                path_f, path_b, f_, b_ = launch_table(ft, 1, nh, L, d, w, dl, code)
+                ltf += f_
+                ltb += b_
+    nf, nb = len(ltf), len(ltb)
 
     gen = torch.Generator(device=dev)
     gen.manual_seed(1234 + rank)
@@ -267,8 +310,8 @@ def main():
         flush = torch.empty(2 * L2_BYTES, device=dev, dtype=torch.uint8)
 
     def step():
-        ft.fwd(q, k, v, w, dil, out=out, lse=lse)
-        ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws)
+        ft.fwd(q, k, v, w, dil, out=out, lse=lse, dilated_heads=hd)
+        ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
 
     for _ in range(args.warmup):
         step()
@@ -292,9 +335,9 @@ def main():
             s0, fe, be, s1 = ev(), [ev() for _ in range(nf)], [ev() for _ in range(nb)], ev()
             s0.record(stream)
             with ft.profile_events(fe):
-                ft.fwd(q, k, v, w, dil, out=out, lse=lse)
+                ft.fwd(q, k, v, w, dil, out=out, lse=lse, dilated_heads=hd)
             with ft.profile_events(be):
-                ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws)
+                ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
             s1.record(stream)
             starts.append(s0); fevs.append(fe); bevs.append(be); ends.append(s1)
         torch.cuda.synchronize()
@@ -320,25 +363,14 @@ def main():
     hbm_peak, bf16_peak, sm_max, peak_src = load_peaks()
     rows = rows_of(B, H, L)
 
-    # dominant kernel roofline
-    kinds = {}
-    if path_f == ft.PATH_TC or path_f == ft.PATH_SIMT:
-        for i in range(nf):
-            kinds[f"fwd{i}"] = "fwd"
-    # backward launches: [rowdot,] bwdA x g, bwdB x g (g residue groups); the band and narrow
-    # kernels have no rowdot
-    # (the fused d = 64 backward, tc_narrow_fused.cu, is one launch per residue group)
-    groups = -(-min(dil, L) // 3)
-    if nb == groups and path_b == ft.PATH_TC and d == 64 and min(w, L) <= 32:
-        kinds.update({f"bwd{i}": "bwdF" for i in range(nb)})
-    else:
-        pre = nb % 2
-        ngrp = (nb - pre) // 2
-        kinds.update({f"bwd{i}": ("rowdot" if i < pre else "bwdA" if i < pre + ngrp else "bwdB") for i in range(nb)})
+    # dominant kernel roofline (kind and rows of every launch: launch_table)
+    kinds = {f"fwd{i}": kd for i, (kd, _) in enumerate(ltf)}
+    kinds.update({f"bwd{i}": kd for i, (kd, _) in enumerate(ltb)})
+    krows = {f"fwd{i}": r for i, (_, r) in enumerate(ltf)}
+    krows.update({f"bwd{i}": r for i, (_, r) in enumerate(ltb)})
     mean_k = {n: sum(x) / len(x) for n, x in kdur.items()}
     dom = max(mean_k, key=mean_k.get)
-    # rows processed per launch: all rows (fwd launches are per residue group)
-    rows_per_launch = rows if not dom.startswith("fwd") or nf == 1 else rows / nf
+    rows_per_launch = krows[dom]
     if args.dtype == "bf16":
         by = kernel_bytes_per_row(kinds[dom], d, e) * rows_per_launch
         ach = by / (mean_k[dom] / 1e3) / 1e9
@@ -407,8 +439,9 @@ def main():
                 s_cmp.wait_event(h2d_done[i])
                 if i >= 2:
                     s_cmp.wait_event(d2h_done[i - 2])   # set i%2's results were read back
-                ft.fwd(tq, tk, tv, w, dil, out=to, lse=tl)
-                ft.bwd(tq, tk, tv, to, tl, tg, w, dil, dq=tdq, dk=tdk, dv=tdv, workspace=tws)
+                ft.fwd(tq, tk, tv, w, dil, out=to, lse=tl, dilated_heads=hd)
+                ft.bwd(tq, tk, tv, to, tl, tg, w, dil, dq=tdq, dk=tdk, dv=tdv, workspace=tws,
+                       dilated_heads=hd)
                 cmp_done[i].record(s_cmp)
             with torch.cuda.stream(s_out):
                 s_out.wait_event(cmp_done[i])

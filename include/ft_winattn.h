@@ -17,7 +17,8 @@
  *     out_i = sum_{j in N(i)} exp(s_ij - lse_i) v_j
  *   backward  (the gradient program of PAPER.md:447-453, P recomputed from lse as in
  *              PAPER.md:489-497 "selective materialization", reading A6):
- *     D_i = dout_i . out_i,  P_ij = exp(s_ij - lse_i),  dS_ij = P_ij (dout_i . v_j - D_i)
+ *     P_ij = exp(s_ij - lse_i),  D_i = sum_j P_ij (dout_i . v_j)  (= dout_i . out_i exactly;
+ *     the kernels form it from the recomputed band, reading R1),  dS_ij = P_ij (dout_i . v_j - D_i)
  *     dq_i = sum_j dS_ij k_j,  dk_j = sum_i dS_ij q_i,  dv_j = sum_i P_ij dout_i
  *
  * Layout (reading A9): q, k, v, out, dout, dq, dk, dv are contiguous row-major
@@ -90,7 +91,26 @@ ft_status ft_winattn_bwd(const void* q, const void* k, const void* v,
                          int64_t w, int64_t dilation, ft_dtype dtype,
                          void* workspace, size_t workspace_bytes, void* stream);
 
-/* Device workspace the backward needs (the per-row D_i = dout_i . out_i, fp32). */
+/* Per-head dilation (Longformer [8] and the FreeTensor artefact's mixed heads, PAPER.md:625;
+ * SURVEY.md §8(f) item 1, reading A4): heads [0, dilated_heads) of every batch element attend
+ * with `dilation`, heads [dilated_heads, heads) with dilation 1.  Arguments, layout, ownership
+ * and errors are those of ft_winattn_fwd / ft_winattn_bwd, plus FT_ERR_INVALID_VALUE when
+ * dilated_heads is outside [0, heads].  The workspace size is ft_winattn_bwd_workspace_bytes
+ * of the same shape.  Both head groups are enqueued on `stream` (one launch set per group when
+ * batch == 1 or one group is empty, else one per group and batch element). */
+ft_status ft_winattn_fwd_mixed(const void* q, const void* k, const void* v,
+                               void* out, float* lse,
+                               int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                               int64_t w, int64_t dilation, int64_t dilated_heads, ft_dtype dtype,
+                               void* stream);
+ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v,
+                               const void* out, const float* lse, const void* dout,
+                               void* dq, void* dk, void* dv,
+                               int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                               int64_t w, int64_t dilation, int64_t dilated_heads, ft_dtype dtype,
+                               void* workspace, size_t workspace_bytes, void* stream);
+
+/* Device workspace the backward needs (the per-row D_i, fp32). */
 size_t ft_winattn_bwd_workspace_bytes(int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
                                       int64_t w, int64_t dilation, ft_dtype dtype);
 

@@ -62,6 +62,10 @@ def load_library(build_if_missing: bool = False):
     lib.ft_winattn_fwd.restype = ctypes.c_int
     lib.ft_winattn_bwd.argtypes = [vp] * 9 + [i64] * 6 + [ctypes.c_int, vp, sz, vp]
     lib.ft_winattn_bwd.restype = ctypes.c_int
+    lib.ft_winattn_fwd_mixed.argtypes = [vp, vp, vp, vp, fp] + [i64] * 7 + [ctypes.c_int, vp]
+    lib.ft_winattn_fwd_mixed.restype = ctypes.c_int
+    lib.ft_winattn_bwd_mixed.argtypes = [vp] * 9 + [i64] * 7 + [ctypes.c_int, vp, sz, vp]
+    lib.ft_winattn_bwd_mixed.restype = ctypes.c_int
     lib.ft_winattn_bwd_workspace_bytes.argtypes = [i64] * 6 + [ctypes.c_int]
     lib.ft_winattn_bwd_workspace_bytes.restype = sz
     lib.ft_winattn_plan.argtypes = [ctypes.c_int] + [i64] * 6 + [ctypes.c_int,
@@ -138,17 +142,26 @@ def plan(is_bwd: bool, batch: int, heads: int, seq_len: int, d: int, w: int, dil
 
 
 def fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, w: int, dilation: int = 1,
-        out: torch.Tensor | None = None, lse: torch.Tensor | None = None):
-    """Forward: returns (out [B,H,L,d] in q.dtype, lse [B,H,L] fp32)."""
+        out: torch.Tensor | None = None, lse: torch.Tensor | None = None,
+        dilated_heads: int | None = None):
+    """Forward: returns (out [B,H,L,d] in q.dtype, lse [B,H,L] fp32).  With ``dilated_heads``
+    only heads [0, dilated_heads) use ``dilation`` and the rest dilation 1
+    (ft_winattn_fwd_mixed)."""
     _check_inputs(q, k, v)
     B, H, L, d = q.shape
     if out is None:
         out = torch.empty_like(q)
     if lse is None:
         lse = torch.empty((B, H, L), dtype=torch.float32, device=q.device)
-    _check(load_library().ft_winattn_fwd(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(),
-                                         lse.data_ptr(), B, H, L, d, int(w), int(dilation),
-                                         _dtype_code(q), _stream(q.device)))
+    lib = load_library()
+    if dilated_heads is None:
+        _check(lib.ft_winattn_fwd(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(),
+                                  lse.data_ptr(), B, H, L, d, int(w), int(dilation),
+                                  _dtype_code(q), _stream(q.device)))
+    else:
+        _check(lib.ft_winattn_fwd_mixed(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(),
+                                        lse.data_ptr(), B, H, L, d, int(w), int(dilation),
+                                        int(dilated_heads), _dtype_code(q), _stream(q.device)))
     return out, lse
 
 
@@ -159,8 +172,8 @@ def workspace_bytes(q: torch.Tensor, w: int, dilation: int = 1) -> int:
 
 
 def bwd(q, k, v, out, lse, dout, w: int, dilation: int = 1, dq=None, dk=None, dv=None,
-        workspace: torch.Tensor | None = None):
-    """Backward: returns (dq, dk, dv) in q.dtype."""
+        workspace: torch.Tensor | None = None, dilated_heads: int | None = None):
+    """Backward: returns (dq, dk, dv) in q.dtype (``dilated_heads``: see fwd)."""
     _check_inputs(q, k, v, out, dout)
     B, H, L, d = q.shape
     if lse.dtype != torch.float32 or not lse.is_contiguous() or lse.shape != (B, H, L):
@@ -171,11 +184,15 @@ def bwd(q, k, v, out, lse, dout, w: int, dilation: int = 1, dq=None, dk=None, dv
     wsb = workspace_bytes(q, w, dilation)
     if workspace is None or workspace.numel() * workspace.element_size() < wsb:
         workspace = torch.empty(max(wsb, 16), dtype=torch.uint8, device=q.device)
-    _check(load_library().ft_winattn_bwd(
-        q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), lse.data_ptr(), dout.data_ptr(),
-        dq.data_ptr(), dk.data_ptr(), dv.data_ptr(), B, H, L, d, int(w), int(dilation),
-        _dtype_code(q), workspace.data_ptr(), workspace.numel() * workspace.element_size(),
-        _stream(q.device)))
+    lib = load_library()
+    ptrs = (q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), lse.data_ptr(), dout.data_ptr(),
+            dq.data_ptr(), dk.data_ptr(), dv.data_ptr(), B, H, L, d, int(w), int(dilation))
+    tail = (_dtype_code(q), workspace.data_ptr(), workspace.numel() * workspace.element_size(),
+            _stream(q.device))
+    if dilated_heads is None:
+        _check(lib.ft_winattn_bwd(*ptrs, *tail))
+    else:
+        _check(lib.ft_winattn_bwd_mixed(*ptrs, int(dilated_heads), *tail))
     return dq, dk, dv
 
 
@@ -183,18 +200,20 @@ class WinAttn(torch.autograd.Function):
     """autograd wrapper: saves (q, k, v, out, lse); backward recomputes P from lse."""
 
     @staticmethod
-    def forward(ctx, q, k, v, w: int, dilation: int = 1):
-        out, lse = fwd(q.contiguous(), k.contiguous(), v.contiguous(), w, dilation)
+    def forward(ctx, q, k, v, w: int, dilation: int = 1, dilated_heads: int | None = None):
+        out, lse = fwd(q.contiguous(), k.contiguous(), v.contiguous(), w, dilation,
+                       dilated_heads=dilated_heads)
         ctx.save_for_backward(q, k, v, out, lse)
-        ctx.w, ctx.dilation = w, dilation
+        ctx.w, ctx.dilation, ctx.dilated_heads = w, dilation, dilated_heads
         return out
 
     @staticmethod
     def backward(ctx, dout):
         q, k, v, out, lse = ctx.saved_tensors
-        dq, dk, dv = bwd(q, k, v, out, lse, dout.contiguous(), ctx.w, ctx.dilation)
-        return dq, dk, dv, None, None
+        dq, dk, dv = bwd(q, k, v, out, lse, dout.contiguous(), ctx.w, ctx.dilation,
+                         dilated_heads=ctx.dilated_heads)
+        return dq, dk, dv, None, None, None
 
 
-def win_attn(q, k, v, w: int, dilation: int = 1):
-    return WinAttn.apply(q, k, v, w, dilation)
+def win_attn(q, k, v, w: int, dilation: int = 1, dilated_heads: int | None = None):
+    return WinAttn.apply(q, k, v, w, dilation, dilated_heads)

@@ -140,9 +140,13 @@ ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_
     return FT_OK;
 }
 
-ft_status ft_winattn_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
-                         int64_t batch, int64_t heads, int64_t seq_len, int64_t d, int64_t w,
-                         int64_t dilation, ft_dtype dtype, void* stream) {
+}  // extern "C"
+
+namespace {
+
+// Argument checks of the forward (before any launch).
+ft_status check_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t batch,
+                    int64_t heads, int64_t seq_len, int64_t d, int64_t w, int64_t dilation, ft_dtype dtype) {
     if (!q || !k || !v || !out || !lse) return FT_ERR_INVALID_VALUE;
     ft_status s = check_scalars(batch, heads, seq_len, d, w, dilation, dtype);
     if (s != FT_OK) return s;
@@ -157,12 +161,18 @@ ft_status ft_winattn_fwd(const void* q, const void* k, const void* v, void* out,
     for (const Span& x : in)
         if (overlap(x, so) || overlap(x, sl)) return FT_ERR_INVALID_VALUE;
     int path = 0;
-    s = choose_path(0, batch * heads, seq_len, d, w, dilation, dtype, &path);
-    if (s != FT_OK) return s;
+    return choose_path(0, batch * heads, seq_len, d, w, dilation, dtype, &path);
+}
 
+// Enqueue a validated forward.
+ft_status run_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t batch,
+                  int64_t heads, int64_t seq_len, int64_t d, int64_t w, int64_t dilation, ft_dtype dtype,
+                  void* stream) {
+    int path = 0;
+    ft_status s = choose_path(0, batch * heads, seq_len, d, w, dilation, dtype, &path);
+    if (s != FT_OK) return s;
     cudaStream_t st = (cudaStream_t)stream;
     cudaError_t e;
-    ftw::prof_reset();
     if (path == FT_PATH_TC) {
         int n = 0;
         e = ftw::tc_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, st, &n);
@@ -172,11 +182,10 @@ ft_status ft_winattn_fwd(const void* q, const void* k, const void* v, void* out,
     return e == cudaSuccess ? FT_OK : cuda_fail(e);
 }
 
-ft_status ft_winattn_bwd(const void* q, const void* k, const void* v, const void* out,
-                         const float* lse, const void* dout, void* dq, void* dk, void* dv,
-                         int64_t batch, int64_t heads, int64_t seq_len, int64_t d, int64_t w,
-                         int64_t dilation, ft_dtype dtype, void* workspace,
-                         size_t workspace_bytes, void* stream) {
+ft_status check_bwd(const void* q, const void* k, const void* v, const void* out, const float* lse,
+                    const void* dout, void* dq, void* dk, void* dv, int64_t batch, int64_t heads,
+                    int64_t seq_len, int64_t d, int64_t w, int64_t dilation, ft_dtype dtype,
+                    void* workspace, size_t workspace_bytes) {
     if (!q || !k || !v || !out || !lse || !dout || !dq || !dk || !dv) return FT_ERR_INVALID_VALUE;
     ft_status s = check_scalars(batch, heads, seq_len, d, w, dilation, dtype);
     if (s != FT_OK) return s;
@@ -202,13 +211,19 @@ ft_status ft_winattn_bwd(const void* q, const void* k, const void* v, const void
             if (outs[b].hi != outs[b].lo && overlap(outs[a], outs[b])) return FT_ERR_INVALID_VALUE;
     }
     int path = 0;
-    s = choose_path(1, batch * heads, seq_len, d, w, dilation, dtype, &path);
-    if (s != FT_OK) return s;
+    return choose_path(1, batch * heads, seq_len, d, w, dilation, dtype, &path);
+}
 
+ft_status run_bwd(const void* q, const void* k, const void* v, const void* out, const float* lse,
+                  const void* dout, void* dq, void* dk, void* dv, int64_t batch, int64_t heads,
+                  int64_t seq_len, int64_t d, int64_t w, int64_t dilation, ft_dtype dtype,
+                  void* workspace, void* stream) {
+    int path = 0;
+    ft_status s = choose_path(1, batch * heads, seq_len, d, w, dilation, dtype, &path);
+    if (s != FT_OK) return s;
     cudaStream_t st = (cudaStream_t)stream;
     float* Dws = (float*)workspace;
     cudaError_t e;
-    ftw::prof_reset();
     if (path == FT_PATH_TC) {
         int n = 0;
         e = ftw::tc_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w,
@@ -218,6 +233,104 @@ ft_status ft_winattn_bwd(const void* q, const void* k, const void* v, const void
                           dilation, dtype, st);
     }
     return e == cudaSuccess ? FT_OK : cuda_fail(e);
+}
+
+// Head groups of a per-head-dilation call: (first head, head count, dilation) per group, and
+// whether the groups are contiguous over the whole batch (batch == 1 or a single group).
+struct Group {
+    int64_t h0, nh, dil;
+};
+int mixed_groups(int64_t heads, int64_t dilation, int64_t hd, Group (&g)[2]) {
+    int n = 0;
+    if (hd > 0) g[n++] = {0, hd, dilation};
+    if (hd < heads) g[n++] = {hd, heads - hd, 1};
+    return n;
+}
+
+}  // namespace
+
+extern "C" {
+
+ft_status ft_winattn_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
+                         int64_t batch, int64_t heads, int64_t seq_len, int64_t d, int64_t w,
+                         int64_t dilation, ft_dtype dtype, void* stream) {
+    ft_status s = check_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype);
+    if (s != FT_OK) return s;
+    ftw::prof_reset();
+    return run_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype, stream);
+}
+
+ft_status ft_winattn_bwd(const void* q, const void* k, const void* v, const void* out,
+                         const float* lse, const void* dout, void* dq, void* dk, void* dv,
+                         int64_t batch, int64_t heads, int64_t seq_len, int64_t d, int64_t w,
+                         int64_t dilation, ft_dtype dtype, void* workspace,
+                         size_t workspace_bytes, void* stream) {
+    ft_status s = check_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, dilation,
+                            dtype, workspace, workspace_bytes);
+    if (s != FT_OK) return s;
+    ftw::prof_reset();
+    return run_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, dilation, dtype,
+                   workspace, stream);
+}
+
+ft_status ft_winattn_fwd_mixed(const void* q, const void* k, const void* v, void* out, float* lse,
+                               int64_t batch, int64_t heads, int64_t seq_len, int64_t d, int64_t w,
+                               int64_t dilation, int64_t dilated_heads, ft_dtype dtype, void* stream) {
+    if (dilated_heads < 0 || heads < 1 || dilated_heads > heads) return FT_ERR_INVALID_VALUE;
+    // every group's configuration is validated before anything is enqueued
+    ft_status s = check_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype);
+    if (s != FT_OK) return s;
+    s = check_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, 1, dtype);
+    if (s != FT_OK) return s;
+    Group g[2];
+    const int ng = mixed_groups(heads, dilation, dilated_heads, g);
+    const size_t e = elt_size(dtype);
+    const int64_t nb = ng == 1 ? 1 : batch;   // one group spans the whole batch contiguously
+    ftw::prof_reset();
+    for (int64_t b = 0; b < nb; ++b) {
+        for (int i = 0; i < ng; ++i) {
+            const int64_t B1 = ng == 1 ? batch : 1, H1 = ng == 1 ? heads : g[i].nh;
+            const int64_t row0 = (b * heads + g[i].h0) * seq_len;   // first (unit, row) of the slice
+            const size_t off = (size_t)row0 * d * e;
+            s = run_fwd((const char*)q + off, (const char*)k + off, (const char*)v + off, (char*)out + off,
+                        lse + row0, B1, H1, seq_len, d, w, g[i].dil, dtype, stream);
+            if (s != FT_OK) return s;
+        }
+    }
+    return FT_OK;
+}
+
+ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v, const void* out,
+                               const float* lse, const void* dout, void* dq, void* dk, void* dv,
+                               int64_t batch, int64_t heads, int64_t seq_len, int64_t d, int64_t w,
+                               int64_t dilation, int64_t dilated_heads, ft_dtype dtype, void* workspace,
+                               size_t workspace_bytes, void* stream) {
+    if (dilated_heads < 0 || heads < 1 || dilated_heads > heads) return FT_ERR_INVALID_VALUE;
+    ft_status s = check_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, dilation,
+                            dtype, workspace, workspace_bytes);
+    if (s != FT_OK) return s;
+    s = check_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, 1, dtype, workspace,
+                  workspace_bytes);
+    if (s != FT_OK) return s;
+    Group g[2];
+    const int ng = mixed_groups(heads, dilation, dilated_heads, g);
+    const size_t e = elt_size(dtype);
+    const int64_t nb = ng == 1 ? 1 : batch;
+    ftw::prof_reset();
+    for (int64_t b = 0; b < nb; ++b) {
+        for (int i = 0; i < ng; ++i) {
+            const int64_t B1 = ng == 1 ? batch : 1, H1 = ng == 1 ? heads : g[i].nh;
+            const int64_t row0 = (b * heads + g[i].h0) * seq_len;
+            const size_t off = (size_t)row0 * d * e;
+            // the workspace holds one fp32 per row: the slice's rows start at row0
+            s = run_bwd((const char*)q + off, (const char*)k + off, (const char*)v + off, (const char*)out + off,
+                        lse + row0, (const char*)dout + off, (char*)dq + off, (char*)dk + off, (char*)dv + off,
+                        B1, H1, seq_len, d, w, g[i].dil, dtype, workspace ? (char*)workspace + row0 * 4 : nullptr,
+                        stream);
+            if (s != FT_OK) return s;
+        }
+    }
+    return FT_OK;
 }
 
 }  // extern "C"

@@ -55,7 +55,7 @@ enum { FWD = 0, BWDQ = 1, BWDKV = 2 };
 
 constexpr int BM = 128;
 constexpr int KB = 64;                   // key-block rows of an output-GEMM B operand
-constexpr int RES_PER_LAUNCH = 3;        // residues per launch (8 tensor maps each)
+constexpr int RES_PER_LAUNCH = 8;        // residues per launch (8 tensor maps each; kernel params up to 32 KB)
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t ABYTES = BM * 128;    // one 128-row x 64-col bf16 slice (SW128)
 constexpr uint32_t OBOX = KB * 128;      // one 64-row x 64-col bf16 box

@@ -47,7 +47,7 @@ constexpr int D = 64;                        // head dim
 constexpr int NK = 192;                      // halo rows (keys m0-w .. m0-w+191), w <= 32
 constexpr int NSTAGE = 3;
 constexpr int NTHREADS = 320;
-constexpr int RES_PER_LAUNCH = 3;
+constexpr int RES_PER_LAUNCH = 8;
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t QBYTES = BM * D * 2;      // 16 KB
 constexpr uint32_t HBYTES = NK * D * 2;      // 24 KB

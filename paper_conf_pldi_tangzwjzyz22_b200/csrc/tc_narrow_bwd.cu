@@ -61,7 +61,7 @@ constexpr int D = 64;
 constexpr int NK = 192;
 constexpr int NSTAGE = 2;
 constexpr int NTHREADS = 352;
-constexpr int RES_PER_LAUNCH = 3;
+constexpr int RES_PER_LAUNCH = 8;
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t ABYTES = BM * D * 2;      // 16 KB: a 128-row tile
 constexpr uint32_t HBYTES = NK * D * 2;      // 24 KB: a 192-row halo

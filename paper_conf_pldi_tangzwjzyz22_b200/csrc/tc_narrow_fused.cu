@@ -70,7 +70,7 @@ constexpr int KB = 64;                       // rows per K / V ring block
 constexpr int RK = 5, RV = 4;                // ring slots
 constexpr int NTHREADS = 640;
 constexpr int NSM = 512;                     // softmax threads (warps 0-15)
-constexpr int RES_PER_LAUNCH = 3;
+constexpr int RES_PER_LAUNCH = 8;
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table");
 constexpr uint32_t TILE = BM * D * 2;        // 16 KB
 constexpr uint32_t BLK = KB * D * 2;         // 8 KB

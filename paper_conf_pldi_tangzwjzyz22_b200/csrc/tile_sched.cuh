@@ -12,7 +12,7 @@
 
 namespace ftw {
 
-constexpr int SCHED_MAX_RES = 4;   // >= every kernel's residues per launch (static_asserts)
+constexpr int SCHED_MAX_RES = 8;   // >= every kernel's residues per launch (static_asserts)
 
 struct SchedParams {
     int tiles;                 // row blocks per residue (of the longest residue of the launch)

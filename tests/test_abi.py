@@ -123,3 +123,22 @@ def test_status_strings(lib):
     for s in range(5):
         assert lib.ft_status_str(s)
     assert b"INVALID" in lib.ft_status_str(1)
+
+
+def test_mixed_validation(lib):
+    """ft_winattn_fwd_mixed / bwd_mixed: dilated_heads outside [0, heads] and every check of the
+    plain entry points fail before any launch (fake pointers are never dereferenced)."""
+    args = [P(i) for i in range(5)]
+    assert lib.ft_winattn_fwd_mixed(*args, 1, 4, 64, 64, 4, 2, 5, 1, None) == INVALID
+    assert lib.ft_winattn_fwd_mixed(*args, 1, 4, 64, 64, 4, 2, -1, 1, None) == INVALID
+    assert lib.ft_winattn_fwd_mixed(*args, 1, 4, 64, 64, 4, 0, 2, 1, None) == INVALID   # dilation 0
+    assert lib.ft_winattn_fwd_mixed(*args, 1, 4, 64, 24, 4, 2, 2, 1, None) == NOTSUP    # d = 24
+    bad = list(args)
+    bad[0] = P(0, 8)
+    assert lib.ft_winattn_fwd_mixed(*bad, 1, 4, 64, 64, 4, 2, 2, 1, None) == MISALIGNED
+    need = lib.ft_winattn_bwd_workspace_bytes(1, 4, 64, 64, 4, 2, 1)
+    b = [P(i) for i in range(9)]
+    assert lib.ft_winattn_bwd_mixed(*b, 1, 4, 64, 64, 4, 2, 7, 1, P(9), need, None) == INVALID
+    assert lib.ft_winattn_bwd_mixed(*b, 1, 4, 64, 64, 4, 2, 2, 1, P(9), 0, None) == INVALID
+    b[7] = b[6]                                                                          # dk aliases dq
+    assert lib.ft_winattn_bwd_mixed(*b, 1, 4, 64, 64, 4, 2, 2, 1, P(9), need, None) == INVALID

@@ -95,8 +95,10 @@ SMALL = [
     (1, 1, 260, 192, 20, 1),     # one 192-column output chunk
     (1, 1, 300, 320, 32, 2),     # chunks of 256 + 64 columns
     (1, 1, 140, 448, 64, 1),     # 256 + 192 columns, widest band (NK = 256)
-    (1, 2, 700, 64, 20, 5),      # 5 residues -> two launch groups
+    (1, 2, 700, 64, 20, 5),      # 5 residues
+    (1, 2, 1300, 64, 20, 11),    # 11 residues -> two launch groups (8 residues per launch)
     (2, 1, 900, 128, 3, 7),      # 7 residues, short windows
+    (1, 1, 1000, 128, 10, 9),    # 9 residues: two band launch groups
 ]
 SIMT_ONLY = [
     (1, 1, 300, 64, 100, 1),     # w > 64
@@ -339,6 +341,7 @@ FUSED = [
     (1, 1, 1, 64, 3, 1),
     (1, 64, 4096, 64, 32, 1),
     (3, 1, 1000, 64, 16, 1),
+    (1, 2, 1500, 64, 16, 10),    # two launch groups
 ]
 
 
@@ -347,5 +350,38 @@ def test_narrow_fused_bwd(ft, shape):
     sh = WinAttnShape(*shape)
     with _env(FT_WINATTN_FUSED="2"):
         p, n = ft.plan(True, sh.batch, sh.heads, sh.seq_len, sh.d, sh.w, sh.dilation, 1)
-        assert p == ft.PATH_TC and n == (min(sh.dilation, sh.seq_len) + 2) // 3
+        assert p == ft.PATH_TC and n == (min(sh.dilation, sh.seq_len) + 7) // 8
         run_case(ft, sh, "bf16", None, seed=6)
+
+
+# Per-head dilation (ft_winattn_fwd_mixed / bwd_mixed): heads
+# [0, hd) with dilation, the rest with 1 -- against the oracle run on each head slice.
+MIXED = [
+    (1, 4, 700, 64, 20, 4, 2, "bf16"),     # C2a-mix-like: two dilated heads of four
+    (2, 3, 300, 64, 32, 3, 1, "bf16"),     # batch > 1: one launch set per group and batch
+    (1, 2, 500, 128, 16, 2, 2, "bf16"),    # every head dilated
+    (2, 2, 260, 64, 8, 5, 0, "bf16"),      # none dilated
+    (1, 3, 200, 32, 6, 2, 1, "f32"),       # SIMT path
+    (1, 4, 300, 512, 32, 4, 2, "bf16"),    # d = 512 band kernels
+]
+
+
+@pytest.mark.parametrize("case", MIXED, ids=lambda c: "x".join(map(str, c)))
+def test_mixed_dilation(ft, case):
+    B, H, L, d, w, dil, hd, dtype = case
+    sh = WinAttnShape(B, H, L, d, w, dil)
+    x = make_inputs(sh, 8, dtype)
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    out, lse = ft.fwd(q, k, v, w, dil, dilated_heads=hd)
+    dq, dk, dv = ft.bwd(q, k, v, out, lse, g, w, dil, dilated_heads=hd)
+    torch.cuda.synchronize()
+    parts = []
+    for h0, h1, dl in ((0, hd, dil), (hd, H, 1)):
+        if h1 > h0:
+            s = {n: x[n + "64"][:, h0:h1].copy() for n in ("q", "k", "v", "dout")}
+            ro, rl = oracle.fwd(s["q"], s["k"], s["v"], w, dl)
+            parts.append((h0, h1, ro, rl) + tuple(oracle.bwd(s["q"], s["k"], s["v"], ro, rl, s["dout"], w, dl)))
+    for h0, h1, ro, rl, rdq, rdk, rdv in parts:
+        for n, a, r in (("out", out, ro), ("lse", lse, rl), ("dq", dq, rdq), ("dk", dk, rdk), ("dv", dv, rdv)):
+            compare(f"{n}[{h0}:{h1}]", a[:, h0:h1].double().cpu().numpy(), r, dtype)
