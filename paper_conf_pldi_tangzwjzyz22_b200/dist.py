@@ -106,3 +106,135 @@ def sharded_fwd_bwd(q, k, v, dout, w: int, dilation: int = 1, shape=None, dtype=
     o, l_, a, b, c = got
     return (o.reshape(B, H, L, d), l_.reshape(B, H, L), a.reshape(B, H, L, d),
             b.reshape(B, H, L, d), c.reshape(B, H, L, d))
+
+
+# ------------------------------------------------------------------ sequence (context) parallel
+# when B*H is smaller than the number of GPUs, or L is very long, each
+# rank holds a contiguous slice of the SEQUENCE of every (batch, head) unit instead.  A query
+# row attends only to keys within h = w * dilation rows (reading A1/A4), so a rank
+# needs h halo rows of K and V from each neighbour -- one NCCL point-to-point exchange -- and,
+# in the backward, returns the dK / dV its queries produced for the neighbours' rows.
+#
+# The local call runs the ordinary single-GPU kernels on the extended slice [halo | own | halo]:
+#   forward : q halo rows are zero; their outputs are discarded.
+#   backward: q, out, dout of the halo rows are zero and their lse is 0, so P = 1 on their band
+#             but dP = dout . v = 0 and D = 0, hence dS = 0 and P^T dout = 0 -- halo queries add
+#             nothing to dK / dV, which therefore hold exactly the contributions of this rank's
+#             queries; the halo rows' dK / dV go back to their owners and are added there.
+
+
+def seq_bounds(L: int, world: int, rank: int) -> tuple[int, int]:
+    """Contiguous rows [lo, hi) of the sequence owned by `rank` (balanced to within one row)."""
+    return shard_bounds(L, world, rank)
+
+
+def _neighbour_exchange(send_left: torch.Tensor | None, send_right: torch.Tensor | None,
+                        recv_left_shape, recv_right_shape, group=None):
+    """Send `send_left` to rank-1 and `send_right` to rank+1; receive tensors of the given shapes
+    (None = no neighbour) from rank-1 and rank+1.  One batched set of P2P ops (NCCL send/recv
+    over NVLink on GPUs, gloo on CPU)."""
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    ops, rl, rr = [], None, None
+    ref = send_left if send_left is not None else send_right
+    if recv_left_shape is not None:
+        rl = torch.empty(recv_left_shape, dtype=ref.dtype, device=ref.device)
+        ops.append(dist.P2POp(dist.irecv, rl, rank - 1, group))
+    if recv_right_shape is not None:
+        rr = torch.empty(recv_right_shape, dtype=ref.dtype, device=ref.device)
+        ops.append(dist.P2POp(dist.irecv, rr, rank + 1, group))
+    if send_left is not None and rank > 0:
+        ops.append(dist.P2POp(dist.isend, send_left.contiguous(), rank - 1, group))
+    if send_right is not None and rank < world - 1:
+        ops.append(dist.P2POp(dist.isend, send_right.contiguous(), rank + 1, group))
+    if ops:
+        for r in dist.batch_isend_irecv(ops):
+            r.wait()
+    return rl, rr
+
+
+def _halos(L: int, w: int, dilation: int, group=None):
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    lo, hi = seq_bounds(L, world, rank)
+    h = min(w * dilation, L)
+    hl = min(h, lo)              # rows of rank-1 this rank needs
+    hr = min(h, L - hi)          # rows of rank+1
+    for r in (rank - 1, rank + 1):
+        if 0 <= r < world:
+            a, b = seq_bounds(L, world, r)
+            if b - a < min(h, L):
+                raise ValueError("context parallel needs every rank to own >= w*dilation rows")
+    return lo, hi, hl, hr
+
+
+def _extend(x: torch.Tensor, hl: int, hr: int, group=None, zero_halo: bool = False):
+    """[B, H, n, ...] local slice -> [B, H, hl + n + hr, ...] with the neighbours' rows (or zeros)."""
+    B, H, n = x.shape[:3]
+    tail = tuple(x.shape[3:])
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    if zero_halo:
+        left = x.new_zeros((B, H, hl) + tail)
+        right = x.new_zeros((B, H, hr) + tail)
+    else:
+        # my first rows are rank-1's right halo and my last rows rank+1's left halo; _halos
+        # guarantees every rank owns >= h rows, so both sides of each link agree on the size
+        send_l = x[:, :, :hl] if rank > 0 else None
+        send_r = x[:, :, n - hr:] if rank < world - 1 else None
+        left, right = _neighbour_exchange(send_l, send_r,
+                                          (B, H, hl) + tail if hl > 0 else None,
+                                          (B, H, hr) + tail if hr > 0 else None, group)
+        left = left if left is not None else x.new_zeros((B, H, 0) + tail)
+        right = right if right is not None else x.new_zeros((B, H, 0) + tail)
+    return torch.cat([left, x, right], dim=2).contiguous()
+
+
+def cp_fwd(q, k, v, w: int, dilation: int, L: int, fwd_fn: Callable | None = None, group=None):
+    """Context-parallel forward.  q, k, v: this rank's rows [lo, hi) of the [B, H, L, d] tensors
+    (seq_bounds).  Returns (out, lse) for those rows.  `fwd_fn(q, k, v, w, dil)` is the local
+    single-device forward (default: the CUDA library)."""
+    if fwd_fn is None:
+        from . import fwd as fwd_fn
+    lo, hi, hl, hr = _halos(L, w, dilation, group)
+    n = hi - lo
+    ke, ve = _extend(k, hl, hr, group), _extend(v, hl, hr, group)
+    qe = _extend(q, hl, hr, group, zero_halo=True)
+    out, lse = fwd_fn(qe, ke, ve, w, dilation)
+    return out[:, :, hl:hl + n].contiguous(), lse[:, :, hl:hl + n].contiguous()
+
+
+def cp_bwd(q, k, v, out, lse, dout, w: int, dilation: int, L: int, bwd_fn: Callable | None = None,
+           group=None):
+    """Context-parallel backward over this rank's rows; returns (dq, dk, dv) for them.  dK / dV
+    of the halo rows (this rank's queries' contributions to its neighbours' keys) are sent back
+    and added by their owners."""
+    if bwd_fn is None:
+        from . import bwd as bwd_fn
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    lo, hi, hl, hr = _halos(L, w, dilation, group)
+    n = hi - lo
+    ke, ve = _extend(k, hl, hr, group), _extend(v, hl, hr, group)
+    qe, oe, ge = (_extend(t, hl, hr, group, zero_halo=True) for t in (q, out, dout))
+    le = _extend(lse, hl, hr, group, zero_halo=True)
+    dqe, dke, dve = bwd_fn(qe, ke, ve, oe, le, ge, w, dilation)
+    dq = dqe[:, :, hl:hl + n].contiguous()
+    dk = dke[:, :, hl:hl + n].clone()
+    dv = dve[:, :, hl:hl + n].clone()
+    # halo parts back to their owners: my left halo rows are rank-1's last rows, the right
+    # halo rows rank+1's first rows
+    hkv_l = torch.cat([dke[:, :, :hl], dve[:, :, :hl]], dim=-1) if rank > 0 else None
+    hkv_r = torch.cat([dke[:, :, hl + n:], dve[:, :, hl + n:]], dim=-1) if rank < world - 1 else None
+    need_prev = hl      # my first rows = rank-1's right halo (same size, see _halos)
+    need_next = hr      # my last rows = rank+1's left halo
+    d2 = dk.shape[-1] * 2
+    B, H = dk.shape[:2]
+    from_prev, from_next = _neighbour_exchange(
+        hkv_l, hkv_r,
+        (B, H, need_prev, d2) if need_prev > 0 else None,
+        (B, H, need_next, d2) if need_next > 0 else None, group)
+    d = dk.shape[-1]
+    if from_prev is not None:   # rank-1's queries -> my first rows
+        dk[:, :, :need_prev] += from_prev[..., :d].to(dk.dtype)
+        dv[:, :, :need_prev] += from_prev[..., d:].to(dv.dtype)
+    if from_next is not None:   # rank+1's queries -> my last rows
+        dk[:, :, n - need_next:] += from_next[..., :d].to(dk.dtype)
+        dv[:, :, n - need_next:] += from_next[..., d:].to(dv.dtype)
+    return dq, dk, dv

@@ -3,8 +3,10 @@
 set -u
 cd "$(dirname "$0")/.."
 cat > /tmp/san_case.py <<'PY'
-import sys, torch
+import os, sys, torch
 sys.path.insert(0, ".")
+if len(sys.argv) > 1:   # "fused": the one-kernel d = 64 backward (tc_narrow_fused.cu) on every d = 64 case
+    os.environ["FT_WINATTN_FUSED"] = "2"
 import paper_conf_pldi_tangzwjzyz22_b200 as ft
 from synth import WinAttnShape, make_inputs
 dev = torch.device("cuda:0")
@@ -17,10 +19,19 @@ for shape, dt in [((1, 2, 300, 64, 32, 3), "bf16"), ((1, 4, 1500, 64, 32, 1), "b
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
     o, l = ft.fwd(q, k, v, s.w, s.dilation)
     ft.bwd(q, k, v, o, l, g, s.w, s.dilation)
+# per-head dilation (ft_winattn_*_mixed)
+s = WinAttnShape(1, 4, 400, 64, 16, 3)
+x = make_inputs(s, 0, "bf16")
+q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+o, l = ft.fwd(q, k, v, s.w, s.dilation, dilated_heads=2)
+ft.bwd(q, k, v, o, l, g, s.w, s.dilation, dilated_heads=2)
 torch.cuda.synchronize()
 print("cases ok")
 PY
-for tool in memcheck racecheck synccheck initcheck; do
-  echo "== $tool"
-  timeout 600 compute-sanitizer --tool $tool --kernel-name kns=tc_ --kernel-name kns=simt --print-limit 10 python /tmp/san_case.py 2>&1 | tail -4
+for variant in default fused; do
+  for tool in memcheck racecheck synccheck initcheck; do
+    echo "== $tool ($variant)"
+    timeout 600 compute-sanitizer --tool $tool --kernel-name kns=tc_ --kernel-name kns=simt --print-limit 10 \
+      python /tmp/san_case.py $([ $variant = fused ] && echo fused) 2>&1 | tail -4
+  done
 done
