@@ -385,7 +385,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 trace_ev(p, j, 0);
                 if (j >= 1) mbar_wait(dp_free, (j - 1) & 1);
                 const uint32_t qa = smem_u32(smem + OFF_QO + (j & 1) * QO);
+                trace_ev(p, j, 25);
                 mbar_wait(&convB[j & 1], (j >> 1) & 1);   // Q_j and its K blocks landed, fp16
+                trace_ev(p, j, 26);
                 tc_fence_after();
                 score(qa, kring, RK, I.bseq % RK, true);
                 mma_commit(&s_full[j & 1]);
@@ -393,8 +395,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 mbar_wait(s_free, j & 1);
                 trace_ev(p, j, 16);
                 for (int g = 0; g < 3; ++g) mbar_wait(&vfull[(I.bseq + g) % RV], ((I.bseq + g) / RV) & 1);
+                trace_ev(p, j, 23);
                 tc_fence_after();
                 score(qa + TILE, vring, RV, I.bseq % RV, false);
+                trace_ev(p, j, 24);
                 mma_commit(dp_full);
                 trace_ev(p, j, 3);
                 for (int g = 0; g < (cn ? 2 : 3); ++g) mma_commit(&vempty[(I.bseq + g) % RV]);

@@ -22,7 +22,8 @@ EV = ["mma iter start", "S(j) issued", "out(j) issued", "dP(j) issued", "sm s_fu
       "sm dp_full seen", "sm p_done", "sm drain(j-1) done", "prod QO(j) issued", "prod K(j) issued",
       "prod V(j) issued", "conv s_full seen", "out A mmas issued", "conv done", "out accfree ok",
       "out(j) conv ok", "mma s_free seen", "sm pair barrier", "out(j) p_done ok", "out dqfree ok",
-      "out mmas issued", "sm drain(j-1) dq ld", "sm drain(j-1) X ld"]
+      "out mmas issued", "sm drain(j-1) dq ld", "sm drain(j-1) X ld", "i1 vfull ok", "i1 dP mmas issued",
+      "i1 dp_free(j-1) ok", "i1 conv(j) ok"]
 
 
 def main():
