@@ -170,6 +170,15 @@ struct FCursor {
     }
 };
 
+// One arrival per softmax warp (the barriers count warps): 512 per-thread arrivals on one
+// mbarrier serialise in the shared-memory atomic unit and delay every other mbarrier / MMA
+// operation of the SM behind them.  Each lane has finished its own TMEM loads (wait::ld +
+// fence::before_thread_sync) or smem writes (fence.proxy.async) before the __syncwarp.
+__device__ __forceinline__ void warp_arrive(uint64_t* bar) {
+    __syncwarp();
+    if ((threadIdx.x & 31u) == 0) mbar_arrive(bar);
+}
+
 __device__ __forceinline__ float fast_exp2(float x) {
     float y;
     asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
@@ -198,7 +207,11 @@ __device__ __forceinline__ void store_rows16(uint16_t* t, int64_t rowbase, int d
 #pragma unroll
     for (int q = 0; q < 2; ++q) {
         const int row = row0 + 2 * pr + q;
+#ifdef FT_EXPERIMENT_NO_DRAIN_STORES   // A/B experiment only: drops the results
+        if (row < -1000000)
+#else
         if (row >= 0 && row < Lr)
+#endif
             *reinterpret_cast<uint4*>(t + (rowbase + (int64_t)row * dil) * D + 16 * pq + 8 * ch) =
                 make_uint4(c[4 * q], c[4 * q + 1], c[4 * q + 2], c[4 * q + 3]);
     }
@@ -268,16 +281,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 mbar_init(&s_full[i], 1);
                 mbar_init(&oq_full[i], 1);
                 mbar_init(&okv_full[i], 1);
-                mbar_init(&accfree[i], NSM);
-                mbar_init(&convB[i], 32);
+                mbar_init(&accfree[i], NSM / 32);
+                mbar_init(&convB[i], 1);
             }
             for (int i = 0; i < RK; ++i) { mbar_init(&kfull[i], 1); mbar_init(&kempty[i], 1); }
             for (int i = 0; i < RV; ++i) { mbar_init(&vfull[i], 1); mbar_init(&vempty[i], 1); }
-            mbar_init(s_free, NSM);
+            mbar_init(s_free, NSM / 32);
             mbar_init(dp_full, 1);
-            mbar_init(dp_free, NSM);
-            mbar_init(p_done, NSM);
-            mbar_init(dqfree, NSM);
+            mbar_init(dp_free, NSM / 32);
+            mbar_init(p_done, NSM / 32);
+            mbar_init(dqfree, NSM / 32);
             mbar_init(opfree, 2);
             fence_barrier_init();
             for (int i = 0; i < p.nr; ++i) {
@@ -339,7 +352,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 to_f16(blk, blk, BLK, lane);
             }
             fence_proxy_async_smem();
-            mbar_arrive(&convB[j & 1]);
+            warp_arrive(&convB[j & 1]);
             if (lane == 0) trace_ev(p, j, 13);
         }
     } else if (warp == 17 || warp == 19) {
@@ -383,18 +396,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 const bool hnext = nx.next(p, N);   // N = item j+1
                 const bool cn = hnext && N.cont;
                 trace_ev(p, j, 0);
-                if (j >= 1) mbar_wait(dp_free, (j - 1) & 1);
+                if (j >= 1) mbar_wait_spin(dp_free, (j - 1) & 1);
                 const uint32_t qa = smem_u32(smem + OFF_QO + (j & 1) * QO);
                 trace_ev(p, j, 25);
-                mbar_wait(&convB[j & 1], (j >> 1) & 1);   // Q_j and its K blocks landed, fp16
+                mbar_wait_spin(&convB[j & 1], (j >> 1) & 1);   // Q_j and its K blocks landed, fp16
                 trace_ev(p, j, 26);
                 tc_fence_after();
                 score(qa, kring, RK, I.bseq % RK, true);
                 mma_commit(&s_full[j & 1]);
                 trace_ev(p, j, 1);
-                mbar_wait(s_free, j & 1);
+                mbar_wait_spin(s_free, j & 1);
                 trace_ev(p, j, 16);
-                for (int g = 0; g < 3; ++g) mbar_wait(&vfull[(I.bseq + g) % RV], ((I.bseq + g) / RV) & 1);
+                for (int g = 0; g < 3; ++g) mbar_wait_spin(&vfull[(I.bseq + g) % RV], ((I.bseq + g) / RV) & 1);
                 trace_ev(p, j, 23);
                 tc_fence_after();
                 score(qa + TILE, vring, RV, I.bseq % RV, false);
@@ -404,10 +417,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 for (int g = 0; g < (cn ? 2 : 3); ++g) mma_commit(&vempty[(I.bseq + g) % RV]);
                 mma_commit(&qo_empty[j & 1]);
                 // dQ(j) = dS K_h: A = dS K-major atoms [dS0|Z], dS1, [Z|dS2]
-                mbar_wait(p_done, j & 1);
+                mbar_wait_spin(p_done, j & 1);
                 trace_ev(p, j, 15);
                 if (!I.warm) {
-                    if (dq_req >= 1) mbar_wait(dqfree, (dq_req - 1) & 1);
+                    if (dq_req >= 1) mbar_wait_spin(dqfree, (dq_req - 1) & 1);
                     tc_fence_after();
                     const uint32_t k2 = kring + ((I.bseq + 2) % RK) * BLK;
                     mma_ss_x4<2, 128>(tbase + T_DQ, sdesc_sw128(opsa + O_DS0, 16, 1024),
@@ -429,13 +442,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
             int x_req[2] = {0, 0}, x_wait[2] = {0, 0};
             auto wait_x = [&](int b) {
                 if (x_req[b] > x_wait[b]) {
-                    mbar_wait(&accfree[b], x_wait[b] & 1);
+                    mbar_wait_spin(&accfree[b], x_wait[b] & 1);
                     ++x_wait[b];
                 }
             };
             for (int i = 0; have; ++i) {
                 const FItem& X = I;
-                mbar_wait(p_done, i & 1);
+                mbar_wait_spin(p_done, i & 1);
                 trace_ev(p, i, 18);
                 const uint32_t qa = smem_u32(smem + OFF_QO + (i & 1) * QO), da = qa + TILE;
                 const int a = i & 1, b = a ^ 1;
@@ -506,7 +519,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 tmem_ld16(tbase + lane_off + T_DQ + 16u * pq, va);
                 tmem_wait_ld();
                 tc_fence_before();
-                mbar_arrive(dqfree);
+                warp_arrive(dqfree);
                 if (threadIdx.x == 0) trace_ev(p, i + 1, 21);
                 store_rows16(p.dq, X.rowbase, p.dil, X.m0 + 32 * wq, X.Lr, pq, lane, va);
                 mbar_wait(&okv_full[i & 1], (i >> 1) & 1);
@@ -516,7 +529,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 tmem_ld16(xa + 64u + 16u * pq, vb);
                 tmem_wait_ld();
                 tc_fence_before();
-                mbar_arrive(&accfree[i & 1]);
+                warp_arrive(&accfree[i & 1]);
                 if (threadIdx.x == 0) trace_ev(p, i + 1, 22);
                 store_rows16(p.dk, X.rowbase, p.dil, X.m0 - w + 32 * wq, X.Lr, pq, lane, va);
                 store_rows16(p.dv, X.rowbase, p.dil, X.m0 - w + 32 * wq, X.Lr, pq, lane, vb);
@@ -529,7 +542,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 tmem_ld16(xb + 64u + 16u * pq, vb);
                 tmem_wait_ld();
                 tc_fence_before();
-                mbar_arrive(&accfree[(i + 1) & 1]);
+                warp_arrive(&accfree[(i + 1) & 1]);
                 store_rows16(p.dk, X.rowbase, p.dil, X.m0 - w + BM + 32 * wq, X.Lr, pq, lane, va);
                 store_rows16(p.dv, X.rowbase, p.dil, X.m0 - w + BM + 32 * wq, X.Lr, pq, lane, vb);
             }
@@ -560,7 +573,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
             tmem_ld8(tbase + lane_off + c0 + 16, &rs[16]);
             tmem_wait_ld();
             tc_fence_before();
-            mbar_arrive(s_free);
+            warp_arrive(s_free);
             uint32_t pk[12];
 #pragma unroll
             for (int e = 0; e < 24; e += 2) {
@@ -585,7 +598,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
             tmem_ld8(tbase + lane_off + c0 + 16, &rd[16]);
             tmem_wait_ld();
             tc_fence_before();
-            mbar_arrive(dp_free);
+            warp_arrive(dp_free);
             float dpart[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
             for (int e = 0; e < 24; ++e) dpart[e & 3] = fmaf(__uint_as_float(rs[e]), __uint_as_float(rd[e]), dpart[e & 3]);
@@ -604,7 +617,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
             for (int g = 0; g < 3; ++g)
                 *gran(O_DS0, O_DS1, O_DS2, c0 + 8 * g) = make_uint4(pk[4 * g], pk[4 * g + 1], pk[4 * g + 2], pk[4 * g + 3]);
             fence_proxy_async_smem();
-            mbar_arrive(p_done);
+            warp_arrive(p_done);
             if (tr) trace_ev(p, j, 6);
             Pv = I;
         }
