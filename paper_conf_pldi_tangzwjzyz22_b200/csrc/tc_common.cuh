@@ -94,6 +94,15 @@ __device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
     }
 }
 
+// One arrival per warp on a barrier whose count is in warps: per-thread arrivals of 128-512
+// threads on one mbarrier serialise in the shared-memory atomic unit and delay the SM's other
+// barrier and MMA traffic (fused backward: 0.626 -> 0.593 ms).  Every lane must have completed
+// (and fenced) its own work before the call; the call must be warp-uniform.
+__device__ __forceinline__ void warp_arrive(uint64_t* bar) {
+    __syncwarp();
+    if ((threadIdx.x & 31u) == 0) mbar_arrive(bar);
+}
+
 // ------------------------------------------------------------------ fences / barriers
 __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");

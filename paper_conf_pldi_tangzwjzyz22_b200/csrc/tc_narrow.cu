@@ -106,9 +106,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
             }
             for (int b = 0; b < 2; ++b) {
                 mbar_init(&s_full[b], 1);
-                mbar_init(&p_full[b], 128);
+                mbar_init(&p_full[b], 4);
                 mbar_init(&o_full[b], 1);
-                mbar_init(&o_free[b], 128);
+                mbar_init(&o_free[b], 4);
             }
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
@@ -241,7 +241,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
             }
             tmem_wait_st();
             tc_fence_before();
-            mbar_arrive(&p_full[g]);
+            warp_arrive(&p_full[g]);
             const float l = (l4[0] + l4[1]) + (l4[2] + l4[3]);
             const int mrow = m0 + t;
             if (mrow < Lr)
@@ -256,7 +256,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
             tmem_ld32(tO + 32, ov[1]);
             tmem_wait_ld();
             tc_fence_before();
-            mbar_arrive(&o_free[g]);
+            warp_arrive(&o_free[g]);
             if (lane == 0) tma_store_wait_read<0>();
             __syncwarp();
 #pragma unroll

@@ -116,7 +116,7 @@ __device__ __forceinline__ void drain_store(uint32_t tacc, uint8_t* stg, const C
     tmem_ld32(tacc + 32, ov[1]);
     tmem_wait_ld();
     tc_fence_before();
-    mbar_arrive(freed);
+    warp_arrive(freed);
     if (lane == 0) tma_store_wait_read<0>();
     __syncwarp();
 #pragma unroll
@@ -168,11 +168,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 mbar_init(&empty[i], 1);
             }
             mbar_init(s_full, 1);
-            mbar_init(dp_free, 256);
-            mbar_init(p_done, 256 + 32);
+            mbar_init(dp_free, 8);
+            mbar_init(p_done, 8 + 1);
             for (int b = 0; b < 2; ++b) {
                 mbar_init(&acc_full[b], 1);
-                mbar_init(&acc_free[b], 256);
+                mbar_init(&acc_free[b], 8);
             }
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
@@ -229,7 +229,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 hb[i] = v4;
             }
             fence_proxy_async_smem();
-            mbar_arrive(p_done);
+            warp_arrive(p_done);
             if (lane == 0) trace_ev(p, j, 12);
         }
     } else if (warp == 9) {
@@ -392,7 +392,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 tmem_wait_ld();
                 if (threadIdx.x == 0) trace_ev(p, i, 16);
                 tc_fence_before();
-                mbar_arrive(&acc_free[b]);
+                warp_arrive(&acc_free[b]);
                 const int mrow = c.m0 + t;
                 if (mrow < c.Lr) {
                     uint4* dst = reinterpret_cast<uint4*>(p.o1 + (c.rowbase + (int64_t)mrow * p.dil) * D + 32 * h);
@@ -435,7 +435,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             tmem_ld16(tP + c0 + 32, *reinterpret_cast<uint32_t(*)[16]>(&rd[32]));
             tmem_wait_ld();
             tc_fence_before();
-            mbar_arrive(dp_free);
+            warp_arrive(dp_free);
             if (tr) trace_ev(p, j, 5);
             uint32_t pk[24], pk2[24];
             if (MODE == NQ) {
@@ -494,7 +494,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 tmem_wait_st();
             }
             tc_fence_before();
-            mbar_arrive(p_done);
+            warp_arrive(p_done);
             if (tr) trace_ev(p, j, 8);
             const St done = cs;
             have = cur.next(p.sc, T);

@@ -170,15 +170,6 @@ struct FCursor {
     }
 };
 
-// One arrival per softmax warp (the barriers count warps): 512 per-thread arrivals on one
-// mbarrier serialise in the shared-memory atomic unit and delay every other mbarrier / MMA
-// operation of the SM behind them.  Each lane has finished its own TMEM loads (wait::ld +
-// fence::before_thread_sync) or smem writes (fence.proxy.async) before the __syncwarp.
-__device__ __forceinline__ void warp_arrive(uint64_t* bar) {
-    __syncwarp();
-    if ((threadIdx.x & 31u) == 0) mbar_arrive(bar);
-}
-
 __device__ __forceinline__ float fast_exp2(float x) {
     float y;
     asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
