@@ -18,7 +18,7 @@ import os
 
 import torch
 
-__all__ = ["fwd", "bwd", "plan", "profile_events", "WinAttn", "win_attn", "lib_path", "load_library",
+__all__ = ["fwd", "bwd", "fwd_tape", "bwd_tape", "tape_bytes", "plan", "profile_events", "WinAttn", "win_attn", "lib_path", "load_library",
            "FT_F32", "FT_BF16", "PATH_SIMT", "PATH_TC", "FtError"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -66,6 +66,12 @@ def load_library(build_if_missing: bool = False):
     lib.ft_winattn_fwd_mixed.restype = ctypes.c_int
     lib.ft_winattn_bwd_mixed.argtypes = [vp] * 9 + [i64] * 7 + [ctypes.c_int, vp, sz, vp]
     lib.ft_winattn_bwd_mixed.restype = ctypes.c_int
+    lib.ft_winattn_tape_bytes.argtypes = [i64] * 4
+    lib.ft_winattn_tape_bytes.restype = sz
+    lib.ft_winattn_fwd_tape.argtypes = [vp, vp, vp, vp, fp, fp] + [i64] * 6 + [ctypes.c_int, vp]
+    lib.ft_winattn_fwd_tape.restype = ctypes.c_int
+    lib.ft_winattn_bwd_tape.argtypes = [vp] * 10 + [i64] * 6 + [ctypes.c_int, vp, sz, vp]
+    lib.ft_winattn_bwd_tape.restype = ctypes.c_int
     lib.ft_winattn_bwd_workspace_bytes.argtypes = [i64] * 6 + [ctypes.c_int]
     lib.ft_winattn_bwd_workspace_bytes.restype = sz
     lib.ft_winattn_plan.argtypes = [ctypes.c_int] + [i64] * 6 + [ctypes.c_int,
@@ -193,6 +199,42 @@ def bwd(q, k, v, out, lse, dout, w: int, dilation: int = 1, dq=None, dk=None, dv
         _check(lib.ft_winattn_bwd(*ptrs, *tail))
     else:
         _check(lib.ft_winattn_bwd_mixed(*ptrs, int(dilated_heads), *tail))
+    return dq, dk, dv
+
+
+def tape_bytes(q: torch.Tensor, w: int) -> int:
+    B, H, L, _ = q.shape
+    return int(load_library().ft_winattn_tape_bytes(B, H, L, int(w)))
+
+
+def fwd_tape(q, k, v, w: int, dilation: int = 1):
+    """Forward that also materializes the band scores (ft_winattn_fwd_tape; CUDA-core kernels).
+    Returns (out, lse, tape) with tape fp32 [B, H, L, 2*min(w, L)+1]."""
+    _check_inputs(q, k, v)
+    B, H, L, d = q.shape
+    out = torch.empty_like(q)
+    lse = torch.empty((B, H, L), dtype=torch.float32, device=q.device)
+    tape = torch.empty((B, H, L, 2 * min(int(w), L) + 1), dtype=torch.float32, device=q.device)
+    _check(load_library().ft_winattn_fwd_tape(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(),
+                                              lse.data_ptr(), tape.data_ptr(), B, H, L, d, int(w),
+                                              int(dilation), _dtype_code(q), _stream(q.device)))
+    return out, lse, tape
+
+
+def bwd_tape(q, k, v, out, lse, tape, dout, w: int, dilation: int = 1):
+    """Backward reading the materialized scores instead of recomputing them (ft_winattn_bwd_tape)."""
+    _check_inputs(q, k, v, out, dout)
+    B, H, L, d = q.shape
+    if tape.dtype != torch.float32 or not tape.is_contiguous() or \
+            tape.numel() * 4 < tape_bytes(q, w):
+        raise ValueError("tape must be the contiguous fp32 tensor fwd_tape returned")
+    dq, dk, dv = torch.empty_like(q), torch.empty_like(q), torch.empty_like(q)
+    wsb = workspace_bytes(q, w, dilation)
+    ws = torch.empty(max(wsb, 16), dtype=torch.uint8, device=q.device)
+    _check(load_library().ft_winattn_bwd_tape(
+        q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), lse.data_ptr(), tape.data_ptr(),
+        dout.data_ptr(), dq.data_ptr(), dk.data_ptr(), dv.data_ptr(), B, H, L, d, int(w), int(dilation),
+        _dtype_code(q), ws.data_ptr(), ws.numel(), _stream(q.device)))
     return dq, dk, dv
 
 

@@ -333,4 +333,39 @@ ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v, cons
     return FT_OK;
 }
 
+size_t ft_winattn_tape_bytes(int64_t batch, int64_t heads, int64_t seq_len, int64_t w) {
+    if (batch < 1 || heads < 1 || seq_len < 1 || w < 0) return 0;
+    const int64_t wc = w < seq_len ? w : seq_len;
+    return (size_t)(batch * heads * seq_len) * (size_t)(2 * wc + 1) * sizeof(float);
+}
+
+ft_status ft_winattn_fwd_tape(const void* q, const void* k, const void* v, void* out, float* lse,
+                              float* tape, int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                              int64_t w, int64_t dilation, ft_dtype dtype, void* stream) {
+    ft_status s = check_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype);
+    if (s != FT_OK) return s;
+    if (!tape) return FT_ERR_INVALID_VALUE;
+    if (!aligned16(tape)) return FT_ERR_MISALIGNED;
+    ftw::prof_reset();
+    const cudaError_t e = ftw::simt_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype,
+                                        (cudaStream_t)stream, tape);
+    return e == cudaSuccess ? FT_OK : cuda_fail(e);
+}
+
+ft_status ft_winattn_bwd_tape(const void* q, const void* k, const void* v, const void* out,
+                              const float* lse, const float* tape, const void* dout, void* dq, void* dk,
+                              void* dv, int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                              int64_t w, int64_t dilation, ft_dtype dtype, void* workspace,
+                              size_t workspace_bytes, void* stream) {
+    ft_status s = check_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, dilation,
+                            dtype, workspace, workspace_bytes);
+    if (s != FT_OK) return s;
+    if (!tape) return FT_ERR_INVALID_VALUE;
+    if (!aligned16(tape)) return FT_ERR_MISALIGNED;
+    ftw::prof_reset();
+    const cudaError_t e = ftw::simt_bwd(q, k, v, out, lse, dout, dq, dk, dv, (float*)workspace, batch,
+                                        heads, seq_len, d, w, dilation, dtype, (cudaStream_t)stream, tape);
+    return e == cudaSuccess ? FT_OK : cuda_fail(e);
+}
+
 }  // extern "C"

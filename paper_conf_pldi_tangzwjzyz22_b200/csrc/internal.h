@@ -42,13 +42,15 @@ inline Geo make_geo(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64
 inline int64_t geo_blocks(const Geo& g) { return g.units * g.nres * g.tiles; }
 
 // SIMT (CUDA-core) kernels -- simt.cu
+// tape (optional): the raw band scores s_ij, fp32 [B*H*L][2w+1] (w clamped to L); the forward
+// writes it and the backward reads it instead of recomputing q_i . k_j (ft_winattn_*_tape).
 cudaError_t simt_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
                      int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
-                     ft_dtype dt, cudaStream_t st);
+                     ft_dtype dt, cudaStream_t st, float* tape = nullptr);
 cudaError_t simt_bwd(const void* q, const void* k, const void* v, const void* out,
                      const float* lse, const void* dout, void* dq, void* dk, void* dv,
                      float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
-                     int64_t dil, ft_dtype dt, cudaStream_t st);
+                     int64_t dil, ft_dtype dt, cudaStream_t st, const float* tape = nullptr);
 int simt_fwd_launches();
 int simt_bwd_launches();
 

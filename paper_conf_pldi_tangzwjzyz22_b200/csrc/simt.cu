@@ -111,12 +111,15 @@ __device__ __forceinline__ float hsum16(float x) {
 }
 
 // ------------------------------------------------------------------------------ forward
+// tape (nullable): the raw band scores s_ij, fp32 [B*H*L][2w+1] indexed by the query's flat
+// row and k + w (residue-space offset k = m_j - m_i) -- the materialized `dot` of Fig. 8 that
+// the tape-based backward reads instead of recomputing it.
 template <typename Tin>
 __global__ void __launch_bounds__(NT) simt_fwd_kernel(const Tin* __restrict__ q,
                                                       const Tin* __restrict__ k,
                                                       const Tin* __restrict__ v,
                                                       Tin* __restrict__ out, float* __restrict__ lse,
-                                                      Geo g) {
+                                                      float* __restrict__ tape, Geo g) {
     constexpr int T = 64, RA = T / 16;
     extern __shared__ float smem[];
     float(*Qs)[SP] = reinterpret_cast<float(*)[SP]>(smem);
@@ -175,6 +178,8 @@ __global__ void __launch_bounds__(NT) simt_fwd_kernel(const Tin* __restrict__ q,
             for (int b = 0; b < 4; ++b) {
                 const int mk = c0 + tx + 16 * b;
                 const bool ok = (mk < kend) && (abs(mk - mq) <= w);
+                if (tape && ok && mq < Lr)
+                    tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)] = s[a][b];
                 s[a][b] = ok ? s[a][b] * LOG2E : -INFINITY;
                 cmax = fmaxf(cmax, s[a][b]);
             }
@@ -244,12 +249,15 @@ __global__ void __launch_bounds__(NT) simt_fwd_kernel(const Tin* __restrict__ q,
 // so one sweep over the band accumulates A_i = sum (P dP) k, B_i = sum P k and D_i, and
 // dq_i = A_i - D_i B_i at the end.  D is also written to the workspace for the key-major
 // kernel.
-template <typename Tin, int T>
+// TAPE: s_ij is read from the forward's tape instead of being recomputed as q_i . k_j, so the
+// score loop stages only dout and V (half its FMAs and shared-memory traffic).
+template <typename Tin, int T, bool TAPE>
 __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
                                                      const Tin* __restrict__ k,
                                                      const Tin* __restrict__ v,
                                                      const Tin* __restrict__ dout,
                                                      const float* __restrict__ lse,
+                                                     const float* __restrict__ tape,
                                                      float* __restrict__ Dws,
                                                      Tin* __restrict__ dq, Geo g) {
     constexpr int RA = T / 16;
@@ -287,23 +295,23 @@ __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
             for (int b = 0; b < 4; ++b) { s[a][b] = 0.f; dp[a][b] = 0.f; }
         for (int col0 = 0; col0 < d; col0 += DS) {
             __syncthreads();
-            load_slice<Tin, T>(Qs, q + tc.off, tc.rstride, m0, Lr, col0, d);
+            if (!TAPE) load_slice<Tin, T>(Qs, q + tc.off, tc.rstride, m0, Lr, col0, d);
             load_slice<Tin, T>(Gs, dout + tc.off, tc.rstride, m0, Lr, col0, d);
-            load_slice<Tin, C>(Ks, k + tc.off, tc.rstride, c0, kend, col0, d);
+            if (!TAPE) load_slice<Tin, C>(Ks, k + tc.off, tc.rstride, c0, kend, col0, d);
             load_slice<Tin, C>(Vs, v + tc.off, tc.rstride, c0, kend, col0, d);
             __syncthreads();
 #pragma unroll 4
             for (int p = 0; p < DS; ++p) {
                 float qa[RA], ga[RA], kb[4], vb[4];
 #pragma unroll
-                for (int a = 0; a < RA; ++a) { qa[a] = Qs[ty + 16 * a][p]; ga[a] = Gs[ty + 16 * a][p]; }
+                for (int a = 0; a < RA; ++a) { if (!TAPE) qa[a] = Qs[ty + 16 * a][p]; ga[a] = Gs[ty + 16 * a][p]; }
 #pragma unroll
-                for (int b = 0; b < 4; ++b) { kb[b] = Ks[tx + 16 * b][p]; vb[b] = Vs[tx + 16 * b][p]; }
+                for (int b = 0; b < 4; ++b) { if (!TAPE) kb[b] = Ks[tx + 16 * b][p]; vb[b] = Vs[tx + 16 * b][p]; }
 #pragma unroll
                 for (int a = 0; a < RA; ++a)
 #pragma unroll
                     for (int b = 0; b < 4; ++b) {
-                        s[a][b] = fmaf(qa[a], kb[b], s[a][b]);
+                        if (!TAPE) s[a][b] = fmaf(qa[a], kb[b], s[a][b]);
                         dp[a][b] = fmaf(ga[a], vb[b], dp[a][b]);
                     }
             }
@@ -314,7 +322,8 @@ __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
 #pragma unroll
             for (int b = 0; b < 4; ++b) {
                 const int mk = c0 + tx + 16 * b;
-                const bool ok = (mk < kend) && (abs(mk - mq) <= w);
+                const bool ok = (mk < kend) && (abs(mk - mq) <= w) && mq < Lr;
+                if (TAPE && ok) s[a][b] = tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)];
                 const float p = ok ? exp2f(s[a][b] * LOG2E - lse2[a]) : 0.f;
                 const float pd = p * dp[a][b];
                 Dacc[a] += pd;
@@ -372,12 +381,13 @@ __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
 // ------------------------------------------------------------------------------ backward: dk, dv
 // Key-major: for owned key rows j, dk_j = sum_i dS_ij q_i and dv_j = sum_i P_ij dout_i over
 // the queries i whose window contains j (the band is symmetric: |m_i - m_j| <= w).
-template <typename Tin, int T>
+template <typename Tin, int T, bool TAPE>
 __global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q,
                                                        const Tin* __restrict__ k,
                                                        const Tin* __restrict__ v,
                                                        const Tin* __restrict__ dout,
                                                        const float* __restrict__ lse,
+                                                       const float* __restrict__ tape,
                                                        const float* __restrict__ Dws,
                                                        Tin* __restrict__ dk, Tin* __restrict__ dv,
                                                        Geo g) {
@@ -417,23 +427,23 @@ __global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q
         }
         for (int col0 = 0; col0 < d; col0 += DS) {
             __syncthreads();
-            load_slice<Tin, T>(Ks, k + tc.off, tc.rstride, m0, Lr, col0, d);
+            if (!TAPE) load_slice<Tin, T>(Ks, k + tc.off, tc.rstride, m0, Lr, col0, d);
             load_slice<Tin, T>(Vs, v + tc.off, tc.rstride, m0, Lr, col0, d);
-            load_slice<Tin, C>(Qs, q + tc.off, tc.rstride, c0, qend, col0, d);
+            if (!TAPE) load_slice<Tin, C>(Qs, q + tc.off, tc.rstride, c0, qend, col0, d);
             load_slice<Tin, C>(Gs, dout + tc.off, tc.rstride, c0, qend, col0, d);
             __syncthreads();
 #pragma unroll 4
             for (int p = 0; p < DS; ++p) {
                 float ka[RA], va[RA], qb[4], gb[4];
 #pragma unroll
-                for (int a = 0; a < RA; ++a) { ka[a] = Ks[ty + 16 * a][p]; va[a] = Vs[ty + 16 * a][p]; }
+                for (int a = 0; a < RA; ++a) { if (!TAPE) ka[a] = Ks[ty + 16 * a][p]; va[a] = Vs[ty + 16 * a][p]; }
 #pragma unroll
-                for (int b = 0; b < 4; ++b) { qb[b] = Qs[tx + 16 * b][p]; gb[b] = Gs[tx + 16 * b][p]; }
+                for (int b = 0; b < 4; ++b) { if (!TAPE) qb[b] = Qs[tx + 16 * b][p]; gb[b] = Gs[tx + 16 * b][p]; }
 #pragma unroll
                 for (int a = 0; a < RA; ++a)
 #pragma unroll
                     for (int b = 0; b < 4; ++b) {
-                        s[a][b] = fmaf(ka[a], qb[b], s[a][b]);
+                        if (!TAPE) s[a][b] = fmaf(ka[a], qb[b], s[a][b]);
                         dp[a][b] = fmaf(va[a], gb[b], dp[a][b]);
                     }
             }
@@ -445,7 +455,8 @@ __global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q
             for (int b = 0; b < 4; ++b) {
                 const int qi = tx + 16 * b;
                 const int mq = c0 + qi;
-                const bool ok = (mq < qend) && (abs(mq - mk) <= w);
+                const bool ok = (mq < qend) && (abs(mq - mk) <= w) && mk < Lr;
+                if (TAPE && ok) s[a][b] = tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)];
                 const float p = ok ? exp2f(s[a][b] * LOG2E - qlse[qi]) : 0.f;
                 Ps[ty + 16 * a][qi] = p;
                 DSs[ty + 16 * a][qi] = p * (dp[a][b] - qD[qi]);
@@ -509,70 +520,70 @@ void set_smem_once(F* f, size_t bytes, std::once_flag& flag) {
 }
 
 template <typename Tin>
-cudaError_t fwd_impl(const void* q, const void* k, const void* v, void* out, float* lse,
+cudaError_t fwd_impl(const void* q, const void* k, const void* v, void* out, float* lse, float* tape,
                      int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                      cudaStream_t st) {
     static std::once_flag once;
     Geo g = make_geo(B, H, L, d, w, dil, 64);
     set_smem_once(simt_fwd_kernel<Tin>, fwd_smem(d), once);
     simt_fwd_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_smem(d), st>>>(
-        (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, g);
+        (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, tape, g);
+    prof_mark(st);
+    return cudaGetLastError();
+}
+
+template <typename Tin, int T, bool TAPE>
+cudaError_t bwd_launch(const void* q, const void* k, const void* v, const float* lse, const float* tape,
+                       const void* dout, void* dq, void* dk, void* dv, float* Dws, const Geo& g,
+                       cudaStream_t st) {
+    static std::once_flag o1, o2;
+    const int64_t d = g.d;
+    set_smem_once(simt_dq_kernel<Tin, T, TAPE>, dq_smem(T, d), o1);
+    simt_dq_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dq_smem(T, d), st>>>(
+        (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dq, g);
+    prof_mark(st);
+    cudaError_t e;
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    set_smem_once(simt_dkdv_kernel<Tin, T, TAPE>, dkdv_smem(T, d), o2);
+    simt_dkdv_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dkdv_smem(T, d), st>>>(
+        (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dk,
+        (Tin*)dv, g);
     prof_mark(st);
     return cudaGetLastError();
 }
 
 template <typename Tin>
 cudaError_t bwd_impl(const void* q, const void* k, const void* v, const void* out,
-                     const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
-                     int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
+                     const float* lse, const float* tape, const void* dout, void* dq, void* dk, void* dv,
+                     float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                      cudaStream_t st) {
     (void)out;   // D_i is recomputed exactly as sum_j P_ij dP_ij (see simt_dq_kernel)
-    static std::once_flag o1, o2, o3, o4;
-    cudaError_t e;
     const int T = d <= 256 ? 64 : 32;
     Geo g = make_geo(B, H, L, d, w, dil, T);
-    if (T == 64) {
-        set_smem_once(simt_dq_kernel<Tin, 64>, dq_smem(64, d), o1);
-        simt_dq_kernel<Tin, 64><<<(unsigned)geo_blocks(g), NT, dq_smem(64, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dq, g);
-    } else {
-        set_smem_once(simt_dq_kernel<Tin, 32>, dq_smem(32, d), o2);
-        simt_dq_kernel<Tin, 32><<<(unsigned)geo_blocks(g), NT, dq_smem(32, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dq, g);
+    if (tape) {
+        return T == 64 ? bwd_launch<Tin, 64, true>(q, k, v, lse, tape, dout, dq, dk, dv, Dws, g, st)
+                       : bwd_launch<Tin, 32, true>(q, k, v, lse, tape, dout, dq, dk, dv, Dws, g, st);
     }
-    prof_mark(st);
-    if ((e = cudaGetLastError()) != cudaSuccess) return e;
-    if (T == 64) {
-        set_smem_once(simt_dkdv_kernel<Tin, 64>, dkdv_smem(64, d), o3);
-        simt_dkdv_kernel<Tin, 64><<<(unsigned)geo_blocks(g), NT, dkdv_smem(64, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dk,
-            (Tin*)dv, g);
-    } else {
-        set_smem_once(simt_dkdv_kernel<Tin, 32>, dkdv_smem(32, d), o4);
-        simt_dkdv_kernel<Tin, 32><<<(unsigned)geo_blocks(g), NT, dkdv_smem(32, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, Dws, (Tin*)dk,
-            (Tin*)dv, g);
-    }
-    prof_mark(st);
-    return cudaGetLastError();
+    return T == 64 ? bwd_launch<Tin, 64, false>(q, k, v, lse, nullptr, dout, dq, dk, dv, Dws, g, st)
+                   : bwd_launch<Tin, 32, false>(q, k, v, lse, nullptr, dout, dq, dk, dv, Dws, g, st);
 }
 
 }  // namespace
 
 cudaError_t simt_fwd(const void* q, const void* k, const void* v, void* out, float* lse,
                      int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
-                     ft_dtype dt, cudaStream_t st) {
-    if (dt == FT_F32) return fwd_impl<float>(q, k, v, out, lse, B, H, L, d, w, dil, st);
-    return fwd_impl<__nv_bfloat16>(q, k, v, out, lse, B, H, L, d, w, dil, st);
+                     ft_dtype dt, cudaStream_t st, float* tape) {
+    if (dt == FT_F32) return fwd_impl<float>(q, k, v, out, lse, tape, B, H, L, d, w, dil, st);
+    return fwd_impl<__nv_bfloat16>(q, k, v, out, lse, tape, B, H, L, d, w, dil, st);
 }
 
 cudaError_t simt_bwd(const void* q, const void* k, const void* v, const void* out,
                      const float* lse, const void* dout, void* dq, void* dk, void* dv,
                      float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
-                     int64_t dil, ft_dtype dt, cudaStream_t st) {
+                     int64_t dil, ft_dtype dt, cudaStream_t st, const float* tape) {
     if (dt == FT_F32)
-        return bwd_impl<float>(q, k, v, out, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st);
-    return bwd_impl<__nv_bfloat16>(q, k, v, out, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st);
+        return bwd_impl<float>(q, k, v, out, lse, tape, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st);
+    return bwd_impl<__nv_bfloat16>(q, k, v, out, lse, tape, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st);
 }
 
 int simt_fwd_launches() { return 1; }

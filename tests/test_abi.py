@@ -142,3 +142,17 @@ def test_mixed_validation(lib):
     assert lib.ft_winattn_bwd_mixed(*b, 1, 4, 64, 64, 4, 2, 2, 1, P(9), 0, None) == INVALID
     b[7] = b[6]                                                                          # dk aliases dq
     assert lib.ft_winattn_bwd_mixed(*b, 1, 4, 64, 64, 4, 2, 2, 1, P(9), need, None) == INVALID
+
+
+def test_tape_validation(lib):
+    assert lib.ft_winattn_tape_bytes(2, 3, 100, 4) == 2 * 3 * 100 * 9 * 4
+    assert lib.ft_winattn_tape_bytes(1, 1, 10, 50) == 10 * 21 * 4      # w clamped to L
+    assert lib.ft_winattn_tape_bytes(0, 1, 10, 5) == 0
+    a = [P(i) for i in range(5)]
+    assert lib.ft_winattn_fwd_tape(*a, None, 1, 1, 64, 64, 4, 1, 1, None) == INVALID
+    assert lib.ft_winattn_fwd_tape(*a, P(5, 4), 1, 1, 64, 64, 4, 1, 1, None) == MISALIGNED
+    assert lib.ft_winattn_fwd_tape(*a, P(5), 1, 1, 64, 24, 4, 1, 1, None) == NOTSUP
+    need = lib.ft_winattn_bwd_workspace_bytes(1, 1, 64, 64, 4, 1, 1)
+    b = [P(i) for i in range(10)]
+    assert lib.ft_winattn_bwd_tape(*b[:5], None, *b[6:10], 1, 1, 64, 64, 4, 1, 1, P(11), need, None) == INVALID
+    assert lib.ft_winattn_bwd_tape(*b, 1, 1, 64, 64, 4, 1, 1, P(11), 0, None) == INVALID

@@ -385,3 +385,41 @@ def test_mixed_dilation(ft, case):
     for h0, h1, ro, rl, rdq, rdk, rdv in parts:
         for n, a, r in (("out", out, ro), ("lse", lse, rl), ("dq", dq, rdq), ("dk", dk, rdk), ("dv", dv, rdv)):
             compare(f"{n}[{h0}:{h1}]", a[:, h0:h1].double().cpu().numpy(), r, dtype)
+
+
+# Tape vs recompute (ft_winattn_fwd_tape / bwd_tape): the backward
+# reads the materialized band scores instead of recomputing them; same results as the oracle.
+TAPE = [
+    (1, 1, 64, 16, 4, 1, "f32"),
+    (1, 2, 300, 64, 32, 3, "f32"),
+    (2, 1, 257, 128, 17, 2, "bf16"),
+    (1, 1, 200, 512, 32, 1, "f32"),
+    (1, 1, 50, 64, 100, 1, "f32"),     # w >= L
+    (1, 1, 130, 64, 0, 1, "bf16"),     # w = 0
+]
+
+
+@pytest.mark.parametrize("case", TAPE, ids=lambda c: "x".join(map(str, c)))
+def test_tape_path(ft, case):
+    B, H, L, d, w, dil, dtype = case
+    sh = WinAttnShape(B, H, L, d, w, dil)
+    x = make_inputs(sh, 11, dtype)
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    out, lse, tape = ft.fwd_tape(q, k, v, w, dil)
+    dq, dk, dv = ft.bwd_tape(q, k, v, out, lse, tape, g, w, dil)
+    torch.cuda.synchronize()
+    ro, rl = oracle.fwd(x["q64"], x["k64"], x["v64"], w, dil)
+    rdq, rdk, rdv = oracle.bwd(x["q64"], x["k64"], x["v64"], ro, rl, x["dout64"], w, dil)
+    for n, a, r in (("out", out, ro), ("lse", lse, rl), ("dq", dq, rdq), ("dk", dk, rdk), ("dv", dv, rdv)):
+        compare(n, a.double().cpu().numpy(), r, dtype)
+    # the tape holds q_i . k_j of every in-sequence band entry (fp32 sums of the stored inputs)
+    qn, kn = x["q64"], x["k64"]
+    t = tape.cpu().numpy()
+    wc = min(w, L)
+    for i in (0, L // 2, L - 1):
+        for kk in range(-wc, wc + 1):
+            j = i + kk * dil
+            if 0 <= j < L:
+                ref = float((qn[0, 0, i] * kn[0, 0, j]).sum())
+                assert abs(t[0, 0, i, kk + wc] - ref) <= 1e-4 * max(1.0, abs(ref)) + 1e-5
