@@ -107,3 +107,42 @@ def make_inputs(shape: WinAttnShape, seed: int, dtype: str = "f32", q_scale: flo
         out[name] = t
         out[name + "64"] = x64
     return out
+
+
+# --------------------------------------------------------------------------- SubdivNet meshes
+def torus_mesh(nx: int, ny: int, shuffle_seed: int | None = None) -> np.ndarray:
+    """Face adjacency [2*nx*ny, 3] (int64) of a closed triangulated torus: an nx x ny grid of
+    quads, each split into two triangles, wrapping in both directions, so every face has exactly
+    three edge-adjacent faces -- the manifold meshes SubdivNet convolves over (PAPER.md
+    Section 2.2).  Triangle A of cell (x, y) borders B of the same cell, B of (x, y-1) and
+    B of (x-1, y); triangle B borders A of the same cell, A of (x, y+1) and A of (x+1, y).
+    With shuffle_seed, face ids are randomly permuted (an unordered mesh).  Pure data
+    generation: no arithmetic of the method."""
+    xs, ys = np.meshgrid(np.arange(nx), np.arange(ny), indexing="ij")
+    cell = lambda x, y: ((x % nx) * ny + (y % ny))  # noqa: E731
+    A = 2 * cell(xs, ys)
+    B = A + 1
+    adjA = np.stack([2 * cell(xs, ys) + 1, 2 * cell(xs, ys - 1) + 1, 2 * cell(xs - 1, ys) + 1], -1)
+    adjB = np.stack([2 * cell(xs, ys), 2 * cell(xs, ys + 1), 2 * cell(xs + 1, ys)], -1)
+    adj = np.empty((2 * nx * ny, 3), dtype=np.int64)
+    adj[A.reshape(-1)] = adjA.reshape(-1, 3)
+    adj[B.reshape(-1)] = adjB.reshape(-1, 3)
+    if shuffle_seed is not None:
+        perm = np.random.Generator(np.random.PCG64(shuffle_seed)).permutation(adj.shape[0])
+        inv = np.empty_like(perm)
+        inv[perm] = np.arange(perm.size)
+        adj = inv[adj[perm]]          # new face f = old face perm[f]
+    return adj
+
+
+def mesh_features(n_faces: int, n_feats: int, seed: int, dtype: str = "f32"):
+    """e and dy, i.i.d. U(-1, 1) drawn with PCG64(seed) in that order, rounded to the storage dtype;
+    returns dict with torch tensors 'e', 'dy' and their exact fp64 numpy copies 'e64', 'dy64'."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    out = {}
+    for name in ("e", "dy"):
+        x = rng.uniform(-1.0, 1.0, size=(n_faces, n_feats))
+        t, x64 = round_to(x, dtype)
+        out[name] = t
+        out[name + "64"] = x64
+    return out
