@@ -37,7 +37,7 @@ def nvcc() -> str:
 
 def _deps():
     return sorted(glob.glob(os.path.join(CSRC, "*.cuh")) + glob.glob(os.path.join(CSRC, "*.h")) +
-                  [os.path.join(INCLUDE, "ft_winattn.h")])
+                  glob.glob(os.path.join(INCLUDE, "*.h")))
 
 
 def _compile(src: str, obj: str, verbose_ptxas: bool) -> str:

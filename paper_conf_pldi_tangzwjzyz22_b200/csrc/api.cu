@@ -76,6 +76,7 @@ ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w
 }  // namespace
 
 namespace ftw {
+ft_status cuda_error(cudaError_t e) { return cuda_fail(e); }
 void prof_reset() { g_prof_i = 0; }
 void* trace_buffer(int mode) { return (mode >= 0 && mode < 3) ? g_trace[mode] : nullptr; }
 void prof_mark(cudaStream_t st) {

@@ -111,6 +111,9 @@ cudaError_t tc_narrow_fused_bwd(const void* q, const void* k, const void* v, con
                                 const void* dout, void* dq, void* dk, void* dv, int64_t B, int64_t H,
                                 int64_t L, int64_t w, int64_t dil, cudaStream_t st, int* launches);
 
+// FT_ERR_CUDA with the CUDA error text recorded for ft_status_str (api.cu)
+ft_status cuda_error(cudaError_t e);
+
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();
 void* trace_buffer(int kernel_mode);   // ft_winattn_debug_trace target for a kernel mode, or null

@@ -14,6 +14,8 @@ import paper_conf_pldi_tangzwjzyz22_b200 as ft
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 HEADER = os.path.join(ROOT, "include", "ft_winattn.h")
+HEADERS = [os.path.join(ROOT, "include", h) for h in sorted(os.listdir(os.path.join(ROOT, "include")))
+           if h.endswith(".h")]
 
 OK, INVALID, NOTSUP, MISALIGNED = 0, 1, 2, 3
 
@@ -24,7 +26,7 @@ def lib():
 
 
 def declared_symbols():
-    src = open(HEADER).read()
+    src = "\n".join(open(h).read() for h in HEADERS)
     return sorted(set(re.findall(r"^\S[^;()]*?\b(ft_\w+)\s*\(", src, flags=re.M)))
 
 
@@ -156,3 +158,27 @@ def test_tape_validation(lib):
     b = [P(i) for i in range(10)]
     assert lib.ft_winattn_bwd_tape(*b[:5], None, *b[6:10], 1, 1, 64, 64, 4, 1, 1, P(11), need, None) == INVALID
     assert lib.ft_winattn_bwd_tape(*b, 1, 1, 64, 64, 4, 1, 1, P(11), 0, None) == INVALID
+
+
+def test_subdiv_validation(lib):
+    """SubdivNet circular difference (include/ft_subdiv.h): argument checks before any launch."""
+    f = lib.ft_subdiv_circdiff_fwd
+    f.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64,
+                  ctypes.c_int, ctypes.c_void_p]
+    assert f(None, P(1), P(2), 100, 64, 0, None) == INVALID
+    assert f(P(0), P(1), P(2), 0, 64, 0, None) == INVALID
+    assert f(P(0), P(1), P(2), 100, 64, 5, None) == NOTSUP
+    assert f(P(0, 8), P(1), P(2), 100, 64, 0, None) == MISALIGNED
+    assert f(P(0), P(1, 2), P(2), 100, 64, 0, None) == MISALIGNED
+    assert f(P(0), P(1), P(0), 100, 64, 0, None) == INVALID           # y aliases e
+    b = lib.ft_subdiv_circdiff_bwd
+    b.argtypes = [ctypes.c_void_p] * 4 + [ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.c_void_p,
+                                          ctypes.c_size_t, ctypes.c_void_p]
+    lib.ft_subdiv_circdiff_bwd_workspace_bytes.restype = ctypes.c_size_t
+    lib.ft_subdiv_circdiff_bwd_workspace_bytes.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int]
+    assert lib.ft_subdiv_circdiff_bwd_workspace_bytes(100, 64, 0) == 0
+    need = lib.ft_subdiv_circdiff_bwd_workspace_bytes(100, 64, 1)
+    assert need >= 100 * 64 * 4
+    assert b(P(0), P(1), P(2), P(3), 100, 64, 1, P(4), 0, None) == INVALID        # workspace too small
+    assert b(P(0), P(1), P(2), P(2), 100, 64, 0, None, 0, None) == INVALID        # de aliases dy
+    assert b(P(0), P(1), P(2), P(3, 4), 100, 64, 0, None, 0, None) == MISALIGNED
