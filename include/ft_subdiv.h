@@ -19,9 +19,17 @@
  * [0, n_faces) (not checked; out-of-range indices are undefined behaviour).  All pointers are
  * DEVICE pointers.  Ownership, async and threading rules are those of ft_winattn.h: the caller
  * owns every buffer (including the workspace), work is enqueued on `stream`, and outputs are
- * fully overwritten.  The backward scatters into de with fp32 atomic adds (each face collects
- * the contributions of the ~3 faces that reference it), so its summation order, and for fp32 its
- * last bit, may vary between runs.
+ * fully overwritten.
+ *
+ * Backward, two algorithms:
+ *   symmetric = 1: adj is the edge adjacency of a closed manifold triangle mesh (f is in adj[g]
+ *     exactly when g is in adj[f], once each; not checked).  Then the faces whose y involves
+ *     e[f] are f's own neighbours, and de[f] is GATHERED from them: one writer per row, no
+ *     atomics, deterministic, no workspace (requires n_feats % 4 == 0 for FT_F32, % 8 for
+ *     FT_BF16; otherwise the scatter below runs).
+ *   symmetric = 0: any adjacency array.  Contributions are SCATTERED into an fp32 accumulator
+ *     (de itself for FT_F32, the workspace for FT_BF16) with atomic adds, so the summation order,
+ *     and for fp32 the last bit, may vary between runs.
  *
  * Errors (checked before any launch; on failure nothing is launched):
  *   FT_ERR_INVALID_VALUE  null pointer, n_faces or n_feats < 1, an output overlapping an input,
@@ -50,8 +58,8 @@ ft_status ft_subdiv_circdiff_fwd(const void* e, const int32_t* adj, void* y, int
 size_t ft_subdiv_circdiff_bwd_workspace_bytes(int64_t n_faces, int64_t n_feats, ft_dtype dtype);
 
 ft_status ft_subdiv_circdiff_bwd(const void* e, const int32_t* adj, const void* dy, void* de,
-                                 int64_t n_faces, int64_t n_feats, ft_dtype dtype, void* workspace,
-                                 size_t workspace_bytes, void* stream);
+                                 int64_t n_faces, int64_t n_feats, ft_dtype dtype, int symmetric,
+                                 void* workspace, size_t workspace_bytes, void* stream);
 
 #ifdef __cplusplus
 }

@@ -160,6 +160,52 @@ __global__ void __launch_bounds__(256) circdiff_bwd_scalar(const T* __restrict__
     }
 }
 
+// Gather backward for edge adjacencies of closed manifold meshes (f in adj[g] <=> g in adj[f],
+// once each): the faces whose circular difference involves e[f] are exactly f's neighbours g,
+// and f's terms in y[g] are the pairs (f, next) and (prev, f) of g's cyclic list, so
+//     de[f] = sum_{g in adj[f]} dy[g] * (sign(e[f] - e[next_g(f)]) + sign(e[f] - e[prev_g(f)]))
+// -- every de row has one writer: no atomics, no zeroing pass, deterministic.  The extra reads
+// (the neighbours' adjacency rows and second-ring features) are L2 hits on a well-ordered mesh.
+template <typename T>
+__global__ void __launch_bounds__(256) circdiff_bwd_gather(const T* __restrict__ e, const int32_t* __restrict__ adj,
+                                                           const T* __restrict__ dy, T* __restrict__ de,
+                                                           int64_t n_faces, int64_t n_feats) {
+    constexpr int N = V8<T>::N;
+    const int64_t nch = n_feats / N, total = n_faces * nch;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t f = idx / nch, c = (idx - f * nch) * N;
+        // three dependent phases, each with all its loads in flight: the neighbour ids, their
+        // adjacency rows, then the nine feature chunks (plus e[f])
+        int32_t g[3], b[3][3];
+#pragma unroll
+        for (int j = 0; j < 3; ++j) g[j] = __ldg(adj + 3 * f + j);
+#pragma unroll
+        for (int j = 0; j < 3; ++j)
+#pragma unroll
+            for (int r = 0; r < 3; ++r) b[j][r] = __ldg(adj + 3 * (int64_t)g[j] + r);
+        float xf[N], xn[3][N], xp[3][N], gg[3][N];
+        V8<T>::load(e + f * n_feats + c, xf);
+#pragma unroll
+        for (int j = 0; j < 3; ++j) {
+            const int32_t nxt = b[j][0] == f ? b[j][1] : (b[j][1] == f ? b[j][2] : b[j][0]);
+            const int32_t prv = b[j][0] == f ? b[j][2] : (b[j][1] == f ? b[j][0] : b[j][1]);
+            V8<T>::load(e + nxt * n_feats + c, xn[j]);
+            V8<T>::load(e + prv * n_feats + c, xp[j]);
+            V8<T>::load(dy + (int64_t)g[j] * n_feats + c, gg[j]);
+        }
+        float acc[N];
+#pragma unroll
+        for (int t = 0; t < N; ++t) {
+            float a = 0.f;
+#pragma unroll
+            for (int j = 0; j < 3; ++j) a = fmaf(gg[j][t], sgnf(xf[t] - xn[j][t]) + sgnf(xf[t] - xp[j][t]), a);
+            acc[t] = a;
+        }
+        V8<T>::store(de + f * n_feats + c, acc);
+    }
+}
+
 __global__ void __launch_bounds__(256) zero_f32(float4* __restrict__ p, int64_t n4, float* __restrict__ tail, int ntail) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x)
         p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -252,8 +298,8 @@ ft_status ft_subdiv_circdiff_fwd(const void* e, const int32_t* adj, void* y, int
 }
 
 ft_status ft_subdiv_circdiff_bwd(const void* e, const int32_t* adj, const void* dy, void* de, int64_t n_faces,
-                                 int64_t n_feats, ft_dtype dtype, void* workspace, size_t workspace_bytes,
-                                 void* stream) {
+                                 int64_t n_feats, ft_dtype dtype, int symmetric, void* workspace,
+                                 size_t workspace_bytes, void* stream) {
     if (!e || !adj || !dy || !de || n_faces < 1 || n_feats < 1) return FT_ERR_INVALID_VALUE;
     if (dtype != FT_F32 && dtype != FT_BF16) return FT_ERR_NOT_SUPPORTED;
     if ((double)n_faces * (double)n_feats >= 1099511627776.0) return FT_ERR_NOT_SUPPORTED;
@@ -274,6 +320,18 @@ ft_status ft_subdiv_circdiff_bwd(const void* e, const int32_t* adj, const void* 
     prof_reset();
     cudaStream_t st = (cudaStream_t)stream;
     cudaError_t err;
+    const int vec = dtype == FT_F32 ? 4 : 8;
+    if (symmetric && n_feats % vec == 0) {
+        if (dtype == FT_F32)
+            circdiff_bwd_gather<float><<<grid_for(n_faces * (n_feats / 4)), 256, 0, st>>>(
+                (const float*)e, adj, (const float*)dy, (float*)de, n_faces, n_feats);
+        else
+            circdiff_bwd_gather<__nv_bfloat16><<<grid_for(n_faces * (n_feats / 8)), 256, 0, st>>>(
+                (const __nv_bfloat16*)e, adj, (const __nv_bfloat16*)dy, (__nv_bfloat16*)de, n_faces, n_feats);
+        prof_mark(st);
+        err = cudaGetLastError();
+        return err == cudaSuccess ? FT_OK : cuda_error(err);
+    }
     if (dtype == FT_F32) {
         err = bwd_t<float>(e, adj, dy, (float*)de, n_faces, n_feats, st);
     } else {

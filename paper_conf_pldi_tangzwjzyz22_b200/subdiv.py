@@ -22,7 +22,8 @@ def _lib():
         vp, i64 = ctypes.c_void_p, ctypes.c_int64
         lib.ft_subdiv_circdiff_fwd.argtypes = [vp, vp, vp, i64, i64, ctypes.c_int, vp]
         lib.ft_subdiv_circdiff_fwd.restype = ctypes.c_int
-        lib.ft_subdiv_circdiff_bwd.argtypes = [vp] * 4 + [i64, i64, ctypes.c_int, vp, ctypes.c_size_t, vp]
+        lib.ft_subdiv_circdiff_bwd.argtypes = [vp] * 4 + [i64, i64, ctypes.c_int, ctypes.c_int, vp,
+                                                          ctypes.c_size_t, vp]
         lib.ft_subdiv_circdiff_bwd.restype = ctypes.c_int
         lib.ft_subdiv_circdiff_bwd_workspace_bytes.argtypes = [i64, i64, ctypes.c_int]
         lib.ft_subdiv_circdiff_bwd_workspace_bytes.restype = ctypes.c_size_t
@@ -57,7 +58,9 @@ def circdiff_fwd(e: torch.Tensor, adj: torch.Tensor, y: torch.Tensor | None = No
 
 
 def circdiff_bwd(e: torch.Tensor, adj: torch.Tensor, dy: torch.Tensor, de: torch.Tensor | None = None,
-                 workspace: torch.Tensor | None = None) -> torch.Tensor:
+                 workspace: torch.Tensor | None = None, symmetric: bool = False) -> torch.Tensor:
+    """de for the loss sum(y * dy).  symmetric=True: adj is a closed manifold mesh's edge
+    adjacency (gather kernel, deterministic); False: any adjacency (atomic scatter)."""
     _check_args(e, adj)
     if dy.shape != e.shape or dy.dtype != e.dtype or not dy.is_contiguous():
         raise ValueError("dy must match e")
@@ -70,22 +73,23 @@ def circdiff_bwd(e: torch.Tensor, adj: torch.Tensor, dy: torch.Tensor, de: torch
     wp = workspace.data_ptr() if need else None
     wb = workspace.numel() * workspace.element_size() if need else 0
     _check(lib.ft_subdiv_circdiff_bwd(e.data_ptr(), adj.data_ptr(), dy.data_ptr(), de.data_ptr(), n, f,
-                                      _code(e), wp, wb, _stream(e.device)))
+                                      _code(e), int(symmetric), wp, wb, _stream(e.device)))
     return de
 
 
 class CircDiff(torch.autograd.Function):
     @staticmethod
-    def forward(ctx, e, adj):
+    def forward(ctx, e, adj, symmetric: bool = False):
         e = e.contiguous()
         ctx.save_for_backward(e, adj)
+        ctx.symmetric = symmetric
         return circdiff_fwd(e, adj)
 
     @staticmethod
     def backward(ctx, dy):
         e, adj = ctx.saved_tensors
-        return circdiff_bwd(e, adj, dy.contiguous()), None
+        return circdiff_bwd(e, adj, dy.contiguous(), symmetric=ctx.symmetric), None, None
 
 
-def circdiff(e, adj):
-    return CircDiff.apply(e, adj)
+def circdiff(e, adj, symmetric: bool = False):
+    return CircDiff.apply(e, adj, symmetric)

@@ -172,13 +172,13 @@ def test_subdiv_validation(lib):
     assert f(P(0), P(1, 2), P(2), 100, 64, 0, None) == MISALIGNED
     assert f(P(0), P(1), P(0), 100, 64, 0, None) == INVALID           # y aliases e
     b = lib.ft_subdiv_circdiff_bwd
-    b.argtypes = [ctypes.c_void_p] * 4 + [ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.c_void_p,
-                                          ctypes.c_size_t, ctypes.c_void_p]
+    b.argtypes = [ctypes.c_void_p] * 4 + [ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.c_int,
+                                          ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p]
     lib.ft_subdiv_circdiff_bwd_workspace_bytes.restype = ctypes.c_size_t
     lib.ft_subdiv_circdiff_bwd_workspace_bytes.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int]
     assert lib.ft_subdiv_circdiff_bwd_workspace_bytes(100, 64, 0) == 0
     need = lib.ft_subdiv_circdiff_bwd_workspace_bytes(100, 64, 1)
     assert need >= 100 * 64 * 4
-    assert b(P(0), P(1), P(2), P(3), 100, 64, 1, P(4), 0, None) == INVALID        # workspace too small
-    assert b(P(0), P(1), P(2), P(2), 100, 64, 0, None, 0, None) == INVALID        # de aliases dy
-    assert b(P(0), P(1), P(2), P(3, 4), 100, 64, 0, None, 0, None) == MISALIGNED
+    assert b(P(0), P(1), P(2), P(3), 100, 64, 1, 0, P(4), 0, None) == INVALID     # workspace too small
+    assert b(P(0), P(1), P(2), P(2), 100, 64, 0, 0, None, 0, None) == INVALID     # de aliases dy
+    assert b(P(0), P(1), P(2), P(3, 4), 100, 64, 0, 1, None, 0, None) == MISALIGNED

@@ -25,14 +25,14 @@ def sd():
     return subdiv
 
 
-def _run(sd, nx, ny, f, dtype, shuffle, seed=0):
+def _run(sd, nx, ny, f, dtype, shuffle, seed=0, symmetric=False):
     adj = torus_mesh(nx, ny, shuffle)
     x = mesh_features(adj.shape[0], f, seed, dtype)
     dev = torch.device("cuda:0")
     e, dy = x["e"].to(dev), x["dy"].to(dev)
     a = torch.from_numpy(adj.astype(np.int32)).to(dev)
     y = sd.circdiff_fwd(e, a)
-    de = sd.circdiff_bwd(e, a, dy)
+    de = sd.circdiff_bwd(e, a, dy, symmetric=symmetric)
     torch.cuda.synchronize()
     compare("y", y.double().cpu().numpy(), osd.fwd(x["e64"], adj), dtype)
     compare("de", de.double().cpu().numpy(), osd.bwd(x["e64"], adj, x["dy64"]), dtype)
@@ -41,14 +41,26 @@ def _run(sd, nx, ny, f, dtype, shuffle, seed=0):
 @pytest.mark.parametrize("f", [13, 64, 128, 8, 4])
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
 @pytest.mark.parametrize("shuffle", [None, 3])
-def test_circdiff_parity(sd, f, dtype, shuffle):
-    _run(sd, 40, 30, f, dtype, shuffle)
+@pytest.mark.parametrize("symmetric", [False, True])
+def test_circdiff_parity(sd, f, dtype, shuffle, symmetric):
+    _run(sd, 40, 30, f, dtype, shuffle, symmetric=symmetric)
 
 
 def test_circdiff_tiny_and_full_size(sd):
     _run(sd, 2, 2, 3, "f32", None)                      # 8 faces
     _run(sd, 1024, 1024, 64, "bf16", None, seed=1)      # 2M faces, bench size
+    _run(sd, 1024, 1024, 64, "f32", None, seed=1, symmetric=True)
     _run(sd, 512, 512, 64, "f32", 5, seed=2)            # shuffled, 512K faces
+
+
+def test_circdiff_gather_is_deterministic(sd):
+    adj = torus_mesh(64, 64, 2)
+    x = mesh_features(adj.shape[0], 32, 6, "f32")
+    dev = torch.device("cuda:0")
+    e, dy = x["e"].to(dev), x["dy"].to(dev)
+    a = torch.from_numpy(adj.astype(np.int32)).to(dev)
+    r = [sd.circdiff_bwd(e, a, dy, symmetric=True) for _ in range(3)]
+    assert all(torch.equal(r[0], t) for t in r[1:])
 
 
 def test_circdiff_autograd(sd):
