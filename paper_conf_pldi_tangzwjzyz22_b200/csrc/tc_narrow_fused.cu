@@ -383,10 +383,37 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 }
             };
             int dq_req = 0;
-            for (int j = 0; have; ++j) {
+            // dQ(i) = dS K_h: A = dS K-major atoms [dS0|Z], dS1, [Z|dS2].  Issued after S(i+1), so
+            // the next tile's score GEMM runs while the softmax finishes tile i
+            auto dq_issue = [&](int i, const FItem& X, bool cn) {
+                mbar_wait_spin(p_done, i & 1);
+                trace_ev(p, i, 15);
+                if (!X.warm) {
+                    if (dq_req >= 1) mbar_wait_spin(dqfree, (dq_req - 1) & 1);
+                    tc_fence_after();
+                    const uint32_t k2 = kring + ((X.bseq + 2) % RK) * BLK;
+                    mma_ss_x4<2, 128>(tbase + T_DQ, sdesc_sw128(opsa + O_DS0, 16, 1024),
+                                      sdesc_sw128(kring + (X.bseq % RK) * BLK, 8192, 1024), idQ, 0);
+                    mma_ss_x4<2, 128>(tbase + T_DQ, sdesc_sw128(opsa + O_DS1, 16, 1024),
+                                      sdesc_sw128(kring + ((X.bseq + 1) % RK) * BLK, 8192, 1024), idQ, 1);
+                    mma_ss_x4<2, 128>(tbase + T_DQ, sdesc_sw128(opsa + O_Z, 16, 1024),
+                                      sdesc_sw128(k2, 8192, 1024), idQ, 1);
+                    ++dq_req;
+                }
+                mma_commit(&oq_full[i & 1]);
+                mma_commit(opfree);
+                for (int g = 0; g < (cn ? 2 : 3); ++g) mma_commit(&kempty[(X.bseq + g) % RK]);
+                trace_ev(p, i, 2);
+            };
+            FItem Pv;
+            int j = 0;
+            for (; have; ++j) {
                 const bool hnext = nx.next(p, N);   // N = item j+1
                 const bool cn = hnext && N.cont;
                 trace_ev(p, j, 0);
+                // a tile that does not continue the previous one loads three fresh K blocks, one
+                // of them into the slot the previous tile's dQ frees: its dQ must go first
+                if (j >= 1 && !I.cont) dq_issue(j - 1, Pv, false);
                 if (j >= 1) mbar_wait_spin(dp_free, (j - 1) & 1);
                 const uint32_t qa = smem_u32(smem + OFF_QO + (j & 1) * QO);
                 trace_ev(p, j, 25);
@@ -396,6 +423,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 score(qa, kring, RK, I.bseq % RK, true);
                 mma_commit(&s_full[j & 1]);
                 trace_ev(p, j, 1);
+                if (j >= 1 && I.cont) dq_issue(j - 1, Pv, true);
                 mbar_wait_spin(s_free, j & 1);
                 trace_ev(p, j, 16);
                 for (int g = 0; g < 3; ++g) mbar_wait_spin(&vfull[(I.bseq + g) % RV], ((I.bseq + g) / RV) & 1);
@@ -407,28 +435,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fused_kernel(const __gr
                 trace_ev(p, j, 3);
                 for (int g = 0; g < (cn ? 2 : 3); ++g) mma_commit(&vempty[(I.bseq + g) % RV]);
                 mma_commit(&qo_empty[j & 1]);
-                // dQ(j) = dS K_h: A = dS K-major atoms [dS0|Z], dS1, [Z|dS2]
-                mbar_wait_spin(p_done, j & 1);
-                trace_ev(p, j, 15);
-                if (!I.warm) {
-                    if (dq_req >= 1) mbar_wait_spin(dqfree, (dq_req - 1) & 1);
-                    tc_fence_after();
-                    const uint32_t k2 = kring + ((I.bseq + 2) % RK) * BLK;
-                    mma_ss_x4<2, 128>(tbase + T_DQ, sdesc_sw128(opsa + O_DS0, 16, 1024),
-                                      sdesc_sw128(kring + (I.bseq % RK) * BLK, 8192, 1024), idQ, 0);
-                    mma_ss_x4<2, 128>(tbase + T_DQ, sdesc_sw128(opsa + O_DS1, 16, 1024),
-                                      sdesc_sw128(kring + ((I.bseq + 1) % RK) * BLK, 8192, 1024), idQ, 1);
-                    mma_ss_x4<2, 128>(tbase + T_DQ, sdesc_sw128(opsa + O_Z, 16, 1024),
-                                      sdesc_sw128(k2, 8192, 1024), idQ, 1);
-                    ++dq_req;
-                }
-                mma_commit(&oq_full[j & 1]);
-                mma_commit(opfree);
-                for (int g = 0; g < (cn ? 2 : 3); ++g) mma_commit(&kempty[(I.bseq + g) % RK]);
-                trace_ev(p, j, 2);
+                Pv = I;
                 I = N;
                 have = hnext;
             }
+            if (j >= 1) dq_issue(j - 1, Pv, false);
         } else if (warp == 19 && lane == 0) {   // ----------------------------------- issuer 2
             int x_req[2] = {0, 0}, x_wait[2] = {0, 0};
             auto wait_x = [&](int b) {
