@@ -285,9 +285,17 @@ def main():
 
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    # FT_BENCH_ONE_GPU=1 (self-test of the multi-rank code path on a one-GPU box): every rank
+    # uses cuda:0 and the gloo backend (NCCL refuses two ranks on one device).  Not for timing.
+    one_gpu = os.environ.get("FT_BENCH_ONE_GPU") == "1"
+    if one_gpu:
+        local_rank = 0
     if world > 1:
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
     ft.load_library()
@@ -362,7 +370,7 @@ def main():
             kdur[n].append(prev.elapsed_time(e1))
             prev = e1
     if world > 1:
-        t = torch.tensor([elapsed_ms], device=dev, dtype=torch.float64)
+        t = torch.tensor([elapsed_ms], device="cpu" if one_gpu else dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         elapsed_ms = float(t.item())
 
@@ -461,7 +469,7 @@ def main():
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1)
         if world > 1:
-            t = torch.tensor([ems], device=dev, dtype=torch.float64)
+            t = torch.tensor([ems], device="cpu" if one_gpu else dev, dtype=torch.float64)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
         e2e = {"value": B * L * world * args.e2e_steps / (ems / 1e3), "unit": "tokens/s",
