@@ -238,11 +238,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             // by the issuers owning a chain of that GEMM (see the MMA issuers below).
             for (int i = 0; i < NST; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], p.two ? 2 : 1); }
             mbar_init(s_full, MODE != FWD && p.two ? 2 : 1);
-            mbar_init(p_full, 4);
+            mbar_init(p_full, 128);
             mbar_init(o_full, dual && p.two ? 2 : 1);
-            mbar_init(o_empty, 4);
+            mbar_init(o_empty, 128);
             mbar_init(p_free, 1);
-            for (int i = 0; i < 4; ++i) mbar_init(&p_blk[i], 4);
+            for (int i = 0; i < 4; ++i) mbar_init(&p_blk[i], 128);
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
                 const Maps& mp = p.maps[i];
@@ -538,7 +538,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 rowScale[(j % 3) * 128 + t] = 1.f / sum;
                 fence_proxy_async_smem();   // P (generic-proxy stores) -> tensor core (async proxy)
                 tc_fence_before();
-                warp_arrive(p_full);
+                mbar_arrive(p_full);
                 if (mrow < Lr) p.lse[rowbase + (int64_t)mrow * p.dil] = (mxs + log2f(sum)) * LN2;
             } else if (MODE == BWDQ) {
                 const float lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
@@ -561,7 +561,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     if (early && (c & 1)) {
                         tmem_wait_st();
                         tc_fence_before();
-                        warp_arrive(&p_blk[c >> 1]);
+                        mbar_arrive(&p_blk[c >> 1]);
                     }
                 };
                 for (int c = 0; c < nch; ++c) {   // pass 2: dS = P (dP - D) -> TMEM (bf16 hi/lo)
@@ -594,7 +594,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 }
                 tmem_wait_st();
                 tc_fence_before();
-                warp_arrive(p_full);
+                mbar_arrive(p_full);
                 if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
             } else {   // BWDKV: rows are keys, columns are halo queries
                 if (j > 0) mbar_wait(p_free, (j - 1) & 1);
@@ -630,7 +630,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 fence_proxy_async_smem();
                 tmem_wait_st();
                 tc_fence_before();
-                warp_arrive(p_full);
+                mbar_arrive(p_full);
             }
             if (t == 0) trace_ev(p, j, 7);
             ++j;
@@ -674,7 +674,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     tmem_wait_ld();
                     if (s0 + ns == nsl_c) {
                         tc_fence_before();
-                        warp_arrive(o_empty);
+                        mbar_arrive(o_empty);
                     }
 #pragma unroll
                     for (int h = 0; h < 2; ++h) {

@@ -25,13 +25,30 @@ x = make_inputs(s, 0, "bf16")
 q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
 o, l = ft.fwd(q, k, v, s.w, s.dilation, dilated_heads=2)
 ft.bwd(q, k, v, o, l, g, s.w, s.dilation, dilated_heads=2)
+# tape path (SIMT kernels with the materialized scores)
+s = WinAttnShape(1, 2, 300, 64, 20, 3)
+x = make_inputs(s, 0, "f32")
+q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+o, l, tp = ft.fwd_tape(q, k, v, s.w, s.dilation)
+ft.bwd_tape(q, k, v, o, l, tp, g, s.w, s.dilation)
+# SubdivNet circular difference: vector / scalar, gather / scatter, fp32 / bf16
+import numpy as np
+from paper_conf_pldi_tangzwjzyz22_b200 import subdiv
+from synth import mesh_features, torus_mesh
+adj = torch.from_numpy(torus_mesh(20, 15, 2).astype(np.int32)).to(dev)
+for f, dt in ((64, "f32"), (13, "f32"), (64, "bf16")):
+    m = mesh_features(adj.shape[0], f, 0, dt)
+    e, dy = m["e"].to(dev), m["dy"].to(dev)
+    subdiv.circdiff_fwd(e, adj)
+    subdiv.circdiff_bwd(e, adj, dy)
+    subdiv.circdiff_bwd(e, adj, dy, symmetric=True)
 torch.cuda.synchronize()
 print("cases ok")
 PY
 for variant in default fused; do
   for tool in memcheck racecheck synccheck initcheck; do
     echo "== $tool ($variant)"
-    timeout 600 compute-sanitizer --tool $tool --kernel-name kns=tc_ --kernel-name kns=simt --print-limit 10 \
+    timeout 600 compute-sanitizer --tool $tool --kernel-name kns=tc_ --kernel-name kns=simt --kernel-name kns=circdiff --kernel-name kns=f32_to_bf16 --kernel-name kns=zero_f32 --print-limit 10 \
       python /tmp/san_case.py $([ $variant = fused ] && echo fused) 2>&1 | tail -4
   done
 done
