@@ -59,6 +59,8 @@ CONFIGS = {
     "C5_small_w32": WinAttnShape(1, 8, 4096, 64, 32, 1),
     "C5_big_w32": WinAttnShape(1, 64, 32768, 64, 32, 1),
     "C5_big_w256": WinAttnShape(1, 64, 32768, 64, 256, 1),
+    # one unit of 2^21 rows: 21-bit row indices, 16384 tiles in one (unit, residue) problem
+    "long_2M": WinAttnShape(1, 1, 2097152, 64, 32, 3),
 }
 
 

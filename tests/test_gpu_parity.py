@@ -3,7 +3,8 @@ seeded inputs.  Run on a B200 with ``pytest -m gpu``.
 
 * element-by-element at sizes the oracle finishes in seconds, spanning several tiles and a
   ragged tail, for both kernel families (FT_WINATTN_PATH=simt|tc forces one);
-* sampled rows at BASELINE.json's full sizes (C2a, C2b, C4), in the launch configuration
+* sampled rows at BASELINE.json's full sizes (C2a, C2b, C4, C5 corners) and one 2^21-row
+  sequence, in the launch configuration
   bench.py times, against the oracle's per-row entry points;
 * edge cases: L=1, w=0, w >= L, dilation >= L, ragged tails, x16 logits.
 """
@@ -285,7 +286,8 @@ def _sample_rows(shape: WinAttnShape, n_mid: int, seed: int):
 
 @pytest.mark.parametrize("name,dtype", [("C2a", "bf16"), ("C2a", "f32"), ("C2a_dil", "bf16"),
                                         ("C2b", "bf16"), ("C4d2", "bf16"), ("C4d4", "bf16"),
-                                        ("C5_big_w32", "bf16")])
+                                        ("C5_big_w32", "bf16"), ("C5_big_w256", "bf16"),
+                                        ("long_2M", "bf16")])
 def test_full_size_sampled(ft, name, dtype):
     shape = CONFIGS[name]
     x = make_inputs(shape, 0, dtype)
