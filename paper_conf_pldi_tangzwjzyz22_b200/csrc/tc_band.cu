@@ -198,6 +198,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int NK = p.NK, nsl = p.nsl, w = p.w, NST = p.nst, d = p.d;
+    // Programmatic dependent launch (BWDQ -> BWDKV, launch_pdl): BWDKV CTAs may take the SMs
+    // BWDQ CTAs leave (its persistent CTAs finish 4 or 5 tiles apart) and stream their first
+    // tiles' q/k/v/dout -- inputs of the whole backward call, complete before BWDQ started --
+    // while BWDQ drains; only BWDKV's softmax warps, which read BWDQ's D, wait for it.
+    if (MODE == BWDQ) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const int nkb = NK / KB;
     const int ncw = (d + 255) / 256;            // output chunks
     // BWDKV with d <= 128: dV and dK accumulate side by side ([256, 256+d) and
@@ -491,6 +496,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
         uint32_t zero16[16];
 #pragma unroll
         for (int e = 0; e < 16; ++e) zero16[e] = 0u;
+        if (MODE == BWDKV) asm volatile("griddepcontrol.wait;" ::: "memory");   // D of BWDQ
         while (cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0;
             const int mrow = m0 + t;
@@ -727,6 +733,12 @@ void set_attr_once() {
     });
 }
 
+// FT_WINATTN_PDL=0 turns the programmatic dependent launch off (A/B timing)
+bool pdl_enabled() {
+    const char* e = getenv("FT_WINATTN_PDL");
+    return !(e && atoi(e) == 0);
+}
+
 int num_sms() {
     static int n = 0;
     static std::once_flag once;
@@ -797,7 +809,22 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         dim3 grid((unsigned)(total < num_sms() ? total : num_sms()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_smem_bytes<MODE>(NK) + (size_t)nst * slot_bytes(NK);
-        tc_band_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
+        if (MODE == BWDKV && r0 == 0 && pdl_enabled()) {
+            // BWDKV directly follows this call's last BWDQ launch on the stream
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = grid;
+            cfg.blockDim = dim3(NTHREADS);
+            cfg.dynamicSmemBytes = smem;
+            cfg.stream = st;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = at;
+            cfg.numAttrs = 1;
+            cudaLaunchKernelEx(&cfg, tc_band_kernel<MODE>, p);
+        } else {
+            tc_band_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
+        }
         prof_mark(st);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
