@@ -248,6 +248,41 @@ def run_reference(args, shape, cfg):
 
 
 # ----------------------------------------------------------------------------- GPU arm
+def scatter_gather_e2e(args, rank, world, dev, tdt, e, shape):
+    """N > 1: the north_star's end-to-end multi-GPU variant (dist.sharded_fwd_bwd).  Rank 0 owns
+    the full [B*N, H, L, d] tensors, scatters (batch, head) slabs with NCCL, every rank runs
+    fwd+bwd on its slab, and out / lse / dq / dk / dv are gathered back.  CUDA events between
+    barriers, max over ranks."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_pldi_tangzwjzyz22_b200.dist import sharded_fwd_bwd
+    B, H, L, d, w, dil = shape
+    full = [None] * 4
+    if rank == 0:
+        gen0 = torch.Generator(device=dev)
+        gen0.manual_seed(99)
+        full = [(torch.rand((B * world, H, L, d), device=dev, generator=gen0) * 2 - 1).to(tdt)
+                for _ in range(4)]
+    run = lambda: sharded_fwd_bwd(*full, w, dil, shape=(B * world, H, L, d), dtype=tdt, device=dev)  # noqa: E731
+    run()   # warm-up
+    torch.cuda.synchronize()
+    dist.barrier()
+    a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a0.record()
+    for _ in range(args.sg_steps):
+        run()
+    a1.record()
+    torch.cuda.synchronize()
+    t = torch.tensor([a0.elapsed_time(a1) / args.sg_steps], device=dev, dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    n_el = B * world * H * L * d
+    return {"value": B * world * L / (ms / 1e3), "unit": "tokens/s", "ms_per_step": ms,
+            "steps": args.sg_steps, "bytes_scattered": 4 * n_el * e,
+            "bytes_gathered": 4 * n_el * e + B * world * H * L * 4,
+            "what": "rank 0 scatters q/k/v/dout (NCCL), per-rank fwd+bwd, gathers out/lse/dq/dk/dv"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -260,6 +295,7 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work (cpu_baseline)")
     ap.add_argument("--ref-rows", type=int, default=0, help="oracle rows per reference step (0 = full L)")
     ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--sg-steps", type=int, default=3, help="N > 1: NCCL scatter/gather end-to-end steps")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -477,6 +513,18 @@ def main():
                "d2h_bytes_per_step": 4 * q.numel() * e + lse.numel() * 4,
                "steps": args.e2e_steps, "pipelined": "2 buffer sets; H2D / compute / D2H streams"}
 
+    # ---------------------------------------------------------------- N > 1: NCCL scatter / gather
+    # The north_star's end-to-end multi-GPU variant (dist.sharded_fwd_bwd): rank 0 owns the full
+    # [B*N, H, L, d] tensors, scatters (batch, head) slabs over NVLink, every rank runs fwd+bwd on
+    # its slab, and out / lse / dq / dk / dv are gathered back.  Timed with CUDA events between
+    # barriers, max over ranks.  Not in one_gpu self-test mode (gloo has no CUDA scatter).
+    sg = None
+    if world > 1 and not one_gpu and args.sg_steps > 0:
+        try:
+            sg = scatter_gather_e2e(args, rank, world, dev, tdt, e, (B, H, L, d, w, dil))
+        except Exception as ex:   # the main line must survive; report why this extra is missing
+            sg = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(shape, args.cpu_budget)
@@ -495,6 +543,7 @@ def main():
             "roofline": roof, "hbm_step": hbm_step,
             "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": args.steps * (nf + nb),
+            **({"e2e_nccl_scatter_gather": sg} if sg is not None else {}),
             "clocks": sampler.summary(),
         }
         print(json.dumps(line), flush=True)
