@@ -193,6 +193,16 @@ def oracle_sample(shape, units: int, rows_cap: int, seed: int = 0):
     return time.perf_counter() - t0, units, Ls
 
 
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def cpu_baseline(shape, budget_s: float = 15.0):
     """The oracle as it stands, on as many whole (batch, head) units of the workload as fit
     in ~budget_s seconds of CPU work (at least one unit), extrapolated per unit."""
@@ -210,6 +220,7 @@ def cpu_baseline(shape, budget_s: float = 15.0):
         reps += extra
     value = reps * (n * Ls / secs) / (B * H) * B
     return {"value": value, "unit": "tokens/s", "cores": oracle.num_threads(), "kind": "oracle",
+            "cpu_model": cpu_model(),
             "sample": f"fp64 oracle fwd+bwd on {n} of {B * H} (batch, head) units at full length "
                       f"{Ls}, {reps} pass(es); {secs:.2f} s of CPU work; tokens/s extrapolated "
                       f"linearly per unit",
@@ -452,6 +463,25 @@ def main():
     hbm_step = {"algorithmic_bytes_per_step": step_alg,
                 "achieved_gbs": step_alg / (elapsed_ms / args.steps / 1e3) / 1e9 / world,
                 "peak": hbm_peak, "frac": step_alg / (elapsed_ms / args.steps / 1e3) / 1e9 / world / hbm_peak}
+    # the step against every ceiling of SURVEY.md §8(d): HBM bytes, tensor (bf16) or FMA (fp32)
+    # flops (fwd 4 d n_i + bwd 8 d n_i per row), MUFU ex2 (n_i per row in each direction); the
+    # binding ceiling is the one with the largest lower-bound time
+    step_s = elapsed_ms / args.steps / 1e3
+    nsum = float(window_sizes(L, w, dil).sum()) * B * H
+    flops = 12.0 * d * nsum
+    exps = 2.0 * nsum
+    sm_mhz = sm_max
+    comp_peak = bf16_peak * 1e12 if args.dtype == "bf16" else 148 * 128 * 2 * sm_mhz * 1e6
+    mufu_peak = 148 * 16 * sm_mhz * 1e6
+    bounds = {"hbm": step_alg / world / (hbm_peak * 1e9), "tensor" if args.dtype == "bf16" else "fma": flops / comp_peak,
+              "mufu": exps / mufu_peak}
+    ceilings = {k: {"lower_bound_us": v * 1e6, "frac": v / step_s} for k, v in bounds.items()}
+    ceilings["binding"] = max(bounds, key=bounds.get)
+    ceilings["peaks"] = {"hbm_gbs": hbm_peak, "compute_tflops": comp_peak / 1e12, "mufu_gops": mufu_peak / 1e9,
+                         "note": "HBM and bf16 measured (MEASURED_PEAKS.json); FMA and MUFU derived from "
+                                 "148 SMs x 128 lanes x 2 / 16 ex2 per clock at sm_max_mhz"}
+    ceilings["step_ms"] = {"mean": elapsed_ms / args.steps, "min": min(step_ms),
+                           "median": sorted(step_ms)[len(step_ms) // 2]}
 
     # ---------------------------------------------------------------- e2e (pinned host buffers)
     # Every step copies its inputs host -> device, runs fwd + bwd through the public API and
@@ -540,7 +570,7 @@ def main():
             "paths": {"fwd": "tc" if path_f == ft.PATH_TC else "simt",
                       "bwd": "tc" if path_b == ft.PATH_TC else "simt"},
             "kernel_ms": {n: sum(x) / len(x) for n, x in kdur.items()},
-            "roofline": roof, "hbm_step": hbm_step,
+            "roofline": roof, "hbm_step": hbm_step, "ceilings": ceilings,
             "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": args.steps * (nf + nb),
             **({"e2e_nccl_scatter_gather": sg} if sg is not None else {}),
