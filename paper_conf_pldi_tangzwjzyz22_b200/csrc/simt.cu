@@ -15,6 +15,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include <mutex>
 
@@ -230,6 +231,243 @@ __global__ void __launch_bounds__(NT) simt_fwd_kernel(const Tin* __restrict__ q,
     if (tx == 0) {
 #pragma unroll
         for (int a = 0; a < RA; ++a) { rowM[ty + 16 * a] = mrow[a]; rowL[ty + 16 * a] = lrow[a]; }
+    }
+    __syncthreads();
+    const int nrows = min(T, Lr - m0);
+    for (int i = threadIdx.x; i < nrows * d; i += NT) {
+        const int row = i / d, col = i % d;
+        Vec<Tin>::store1(out + tc.off + (int64_t)(m0 + row) * tc.rstride + col, Os[i] / rowL[row]);
+    }
+    for (int row = threadIdx.x; row < nrows; row += NT)
+        lse[tc.row0 + (int64_t)(m0 + row) * g.dil] = (rowM[row] + log2f(rowL[row])) * LN2;
+}
+
+// ------------------------------------------------------------------------------ forward, v2
+// Same algorithm as simt_fwd_kernel, with the shared-memory traffic of the two micro-GEMMs cut
+// four-fold: Q and K slices are staged TRANSPOSED ([d column][row], rows padded to 68 floats) so
+// a thread's four rows (4ty..4ty+3) and four keys (4tx..4tx+3) are one 16-byte load each per
+// d column, and P is staged transposed ([key][row]) so the P.V loop reads a thread's four rows
+// of P with one 16-byte load and two V columns (2tx, 2tx+1) with one 8-byte load.  The scalar
+// version issued eight 4-byte loads per 16 FMAs and was bound by shared-memory instructions
+// (ncu: 34 % issue utilisation at one 8-warp CTA per SM).
+constexpr int TP = 64 + 4;     // padded row count of a transposed slice (16-byte aligned rows)
+constexpr int VSP = DS + 4;    // padded V slice row (16-byte aligned)
+
+template <typename Tin, int R>
+__device__ __forceinline__ void load_slice_t(float* dst, const Tin* __restrict__ base, int64_t rstride,
+                                             int mbase, int Lr, int col0, int d) {
+    constexpr int V = Vec<Tin>::N;
+    constexpr int NV = DS / V;
+    for (int idx = threadIdx.x; idx < R * NV; idx += NT) {
+        const int row = idx / NV, cv = idx % NV;
+        const int m = mbase + row, c = col0 + cv * V;
+        float vals[V];
+        if (m >= 0 && m < Lr && c < d) {
+            Vec<Tin>::load(base + (int64_t)m * rstride + c, vals);
+        } else {
+#pragma unroll
+            for (int e = 0; e < V; ++e) vals[e] = 0.f;
+        }
+#pragma unroll
+        for (int e = 0; e < V; ++e) dst[(cv * V + e) * TP + row] = vals[e];
+    }
+}
+
+template <typename Tin, int R>
+__device__ __forceinline__ void load_slice_v(float* dst, const Tin* __restrict__ base, int64_t rstride,
+                                             int mbase, int Lr, int col0, int d) {
+    constexpr int V = Vec<Tin>::N;
+    constexpr int NV = DS / V;
+    for (int idx = threadIdx.x; idx < R * NV; idx += NT) {
+        const int row = idx / NV, cv = idx % NV;
+        const int m = mbase + row, c = col0 + cv * V;
+        float vals[V];
+        if (m >= 0 && m < Lr && c < d) {
+            Vec<Tin>::load(base + (int64_t)m * rstride + c, vals);
+        } else {
+#pragma unroll
+            for (int e = 0; e < V; ++e) vals[e] = 0.f;
+        }
+#pragma unroll
+        for (int e = 0; e < V; e += 4)
+            *reinterpret_cast<float4*>(&dst[row * VSP + cv * V + e]) = make_float4(vals[e], vals[e + 1], vals[e + 2], vals[e + 3]);
+    }
+}
+
+// Register-staged slice loads for software pipelining: a thread fetches its share of slice
+// i+1 from HBM into registers while the CTA computes on slice i in shared memory, then stores it
+// after the barrier -- the global latency is hidden behind the micro-GEMM instead of being paid
+// by every slice (one 8-warp CTA per SM cannot hide it by occupancy).
+template <typename Tin, int R>
+struct SliceRegs {
+    static constexpr int V = Vec<Tin>::N, NV = DS / V, PER = (R * NV + NT - 1) / NT;
+    float vals[PER][V];
+    __device__ void fetch(const Tin* __restrict__ base, int64_t rstride, int mbase, int Lr, int col0, int d) {
+#pragma unroll
+        for (int it = 0; it < PER; ++it) {
+            const int idx = threadIdx.x + it * NT;
+            const int row = idx / NV, cv = idx % NV;
+            const int m = mbase + row, c = col0 + cv * V;
+            if (idx < R * NV && m >= 0 && m < Lr && c < d) {
+                Vec<Tin>::load(base + (int64_t)m * rstride + c, vals[it]);
+            } else {
+#pragma unroll
+                for (int e = 0; e < V; ++e) vals[it][e] = 0.f;
+            }
+        }
+    }
+    __device__ void store_t(float* dst) const {   // transposed: [col][row], rows padded to TP
+#pragma unroll
+        for (int it = 0; it < PER; ++it) {
+            const int idx = threadIdx.x + it * NT;
+            if (idx >= R * NV) break;
+            const int row = idx / NV, cv = idx % NV;
+#pragma unroll
+            for (int e = 0; e < V; ++e) dst[(cv * V + e) * TP + row] = vals[it][e];
+        }
+    }
+    __device__ void store_v(float* dst) const {   // row-major, rows padded to VSP
+#pragma unroll
+        for (int it = 0; it < PER; ++it) {
+            const int idx = threadIdx.x + it * NT;
+            if (idx >= R * NV) break;
+            const int row = idx / NV, cv = idx % NV;
+#pragma unroll
+            for (int e = 0; e < V; e += 4)
+                *reinterpret_cast<float4*>(&dst[row * VSP + cv * V + e]) =
+                    make_float4(vals[it][e], vals[it][e + 1], vals[it][e + 2], vals[it][e + 3]);
+        }
+    }
+};
+
+template <typename Tin>
+__global__ void __launch_bounds__(NT) simt_fwd_v2_kernel(const Tin* __restrict__ q,
+                                                         const Tin* __restrict__ k,
+                                                         const Tin* __restrict__ v,
+                                                         Tin* __restrict__ out, float* __restrict__ lse,
+                                                         float* __restrict__ tape, Geo g) {
+    constexpr int T = 64;
+    extern __shared__ float smem[];
+    float* Qt = smem;                 // [DS][TP]
+    float* Kt = Qt + DS * TP;         // [DS][TP]
+    float* Vs = Kt + DS * TP;         // [C][VSP]
+    float* Pt = Vs + C * VSP;         // [C][TP]   P transposed: key-major
+    float* Os = Pt + C * TP;          // [T][d]
+    float* rowM = Os + T * g.d;
+    float* rowL = rowM + T;
+
+    TileCoord tc;
+    if (!decode(g, tc)) return;
+    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
+    const Tin* Qb = q + tc.off;
+    const Tin* Kb = k + tc.off;
+    const Tin* Vb = v + tc.off;
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+
+    for (int i = threadIdx.x; i < T * d; i += NT) Os[i] = 0.f;
+    float mrow[4], lrow[4];
+#pragma unroll
+    for (int a = 0; a < 4; ++a) { mrow[a] = -INFINITY; lrow[a] = 0.f; }
+
+    const int kbeg = max(0, m0 - w);
+    const int kend = min(Lr, m0 + T + w);
+    for (int c0 = kbeg; c0 < kend; c0 += C) {
+        float s[4][4];
+#pragma unroll
+        for (int a = 0; a < 4; ++a)
+#pragma unroll
+            for (int b = 0; b < 4; ++b) s[a][b] = 0.f;
+        SliceRegs<Tin, T> rq;
+        SliceRegs<Tin, C> rk;
+        rq.fetch(Qb, tc.rstride, m0, Lr, 0, d);
+        rk.fetch(Kb, tc.rstride, c0, kend, 0, d);
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            rq.store_t(Qt);
+            rk.store_t(Kt);
+            __syncthreads();
+            if (col0 + DS < d) {   // next slice in flight during this one's micro-GEMM
+                rq.fetch(Qb, tc.rstride, m0, Lr, col0 + DS, d);
+                rk.fetch(Kb, tc.rstride, c0, kend, col0 + DS, d);
+            }
+#pragma unroll 8
+            for (int p = 0; p < DS; ++p) {
+                const float4 qa = *reinterpret_cast<const float4*>(&Qt[p * TP + 4 * ty]);
+                const float4 kb = *reinterpret_cast<const float4*>(&Kt[p * TP + 4 * tx]);
+                const float qv[4] = {qa.x, qa.y, qa.z, qa.w}, kv[4] = {kb.x, kb.y, kb.z, kb.w};
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) s[a][b] = fmaf(qv[a], kv[b], s[a][b]);
+            }
+        }
+        // band mask + online softmax (log2 domain); rows 4ty+a are shared by the 16 tx lanes
+        float alpha[4];
+        __syncthreads();   // the previous chunk's P.V reads of Pt are done
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            const int mq = m0 + 4 * ty + a;
+            float cmax = -INFINITY;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int mk = c0 + 4 * tx + b;
+                const bool ok = (mk < kend) && (abs(mk - mq) <= w);
+                if (tape && ok && mq < Lr)
+                    tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)] = s[a][b];
+                s[a][b] = ok ? s[a][b] * LOG2E : -INFINITY;
+                cmax = fmaxf(cmax, s[a][b]);
+            }
+            cmax = hmax16(cmax);
+            const float mnew = fmaxf(mrow[a], cmax);
+            alpha[a] = (mnew == -INFINITY) ? 1.f : exp2f(mrow[a] - mnew);
+            float sum = 0.f;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const float pv = (s[a][b] == -INFINITY) ? 0.f : exp2f(s[a][b] - mnew);
+                Pt[(4 * tx + b) * TP + 4 * ty + a] = pv;
+                sum += pv;
+            }
+            sum = hsum16(sum);
+            lrow[a] = lrow[a] * alpha[a] + sum;
+            mrow[a] = mnew;
+        }
+        // O = alpha * O + P V, 32 output columns per staged V slice
+        SliceRegs<Tin, C> rv;
+        rv.fetch(Vb, tc.rstride, c0, kend, 0, d);
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            rv.store_v(Vs);
+            __syncthreads();
+            if (col0 + DS < d) rv.fetch(Vb, tc.rstride, c0, kend, col0 + DS, d);
+            float acc[4][2];
+#pragma unroll
+            for (int a = 0; a < 4; ++a) { acc[a][0] = 0.f; acc[a][1] = 0.f; }
+#pragma unroll 8
+            for (int kk = 0; kk < C; ++kk) {
+                const float4 pv = *reinterpret_cast<const float4*>(&Pt[kk * TP + 4 * ty]);
+                const float2 vv = *reinterpret_cast<const float2*>(&Vs[kk * VSP + 2 * tx]);
+                const float pa[4] = {pv.x, pv.y, pv.z, pv.w};
+#pragma unroll
+                for (int a = 0; a < 4; ++a) {
+                    acc[a][0] = fmaf(pa[a], vv.x, acc[a][0]);
+                    acc[a][1] = fmaf(pa[a], vv.y, acc[a][1]);
+                }
+            }
+#pragma unroll
+            for (int a = 0; a < 4; ++a)
+#pragma unroll
+                for (int b = 0; b < 2; ++b) {
+                    const int col = col0 + 2 * tx + b;
+                    if (col < d) {
+                        float* o = &Os[(4 * ty + a) * d + col];
+                        *o = *o * alpha[a] + acc[a][b];
+                    }
+                }
+        }
+    }
+    if (tx == 0) {
+#pragma unroll
+        for (int a = 0; a < 4; ++a) { rowM[4 * ty + a] = mrow[a]; rowL[4 * ty + a] = lrow[a]; }
     }
     __syncthreads();
     const int nrows = min(T, Lr - m0);
@@ -505,6 +743,7 @@ __global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q
     }
 }
 
+size_t fwd_v2_smem(int64_t d) { return sizeof(float) * (2 * DS * TP + C * VSP + C * TP + 64 * d + 128); }
 size_t fwd_smem(int64_t d) { return sizeof(float) * (64 * SP + C * SP + 64 * (C + 1) + 64 * d + 128); }
 size_t dq_smem(int T, int64_t d) { return sizeof(float) * (2 * T * SP + 2 * C * SP + 2 * T * (C + 1) + T + 2 * T * d); }
 size_t dkdv_smem(int T, int64_t d) {
@@ -523,11 +762,18 @@ template <typename Tin>
 cudaError_t fwd_impl(const void* q, const void* k, const void* v, void* out, float* lse, float* tape,
                      int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                      cudaStream_t st) {
-    static std::once_flag once;
+    static std::once_flag once, once2;
     Geo g = make_geo(B, H, L, d, w, dil, 64);
-    set_smem_once(simt_fwd_kernel<Tin>, fwd_smem(d), once);
-    simt_fwd_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_smem(d), st>>>(
-        (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, tape, g);
+    const char* e1 = getenv("FT_WINATTN_SIMT_V1");   // A/B timing: the scalar-load version
+    if (e1 && atoi(e1) == 1) {
+        set_smem_once(simt_fwd_kernel<Tin>, fwd_smem(d), once);
+        simt_fwd_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_smem(d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, tape, g);
+    } else {
+        set_smem_once(simt_fwd_v2_kernel<Tin>, fwd_v2_smem(d), once2);
+        simt_fwd_v2_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_v2_smem(d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, tape, g);
+    }
     prof_mark(st);
     return cudaGetLastError();
 }
