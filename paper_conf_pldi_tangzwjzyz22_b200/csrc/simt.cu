@@ -253,47 +253,6 @@ __global__ void __launch_bounds__(NT) simt_fwd_kernel(const Tin* __restrict__ q,
 constexpr int TP = 64 + 4;     // padded row count of a transposed slice (16-byte aligned rows)
 constexpr int VSP = DS + 4;    // padded V slice row (16-byte aligned)
 
-template <typename Tin, int R>
-__device__ __forceinline__ void load_slice_t(float* dst, const Tin* __restrict__ base, int64_t rstride,
-                                             int mbase, int Lr, int col0, int d) {
-    constexpr int V = Vec<Tin>::N;
-    constexpr int NV = DS / V;
-    for (int idx = threadIdx.x; idx < R * NV; idx += NT) {
-        const int row = idx / NV, cv = idx % NV;
-        const int m = mbase + row, c = col0 + cv * V;
-        float vals[V];
-        if (m >= 0 && m < Lr && c < d) {
-            Vec<Tin>::load(base + (int64_t)m * rstride + c, vals);
-        } else {
-#pragma unroll
-            for (int e = 0; e < V; ++e) vals[e] = 0.f;
-        }
-#pragma unroll
-        for (int e = 0; e < V; ++e) dst[(cv * V + e) * TP + row] = vals[e];
-    }
-}
-
-template <typename Tin, int R>
-__device__ __forceinline__ void load_slice_v(float* dst, const Tin* __restrict__ base, int64_t rstride,
-                                             int mbase, int Lr, int col0, int d) {
-    constexpr int V = Vec<Tin>::N;
-    constexpr int NV = DS / V;
-    for (int idx = threadIdx.x; idx < R * NV; idx += NT) {
-        const int row = idx / NV, cv = idx % NV;
-        const int m = mbase + row, c = col0 + cv * V;
-        float vals[V];
-        if (m >= 0 && m < Lr && c < d) {
-            Vec<Tin>::load(base + (int64_t)m * rstride + c, vals);
-        } else {
-#pragma unroll
-            for (int e = 0; e < V; ++e) vals[e] = 0.f;
-        }
-#pragma unroll
-        for (int e = 0; e < V; e += 4)
-            *reinterpret_cast<float4*>(&dst[row * VSP + cv * V + e]) = make_float4(vals[e], vals[e + 1], vals[e + 2], vals[e + 3]);
-    }
-}
-
 // Register-staged slice loads for software pipelining: a thread fetches its share of slice
 // i+1 from HBM into registers while the CTA computes on slice i in shared memory, then stores it
 // after the barrier -- the global latency is hidden behind the micro-GEMM instead of being paid
@@ -324,6 +283,16 @@ struct SliceRegs {
             const int row = idx / NV, cv = idx % NV;
 #pragma unroll
             for (int e = 0; e < V; ++e) dst[(cv * V + e) * TP + row] = vals[it][e];
+        }
+    }
+    __device__ void store_p(float (*dst)[SP]) const {   // row-major, rows padded to SP
+#pragma unroll
+        for (int it = 0; it < PER; ++it) {
+            const int idx = threadIdx.x + it * NT;
+            if (idx >= R * NV) break;
+            const int row = idx / NV, cv = idx % NV;
+#pragma unroll
+            for (int e = 0; e < V; ++e) dst[row][cv * V + e] = vals[it][e];
         }
     }
     __device__ void store_v(float* dst) const {   // row-major, rows padded to VSP
@@ -531,13 +500,23 @@ __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
         for (int a = 0; a < RA; ++a)
 #pragma unroll
             for (int b = 0; b < 4; ++b) { s[a][b] = 0.f; dp[a][b] = 0.f; }
+        SliceRegs<Tin, T> rq, rg;
+        SliceRegs<Tin, C> rk, rv;
+        auto fetch = [&](int col0) {   // slice col0 into registers (software pipelining)
+            if (!TAPE) rq.fetch(q + tc.off, tc.rstride, m0, Lr, col0, d);
+            rg.fetch(dout + tc.off, tc.rstride, m0, Lr, col0, d);
+            if (!TAPE) rk.fetch(k + tc.off, tc.rstride, c0, kend, col0, d);
+            rv.fetch(v + tc.off, tc.rstride, c0, kend, col0, d);
+        };
+        fetch(0);
         for (int col0 = 0; col0 < d; col0 += DS) {
             __syncthreads();
-            if (!TAPE) load_slice<Tin, T>(Qs, q + tc.off, tc.rstride, m0, Lr, col0, d);
-            load_slice<Tin, T>(Gs, dout + tc.off, tc.rstride, m0, Lr, col0, d);
-            if (!TAPE) load_slice<Tin, C>(Ks, k + tc.off, tc.rstride, c0, kend, col0, d);
-            load_slice<Tin, C>(Vs, v + tc.off, tc.rstride, c0, kend, col0, d);
+            if (!TAPE) rq.store_p(Qs);
+            rg.store_p(Gs);
+            if (!TAPE) rk.store_p(Ks);
+            rv.store_p(Vs);
             __syncthreads();
+            if (col0 + DS < d) fetch(col0 + DS);
 #pragma unroll 4
             for (int p = 0; p < DS; ++p) {
                 float qa[RA], ga[RA], kb[4], vb[4];
@@ -569,10 +548,13 @@ __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
                 Ps[ty + 16 * a][tx + 16 * b] = p;
             }
         }
+        SliceRegs<Tin, C> rk2;
+        rk2.fetch(k + tc.off, tc.rstride, c0, kend, 0, d);
         for (int col0 = 0; col0 < d; col0 += DS) {
             __syncthreads();
-            load_slice<Tin, C>(Ks, k + tc.off, tc.rstride, c0, kend, col0, d);
+            rk2.store_p(Ks);
             __syncthreads();
+            if (col0 + DS < d) rk2.fetch(k + tc.off, tc.rstride, c0, kend, col0 + DS, d);
             float aA[RA][2], aB[RA][2];
 #pragma unroll
             for (int a = 0; a < RA; ++a) { aA[a][0] = aA[a][1] = aB[a][0] = aB[a][1] = 0.f; }
@@ -663,13 +645,23 @@ __global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q
             qlse[i] = mq < qend ? lse[fr] * LOG2E : 0.f;
             qD[i] = mq < qend ? Dws[fr] : 0.f;
         }
+        SliceRegs<Tin, T> rk, rv;
+        SliceRegs<Tin, C> rq, rg;
+        auto fetch = [&](int col0) {   // slice col0 into registers (software pipelining)
+            if (!TAPE) rk.fetch(k + tc.off, tc.rstride, m0, Lr, col0, d);
+            rv.fetch(v + tc.off, tc.rstride, m0, Lr, col0, d);
+            if (!TAPE) rq.fetch(q + tc.off, tc.rstride, c0, qend, col0, d);
+            rg.fetch(dout + tc.off, tc.rstride, c0, qend, col0, d);
+        };
+        fetch(0);
         for (int col0 = 0; col0 < d; col0 += DS) {
             __syncthreads();
-            if (!TAPE) load_slice<Tin, T>(Ks, k + tc.off, tc.rstride, m0, Lr, col0, d);
-            load_slice<Tin, T>(Vs, v + tc.off, tc.rstride, m0, Lr, col0, d);
-            if (!TAPE) load_slice<Tin, C>(Qs, q + tc.off, tc.rstride, c0, qend, col0, d);
-            load_slice<Tin, C>(Gs, dout + tc.off, tc.rstride, c0, qend, col0, d);
+            if (!TAPE) rk.store_p(Ks);
+            rv.store_p(Vs);
+            if (!TAPE) rq.store_p(Qs);
+            rg.store_p(Gs);
             __syncthreads();
+            if (col0 + DS < d) fetch(col0 + DS);
 #pragma unroll 4
             for (int p = 0; p < DS; ++p) {
                 float ka[RA], va[RA], qb[4], gb[4];
@@ -700,11 +692,18 @@ __global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q
                 DSs[ty + 16 * a][qi] = p * (dp[a][b] - qD[qi]);
             }
         }
+        SliceRegs<Tin, C> rq2, rg2;
+        rq2.fetch(q + tc.off, tc.rstride, c0, qend, 0, d);
+        rg2.fetch(dout + tc.off, tc.rstride, c0, qend, 0, d);
         for (int col0 = 0; col0 < d; col0 += DS) {
             __syncthreads();
-            load_slice<Tin, C>(Qs, q + tc.off, tc.rstride, c0, qend, col0, d);
-            load_slice<Tin, C>(Gs, dout + tc.off, tc.rstride, c0, qend, col0, d);
+            rq2.store_p(Qs);
+            rg2.store_p(Gs);
             __syncthreads();
+            if (col0 + DS < d) {
+                rq2.fetch(q + tc.off, tc.rstride, c0, qend, col0 + DS, d);
+                rg2.fetch(dout + tc.off, tc.rstride, c0, qend, col0 + DS, d);
+            }
             float ak[RA][2], av[RA][2];
 #pragma unroll
             for (int a = 0; a < RA; ++a) { ak[a][0] = ak[a][1] = av[a][0] = av[a][1] = 0.f; }
