@@ -275,14 +275,15 @@ struct SliceRegs {
             }
         }
     }
-    __device__ void store_t(float* dst) const {   // transposed: [col][row], rows padded to TP
+    template <int RP = TP>
+    __device__ void store_t(float* dst) const {   // transposed: [col][row], rows padded to RP
 #pragma unroll
         for (int it = 0; it < PER; ++it) {
             const int idx = threadIdx.x + it * NT;
             if (idx >= R * NV) break;
             const int row = idx / NV, cv = idx % NV;
 #pragma unroll
-            for (int e = 0; e < V; ++e) dst[(cv * V + e) * TP + row] = vals[it][e];
+            for (int e = 0; e < V; ++e) dst[(cv * V + e) * RP + row] = vals[it][e];
         }
     }
     __device__ void store_p(float (*dst)[SP]) const {   // row-major, rows padded to SP
@@ -598,6 +599,168 @@ __global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
         Dws[tc.row0 + (int64_t)(m0 + row) * g.dil] = rowD[row];
 }
 
+// dq, v2: the same sweep with the vectorised staging of simt_fwd_v2_kernel -- a thread owns the
+// RA consecutive rows RA*ty.. and the four consecutive keys 4tx.., Q / dO / K / V slices are
+// staged transposed ([d column][row]) and P, P*dP transposed ([key][row]), so every operand of
+// both micro-GEMMs is one 8- or 16-byte shared load.
+template <int RA>
+__device__ __forceinline__ void ldrows(const float* p, float (&o)[RA]) {
+    if (RA == 4) {
+        const float4 x = *reinterpret_cast<const float4*>(p);
+        o[0] = x.x; o[1] = x.y; o[RA > 2 ? 2 : 0] = x.z; o[RA > 3 ? 3 : 0] = x.w;
+    } else {
+        const float2 x = *reinterpret_cast<const float2*>(p);
+        o[0] = x.x; o[1] = x.y;
+    }
+}
+
+template <typename Tin, int T, bool TAPE>
+__global__ void __launch_bounds__(NT, T == 32 ? 1 : 0) simt_dq_v2_kernel(const Tin* __restrict__ q,
+                                                        const Tin* __restrict__ k,
+                                                        const Tin* __restrict__ v,
+                                                        const Tin* __restrict__ dout,
+                                                        const float* __restrict__ lse,
+                                                        const float* __restrict__ tape,
+                                                        float* __restrict__ Dws,
+                                                        Tin* __restrict__ dq, Geo g) {
+    constexpr int RA = T / 16;
+    constexpr int RP = T + 4;                 // padded row count of a transposed T-row slice
+    extern __shared__ float smem[];
+    float* Qt = smem;                         // [DS][RP]
+    float* Gt = Qt + DS * RP;                 // [DS][RP]
+    float* Kt = Gt + DS * RP;                 // [DS][TP]
+    float* Vt = Kt + DS * TP;                 // [DS][TP]
+    float* PDt = Vt + DS * TP;                // [C][RP]  (P * dP) transposed
+    float* Pt = PDt + C * RP;                 // [C][RP]
+    float* Ko = Qt;                           // [C][VSP] output-loop K slices (reuses Qt / Gt)
+    float* rowD = Pt + C * RP;
+    float* OsA = rowD + T;
+    float* OsB = OsA + T * g.d;
+    static_assert(C * VSP <= 2 * DS * RP, "output K slice fits in the Q / dO staging");
+
+    TileCoord tc;
+    if (!decode(g, tc)) return;
+    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+    for (int i = threadIdx.x; i < T * d; i += NT) { OsA[i] = 0.f; OsB[i] = 0.f; }
+
+    float lse2[RA], Dacc[RA];
+#pragma unroll
+    for (int a = 0; a < RA; ++a) {
+        const int mq = m0 + RA * ty + a;
+        lse2[a] = mq < Lr ? lse[tc.row0 + (int64_t)mq * g.dil] * LOG2E : 0.f;
+        Dacc[a] = 0.f;
+    }
+    const int kbeg = max(0, m0 - w);
+    const int kend = min(Lr, m0 + T + w);
+    for (int c0 = kbeg; c0 < kend; c0 += C) {
+        float s[RA][4], dp[RA][4];
+#pragma unroll
+        for (int a = 0; a < RA; ++a)
+#pragma unroll
+            for (int b = 0; b < 4; ++b) { s[a][b] = 0.f; dp[a][b] = 0.f; }
+        SliceRegs<Tin, T> rq, rg;
+        SliceRegs<Tin, C> rk, rv;
+        auto fetch = [&](int col0) {
+            if (!TAPE) rq.fetch(q + tc.off, tc.rstride, m0, Lr, col0, d);
+            rg.fetch(dout + tc.off, tc.rstride, m0, Lr, col0, d);
+            if (!TAPE) rk.fetch(k + tc.off, tc.rstride, c0, kend, col0, d);
+            rv.fetch(v + tc.off, tc.rstride, c0, kend, col0, d);
+        };
+        fetch(0);
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            if (!TAPE) rq.template store_t<RP>(Qt);
+            rg.template store_t<RP>(Gt);
+            if (!TAPE) rk.template store_t<TP>(Kt);
+            rv.template store_t<TP>(Vt);
+            __syncthreads();
+            if (col0 + DS < d) fetch(col0 + DS);
+#pragma unroll 4
+            for (int p = 0; p < DS; ++p) {
+                float qa[RA], ga[RA];
+                if (!TAPE) ldrows<RA>(&Qt[p * RP + RA * ty], qa);
+                ldrows<RA>(&Gt[p * RP + RA * ty], ga);
+                float4 kb4 = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (!TAPE) kb4 = *reinterpret_cast<const float4*>(&Kt[p * TP + 4 * tx]);
+                const float4 vb4 = *reinterpret_cast<const float4*>(&Vt[p * TP + 4 * tx]);
+                const float kb[4] = {kb4.x, kb4.y, kb4.z, kb4.w}, vb[4] = {vb4.x, vb4.y, vb4.z, vb4.w};
+#pragma unroll
+                for (int a = 0; a < RA; ++a)
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) {
+                        if (!TAPE) s[a][b] = fmaf(qa[a], kb[b], s[a][b]);
+                        dp[a][b] = fmaf(ga[a], vb[b], dp[a][b]);
+                    }
+            }
+        }
+#pragma unroll
+        for (int a = 0; a < RA; ++a) {
+            const int mq = m0 + RA * ty + a;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int mk = c0 + 4 * tx + b;
+                const bool ok = (mk < kend) && (abs(mk - mq) <= w) && mq < Lr;
+                if (TAPE && ok) s[a][b] = tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)];
+                const float pv = ok ? exp2f(s[a][b] * LOG2E - lse2[a]) : 0.f;
+                const float pd = pv * dp[a][b];
+                Dacc[a] += pd;
+                PDt[(4 * tx + b) * RP + RA * ty + a] = pd;
+                Pt[(4 * tx + b) * RP + RA * ty + a] = pv;
+            }
+        }
+        SliceRegs<Tin, C> rk2;
+        rk2.fetch(k + tc.off, tc.rstride, c0, kend, 0, d);
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            rk2.store_v(Ko);
+            __syncthreads();
+            if (col0 + DS < d) rk2.fetch(k + tc.off, tc.rstride, c0, kend, col0 + DS, d);
+            float aA[RA][2], aB[RA][2];
+#pragma unroll
+            for (int a = 0; a < RA; ++a) { aA[a][0] = aA[a][1] = aB[a][0] = aB[a][1] = 0.f; }
+#pragma unroll 4
+            for (int kk = 0; kk < C; ++kk) {
+                const float2 kv = *reinterpret_cast<const float2*>(&Ko[kk * VSP + 2 * tx]);
+                float pd[RA], pv[RA];
+                ldrows<RA>(&PDt[kk * RP + RA * ty], pd);
+                ldrows<RA>(&Pt[kk * RP + RA * ty], pv);
+#pragma unroll
+                for (int a = 0; a < RA; ++a) {
+                    aA[a][0] = fmaf(pd[a], kv.x, aA[a][0]);
+                    aA[a][1] = fmaf(pd[a], kv.y, aA[a][1]);
+                    aB[a][0] = fmaf(pv[a], kv.x, aB[a][0]);
+                    aB[a][1] = fmaf(pv[a], kv.y, aB[a][1]);
+                }
+            }
+#pragma unroll
+            for (int a = 0; a < RA; ++a)
+#pragma unroll
+                for (int b = 0; b < 2; ++b) {
+                    const int col = col0 + 2 * tx + b;
+                    if (col < d) {
+                        OsA[(RA * ty + a) * d + col] += aA[a][b];
+                        OsB[(RA * ty + a) * d + col] += aB[a][b];
+                    }
+                }
+        }
+    }
+#pragma unroll
+    for (int a = 0; a < RA; ++a) {
+        const float D = hsum16(Dacc[a]);
+        if (tx == 0) rowD[RA * ty + a] = D;
+    }
+    __syncthreads();
+    const int nrows = min(T, Lr - m0);
+    for (int i = threadIdx.x; i < nrows * d; i += NT) {
+        const int row = i / d, col = i % d;
+        Vec<Tin>::store1(dq + tc.off + (int64_t)(m0 + row) * tc.rstride + col,
+                         OsA[i] - rowD[row] * OsB[i]);
+    }
+    for (int row = threadIdx.x; row < nrows; row += NT)
+        Dws[tc.row0 + (int64_t)(m0 + row) * g.dil] = rowD[row];
+}
+
 // ------------------------------------------------------------------------------ backward: dk, dv
 // Key-major: for owned key rows j, dk_j = sum_i dS_ij q_i and dv_j = sum_i P_ij dout_i over
 // the queries i whose window contains j (the band is symmetric: |m_i - m_j| <= w).
@@ -742,8 +905,166 @@ __global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q
     }
 }
 
+// dk / dv, v2: simt_dkdv_kernel with the staging of simt_dq_v2_kernel -- a thread owns key
+// rows RA*ty.. and the four consecutive queries 4tx..; K / V / Q / dO slices transposed, P and
+// dS transposed ([query][key row]), the output loop's Q / dO slices row-major (float2 loads).
+template <typename Tin, int T, bool TAPE>
+__global__ void __launch_bounds__(NT) simt_dkdv_v2_kernel(const Tin* __restrict__ q,
+                                                          const Tin* __restrict__ k,
+                                                          const Tin* __restrict__ v,
+                                                          const Tin* __restrict__ dout,
+                                                          const float* __restrict__ lse,
+                                                          const float* __restrict__ tape,
+                                                          const float* __restrict__ Dws,
+                                                          Tin* __restrict__ dk, Tin* __restrict__ dv,
+                                                          Geo g) {
+    constexpr int RA = T / 16;
+    constexpr int RP = T + 4;
+    extern __shared__ float smem[];
+    float* Kt = smem;                 // [DS][RP]
+    float* Vt = Kt + DS * RP;         // [DS][RP]
+    float* Qt = Vt + DS * RP;         // [DS][TP]
+    float* Gt = Qt + DS * TP;         // [DS][TP]
+    float* Pt = Gt + DS * TP;         // [C][RP]
+    float* DSt = Pt + C * RP;         // [C][RP]
+    float* Qo = smem;                 // [C][VSP] output-loop slices (reuse Kt .. Gt)
+    float* Go = Qo + C * VSP;
+    float* qlse = DSt + C * RP;
+    float* qD = qlse + C;
+    float* OsK = qD + C;
+    float* OsV = OsK + T * g.d;
+    static_assert(2 * C * VSP <= 2 * DS * RP + 2 * DS * TP, "output slices fit in the staging");
+
+    TileCoord tc;
+    if (!decode(g, tc)) return;
+    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+    for (int i = threadIdx.x; i < T * d; i += NT) { OsK[i] = 0.f; OsV[i] = 0.f; }
+
+    const int qbeg = max(0, m0 - w);
+    const int qend = min(Lr, m0 + T + w);
+    for (int c0 = qbeg; c0 < qend; c0 += C) {
+        float s[RA][4], dp[RA][4];
+#pragma unroll
+        for (int a = 0; a < RA; ++a)
+#pragma unroll
+            for (int b = 0; b < 4; ++b) { s[a][b] = 0.f; dp[a][b] = 0.f; }
+        __syncthreads();
+        for (int i = threadIdx.x; i < C; i += NT) {
+            const int mq = c0 + i;
+            const int64_t fr = tc.row0 + (int64_t)mq * g.dil;
+            qlse[i] = mq < qend ? lse[fr] * LOG2E : 0.f;
+            qD[i] = mq < qend ? Dws[fr] : 0.f;
+        }
+        SliceRegs<Tin, T> rk, rv;
+        SliceRegs<Tin, C> rq, rg;
+        auto fetch = [&](int col0) {
+            if (!TAPE) rk.fetch(k + tc.off, tc.rstride, m0, Lr, col0, d);
+            rv.fetch(v + tc.off, tc.rstride, m0, Lr, col0, d);
+            if (!TAPE) rq.fetch(q + tc.off, tc.rstride, c0, qend, col0, d);
+            rg.fetch(dout + tc.off, tc.rstride, c0, qend, col0, d);
+        };
+        fetch(0);
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            if (!TAPE) rk.template store_t<RP>(Kt);
+            rv.template store_t<RP>(Vt);
+            if (!TAPE) rq.template store_t<TP>(Qt);
+            rg.template store_t<TP>(Gt);
+            __syncthreads();
+            if (col0 + DS < d) fetch(col0 + DS);
+#pragma unroll 4
+            for (int p = 0; p < DS; ++p) {
+                float ka[RA], va[RA];
+                if (!TAPE) ldrows<RA>(&Kt[p * RP + RA * ty], ka);
+                ldrows<RA>(&Vt[p * RP + RA * ty], va);
+                float4 qb4 = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (!TAPE) qb4 = *reinterpret_cast<const float4*>(&Qt[p * TP + 4 * tx]);
+                const float4 gb4 = *reinterpret_cast<const float4*>(&Gt[p * TP + 4 * tx]);
+                const float qb[4] = {qb4.x, qb4.y, qb4.z, qb4.w}, gb[4] = {gb4.x, gb4.y, gb4.z, gb4.w};
+#pragma unroll
+                for (int a = 0; a < RA; ++a)
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) {
+                        if (!TAPE) s[a][b] = fmaf(ka[a], qb[b], s[a][b]);
+                        dp[a][b] = fmaf(va[a], gb[b], dp[a][b]);
+                    }
+            }
+        }
+#pragma unroll
+        for (int a = 0; a < RA; ++a) {
+            const int mk = m0 + RA * ty + a;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int qi = 4 * tx + b;
+                const int mq = c0 + qi;
+                const bool ok = (mq < qend) && (abs(mq - mk) <= w) && mk < Lr;
+                if (TAPE && ok) s[a][b] = tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)];
+                const float p = ok ? exp2f(s[a][b] * LOG2E - qlse[qi]) : 0.f;
+                Pt[qi * RP + RA * ty + a] = p;
+                DSt[qi * RP + RA * ty + a] = p * (dp[a][b] - qD[qi]);
+            }
+        }
+        SliceRegs<Tin, C> rq2, rg2;
+        rq2.fetch(q + tc.off, tc.rstride, c0, qend, 0, d);
+        rg2.fetch(dout + tc.off, tc.rstride, c0, qend, 0, d);
+        for (int col0 = 0; col0 < d; col0 += DS) {
+            __syncthreads();
+            rq2.store_v(Qo);
+            rg2.store_v(Go);
+            __syncthreads();
+            if (col0 + DS < d) {
+                rq2.fetch(q + tc.off, tc.rstride, c0, qend, col0 + DS, d);
+                rg2.fetch(dout + tc.off, tc.rstride, c0, qend, col0 + DS, d);
+            }
+            float ak[RA][2], av[RA][2];
+#pragma unroll
+            for (int a = 0; a < RA; ++a) { ak[a][0] = ak[a][1] = av[a][0] = av[a][1] = 0.f; }
+#pragma unroll 4
+            for (int qi = 0; qi < C; ++qi) {
+                const float2 qv = *reinterpret_cast<const float2*>(&Qo[qi * VSP + 2 * tx]);
+                const float2 gv = *reinterpret_cast<const float2*>(&Go[qi * VSP + 2 * tx]);
+                float ds[RA], pv[RA];
+                ldrows<RA>(&DSt[qi * RP + RA * ty], ds);
+                ldrows<RA>(&Pt[qi * RP + RA * ty], pv);
+#pragma unroll
+                for (int a = 0; a < RA; ++a) {
+                    ak[a][0] = fmaf(ds[a], qv.x, ak[a][0]);
+                    ak[a][1] = fmaf(ds[a], qv.y, ak[a][1]);
+                    av[a][0] = fmaf(pv[a], gv.x, av[a][0]);
+                    av[a][1] = fmaf(pv[a], gv.y, av[a][1]);
+                }
+            }
+#pragma unroll
+            for (int a = 0; a < RA; ++a)
+#pragma unroll
+                for (int b = 0; b < 2; ++b) {
+                    const int col = col0 + 2 * tx + b;
+                    if (col < d) {
+                        OsK[(RA * ty + a) * d + col] += ak[a][b];
+                        OsV[(RA * ty + a) * d + col] += av[a][b];
+                    }
+                }
+        }
+    }
+    __syncthreads();
+    const int nrows = min(T, Lr - m0);
+    for (int i = threadIdx.x; i < nrows * d; i += NT) {
+        const int row = i / d, col = i % d;
+        const int64_t o = tc.off + (int64_t)(m0 + row) * tc.rstride + col;
+        Vec<Tin>::store1(dk + o, OsK[i]);
+        Vec<Tin>::store1(dv + o, OsV[i]);
+    }
+}
+
+size_t dkdv_v2_smem(int T, int64_t d) {
+    return sizeof(float) * (2 * DS * (T + 4) + 2 * DS * TP + 2 * C * (T + 4) + 2 * C + 2 * T * d);
+}
 size_t fwd_v2_smem(int64_t d) { return sizeof(float) * (2 * DS * TP + C * VSP + C * TP + 64 * d + 128); }
 size_t fwd_smem(int64_t d) { return sizeof(float) * (64 * SP + C * SP + 64 * (C + 1) + 64 * d + 128); }
+size_t dq_v2_smem(int T, int64_t d) {
+    return sizeof(float) * (2 * DS * (T + 4) + 2 * DS * TP + 2 * C * (T + 4) + T + 2 * T * d);
+}
 size_t dq_smem(int T, int64_t d) { return sizeof(float) * (2 * T * SP + 2 * C * SP + 2 * T * (C + 1) + T + 2 * T * d); }
 size_t dkdv_smem(int T, int64_t d) {
     return sizeof(float) * (2 * T * SP + 2 * C * SP + 2 * T * (C + 1) + 2 * C + 2 * T * d);
@@ -781,18 +1102,32 @@ template <typename Tin, int T, bool TAPE>
 cudaError_t bwd_launch(const void* q, const void* k, const void* v, const float* lse, const float* tape,
                        const void* dout, void* dq, void* dk, void* dv, float* Dws, const Geo& g,
                        cudaStream_t st) {
-    static std::once_flag o1, o2;
+    static std::once_flag o1, o2, o3, o4;
     const int64_t d = g.d;
-    set_smem_once(simt_dq_kernel<Tin, T, TAPE>, dq_smem(T, d), o1);
-    simt_dq_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dq_smem(T, d), st>>>(
-        (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dq, g);
+    const char* e1 = getenv("FT_WINATTN_SIMT_V1");   // A/B timing: the scalar-load version
+    if (e1 && atoi(e1) == 1) {
+        set_smem_once(simt_dq_kernel<Tin, T, TAPE>, dq_smem(T, d), o1);
+        simt_dq_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dq_smem(T, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dq, g);
+    } else {
+        set_smem_once(simt_dq_v2_kernel<Tin, T, TAPE>, dq_v2_smem(T, d), o3);
+        simt_dq_v2_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dq_v2_smem(T, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dq, g);
+    }
     prof_mark(st);
     cudaError_t e;
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
-    set_smem_once(simt_dkdv_kernel<Tin, T, TAPE>, dkdv_smem(T, d), o2);
-    simt_dkdv_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dkdv_smem(T, d), st>>>(
-        (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dk,
-        (Tin*)dv, g);
+    if (e1 && atoi(e1) == 1) {
+        set_smem_once(simt_dkdv_kernel<Tin, T, TAPE>, dkdv_smem(T, d), o2);
+        simt_dkdv_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dkdv_smem(T, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dk,
+            (Tin*)dv, g);
+    } else {
+        set_smem_once(simt_dkdv_v2_kernel<Tin, T, TAPE>, dkdv_v2_smem(T, d), o4);
+        simt_dkdv_v2_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dkdv_v2_smem(T, d), st>>>(
+            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dk,
+            (Tin*)dv, g);
+    }
     prof_mark(st);
     return cudaGetLastError();
 }
