@@ -16,7 +16,9 @@ global_batch = N), timed between a barrier + synchronize on both sides, and the 
 time is the max over ranks.
 
 Keys beyond the base contract: "roofline" (dominant kernel, CUDA events on the launching
-stream via the ft_winattn_profile_events hook), "hbm_step" (whole step vs SURVEY.md §8(d)
+stream via the ft_winattn_profile_events hook, recorded in a second pass of the same steps:
+an event between two launches would stop the BWDQ -> BWDKV programmatic dependent launch
+overlap inside the timed region), "hbm_step" (whole step vs SURVEY.md §8(d)
 algorithmic bytes), "cpu_baseline" (the fp64 oracle on a bounded sample, rank 0, N=1),
 "e2e" (pinned host buffers, H2D + fwd + bwd + D2H inside the timed region), "clocks"
 (NVML samples during the timed region) and "gpu_launches".
@@ -386,7 +388,7 @@ def main():
         e_ = torch.cuda.Event(enable_timing=True)
         e_.record(stream)   # materialise the CUDA event so its handle can go through the ABI
         return e_
-    starts, fevs, bevs, ends = [], [], [], []
+    starts, ends = [], []
     sampler = ClockSampler(dev.index if dev.index is not None else 0)
     if world > 1:
         dist.barrier()
@@ -395,23 +397,37 @@ def main():
         for _ in range(args.steps):
             if flush is not None:
                 flush.zero_()   # outside the events: evicts q/k/v/dout from L2
-            s0, fe, be, s1 = ev(), [ev() for _ in range(nf)], [ev() for _ in range(nb)], ev()
+            s0, s1 = ev(), ev()
             s0.record(stream)
-            with ft.profile_events(fe):
-                ft.fwd(q, k, v, w, dil, out=out, lse=lse, dilated_heads=hd)
-            with ft.profile_events(be):
-                ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
+            step()
             s1.record(stream)
-            starts.append(s0); fevs.append(fe); bevs.append(be); ends.append(s1)
+            starts.append(s0); ends.append(s1)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in zip(starts, ends)]
     elapsed_ms = sum(step_ms)
-    # per-kernel durations (each launch timed from the previous event on the same stream)
+    # Per-kernel durations: a second pass over the same steps with an event recorded after
+    # every launch (each launch timed from the previous event on the same stream).  It is
+    # kept out of the timed region because an event between two launches stops the
+    # programmatic-dependent-launch overlap (BWDQ -> BWDKV): these durations are serialised,
+    # i.e. conservative for the roofline.
     names = [f"fwd{i}" for i in range(nf)] + [f"bwd{i}" for i in range(nb)]
     kdur = {n: [] for n in names}
-    for s0, fe, be in zip(starts, fevs, bevs):
+    kpass = min(args.steps, 50)
+    rec = []
+    for _ in range(kpass):
+        if flush is not None:
+            flush.zero_()
+        s0, fe, be = ev(), [ev() for _ in range(nf)], [ev() for _ in range(nb)]
+        s0.record(stream)
+        with ft.profile_events(fe):
+            ft.fwd(q, k, v, w, dil, out=out, lse=lse, dilated_heads=hd)
+        with ft.profile_events(be):
+            ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
+        rec.append((s0, fe, be))
+    torch.cuda.synchronize()
+    for s0, fe, be in rec:
         prev = s0
         for n, e1 in zip(names, fe + be):
             kdur[n].append(prev.elapsed_time(e1))
@@ -570,6 +586,8 @@ def main():
             "paths": {"fwd": "tc" if path_f == ft.PATH_TC else "simt",
                       "bwd": "tc" if path_b == ft.PATH_TC else "simt"},
             "kernel_ms": {n: sum(x) / len(x) for n, x in kdur.items()},
+            "kernel_timing": f"separate pass of {kpass} steps with an event after every launch "
+                             "(serialised: no PDL overlap); the timed region has no per-launch events",
             "roofline": roof, "hbm_step": hbm_step, "ceilings": ceilings,
             "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": args.steps * (nf + nb),

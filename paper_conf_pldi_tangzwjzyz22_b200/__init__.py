@@ -125,6 +125,9 @@ class profile_events:
 
     def __init__(self, events):
         self.events = list(events)
+        for e in self.events:
+            if not e.cuda_event:
+                e.record()   # torch creates the CUDA event lazily; materialise its handle
         self._arr = (ctypes.c_void_p * max(1, len(self.events)))(
             *[ctypes.c_void_p(e.cuda_event) for e in self.events])
 

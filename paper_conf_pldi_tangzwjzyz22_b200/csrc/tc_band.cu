@@ -87,7 +87,22 @@ struct Params {
     SchedParams sc;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace)
     int two;                     // 1: two MMA issuers (warps 9, 10); 0: warp 9 issues all
+    int dpoll;                   // BWDKV: poll D row by row instead of waiting for all of BWDQ
 };
+
+// D rows not yet written by BWDQ hold D_UNSET (each BWDQ CTA stores it into the rows of its
+// tiles before it triggers the dependent BWDKV launch).  Arithmetic never produces this bit pattern: a NaN from the FP units is the
+// canonical 0x7FFFFFFF, so D_UNSET is never a value BWDQ stores.
+constexpr uint32_t D_UNSET = 0xFFFFFFFFu;
+__device__ __forceinline__ float ld_D_ready(const float* ptr) {
+    uint32_t x;
+    for (;;) {
+        asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr) : "memory");
+        if (x != D_UNSET) break;
+        __nanosleep(128);
+    }
+    return __uint_as_float(x);
+}
 
 // Phase trace: per CTA and local tile j < TRACE_TILES, clock64 stamps (SM cycles) of
 // 0 producer first score-GEMM load, 1 producer last output load, 2 MMA score GEMM first
@@ -202,6 +217,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     // BWDQ CTAs leave (its persistent CTAs finish 4 or 5 tiles apart) and stream their first
     // tiles' q/k/v/dout -- inputs of the whole backward call, complete before BWDQ started --
     // while BWDQ drains; only BWDKV's softmax warps, which read BWDQ's D, wait for it.
+    if (MODE == BWDQ && p.dpoll) {
+        // mark this CTA's D rows unset before BWDKV may launch (ld_D_ready); the CTA stores
+        // the real values of the same rows later, ordered after this by the barrier
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T)) {
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+            for (int i = threadIdx.x; i < BM && T.m0 + i < T.Lr; i += NTHREADS)
+                reinterpret_cast<uint32_t*>(p.D)[rowbase + (int64_t)(T.m0 + i) * p.dil] = D_UNSET;
+        }
+        __threadfence();
+        __syncthreads();
+    }
     if (MODE == BWDQ) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const int nkb = NK / KB;
     const int ncw = (d + 255) / 256;            // output chunks
@@ -496,7 +524,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
         uint32_t zero16[16];
 #pragma unroll
         for (int e = 0; e < 16; ++e) zero16[e] = 0u;
-        if (MODE == BWDKV) asm volatile("griddepcontrol.wait;" ::: "memory");   // D of BWDQ
+        // D of BWDQ: either wait for the whole BWDQ grid, or (dpoll) read each D row as soon
+        // as its BWDQ tile has stored it, so BWDKV's first tiles overlap BWDQ's last ones
+        if (MODE == BWDKV && !p.dpoll) asm volatile("griddepcontrol.wait;" ::: "memory");
         while (cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0;
             const int mrow = m0 + t;
@@ -509,7 +539,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     const int mc = kb + n;
                     const bool ok = mc >= 0 && mc < Lr;
                     colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
-                    colD[n] = ok ? p.D[rowbase + (int64_t)mc * p.dil] : 0.f;
+                    colD[n] = !ok ? 0.f
+                              : p.dpoll ? ld_D_ready(p.D + rowbase + (int64_t)mc * p.dil)
+                                        : p.D[rowbase + (int64_t)mc * p.dil];
                 }
                 named_bar_sync(1, 128);
             }
@@ -739,6 +771,13 @@ bool pdl_enabled() {
     return !(e && atoi(e) == 0);
 }
 
+// FT_WINATTN_DPOLL=0: BWDKV waits for the whole BWDQ grid (griddepcontrol.wait) instead of
+// polling D row by row (A/B timing)
+bool dpoll_enabled() {
+    const char* e = getenv("FT_WINATTN_DPOLL");
+    return !(e && atoi(e) == 0);
+}
+
 int num_sms() {
     static int n = 0;
     static std::once_flag once;
@@ -804,6 +843,7 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
             const char* e = getenv("FT_WINATTN_ISSUERS");
             p.two = !(e && atoi(e) == 1);
         }
+        p.dpoll = MODE != FWD && dpoll_enabled();
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms() ? total : num_sms()));
