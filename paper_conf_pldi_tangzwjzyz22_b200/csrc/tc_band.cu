@@ -90,19 +90,6 @@ struct Params {
     int dpoll;                   // BWDKV: poll D row by row instead of waiting for all of BWDQ
 };
 
-// D rows not yet written by BWDQ hold D_UNSET (each BWDQ CTA stores it into the rows of its
-// tiles before it triggers the dependent BWDKV launch).  Arithmetic never produces this bit pattern: a NaN from the FP units is the
-// canonical 0x7FFFFFFF, so D_UNSET is never a value BWDQ stores.
-constexpr uint32_t D_UNSET = 0xFFFFFFFFu;
-__device__ __forceinline__ float ld_D_ready(const float* ptr) {
-    uint32_t x;
-    for (;;) {
-        asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr) : "memory");
-        if (x != D_UNSET) break;
-        __nanosleep(128);
-    }
-    return __uint_as_float(x);
-}
 
 // Phase trace: per CTA and local tile j < TRACE_TILES, clock64 stamps (SM cycles) of
 // 0 producer first score-GEMM load, 1 producer last output load, 2 MMA score GEMM first
@@ -768,13 +755,6 @@ void set_attr_once() {
 // FT_WINATTN_PDL=0 turns the programmatic dependent launch off (A/B timing)
 bool pdl_enabled() {
     const char* e = getenv("FT_WINATTN_PDL");
-    return !(e && atoi(e) == 0);
-}
-
-// FT_WINATTN_DPOLL=0: BWDKV waits for the whole BWDQ grid (griddepcontrol.wait) instead of
-// polling D row by row (A/B timing)
-bool dpoll_enabled() {
-    const char* e = getenv("FT_WINATTN_DPOLL");
     return !(e && atoi(e) == 0);
 }
 

@@ -9,6 +9,7 @@
 //   instr desc (kind::f16): [4,6) D fmt (1=f32), [7,10) A fmt (1=bf16), [10,13) B fmt,
 //              [15] A major (1=MN), [16] B major, [17,23) N>>3, [24,29) M>>4
 #pragma once
+#include <stdlib.h>
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
@@ -353,6 +354,28 @@ __device__ __forceinline__ uint32_t elect_one() {
     asm volatile("{\n\t.reg .pred p;\n\telect.sync _|p, 0xffffffff;\n\tselp.u32 %0, 1, 0, p;\n\t}"
                  : "=r"(e));
     return e;
+}
+
+// ---- D hand-off between the two kernels of a split backward (dQ kernel -> dK/dV kernel).
+// The dQ kernel's CTAs first mark the D rows of their tiles D_UNSET, then trigger the
+// programmatic dependent launch; the dK/dV kernel, launched with PDL, reads each D row with
+// ld_D_ready as soon as it is stored, so its first tiles overlap the dQ kernel's last ones.
+// Arithmetic never produces D_UNSET: a NaN from the FP units is the canonical 0x7FFFFFFF.
+constexpr uint32_t D_UNSET = 0xFFFFFFFFu;
+__device__ __forceinline__ float ld_D_ready(const float* ptr) {
+    uint32_t x;
+    for (;;) {
+        asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr) : "memory");
+        if (x != D_UNSET) break;
+        __nanosleep(128);
+    }
+    return __uint_as_float(x);
+}
+
+// FT_WINATTN_DPOLL=0: the dK/dV kernel waits for the whole dQ grid instead (A/B timing)
+inline bool dpoll_enabled() {
+    const char* e = getenv("FT_WINATTN_DPOLL");
+    return !(e && atoi(e) == 0);
 }
 
 }  // namespace tc

@@ -76,6 +76,7 @@ struct BParams {
     const uint16_t* dout;   // WQ (wqc): raw dout / out rows for D~ = dout . out
     const uint16_t* out;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, mode 1 / 2)
+    int dpoll;                   // D hand-off by row polling (tc_common.cuh ld_D_ready)
 };
 
 // Phase trace, per CTA and local tile j < 8, 48 uint64 slots (ns sums over the tile):
@@ -133,6 +134,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
     const int d = p.d, w = p.w, nkc = p.nkc, nds = d / 64;
     const bool wqc = MODE == WQ && p.wqc;
     const int ACC = acc_cols<MODE>(d, p.wqc), NREG = n_regions<MODE>(d, p.wqc);
+    if (MODE == WQ && p.dpoll) {   // this CTA's D rows: unset, before WKV may launch
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T)) {
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+            for (int i = threadIdx.x; i < BM && T.m0 + i < T.Lr; i += NTHREADS)
+                reinterpret_cast<uint32_t*>(p.D)[rowbase + (int64_t)(T.m0 + i) * p.dil] = D_UNSET;
+        }
+        __threadfence();
+        __syncthreads();
+    }
+    if (MODE == WQ) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const int nsteps = (MODE == WQ && !wqc ? 2 : 1) * nkc;   // steps per tile
     const uint32_t RB = row_bytes(d), SB = slot_bytes(d);
     const int NKt = nkc * KC;
@@ -379,7 +392,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     const int mc = kb + n;
                     const bool ok = mc >= 0 && mc < Lr;
                     colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
-                    colD[n] = ok ? p.D[rowbase + (int64_t)mc * p.dil] : 0.f;
+                    colD[n] = !ok ? 0.f
+                              : p.dpoll ? ld_D_ready(p.D + rowbase + (int64_t)mc * p.dil)
+                                        : p.D[rowbase + (int64_t)mc * p.dil];
                 }
                 named_bar_sync(1, 256);
             } else {
@@ -689,7 +704,24 @@ cudaError_t launch(const void* a1, const void* a2, const void* b1, const void* b
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_bytes<MODE>((int)d, nkc) + (size_t)na * 2 * row_bytes((int)d) +
                             (size_t)(n1 + n2) * slot_bytes((int)d);
-        tc_wide_bwd_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
+        p.dpoll = dpoll_enabled();
+        if (MODE == WKV && r0 == 0 && p.dpoll) {
+            // WKV directly follows this call's last WQ launch on the stream: programmatic
+            // dependent launch, D handed over row by row
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = grid;
+            cfg.blockDim = dim3(NTHREADS);
+            cfg.dynamicSmemBytes = smem;
+            cfg.stream = st;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = at;
+            cfg.numAttrs = 1;
+            cudaLaunchKernelEx(&cfg, tc_wide_bwd_kernel<MODE>, p);
+        } else {
+            tc_wide_bwd_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
+        }
         prof_mark(st);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
