@@ -372,6 +372,14 @@ __device__ __forceinline__ float ld_D_ready(const float* ptr) {
     return __uint_as_float(x);
 }
 
+// one relaxed load (no memory clobber: a thread's loads of a halo issue back to back; the
+// few still D_UNSET are then re-read with ld_D_ready)
+__device__ __forceinline__ float ld_D_first(const float* ptr) {
+    uint32_t x;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr));
+    return __uint_as_float(x);
+}
+
 // FT_WINATTN_DPOLL=0: the dK/dV kernel waits for the whole dQ grid instead (A/B timing)
 inline bool dpoll_enabled() {
     const char* e = getenv("FT_WINATTN_DPOLL");

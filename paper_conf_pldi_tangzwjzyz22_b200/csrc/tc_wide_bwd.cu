@@ -393,9 +393,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     const bool ok = mc >= 0 && mc < Lr;
                     colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
                     colD[n] = !ok ? 0.f
-                              : p.dpoll ? ld_D_ready(p.D + rowbase + (int64_t)mc * p.dil)
+                              : p.dpoll ? ld_D_first(p.D + rowbase + (int64_t)mc * p.dil)
                                         : p.D[rowbase + (int64_t)mc * p.dil];
                 }
+                if (p.dpoll)   // rows whose WQ tile had not stored D yet
+                    for (int n = warp * 32 + lane; n < NKt; n += 256)
+                        if (__float_as_uint(colD[n]) == D_UNSET)
+                            colD[n] = ld_D_ready(p.D + rowbase + (int64_t)(kb + n) * p.dil);
                 named_bar_sync(1, 256);
             } else {
                 lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
