@@ -464,3 +464,35 @@ def test_autograd_mixed_dilation(ft):
         compare("out", out[:, h0:h1].detach().double().cpu().numpy(), ro, "bf16")
         for n, t, b in zip(("dq", "dk", "dv"), (q, k, v), r):
             compare(n, t.grad[:, h0:h1].double().cpu().numpy(), b, "bf16")
+
+
+@pytest.mark.parametrize("shape", [(1, 2, 700, 512, 32, 1), (1, 3, 900, 512, 20, 3), (1, 2, 700, 64, 100, 2),
+                                   (2, 3, 1500, 128, 80, 1), (1, 2, 40000, 512, 32, 1)],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_d_handoff_stale_workspace(ft, shape):
+    """The split backward hands D from the dQ kernel to the dK/dV kernel row by row
+    (tc_common.cuh ld_D_ready). Whatever the workspace
+    holds before the call -- the unset marker everywhere, D of different inputs from an
+    earlier call, zeros -- the gradients must be bit-identical to the grid-wide-wait
+    schedule (FT_WINATTN_DPOLL=0), and equal the oracle on sampled rows."""
+    sh = WinAttnShape(*shape)
+    x = make_inputs(sh, 21, "bf16")
+    y = make_inputs(sh, 22, "bf16")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    out, lse = ft.fwd(q, k, v, sh.w, sh.dilation)
+    with _env(FT_WINATTN_DPOLL="0"):
+        want = ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation)
+    nbytes = ft.workspace_bytes(q, sh.w, sh.dilation)
+    ws = torch.empty(max(nbytes, 16), dtype=torch.uint8, device=dev)
+    # stale D of other inputs (same shape) left by an earlier call
+    q2, k2, v2, g2 = (y[n].to(dev) for n in ("q", "k", "v", "dout"))
+    o2, l2 = ft.fwd(q2, k2, v2, sh.w, sh.dilation)
+    fills = [lambda: ws.fill_(0xFF), lambda: ws.zero_(),
+             lambda: ft.bwd(q2, k2, v2, o2, l2, g2, sh.w, sh.dilation, workspace=ws)]
+    for fill in fills:
+        fill()
+        got = ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation, workspace=ws)
+        torch.cuda.synchronize()
+        for a, b in zip(got, want):
+            assert torch.equal(a, b)
