@@ -87,6 +87,7 @@ struct BParams {
     int w, dil;
     SchedParams sc;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, modes 1 / 2)
+    int dpoll;                   // D hand-off by row polling (tc_common.cuh ld_D_ready)
 };
 
 // Phase trace: per CTA and local tile j < 8, clock64 stamps (tools/trace_narrow.py).
@@ -142,6 +143,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw_u32 = smem_u32(smem_raw);
     uint8_t* smem = smem_raw + (((raw_u32 + 1023u) & ~1023u) - raw_u32);
+    if (MODE == NQ && p.dpoll) {   // this CTA's D rows: unset, before NKV may launch
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T)) {
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+            for (int i = threadIdx.x; i < BM && T.m0 + i < T.Lr; i += NTHREADS)
+                reinterpret_cast<uint32_t*>(p.D)[rowbase + (int64_t)(T.m0 + i) * p.dil] = D_UNSET;
+        }
+        __threadfence();
+        __syncthreads();
+    }
+    if (MODE == NQ) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     uint8_t* stages = smem;                                        // [NSTAGE] {A1, A2, B1, B2}
     uint8_t* xbuf = smem + (size_t)NSTAGE * STAGE;                 // NQ: dS operand; NKV: staging
     float* colv = reinterpret_cast<float*>(xbuf + XBYTES);         // NKV [2][2][NK]: lse, D of columns
@@ -369,6 +382,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             c.Lr = X.Lr; c.m0 = X.m0; c.kb = X.m0 - w; c.u = X.u; c.rl = X.rl;
             c.rowbase = (int64_t)X.u * p.L + X.r;
             cp_async_wait_all();   // this tile's values (copied a tile ago)
+            if (MODE == NKV && p.dpoll && threadIdx.x < NK) {   // D rows NQ had not stored yet
+                float* cd = colv + (jx & 1) * 2 * NK + NK + threadIdx.x;
+                if (__float_as_uint(*cd) == D_UNSET)
+                    *cd = ld_D_ready(p.D + c.rowbase + (int64_t)(c.kb + (int)threadIdx.x) * p.dil);
+            }
             c.lse2 = MODE == NQ ? lpre[(jx & 1) * 256 + threadIdx.x] * LOG2E : 0.f;
             if (MODE == NKV) named_bar_sync(5, 256);   // every thread's columns landed
             hn = nxt.next(p.sc, Tn);
@@ -573,7 +591,24 @@ cudaError_t launch_nb(const void* a1, const void* a2, const void* b1, const void
         const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms_nb() ? total : num_sms_nb()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
-        tc_narrow_bwd_kernel<MODE><<<grid, NTHREADS, SMEM_BYTES, st>>>(p);
+        p.dpoll = dpoll_enabled();
+        if (MODE == NKV && r0 == 0 && p.dpoll) {
+            // NKV directly follows this call's last NQ launch: programmatic dependent launch,
+            // D handed over row by row
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = grid;
+            cfg.blockDim = dim3(NTHREADS);
+            cfg.dynamicSmemBytes = SMEM_BYTES;
+            cfg.stream = st;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = at;
+            cfg.numAttrs = 1;
+            cudaLaunchKernelEx(&cfg, tc_narrow_bwd_kernel<MODE>, p);
+        } else {
+            tc_narrow_bwd_kernel<MODE><<<grid, NTHREADS, SMEM_BYTES, st>>>(p);
+        }
         prof_mark(st);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
