@@ -467,7 +467,8 @@ def test_autograd_mixed_dilation(ft):
 
 
 @pytest.mark.parametrize("shape", [(1, 2, 700, 512, 32, 1), (1, 3, 900, 512, 20, 3), (1, 2, 700, 64, 100, 2),
-                                   (2, 3, 1500, 128, 80, 1), (1, 2, 40000, 512, 32, 1)],
+                                   (2, 3, 1500, 128, 80, 1), (1, 2, 40000, 512, 32, 1),
+                                   (1, 2, 700, 64, 32, 1), (1, 8, 4096, 64, 32, 1), (1, 3, 5000, 64, 16, 3)],
                          ids=lambda s: "x".join(map(str, s)))
 def test_d_handoff_stale_workspace(ft, shape):
     """The split backward hands D from the dQ kernel to the dK/dV kernel row by row
