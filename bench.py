@@ -416,6 +416,10 @@ def main():
     kdur = {n: [] for n in names}
     kpass = min(args.steps, 50)
     rec = []
+    # a mixed call runs its head groups on two streams; events chained across them would not
+    # time one launch each, so this pass enqueues every launch on the timed stream
+    prev_serial = os.environ.get("FT_WINATTN_MIXED_SERIAL")
+    os.environ["FT_WINATTN_MIXED_SERIAL"] = "1"
     for _ in range(kpass):
         if flush is not None:
             flush.zero_()
@@ -427,6 +431,10 @@ def main():
             ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
         rec.append((s0, fe, be))
     torch.cuda.synchronize()
+    if prev_serial is None:
+        os.environ.pop("FT_WINATTN_MIXED_SERIAL", None)
+    else:
+        os.environ["FT_WINATTN_MIXED_SERIAL"] = prev_serial
     for s0, fe, be in rec:
         prev = s0
         for n, e1 in zip(names, fe + be):

@@ -96,8 +96,13 @@ ft_status ft_winattn_bwd(const void* q, const void* k, const void* v,
  * with `dilation`, heads [dilated_heads, heads) with dilation 1.  Arguments, layout, ownership
  * and errors are those of ft_winattn_fwd / ft_winattn_bwd, plus FT_ERR_INVALID_VALUE when
  * dilated_heads is outside [0, heads].  The workspace size is ft_winattn_bwd_workspace_bytes
- * of the same shape.  Both head groups are enqueued on `stream` (one launch set per group when
- * batch == 1 or one group is empty, else one per group and batch element). */
+ * of the same shape.  One launch set per head group when batch == 1 or one group is empty,
+ * else one per group and batch element.  The slices are independent and alternate between
+ * `stream` and a side stream the library creates once per device (with two events): the side
+ * stream waits on an event recorded on `stream` before the first slice, and `stream` waits
+ * on the side stream's last slice, so the call stays asynchronous, ordered with respect to
+ * `stream` and capturable in a CUDA graph.  FT_WINATTN_MIXED_SERIAL=1 (environment) keeps
+ * every slice on `stream`. */
 ft_status ft_winattn_fwd_mixed(const void* q, const void* k, const void* v,
                                void* out, float* lse,
                                int64_t batch, int64_t heads, int64_t seq_len, int64_t d,

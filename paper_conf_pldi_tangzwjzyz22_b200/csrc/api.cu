@@ -11,6 +11,7 @@
 #include <string.h>
 
 #include "ft_winattn.h"
+#include <mutex>
 #include "internal.h"
 
 namespace {
@@ -248,6 +249,60 @@ int mixed_groups(int64_t heads, int64_t dilation, int64_t hd, Group (&g)[2]) {
     return n;
 }
 
+// The slices of a mixed call are independent: they alternate between the caller's stream and
+// one library-owned side stream per device (fork / join through events, so the call stays
+// asynchronous and capturable in a CUDA graph). Each slice's persistent kernels then take the
+// SMs the other slice's last CTAs leave, instead of running their own partial last waves one
+// after the other. FT_WINATTN_MIXED_SERIAL=1 keeps every slice on the caller's stream.
+struct Side {
+    cudaStream_t s = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr;
+    bool ok = false;
+};
+Side* side_stream() {
+    const char* e = getenv("FT_WINATTN_MIXED_SERIAL");
+    if (e && atoi(e) == 1) return nullptr;
+    constexpr int MAXDEV = 64;
+    static Side sides[MAXDEV];
+    static std::once_flag once[MAXDEV];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= MAXDEV) return nullptr;
+    std::call_once(once[dev], [dev] {
+        Side& x = sides[dev];
+        x.ok = cudaStreamCreateWithFlags(&x.s, cudaStreamNonBlocking) == cudaSuccess &&
+               cudaEventCreateWithFlags(&x.fork, cudaEventDisableTiming) == cudaSuccess &&
+               cudaEventCreateWithFlags(&x.join, cudaEventDisableTiming) == cudaSuccess;
+    });
+    return sides[dev].ok ? &sides[dev] : nullptr;
+}
+// stream of slice i (fork before the first slice, join after the last)
+struct ForkJoin {
+    Side* side;
+    cudaStream_t main;
+    bool forked = false;
+    ForkJoin(cudaStream_t st, int nslices) : side(nslices > 1 ? side_stream() : nullptr), main(st) {
+        stream_of(1);   // fork now, before any slice is enqueued on the caller's stream
+    }
+    cudaStream_t stream_of(int i) {
+        if (!side || i % 2 == 0) return main;
+        if (!forked) {   // called before slice 0 is enqueued: the side stream must not wait for it
+            cudaEventRecord(side->fork, main);
+            cudaStreamWaitEvent(side->s, side->fork, 0);
+            forked = true;
+        }
+        return side->s;
+    }
+    ft_status finish(ft_status s) {
+        if (forked) {
+            cudaEventRecord(side->join, side->s);
+            cudaStreamWaitEvent(main, side->join, 0);
+            const cudaError_t e = cudaGetLastError();
+            if (s == FT_OK && e != cudaSuccess) return cuda_fail(e);
+        }
+        return s;
+    }
+};
+
 }  // namespace
 
 extern "C" {
@@ -288,17 +343,18 @@ ft_status ft_winattn_fwd_mixed(const void* q, const void* k, const void* v, void
     const size_t e = elt_size(dtype);
     const int64_t nb = ng == 1 ? 1 : batch;   // one group spans the whole batch contiguously
     ftw::prof_reset();
+    ForkJoin fj((cudaStream_t)stream, (int)(nb * ng));
     for (int64_t b = 0; b < nb; ++b) {
         for (int i = 0; i < ng; ++i) {
             const int64_t B1 = ng == 1 ? batch : 1, H1 = ng == 1 ? heads : g[i].nh;
             const int64_t row0 = (b * heads + g[i].h0) * seq_len;   // first (unit, row) of the slice
             const size_t off = (size_t)row0 * d * e;
             s = run_fwd((const char*)q + off, (const char*)k + off, (const char*)v + off, (char*)out + off,
-                        lse + row0, B1, H1, seq_len, d, w, g[i].dil, dtype, stream);
-            if (s != FT_OK) return s;
+                        lse + row0, B1, H1, seq_len, d, w, g[i].dil, dtype, fj.stream_of((int)(b * ng + i)));
+            if (s != FT_OK) return fj.finish(s);
         }
     }
-    return FT_OK;
+    return fj.finish(FT_OK);
 }
 
 ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v, const void* out,
@@ -318,6 +374,7 @@ ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v, cons
     const size_t e = elt_size(dtype);
     const int64_t nb = ng == 1 ? 1 : batch;
     ftw::prof_reset();
+    ForkJoin fj((cudaStream_t)stream, (int)(nb * ng));
     for (int64_t b = 0; b < nb; ++b) {
         for (int i = 0; i < ng; ++i) {
             const int64_t B1 = ng == 1 ? batch : 1, H1 = ng == 1 ? heads : g[i].nh;
@@ -327,11 +384,11 @@ ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v, cons
             s = run_bwd((const char*)q + off, (const char*)k + off, (const char*)v + off, (const char*)out + off,
                         lse + row0, (const char*)dout + off, (char*)dq + off, (char*)dk + off, (char*)dv + off,
                         B1, H1, seq_len, d, w, g[i].dil, dtype, workspace ? (char*)workspace + row0 * 4 : nullptr,
-                        stream);
-            if (s != FT_OK) return s;
+                        fj.stream_of((int)(b * ng + i)));
+            if (s != FT_OK) return fj.finish(s);
         }
     }
-    return FT_OK;
+    return fj.finish(FT_OK);
 }
 
 size_t ft_winattn_tape_bytes(int64_t batch, int64_t heads, int64_t seq_len, int64_t w) {

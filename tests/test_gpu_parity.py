@@ -497,3 +497,45 @@ def test_d_handoff_stale_workspace(ft, shape):
         torch.cuda.synchronize()
         for a, b in zip(got, want):
             assert torch.equal(a, b)
+
+
+@pytest.mark.parametrize("shape", [(1, 4, 1200, 512, 32, 4, 1), (2, 3, 900, 64, 32, 2, 2), (2, 3, 700, 64, 100, 3, 1)],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_mixed_side_stream_and_graph(ft, shape):
+    """ft_winattn_*_mixed runs its head-group slices on the caller's stream and a library side
+    stream (fork / join through events). The result must be bit-identical to the all-on-one-
+    stream schedule (FT_WINATTN_MIXED_SERIAL=1), and the call must be capturable in a CUDA
+    graph whose replay gives the same result again."""
+    B, H, L, d, w, dil, hd = shape
+    sh = WinAttnShape(B, H, L, d, w, dil)
+    x = make_inputs(sh, 31, "bf16")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    with _env(FT_WINATTN_MIXED_SERIAL="1"):
+        o1, l1 = ft.fwd(q, k, v, w, dil, dilated_heads=hd)
+        want = (o1, l1) + ft.bwd(q, k, v, o1, l1, g, w, dil, dilated_heads=hd)
+    o2, l2 = ft.fwd(q, k, v, w, dil, dilated_heads=hd)
+    got = (o2, l2) + ft.bwd(q, k, v, o2, l2, g, w, dil, dilated_heads=hd)
+    torch.cuda.synchronize()
+    for a, b in zip(got, want):
+        assert torch.equal(a, b)
+    # CUDA graph capture of the two-stream call
+    out = torch.empty_like(q)
+    lse = torch.empty((B, H, L), device=dev, dtype=torch.float32)
+    dq, dk, dv = (torch.empty_like(q) for _ in range(3))
+    ws = torch.empty(max(ft.workspace_bytes(q, w, dil), 16), dtype=torch.uint8, device=dev)
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):   # warm-up outside the capture (one-time attribute / stream setup)
+        ft.fwd(q, k, v, w, dil, out=out, lse=lse, dilated_heads=hd)
+    torch.cuda.current_stream().wait_stream(s)
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        ft.fwd(q, k, v, w, dil, out=out, lse=lse, dilated_heads=hd)
+        ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
+    for t in (out, lse, dq, dk, dv):
+        t.zero_()
+    graph.replay()
+    torch.cuda.synchronize()
+    for a, b in zip((out, lse, dq, dk, dv), want):
+        assert torch.equal(a, b)

@@ -14,11 +14,13 @@ CHILD = r"""
 import sys, torch
 sys.path.insert(0, %r)
 import bench, paper_conf_pldi_tangzwjzyz22_b200 as ft
-B, H, L, d, w, dil = bench.WORKLOADS[%r][:6]
+WL = bench.WORKLOADS[%r]
+B, H, L, d, w, dil = WL[:6]
+hd = WL[7] if len(WL) > 7 else None
 dev = torch.device("cuda:0")
 g = torch.Generator(device=dev).manual_seed(0)
 q, k, v, dout = (torch.randn(B, H, L, d, device=dev, dtype=torch.bfloat16, generator=g) for _ in range(4))
-out, lse = ft.fwd(q, k, v, w, dil)
+out, lse = ft.fwd(q, k, v, w, dil, dilated_heads=hd)
 dq, dk, dv = (torch.empty_like(q) for _ in range(3))
 ws = torch.empty(max(ft.workspace_bytes(q, w, dil), 16), dtype=torch.uint8, device=dev)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
@@ -27,8 +29,8 @@ for i in range(60):
     flush.zero_()
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     a.record()
-    ft.fwd(q, k, v, w, dil, out=out, lse=lse)
-    ft.bwd(q, k, v, out, lse, dout, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws)
+    ft.fwd(q, k, v, w, dil, out=out, lse=lse, dilated_heads=hd)
+    ft.bwd(q, k, v, out, lse, dout, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
     b.record()
     torch.cuda.synchronize()
     if i >= 10:
