@@ -88,6 +88,8 @@ struct Params {
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace)
     int two;                     // 1: two MMA issuers (warps 9, 10); 0: warp 9 issues all
     int dpoll;                   // BWDKV: poll D row by row instead of waiting for all of BWDQ
+    int lsepoll;                 // FWD -> BWDQ lse hand-off: FWD marks its lse rows unset and
+                                 // triggers; BWDQ (PDL) and BWDKV poll lse rows
 };
 
 
@@ -217,7 +219,20 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
         __threadfence();
         __syncthreads();
     }
-    if (MODE == BWDQ) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    if (MODE == FWD && p.lsepoll) {
+        // lse hand-off to a following BWDQ launched with PDL: same scheme as D (ld_lse_ready)
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T)) {
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+            for (int i = threadIdx.x; i < BM && T.m0 + i < T.Lr; i += NTHREADS)
+                reinterpret_cast<uint32_t*>(p.lse)[rowbase + (int64_t)(T.m0 + i) * p.dil] = D_UNSET;
+        }
+        __threadfence();
+        __syncthreads();
+    }
+    if (MODE == BWDQ || (MODE == FWD && p.lsepoll))
+        asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const int nkb = NK / KB;
     const int ncw = (d + 255) / 256;            // output chunks
     // BWDKV with d <= 128: dV and dK accumulate side by side ([256, 256+d) and
@@ -514,6 +529,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
         // D of BWDQ: either wait for the whole BWDQ grid, or (dpoll) read each D row as soon
         // as its BWDQ tile has stored it, so BWDKV's first tiles overlap BWDQ's last ones
         if (MODE == BWDKV && !p.dpoll) asm volatile("griddepcontrol.wait;" ::: "memory");
+        bool lse_settled = false;   // ld_lse_ready fell back to griddepcontrol.wait
         while (cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0;
             const int mrow = m0 + t;
@@ -525,7 +541,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 for (int n = t; n < NK; n += 128) {
                     const int mc = kb + n;
                     const bool ok = mc >= 0 && mc < Lr;
-                    colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
+                    colLse[n] = !ok ? 0.f
+                                : p.lsepoll ? ld_D_first(p.lse + rowbase + (int64_t)mc * p.dil)
+                                            : p.lse[rowbase + (int64_t)mc * p.dil];
                     colD[n] = !ok ? 0.f
                               : p.dpoll ? ld_D_first(p.D + rowbase + (int64_t)mc * p.dil)
                                         : p.D[rowbase + (int64_t)mc * p.dil];
@@ -534,6 +552,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     for (int n = t; n < NK; n += 128)
                         if (__float_as_uint(colD[n]) == D_UNSET)
                             colD[n] = ld_D_ready(p.D + rowbase + (int64_t)(kb + n) * p.dil);
+                for (int n = t; n < NK; n += 128) {   // lse rows FWD had not stored yet
+                    if (p.lsepoll && __float_as_uint(colLse[n]) == D_UNSET)
+                        colLse[n] = ld_lse_ready(p.lse + rowbase + (int64_t)(kb + n) * p.dil, lse_settled);
+                    colLse[n] *= LOG2E;
+                }
                 named_bar_sync(1, 128);
             }
             mbar_wait(s_full, j & 1);
@@ -570,7 +593,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 mbar_arrive(p_full);
                 if (mrow < Lr) p.lse[rowbase + (int64_t)mrow * p.dil] = (mxs + log2f(sum)) * LN2;
             } else if (MODE == BWDQ) {
-                const float lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
+                const float lse2 = mrow >= Lr ? 0.f
+                                   : (p.lsepoll ? ld_lse_ready(p.lse + rowbase + (int64_t)mrow * p.dil, lse_settled)
+                                                : p.lse[rowbase + (int64_t)mrow * p.dil]) * LOG2E;
                 float D = 0.f;
                 for (int c = c_lo; c <= c_hi; ++c) {   // pass 1: D = sum_j P_ij dP_ij
                     uint32_t rs[32], rd[32];
@@ -685,6 +710,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 const int nsl_c = (dual ? 2 : 1) * cw / 64;
                 mbar_wait(o_full, ga & 1);
                 tc_fence_after();
+                // BWDQ launched early (lse hand-off): its first global store waits for the
+                // preceding grid, so stream order holds for every buffer it writes
+                if (MODE == BWDQ && p.lsepoll && ga == 0) asm volatile("griddepcontrol.wait;" ::: "memory");
                 if (lane == 0 && ew == 0 && a == 0) trace_ev(p, j, 8);
                 // Drain the accumulator 128 columns at a time: both 64-column halves are
                 // loaded before the wait, and o_empty is released as soon as every column is
@@ -762,6 +790,12 @@ bool pdl_enabled() {
     return !(e && atoi(e) == 0);
 }
 
+// FT_WINATTN_LSEPOLL=0: no FWD -> BWDQ lse hand-off (BWDQ waits for the whole preceding grid)
+static int lsepoll_enabled() {
+    const char* e = getenv("FT_WINATTN_LSEPOLL");
+    return pdl_enabled() && dpoll_enabled() && !(e && atoi(e) == 0);
+}
+
 int num_sms() {
     static int n = 0;
     static std::once_flag once;
@@ -828,13 +862,15 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
             p.two = !(e && atoi(e) == 1);
         }
         p.dpoll = MODE != FWD && dpoll_enabled();
+        p.lsepoll = lsepoll_enabled() && r0 == 0;
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms() ? total : num_sms()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_smem_bytes<MODE>(NK) + (size_t)nst * slot_bytes(NK);
-        if (MODE == BWDKV && r0 == 0 && pdl_enabled()) {
-            // BWDKV directly follows this call's last BWDQ launch on the stream
+        if (MODE != FWD && r0 == 0 && pdl_enabled() && (MODE == BWDKV || p.lsepoll)) {
+            // BWDKV directly follows this call's last BWDQ launch on the stream; BWDQ
+            // (lse hand-off) typically follows the forward's band launch
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = grid;
             cfg.blockDim = dim3(NTHREADS);

@@ -380,6 +380,25 @@ __device__ __forceinline__ float ld_D_first(const float* ptr) {
     return __uint_as_float(x);
 }
 
+// lse hand-off (forward band kernel -> dQ kernel): the forward's CTAs mark their lse rows
+// D_UNSET before triggering.  Unlike D, lse is a caller's buffer that may hold any bits when
+// the preceding grid is not that forward, so the poll is bounded: after ~1 ms it waits for
+// the preceding grid to complete (griddepcontrol.wait) and takes the value as stored;
+// `settled` remembers that wait, after which every value is final and read once.
+__device__ __forceinline__ float ld_lse_ready(const float* ptr, bool& settled) {
+    uint32_t x;
+    for (int i = 0; i < (settled ? 1 : 8192); ++i) {
+        asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr) : "memory");
+        if (x != D_UNSET) return __uint_as_float(x);
+        __nanosleep(128);
+    }
+    if (settled) return __uint_as_float(x);
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    settled = true;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr) : "memory");
+    return __uint_as_float(x);
+}
+
 // FT_WINATTN_DPOLL=0: the dK/dV kernel waits for the whole dQ grid instead (A/B timing)
 inline bool dpoll_enabled() {
     const char* e = getenv("FT_WINATTN_DPOLL");

@@ -499,6 +499,45 @@ def test_d_handoff_stale_workspace(ft, shape):
             assert torch.equal(a, b)
 
 
+@pytest.mark.parametrize("shape", [(1, 2, 700, 512, 32, 1), (1, 3, 900, 512, 20, 3), (1, 8, 10000, 512, 32, 1),
+                                   (1, 2, 3000, 512, 32, 11), (2, 3, 1500, 128, 48, 1)],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_lse_handoff(ft, shape):
+    """The band forward marks its lse rows unset and triggers a programmatic dependent launch
+    of the dQ kernel, which polls lse row by row (tc_common.cuh ld_lse_ready; DESIGN.md
+    'lse hand-off'). Directly after its own forward, after the forward of OTHER inputs (so
+    the polled lse is a different, complete buffer), and with an lse buffer that holds the
+    unset marker itself (bounded poll, then a grid-wide wait: must not hang), the results must
+    be bit-identical to the schedule without the hand-off (FT_WINATTN_LSEPOLL=0)."""
+    sh = WinAttnShape(*shape)
+    x = make_inputs(sh, 41, "bf16")
+    y = make_inputs(sh, 42, "bf16")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    q2, k2, v2 = (y[n].to(dev) for n in ("q", "k", "v"))
+    with _env(FT_WINATTN_LSEPOLL="0"):
+        o0, l0 = ft.fwd(q, k, v, sh.w, sh.dilation)
+        want = ft.bwd(q, k, v, o0, l0, g, sh.w, sh.dilation)
+        bad = torch.full_like(l0, float("nan")).view(torch.int32).fill_(-1).view(torch.float32)
+        want_bad = ft.bwd(q, k, v, o0, bad, g, sh.w, sh.dilation)
+    o1, l1 = ft.fwd(q, k, v, sh.w, sh.dilation)
+    got = ft.bwd(q, k, v, o1, l1, g, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    assert torch.equal(o1, o0) and torch.equal(l1, l0)
+    for a, b in zip(got, want):
+        assert torch.equal(a, b)
+    ft.fwd(q2, k2, v2, sh.w, sh.dilation)   # another problem's forward precedes the backward
+    got = ft.bwd(q, k, v, o0, l0, g, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    for a, b in zip(got, want):
+        assert torch.equal(a, b)
+    ft.fwd(q2, k2, v2, sh.w, sh.dilation)
+    got = ft.bwd(q, k, v, o0, bad, g, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    for a, b in zip(got, want_bad):
+        assert torch.equal(a.isnan(), b.isnan())
+
+
 @pytest.mark.parametrize("shape", [(1, 4, 1200, 512, 32, 4, 1), (2, 3, 900, 64, 32, 2, 2), (2, 3, 700, 64, 100, 3, 1)],
                          ids=lambda s: "x".join(map(str, s)))
 def test_mixed_side_stream_and_graph(ft, shape):
