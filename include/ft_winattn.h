@@ -30,7 +30,12 @@
  * overwritten, never accumulated into.
  *
  * Async: work is enqueued on `stream` (a cudaStream_t passed as void*; NULL = legacy
- * default stream) and the call returns immediately.
+ * default stream) and the call returns immediately.  Stream order is preserved for the
+ * caller.  Inside a forward -> backward pair on one stream, the backward's first kernel may
+ * start while the forward drains (programmatic dependent launch).  It reads lse rows as the
+ * forward stores them and writes nothing the caller can see before the forward completes
+ * ("lse hand-off").  While a forward runs, its lse rows temporarily hold the
+ * bit pattern 0xFFFFFFFF.
  *
  * Errors: all argument checks run before any launch; on failure nothing is launched
  * and the outputs are untouched.
