@@ -790,12 +790,6 @@ bool pdl_enabled() {
     return !(e && atoi(e) == 0);
 }
 
-// FT_WINATTN_LSEPOLL=0: no FWD -> BWDQ lse hand-off (BWDQ waits for the whole preceding grid)
-static int lsepoll_enabled() {
-    const char* e = getenv("FT_WINATTN_LSEPOLL");
-    return pdl_enabled() && dpoll_enabled() && !(e && atoi(e) == 0);
-}
-
 int num_sms() {
     static int n = 0;
     static std::once_flag once;
@@ -862,9 +856,9 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
             p.two = !(e && atoi(e) == 1);
         }
         p.dpoll = MODE != FWD && dpoll_enabled();
-        p.lsepoll = lsepoll_enabled() && r0 == 0;
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
+        p.lsepoll = lsepoll_enabled() && r0 == 0 && lsepoll_worth(total, num_sms());
         dim3 grid((unsigned)(total < num_sms() ? total : num_sms()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_smem_bytes<MODE>(NK) + (size_t)nst * slot_bytes(NK);

@@ -399,6 +399,19 @@ __device__ __forceinline__ float ld_lse_ready(const float* ptr, bool& settled) {
     return __uint_as_float(x);
 }
 
+// FT_WINATTN_LSEPOLL=0: no forward -> dQ-kernel lse hand-off (also off with DPOLL=0 or PDL=0)
+inline bool lsepoll_enabled() {
+    const char* e = getenv("FT_WINATTN_LSEPOLL");
+    const char* d = getenv("FT_WINATTN_DPOLL");
+    const char* p = getenv("FT_WINATTN_PDL");
+    return !(e && atoi(e) == 0) && !(d && atoi(d) == 0) && !(p && atoi(p) == 0);
+}
+
+// The hand-off pays only when the forward's last partial wave is a visible share of it: with
+// many tiles per SM the forward's marking pass costs more than the overlap gains (narrow
+// C5_w32, 110 tiles per SM: forward 0.176 -> 0.194 ms).  Used by both sides of a call.
+inline bool lsepoll_worth(int64_t tiles, int sms) { return tiles < 8 * (int64_t)sms; }
+
 // FT_WINATTN_DPOLL=0: the dK/dV kernel waits for the whole dQ grid instead (A/B timing)
 inline bool dpoll_enabled() {
     const char* e = getenv("FT_WINATTN_DPOLL");

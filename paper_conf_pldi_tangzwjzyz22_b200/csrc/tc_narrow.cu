@@ -67,6 +67,7 @@ struct NParams {
     int64_t L;
     int w, dil;
     SchedParams sc;
+    int lsepoll;   // lse hand-off to the narrow dQ kernel (tc_common.cuh ld_lse_ready)
 };
 
 using Tile = SchedTile;
@@ -97,6 +98,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_fwd_kernel(const __grid
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int w = p.w;
 
+    if (p.lsepoll) {   // lse rows unset, then let the dQ kernel (PDL) launch
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T)) {
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+            for (int i = threadIdx.x; i < BM && T.m0 + i < T.Lr; i += NTHREADS)
+                reinterpret_cast<uint32_t*>(p.lse)[rowbase + (int64_t)(T.m0 + i) * p.dil] = D_UNSET;
+        }
+        __threadfence();
+        __syncthreads();
+        asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    }
     if (warp == 8) {
         if (lane == 0) {
             for (int i = 0; i < NSTAGE; ++i) {
@@ -351,6 +364,9 @@ cudaError_t tc_narrow_fwd(const void* q, const void* k, const void* v, void* out
         const int64_t Lr0 = ceil_div(L - r0, dil);
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
+        // only when the split backward (NQ, PDL-launched) follows; the fused one is not
+        p.lsepoll = r0 == 0 && lsepoll_enabled() && lsepoll_worth(total, num_sms_n()) &&
+                    !tc_narrow_fused_ok(units, L, d, w, dil);
         dim3 grid((unsigned)(total < num_sms_n() ? total : num_sms_n()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         tc_narrow_fwd_kernel<<<grid, NTHREADS, SMEM_BYTES, st>>>(p);

@@ -88,6 +88,7 @@ struct BParams {
     SchedParams sc;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, modes 1 / 2)
     int dpoll;                   // D hand-off by row polling (tc_common.cuh ld_D_ready)
+    int lsepoll;                 // lse hand-off from the narrow forward (ld_lse_ready)
 };
 
 // Phase trace: per CTA and local tile j < 8, clock64 stamps (tools/trace_narrow.py).
@@ -350,6 +351,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
         TileCursor cur(p.sc), nxt(p.sc);
         Tile T, Tn;
         bool hn = nxt.next(p.sc, Tn);
+        bool lse_settled = false;   // ld_lse_ready fell back to griddepcontrol.wait
+        bool first_store = true;    // NQ launched early: wait for the preceding grid first
         auto prefetch = [&](const Tile& X, int jx) {
             const int64_t rb = (int64_t)X.u * p.L + X.r;
             if (MODE == NKV) {
@@ -382,6 +385,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             c.Lr = X.Lr; c.m0 = X.m0; c.kb = X.m0 - w; c.u = X.u; c.rl = X.rl;
             c.rowbase = (int64_t)X.u * p.L + X.r;
             cp_async_wait_all();   // this tile's values (copied a tile ago)
+            if (p.lsepoll) {   // lse rows the forward had not stored yet
+                if (MODE == NQ) {
+                    float* cl = lpre + (jx & 1) * 256 + threadIdx.x;
+                    if (__float_as_uint(*cl) == D_UNSET)
+                        *cl = ld_lse_ready(p.lse + c.rowbase + (int64_t)(c.m0 + t) * p.dil, lse_settled);
+                } else if (threadIdx.x < NK) {
+                    float* cl = colv + (jx & 1) * 2 * NK + threadIdx.x;
+                    if (__float_as_uint(*cl) == D_UNSET)
+                        *cl = ld_lse_ready(p.lse + c.rowbase + (int64_t)(c.kb + (int)threadIdx.x) * p.dil, lse_settled);
+                }
+            }
             if (MODE == NKV && p.dpoll && threadIdx.x < NK) {   // D rows NQ had not stored yet
                 float* cd = colv + (jx & 1) * 2 * NK + NK + threadIdx.x;
                 if (__float_as_uint(*cd) == D_UNSET)
@@ -404,6 +418,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             mbar_wait(&acc_full[b], MODE == NQ ? (i >> 1) & 1 : i & 1);
             tc_fence_after();
             if (threadIdx.x == 0) trace_ev(p, i, 9);
+            if (MODE == NQ && p.lsepoll && first_store) {
+                asm volatile("griddepcontrol.wait;" ::: "memory");
+                first_store = false;
+            }
             if (MODE == NQ) {
                 uint32_t ov[32];
                 tmem_ld32(tbase + lane_off + TACC + 64u * b + 32u * h, ov);
@@ -592,7 +610,8 @@ cudaError_t launch_nb(const void* a1, const void* a2, const void* b1, const void
         dim3 grid((unsigned)(total < num_sms_nb() ? total : num_sms_nb()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         p.dpoll = dpoll_enabled();
-        if (MODE == NKV && r0 == 0 && p.dpoll) {
+        p.lsepoll = r0 == 0 && lsepoll_enabled() && lsepoll_worth(total, num_sms_nb());
+        if (r0 == 0 && ((MODE == NKV && p.dpoll) || (MODE == NQ && p.lsepoll))) {
             // NKV directly follows this call's last NQ launch: programmatic dependent launch,
             // D handed over row by row
             cudaLaunchConfig_t cfg = {};

@@ -500,11 +500,13 @@ def test_d_handoff_stale_workspace(ft, shape):
 
 
 @pytest.mark.parametrize("shape", [(1, 2, 700, 512, 32, 1), (1, 3, 900, 512, 20, 3), (1, 8, 10000, 512, 32, 1),
-                                   (1, 2, 3000, 512, 32, 11), (2, 3, 1500, 128, 48, 1)],
+                                   (1, 2, 3000, 512, 32, 11), (2, 3, 1500, 128, 48, 1),
+                                   (1, 8, 4096, 64, 32, 1), (1, 2, 700, 64, 32, 1), (1, 3, 5000, 64, 16, 3),
+                                   (1, 48, 2048, 64, 32, 1)],
                          ids=lambda s: "x".join(map(str, s)))
 def test_lse_handoff(ft, shape):
-    """The band forward marks its lse rows unset and triggers a programmatic dependent launch
-    of the dQ kernel, which polls lse row by row (tc_common.cuh ld_lse_ready; DESIGN.md
+    """The band and narrow forwards mark their lse rows unset and trigger a programmatic
+    dependent launch of the dQ kernel, which polls lse row by row (tc_common.cuh ld_lse_ready; DESIGN.md
     'lse hand-off'). Directly after its own forward, after the forward of OTHER inputs (so
     the polled lse is a different, complete buffer), and with an lse buffer that holds the
     unset marker itself (bounded poll, then a grid-wide wait: must not hang), the results must
