@@ -81,10 +81,9 @@ def kernel_bytes_per_row(kind: str, d: int, e: int) -> int:
     fwd : read q, k, v ; write o (dtype) and lse (fp32)                 = 4de + 4
     bwdA: read q, k, v, dout, lse ; write dq, D                          = 5de + 8
     bwdB: read q, k, v, dout, lse, D ; write dk, dv                      = 6de + 8
-    rowdot (wide windows): read dout, o ; write D                        = 2de + 4
-    bwdF (d = 64, w <= 32, one kernel): read q, k, v, dout, lse ; write dq, dk, dv = 7de + 4"""
+    rowdot (wide windows): read dout, o ; write D                        = 2de + 4"""
     return {"fwd": 4 * d * e + 4, "bwdA": 5 * d * e + 8, "bwdB": 6 * d * e + 8,
-            "rowdot": 2 * d * e + 4, "bwdF": 7 * d * e + 4}[kind]
+            "rowdot": 2 * d * e + 4}[kind]
 
 
 def step_bytes_per_row(d: int, e: int) -> int:
@@ -109,10 +108,7 @@ def launch_table(ft, B, H, L, d, w, dil, code):
 
     res = 8 if min(w, L) <= 64 else 4
     fwd = [("fwd", r) for r in (split(nf, res) if path_f == ft.PATH_TC else [rows] * nf)]
-    groups = -(-nres // res)
-    if path_b == ft.PATH_TC and nb == groups and d == 64 and min(w, L) <= 32:
-        bwd = [("bwdF", r) for r in split(nb, 8)]        # fused d = 64 backward (tc_narrow_fused.cu)
-    elif path_b == ft.PATH_TC:
+    if path_b == ft.PATH_TC:
         pre = nb % 2                                     # wide windows: optional rowdot pre-pass
         g = (nb - pre) // 2
         per = split(g, res)
@@ -418,8 +414,8 @@ def main():
     rec = []
     # a mixed call runs its head groups on two streams; events chained across them would not
     # time one launch each, so this pass enqueues every launch on the timed stream
-    prev_serial = os.environ.get("FT_WINATTN_MIXED_SERIAL")
-    os.environ["FT_WINATTN_MIXED_SERIAL"] = "1"
+    serial = ft.knobs(side=0)
+    serial.__enter__()
     for _ in range(kpass):
         if flush is not None:
             flush.zero_()
@@ -431,10 +427,7 @@ def main():
             ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
         rec.append((s0, fe, be))
     torch.cuda.synchronize()
-    if prev_serial is None:
-        os.environ.pop("FT_WINATTN_MIXED_SERIAL", None)
-    else:
-        os.environ["FT_WINATTN_MIXED_SERIAL"] = prev_serial
+    serial.__exit__()
     for s0, fe, be in rec:
         prev = s0
         for n, e1 in zip(names, fe + be):

@@ -31,11 +31,12 @@
  *
  * Async: work is enqueued on `stream` (a cudaStream_t passed as void*; NULL = legacy
  * default stream) and the call returns immediately.  Stream order is preserved for the
- * caller.  Inside a forward -> backward pair on one stream, the backward's first kernel may
- * start while the forward drains (programmatic dependent launch).  It reads lse rows as the
- * forward stores them and writes nothing the caller can see before the forward completes
- * ("lse hand-off").  While a forward runs, its lse rows temporarily hold the
- * bit pattern 0xFFFFFFFF.
+ * caller: every kernel of a call starts after all work enqueued on `stream` before the call
+ * has completed, and work enqueued after the call starts after it.  Inside ONE call the
+ * library may overlap its own kernels (programmatic dependent launch: ft_winattn_bwd's dK/dV
+ * kernel reads D rows as its dQ kernel stores them; ft_winattn_fwd_bwd's dQ kernel reads lse
+ * rows as its forward stores them), never across calls.  No kernel of a call reads an input
+ * or writes any memory before the previous work on `stream` is complete.
  *
  * Errors: all argument checks run before any launch; on failure nothing is launched
  * and the outputs are untouched.
@@ -59,7 +60,7 @@
 extern "C" {
 #endif
 
-#define FT_WINATTN_ABI_VERSION 1
+#define FT_WINATTN_ABI_VERSION 2
 
 typedef enum {
     FT_OK = 0,
@@ -71,8 +72,8 @@ typedef enum {
 
 typedef enum { FT_F32 = 0, FT_BF16 = 1 } ft_dtype;
 
-/* Kernel family chosen for a call (reported by ft_winattn_plan; tests may force one
- * through the environment variable FT_WINATTN_PATH=simt|tc). */
+/* Kernel family chosen for a call (reported by ft_winattn_plan; tests may force one with
+ * ft_winattn_debug_set(FT_KNOB_PATH, ...)). */
 typedef enum {
     FT_PATH_SIMT = 0,   /* CUDA-core FMA kernels (fp32 math), any dtype / d / w      */
     FT_PATH_TC = 1      /* tcgen05/TMEM tensor-core kernels, bf16 only               */
@@ -96,6 +97,20 @@ ft_status ft_winattn_bwd(const void* q, const void* k, const void* v,
                          int64_t w, int64_t dilation, ft_dtype dtype,
                          void* workspace, size_t workspace_bytes, void* stream);
 
+/* Forward then backward in one call, for the recompute / activation-checkpointing pattern
+ * (the gradient program of PAPER.md:449, 523 as one unit): computes out and lse exactly as
+ * ft_winattn_fwd and dq, dk, dv exactly as ft_winattn_bwd with that out and lse.  Inputs q, k,
+ * v, dout; outputs out, lse, dq, dk, dv, workspace (ft_winattn_bwd_workspace_bytes).  Because
+ * both halves are enqueued by the library, its dQ kernel may start while the forward drains and
+ * read each lse row as the forward stores it (the forward marks its lse rows with the bit
+ * pattern 0xFFFFFFFF first; DESIGN.md §7 "lse hand-off").  Errors: those of ft_winattn_fwd and
+ * ft_winattn_bwd, plus FT_ERR_INVALID_VALUE when dout overlaps out or lse. */
+ft_status ft_winattn_fwd_bwd(const void* q, const void* k, const void* v, const void* dout,
+                             void* out, float* lse, void* dq, void* dk, void* dv,
+                             int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                             int64_t w, int64_t dilation, ft_dtype dtype,
+                             void* workspace, size_t workspace_bytes, void* stream);
+
 /* Per-head dilation (Longformer [8] and the FreeTensor artefact's mixed heads, PAPER.md:625;
  * SURVEY.md §8(f) item 1, reading A4): heads [0, dilated_heads) of every batch element attend
  * with `dilation`, heads [dilated_heads, heads) with dilation 1.  Arguments, layout, ownership
@@ -103,11 +118,12 @@ ft_status ft_winattn_bwd(const void* q, const void* k, const void* v,
  * dilated_heads is outside [0, heads].  The workspace size is ft_winattn_bwd_workspace_bytes
  * of the same shape.  One launch set per head group when batch == 1 or one group is empty,
  * else one per group and batch element.  The slices are independent and alternate between
- * `stream` and a side stream the library creates once per device (with two events): the side
+ * `stream` and a side stream the library creates per host thread and device (with two events): the side
  * stream waits on an event recorded on `stream` before the first slice, and `stream` waits
  * on the side stream's last slice, so the call stays asynchronous, ordered with respect to
- * `stream` and capturable in a CUDA graph.  FT_WINATTN_MIXED_SERIAL=1 (environment) keeps
- * every slice on `stream`. */
+ * `stream` and capturable in a CUDA graph.  The side stream and events belong to the calling
+ * host thread (one set per thread and device).  FT_KNOB_SIDE = 0 keeps every slice on
+ * `stream`. */
 ft_status ft_winattn_fwd_mixed(const void* q, const void* k, const void* v,
                                void* out, float* lse,
                                int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
@@ -168,6 +184,23 @@ ft_status ft_winattn_profile_events(void* const* events, int n);
  * csrc/tc_wide.cu).  The buffer must hold 148*8*48*8 bytes per SM-sized grid.  Profiling
  * only. */
 ft_status ft_winattn_debug_trace(int kernel_mode, void* device_buffer);
+
+/* Debug / A-B knobs (tests and profiling only; process-wide, initialised once from the
+ * environment variable named in brackets).  Every setting computes the same result; they select
+ * among kernel families or launch schedules:
+ *   0 FT_KNOB_PATH    0 auto, 1 CUDA-core kernels, 2 tensor-core kernels (FT_ERR_NOT_SUPPORTED
+ *                     from calls they cannot serve)              [FT_WINATTN_PATH=simt|tc]
+ *   1 FT_KNOB_PDL     1 programmatic dependent launch inside a call, 0 plain stream order
+ *                                                                [FT_WINATTN_PDL=0]
+ *   2 FT_KNOB_NARROW  1 the d = 64, w <= 32 kernels, 0 the band kernels  [FT_WINATTN_NARROW=0]
+ *   3 FT_KNOB_WIDE    1 the w > 64 wide kernels, 0 the chunked fallback  [FT_WINATTN_WIDE=0]
+ *   4 FT_KNOB_SIDE    1 per-head-dilation calls use a side stream, 0 serial
+ *                                                                [FT_WINATTN_MIXED_SERIAL=1]
+ * ft_winattn_debug_set returns FT_ERR_INVALID_VALUE for an unknown knob or value;
+ * ft_winattn_debug_get returns the current value (-1 for an unknown knob). */
+enum { FT_KNOB_PATH = 0, FT_KNOB_PDL = 1, FT_KNOB_NARROW = 2, FT_KNOB_WIDE = 3, FT_KNOB_SIDE = 4 };
+ft_status ft_winattn_debug_set(int knob, int value);
+int       ft_winattn_debug_get(int knob);
 
 /* Human-readable text for a status (static storage, never NULL).  For FT_ERR_CUDA it
  * includes the CUDA error string of the last failure on the calling thread. */

@@ -18,7 +18,7 @@ import os
 
 import torch
 
-__all__ = ["fwd", "bwd", "fwd_tape", "bwd_tape", "tape_bytes", "plan", "profile_events", "WinAttn", "win_attn", "lib_path", "load_library",
+__all__ = ["fwd", "bwd", "fwd_bwd", "knobs", "debug_set", "debug_get", "fwd_tape", "bwd_tape", "tape_bytes", "plan", "profile_events", "WinAttn", "win_attn", "lib_path", "load_library",
            "FT_F32", "FT_BF16", "PATH_SIMT", "PATH_TC", "FtError"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -62,6 +62,12 @@ def load_library(build_if_missing: bool = False):
     lib.ft_winattn_fwd.restype = ctypes.c_int
     lib.ft_winattn_bwd.argtypes = [vp] * 9 + [i64] * 6 + [ctypes.c_int, vp, sz, vp]
     lib.ft_winattn_bwd.restype = ctypes.c_int
+    lib.ft_winattn_fwd_bwd.argtypes = [vp] * 9 + [i64] * 6 + [ctypes.c_int, vp, sz, vp]
+    lib.ft_winattn_fwd_bwd.restype = ctypes.c_int
+    lib.ft_winattn_debug_set.argtypes = [ctypes.c_int, ctypes.c_int]
+    lib.ft_winattn_debug_set.restype = ctypes.c_int
+    lib.ft_winattn_debug_get.argtypes = [ctypes.c_int]
+    lib.ft_winattn_debug_get.restype = ctypes.c_int
     lib.ft_winattn_fwd_mixed.argtypes = [vp, vp, vp, vp, fp] + [i64] * 7 + [ctypes.c_int, vp]
     lib.ft_winattn_fwd_mixed.restype = ctypes.c_int
     lib.ft_winattn_bwd_mixed.argtypes = [vp] * 9 + [i64] * 7 + [ctypes.c_int, vp, sz, vp]
@@ -85,6 +91,39 @@ def load_library(build_if_missing: bool = False):
     lib.ft_winattn_profile_events.restype = ctypes.c_int
     _lib = lib
     return lib
+
+
+_KNOBS = {"path": 0, "pdl": 1, "narrow": 2, "wide": 3, "side": 4}
+_PATHS = {"auto": 0, "simt": 1, "tc": 2}
+
+
+def debug_set(name: str, value) -> None:
+    """Set a debug / A-B knob of include/ft_winattn.h (path: auto|simt|tc; pdl, narrow, wide,
+    side: 0|1).  Process-wide; every setting computes the same result."""
+    v = _PATHS[value] if name == "path" and isinstance(value, str) else int(value)
+    _check(load_library().ft_winattn_debug_set(_KNOBS[name], v))
+
+
+def debug_get(name: str) -> int:
+    return int(load_library().ft_winattn_debug_get(_KNOBS[name]))
+
+
+class knobs:
+    """Context manager: ``with knobs(path="simt", pdl=0): ...`` sets debug knobs and restores
+    the previous values on exit."""
+
+    def __init__(self, **kv):
+        self.kv = kv
+
+    def __enter__(self):
+        self.old = {k: debug_get(k) for k in self.kv}
+        for k, v in self.kv.items():
+            debug_set(k, v)
+        return self
+
+    def __exit__(self, *a):
+        for k, v in self.old.items():
+            debug_set(k, v)
 
 
 def _dtype_code(t: torch.Tensor) -> int:
@@ -205,6 +244,28 @@ def bwd(q, k, v, out, lse, dout, w: int, dilation: int = 1, dq=None, dk=None, dv
     return dq, dk, dv
 
 
+def fwd_bwd(q, k, v, dout, w: int, dilation: int = 1, out=None, lse=None, dq=None, dk=None, dv=None,
+            workspace: torch.Tensor | None = None):
+    """Forward then backward in one call (ft_winattn_fwd_bwd; the recompute / checkpointing
+    pattern): returns (out, lse, dq, dk, dv).  Inside the call the dQ kernel may read each lse
+    row as the forward stores it."""
+    _check_inputs(q, k, v, dout)
+    B, H, L, d = q.shape
+    out = torch.empty_like(q) if out is None else out
+    lse = torch.empty((B, H, L), dtype=torch.float32, device=q.device) if lse is None else lse
+    dq = torch.empty_like(q) if dq is None else dq
+    dk = torch.empty_like(q) if dk is None else dk
+    dv = torch.empty_like(q) if dv is None else dv
+    wsb = workspace_bytes(q, w, dilation)
+    if workspace is None or workspace.numel() * workspace.element_size() < wsb:
+        workspace = torch.empty(max(wsb, 16), dtype=torch.uint8, device=q.device)
+    _check(load_library().ft_winattn_fwd_bwd(
+        q.data_ptr(), k.data_ptr(), v.data_ptr(), dout.data_ptr(), out.data_ptr(), lse.data_ptr(),
+        dq.data_ptr(), dk.data_ptr(), dv.data_ptr(), B, H, L, d, int(w), int(dilation), _dtype_code(q),
+        workspace.data_ptr(), workspace.numel() * workspace.element_size(), _stream(q.device)))
+    return out, lse, dq, dk, dv
+
+
 def tape_bytes(q: torch.Tensor, w: int) -> int:
     B, H, L, _ = q.shape
     return int(load_library().ft_winattn_tape_bytes(B, H, L, int(w)))
@@ -246,8 +307,10 @@ class WinAttn(torch.autograd.Function):
 
     @staticmethod
     def forward(ctx, q, k, v, w: int, dilation: int = 1, dilated_heads: int | None = None):
-        out, lse = fwd(q.contiguous(), k.contiguous(), v.contiguous(), w, dilation,
-                       dilated_heads=dilated_heads)
+        # the kernels take contiguous [B, H, L, d]: save the copies they read (a common layout,
+        # x.view(B, L, H, d).transpose(1, 2), is not contiguous)
+        q, k, v = q.contiguous(), k.contiguous(), v.contiguous()
+        out, lse = fwd(q, k, v, w, dilation, dilated_heads=dilated_heads)
         ctx.save_for_backward(q, k, v, out, lse)
         ctx.w, ctx.dilation, ctx.dilated_heads = w, dilation, dilated_heads
         return out

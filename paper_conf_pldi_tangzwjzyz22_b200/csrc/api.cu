@@ -11,6 +11,7 @@
 #include <string.h>
 
 #include "ft_winattn.h"
+#include <atomic>
 #include <mutex>
 #include "internal.h"
 
@@ -50,14 +51,26 @@ struct Span {
 };
 bool overlap(Span a, Span b) { return a.lo < b.hi && b.lo < a.hi; }
 
-// 0 = auto, 1 = force SIMT, 2 = force tensor cores (test-only override).
-int forced_path() {
-    const char* s = getenv("FT_WINATTN_PATH");
-    if (!s || !*s) return 0;
-    if (!strcmp(s, "simt")) return 1;
-    if (!strcmp(s, "tc")) return 2;
-    return 0;
+// Debug / A-B knobs (ft_winattn_debug_set), initialised once from the environment.
+std::atomic<int> g_knob[ftw::K_NUM];
+std::once_flag g_knob_once;
+int env_int(const char* name, int dflt) {
+    const char* s = getenv(name);
+    return (s && *s) ? atoi(s) : dflt;
 }
+void knob_init() {
+    std::call_once(g_knob_once, [] {
+        const char* s = getenv("FT_WINATTN_PATH");
+        g_knob[ftw::K_PATH] = (s && !strcmp(s, "simt")) ? 1 : (s && !strcmp(s, "tc")) ? 2 : 0;
+        g_knob[ftw::K_PDL] = env_int("FT_WINATTN_PDL", 1) != 0;
+        g_knob[ftw::K_NARROW] = env_int("FT_WINATTN_NARROW", 1) != 0;
+        g_knob[ftw::K_WIDE] = env_int("FT_WINATTN_WIDE", 1) != 0;
+        g_knob[ftw::K_SIDE] = env_int("FT_WINATTN_MIXED_SERIAL", 0) != 1;
+    });
+}
+thread_local bool g_handoff = false;   // inside ft_winattn_fwd_bwd
+
+int forced_path() { return ftw::knob(ftw::K_PATH); }
 
 ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil, ft_dtype dt,
                       int* path) {
@@ -77,6 +90,11 @@ ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w
 }  // namespace
 
 namespace ftw {
+int knob(Knob k) {
+    knob_init();
+    return g_knob[k].load(std::memory_order_relaxed);
+}
+bool call_handoff() { return g_handoff; }
 ft_status cuda_error(cudaError_t e) { return cuda_fail(e); }
 void prof_reset() { g_prof_i = 0; }
 void* trace_buffer(int mode) { return (mode >= 0 && mode < 3) ? g_trace[mode] : nullptr; }
@@ -103,6 +121,19 @@ ft_status ft_winattn_profile_events(void* const* events, int n) {
 }
 
 int ft_winattn_abi_version(void) { return FT_WINATTN_ABI_VERSION; }
+
+ft_status ft_winattn_debug_set(int which, int value) {
+    if (which < 0 || which >= ftw::K_NUM) return FT_ERR_INVALID_VALUE;
+    if (which == ftw::K_PATH ? (value < 0 || value > 2) : (value < 0 || value > 1)) return FT_ERR_INVALID_VALUE;
+    knob_init();
+    g_knob[which].store(value, std::memory_order_relaxed);
+    return FT_OK;
+}
+
+int ft_winattn_debug_get(int which) {
+    if (which < 0 || which >= ftw::K_NUM) return -1;
+    return ftw::knob((ftw::Knob)which);
+}
 
 const char* ft_status_str(ft_status s) {
     switch (s) {
@@ -259,21 +290,34 @@ struct Side {
     cudaEvent_t fork = nullptr, join = nullptr;
     bool ok = false;
 };
+// One side stream and fork / join event pair per host thread and device: two threads calling
+// concurrently never share the events (a record on one thread's stream could otherwise be
+// overwritten by the other's before the wait is enqueued).  They live for the thread.
 Side* side_stream() {
-    const char* e = getenv("FT_WINATTN_MIXED_SERIAL");
-    if (e && atoi(e) == 1) return nullptr;
+    if (!ftw::knob(ftw::K_SIDE)) return nullptr;
     constexpr int MAXDEV = 64;
-    static Side sides[MAXDEV];
-    static std::once_flag once[MAXDEV];
+    struct PerThread {
+        Side sides[MAXDEV];
+        bool tried[MAXDEV] = {};
+        ~PerThread() {
+            for (Side& x : sides) {
+                if (x.fork) cudaEventDestroy(x.fork);
+                if (x.join) cudaEventDestroy(x.join);
+                if (x.s) cudaStreamDestroy(x.s);
+            }
+        }
+    };
+    thread_local PerThread pt;
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= MAXDEV) return nullptr;
-    std::call_once(once[dev], [dev] {
-        Side& x = sides[dev];
+    Side& x = pt.sides[dev];
+    if (!pt.tried[dev]) {
+        pt.tried[dev] = true;
         x.ok = cudaStreamCreateWithFlags(&x.s, cudaStreamNonBlocking) == cudaSuccess &&
                cudaEventCreateWithFlags(&x.fork, cudaEventDisableTiming) == cudaSuccess &&
                cudaEventCreateWithFlags(&x.join, cudaEventDisableTiming) == cudaSuccess;
-    });
-    return sides[dev].ok ? &sides[dev] : nullptr;
+    }
+    return x.ok ? &x : nullptr;
 }
 // stream of slice i (fork before the first slice, join after the last)
 struct ForkJoin {
@@ -424,6 +468,34 @@ ft_status ft_winattn_bwd_tape(const void* q, const void* k, const void* v, const
     const cudaError_t e = ftw::simt_bwd(q, k, v, out, lse, dout, dq, dk, dv, (float*)workspace, batch,
                                         heads, seq_len, d, w, dilation, dtype, (cudaStream_t)stream, tape);
     return e == cudaSuccess ? FT_OK : cuda_fail(e);
+}
+
+
+ft_status ft_winattn_fwd_bwd(const void* q, const void* k, const void* v, const void* dout, void* out,
+                             float* lse, void* dq, void* dk, void* dv, int64_t batch, int64_t heads,
+                             int64_t seq_len, int64_t d, int64_t w, int64_t dilation, ft_dtype dtype,
+                             void* workspace, size_t workspace_bytes, void* stream) {
+    if (!dout || !dq || !dk || !dv) return FT_ERR_INVALID_VALUE;
+    ft_status s = check_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype);
+    if (s != FT_OK) return s;
+    s = check_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, dilation, dtype,
+                  workspace, workspace_bytes);
+    if (s != FT_OK) return s;
+    // out and lse are outputs here: dout must not overlap them either (check_bwd treats them as
+    // inputs, so it allowed dout == out)
+    const size_t nb = (size_t)(batch * heads * seq_len * d) * elt_size(dtype);
+    const size_t lb = (size_t)(batch * heads * seq_len) * sizeof(float);
+    const Span sdo = {(uintptr_t)dout, (uintptr_t)dout + nb};
+    if (overlap(sdo, {(uintptr_t)out, (uintptr_t)out + nb}) || overlap(sdo, {(uintptr_t)lse, (uintptr_t)lse + lb}))
+        return FT_ERR_INVALID_VALUE;
+    ftw::prof_reset();
+    g_handoff = true;
+    s = run_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype, stream);
+    if (s == FT_OK)
+        s = run_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, dilation, dtype,
+                    workspace, stream);
+    g_handoff = false;
+    return s;
 }
 
 }  // extern "C"

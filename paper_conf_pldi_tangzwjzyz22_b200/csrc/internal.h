@@ -103,16 +103,28 @@ cudaError_t tc_narrow_bwd(const void* q, const void* k, const void* v, const flo
                           int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
                           int* launches);
 
-// d = 64, w <= 32 backward in ONE kernel (query-major strips, dK/dV key blocks in TMEM) --
-// tc_narrow_fused.cu.  Used instead of tc_narrow_bwd when there are >= ~4 tiles per SM.
-bool tc_narrow_fused_ok(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
-int tc_narrow_fused_launches(int64_t L, int64_t dil);
-cudaError_t tc_narrow_fused_bwd(const void* q, const void* k, const void* v, const float* lse,
-                                const void* dout, void* dq, void* dk, void* dv, int64_t B, int64_t H,
-                                int64_t L, int64_t w, int64_t dil, cudaStream_t st, int* launches);
-
 // FT_ERR_CUDA with the CUDA error text recorded for ft_status_str (api.cu)
 ft_status cuda_error(cudaError_t e);
+
+// Debug / A-B knobs (ft_winattn_debug_set; initialised once from the environment, see
+// include/ft_winattn.h).  They pick among kernels that compute the same result.
+enum Knob {
+    K_PATH = 0,     // 0 auto, 1 CUDA-core (SIMT) kernels, 2 tensor-core kernels (FT_WINATTN_PATH=simt|tc)
+    K_PDL = 1,      // 1: programmatic dependent launch inside a call; 0: plain stream order (FT_WINATTN_PDL=0)
+    K_NARROW = 2,   // 1: d = 64, w <= 32 narrow kernels; 0: band kernels (FT_WINATTN_NARROW=0)
+    K_WIDE = 3,     // 1: w > 64 wide kernels; 0: the chunked fallback kernels (FT_WINATTN_WIDE=0)
+    K_SIDE = 4,     // 1: per-head-dilation calls use a side stream; 0: serial (FT_WINATTN_MIXED_SERIAL=1)
+    K_NUM = 5
+};
+int knob(Knob k);
+
+// True while ft_winattn_fwd_bwd enqueues its forward and backward back to back on one stream
+// (the forward -> dQ-kernel lse hand-off is allowed only then).
+bool call_handoff();
+// The forward marks its lse rows and triggers, and the dQ kernel (PDL) polls them, only inside
+// ft_winattn_fwd_bwd; the dQ -> dK/dV kernel D hand-off (always inside one call) needs PDL on.
+inline bool lsepoll_enabled() { return call_handoff() && knob(K_PDL) != 0; }
+inline bool dpoll_enabled() { return knob(K_PDL) != 0; }
 
 // Profiling hook (ft_winattn_profile_events): record the next caller event after a launch.
 void prof_reset();

@@ -56,27 +56,6 @@ template <> struct Vec<__nv_bfloat16> {
     __device__ static float to_f(__nv_bfloat16 x) { return __bfloat162float(x); }
 };
 
-// Stage rows [mbase, mbase+R) x cols [col0, col0+DS) of a strided band view into dst[R][SP].
-// Rows outside [0, Lr) and columns >= d read as zero.
-template <typename Tin, int R>
-__device__ __forceinline__ void load_slice(float (*dst)[SP], const Tin* __restrict__ base,
-                                           int64_t rstride, int mbase, int Lr, int col0, int d) {
-    constexpr int V = Vec<Tin>::N;
-    constexpr int NV = DS / V;
-    for (int idx = threadIdx.x; idx < R * NV; idx += NT) {
-        const int row = idx / NV, cv = idx % NV;
-        const int m = mbase + row, c = col0 + cv * V;
-        float vals[V];
-        if (m >= 0 && m < Lr && c < d) {
-            Vec<Tin>::load(base + (int64_t)m * rstride + c, vals);
-        } else {
-#pragma unroll
-            for (int e = 0; e < V; ++e) vals[e] = 0.f;
-        }
-#pragma unroll
-        for (int e = 0; e < V; ++e) dst[row][cv * V + e] = vals[e];
-    }
-}
 
 struct TileCoord {
     int64_t u, r;
@@ -115,136 +94,10 @@ __device__ __forceinline__ float hsum16(float x) {
 // tape (nullable): the raw band scores s_ij, fp32 [B*H*L][2w+1] indexed by the query's flat
 // row and k + w (residue-space offset k = m_j - m_i) -- the materialized `dot` of Fig. 8 that
 // the tape-based backward reads instead of recomputing it.
-template <typename Tin>
-__global__ void __launch_bounds__(NT) simt_fwd_kernel(const Tin* __restrict__ q,
-                                                      const Tin* __restrict__ k,
-                                                      const Tin* __restrict__ v,
-                                                      Tin* __restrict__ out, float* __restrict__ lse,
-                                                      float* __restrict__ tape, Geo g) {
-    constexpr int T = 64, RA = T / 16;
-    extern __shared__ float smem[];
-    float(*Qs)[SP] = reinterpret_cast<float(*)[SP]>(smem);
-    float(*Ks)[SP] = Qs + T;                                   // K slice, then V slice
-    float(*Ps)[C + 1] = reinterpret_cast<float(*)[C + 1]>(Ks + C);
-    float* Os = reinterpret_cast<float*>(Ps + T);              // T x d accumulator
-    float* rowM = Os + T * g.d;
-    float* rowL = rowM + T;
-
-    TileCoord tc;
-    if (!decode(g, tc)) return;
-    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
-    const Tin* Qb = q + tc.off;
-    const Tin* Kb = k + tc.off;
-    const Tin* Vb = v + tc.off;
-    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
-
-    for (int i = threadIdx.x; i < T * d; i += NT) Os[i] = 0.f;
-    float mrow[RA], lrow[RA];
-#pragma unroll
-    for (int a = 0; a < RA; ++a) { mrow[a] = -INFINITY; lrow[a] = 0.f; }
-
-    const int kbeg = max(0, m0 - w);
-    const int kend = min(Lr, m0 + T + w);
-    for (int c0 = kbeg; c0 < kend; c0 += C) {
-        float s[RA][4];
-#pragma unroll
-        for (int a = 0; a < RA; ++a)
-#pragma unroll
-            for (int b = 0; b < 4; ++b) s[a][b] = 0.f;
-        for (int col0 = 0; col0 < d; col0 += DS) {
-            __syncthreads();
-            load_slice<Tin, T>(Qs, Qb, tc.rstride, m0, Lr, col0, d);
-            load_slice<Tin, C>(Ks, Kb, tc.rstride, c0, kend, col0, d);
-            __syncthreads();
-#pragma unroll 8
-            for (int p = 0; p < DS; ++p) {
-                float qa[RA], kb[4];
-#pragma unroll
-                for (int a = 0; a < RA; ++a) qa[a] = Qs[ty + 16 * a][p];
-#pragma unroll
-                for (int b = 0; b < 4; ++b) kb[b] = Ks[tx + 16 * b][p];
-#pragma unroll
-                for (int a = 0; a < RA; ++a)
-#pragma unroll
-                    for (int b = 0; b < 4; ++b) s[a][b] = fmaf(qa[a], kb[b], s[a][b]);
-            }
-        }
-        // band mask + online softmax (log2 domain)
-        float alpha[RA];
-#pragma unroll
-        for (int a = 0; a < RA; ++a) {
-            const int mq = m0 + ty + 16 * a;
-            float cmax = -INFINITY;
-#pragma unroll
-            for (int b = 0; b < 4; ++b) {
-                const int mk = c0 + tx + 16 * b;
-                const bool ok = (mk < kend) && (abs(mk - mq) <= w);
-                if (tape && ok && mq < Lr)
-                    tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)] = s[a][b];
-                s[a][b] = ok ? s[a][b] * LOG2E : -INFINITY;
-                cmax = fmaxf(cmax, s[a][b]);
-            }
-            cmax = hmax16(cmax);
-            const float mnew = fmaxf(mrow[a], cmax);
-            alpha[a] = (mnew == -INFINITY) ? 1.f : exp2f(mrow[a] - mnew);
-            float sum = 0.f;
-#pragma unroll
-            for (int b = 0; b < 4; ++b) {
-                const float p = (s[a][b] == -INFINITY) ? 0.f : exp2f(s[a][b] - mnew);
-                Ps[ty + 16 * a][tx + 16 * b] = p;
-                sum += p;
-            }
-            sum = hsum16(sum);
-            lrow[a] = lrow[a] * alpha[a] + sum;
-            mrow[a] = mnew;
-        }
-        // O = alpha * O + P V
-        for (int col0 = 0; col0 < d; col0 += DS) {
-            __syncthreads();
-            load_slice<Tin, C>(Ks, Vb, tc.rstride, c0, kend, col0, d);
-            __syncthreads();
-            float acc[RA][2];
-#pragma unroll
-            for (int a = 0; a < RA; ++a) { acc[a][0] = 0.f; acc[a][1] = 0.f; }
-#pragma unroll 8
-            for (int kk = 0; kk < C; ++kk) {
-                const float v0 = Ks[kk][tx], v1 = Ks[kk][tx + 16];
-#pragma unroll
-                for (int a = 0; a < RA; ++a) {
-                    const float p = Ps[ty + 16 * a][kk];
-                    acc[a][0] = fmaf(p, v0, acc[a][0]);
-                    acc[a][1] = fmaf(p, v1, acc[a][1]);
-                }
-            }
-#pragma unroll
-            for (int a = 0; a < RA; ++a)
-#pragma unroll
-                for (int b = 0; b < 2; ++b) {
-                    const int col = col0 + tx + 16 * b;
-                    if (col < d) {
-                        float* o = &Os[(ty + 16 * a) * d + col];
-                        *o = *o * alpha[a] + acc[a][b];
-                    }
-                }
-        }
-    }
-    if (tx == 0) {
-#pragma unroll
-        for (int a = 0; a < RA; ++a) { rowM[ty + 16 * a] = mrow[a]; rowL[ty + 16 * a] = lrow[a]; }
-    }
-    __syncthreads();
-    const int nrows = min(T, Lr - m0);
-    for (int i = threadIdx.x; i < nrows * d; i += NT) {
-        const int row = i / d, col = i % d;
-        Vec<Tin>::store1(out + tc.off + (int64_t)(m0 + row) * tc.rstride + col, Os[i] / rowL[row]);
-    }
-    for (int row = threadIdx.x; row < nrows; row += NT)
-        lse[tc.row0 + (int64_t)(m0 + row) * g.dil] = (rowM[row] + log2f(rowL[row])) * LN2;
-}
-
-// ------------------------------------------------------------------------------ forward, v2
-// Same algorithm as simt_fwd_kernel, with the shared-memory traffic of the two micro-GEMMs cut
-// four-fold: Q and K slices are staged TRANSPOSED ([d column][row], rows padded to 68 floats) so
+// ------------------------------------------------------------------------------ forward
+// A CTA owns 64 rows of one (unit, residue) problem and streams the 64-key chunks of its band:
+// S = Q K^T over d-slices, online row max / sum, O += P V.  The shared-memory traffic of the two
+// micro-GEMMs is cut four-fold: Q and K slices are staged TRANSPOSED ([d column][row], rows padded to 68 floats) so
 // a thread's four rows (4ty..4ty+3) and four keys (4tx..4tx+3) are one 16-byte load each per
 // d column, and P is staged transposed ([key][row]) so the P.V loop reads a thread's four rows
 // of P with one 16-byte load and two V columns (2tx, 2tx+1) with one 8-byte load.  The scalar
@@ -459,146 +312,6 @@ __global__ void __launch_bounds__(NT) simt_fwd_v2_kernel(const Tin* __restrict__
 // kernel.
 // TAPE: s_ij is read from the forward's tape instead of being recomputed as q_i . k_j, so the
 // score loop stages only dout and V (half its FMAs and shared-memory traffic).
-template <typename Tin, int T, bool TAPE>
-__global__ void __launch_bounds__(NT) simt_dq_kernel(const Tin* __restrict__ q,
-                                                     const Tin* __restrict__ k,
-                                                     const Tin* __restrict__ v,
-                                                     const Tin* __restrict__ dout,
-                                                     const float* __restrict__ lse,
-                                                     const float* __restrict__ tape,
-                                                     float* __restrict__ Dws,
-                                                     Tin* __restrict__ dq, Geo g) {
-    constexpr int RA = T / 16;
-    extern __shared__ float smem[];
-    float(*Qs)[SP] = reinterpret_cast<float(*)[SP]>(smem);
-    float(*Gs)[SP] = Qs + T;   // dout rows
-    float(*Ks)[SP] = Gs + T;
-    float(*Vs)[SP] = Ks + C;
-    float(*PDs)[C + 1] = reinterpret_cast<float(*)[C + 1]>(Vs + C);   // P * dP
-    float(*Ps)[C + 1] = PDs + T;                                        // P
-    float* rowD = reinterpret_cast<float*>(Ps + T);
-    float* OsA = rowD + T;
-    float* OsB = OsA + T * g.d;
-
-    TileCoord tc;
-    if (!decode(g, tc)) return;
-    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
-    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
-    for (int i = threadIdx.x; i < T * d; i += NT) { OsA[i] = 0.f; OsB[i] = 0.f; }
-
-    float lse2[RA], Dacc[RA];
-#pragma unroll
-    for (int a = 0; a < RA; ++a) {
-        const int mq = m0 + ty + 16 * a;
-        lse2[a] = mq < Lr ? lse[tc.row0 + (int64_t)mq * g.dil] * LOG2E : 0.f;
-        Dacc[a] = 0.f;
-    }
-    const int kbeg = max(0, m0 - w);
-    const int kend = min(Lr, m0 + T + w);
-    for (int c0 = kbeg; c0 < kend; c0 += C) {
-        float s[RA][4], dp[RA][4];
-#pragma unroll
-        for (int a = 0; a < RA; ++a)
-#pragma unroll
-            for (int b = 0; b < 4; ++b) { s[a][b] = 0.f; dp[a][b] = 0.f; }
-        SliceRegs<Tin, T> rq, rg;
-        SliceRegs<Tin, C> rk, rv;
-        auto fetch = [&](int col0) {   // slice col0 into registers (software pipelining)
-            if (!TAPE) rq.fetch(q + tc.off, tc.rstride, m0, Lr, col0, d);
-            rg.fetch(dout + tc.off, tc.rstride, m0, Lr, col0, d);
-            if (!TAPE) rk.fetch(k + tc.off, tc.rstride, c0, kend, col0, d);
-            rv.fetch(v + tc.off, tc.rstride, c0, kend, col0, d);
-        };
-        fetch(0);
-        for (int col0 = 0; col0 < d; col0 += DS) {
-            __syncthreads();
-            if (!TAPE) rq.store_p(Qs);
-            rg.store_p(Gs);
-            if (!TAPE) rk.store_p(Ks);
-            rv.store_p(Vs);
-            __syncthreads();
-            if (col0 + DS < d) fetch(col0 + DS);
-#pragma unroll 4
-            for (int p = 0; p < DS; ++p) {
-                float qa[RA], ga[RA], kb[4], vb[4];
-#pragma unroll
-                for (int a = 0; a < RA; ++a) { if (!TAPE) qa[a] = Qs[ty + 16 * a][p]; ga[a] = Gs[ty + 16 * a][p]; }
-#pragma unroll
-                for (int b = 0; b < 4; ++b) { if (!TAPE) kb[b] = Ks[tx + 16 * b][p]; vb[b] = Vs[tx + 16 * b][p]; }
-#pragma unroll
-                for (int a = 0; a < RA; ++a)
-#pragma unroll
-                    for (int b = 0; b < 4; ++b) {
-                        if (!TAPE) s[a][b] = fmaf(qa[a], kb[b], s[a][b]);
-                        dp[a][b] = fmaf(ga[a], vb[b], dp[a][b]);
-                    }
-            }
-        }
-#pragma unroll
-        for (int a = 0; a < RA; ++a) {
-            const int mq = m0 + ty + 16 * a;
-#pragma unroll
-            for (int b = 0; b < 4; ++b) {
-                const int mk = c0 + tx + 16 * b;
-                const bool ok = (mk < kend) && (abs(mk - mq) <= w) && mq < Lr;
-                if (TAPE && ok) s[a][b] = tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)];
-                const float p = ok ? exp2f(s[a][b] * LOG2E - lse2[a]) : 0.f;
-                const float pd = p * dp[a][b];
-                Dacc[a] += pd;
-                PDs[ty + 16 * a][tx + 16 * b] = pd;
-                Ps[ty + 16 * a][tx + 16 * b] = p;
-            }
-        }
-        SliceRegs<Tin, C> rk2;
-        rk2.fetch(k + tc.off, tc.rstride, c0, kend, 0, d);
-        for (int col0 = 0; col0 < d; col0 += DS) {
-            __syncthreads();
-            rk2.store_p(Ks);
-            __syncthreads();
-            if (col0 + DS < d) rk2.fetch(k + tc.off, tc.rstride, c0, kend, col0 + DS, d);
-            float aA[RA][2], aB[RA][2];
-#pragma unroll
-            for (int a = 0; a < RA; ++a) { aA[a][0] = aA[a][1] = aB[a][0] = aB[a][1] = 0.f; }
-#pragma unroll 4
-            for (int kk = 0; kk < C; ++kk) {
-                const float k0 = Ks[kk][tx], k1 = Ks[kk][tx + 16];
-#pragma unroll
-                for (int a = 0; a < RA; ++a) {
-                    const float pd = PDs[ty + 16 * a][kk], p = Ps[ty + 16 * a][kk];
-                    aA[a][0] = fmaf(pd, k0, aA[a][0]);
-                    aA[a][1] = fmaf(pd, k1, aA[a][1]);
-                    aB[a][0] = fmaf(p, k0, aB[a][0]);
-                    aB[a][1] = fmaf(p, k1, aB[a][1]);
-                }
-            }
-#pragma unroll
-            for (int a = 0; a < RA; ++a)
-#pragma unroll
-                for (int b = 0; b < 2; ++b) {
-                    const int col = col0 + tx + 16 * b;
-                    if (col < d) {
-                        OsA[(ty + 16 * a) * d + col] += aA[a][b];
-                        OsB[(ty + 16 * a) * d + col] += aB[a][b];
-                    }
-                }
-        }
-    }
-#pragma unroll
-    for (int a = 0; a < RA; ++a) {
-        const float D = hsum16(Dacc[a]);
-        if (tx == 0) rowD[ty + 16 * a] = D;
-    }
-    __syncthreads();
-    const int nrows = min(T, Lr - m0);
-    for (int i = threadIdx.x; i < nrows * d; i += NT) {
-        const int row = i / d, col = i % d;
-        Vec<Tin>::store1(dq + tc.off + (int64_t)(m0 + row) * tc.rstride + col,
-                         OsA[i] - rowD[row] * OsB[i]);
-    }
-    for (int row = threadIdx.x; row < nrows; row += NT)
-        Dws[tc.row0 + (int64_t)(m0 + row) * g.dil] = rowD[row];
-}
-
 // dq, v2: the same sweep with the vectorised staging of simt_fwd_v2_kernel -- a thread owns the
 // RA consecutive rows RA*ty.. and the four consecutive keys 4tx.., Q / dO / K / V slices are
 // staged transposed ([d column][row]) and P, P*dP transposed ([key][row]), so every operand of
@@ -764,148 +477,7 @@ __global__ void __launch_bounds__(NT, T == 32 ? 1 : 0) simt_dq_v2_kernel(const T
 // ------------------------------------------------------------------------------ backward: dk, dv
 // Key-major: for owned key rows j, dk_j = sum_i dS_ij q_i and dv_j = sum_i P_ij dout_i over
 // the queries i whose window contains j (the band is symmetric: |m_i - m_j| <= w).
-template <typename Tin, int T, bool TAPE>
-__global__ void __launch_bounds__(NT) simt_dkdv_kernel(const Tin* __restrict__ q,
-                                                       const Tin* __restrict__ k,
-                                                       const Tin* __restrict__ v,
-                                                       const Tin* __restrict__ dout,
-                                                       const float* __restrict__ lse,
-                                                       const float* __restrict__ tape,
-                                                       const float* __restrict__ Dws,
-                                                       Tin* __restrict__ dk, Tin* __restrict__ dv,
-                                                       Geo g) {
-    constexpr int RA = T / 16;
-    extern __shared__ float smem[];
-    float(*Ks)[SP] = reinterpret_cast<float(*)[SP]>(smem);
-    float(*Vs)[SP] = Ks + T;
-    float(*Qs)[SP] = Vs + T;   // query rows of the chunk
-    float(*Gs)[SP] = Qs + C;   // dout rows of the chunk
-    float(*Ps)[C + 1] = reinterpret_cast<float(*)[C + 1]>(Gs + C);
-    float(*DSs)[C + 1] = Ps + T;
-    float* qlse = reinterpret_cast<float*>(DSs + T);
-    float* qD = qlse + C;
-    float* OsK = qD + C;
-    float* OsV = OsK + T * g.d;
-
-    TileCoord tc;
-    if (!decode(g, tc)) return;
-    const int d = (int)g.d, w = (int)g.w, Lr = tc.Lr, m0 = tc.m0;
-    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
-    for (int i = threadIdx.x; i < T * d; i += NT) { OsK[i] = 0.f; OsV[i] = 0.f; }
-
-    const int qbeg = max(0, m0 - w);
-    const int qend = min(Lr, m0 + T + w);
-    for (int c0 = qbeg; c0 < qend; c0 += C) {
-        float s[RA][4], dp[RA][4];
-#pragma unroll
-        for (int a = 0; a < RA; ++a)
-#pragma unroll
-            for (int b = 0; b < 4; ++b) { s[a][b] = 0.f; dp[a][b] = 0.f; }
-        __syncthreads();
-        for (int i = threadIdx.x; i < C; i += NT) {
-            const int mq = c0 + i;
-            const int64_t fr = tc.row0 + (int64_t)mq * g.dil;
-            qlse[i] = mq < qend ? lse[fr] * LOG2E : 0.f;
-            qD[i] = mq < qend ? Dws[fr] : 0.f;
-        }
-        SliceRegs<Tin, T> rk, rv;
-        SliceRegs<Tin, C> rq, rg;
-        auto fetch = [&](int col0) {   // slice col0 into registers (software pipelining)
-            if (!TAPE) rk.fetch(k + tc.off, tc.rstride, m0, Lr, col0, d);
-            rv.fetch(v + tc.off, tc.rstride, m0, Lr, col0, d);
-            if (!TAPE) rq.fetch(q + tc.off, tc.rstride, c0, qend, col0, d);
-            rg.fetch(dout + tc.off, tc.rstride, c0, qend, col0, d);
-        };
-        fetch(0);
-        for (int col0 = 0; col0 < d; col0 += DS) {
-            __syncthreads();
-            if (!TAPE) rk.store_p(Ks);
-            rv.store_p(Vs);
-            if (!TAPE) rq.store_p(Qs);
-            rg.store_p(Gs);
-            __syncthreads();
-            if (col0 + DS < d) fetch(col0 + DS);
-#pragma unroll 4
-            for (int p = 0; p < DS; ++p) {
-                float ka[RA], va[RA], qb[4], gb[4];
-#pragma unroll
-                for (int a = 0; a < RA; ++a) { if (!TAPE) ka[a] = Ks[ty + 16 * a][p]; va[a] = Vs[ty + 16 * a][p]; }
-#pragma unroll
-                for (int b = 0; b < 4; ++b) { if (!TAPE) qb[b] = Qs[tx + 16 * b][p]; gb[b] = Gs[tx + 16 * b][p]; }
-#pragma unroll
-                for (int a = 0; a < RA; ++a)
-#pragma unroll
-                    for (int b = 0; b < 4; ++b) {
-                        if (!TAPE) s[a][b] = fmaf(ka[a], qb[b], s[a][b]);
-                        dp[a][b] = fmaf(va[a], gb[b], dp[a][b]);
-                    }
-            }
-        }
-#pragma unroll
-        for (int a = 0; a < RA; ++a) {
-            const int mk = m0 + ty + 16 * a;
-#pragma unroll
-            for (int b = 0; b < 4; ++b) {
-                const int qi = tx + 16 * b;
-                const int mq = c0 + qi;
-                const bool ok = (mq < qend) && (abs(mq - mk) <= w) && mk < Lr;
-                if (TAPE && ok) s[a][b] = tape[(tc.row0 + (int64_t)mq * g.dil) * (2 * w + 1) + (mk - mq + w)];
-                const float p = ok ? exp2f(s[a][b] * LOG2E - qlse[qi]) : 0.f;
-                Ps[ty + 16 * a][qi] = p;
-                DSs[ty + 16 * a][qi] = p * (dp[a][b] - qD[qi]);
-            }
-        }
-        SliceRegs<Tin, C> rq2, rg2;
-        rq2.fetch(q + tc.off, tc.rstride, c0, qend, 0, d);
-        rg2.fetch(dout + tc.off, tc.rstride, c0, qend, 0, d);
-        for (int col0 = 0; col0 < d; col0 += DS) {
-            __syncthreads();
-            rq2.store_p(Qs);
-            rg2.store_p(Gs);
-            __syncthreads();
-            if (col0 + DS < d) {
-                rq2.fetch(q + tc.off, tc.rstride, c0, qend, col0 + DS, d);
-                rg2.fetch(dout + tc.off, tc.rstride, c0, qend, col0 + DS, d);
-            }
-            float ak[RA][2], av[RA][2];
-#pragma unroll
-            for (int a = 0; a < RA; ++a) { ak[a][0] = ak[a][1] = av[a][0] = av[a][1] = 0.f; }
-#pragma unroll 4
-            for (int qi = 0; qi < C; ++qi) {
-                const float q0 = Qs[qi][tx], q1 = Qs[qi][tx + 16];
-                const float g0 = Gs[qi][tx], g1 = Gs[qi][tx + 16];
-#pragma unroll
-                for (int a = 0; a < RA; ++a) {
-                    const float ds = DSs[ty + 16 * a][qi], p = Ps[ty + 16 * a][qi];
-                    ak[a][0] = fmaf(ds, q0, ak[a][0]);
-                    ak[a][1] = fmaf(ds, q1, ak[a][1]);
-                    av[a][0] = fmaf(p, g0, av[a][0]);
-                    av[a][1] = fmaf(p, g1, av[a][1]);
-                }
-            }
-#pragma unroll
-            for (int a = 0; a < RA; ++a)
-#pragma unroll
-                for (int b = 0; b < 2; ++b) {
-                    const int col = col0 + tx + 16 * b;
-                    if (col < d) {
-                        OsK[(ty + 16 * a) * d + col] += ak[a][b];
-                        OsV[(ty + 16 * a) * d + col] += av[a][b];
-                    }
-                }
-        }
-    }
-    __syncthreads();
-    const int nrows = min(T, Lr - m0);
-    for (int i = threadIdx.x; i < nrows * d; i += NT) {
-        const int row = i / d, col = i % d;
-        const int64_t o = tc.off + (int64_t)(m0 + row) * tc.rstride + col;
-        Vec<Tin>::store1(dk + o, OsK[i]);
-        Vec<Tin>::store1(dv + o, OsV[i]);
-    }
-}
-
-// dk / dv, v2: simt_dkdv_kernel with the staging of simt_dq_v2_kernel -- a thread owns key
+// dk / dv: key-major, with the staging of simt_dq_v2_kernel -- a thread owns key
 // rows RA*ty.. and the four consecutive queries 4tx..; K / V / Q / dO slices transposed, P and
 // dS transposed ([query][key row]), the output loop's Q / dO slices row-major (float2 loads).
 template <typename Tin, int T, bool TAPE>
@@ -1061,13 +633,8 @@ size_t dkdv_v2_smem(int T, int64_t d) {
     return sizeof(float) * (2 * DS * (T + 4) + 2 * DS * TP + 2 * C * (T + 4) + 2 * C + 2 * T * d);
 }
 size_t fwd_v2_smem(int64_t d) { return sizeof(float) * (2 * DS * TP + C * VSP + C * TP + 64 * d + 128); }
-size_t fwd_smem(int64_t d) { return sizeof(float) * (64 * SP + C * SP + 64 * (C + 1) + 64 * d + 128); }
 size_t dq_v2_smem(int T, int64_t d) {
     return sizeof(float) * (2 * DS * (T + 4) + 2 * DS * TP + 2 * C * (T + 4) + T + 2 * T * d);
-}
-size_t dq_smem(int T, int64_t d) { return sizeof(float) * (2 * T * SP + 2 * C * SP + 2 * T * (C + 1) + T + 2 * T * d); }
-size_t dkdv_smem(int T, int64_t d) {
-    return sizeof(float) * (2 * T * SP + 2 * C * SP + 2 * T * (C + 1) + 2 * C + 2 * T * d);
 }
 
 template <typename F>
@@ -1082,18 +649,11 @@ template <typename Tin>
 cudaError_t fwd_impl(const void* q, const void* k, const void* v, void* out, float* lse, float* tape,
                      int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                      cudaStream_t st) {
-    static std::once_flag once, once2;
+    static std::once_flag once;
     Geo g = make_geo(B, H, L, d, w, dil, 64);
-    const char* e1 = getenv("FT_WINATTN_SIMT_V1");   // A/B timing: the scalar-load version
-    if (e1 && atoi(e1) == 1) {
-        set_smem_once(simt_fwd_kernel<Tin>, fwd_smem(d), once);
-        simt_fwd_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_smem(d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, tape, g);
-    } else {
-        set_smem_once(simt_fwd_v2_kernel<Tin>, fwd_v2_smem(d), once2);
-        simt_fwd_v2_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_v2_smem(d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, tape, g);
-    }
+    set_smem_once(simt_fwd_v2_kernel<Tin>, fwd_v2_smem(d), once);
+    simt_fwd_v2_kernel<Tin><<<(unsigned)geo_blocks(g), NT, fwd_v2_smem(d), st>>>(
+        (const Tin*)q, (const Tin*)k, (const Tin*)v, (Tin*)out, lse, tape, g);
     prof_mark(st);
     return cudaGetLastError();
 }
@@ -1102,32 +662,18 @@ template <typename Tin, int T, bool TAPE>
 cudaError_t bwd_launch(const void* q, const void* k, const void* v, const float* lse, const float* tape,
                        const void* dout, void* dq, void* dk, void* dv, float* Dws, const Geo& g,
                        cudaStream_t st) {
-    static std::once_flag o1, o2, o3, o4;
+    static std::once_flag o1, o2;
     const int64_t d = g.d;
-    const char* e1 = getenv("FT_WINATTN_SIMT_V1");   // A/B timing: the scalar-load version
-    if (e1 && atoi(e1) == 1) {
-        set_smem_once(simt_dq_kernel<Tin, T, TAPE>, dq_smem(T, d), o1);
-        simt_dq_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dq_smem(T, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dq, g);
-    } else {
-        set_smem_once(simt_dq_v2_kernel<Tin, T, TAPE>, dq_v2_smem(T, d), o3);
-        simt_dq_v2_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dq_v2_smem(T, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dq, g);
-    }
+    set_smem_once(simt_dq_v2_kernel<Tin, T, TAPE>, dq_v2_smem(T, d), o1);
+    simt_dq_v2_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dq_v2_smem(T, d), st>>>(
+        (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dq, g);
     prof_mark(st);
     cudaError_t e;
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
-    if (e1 && atoi(e1) == 1) {
-        set_smem_once(simt_dkdv_kernel<Tin, T, TAPE>, dkdv_smem(T, d), o2);
-        simt_dkdv_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dkdv_smem(T, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dk,
-            (Tin*)dv, g);
-    } else {
-        set_smem_once(simt_dkdv_v2_kernel<Tin, T, TAPE>, dkdv_v2_smem(T, d), o4);
-        simt_dkdv_v2_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dkdv_v2_smem(T, d), st>>>(
-            (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dk,
-            (Tin*)dv, g);
-    }
+    set_smem_once(simt_dkdv_v2_kernel<Tin, T, TAPE>, dkdv_v2_smem(T, d), o2);
+    simt_dkdv_v2_kernel<Tin, T, TAPE><<<(unsigned)geo_blocks(g), NT, dkdv_v2_smem(T, d), st>>>(
+        (const Tin*)q, (const Tin*)k, (const Tin*)v, (const Tin*)dout, lse, tape, Dws, (Tin*)dk,
+        (Tin*)dv, g);
     prof_mark(st);
     return cudaGetLastError();
 }
@@ -1137,7 +683,7 @@ cudaError_t bwd_impl(const void* q, const void* k, const void* v, const void* ou
                      const float* lse, const float* tape, const void* dout, void* dq, void* dk, void* dv,
                      float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                      cudaStream_t st) {
-    (void)out;   // D_i is recomputed exactly as sum_j P_ij dP_ij (see simt_dq_kernel)
+    (void)out;   // D_i is recomputed exactly as sum_j P_ij dP_ij (see simt_dq_v2_kernel)
     const int T = d <= 256 ? 64 : 32;
     Geo g = make_geo(B, H, L, d, w, dil, T);
     if (tape) {

@@ -784,11 +784,7 @@ void set_attr_once() {
     });
 }
 
-// FT_WINATTN_PDL=0 turns the programmatic dependent launch off (A/B timing)
-bool pdl_enabled() {
-    const char* e = getenv("FT_WINATTN_PDL");
-    return !(e && atoi(e) == 0);
-}
+bool pdl_enabled() { return knob(K_PDL) != 0; }
 
 int num_sms() {
     static int n = 0;
@@ -849,12 +845,7 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         p.nst = nst;
         const int64_t Lr0 = ceil_div(L - r0, dil);   // longest residue of this group
         p.trace = (unsigned long long*)trace_buffer(MODE);
-        {
-            // Two issuers (measured faster for every mode and d, profiles/README.md);
-            // FT_WINATTN_ISSUERS=1 restores the single-issuer schedule for A/B timing.
-            const char* e = getenv("FT_WINATTN_ISSUERS");
-            p.two = !(e && atoi(e) == 1);
-        }
+        p.two = 1;   // two MMA issuers (measured faster for every mode and d, profiles/README.md)
         p.dpoll = MODE != FWD && dpoll_enabled();
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
@@ -915,7 +906,6 @@ int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
     return halo_rows(L, w) <= 256 ? band_launches(L, dil) : tc_chunk_launches(L, dil);
 }
 int tc_bwd_launches(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
-    if (tc_narrow_fused_ok(units, L, d, w, dil)) return tc_narrow_fused_launches(L, dil);
     if (tc_narrow_bwd_supported(1, L, d, w, dil)) return 2 * tc_narrow_launches(L, dil);
     if (halo_rows(L, w) <= 256) return 2 * band_launches(L, dil);
     return 2 * tc_chunk_launches(L, dil);
@@ -926,8 +916,7 @@ cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float
                    int* launches) {
     if (launches) *launches = 0;
     if (halo_rows(L, w) > 256) {
-        const char* v1 = getenv("FT_WINATTN_WIDE_V1");   // A/B timing: previous chunk kernel
-        if ((v1 && atoi(v1) == 1) || !tc_wide_supported(B * H, L, d, w, dil))
+        if (!knob(K_WIDE) || !tc_wide_supported(B * H, L, d, w, dil))
             return tc_chunk_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
         return tc_wide_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
     }
@@ -945,13 +934,10 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
     // wide kernels also compute it exactly, and read out only for the first-guess D~
     if (launches) *launches = 0;
     if (halo_rows(L, w) > 256) {
-        const char* v1 = getenv("FT_WINATTN_WIDE_V1");   // A/B timing: previous chunk kernels
-        if ((v1 && atoi(v1) == 1) || !tc_wide_bwd_supported(B * H, L, d, w, dil))
+        if (!knob(K_WIDE) || !tc_wide_bwd_supported(B * H, L, d, w, dil))
             return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
         return tc_wide_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     }
-    if (tc_narrow_fused_ok(B * H, L, d, w, dil))
-        return tc_narrow_fused_bwd(q, k, v, lse, dout, dq, dk, dv, B, H, L, w, dil, st, launches);
     if (tc_narrow_bwd_supported(B * H, L, d, w, dil))
         return tc_narrow_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     cudaError_t e = launch<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse),

@@ -363,10 +363,13 @@ __device__ __forceinline__ uint32_t elect_one() {
 // Arithmetic never produces D_UNSET: a NaN from the FP units is the canonical 0x7FFFFFFF.
 constexpr uint32_t D_UNSET = 0xFFFFFFFFu;
 __device__ __forceinline__ float ld_D_ready(const float* ptr) {
-    uint32_t x;
+    // D is stored by the dQ kernel of the same call, which is resident (the dependent grid
+    // launches only after every dQ CTA triggered): a protocol bug traps instead of hanging
+    uint32_t x, spins = 0;
     for (;;) {
         asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr) : "memory");
         if (x != D_UNSET) break;
+        if (++spins == FT_WATCHDOG_SPINS) __trap();
         __nanosleep(128);
     }
     return __uint_as_float(x);
@@ -399,24 +402,10 @@ __device__ __forceinline__ float ld_lse_ready(const float* ptr, bool& settled) {
     return __uint_as_float(x);
 }
 
-// FT_WINATTN_LSEPOLL=0: no forward -> dQ-kernel lse hand-off (also off with DPOLL=0 or PDL=0)
-inline bool lsepoll_enabled() {
-    const char* e = getenv("FT_WINATTN_LSEPOLL");
-    const char* d = getenv("FT_WINATTN_DPOLL");
-    const char* p = getenv("FT_WINATTN_PDL");
-    return !(e && atoi(e) == 0) && !(d && atoi(d) == 0) && !(p && atoi(p) == 0);
-}
-
 // The hand-off pays only when the forward's last partial wave is a visible share of it: with
 // many tiles per SM the forward's marking pass costs more than the overlap gains (narrow
 // C5_w32, 110 tiles per SM: forward 0.176 -> 0.194 ms).  Used by both sides of a call.
 inline bool lsepoll_worth(int64_t tiles, int sms) { return tiles < 8 * (int64_t)sms; }
-
-// FT_WINATTN_DPOLL=0: the dK/dV kernel waits for the whole dQ grid instead (A/B timing)
-inline bool dpoll_enabled() {
-    const char* e = getenv("FT_WINATTN_DPOLL");
-    return !(e && atoi(e) == 0);
-}
 
 }  // namespace tc
 }  // namespace ftw

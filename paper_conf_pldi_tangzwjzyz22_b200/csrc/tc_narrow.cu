@@ -315,14 +315,11 @@ int num_sms_n() {
 
 bool tc_narrow_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
     const int64_t wc = w < L ? w : L;
-    const char* e = getenv("FT_WINATTN_NARROW");   // A/B timing: 0 falls back to tc_band
-    if (e && atoi(e) == 0) return false;
+    if (!knob(K_NARROW)) return false;   // A/B: the band kernels
     return d == D && wc <= 32 && dil <= 256 && units * ((L + BM - 1) / BM) < (1 << 30);
 }
 
 bool tc_narrow_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
-    const char* e = getenv("FT_WINATTN_NARROW_BWD");   // A/B timing: 0 falls back to tc_band
-    if (e && atoi(e) == 0) return false;
     return tc_narrow_supported(units, L, d, w, dil);
 }
 
@@ -364,9 +361,8 @@ cudaError_t tc_narrow_fwd(const void* q, const void* k, const void* v, void* out
         const int64_t Lr0 = ceil_div(L - r0, dil);
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
-        // only when the split backward (NQ, PDL-launched) follows; the fused one is not
-        p.lsepoll = r0 == 0 && lsepoll_enabled() && lsepoll_worth(total, num_sms_n()) &&
-                    !tc_narrow_fused_ok(units, L, d, w, dil);
+        // only inside ft_winattn_fwd_bwd, where the dQ kernel (NQ, PDL-launched) follows
+        p.lsepoll = r0 == 0 && lsepoll_enabled() && lsepoll_worth(total, num_sms_n());
         dim3 grid((unsigned)(total < num_sms_n() ? total : num_sms_n()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         tc_narrow_fwd_kernel<<<grid, NTHREADS, SMEM_BYTES, st>>>(p);

@@ -20,13 +20,19 @@
 // (tcgen05.mma executes in issue order).  Per tile the tensor pipe runs S(j+1), out(j),
 // dP(j+1) while the softmax warps drain tile j's accumulator.
 //
-// dS enters its output MMA as fp16, with the bf16 halo it multiplies (K_h for dQ, Q_h for
-// dK) converted to fp16 in shared memory once the score GEMM has read it (exact for bf16
-// values of magnitude 6.1e-5 .. 65504).  A single bf16 dS put dq 1.1e-2 off at one element of
-// 8.4M in the 16 x 8192 parity case; fp16's 11-bit significand is 8x finer, and unlike a bf16
-// hi + lo pair it costs one operand: NQ writes dS over S, NKV writes P^T (bf16) | dS^T (fp16)
-// over S^T, and the dP region is free as soon as the softmax holds dP in registers
-// (reading A10).
+// dS enters its output MMA as fp16 (11-bit significand) with power-of-two scales, so the
+// result does not depend on the magnitude of the inputs (reading A10): the converter warp
+// turns the bf16 halo the dS GEMM multiplies (K_h for dQ, Q_h for dK) into fp16 row by row,
+// each row c scaled by 2^f_c so that its largest |value| lands in [2^14, 2^15), once the
+// score GEMM has read it, and publishes 2^-f_c; the softmax forms dS'_rc = dS_rc 2^-f_c,
+// scales its row r by 2^e_r (largest |dS'| in [2^14, 2^15)) and stores it as fp16.  The MMA
+// then accumulates 2^e_r sum_c dS_rc x_c exactly up to fp16 rounding of the two operands, and
+// the drain multiplies the row by 2^-e_r.  Powers of two are exact, so a gradient scaled by
+// 2^16 (loss scaling) or 2^-24 gives the same relative error, with no overflow to inf and no
+// fp16 subnormals (tests/test_gpu_parity.py::test_scale_equivariance).  A single bf16 dS
+// failed the 2e-2 / 1e-2 bound at one element of 8.4 M (16 x 8192 case); the bf16 hi + lo
+// pair of the band kernels would need a second operand, which does not fit (NQ: smem; NKV:
+// the P^T | dS^T pair fills the 192 columns over S^T).
 //
 // Roles (320 threads): warps 0-7 softmax -- warp w reads TMEM lanes 32*(w%4).. (thread <->
 // row) and column half h = w/4 of the row's 96-column band range; warp 8 TMA producer +
@@ -70,7 +76,10 @@ constexpr uint32_t STG = 32 * 128;
 constexpr uint32_t XBYTES = 3 * 16384;      // NQ: dS operand (fp16, 128 x 192); NKV: 8 x STG staging
 // per-tile scratch: NKV [2][2][NK] column lse / D; NQ [2][2][BM] D halves + [2][256] row lse
 constexpr int SCRATCH_FLOATS = 2 * 2 * BM + 2 * 256 > 2 * 2 * NK ? 2 * 2 * BM + 2 * 256 : 2 * 2 * NK;
-constexpr size_t SMEM_BYTES = 1024 + (size_t)NSTAGE * STAGE + XBYTES + SCRATCH_FLOATS * 4 + 256;
+// halo row scales 2^-f_c [2][NK] and the two halves' row maxima of |dS'| [2][2][BM]
+constexpr int SCALE_FLOATS = 2 * NK + 2 * 2 * BM;
+constexpr size_t SMEM_BYTES = 1024 + (size_t)NSTAGE * STAGE + XBYTES + (SCRATCH_FLOATS + SCALE_FLOATS) * 4 + 256;
+static_assert(SMEM_BYTES <= 232448, "shared memory plan");
 constexpr float LOG2E = 1.4426950408889634f;
 constexpr uint32_t TACC = 384;
 
@@ -103,6 +112,16 @@ __device__ __forceinline__ void trace_ev(const BParams& p, int j, int ev) {
 using Tile = SchedTile;
 using TileCursor = SchedCursor<BM>;
 
+// f with max|x| * 2^f in [2^14, 2^15) for a biased binary exponent E of max|x| (fp32 and bf16
+// share the field), clamped so that 2^f and 2^-f are both normal floats
+__device__ __forceinline__ int pow2_exp_fp16(int E) { return min(126, max(-126, 141 - E)); }
+// 2^e and 2^-e of a row whose largest |value| is mx (e = 0 for an all-zero row)
+__device__ __forceinline__ void row_pow2(float mx, float& up, float& down) {
+    const int f = mx > 0.f ? pow2_exp_fp16(int(__float_as_uint(mx) >> 23) & 0xFF) : 0;
+    up = __uint_as_float((uint32_t)(127 + f) << 23);
+    down = __uint_as_float((uint32_t)(127 - f) << 23);
+}
+
 __device__ __forceinline__ float fast_exp2(float x) {
     float y;
     asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
@@ -112,7 +131,7 @@ __device__ __forceinline__ float fast_exp2(float x) {
 // rows 32*wq .. +31 of a 64-column accumulator -> bf16 -> this warp's staging -> TMA store
 // (the accumulator is released on `freed` as soon as it is in registers)
 __device__ __forceinline__ void drain_store(uint32_t tacc, uint8_t* stg, const CUtensorMap* m, int row0,
-                                           int u, int lane, uint64_t* freed) {
+                                           int u, int lane, uint64_t* freed, float scale) {
     uint32_t ov[2][32];
     tmem_ld32(tacc, ov[0]);
     tmem_ld32(tacc + 32, ov[1]);
@@ -125,10 +144,11 @@ __device__ __forceinline__ void drain_store(uint32_t tacc, uint8_t* stg, const C
     for (int q = 0; q < 8; ++q) {
         const uint32_t* src = &ov[q >> 2][(q & 3) * 8];
         uint4 val;
-        val.x = pack_bf16x2(__uint_as_float(src[0]), __uint_as_float(src[1]));
-        val.y = pack_bf16x2(__uint_as_float(src[2]), __uint_as_float(src[3]));
-        val.z = pack_bf16x2(__uint_as_float(src[4]), __uint_as_float(src[5]));
-        val.w = pack_bf16x2(__uint_as_float(src[6]), __uint_as_float(src[7]));
+        const float* f = reinterpret_cast<const float*>(src);
+        val.x = pack_bf16x2(f[0] * scale, f[1] * scale);
+        val.y = pack_bf16x2(f[2] * scale, f[3] * scale);
+        val.z = pack_bf16x2(f[4] * scale, f[5] * scale);
+        val.w = pack_bf16x2(f[6] * scale, f[7] * scale);
         *reinterpret_cast<uint4*>(stg + lane * 128 + ((q ^ (lane & 7)) * 16)) = val;
     }
     fence_proxy_async_smem();
@@ -160,7 +180,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
     uint8_t* xbuf = smem + (size_t)NSTAGE * STAGE;                 // NQ: dS operand; NKV: staging
     float* colv = reinterpret_cast<float*>(xbuf + XBYTES);         // NKV [2][2][NK]: lse, D of columns
     float* dx = colv;                                              // NQ [2][2][BM]: D halves, then [2][256] lse
-    uint64_t* bars = reinterpret_cast<uint64_t*>(colv + SCRATCH_FLOATS);
+    float* hscale = colv + SCRATCH_FLOATS;                         // [2][NK] 2^-f of the halo rows
+    float* mxh = hscale + 2 * NK;                                  // [2][2][BM] row max halves
+    uint64_t* bars = reinterpret_cast<uint64_t*>(colv + SCRATCH_FLOATS + SCALE_FLOATS);
     uint64_t* full1 = bars;                 // [NSTAGE] A1 + B1
     uint64_t* full2 = bars + NSTAGE;        // [NSTAGE] A2 + B2
     uint64_t* empty = bars + 2 * NSTAGE;    // [NSTAGE]
@@ -169,7 +191,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
     uint64_t* p_done = s_full + 2;          // operands written and the dS halo converted
     uint64_t* acc_full = s_full + 3;        // [2]
     uint64_t* acc_free = s_full + 5;        // [2]
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 7);
+    uint64_t* hs_full = s_full + 7;         // [2] halo row scales of tile j published
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 9);
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int w = p.w;
@@ -187,6 +210,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             for (int b = 0; b < 2; ++b) {
                 mbar_init(&acc_full[b], 1);
                 mbar_init(&acc_free[b], 8);
+                mbar_init(&hs_full[b], 1);
             }
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
@@ -224,23 +248,48 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
         }
     } else if (warp == 10) {   // ------------------------------------------ halo converter
         // the halo of the dS GEMM (NQ: K_h, NKV: Q_h) to fp16 in place, once the score GEMM
-        // has read it as bf16 (s_full); the output MMAs read it after p_done
+        // has read it as bf16 (s_full): pass 1 finds each row's largest |value| and publishes
+        // 2^-f (hs_full), pass 2 writes the row times 2^f as fp16; the output MMAs read it
+        // after p_done.  Lane l owns halo rows l, l + 32, ...
         TileCursor cur(p.sc);
         Tile T;
         for (int j = 0; cur.next(p.sc, T); ++j) {
             mbar_wait(s_full, j & 1);
             if (lane == 0) trace_ev(p, j, 14);
-            uint4* hb = reinterpret_cast<uint4*>(stages + (size_t)(j % NSTAGE) * STAGE + 2 * ABYTES);
-#pragma unroll 4
-            for (int i = lane; i < (int)(HBYTES / 16); i += 32) {
-                uint4 v4 = hb[i];
-                uint32_t* wv = reinterpret_cast<uint32_t*>(&v4);
+            uint8_t* hb = stages + (size_t)(j % NSTAGE) * STAGE + 2 * ABYTES;
+            float* tab = hscale + (j & 1) * NK;
+            float sc[NK / 32];
 #pragma unroll
-                for (int x = 0; x < 4; ++x) {
-                    const float2 f = __bfloat1622float2(*reinterpret_cast<__nv_bfloat162*>(&wv[x]));
-                    wv[x] = pack_f16x2(f.x, f.y);
+            for (int q = 0; q < NK / 32; ++q) {
+                const uint4* row = reinterpret_cast<const uint4*>(hb + (lane + 32 * q) * 128);
+                uint32_t m = 0;
+#pragma unroll
+                for (int g = 0; g < 8; ++g) {
+                    const uint4 v4 = row[g];
+                    m = __vmaxu2(m, __vmaxu2(__vmaxu2(v4.x & 0x7FFF7FFFu, v4.y & 0x7FFF7FFFu),
+                                             __vmaxu2(v4.z & 0x7FFF7FFFu, v4.w & 0x7FFF7FFFu)));
                 }
-                hb[i] = v4;
+                m = max(m & 0xFFFFu, m >> 16);                  // bf16 bits of the row's max |x|
+                const int f = m == 0 ? 0 : pow2_exp_fp16(int(m >> 7));
+                sc[q] = __uint_as_float((uint32_t)(127 + f) << 23);
+                tab[lane + 32 * q] = __uint_as_float((uint32_t)(127 - f) << 23);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&hs_full[j & 1]);
+#pragma unroll
+            for (int q = 0; q < NK / 32; ++q) {
+                uint4* row = reinterpret_cast<uint4*>(hb + (lane + 32 * q) * 128);
+#pragma unroll
+                for (int g = 0; g < 8; ++g) {
+                    uint4 v4 = row[g];
+                    uint32_t* wv = reinterpret_cast<uint32_t*>(&v4);
+#pragma unroll
+                    for (int x = 0; x < 4; ++x) {
+                        const float2 f2 = __bfloat1622float2(*reinterpret_cast<__nv_bfloat162*>(&wv[x]));
+                        wv[x] = pack_f16x2(f2.x * sc[q], f2.y * sc[q]);
+                    }
+                    row[g] = v4;
+                }
             }
             fence_proxy_async_smem();
             warp_arrive(p_done);
@@ -379,9 +428,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             int64_t rowbase;
             float lse2;
             uint64_t bits;
+            float rsc;   // 2^-e of this row's dS (NQ: dq row; NKV: dk row), set by the softmax
         };
         auto setup = [&](const Tile& X, int jx) -> St {
             St c;
+            c.rsc = 1.f;
             c.Lr = X.Lr; c.m0 = X.m0; c.kb = X.m0 - w; c.u = X.u; c.rl = X.rl;
             c.rowbase = (int64_t)X.u * p.L + X.r;
             cp_async_wait_all();   // this tile's values (copied a tile ago)
@@ -433,16 +484,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 if (mrow < c.Lr) {
                     uint4* dst = reinterpret_cast<uint4*>(p.o1 + (c.rowbase + (int64_t)mrow * p.dil) * D + 32 * h);
 #pragma unroll
-                    for (int q = 0; q < 4; ++q)
-                        dst[q] = make_uint4(pack_bf16x2(__uint_as_float(ov[8 * q]), __uint_as_float(ov[8 * q + 1])),
-                                            pack_bf16x2(__uint_as_float(ov[8 * q + 2]), __uint_as_float(ov[8 * q + 3])),
-                                            pack_bf16x2(__uint_as_float(ov[8 * q + 4]), __uint_as_float(ov[8 * q + 5])),
-                                            pack_bf16x2(__uint_as_float(ov[8 * q + 6]), __uint_as_float(ov[8 * q + 7])));
+                    for (int q = 0; q < 4; ++q) {
+                        const float* o = reinterpret_cast<const float*>(&ov[8 * q]);
+                        const float r = c.rsc;
+                        dst[q] = make_uint4(pack_bf16x2(o[0] * r, o[1] * r), pack_bf16x2(o[2] * r, o[3] * r),
+                                            pack_bf16x2(o[4] * r, o[5] * r), pack_bf16x2(o[6] * r, o[7] * r));
+                    }
                 }
             } else {
                 const BMaps& mp = p.maps[c.rl];
                 drain_store(tbase + lane_off + TACC + 64u * h, xbuf + warp * STG, h == 0 ? &mp.o1 : &mp.o2,
-                            c.m0 + 32 * wq, c.u, lane, &acc_free[0]);
+                            c.m0 + 32 * wq, c.u, lane, &acc_free[0], h == 0 ? 1.f : c.rsc);
             }
             if (threadIdx.x == 0) trace_ev(p, i, 10);
         };
@@ -487,12 +539,25 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 named_bar_sync(1 + wq, 64);   // both halves posted their D part
                 if (tr) trace_ev(p, j, 7);
                 const float Dv = dxb[t] + dxb[BM + t];
+                // dS' = P (dP - D) 2^-f_c (halo row scales), then this row's power of two
+                mbar_wait(&hs_full[j & 1], (j >> 1) & 1);
+                const float* tab = hscale + (j & 1) * NK + c0;
+                float mx = 0.f;
 #pragma unroll
-                for (int e = 0; e < 48; e += 2) {
-                    const float d0 = __uint_as_float(rs[e]) * (__uint_as_float(rd[e]) - Dv);
-                    const float d1 = __uint_as_float(rs[e + 1]) * (__uint_as_float(rd[e + 1]) - Dv);
-                    pk[e / 2] = pack_f16x2(d0, d1);
+                for (int e = 0; e < 48; ++e) {
+                    const float dsv = __uint_as_float(rs[e]) * (__uint_as_float(rd[e]) - Dv) * tab[e];
+                    rs[e] = __float_as_uint(dsv);
+                    mx = fmaxf(mx, fabsf(dsv));
                 }
+                float* mxb = mxh + (j & 1) * 2 * BM;
+                mxb[h * BM + t] = mx;
+                named_bar_sync(1 + wq, 64);   // both halves posted their row max
+                float up, down;
+                row_pow2(fmaxf(mxb[t], mxb[BM + t]), up, down);
+                cs.rsc = down;
+#pragma unroll
+                for (int e = 0; e < 48; e += 2)
+                    pk[e / 2] = pack_f16x2(__uint_as_float(rs[e]) * up, __uint_as_float(rs[e + 1]) * up);
                 // the dS buffer is free once out(j-1) completed
                 if (j >= 1) mbar_wait(&acc_full[(j - 1) & 1], ((j - 1) >> 1) & 1);
                 if (tr) trace_ev(p, j, 6);
@@ -505,25 +570,36 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             } else {
                 const float4* cL = reinterpret_cast<const float4*>(cl + c0);
                 const float4* cD = reinterpret_cast<const float4*>(cl + NK + c0);
+                mbar_wait(&hs_full[j & 1], (j >> 1) & 1);
+                const float* tab = hscale + (j & 1) * NK + c0;   // 2^-f of the Q_h rows (columns)
+                float mx = 0.f;
 #pragma unroll
                 for (int e4 = 0; e4 < 12; ++e4) {
                     const float4 l4 = cL[e4], d4 = cD[e4];
                     const float lv[4] = {l4.x * LOG2E, l4.y * LOG2E, l4.z * LOG2E, l4.w * LOG2E};
                     const float dvv[4] = {d4.x, d4.y, d4.z, d4.w};
-                    float pv[4], dv[4];
+                    float pv[4];
 #pragma unroll
                     for (int x = 0; x < 4; ++x) {
                         const int e = 4 * e4 + x;
                         pv[x] = ((bits >> e) & 1ull) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lv[x])) : 0.f;
-                        dv[x] = pv[x] * (__uint_as_float(rd[e]) - dvv[x]);
+                        const float dsv = pv[x] * (__uint_as_float(rd[e]) - dvv[x]) * tab[e];
+                        rd[e] = __float_as_uint(dsv);
+                        mx = fmaxf(mx, fabsf(dsv));
                     }
                     pk[2 * e4] = pack_bf16x2(pv[0], pv[1]);
                     pk[2 * e4 + 1] = pack_bf16x2(pv[2], pv[3]);
-                    pk2[2 * e4] = pack_f16x2(dv[0], dv[1]);
-                    pk2[2 * e4 + 1] = pack_f16x2(dv[2], dv[3]);
                 }
-                named_bar_sync(1 + wq, 64);   // both halves read S^T / dP^T
+                float* mxb = mxh + (j & 1) * 2 * BM;
+                mxb[h * BM + t] = mx;
+                named_bar_sync(1 + wq, 64);   // both halves read S^T / dP^T and posted their row max
                 if (tr) trace_ev(p, j, 7);
+                float up, down;
+                row_pow2(fmaxf(mxb[t], mxb[BM + t]), up, down);
+                cs.rsc = down;
+#pragma unroll
+                for (int e = 0; e < 48; e += 2)
+                    pk2[e / 2] = pack_f16x2(__uint_as_float(rd[e]) * up, __uint_as_float(rd[e + 1]) * up);
                 // P^T (bf16) | dS^T (fp16) over S^T
                 st_operand(tS, pk);
                 st_operand(tS + 96, pk2);

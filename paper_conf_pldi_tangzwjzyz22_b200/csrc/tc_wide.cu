@@ -83,9 +83,6 @@ struct WParams {
     SchedParams sc;
     int nq, nks, nvs;   // Q buffers, K ring slots, V ring slots
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace, mode 0)
-    int dbg;                     // 0 unless built with FT_WIDE_DBG_KNOBS; timing experiments only
-                                 // (FT_WIDE_DBG): 1 no softmax math,
-                                 // 2 no O MMAs, 4 no S MMAs, 8 no TMA loads -- results are wrong
 };
 
 // Phase trace, per CTA and local tile j < 8, 48 uint64 slots (ns): softmax 0 tile start,
@@ -227,22 +224,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                 for (int i = 0; i < nkc; ++i) {
                     const int c = (mid + i) % nkc, row = T.m0 - w + c * KC;
                     mbar_wait(&k_empty[kr.s], kr.ph ^ 1u);
-                    if (p.dbg & 8) {
-                        mbar_arrive(&k_full[kr.s]);
-                    } else {
-                        mbar_arrive_expect_tx(&k_full[kr.s], TB);
-                        for (int s = 0; s < nds; ++s)
-                            tma_load_3d(sK + (size_t)kr.s * TB + s * BOX, &mp.k, &k_full[kr.s], s * 64, row, T.u);
-                    }
+                    mbar_arrive_expect_tx(&k_full[kr.s], TB);
+                    for (int s = 0; s < nds; ++s)
+                        tma_load_3d(sK + (size_t)kr.s * TB + s * BOX, &mp.k, &k_full[kr.s], s * 64, row, T.u);
                     kr.adv(p.nks);
                     mbar_wait(&v_empty[vr.s], vr.ph ^ 1u);
-                    if (p.dbg & 8) {
-                        mbar_arrive(&v_full[vr.s]);
-                    } else {
-                        mbar_arrive_expect_tx(&v_full[vr.s], TB);
-                        for (int s = 0; s < nds; ++s)
-                            tma_load_3d(sV + (size_t)vr.s * TB + s * BOX, &mp.v, &v_full[vr.s], s * 64, row, T.u);
-                    }
+                    mbar_arrive_expect_tx(&v_full[vr.s], TB);
+                    for (int s = 0; s < nds; ++s)
+                        tma_load_3d(sV + (size_t)vr.s * TB + s * BOX, &mp.v, &v_full[vr.s], s * 64, row, T.u);
                     vr.adv(p.nvs);
                 }
                 ++j;
@@ -276,7 +265,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                     tc_fence_after();
                     if (tr) w_k += gtime() - t0;
                     const uint32_t sb = smem_u32(sK + (size_t)kr.s * TB);
-                    for (int s = 0; s < ((p.dbg & 4) ? 0 : nds); ++s)
+                    for (int s = 0; s < nds; ++s)
                         mma_ss_x4<2, 2>(tbase + 128u * b, sdesc_sw128(sa + s * BOX, 16, 1024),
                                         sdesc_sw128(sb + s * BOX, 16, 1024), idS, s != 0);
                     mma_commit(&k_empty[kr.s]);
@@ -319,7 +308,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                     const uint32_t tO0 = tbase + 256u + (uint32_t)(ob * 2 * d);
                     const uint32_t tO1 = tO0 + (uint32_t)d;
                     const uint32_t sPa = smem_u32(sP + (size_t)b * PBUF);
-                    if (!(p.dbg & 2)) {   // 4 K-steps per partial, one asm block each
+                    {   // 4 K-steps per partial, one asm block each
                         const uint32_t acc = i > 0 ? 1u : 0u;
                         if (PSM) {   // P_c from smem: 64-key atoms of 16 KB, 32 B per step
                             mma_ss_x4<2, 128>(tO0, sdesc_sw128(sPa, 16, 1024), sdesc_sw128(sb, BOX, 1024), idO, acc);
@@ -381,10 +370,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                 mbar_wait(&s_full[b], (gk >> 1) & 1);
                 tc_fence_after();
                 if (tr) { t1 = gtime(); acc_t[0] += t1 - t0; t0 = t1; }
-                const bool dead = p.dbg & 1;
                 // Live: some row of the warp has band columns in sub-chunk sc (warp-uniform);
                 // inner: every row / column of it is in the band and the sequence.
-                auto live = [&](int sc) { const int h0 = c * KC + sc * 32; return !dead && h0 + 31 >= hlo && h0 <= hhi; };
+                auto live = [&](int sc) { const int h0 = c * KC + sc * 32; return h0 + 31 >= hlo && h0 <= hhi; };
                 auto inner = [&](int sc) {
                     const int h0 = c * KC + sc * 32;
                     return h0 >= hlo + 31 && h0 + 31 <= hlo + 2 * w && kb + h0 >= 0 && kb + h0 + 31 < Lr;
@@ -672,12 +660,6 @@ cudaError_t tc_wide_fwd(const void* q, const void* k, const void* v, void* out, 
         p.nks = nks;
         p.nvs = nvs;
         p.trace = (unsigned long long*)trace_buffer(0);
-#ifdef FT_WIDE_DBG_KNOBS   // deletion experiments of profiles/README.md; never in the default build
-        {
-            const char* e = getenv("FT_WIDE_DBG");
-            p.dbg = e ? atoi(e) : 0;
-        }
-#endif
         const int64_t Lr0 = ceil_div(L - r0, dil);
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;

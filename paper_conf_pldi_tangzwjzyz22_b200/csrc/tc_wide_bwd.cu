@@ -749,10 +749,8 @@ cudaError_t tc_wide_bwd(const void* q, const void* k, const void* v, const void*
                         const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
                         int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
                         cudaStream_t st, int* launches) {
-    // WQ in one pass with the D correction; FT_WINATTN_WQ_TWOPASS=1 restores the two-pass
-    // schedule (exact D first, then dS = P (dP - D)) for A/B timing
-    const char* e2 = getenv("FT_WINATTN_WQ_TWOPASS");
-    const int wqc = (e2 && atoi(e2) == 1) ? 0 : 1;
+    // WQ in one pass with the D correction (reading R1)
+    const int wqc = 1;
     // WQ: rows Q (a1) / dO (a2), halo K (b1) / V (b2) -> dQ;  WKV: rows K / V, halo Q / dO -> dV, dK
     cudaError_t e = launch<WQ>(q, dout, k, v, dq, nullptr, lse, Dws, B, H, L, d, w, dil, wqc, dout, out, st,
                                launches);

@@ -158,11 +158,12 @@ def _halos(L: int, w: int, dilation: int, group=None):
     h = min(w * dilation, L)
     hl = min(h, lo)              # rows of rank-1 this rank needs
     hr = min(h, L - hi)          # rows of rank+1
-    for r in (rank - 1, rank + 1):
-        if 0 <= r < world:
-            a, b = seq_bounds(L, world, r)
-            if b - a < min(h, L):
-                raise ValueError("context parallel needs every rank to own >= w*dilation rows")
+    # rank-independent condition (the smallest slice, L // world rows, must hold a whole halo),
+    # so that every rank raises before any communication instead of some ranks waiting on a
+    # peer that raised
+    if world > 1 and L // world < h:
+        raise ValueError(f"context parallel needs every rank to own >= w*dilation = {h} rows "
+                         f"(L = {L} over {world} ranks gives {L // world})")
     return lo, hi, hl, hr
 
 

@@ -32,7 +32,7 @@ def declared_symbols():
 
 def test_header_declares_the_boundary():
     syms = declared_symbols()
-    for s in ("ft_winattn_fwd", "ft_winattn_bwd", "ft_winattn_bwd_workspace_bytes",
+    for s in ("ft_winattn_fwd", "ft_winattn_bwd", "ft_winattn_fwd_bwd", "ft_winattn_bwd_workspace_bytes",
               "ft_winattn_plan", "ft_status_str", "ft_winattn_abi_version"):
         assert s in syms
 
@@ -43,7 +43,7 @@ def test_library_exports_every_declared_symbol(lib):
     exported = set(re.findall(r"\bT\s+(\w+)", out))
     missing = [s for s in declared_symbols() if s not in exported]
     assert not missing, missing
-    assert lib.ft_winattn_abi_version() == 1
+    assert lib.ft_winattn_abi_version() == 2
 
 
 def test_library_is_sm100a(lib):
@@ -106,6 +106,51 @@ def test_bwd_validation(lib):
     assert bwd_call(lib, alias=(6, 0)) == INVALID        # dq aliases q
     assert bwd_call(lib, alias=(7, 6)) == INVALID        # dk aliases dq
     assert bwd_call(lib, d=8) == NOTSUP
+
+
+def fwd_bwd_call(lib, alias=None, B=1, H=1, L=64, d=64, w=4, dil=1, dt=1, ws_bytes=None):
+    """ft_winattn_fwd_bwd(q, k, v, dout, out, lse, dq, dk, dv, ..., workspace, bytes, stream)"""
+    need = lib.ft_winattn_bwd_workspace_bytes(B, H, L, d, w, dil, dt)
+    args = [P(i) for i in range(9)]
+    if alias:
+        args[alias[0]] = args[alias[1]]
+    return lib.ft_winattn_fwd_bwd(*args, B, H, L, d, w, dil, dt, P(9),
+                                  need if ws_bytes is None else ws_bytes, None)
+
+
+def test_fwd_bwd_validation(lib):
+    """the combined call rejects what either half rejects, and also dout overlapping out / lse
+    (out and lse are outputs of the call)"""
+    assert fwd_bwd_call(lib, w=-1) == INVALID
+    assert fwd_bwd_call(lib, ws_bytes=0) == INVALID
+    assert fwd_bwd_call(lib, alias=(4, 3)) == INVALID    # out aliases dout
+    assert fwd_bwd_call(lib, alias=(5, 3)) == INVALID    # lse aliases dout
+    assert fwd_bwd_call(lib, alias=(4, 0)) == INVALID    # out aliases q
+    assert fwd_bwd_call(lib, alias=(6, 4)) == INVALID    # dq aliases out
+    assert fwd_bwd_call(lib, alias=(8, 5)) == INVALID    # dv aliases lse
+    assert fwd_bwd_call(lib, d=24) == NOTSUP
+    bad = [P(i) for i in range(9)]
+    bad[3] = P(3, 8)
+    need = lib.ft_winattn_bwd_workspace_bytes(1, 1, 64, 64, 4, 1, 1)
+    assert lib.ft_winattn_fwd_bwd(*bad, 1, 1, 64, 64, 4, 1, 1, P(9), need, None) == MISALIGNED
+
+
+def test_debug_knobs(lib):
+    """ft_winattn_debug_set / get: documented knobs and values only; plan() follows the path knob"""
+    assert lib.ft_winattn_debug_set(7, 1) == INVALID
+    assert lib.ft_winattn_debug_set(0, 3) == INVALID
+    assert lib.ft_winattn_debug_set(1, 2) == INVALID
+    assert lib.ft_winattn_debug_get(9) == -1
+    with ft.knobs(path="simt"):
+        assert ft.debug_get("path") == 1
+        assert ft.plan(False, 1, 8, 10000, 512, 32, 1, ft.FT_BF16)[0] == ft.PATH_SIMT
+    with ft.knobs(path="tc"):
+        with pytest.raises(ft.FtError):   # no tensor-core kernel for d = 48
+            ft.plan(False, 1, 1, 300, 48, 4, 1, ft.FT_BF16)
+    assert ft.debug_get("path") == 0
+    with ft.knobs(narrow=0, pdl=0):
+        assert ft.debug_get("narrow") == 0 and ft.debug_get("pdl") == 0
+    assert ft.debug_get("narrow") == 1 and ft.debug_get("pdl") == 1
 
 
 def test_workspace_and_plan(lib):

@@ -132,3 +132,37 @@ def test_context_parallel_matches_full_sequence(world, shape):
         p.join(timeout=60)
     for rank, errs in res:
         assert max(errs) < 1e-12, (rank, errs)
+
+
+def _halo_check_worker(rank, world, port, L, w, dil, result_q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_pldi_tangzwjzyz22_b200.dist import cp_fwd, seq_bounds
+        lo, hi = seq_bounds(L, world, rank)
+        x = torch.zeros(1, 1, hi - lo, 8, dtype=torch.float64)
+        try:
+            cp_fwd(x, x, x, w, dil, L, fwd_fn=_oracle_fwd_t)
+            result_q.put((rank, "ran"))
+        except ValueError:
+            result_q.put((rank, "raised"))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_context_parallel_rejects_short_slices_on_every_rank():
+    """L = 11 over 3 ranks (slices 4 / 4 / 3) with a halo of 4 rows: the smallest slice cannot
+    hold a halo, and EVERY rank must raise before any communication (a rank-dependent check
+    would leave the others waiting on it)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_halo_check_worker, args=(r, 3, port, 11, 4, 1, q)) for r in range(3)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=120) for _ in range(3))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert res == {0: "raised", 1: "raised", 2: "raised"}

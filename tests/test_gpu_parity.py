@@ -2,7 +2,7 @@
 seeded inputs.  Run on a B200 with ``pytest -m gpu``.
 
 * element-by-element at sizes the oracle finishes in seconds, spanning several tiles and a
-  ragged tail, for both kernel families (FT_WINATTN_PATH=simt|tc forces one);
+  ragged tail, for both kernel families (ft.knobs(path="simt"|"tc") forces one);
 * sampled rows at BASELINE.json's full sizes (C2a, C2b, C4, C5 corners) and one 2^21-row
   sequence, in the launch configuration
   bench.py times, against the oracle's per-row entry points;
@@ -33,22 +33,11 @@ def ft():
     return ft
 
 
-class forced_path:
-    def __init__(self, path):
-        self.path = path
+def forced_path(path):
+    """force a kernel family for the block (debug knob FT_KNOB_PATH), None = automatic"""
+    import paper_conf_pldi_tangzwjzyz22_b200 as ft
 
-    def __enter__(self):
-        self.old = os.environ.get("FT_WINATTN_PATH")
-        if self.path:
-            os.environ["FT_WINATTN_PATH"] = self.path
-        else:
-            os.environ.pop("FT_WINATTN_PATH", None)
-
-    def __exit__(self, *a):
-        if self.old is None:
-            os.environ.pop("FT_WINATTN_PATH", None)
-        else:
-            os.environ["FT_WINATTN_PATH"] = self.old
+    return ft.knobs(path=path or "auto")
 
 
 def _dtype_code(dtype):
@@ -125,14 +114,12 @@ def test_simt_parity(ft, shape, dtype):
 
 def _tc_ok(ft, shape, bwd=False):
     B, H, L, d, w, dil = shape
-    os.environ["FT_WINATTN_PATH"] = "tc"
-    try:
-        ft.plan(bwd, B, H, L, d, w, dil, 1)
-        return True
-    except ft.FtError:
-        return False
-    finally:
-        os.environ.pop("FT_WINATTN_PATH", None)
+    with ft.knobs(path="tc"):
+        try:
+            ft.plan(bwd, B, H, L, d, w, dil, 1)
+            return True
+        except ft.FtError:
+            return False
 
 
 @pytest.mark.parametrize("shape", SMALL + WIDE, ids=lambda s: "x".join(map(str, s)))
@@ -284,10 +271,46 @@ def _sample_rows(shape: WinAttnShape, n_mid: int, seed: int):
     return np.array(sorted(rows), dtype=np.int64)
 
 
-@pytest.mark.parametrize("name,dtype", [("C2a", "bf16"), ("C2a", "f32"), ("C2a_dil", "bf16"),
-                                        ("C2b", "bf16"), ("C4d2", "bf16"), ("C4d4", "bf16"),
-                                        ("C5_big_w32", "bf16"), ("C5_big_w256", "bf16"),
-                                        ("long_2M", "bf16")])
+@pytest.mark.parametrize("name,dtype", [("C2a", "bf16"), ("C2a", "f32"), ("C2b", "bf16"), ("C2b", "f32"),
+                                        ("C2a_dil", "bf16")])
+def test_full_size_elementwise(ft, name, dtype):
+    """SURVEY.md §8(d) "run the full oracle for C1-C3": every element of out, lse, dq, dk, dv at
+    the paper-shaped sizes, in the launch configuration bench.py times."""
+    shape = CONFIGS[name]
+    x = make_inputs(shape, 0, dtype)
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    out, lse = ft.fwd(q, k, v, shape.w, shape.dilation)
+    dq, dk, dv = ft.bwd(q, k, v, out, lse, g, shape.w, shape.dilation)
+    torch.cuda.synchronize()
+    ro, rl = oracle.fwd(x["q64"], x["k64"], x["v64"], shape.w, shape.dilation)
+    rq, rk, rv = oracle.bwd(x["q64"], x["k64"], x["v64"], ro, rl, x["dout64"], shape.w, shape.dilation)
+    for n, a, r in (("out", out, ro), ("lse", lse, rl), ("dq", dq, rq), ("dk", dk, rk), ("dv", dv, rv)):
+        compare(n, a.double().cpu().numpy(), r, dtype)
+
+
+@pytest.mark.parametrize("name", ["C4d2", "C4d4", "C5_big_w32", "C5_big_w256", "C5_small_w32"])
+def test_full_size_whole_units(ft, name):
+    """C4 / C5 at full size: the first and last (batch, head) units compared element by element
+    (units are independent problems, Fig. 8's outer loop), every value finite."""
+    shape = CONFIGS[name]
+    x = make_inputs(shape, 0, "bf16")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    out, lse = ft.fwd(q, k, v, shape.w, shape.dilation)
+    dq, dk, dv = ft.bwd(q, k, v, out, lse, g, shape.w, shape.dilation)
+    torch.cuda.synchronize()
+    for t in (out, lse, dq, dk, dv):
+        assert torch.isfinite(t).all()
+    for h in sorted({0, shape.heads - 1}):
+        s = {n: np.ascontiguousarray(x[n + "64"][:, h:h + 1]) for n in ("q", "k", "v", "dout")}
+        ro, rl = oracle.fwd(s["q"], s["k"], s["v"], shape.w, shape.dilation)
+        rq, rk, rv = oracle.bwd(s["q"], s["k"], s["v"], ro, rl, s["dout"], shape.w, shape.dilation)
+        for n, a, r in (("out", out, ro), ("lse", lse, rl), ("dq", dq, rq), ("dk", dk, rk), ("dv", dv, rv)):
+            compare(f"{n}[head {h}]", a[:, h:h + 1].double().cpu().numpy(), r, "bf16")
+
+
+@pytest.mark.parametrize("name,dtype", [("C2a_dil", "f32"), ("long_2M", "bf16")])
 def test_full_size_sampled(ft, name, dtype):
     shape = CONFIGS[name]
     x = make_inputs(shape, 0, dtype)
@@ -312,27 +335,10 @@ def test_full_size_sampled(ft, name, dtype):
         assert torch.isfinite(t).all()
 
 
-class _env:
-    def __init__(self, **kv):
-        self.kv = kv
-
-    def __enter__(self):
-        self.old = {k: os.environ.get(k) for k in self.kv}
-        os.environ.update(self.kv)
-
-    def __exit__(self, *a):
-        for k, v in self.old.items():
-            if v is None:
-                os.environ.pop(k, None)
-            else:
-                os.environ[k] = v
-
-
-# d = 64, w <= 32 backward in one kernel (tc_narrow_fused.cu), forced even where the dispatcher
-# would pick the split kernels: strips of one tile (every CTA starts with a warm-up tile), strips
-# crossing (unit, residue) boundaries, tails of ragged residues, two launch groups, w = 0 and
-# w < 32, and enough tiles per CTA that the K (5-slot) and V (4-slot) rings wrap many times.
-FUSED = [
+# d = 64, w <= 32 backward (tc_narrow_bwd.cu NQ + NKV): strips crossing (unit, residue)
+# boundaries, tails of ragged residues, two launch groups, w = 0 and w < 32, one-tile problems,
+# and enough tiles per CTA that the 2-stage ring and the TMEM region rotation wrap many times.
+NARROW = [
     (1, 3, 129, 64, 31, 1),
     (1, 2, 300, 64, 32, 3),
     (1, 6, 5000, 64, 7, 3),
@@ -347,13 +353,72 @@ FUSED = [
 ]
 
 
-@pytest.mark.parametrize("shape", FUSED, ids=lambda s: "x".join(map(str, s)))
-def test_narrow_fused_bwd(ft, shape):
+@pytest.mark.parametrize("shape", NARROW, ids=lambda s: "x".join(map(str, s)))
+def test_narrow_bwd(ft, shape):
     sh = WinAttnShape(*shape)
-    with _env(FT_WINATTN_FUSED="2"):
-        p, n = ft.plan(True, sh.batch, sh.heads, sh.seq_len, sh.d, sh.w, sh.dilation, 1)
-        assert p == ft.PATH_TC and n == (min(sh.dilation, sh.seq_len) + 7) // 8
-        run_case(ft, sh, "bf16", None, seed=6)
+    p, n = ft.plan(True, sh.batch, sh.heads, sh.seq_len, sh.d, sh.w, sh.dilation, 1)
+    assert p == ft.PATH_TC and n == 2 * ((min(sh.dilation, sh.seq_len) + 7) // 8)
+    run_case(ft, sh, "bf16", None, seed=6)
+
+
+# Scale equivariance (reading A10): q -> c q, k -> k / c leaves every score, out and lse unchanged
+# and scales dq by g / c, dk by g c, dv by g when dout -> g dout.  With powers of two the bf16
+# inputs scale exactly, so the oracle of the scaled problem is the scaled oracle; every kernel
+# family must meet the same bound relative to the scaled references (no overflow to inf at
+# |q| ~ 1e5 or a 2^16 loss scale, no loss of precision at 2^-24).  Families: narrow (d = 64,
+# w <= 32), band (d = 128, 512; d = 64 with the narrow kernels off), wide (w > 64) and the
+# chunked wide fallback, and the CUDA-core kernels in fp32.
+SCALES = [(2.0 ** 17, 1.0), (2.0 ** -17, 1.0), (1.0, 2.0 ** 16), (1.0, 2.0 ** -24), (2.0 ** 10, 2.0 ** 12)]
+FAMILIES = [
+    ((1, 4, 3000, 64, 32, 1), "bf16", {}),
+    ((1, 2, 1000, 64, 17, 3), "bf16", {}),
+    ((1, 2, 900, 64, 32, 1), "bf16", {"narrow": 0}),
+    ((1, 2, 700, 128, 40, 1), "bf16", {}),
+    ((1, 2, 500, 512, 32, 1), "bf16", {}),
+    ((1, 2, 800, 64, 100, 1), "bf16", {}),
+    ((1, 2, 700, 128, 130, 2), "bf16", {}),
+    ((1, 2, 800, 64, 100, 1), "bf16", {"wide": 0}),
+    ((1, 2, 300, 64, 20, 1), "f32", {}),
+]
+
+
+@pytest.mark.parametrize("case", FAMILIES, ids=lambda c: "x".join(map(str, c[0])) + c[1] + "".join(c[2]))
+def test_scale_equivariance(ft, case):
+    shape, dtype, kn = case
+    sh = WinAttnShape(*shape)
+    x = make_inputs(sh, 14, dtype)
+    dev = torch.device("cuda:0")
+    ro, rl = oracle.fwd(x["q64"], x["k64"], x["v64"], sh.w, sh.dilation)
+    rdq, rdk, rdv = oracle.bwd(x["q64"], x["k64"], x["v64"], ro, rl, x["dout64"], sh.w, sh.dilation)
+    for c, gs in SCALES:
+        q = (x["q"].double() * c).to(x["q"].dtype).to(dev)
+        k = (x["k"].double() / c).to(x["k"].dtype).to(dev)
+        v, g = x["v"].to(dev), (x["dout"].double() * gs).to(x["dout"].dtype).to(dev)
+        with ft.knobs(**kn):
+            out, lse = ft.fwd(q, k, v, sh.w, sh.dilation)
+            dq, dk, dv = ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation)
+        torch.cuda.synchronize()
+        tag = f"c={c:g} g={gs:g} "
+        compare(tag + "out", out.double().cpu().numpy(), ro, dtype)
+        compare(tag + "lse", lse.double().cpu().numpy(), rl, dtype)
+        compare(tag + "dq", dq.double().cpu().numpy() * (c / gs), rdq, dtype)
+        compare(tag + "dk", dk.double().cpu().numpy() / (c * gs), rdk, dtype)
+        compare(tag + "dv", dv.double().cpu().numpy() / gs, rdv, dtype)
+
+
+# Windows wider than the wide kernels' shared-memory plan (halo > ~4096 rows) take the chunked
+# kernels (tc_chunk.cu), as does w >= L at long L; the knob forces them at smaller windows too.
+@pytest.mark.parametrize("case", [((1, 1, 5000, 64, 2000, 1), {}), ((1, 1, 5000, 64, 4096, 1), {}),
+                                  ((1, 1, 5000, 64, 6000, 1), {}), ((1, 2, 5000, 128, 2100, 1), {}),
+                                  ((1, 2, 1100, 64, 256, 3), {"wide": 0}),
+                                  ((2, 1, 300, 128, 130, 1), {"wide": 0}),
+                                  ((1, 1, 90, 64, 100, 1), {"wide": 0})],
+                         ids=lambda c: "x".join(map(str, c[0])) + "".join(c[1]))
+def test_chunk_fallback(ft, case):
+    shape, kn = case
+    sh = WinAttnShape(*shape)
+    with ft.knobs(path="tc", **kn):
+        run_case(ft, sh, "bf16", "tc", seed=15)
 
 
 # Per-head dilation (ft_winattn_fwd_mixed / bwd_mixed): heads
@@ -432,19 +497,21 @@ def test_tape_path(ft, case):
                          ids=lambda s: "x".join(map(str, s)))
 def test_determinism_every_family(ft, shape):
     """Every tensor-core family writes each output row from one CTA without atomics (tile
-    ownership, Fig. 13(d)): split and fused narrow, band (d = 512) and wide kernels give
-    bit-identical results on repeated runs; the fused one also when forced at a small size."""
+    ownership, Fig. 13(d)): narrow, band (d = 512) and wide kernels give bit-identical
+    results on repeated runs, with and without programmatic dependent launch, and through
+    ft_winattn_fwd_bwd."""
     sh = WinAttnShape(*shape)
     x = make_inputs(sh, 12, "bf16")
     dev = torch.device("cuda:0")
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
-    for fused in ("1", "2"):
-        with _env(FT_WINATTN_FUSED=fused):
-            runs = []
-            for _ in range(2):
-                out, lse = ft.fwd(q, k, v, sh.w, sh.dilation)
-                runs.append((out, lse) + ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation))
-        for a, b in zip(*runs):
+    runs = []
+    for pdl in (1, 1, 0):
+        with ft.knobs(pdl=pdl):
+            out, lse = ft.fwd(q, k, v, sh.w, sh.dilation)
+            runs.append((out, lse) + ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation))
+    runs.append(ft.fwd_bwd(q, k, v, g, sh.w, sh.dilation))
+    for r in runs[1:]:
+        for a, b in zip(runs[0], r):
             assert torch.equal(a, b)
 
 
@@ -475,14 +542,14 @@ def test_d_handoff_stale_workspace(ft, shape):
     (tc_common.cuh ld_D_ready). Whatever the workspace
     holds before the call -- the unset marker everywhere, D of different inputs from an
     earlier call, zeros -- the gradients must be bit-identical to the grid-wide-wait
-    schedule (FT_WINATTN_DPOLL=0), and equal the oracle on sampled rows."""
+    schedule (PDL off: FT_KNOB_PDL = 0)."""
     sh = WinAttnShape(*shape)
     x = make_inputs(sh, 21, "bf16")
     y = make_inputs(sh, 22, "bf16")
     dev = torch.device("cuda:0")
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
     out, lse = ft.fwd(q, k, v, sh.w, sh.dilation)
-    with _env(FT_WINATTN_DPOLL="0"):
+    with ft.knobs(pdl=0):
         want = ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation)
     nbytes = ft.workspace_bytes(q, sh.w, sh.dilation)
     ws = torch.empty(max(nbytes, 16), dtype=torch.uint8, device=dev)
@@ -502,42 +569,90 @@ def test_d_handoff_stale_workspace(ft, shape):
 @pytest.mark.parametrize("shape", [(1, 2, 700, 512, 32, 1), (1, 3, 900, 512, 20, 3), (1, 8, 10000, 512, 32, 1),
                                    (1, 2, 3000, 512, 32, 11), (2, 3, 1500, 128, 48, 1),
                                    (1, 8, 4096, 64, 32, 1), (1, 2, 700, 64, 32, 1), (1, 3, 5000, 64, 16, 3),
-                                   (1, 48, 2048, 64, 32, 1)],
+                                   (1, 48, 2048, 64, 32, 1), (1, 2, 900, 64, 100, 1)],
                          ids=lambda s: "x".join(map(str, s)))
-def test_lse_handoff(ft, shape):
-    """The band and narrow forwards mark their lse rows unset and trigger a programmatic
-    dependent launch of the dQ kernel, which polls lse row by row (tc_common.cuh ld_lse_ready; DESIGN.md
-    'lse hand-off'). Directly after its own forward, after the forward of OTHER inputs (so
-    the polled lse is a different, complete buffer), and with an lse buffer that holds the
-    unset marker itself (bounded poll, then a grid-wide wait: must not hang), the results must
-    be bit-identical to the schedule without the hand-off (FT_WINATTN_LSEPOLL=0)."""
+def test_fwd_bwd_handoff(ft, shape):
+    """ft_winattn_fwd_bwd: its forward marks the lse rows and its dQ kernel (PDL) reads each row as
+    the forward stores it (tc_common.cuh ld_lse_ready).  The result
+    must be bit-identical to separate ft_winattn_fwd + ft_winattn_bwd calls and to the schedule
+    without programmatic dependent launch."""
     sh = WinAttnShape(*shape)
     x = make_inputs(sh, 41, "bf16")
-    y = make_inputs(sh, 42, "bf16")
     dev = torch.device("cuda:0")
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
-    q2, k2, v2 = (y[n].to(dev) for n in ("q", "k", "v"))
-    with _env(FT_WINATTN_LSEPOLL="0"):
-        o0, l0 = ft.fwd(q, k, v, sh.w, sh.dilation)
-        want = ft.bwd(q, k, v, o0, l0, g, sh.w, sh.dilation)
-        bad = torch.full_like(l0, float("nan")).view(torch.int32).fill_(-1).view(torch.float32)
-        want_bad = ft.bwd(q, k, v, o0, bad, g, sh.w, sh.dilation)
+    o0, l0 = ft.fwd(q, k, v, sh.w, sh.dilation)
+    want = (o0, l0) + ft.bwd(q, k, v, o0, l0, g, sh.w, sh.dilation)
+    got = ft.fwd_bwd(q, k, v, g, sh.w, sh.dilation)
+    with ft.knobs(pdl=0):
+        got0 = ft.fwd_bwd(q, k, v, g, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    for a, b, c in zip(got, want, got0):
+        assert torch.equal(a, b) and torch.equal(c, b)
+
+
+@pytest.mark.parametrize("shape", [(1, 8, 10000, 512, 32, 1), (1, 2, 700, 512, 32, 1), (1, 8, 4096, 64, 32, 1),
+                                   (1, 48, 2048, 64, 32, 1), (1, 2, 900, 64, 100, 1), (1, 3, 900, 512, 20, 3)],
+                         ids=lambda s: "x".join(map(str, s)))
+def _early_trigger_lib():
+    import ctypes
+    import subprocess
+    import tempfile
+
+    src = os.path.join(os.path.dirname(os.path.abspath(__file__)), "helpers", "early_trigger.cu")
+    so = os.path.join(tempfile.mkdtemp(prefix="ft_early_"), "libearly.so")
+    subprocess.run(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O2", "-shared", "-Xcompiler",
+                    "-fPIC", "-o", so, src], check=True)
+    lib = ctypes.CDLL(so)
+    lib.early_trigger_copy_launch.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_longlong,
+                                              ctypes.c_longlong, ctypes.c_void_p]
+    lib.early_trigger_copy_launch.restype = ctypes.c_int
+    return lib
+
+
+def test_stream_order_aliasing(ft, shape):
+    """ft_winattn_bwd never starts before the work enqueued ahead of it (include/ft_winattn.h
+    "Async").  (i) out.backward(out): dout IS the out the forward just wrote, enqueued directly
+    after that forward; (ii) the workspace and gradients come from blocks the caching allocator
+    freed right after a still-running forward (its discarded out / lse); (iii) dout is produced
+    by an unrelated kernel directly before the backward.  Each must equal the same calls with a
+    device synchronize in between."""
+    sh = WinAttnShape(*shape)
+    x = make_inputs(sh, 43, "bf16")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    # reference: fully serialised
+    o, l = ft.fwd(q, k, v, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    want_i = ft.bwd(q, k, v, o, l, o, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    want = ft.bwd(q, k, v, o, l, g, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    # (i) dout = out of the forward enqueued just before
     o1, l1 = ft.fwd(q, k, v, sh.w, sh.dilation)
-    got = ft.bwd(q, k, v, o1, l1, g, sh.w, sh.dilation)
+    got = ft.bwd(q, k, v, o1, l1, o1, sh.w, sh.dilation)
     torch.cuda.synchronize()
-    assert torch.equal(o1, o0) and torch.equal(l1, l0)
-    for a, b in zip(got, want):
+    for a, b in zip(got, want_i):
         assert torch.equal(a, b)
-    ft.fwd(q2, k2, v2, sh.w, sh.dilation)   # another problem's forward precedes the backward
-    got = ft.bwd(q, k, v, o0, l0, g, sh.w, sh.dilation)
-    torch.cuda.synchronize()
-    for a, b in zip(got, want):
-        assert torch.equal(a, b)
-    ft.fwd(q2, k2, v2, sh.w, sh.dilation)
-    got = ft.bwd(q, k, v, o0, bad, g, sh.w, sh.dilation)
-    torch.cuda.synchronize()
-    for a, b in zip(got, want_bad):
-        assert torch.equal(a.isnan(), b.isnan())
+    # (ii) a forward whose outputs are freed at once; the backward's buffers reuse those blocks
+    for _ in range(3):
+        tmp_o, tmp_l = ft.fwd(q, k, v, sh.w, sh.dilation)
+        del tmp_o, tmp_l
+        got = ft.bwd(q, k, v, o, l, g, sh.w, sh.dilation)   # allocates ws / dq / dk / dv
+        torch.cuda.synchronize()
+        for a, b in zip(got, want):
+            assert torch.equal(a, b)
+    # (iii) dout written right before the backward by a foreign kernel that triggers its
+    # dependents at once and stores only after ~0.3 ms (tests/helpers/early_trigger.cu)
+    helper = _early_trigger_lib()
+    gbuf = torch.empty_like(g)
+    for _ in range(3):
+        gbuf.zero_()
+        assert helper.early_trigger_copy_launch(g.data_ptr(), gbuf.data_ptr(), g.numel() * g.element_size(),
+                                                300_000, torch.cuda.current_stream().cuda_stream) == 0
+        got = ft.bwd(q, k, v, o, l, gbuf, sh.w, sh.dilation)
+        torch.cuda.synchronize()
+        for a, b in zip(got, want):
+            assert torch.equal(a, b)
 
 
 @pytest.mark.parametrize("shape", [(1, 4, 1200, 512, 32, 4, 1), (2, 3, 900, 64, 32, 2, 2), (2, 3, 700, 64, 100, 3, 1)],
@@ -545,14 +660,14 @@ def test_lse_handoff(ft, shape):
 def test_mixed_side_stream_and_graph(ft, shape):
     """ft_winattn_*_mixed runs its head-group slices on the caller's stream and a library side
     stream (fork / join through events). The result must be bit-identical to the all-on-one-
-    stream schedule (FT_WINATTN_MIXED_SERIAL=1), and the call must be capturable in a CUDA
+    stream schedule (FT_KNOB_SIDE = 0), and the call must be capturable in a CUDA
     graph whose replay gives the same result again."""
     B, H, L, d, w, dil, hd = shape
     sh = WinAttnShape(B, H, L, d, w, dil)
     x = make_inputs(sh, 31, "bf16")
     dev = torch.device("cuda:0")
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
-    with _env(FT_WINATTN_MIXED_SERIAL="1"):
+    with ft.knobs(side=0):
         o1, l1 = ft.fwd(q, k, v, w, dil, dilated_heads=hd)
         want = (o1, l1) + ft.bwd(q, k, v, o1, l1, g, w, dil, dilated_heads=hd)
     o2, l2 = ft.fwd(q, k, v, w, dil, dilated_heads=hd)
