@@ -411,13 +411,14 @@ def test_scale_equivariance(ft, case):
 @pytest.mark.parametrize("case", [((1, 1, 5000, 64, 2000, 1), {}), ((1, 1, 5000, 64, 4096, 1), {}),
                                   ((1, 1, 5000, 64, 6000, 1), {}), ((2, 1, 3000, 64, 1990, 1), {}),
                                   ((1, 2, 1100, 64, 256, 3), {"wide": 0}),
-                                  ((2, 1, 300, 128, 130, 1), {"wide": 0}),
+                                  ((2, 1, 300, 64, 130, 1), {"wide": 0}),
                                   ((1, 1, 90, 64, 100, 1), {"wide": 0})],
                          ids=lambda c: "x".join(map(str, c[0])) + "".join(c[1]))
 def test_chunk_fallback(ft, case):
     shape, kn = case
     sh = WinAttnShape(*shape)
-    with ft.knobs(path="tc", **kn):
+    with ft.knobs(**kn):
+        assert _tc_ok(ft, shape) and _tc_ok(ft, shape, bwd=True)
         run_case(ft, sh, "bf16", "tc", seed=15)
 
 
@@ -590,9 +591,6 @@ def test_fwd_bwd_handoff(ft, shape):
         assert torch.equal(a, b) and torch.equal(c, b)
 
 
-@pytest.mark.parametrize("shape", [(1, 8, 10000, 512, 32, 1), (1, 2, 700, 512, 32, 1), (1, 8, 4096, 64, 32, 1),
-                                   (1, 48, 2048, 64, 32, 1), (1, 2, 900, 64, 100, 1), (1, 3, 900, 512, 20, 3)],
-                         ids=lambda s: "x".join(map(str, s)))
 def _early_trigger_lib():
     import ctypes
     import subprocess
@@ -609,6 +607,9 @@ def _early_trigger_lib():
     return lib
 
 
+@pytest.mark.parametrize("shape", [(1, 8, 10000, 512, 32, 1), (1, 2, 700, 512, 32, 1), (1, 8, 4096, 64, 32, 1),
+                                   (1, 48, 2048, 64, 32, 1), (1, 2, 900, 64, 100, 1), (1, 3, 900, 512, 20, 3)],
+                         ids=lambda s: "x".join(map(str, s)))
 def test_stream_order_aliasing(ft, shape):
     """ft_winattn_bwd never starts before the work enqueued ahead of it (include/ft_winattn.h
     "Async").  (i) out.backward(out): dout IS the out the forward just wrote, enqueued directly
