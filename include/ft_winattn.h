@@ -76,7 +76,9 @@ typedef enum { FT_F32 = 0, FT_BF16 = 1 } ft_dtype;
  * ft_winattn_debug_set(FT_KNOB_PATH, ...)). */
 typedef enum {
     FT_PATH_SIMT = 0,   /* CUDA-core FMA kernels (fp32 math), any dtype / d / w      */
-    FT_PATH_TC = 1      /* tcgen05/TMEM tensor-core kernels, bf16 only               */
+    FT_PATH_TC = 1      /* tcgen05/TMEM tensor-core kernels: bf16 (any w, d % 64 == 0,
+                           d <= 512 for w <= 64; d in {64, 128} above), and fp32 as bf16
+                           hi / lo planes with 3 products (w <= 32, d % 64 == 0)        */
 } ft_path;
 
 /* Forward.  q, k, v: [B,H,L,d] dtype (inputs).  out: [B,H,L,d] dtype, lse: [B,H,L]

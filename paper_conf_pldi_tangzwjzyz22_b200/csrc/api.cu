@@ -74,8 +74,9 @@ int forced_path() { return ftw::knob(ftw::K_PATH); }
 
 ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil, ft_dtype dt,
                       int* path) {
-    const bool tc_ok = dt == FT_BF16 && (is_bwd ? ftw::tc_bwd_supported(units, L, d, w, dil)
-                                                : ftw::tc_fwd_supported(units, L, d, w, dil));
+    const bool tc_ok = dt == FT_BF16 ? (is_bwd ? ftw::tc_bwd_supported(units, L, d, w, dil)
+                                               : ftw::tc_fwd_supported(units, L, d, w, dil))
+                                     : ftw::tc32_supported(units, L, d, w, dil);
     const int f = forced_path();
     if (f == 1) { *path = FT_PATH_SIMT; return FT_OK; }
     if (f == 2) {
@@ -163,7 +164,9 @@ ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_
     s = choose_path(is_bwd, batch * heads, seq_len, d, w, dilation, dtype, &p);
     if (s != FT_OK) return s;
     int n;
-    if (p == FT_PATH_TC)
+    if (p == FT_PATH_TC && dtype == FT_F32)
+        n = is_bwd ? ftw::tc32_bwd_launches(seq_len, dilation) : ftw::tc32_fwd_launches(seq_len, dilation);
+    else if (p == FT_PATH_TC)
         n = is_bwd ? ftw::tc_bwd_launches(batch * heads, seq_len, d, w, dilation)
                    : ftw::tc_fwd_launches(seq_len, d, w, dilation);
     else
@@ -206,7 +209,10 @@ ft_status run_fwd(const void* q, const void* k, const void* v, void* out, float*
     if (s != FT_OK) return s;
     cudaStream_t st = (cudaStream_t)stream;
     cudaError_t e;
-    if (path == FT_PATH_TC) {
+    if (path == FT_PATH_TC && dtype == FT_F32) {
+        int n = 0;
+        e = ftw::tc32_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, st, &n);
+    } else if (path == FT_PATH_TC) {
         int n = 0;
         e = ftw::tc_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, st, &n);
     } else {
@@ -257,7 +263,10 @@ ft_status run_bwd(const void* q, const void* k, const void* v, const void* out, 
     cudaStream_t st = (cudaStream_t)stream;
     float* Dws = (float*)workspace;
     cudaError_t e;
-    if (path == FT_PATH_TC) {
+    if (path == FT_PATH_TC && dtype == FT_F32) {
+        int n = 0;
+        e = ftw::tc32_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w, dilation, st, &n);
+    } else if (path == FT_PATH_TC) {
         int n = 0;
         e = ftw::tc_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w,
                         dilation, st, &n);

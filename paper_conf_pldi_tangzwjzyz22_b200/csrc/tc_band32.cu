@@ -1,0 +1,713 @@
+// tc_band32.cu -- tensor-core kernels for fp32 window attention on sm_100a (the paper's precision:
+// "f32", Fig. 8), windows with w <= 32 (halo NK = round_up(128 + 2w, 64) <= 192
+// rows), d a multiple of 64 up to 512: the C2a shape of BASELINE configs[1-2].
+//
+// Arithmetic.  Every fp32 operand x enters the tensor cores as a pair of bf16 planes,
+// hi = bf16(x) and lo = bf16(x - hi) (16 significant bits), and every product as three bf16 MMAs
+// hi.hi + hi.lo + lo.hi into an fp32 TMEM accumulator; the dropped lo.lo term and the rounding of
+// lo are ~2^-17 relative.  Softmax, lse, D and all accumulations stay fp32.  A simulation of this
+// arithmetic on the C2a shape puts every output within 0.41 of the north_star bound (rtol 1e-4,
+// atol 1e-4 max|R|); tests/test_gpu_parity.py checks the kernels element by element.  kind::tf32
+// would need 3 MMAs at half the bf16 rate and K-major operands only (tools/tf32_modes_probe.cu:
+// MN-major tf32 B operands are not executed), i.e. transposed copies of V, K, dO, Q for the
+// output products; the bf16 planes keep the MN-major B operands of tc_band.cu.
+//
+// Data movement.  TMA loads fp32 boxes of 32 columns (128-byte rows, SWIZZLE_128B) into a ring
+// slot; two converter warps then rewrite each row IN PLACE as its two bf16 planes: the 64 fp32
+// values of a row held by the box pair (cols 0-31 | cols 32-63, at the same row offset of two
+// boxes) become the 64-column hi row (over the first box) and lo row (over the second), which
+// are exactly the K-major SWIZZLE_128B bf16 layouts the MMAs read (score GEMMs), or, for the
+// 64-key x 128-column output blocks, the MN-major bf16 boxes (LBO 16 KB between the two 64-column
+// groups).  So a slot holds fp32 and its planes in the same 80 KB, and the HBM bytes are those of
+// the fp32 tensors: 4de + 4 per row forward, 5de + 8 / 6de + 8 per row for the two backward
+// kernels (the same kernel split as tc_band.cu).
+//
+// One persistent kernel template, three modes; a CTA owns BM = 128 rows of one (unit, residue)
+// band problem and its NK-row halo (the cached window of PAPER.md Fig. 14):
+//   FWD   S = Q K_h^T -> max, exp, sum (Fig. 8 / 10 dot, dot_max, softmax, PAPER.md:215-231,
+//         306-321), lse -> HBM, P (hi|lo packed over S in TMEM) ; O_c = P V_h,c per 128-column
+//         chunk, scaled by 1/l.  S alternates between two TMEM regions so the next tile's score
+//         GEMM runs while this tile's softmax and output GEMMs do.
+//   BWDQ  S = Q K_h^T, dP = dO V_h^T; P = exp(S - lse) (recomputed from the saved lse, PAPER.md:
+//         489-497); D = sum_j P dP (exact, reading R1) -> workspace; dS = P (dP - D) (hi|lo over
+//         S) ; dQ_c = dS K_h,c.
+//   BWDKV rows = keys (each dk / dv row has one writer, Fig. 13(d)); S^T = K Q_h^T,
+//         dP^T = V dO_h^T; P^T (hi|lo over dP^T), dS^T (hi|lo over S^T); dV_c = P^T dO_h,c,
+//         dK_c = dS^T Q_h,c.
+//
+// Roles (384 threads): warps 0-3 softmax (thread t <-> row m0 + t <-> TMEM lane t), 4-7
+// epilogue (TMEM -> fp32 -> smem -> TMA store), 8 TMA producer + TMEM allocator, 9 MMA issuer,
+// 10-11 converters (12 warps keep the register cap at 168 per thread).  TMEM: R0 = [0, 192),
+// R1 = [192, 384), the output accumulator [384, 512).
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <mutex>
+
+#include "internal.h"
+#include "tc_common.cuh"
+#include "tile_sched.cuh"
+#include "tmap.h"
+
+namespace ftw {
+namespace {
+
+using namespace tc;
+
+enum { FWD = 0, BWDQ = 1, BWDKV = 2 };
+
+constexpr int BM = 128;
+constexpr int KB = 64;                    // keys per output block
+constexpr int CW = 128;                   // output columns per accumulation
+constexpr int NST = 2;                    // ring slots
+constexpr uint32_t SLOT = 80 * 1024;      // fp32 score slice (128 + 192 rows x 64 cols) / 64 x 128 block
+constexpr uint32_t STG = 32 * 128;        // one epilogue warp's 32-row x 32-col fp32 staging box
+constexpr int NSTG = 2;                   // staging boxes per epilogue warp
+constexpr int NTHREADS = 384;
+constexpr int NCONV = 2;                  // converter warps
+constexpr int RES_PER_LAUNCH = 8;
+static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
+constexpr uint32_t R0 = 0, R1 = 192, RACC = 384;
+constexpr float LOG2E = 1.4426950408889634f;
+constexpr float LN2 = 0.6931471805599453f;
+
+// a1/b1, a2/b2: score-GEMM operands (box rows BM / NK); ob1/ob2: output-GEMM B operands (box
+// rows KB); o1/o2: outputs (box rows 32).  All fp32, 32-column SWIZZLE_128B boxes.
+struct Maps {
+    CUtensorMap a1, b1, a2, b2, ob1, ob2, o1, o2;
+};
+struct Params {
+    Maps maps[RES_PER_LAUNCH];
+    float* lse;   // FWD: written; BWD: read
+    float* D;     // BWDQ: written; BWDKV: read
+    int64_t L;
+    int d, w, dil, NK, nsl;
+    SchedParams sc;
+    int dpoll;    // BWDKV: poll D row by row (BWDQ marked its rows D_UNSET, PDL launch)
+};
+
+constexpr size_t SCRATCH = 3 * 128 * 4 + 2 * 192 * 4;   // FWD row 1/l [3][128]; BWDKV column lse / D
+constexpr size_t SMEM_BYTES = 1024 + NST * SLOT + 4 * NSTG * STG + SCRATCH + 256;
+static_assert(SMEM_BYTES <= 227 * 1024, "shared memory plan");
+
+using Tile = SchedTile;
+using TileCursor = SchedCursor<BM>;
+
+__device__ __forceinline__ float fast_exp2(float x) {
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+// x -> (bf16(x), bf16(x - bf16(x))) for two values, packed as bf16x2 words
+__device__ __forceinline__ void split2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(x0, x1);
+    const float2 hf = __bfloat1622float2(h);
+    hi = *reinterpret_cast<uint32_t*>(&h);
+    lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
+}
+__device__ __forceinline__ bool band_ok(int n, int t, int w, int mcol, int Lr) {
+    return (unsigned)(n - t) <= (unsigned)(2 * w) && mcol >= 0 && mcol < Lr;
+}
+
+// The R rows of an fp32 box pair (box0 at p, box1 at p + R * 128; 128-byte rows, SWIZZLE_128B)
+// -> in place, the bf16 hi row over box0 and the lo row over box1.  Four threads per row, 16 fp32
+// columns each; the row's four threads are in one warp (reads complete before __syncwarp, writes
+// after).  ct: converter thread 0 .. 32 NCONV - 1.
+__device__ __forceinline__ void convert_pair(uint8_t* p, int R, int ct) {
+    const int q = ct & 3;                        // 16-column quarter of the 64-column row
+    uint8_t* src = p + (q >> 1) * R * 128;       // box holding fp32 columns 16q .. 16q + 15
+    for (int r0 = 0; r0 < R; r0 += 8 * NCONV) {
+        const int r = r0 + (ct >> 2);
+        uint4 v[4];
+        if (r < R) {
+#pragma unroll
+            for (int x = 0; x < 4; ++x) {
+                const int g = 4 * (q & 1) + x;   // logical 16-byte granule (fp32 cols 4g .. 4g + 3)
+                v[x] = *reinterpret_cast<const uint4*>(src + r * 128 + ((g ^ (r & 7)) << 4));
+            }
+        }
+        __syncwarp();
+        if (r < R) {
+            uint32_t hi[8], lo[8];
+#pragma unroll
+            for (int x = 0; x < 4; ++x) {
+                split2(__uint_as_float(v[x].x), __uint_as_float(v[x].y), hi[2 * x], lo[2 * x]);
+                split2(__uint_as_float(v[x].z), __uint_as_float(v[x].w), hi[2 * x + 1], lo[2 * x + 1]);
+            }
+            // bf16 columns 16q .. 16q + 15 = logical granules 2q, 2q + 1 of the plane rows
+#pragma unroll
+            for (int y = 0; y < 2; ++y) {
+                const int G = 2 * q + y;
+                const uint32_t off = r * 128 + ((G ^ (r & 7)) << 4);
+                *reinterpret_cast<uint4*>(p + off) = make_uint4(hi[4 * y], hi[4 * y + 1], hi[4 * y + 2], hi[4 * y + 3]);
+                *reinterpret_cast<uint4*>(p + R * 128 + off) =
+                    make_uint4(lo[4 * y], lo[4 * y + 1], lo[4 * y + 2], lo[4 * y + 3]);
+            }
+        }
+        __syncwarp();
+    }
+}
+
+// The slot sequence every role walks in the same order.  FWD: G(0), then per tile j: G(j+1),
+// O(j).  BWD: per tile: G(j), O(j).  G = nsl score slices (BWD: two slots per slice, S then dP);
+// O = nacc accumulations x nkb key blocks.
+template <int MODE>
+struct Seq {
+    static constexpr int NA = MODE == FWD ? 1 : 2;
+    static constexpr int NOUT = MODE == BWDKV ? 2 : 1;
+};
+
+template <int MODE>
+__global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_constant__ Params p) {
+    using C = Seq<MODE>;
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t raw_u32 = smem_u32(smem_raw);
+    uint8_t* smem = smem_raw + (((raw_u32 + 1023u) & ~1023u) - raw_u32);
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    const int NK = p.NK, nsl = p.nsl, w = p.w, d = p.d;
+    const int nkb = NK / KB, nch = NK / 32;
+    const int ncw = d / CW;                 // output chunks per tensor
+    const int nacc = ncw * C::NOUT;         // accumulations per tile
+
+    if (MODE == BWDQ && p.dpoll) {   // mark this CTA's D rows unset before BWDKV may launch
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T)) {
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+            for (int i = threadIdx.x; i < BM && T.m0 + i < T.Lr; i += NTHREADS)
+                reinterpret_cast<uint32_t*>(p.D)[rowbase + (int64_t)(T.m0 + i) * p.dil] = D_UNSET;
+        }
+        __threadfence();
+        __syncthreads();
+    }
+    if (MODE == BWDQ) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+
+    uint8_t* slots = smem;
+    uint8_t* stg = smem + NST * SLOT;                                   // [4 warps][NSTG] fp32 boxes
+    float* scratch = reinterpret_cast<float*>(stg + 4 * NSTG * STG);
+    float* rowScale = scratch;                                          // FWD [3][128]
+    float* colLse = scratch + 3 * 128;                                  // BWDKV [192] lse * log2e
+    float* colD = colLse + 192;                                         // BWDKV [192]
+    uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(scratch) + SCRATCH);
+    uint64_t* full = bars;             // [NST] TMA bytes landed
+    uint64_t* conv = bars + NST;       // [NST] planes written (4 converter warps)
+    uint64_t* empty = bars + 2 * NST;  // [NST] MMAs done with the slot
+    uint64_t* s_full = bars + 3 * NST; // [2] score GEMMs of a tile done (FWD: region j & 1)
+    uint64_t* p_full = s_full + 2;     // [2] softmax wrote the MMA operands of a tile (4 warps)
+    uint64_t* o_full = s_full + 4;     // accumulation done
+    uint64_t* o_empty = s_full + 5;    // accumulator drained (4 epilogue warps)
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 6);
+
+    if (warp == 8) {
+        if (lane == 0) {
+            for (int i = 0; i < NST; ++i) {
+                mbar_init(&full[i], 1);
+                mbar_init(&conv[i], NCONV);
+                mbar_init(&empty[i], 1);
+            }
+            for (int i = 0; i < 2; ++i) {
+                mbar_init(&s_full[i], 1);
+                mbar_init(&p_full[i], 4);
+            }
+            mbar_init(o_full, 1);
+            mbar_init(o_empty, 4);
+            fence_barrier_init();
+            for (int i = 0; i < p.sc.nr; ++i) {
+                const Maps& mp = p.maps[i];
+                tma_prefetch(&mp.a1); tma_prefetch(&mp.b1); tma_prefetch(&mp.ob1); tma_prefetch(&mp.o1);
+                if (C::NA == 2) { tma_prefetch(&mp.a2); tma_prefetch(&mp.b2); }
+                if (C::NOUT == 2) { tma_prefetch(&mp.ob2); tma_prefetch(&mp.o2); }
+            }
+        }
+        __syncwarp();
+        tmem_alloc(tmem_holder, 512);
+        tmem_relinquish();
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tbase = *tmem_holder;
+
+    // ------------------------------------------------------------------ shared slot walker
+    // fn(kind, T, a, b): kind 0 = score slot (slice a, operand pair b = 0 S / 1 dP), 1 = output
+    // block (accumulation a, key block b).  Called in slot order.
+    auto walk = [&](auto&& fn) {
+        TileCursor cg(p.sc), co(p.sc);
+        Tile Tg, To;
+        bool hg = cg.next(p.sc, Tg);
+        if (MODE == FWD) {
+            if (hg) {
+                for (int s = 0; s < nsl; ++s) fn(0, Tg, s, 0);
+                hg = cg.next(p.sc, Tg);
+            }
+            while (co.next(p.sc, To)) {
+                if (hg) {
+                    for (int s = 0; s < nsl; ++s) fn(0, Tg, s, 0);
+                    hg = cg.next(p.sc, Tg);
+                }
+                for (int a = 0; a < nacc; ++a)
+                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
+            }
+        } else {
+            while (co.next(p.sc, To)) {
+                for (int s = 0; s < nsl; ++s) {
+                    fn(0, To, s, 0);
+                    fn(0, To, s, 1);
+                }
+                for (int a = 0; a < nacc; ++a)
+                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
+            }
+        }
+    };
+
+    if (warp == 8) {
+        if (lane == 0) {   // -------------------------------------------------- TMA producer
+            int st = 0;
+            uint32_t ph = 0;
+            walk([&](int kind, const Tile& T, int a, int b) {
+                mbar_wait(&empty[st], ph ^ 1u);
+                uint8_t* sp = slots + (size_t)st * SLOT;
+                const Maps& mp = p.maps[T.rl];
+                if (kind == 0) {
+                    const CUtensorMap* ma = b ? &mp.a2 : &mp.a1;
+                    const CUtensorMap* mb = b ? &mp.b2 : &mp.b1;
+                    mbar_arrive_expect_tx(&full[st], (uint32_t)(2 * BM + 2 * NK) * 128u);
+                    for (int h = 0; h < 2; ++h) {
+                        tma_load_3d(sp + h * BM * 128, ma, &full[st], 64 * a + 32 * h, T.m0, T.u);
+                        tma_load_3d(sp + 2 * BM * 128 + h * NK * 128, mb, &full[st], 64 * a + 32 * h, T.m0 - w, T.u);
+                    }
+                } else {
+                    const int c = C::NOUT == 2 ? a % ncw : a;
+                    const CUtensorMap* m = (C::NOUT == 2 && a >= ncw) ? &mp.ob2 : &mp.ob1;
+                    mbar_arrive_expect_tx(&full[st], 4u * KB * 128u);
+                    for (int x = 0; x < 4; ++x)
+                        tma_load_3d(sp + x * KB * 128, m, &full[st], CW * c + 32 * x, T.m0 - w + KB * b, T.u);
+                }
+                if (++st == NST) { st = 0; ph ^= 1u; }
+            });
+        }
+    } else if (warp >= 10) {   // ------------------------------------------------- converters
+        const int ct = threadIdx.x - 320;   // 0 .. 32 NCONV - 1
+        int st = 0;
+        uint32_t ph = 0;
+        walk([&](int kind, const Tile&, int, int) {
+            mbar_wait(&full[st], ph);
+            uint8_t* sp = slots + (size_t)st * SLOT;
+            if (kind == 0) {
+                convert_pair(sp, BM, ct);
+                convert_pair(sp + 2 * BM * 128, NK, ct);
+            } else {
+                convert_pair(sp, KB, ct);
+                convert_pair(sp + 2 * KB * 128, KB, ct);
+            }
+            fence_proxy_async_smem();
+            warp_arrive(&conv[st]);
+            if (++st == NST) { st = 0; ph ^= 1u; }
+        });
+    } else if (warp == 9) {
+        if (lane == 0) {   // ------------------------------------------------------ MMA issuer
+            const uint32_t idS = idesc_bf16(BM, NK, false, false);
+            const uint32_t idO = idesc_bf16(BM, CW, false, true);
+            int st = 0, ga = 0;
+            uint32_t ph = 0;
+            int jg = 0;          // score GEMMs: tile counter
+            int jo = 0;          // output GEMMs: tile counter
+            walk([&](int kind, const Tile&, int a, int b) {
+                const uint32_t sa = smem_u32(slots + (size_t)st * SLOT);
+                if (kind == 0) {
+                    // FWD: S(jg) into region jg & 1; BWD: S into R0, dP into R1
+                    const uint32_t dst = tbase + (MODE == FWD ? ((jg & 1) ? R1 : R0) : (b ? R1 : R0));
+                    if (MODE != FWD && a == 0 && b == 0 && jg > 0) {
+                        // R1 (dP) is free once the softmax of the previous tile read it (p_full);
+                        // R0 (dS) once the previous tile's output MMAs read it (issue order)
+                        mbar_wait(&p_full[(jg - 1) & 1], ((jg - 1) >> 1) & 1);
+                        tc_fence_after();
+                    }
+                    mbar_wait(&conv[st], ph);
+                    tc_fence_after();
+                    const uint32_t ahi = sa, alo = sa + BM * 128, bhi = sa + 2 * BM * 128, blo = bhi + NK * 128;
+#pragma unroll
+                    for (int kk = 0; kk < 4; ++kk) {
+                        const uint64_t dah = sdesc_sw128(ahi + kk * 32, 16, 1024), dal = sdesc_sw128(alo + kk * 32, 16, 1024);
+                        const uint64_t dbh = sdesc_sw128(bhi + kk * 32, 16, 1024), dbl = sdesc_sw128(blo + kk * 32, 16, 1024);
+                        mma_ss(dst, dah, dbh, idS, (a | kk) != 0);
+                        mma_ss(dst, dah, dbl, idS, 1);
+                        mma_ss(dst, dal, dbh, idS, 1);
+                    }
+                    mma_commit(&empty[st]);
+                    if (a == nsl - 1 && b == C::NA - 1) {
+                        mma_commit(&s_full[MODE == FWD ? (jg & 1) : 0]);
+                        ++jg;
+                    }
+                } else {
+                    // output block b of accumulation a of tile jo.  A: packed hi | lo operand in TMEM
+                    // (FWD: P over S(jo); BWDQ: dS over S; BWDKV: P^T over dP^T (dV), dS^T over S^T (dK))
+                    if (a == 0 && b == 0) {
+                        mbar_wait(&p_full[jo & 1], (jo >> 1) & 1);
+                        tc_fence_after();
+                    }
+                    if (b == 0 && ga > 0) {
+                        mbar_wait(o_empty, (ga - 1) & 1);
+                        tc_fence_after();
+                    }
+                    const uint32_t Areg = tbase + (MODE == FWD ? ((jo & 1) ? R1 : R0)
+                                                   : (MODE == BWDKV && a < ncw) ? R1 : R0);
+                    mbar_wait(&conv[st], ph);
+                    tc_fence_after();
+#pragma unroll
+                    for (int kk = 0; kk < 4; ++kk) {
+                        const int g = 4 * b + kk;   // 16-key step over the halo
+                        const uint32_t tA = Areg + 32u * (g >> 1) + 8u * (g & 1);
+                        const uint64_t dbh = sdesc_sw128(sa + kk * 2048, 2 * KB * 128, 1024);
+                        const uint64_t dbl = sdesc_sw128(sa + KB * 128 + kk * 2048, 2 * KB * 128, 1024);
+                        mma_ts(tbase + RACC, tA, dbh, idO, g != 0);
+                        mma_ts(tbase + RACC, tA, dbl, idO, 1);
+                        mma_ts(tbase + RACC, tA + 16, dbh, idO, 1);
+                    }
+                    mma_commit(&empty[st]);
+                    if (b == nkb - 1) {
+                        mma_commit(o_full);
+                        ++ga;
+                        if (a == nacc - 1) ++jo;
+                    }
+                }
+                if (++st == NST) { st = 0; ph ^= 1u; }
+            });
+        }
+    } else if (warp < 4) {   // ------------------------------------------------ softmax warps
+        const int t = warp * 32 + lane;
+        const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+        // chunks holding any band column of this warp's rows: [32 warp, 32 warp + 31 + 2w]
+        const int c_lo = warp, c_hi = min(nch - 1, (32 * warp + 31 + 2 * w) / 32);
+        uint32_t zero16[16];
+#pragma unroll
+        for (int e = 0; e < 16; ++e) zero16[e] = 0u;
+        TileCursor cur(p.sc);
+        Tile T;
+        int j = 0;
+        if (MODE == BWDKV && !p.dpoll) asm volatile("griddepcontrol.wait;" ::: "memory");
+        while (cur.next(p.sc, T)) {
+            const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t, kb = m0 - w;
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+            if (MODE == BWDKV) {
+                named_bar_sync(1, 128);   // everyone is done with the previous tile's columns
+                for (int n = t; n < NK; n += 128) {
+                    const int mc = kb + n;
+                    const bool ok = mc >= 0 && mc < Lr;
+                    colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
+                    float dv = 0.f;
+                    if (ok) dv = p.dpoll ? ld_D_ready(p.D + rowbase + (int64_t)mc * p.dil) : p.D[rowbase + (int64_t)mc * p.dil];
+                    colD[n] = dv;
+                }
+                named_bar_sync(1, 128);
+            }
+            const int sidx = MODE == FWD ? (j & 1) : 0;
+            const uint32_t sph = MODE == FWD ? ((j >> 1) & 1) : (j & 1);
+            mbar_wait(&s_full[sidx], sph);
+            tc_fence_after();
+            const uint32_t rS = tbase + lane_off + (MODE == FWD && (j & 1) ? R1 : R0);
+            const uint32_t rP = tbase + lane_off + R1;
+            if (MODE == FWD) {
+                float mx = -INFINITY;
+                for (int c = c_lo; c <= c_hi; ++c) {
+                    uint32_t rr[32];
+                    tmem_ld32(rS + c * 32, rr);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int e = 0; e < 32; ++e)
+                        if (band_ok(c * 32 + e, t, w, kb + c * 32 + e, Lr)) mx = fmaxf(mx, __uint_as_float(rr[e]));
+                }
+                if (mx == -INFINITY) mx = 0.f;   // rows beyond the sequence (never stored)
+                const float mxs = mx * LOG2E;
+                float sum = 0.f;
+                for (int c = 0; c < nch; ++c) {
+                    if (c < c_lo || c > c_hi) {
+                        tmem_st16(rS + c * 32, zero16);
+                        tmem_st16(rS + c * 32 + 16, zero16);
+                        continue;
+                    }
+                    uint32_t rr[32], pk[16], pl[16];
+                    tmem_ld32(rS + c * 32, rr);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int e = 0; e < 32; e += 2) {
+                        float pv[2];
+#pragma unroll
+                        for (int h = 0; h < 2; ++h) {
+                            const int n = c * 32 + e + h;
+                            pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rr[e + h]), LOG2E, -mxs)) : 0.f;
+                            sum += pv[h];
+                        }
+                        split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
+                    }
+                    tmem_st16(rS + c * 32, pk);
+                    tmem_st16(rS + c * 32 + 16, pl);
+                }
+                rowScale[(j % 3) * 128 + t] = 1.f / sum;
+                tmem_wait_st();
+                tc_fence_before();
+                warp_arrive(&p_full[j & 1]);
+                if (mrow < Lr) p.lse[rowbase + (int64_t)mrow * p.dil] = (mxs + log2f(sum)) * LN2;
+            } else if (MODE == BWDQ) {
+                const float lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
+                float D = 0.f;
+                for (int c = c_lo; c <= c_hi; ++c) {   // pass 1: D = sum_j P_ij dP_ij
+                    uint32_t rs[32], rd[32];
+                    tmem_ld32(rS + c * 32, rs);
+                    tmem_ld32(rP + c * 32, rd);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int e = 0; e < 32; ++e) {
+                        const int n = c * 32 + e;
+                        const float pv = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f;
+                        D = fmaf(pv, __uint_as_float(rd[e]), D);
+                    }
+                }
+                for (int c = 0; c < nch; ++c) {   // pass 2: dS = P (dP - D) -> hi | lo over S
+                    if (c < c_lo || c > c_hi) {
+                        tmem_st16(rS + c * 32, zero16);
+                        tmem_st16(rS + c * 32 + 16, zero16);
+                        continue;
+                    }
+                    uint32_t rs[32], rd[32], pk[16], pl[16];
+                    tmem_ld32(rS + c * 32, rs);
+                    tmem_ld32(rP + c * 32, rd);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int e = 0; e < 32; e += 2) {
+                        float dv[2];
+#pragma unroll
+                        for (int h = 0; h < 2; ++h) {
+                            const int n = c * 32 + e + h;
+                            const float pv = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -lse2)) : 0.f;
+                            dv[h] = pv * (__uint_as_float(rd[e + h]) - D);
+                        }
+                        split2(dv[0], dv[1], pk[e / 2], pl[e / 2]);
+                    }
+                    tmem_st16(rS + c * 32, pk);
+                    tmem_st16(rS + c * 32 + 16, pl);
+                }
+                tmem_wait_st();
+                tc_fence_before();
+                warp_arrive(&p_full[j & 1]);
+                if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
+            } else {   // BWDKV: rows are keys, columns halo queries
+                for (int c = 0; c < nch; ++c) {
+                    if (c < c_lo || c > c_hi) {
+                        tmem_st16(rS + c * 32, zero16);
+                        tmem_st16(rS + c * 32 + 16, zero16);
+                        tmem_st16(rP + c * 32, zero16);
+                        tmem_st16(rP + c * 32 + 16, zero16);
+                        continue;
+                    }
+                    uint32_t rs[32], rd[32], pk[16], pl[16], dk[16], dl[16];
+                    tmem_ld32(rS + c * 32, rs);
+                    tmem_ld32(rP + c * 32, rd);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int e = 0; e < 32; e += 2) {
+                        float pv[2], dv[2];
+#pragma unroll
+                        for (int h = 0; h < 2; ++h) {
+                            const int n = c * 32 + e + h;
+                            pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -colLse[n])) : 0.f;
+                            dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
+                        }
+                        split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
+                        split2(dv[0], dv[1], dk[e / 2], dl[e / 2]);
+                    }
+                    tmem_st16(rS + c * 32, dk);
+                    tmem_st16(rS + c * 32 + 16, dl);
+                    tmem_st16(rP + c * 32, pk);
+                    tmem_st16(rP + c * 32 + 16, pl);
+                }
+                tmem_wait_st();
+                tc_fence_before();
+                warp_arrive(&p_full[j & 1]);
+            }
+            ++j;
+        }
+    } else if (warp < 8) {   // ----------------------------------------------- epilogue warps
+        const int ew = warp - 4;   // TMEM lanes 32 ew ..
+        const uint32_t trow = tbase + ((uint32_t)(ew * 32) << 16) + RACC;
+        uint8_t* mystg = stg + ew * NSTG * STG;
+        TileCursor cur(p.sc);
+        Tile T;
+        int j = 0, ga = 0, sidx = 0;
+        while (cur.next(p.sc, T)) {
+            const Maps& mp = p.maps[T.rl];
+            float scale = 1.f;
+            if (MODE == FWD) {   // 1/l of this row, published before p_full
+                mbar_wait(&p_full[j & 1], (j >> 1) & 1);
+                scale = rowScale[(j % 3) * 128 + ew * 32 + lane];
+            }
+            for (int a = 0; a < nacc; ++a, ++ga) {
+                const int c = C::NOUT == 2 ? a % ncw : a;
+                const CUtensorMap* om = (C::NOUT == 2 && a < ncw) ? &mp.o2 : &mp.o1;   // BWDKV: dV first
+                mbar_wait(o_full, ga & 1);
+                tc_fence_after();
+                uint32_t ov[4][32];
+#pragma unroll
+                for (int x = 0; x < 4; ++x) tmem_ld32(trow + 32 * x, ov[x]);
+                tmem_wait_ld();
+                tc_fence_before();
+                warp_arrive(o_empty);
+#pragma unroll
+                for (int x = 0; x < 4; ++x) {
+                    uint8_t* sb = mystg + (sidx % NSTG) * STG;
+                    if (lane == 0 && sidx >= NSTG) tma_store_wait_read<NSTG - 1>();
+                    __syncwarp();
+#pragma unroll
+                    for (int g = 0; g < 8; ++g) {
+                        uint4 val;
+                        val.x = __float_as_uint(__uint_as_float(ov[x][4 * g + 0]) * scale);
+                        val.y = __float_as_uint(__uint_as_float(ov[x][4 * g + 1]) * scale);
+                        val.z = __float_as_uint(__uint_as_float(ov[x][4 * g + 2]) * scale);
+                        val.w = __float_as_uint(__uint_as_float(ov[x][4 * g + 3]) * scale);
+                        *reinterpret_cast<uint4*>(sb + lane * 128 + ((g ^ (lane & 7)) << 4)) = val;
+                    }
+                    fence_proxy_async_smem();
+                    __syncwarp();
+                    if (lane == 0) {
+                        tma_store_3d(om, sb, CW * c + 32 * x, T.m0 + 32 * ew, T.u);
+                        tma_store_commit();
+                    }
+                    ++sidx;
+                }
+            }
+            ++j;
+        }
+        if (lane == 0) tma_store_wait_all<0>();
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 8) {
+        tc_fence_after();
+        tmem_dealloc(tbase, 512);
+    }
+}
+
+int num_sms32() {
+    static int n = 0;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0)
+            n = 148;
+    });
+    return n;
+}
+
+int halo_rows32(int64_t L, int64_t w) {
+    const int64_t wc = w < L ? w : L;
+    return (int)(((BM + 2 * wc) + 63) / 64 * 64);
+}
+
+template <int MODE>
+cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void* b2, const void* ob1,
+                     const void* ob2, void* o1, void* o2, float* lse, float* D, int64_t B, int64_t H,
+                     int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaFuncSetAttribute(tc_band32_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES);
+    });
+    const int64_t wc = w < L ? w : L;
+    const int NK = halo_rows32(L, w);
+    const int64_t units = B * H;
+    const int64_t nres = dil < L ? dil : L;
+    int n = 0;
+    for (int64_t r0 = 0; r0 < nres; r0 += RES_PER_LAUNCH) {
+        Params p;
+        memset(&p, 0, sizeof(p));
+        const int nr = (int)(nres - r0 < RES_PER_LAUNCH ? nres - r0 : RES_PER_LAUNCH);
+        for (int i = 0; i < nr; ++i) {
+            const int64_t r = r0 + i;
+            Maps& m = p.maps[i];
+            bool ok = make_residue_map_f32(&m.a1, a1, L, d, units, dil, r, BM) &&
+                      make_residue_map_f32(&m.b1, b1, L, d, units, dil, r, NK) &&
+                      make_residue_map_f32(&m.ob1, ob1, L, d, units, dil, r, KB) &&
+                      make_residue_map_f32(&m.o1, o1, L, d, units, dil, r, 32);
+            if (ok && a2) ok = make_residue_map_f32(&m.a2, a2, L, d, units, dil, r, BM);
+            if (ok && b2) ok = make_residue_map_f32(&m.b2, b2, L, d, units, dil, r, NK);
+            if (ok && ob2) ok = make_residue_map_f32(&m.ob2, ob2, L, d, units, dil, r, KB);
+            if (ok && o2) ok = make_residue_map_f32(&m.o2, o2, L, d, units, dil, r, 32);
+            if (!ok) return cudaErrorInvalidValue;
+        }
+        p.lse = lse;
+        p.D = D;
+        p.L = L;
+        p.d = (int)d;
+        p.w = (int)wc;
+        p.dil = (int)dil;
+        p.NK = NK;
+        p.nsl = (int)(d / 64);
+        p.dpoll = MODE == BWDKV && dpoll_enabled();
+        const int64_t Lr0 = ceil_div(L - r0, dil);
+        const int tiles = (int)ceil_div(Lr0, BM);
+        const int64_t total = units * nr * tiles;
+        dim3 grid((unsigned)(total < num_sms32() ? total : num_sms32()));
+        sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
+        if (MODE == BWDKV && r0 == 0 && p.dpoll) {   // directly after this call's last BWDQ launch
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = grid;
+            cfg.blockDim = dim3(NTHREADS);
+            cfg.dynamicSmemBytes = SMEM_BYTES;
+            cfg.stream = st;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = at;
+            cfg.numAttrs = 1;
+            cudaLaunchKernelEx(&cfg, tc_band32_kernel<MODE>, p);
+        } else {
+            tc_band32_kernel<MODE><<<grid, NTHREADS, SMEM_BYTES, st>>>(p);
+        }
+        prof_mark(st);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        ++n;
+    }
+    if (launches) *launches += n;
+    return cudaSuccess;
+}
+
+int band32_launches(int64_t L, int64_t dil) {
+    const int64_t nres = dil < L ? dil : L;
+    return (int)ceil_div(nres, RES_PER_LAUNCH);
+}
+
+}  // namespace
+
+bool tc32_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    const int64_t wc = w < L ? w : L;
+    return d % 64 == 0 && d <= 512 && wc <= 32 && dil <= 256 && units * ((L + 127) / 128) < (1 << 30);
+}
+int tc32_fwd_launches(int64_t L, int64_t dil) { return band32_launches(L, dil); }
+int tc32_bwd_launches(int64_t L, int64_t dil) { return 2 * band32_launches(L, dil); }
+
+cudaError_t tc32_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B, int64_t H,
+                     int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
+    if (launches) *launches = 0;
+    return launch32<FWD>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, B, H, L, d, w, dil, st,
+                         launches);
+}
+
+cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const float* lse, const void* dout, void* dq,
+                     void* dk, void* dv, float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
+                     int64_t dil, cudaStream_t st, int* launches) {
+    if (launches) *launches = 0;
+    // BWDQ: S = Q K_h^T (a1 = q, b1 = k), dP = dO V_h^T (a2 = dout, b2 = v), dQ = dS K_h (ob1 = k)
+    cudaError_t e = launch32<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse), Dws, B, H, L,
+                                   d, w, dil, st, launches);
+    if (e != cudaSuccess) return e;
+    // BWDKV: S^T = K Q_h^T, dP^T = V dO_h^T; dV = P^T dO_h (ob1 = dout -> o2 = dv), dK = dS^T Q_h
+    // (ob2 = q -> o1 = dk).  Accumulations: dV chunks (a < ncw, o2), then dK chunks (o1).
+    return launch32<BWDKV>(k, q, v, dout, dout, q, dk, dv, const_cast<float*>(lse), Dws, B, H, L, d, w, dil, st,
+                           launches);
+}
+
+}  // namespace ftw

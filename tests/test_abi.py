@@ -158,8 +158,12 @@ def test_workspace_and_plan(lib):
     assert lib.ft_winattn_bwd_workspace_bytes(0, 3, 100, 64, 4, 1, 1) == 0
     path, n = ft.plan(False, 1, 8, 10000, 512, 32, 1, ft.FT_BF16)
     assert path == ft.PATH_TC and n == 1
-    path, n = ft.plan(False, 1, 8, 10000, 512, 32, 1, ft.FT_F32)
-    assert path == ft.PATH_SIMT and n >= 1
+    path, n = ft.plan(False, 1, 8, 10000, 512, 32, 1, ft.FT_F32)   # fp32 tensor-core kernels
+    assert path == ft.PATH_TC and n == 1
+    path, n = ft.plan(True, 1, 8, 10000, 512, 32, 1, ft.FT_F32)
+    assert path == ft.PATH_TC and n == 2
+    path, n = ft.plan(False, 1, 8, 4096, 64, 256, 1, ft.FT_F32)    # w > 32: CUDA cores
+    assert path == ft.PATH_SIMT
     path, n = ft.plan(True, 1, 1, 64, 16, 4, 1, ft.FT_F32)
     assert path == ft.PATH_SIMT and n >= 1
     with pytest.raises(ft.FtError):

@@ -136,6 +136,14 @@ def test_tc_bwd_parity(ft, shape):
     run_case(ft, WinAttnShape(*shape), "bf16", "tc", seed=3)
 
 
+# fp32 on the tensor cores (tc_band32.cu: bf16 hi / lo planes, three products per MMA step),
+# against the 1e-4 bound of the fp32 path
+@pytest.mark.parametrize("shape", [s for s in SMALL if s[3] % 64 == 0 and min(s[4], s[2]) <= 32],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_tc32_parity(ft, shape):
+    run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=16)
+
+
 @pytest.mark.parametrize("seed", [0, 1, 2])
 def test_default_path_seeds(ft, seed):
     run_case(ft, WinAttnShape(1, 2, 384, 64, 32, 1), "bf16", None, seed=seed)

@@ -32,7 +32,7 @@ __device__ __forceinline__ void mma_ts32(uint32_t d, uint32_t a, uint64_t b, uin
 
 __device__ __forceinline__ float lo_of(float x) { return x - __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
 
-__global__ void kern(const float* A, const float* B, float* D, int mode) {
+__global__ void kern(const float* A, const float* B, float* D, int mode, uint32_t lbo, uint32_t sbo) {
     extern __shared__ __align__(1024) uint8_t smem[];
     __shared__ uint32_t holder;
     __shared__ uint64_t bar;
@@ -87,9 +87,9 @@ __global__ void kern(const float* A, const float* B, float* D, int mode) {
     if (t == 32) {
         const uint32_t id = idesc_tf32(128, 64, false, bmn);
         for (int kk = 0; kk < 4; ++kk) {   // K = 8 per MMA
-            const uint64_t b = bmn ? sdesc_sw128(smem_u32(sB) + kk * 1024, 4096, 1024)
+            const uint64_t b = bmn ? sdesc_sw128(smem_u32(sB) + kk * 1024, lbo, sbo)
                                    : sdesc_sw128(smem_u32(sB) + kk * 32, 16, 1024);
-            const uint64_t bl = bmn ? sdesc_sw128(smem_u32(sBl) + kk * 1024, 4096, 1024)
+            const uint64_t bl = bmn ? sdesc_sw128(smem_u32(sBl) + kk * 1024, lbo, sbo)
                                     : sdesc_sw128(smem_u32(sBl) + kk * 32, 16, 1024);
             if (!ts) {
                 const uint64_t a = sdesc_sw128(smem_u32(sA) + kk * 32, 16, 1024);
@@ -137,9 +137,12 @@ int main() {
     for (int i = 0; i < N * K; ++i) hB[i] = (float)rnd();
     cudaMemcpy(dA, hA, sizeof(hA), cudaMemcpyHostToDevice);
     cudaMemcpy(dB, hB, sizeof(hB), cudaMemcpyHostToDevice);
-    for (int mode = 0; mode < 5; ++mode) {
+    const uint32_t LB[7] = {16, 16, 4096, 16, 4096, 1024, 4096};
+    const uint32_t SB[7] = {1024, 1024, 1024, 1024, 1024, 4096, 4096};
+    for (int m7 = 0; m7 < 7; ++m7) {
+        const int mode = m7 < 5 ? m7 : 2;
         cudaMemset(dD, 0, sizeof(hD));
-        kern<<<1, 128, 64 * 1024>>>(dA, dB, dD, mode);
+        kern<<<1, 128, 64 * 1024>>>(dA, dB, dD, mode, LB[m7], SB[m7]);
         cudaError_t e = cudaDeviceSynchronize();
         cudaMemcpy(hD, dD, sizeof(hD), cudaMemcpyDeviceToHost);
         double maxe = 0, maxr = 0;
@@ -150,8 +153,15 @@ int main() {
                 maxe = fmax(maxe, fabs(hD[m * N + n] - r));
                 maxr = fmax(maxr, fabs(r));
             }
-        printf("mode %d (%s): max abs err %.3e  (max |ref| %.3f, rel %.3e)\n", mode, cudaGetErrorString(e),
-               maxe, maxr, maxe / maxr);
+        double e32 = 0;   // columns 0..31 only (first MN group)
+        for (int m = 0; m < M; ++m)
+            for (int n = 0; n < 32; ++n) {
+                double r = 0;
+                for (int k = 0; k < K; ++k) r += (double)hA[m * K + k] * hB[n * K + k];
+                e32 = fmax(e32, fabs(hD[m * N + n] - r));
+            }
+        printf("mode %d lbo %u sbo %u (%s): max abs err %.3e (cols 0-31: %.3e) (max |ref| %.3f)  D[0][0..3] = %g %g %g %g\n",
+               mode, LB[m7], SB[m7], cudaGetErrorString(e), maxe, e32, maxr, hD[0], hD[1], hD[2], hD[3]);
         if (e != cudaSuccess) return 1;
     }
     return 0;
