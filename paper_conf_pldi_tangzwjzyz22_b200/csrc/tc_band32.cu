@@ -108,6 +108,7 @@ __device__ __forceinline__ void split2(float x0, float x1, uint32_t& hi, uint32_
     hi = *reinterpret_cast<uint32_t*>(&h);
     lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
 }
+__device__ __forceinline__ int chunk_w(int d, int c) { return d - CW * c < CW ? d - CW * c : CW; }
 __device__ __forceinline__ bool band_ok(int n, int t, int w, int mcol, int Lr) {
     return (unsigned)(n - t) <= (unsigned)(2 * w) && mcol >= 0 && mcol < Lr;
 }
@@ -169,7 +170,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int NK = p.NK, nsl = p.nsl, w = p.w, d = p.d;
     const int nkb = NK / KB, nch = NK / 32;
-    const int ncw = d / CW;                 // output chunks per tensor
+    const int ncw = (d + CW - 1) / CW;      // output chunks per tensor (the last may be 64 wide)
     const int nacc = ncw * C::NOUT;         // accumulations per tile
 
     if (MODE == BWDQ && p.dpoll) {   // mark this CTA's D rows unset before BWDKV may launch
@@ -281,9 +282,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     }
                 } else {
                     const int c = C::NOUT == 2 ? a % ncw : a;
+                    const int nbox = chunk_w(d, c) / 32;
                     const CUtensorMap* m = (C::NOUT == 2 && a >= ncw) ? &mp.ob2 : &mp.ob1;
-                    mbar_arrive_expect_tx(&full[st], 4u * KB * 128u);
-                    for (int x = 0; x < 4; ++x)
+                    mbar_arrive_expect_tx(&full[st], (uint32_t)nbox * KB * 128u);
+                    for (int x = 0; x < nbox; ++x)
                         tma_load_3d(sp + x * KB * 128, m, &full[st], CW * c + 32 * x, T.m0 - w + KB * b, T.u);
                 }
                 if (++st == NST) { st = 0; ph ^= 1u; }
@@ -293,7 +295,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         const int ct = threadIdx.x - 320;   // 0 .. 32 NCONV - 1
         int st = 0;
         uint32_t ph = 0;
-        walk([&](int kind, const Tile&, int, int) {
+        walk([&](int kind, const Tile&, int a, int) {
             mbar_wait(&full[st], ph);
             uint8_t* sp = slots + (size_t)st * SLOT;
             if (kind == 0) {
@@ -301,7 +303,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 convert_pair(sp + 2 * BM * 128, NK, ct);
             } else {
                 convert_pair(sp, KB, ct);
-                convert_pair(sp + 2 * KB * 128, KB, ct);
+                if (chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW) convert_pair(sp + 2 * KB * 128, KB, ct);
             }
             fence_proxy_async_smem();
             warp_arrive(&conv[st]);
@@ -311,6 +313,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         if (lane == 0) {   // ------------------------------------------------------ MMA issuer
             const uint32_t idS = idesc_bf16(BM, NK, false, false);
             const uint32_t idO = idesc_bf16(BM, CW, false, true);
+            const uint32_t idO64 = idesc_bf16(BM, 64, false, true);   // a 64-column last chunk
             int st = 0, ga = 0;
             uint32_t ph = 0;
             int jg = 0;          // score GEMMs: tile counter
@@ -355,6 +358,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     }
                     const uint32_t Areg = tbase + (MODE == FWD ? ((jo & 1) ? R1 : R0)
                                                    : (MODE == BWDKV && a < ncw) ? R1 : R0);
+                    const uint32_t id = chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW ? idO : idO64;
                     mbar_wait(&conv[st], ph);
                     tc_fence_after();
 #pragma unroll
@@ -363,9 +367,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         const uint32_t tA = Areg + 32u * (g >> 1) + 8u * (g & 1);
                         const uint64_t dbh = sdesc_sw128(sa + kk * 2048, 2 * KB * 128, 1024);
                         const uint64_t dbl = sdesc_sw128(sa + KB * 128 + kk * 2048, 2 * KB * 128, 1024);
-                        mma_ts(tbase + RACC, tA, dbh, idO, g != 0);
-                        mma_ts(tbase + RACC, tA, dbl, idO, 1);
-                        mma_ts(tbase + RACC, tA + 16, dbh, idO, 1);
+                        mma_ts(tbase + RACC, tA, dbh, id, g != 0);
+                        mma_ts(tbase + RACC, tA, dbl, id, 1);
+                        mma_ts(tbase + RACC, tA + 16, dbh, id, 1);
                     }
                     mma_commit(&empty[st]);
                     if (b == nkb - 1) {
@@ -547,16 +551,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             for (int a = 0; a < nacc; ++a, ++ga) {
                 const int c = C::NOUT == 2 ? a % ncw : a;
                 const CUtensorMap* om = (C::NOUT == 2 && a < ncw) ? &mp.o2 : &mp.o1;   // BWDKV: dV first
+                const int ngrp = chunk_w(d, c) / 32;
                 mbar_wait(o_full, ga & 1);
                 tc_fence_after();
                 uint32_t ov[4][32];
 #pragma unroll
-                for (int x = 0; x < 4; ++x) tmem_ld32(trow + 32 * x, ov[x]);
+                for (int x = 0; x < 4; ++x)
+                    if (x < ngrp) tmem_ld32(trow + 32 * x, ov[x]);
                 tmem_wait_ld();
                 tc_fence_before();
                 warp_arrive(o_empty);
 #pragma unroll
                 for (int x = 0; x < 4; ++x) {
+                    if (x >= ngrp) break;
                     uint8_t* sb = mystg + (sidx % NSTG) * STG;
                     if (lane == 0 && sidx >= NSTG) tma_store_wait_read<NSTG - 1>();
                     __syncwarp();
@@ -645,7 +652,7 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         p.dil = (int)dil;
         p.NK = NK;
         p.nsl = (int)(d / 64);
-        p.dpoll = MODE == BWDKV && dpoll_enabled();
+        p.dpoll = MODE != FWD && dpoll_enabled();   // BWDQ marks its D rows, BWDKV polls them
         const int64_t Lr0 = ceil_div(L - r0, dil);
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
