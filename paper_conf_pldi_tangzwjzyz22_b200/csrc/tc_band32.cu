@@ -12,13 +12,14 @@
 // MN-major tf32 B operands are not executed), i.e. transposed copies of V, K, dO, Q for the
 // output products; the bf16 planes keep the MN-major B operands of tc_band.cu.
 //
-// Data movement.  TMA loads fp32 boxes of 32 columns (128-byte rows, SWIZZLE_128B) into a ring
-// slot; two converter warps then rewrite each row IN PLACE as its two bf16 planes: the 64 fp32
-// values of a row held by the box pair (cols 0-31 | cols 32-63, at the same row offset of two
-// boxes) become the 64-column hi row (over the first box) and lo row (over the second), which
-// are exactly the K-major SWIZZLE_128B bf16 layouts the MMAs read (score GEMMs), or, for the
-// 64-key x 128-column output blocks, the MN-major bf16 boxes (LBO 16 KB between the two 64-column
-// groups).  So a slot holds fp32 and its planes in the same 80 KB, and the HBM bytes are those of
+// Data movement.  TMA loads fp32 box pairs into a ring slot; two converter warps then rewrite
+// each row IN PLACE as its two bf16 planes: the fp32 values of a row held by the box pair (the
+// same row offset of two boxes) become the bf16 hi row (over the first box) and lo row (over the
+// second), which are exactly the layouts the MMAs read.  Score slices: 32 columns as two 16-column
+// boxes (64-byte rows, SWIZZLE_64B) -> K-major SWIZZLE_64B planes, 40 KB per slot (128 + 192 rows),
+// so the 160 KB ring holds four slices in flight; output blocks: 64 keys x 128 columns as four
+// 32-column boxes (SWIZZLE_128B) -> MN-major bf16 boxes (LBO 16 KB between the two 64-column
+// groups).  A slot holds fp32 and its planes in the same bytes, and the HBM bytes are those of
 // the fp32 tensors: 4de + 4 per row forward, 5de + 8 / 6de + 8 per row for the two backward
 // kernels (the same kernel split as tc_band.cu).
 //
@@ -35,9 +36,11 @@
 //         dP^T = V dO_h^T; P^T (hi|lo over dP^T), dS^T (hi|lo over S^T); dV_c = P^T dO_h,c,
 //         dK_c = dS^T Q_h,c.
 //
-// Roles (384 threads): warps 0-3 softmax (thread t <-> row m0 + t <-> TMEM lane t), 4-7
+// Roles (512 threads): warps 0-3 softmax (thread t <-> row m0 + t <-> TMEM lane t), 4-7
 // epilogue (TMEM -> fp32 -> smem -> TMA store), 8 TMA producer + TMEM allocator, 9 MMA issuer,
-// 10-11 converters (12 warps keep the register cap at 168 per thread).  TMEM: R0 = [0, 192),
+// 10-15 converters (the conversion is latency bound per warp: 2 warps converted a 40 KB slot in
+// ~4 kclk, tools/trace32.py; the softmax and epilogue work in 16-column pieces to stay within
+// the 128 registers per thread of 16 warps).  TMEM: R0 = [0, 192),
 // R1 = [192, 384), the output accumulator [384, 512).
 #include <cuda.h>
 #include <cuda_bf16.h>
@@ -62,12 +65,12 @@ enum { FWD = 0, BWDQ = 1, BWDKV = 2 };
 constexpr int BM = 128;
 constexpr int KB = 64;                    // keys per output block
 constexpr int CW = 128;                   // output columns per accumulation
-constexpr int NST = 2;                    // ring slots
-constexpr uint32_t SLOT = 80 * 1024;      // fp32 score slice (128 + 192 rows x 64 cols) / 64 x 128 block
+constexpr int NST = 4;                    // ring slots
+constexpr uint32_t SLOT = 40 * 1024;      // fp32 score slice (128 + 192 rows x 32 cols) / 64 x 128 block
 constexpr uint32_t STG = 32 * 128;        // one epilogue warp's 32-row x 32-col fp32 staging box
 constexpr int NSTG = 2;                   // staging boxes per epilogue warp
-constexpr int NTHREADS = 384;
-constexpr int NCONV = 2;                  // converter warps
+constexpr int NTHREADS = 512;
+constexpr int NCONV = 6;                  // converter warps
 constexpr int RES_PER_LAUNCH = 8;
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t R0 = 0, R1 = 192, RACC = 384;
@@ -87,7 +90,20 @@ struct Params {
     int d, w, dil, NK, nsl;
     SchedParams sc;
     int dpoll;    // BWDKV: poll D row by row (BWDQ marked its rows D_UNSET, PDL launch)
+    unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace), see trace32()
 };
+
+// Phase trace (profiling only): per CTA, clock64 stamps of its first TR_SLOTS slots --
+// [0] producer issued the TMA, [1] converter started, [2] converter done, [3] MMA issue start,
+// [4] MMA issue end -- and of its first TR_TILES tiles at [TR_SLOTS * 5 + tile * 8 + e]:
+// 0 softmax s_full seen, 1 softmax p_full arrived, 2.. epilogue o_full seen per accumulation.
+constexpr int TR_SLOTS = 96, TR_TILES = 4, TR_PER_CTA = TR_SLOTS * 5 + TR_TILES * 8;
+__device__ __forceinline__ void trace_slot(const Params& p, int k, int e) {
+    if (p.trace && k < TR_SLOTS) p.trace[(size_t)blockIdx.x * TR_PER_CTA + k * 5 + e] = clock64();
+}
+__device__ __forceinline__ void trace_tile(const Params& p, int j, int e) {
+    if (p.trace && j < TR_TILES && e < 8) p.trace[(size_t)blockIdx.x * TR_PER_CTA + TR_SLOTS * 5 + j * 8 + e] = clock64();
+}
 
 constexpr size_t SCRATCH = 3 * 128 * 4 + 2 * 192 * 4;   // FWD row 1/l [3][128]; BWDKV column lse / D
 constexpr size_t SMEM_BYTES = 1024 + NST * SLOT + 4 * NSTG * STG + SCRATCH + 256;
@@ -103,53 +119,78 @@ __device__ __forceinline__ float fast_exp2(float x) {
 }
 // x -> (bf16(x), bf16(x - bf16(x))) for two values, packed as bf16x2 words
 __device__ __forceinline__ void split2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
-    __nv_bfloat162 h = __floats2bfloat162_rn(x0, x1);
-    const float2 hf = __bfloat1622float2(h);
-    hi = *reinterpret_cast<uint32_t*>(&h);
-    lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
+    hi = pack_bf16x2(x0, x1);   // RN; x0 in the low half
+    lo = pack_bf16x2(x0 - __uint_as_float(hi << 16), x1 - __uint_as_float(hi & 0xFFFF0000u));
 }
 __device__ __forceinline__ int chunk_w(int d, int c) { return d - CW * c < CW ? d - CW * c : CW; }
 __device__ __forceinline__ bool band_ok(int n, int t, int w, int mcol, int Lr) {
     return (unsigned)(n - t) <= (unsigned)(2 * w) && mcol >= 0 && mcol < Lr;
 }
 
-// The R rows of an fp32 box pair (box0 at p, box1 at p + R * 128; 128-byte rows, SWIZZLE_128B)
-// -> in place, the bf16 hi row over box0 and the lo row over box1.  Four threads per row, 16 fp32
-// columns each; the row's four threads are in one warp (reads complete before __syncwarp, writes
-// after).  ct: converter thread 0 .. 32 NCONV - 1.
-__device__ __forceinline__ void convert_pair(uint8_t* p, int R, int ct) {
-    const int q = ct & 3;                        // 16-column quarter of the 64-column row
-    uint8_t* src = p + (q >> 1) * R * 128;       // box holding fp32 columns 16q .. 16q + 15
-    for (int r0 = 0; r0 < R; r0 += 8 * NCONV) {
-        const int r = r0 + (ct >> 2);
-        uint4 v[4];
-        if (r < R) {
+// In-place fp32 -> bf16 hi / lo planes for the R rows of a box pair: box0 at p, box1 at p + R * RB,
+// RB-byte rows (RB = 128: 32 fp32 per box row, SWIZZLE_128B, 16-byte granule g of row r at
+// (g ^ (r & 7)) * 16; RB = 64: 16 fp32, SWIZZLE_64B, granule g at (g ^ ((r >> 1) & 3)) * 16).
+// The 2 * RB / 4 fp32 of row r (box0 columns first) become the bf16 hi row over box0 and the lo row
+// over box1 -- the K-major (score slices) or MN-major (output blocks) bf16 operand rows.  Four
+// threads per row (one warp holds whole rows): thread q reads fp32 columns [q, q + 1) * RB / 8 and
+// writes bf16 granule(s) of the same columns in both planes, after a __syncwarp separating every
+// read of the row from every write.  UNR row passes per iteration keep 2 UNR RB / 64 loads in
+// flight per thread (one pass per iteration was load-latency bound: ~4.2 kclk per 40 KB score
+// slot, tools/trace32.py).  ct: converter thread 0 .. 32 NCONV - 1.
+template <int RB>
+__device__ __forceinline__ int swz(int g, int r) { return RB == 128 ? (g ^ (r & 7)) : (g ^ ((r >> 1) & 3)); }
+
+template <int RB, int UNR>
+__device__ __forceinline__ void convert_rows(uint8_t* p, int R, int ct) {
+    constexpr int NG = RB / 32;                  // 16-byte fp32 granules read per thread per row
+    const int q = ct & 3;
+    uint8_t* src = p + (q >> 1) * R * RB;        // box holding this thread's fp32 columns
+    constexpr int PASS = 8 * NCONV;              // rows per pass
+    for (int r0 = 0; r0 < R; r0 += UNR * PASS) {
+        uint4 v[UNR][NG];
 #pragma unroll
-            for (int x = 0; x < 4; ++x) {
-                const int g = 4 * (q & 1) + x;   // logical 16-byte granule (fp32 cols 4g .. 4g + 3)
-                v[x] = *reinterpret_cast<const uint4*>(src + r * 128 + ((g ^ (r & 7)) << 4));
+        for (int u = 0; u < UNR; ++u) {
+            const int r = r0 + u * PASS + (ct >> 2);
+            if (r < R) {
+#pragma unroll
+                for (int x = 0; x < NG; ++x)
+                    v[u][x] = *reinterpret_cast<const uint4*>(src + r * RB + (swz<RB>(NG * (q & 1) + x, r) << 4));
             }
         }
         __syncwarp();
-        if (r < R) {
-            uint32_t hi[8], lo[8];
 #pragma unroll
-            for (int x = 0; x < 4; ++x) {
-                split2(__uint_as_float(v[x].x), __uint_as_float(v[x].y), hi[2 * x], lo[2 * x]);
-                split2(__uint_as_float(v[x].z), __uint_as_float(v[x].w), hi[2 * x + 1], lo[2 * x + 1]);
-            }
-            // bf16 columns 16q .. 16q + 15 = logical granules 2q, 2q + 1 of the plane rows
+        for (int u = 0; u < UNR; ++u) {
+            const int r = r0 + u * PASS + (ct >> 2);
+            if (r < R) {
+                uint32_t hi[2 * NG], lo[2 * NG];
 #pragma unroll
-            for (int y = 0; y < 2; ++y) {
-                const int G = 2 * q + y;
-                const uint32_t off = r * 128 + ((G ^ (r & 7)) << 4);
-                *reinterpret_cast<uint4*>(p + off) = make_uint4(hi[4 * y], hi[4 * y + 1], hi[4 * y + 2], hi[4 * y + 3]);
-                *reinterpret_cast<uint4*>(p + R * 128 + off) =
-                    make_uint4(lo[4 * y], lo[4 * y + 1], lo[4 * y + 2], lo[4 * y + 3]);
+                for (int x = 0; x < NG; ++x) {
+                    split2(__uint_as_float(v[u][x].x), __uint_as_float(v[u][x].y), hi[2 * x], lo[2 * x]);
+                    split2(__uint_as_float(v[u][x].z), __uint_as_float(v[u][x].w), hi[2 * x + 1], lo[2 * x + 1]);
+                }
+                // bf16 columns of this thread: granules NG / 2 * q .. of the plane rows
+#pragma unroll
+                for (int y = 0; y < NG / 2; ++y) {
+                    const uint32_t off = r * RB + (swz<RB>((NG / 2) * q + y, r) << 4);
+                    *reinterpret_cast<uint4*>(p + off) = make_uint4(hi[4 * y], hi[4 * y + 1], hi[4 * y + 2], hi[4 * y + 3]);
+                    *reinterpret_cast<uint4*>(p + R * RB + off) =
+                        make_uint4(lo[4 * y], lo[4 * y + 1], lo[4 * y + 2], lo[4 * y + 3]);
+                }
             }
         }
         __syncwarp();
     }
+}
+
+// K-major SWIZZLE_64B smem descriptor (64-byte rows; SBO = 8 rows x 64 B)
+__device__ __forceinline__ uint64_t sdesc_sw64(uint32_t saddr) {
+    uint64_t desc = 0;
+    desc |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+    desc |= (uint64_t)1 << 16;
+    desc |= (uint64_t)(512u >> 4) << 32;
+    desc |= (uint64_t)1 << 46;   // version (sm_100)
+    desc |= (uint64_t)4 << 61;   // SWIZZLE_64B
+    return desc;
 }
 
 // The slot sequence every role walks in the same order.  FWD: G(0), then per tile j: G(j+1),
@@ -266,19 +307,20 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
 
     if (warp == 8) {
         if (lane == 0) {   // -------------------------------------------------- TMA producer
-            int st = 0;
+            int st = 0, k = 0;
             uint32_t ph = 0;
             walk([&](int kind, const Tile& T, int a, int b) {
                 mbar_wait(&empty[st], ph ^ 1u);
+                trace_slot(p, k++, 0);
                 uint8_t* sp = slots + (size_t)st * SLOT;
                 const Maps& mp = p.maps[T.rl];
-                if (kind == 0) {
+                if (kind == 0) {   // 32 columns: two 16-column boxes of each operand
                     const CUtensorMap* ma = b ? &mp.a2 : &mp.a1;
                     const CUtensorMap* mb = b ? &mp.b2 : &mp.b1;
-                    mbar_arrive_expect_tx(&full[st], (uint32_t)(2 * BM + 2 * NK) * 128u);
+                    mbar_arrive_expect_tx(&full[st], (uint32_t)(2 * BM + 2 * NK) * 64u);
                     for (int h = 0; h < 2; ++h) {
-                        tma_load_3d(sp + h * BM * 128, ma, &full[st], 64 * a + 32 * h, T.m0, T.u);
-                        tma_load_3d(sp + 2 * BM * 128 + h * NK * 128, mb, &full[st], 64 * a + 32 * h, T.m0 - w, T.u);
+                        tma_load_3d(sp + h * BM * 64, ma, &full[st], 32 * a + 16 * h, T.m0, T.u);
+                        tma_load_3d(sp + 2 * BM * 64 + h * NK * 64, mb, &full[st], 32 * a + 16 * h, T.m0 - w, T.u);
                     }
                 } else {
                     const int c = C::NOUT == 2 ? a % ncw : a;
@@ -293,20 +335,23 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         }
     } else if (warp >= 10) {   // ------------------------------------------------- converters
         const int ct = threadIdx.x - 320;   // 0 .. 32 NCONV - 1
-        int st = 0;
+        int st = 0, k = 0;
         uint32_t ph = 0;
         walk([&](int kind, const Tile&, int a, int) {
             mbar_wait(&full[st], ph);
+            if (ct == 0) trace_slot(p, k, 1);
             uint8_t* sp = slots + (size_t)st * SLOT;
             if (kind == 0) {
-                convert_pair(sp, BM, ct);
-                convert_pair(sp + 2 * BM * 128, NK, ct);
+                convert_rows<64, 1>(sp, BM, ct);
+                convert_rows<64, 1>(sp + 2 * BM * 64, NK, ct);
             } else {
-                convert_pair(sp, KB, ct);
-                if (chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW) convert_pair(sp + 2 * KB * 128, KB, ct);
+                convert_rows<128, 1>(sp, KB, ct);
+                if (chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW) convert_rows<128, 1>(sp + 2 * KB * 128, KB, ct);
             }
             fence_proxy_async_smem();
             warp_arrive(&conv[st]);
+            if (ct == 0) trace_slot(p, k, 2);
+            ++k;
             if (++st == NST) { st = 0; ph ^= 1u; }
         });
     } else if (warp == 9) {
@@ -314,7 +359,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             const uint32_t idS = idesc_bf16(BM, NK, false, false);
             const uint32_t idO = idesc_bf16(BM, CW, false, true);
             const uint32_t idO64 = idesc_bf16(BM, 64, false, true);   // a 64-column last chunk
-            int st = 0, ga = 0;
+            int st = 0, ga = 0, k = 0;
             uint32_t ph = 0;
             int jg = 0;          // score GEMMs: tile counter
             int jo = 0;          // output GEMMs: tile counter
@@ -331,11 +376,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     }
                     mbar_wait(&conv[st], ph);
                     tc_fence_after();
-                    const uint32_t ahi = sa, alo = sa + BM * 128, bhi = sa + 2 * BM * 128, blo = bhi + NK * 128;
+                    trace_slot(p, k, 3);
+                    const uint32_t ahi = sa, alo = sa + BM * 64, bhi = sa + 2 * BM * 64, blo = bhi + NK * 64;
 #pragma unroll
-                    for (int kk = 0; kk < 4; ++kk) {
-                        const uint64_t dah = sdesc_sw128(ahi + kk * 32, 16, 1024), dal = sdesc_sw128(alo + kk * 32, 16, 1024);
-                        const uint64_t dbh = sdesc_sw128(bhi + kk * 32, 16, 1024), dbl = sdesc_sw128(blo + kk * 32, 16, 1024);
+                    for (int kk = 0; kk < 2; ++kk) {
+                        const uint64_t dah = sdesc_sw64(ahi + kk * 32), dal = sdesc_sw64(alo + kk * 32);
+                        const uint64_t dbh = sdesc_sw64(bhi + kk * 32), dbl = sdesc_sw64(blo + kk * 32);
                         mma_ss(dst, dah, dbh, idS, (a | kk) != 0);
                         mma_ss(dst, dah, dbl, idS, 1);
                         mma_ss(dst, dal, dbh, idS, 1);
@@ -361,15 +407,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     const uint32_t id = chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW ? idO : idO64;
                     mbar_wait(&conv[st], ph);
                     tc_fence_after();
+                    trace_slot(p, k, 3);
 #pragma unroll
                     for (int kk = 0; kk < 4; ++kk) {
                         const int g = 4 * b + kk;   // 16-key step over the halo
-                        const uint32_t tA = Areg + 32u * (g >> 1) + 8u * (g & 1);
+                        const uint32_t tA = Areg + 16u * g;   // hi words; lo words at + 8
                         const uint64_t dbh = sdesc_sw128(sa + kk * 2048, 2 * KB * 128, 1024);
                         const uint64_t dbl = sdesc_sw128(sa + KB * 128 + kk * 2048, 2 * KB * 128, 1024);
                         mma_ts(tbase + RACC, tA, dbh, id, g != 0);
                         mma_ts(tbase + RACC, tA, dbl, id, 1);
-                        mma_ts(tbase + RACC, tA + 16, dbh, id, 1);
+                        mma_ts(tbase + RACC, tA + 8, dbh, id, 1);
                     }
                     mma_commit(&empty[st]);
                     if (b == nkb - 1) {
@@ -378,6 +425,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         if (a == nacc - 1) ++jo;
                     }
                 }
+                trace_slot(p, k++, 4);
                 if (++st == NST) { st = 0; ph ^= 1u; }
             });
         }
@@ -412,8 +460,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             const uint32_t sph = MODE == FWD ? ((j >> 1) & 1) : (j & 1);
             mbar_wait(&s_full[sidx], sph);
             tc_fence_after();
+            if (t == 0) trace_tile(p, j, 0);
             const uint32_t rS = tbase + lane_off + (MODE == FWD && (j & 1) ? R1 : R0);
             const uint32_t rP = tbase + lane_off + R1;
+            // The bf16 operand of 16 keys (K-step g = key / 16) is packed in place over those keys'
+            // 16 fp32 columns: hi words at columns [16 g, 16 g + 8), lo words at [16 g + 8, 16 g + 16).
             if (MODE == FWD) {
                 float mx = -INFINITY;
                 for (int c = c_lo; c <= c_hi; ++c) {
@@ -433,41 +484,50 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tmem_st16(rS + c * 32 + 16, zero16);
                         continue;
                     }
-                    uint32_t rr[32], pk[16], pl[16];
-                    tmem_ld32(rS + c * 32, rr);
-                    tmem_wait_ld();
 #pragma unroll
-                    for (int e = 0; e < 32; e += 2) {
-                        float pv[2];
+                    for (int hh = 0; hh < 2; ++hh) {
+                        const int n0 = c * 32 + 16 * hh;
+                        uint32_t rr[16], pk[8], pl[8];
+                        tmem_ld16(rS + n0, rr);
+                        tmem_wait_ld();
 #pragma unroll
-                        for (int h = 0; h < 2; ++h) {
-                            const int n = c * 32 + e + h;
-                            pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rr[e + h]), LOG2E, -mxs)) : 0.f;
-                            sum += pv[h];
+                        for (int e = 0; e < 16; e += 2) {
+                            float pv[2];
+#pragma unroll
+                            for (int h = 0; h < 2; ++h) {
+                                const int n = n0 + e + h;
+                                pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rr[e + h]), LOG2E, -mxs)) : 0.f;
+                                sum += pv[h];
+                            }
+                            split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
                         }
-                        split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
+                        tmem_st8(rS + n0, pk);
+                        tmem_st8(rS + n0 + 8, pl);
                     }
-                    tmem_st16(rS + c * 32, pk);
-                    tmem_st16(rS + c * 32 + 16, pl);
                 }
                 rowScale[(j % 3) * 128 + t] = 1.f / sum;
                 tmem_wait_st();
                 tc_fence_before();
                 warp_arrive(&p_full[j & 1]);
+                if (t == 0) trace_tile(p, j, 1);
                 if (mrow < Lr) p.lse[rowbase + (int64_t)mrow * p.dil] = (mxs + log2f(sum)) * LN2;
             } else if (MODE == BWDQ) {
                 const float lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
                 float D = 0.f;
                 for (int c = c_lo; c <= c_hi; ++c) {   // pass 1: D = sum_j P_ij dP_ij
-                    uint32_t rs[32], rd[32];
-                    tmem_ld32(rS + c * 32, rs);
-                    tmem_ld32(rP + c * 32, rd);
-                    tmem_wait_ld();
 #pragma unroll
-                    for (int e = 0; e < 32; ++e) {
-                        const int n = c * 32 + e;
-                        const float pv = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f;
-                        D = fmaf(pv, __uint_as_float(rd[e]), D);
+                    for (int hh = 0; hh < 2; ++hh) {
+                        const int n0 = c * 32 + 16 * hh;
+                        uint32_t rs[16], rd[16];
+                        tmem_ld16(rS + n0, rs);
+                        tmem_ld16(rP + n0, rd);
+                        tmem_wait_ld();
+#pragma unroll
+                        for (int e = 0; e < 16; ++e) {
+                            const int n = n0 + e;
+                            const float pv = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f;
+                            D = fmaf(pv, __uint_as_float(rd[e]), D);
+                        }
                     }
                 }
                 for (int c = 0; c < nch; ++c) {   // pass 2: dS = P (dP - D) -> hi | lo over S
@@ -476,23 +536,27 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tmem_st16(rS + c * 32 + 16, zero16);
                         continue;
                     }
-                    uint32_t rs[32], rd[32], pk[16], pl[16];
-                    tmem_ld32(rS + c * 32, rs);
-                    tmem_ld32(rP + c * 32, rd);
-                    tmem_wait_ld();
 #pragma unroll
-                    for (int e = 0; e < 32; e += 2) {
-                        float dv[2];
+                    for (int hh = 0; hh < 2; ++hh) {
+                        const int n0 = c * 32 + 16 * hh;
+                        uint32_t rs[16], rd[16], pk[8], pl[8];
+                        tmem_ld16(rS + n0, rs);
+                        tmem_ld16(rP + n0, rd);
+                        tmem_wait_ld();
 #pragma unroll
-                        for (int h = 0; h < 2; ++h) {
-                            const int n = c * 32 + e + h;
-                            const float pv = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -lse2)) : 0.f;
-                            dv[h] = pv * (__uint_as_float(rd[e + h]) - D);
+                        for (int e = 0; e < 16; e += 2) {
+                            float dv[2];
+#pragma unroll
+                            for (int h = 0; h < 2; ++h) {
+                                const int n = n0 + e + h;
+                                const float pv = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -lse2)) : 0.f;
+                                dv[h] = pv * (__uint_as_float(rd[e + h]) - D);
+                            }
+                            split2(dv[0], dv[1], pk[e / 2], pl[e / 2]);
                         }
-                        split2(dv[0], dv[1], pk[e / 2], pl[e / 2]);
+                        tmem_st8(rS + n0, pk);
+                        tmem_st8(rS + n0 + 8, pl);
                     }
-                    tmem_st16(rS + c * 32, pk);
-                    tmem_st16(rS + c * 32 + 16, pl);
                 }
                 tmem_wait_st();
                 tc_fence_before();
@@ -507,26 +571,30 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tmem_st16(rP + c * 32 + 16, zero16);
                         continue;
                     }
-                    uint32_t rs[32], rd[32], pk[16], pl[16], dk[16], dl[16];
-                    tmem_ld32(rS + c * 32, rs);
-                    tmem_ld32(rP + c * 32, rd);
-                    tmem_wait_ld();
 #pragma unroll
-                    for (int e = 0; e < 32; e += 2) {
-                        float pv[2], dv[2];
+                    for (int hh = 0; hh < 2; ++hh) {
+                        const int n0 = c * 32 + 16 * hh;
+                        uint32_t rs[16], rd[16], pk[8], pl[8], dk[8], dl[8];
+                        tmem_ld16(rS + n0, rs);
+                        tmem_ld16(rP + n0, rd);
+                        tmem_wait_ld();
 #pragma unroll
-                        for (int h = 0; h < 2; ++h) {
-                            const int n = c * 32 + e + h;
-                            pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -colLse[n])) : 0.f;
-                            dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
+                        for (int e = 0; e < 16; e += 2) {
+                            float pv[2], dv[2];
+#pragma unroll
+                            for (int h = 0; h < 2; ++h) {
+                                const int n = n0 + e + h;
+                                pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -colLse[n])) : 0.f;
+                                dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
+                            }
+                            split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
+                            split2(dv[0], dv[1], dk[e / 2], dl[e / 2]);
                         }
-                        split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
-                        split2(dv[0], dv[1], dk[e / 2], dl[e / 2]);
+                        tmem_st8(rS + n0, dk);          // dS^T over S^T
+                        tmem_st8(rS + n0 + 8, dl);
+                        tmem_st8(rP + n0, pk);          // P^T over dP^T
+                        tmem_st8(rP + n0 + 8, pl);
                     }
-                    tmem_st16(rS + c * 32, dk);
-                    tmem_st16(rS + c * 32 + 16, dl);
-                    tmem_st16(rP + c * 32, pk);
-                    tmem_st16(rP + c * 32 + 16, pl);
                 }
                 tmem_wait_st();
                 tc_fence_before();
@@ -554,26 +622,29 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 const int ngrp = chunk_w(d, c) / 32;
                 mbar_wait(o_full, ga & 1);
                 tc_fence_after();
-                uint32_t ov[4][32];
-#pragma unroll
-                for (int x = 0; x < 4; ++x)
-                    if (x < ngrp) tmem_ld32(trow + 32 * x, ov[x]);
-                tmem_wait_ld();
-                tc_fence_before();
-                warp_arrive(o_empty);
+                if (ew == 0 && lane == 0) trace_tile(p, j, 2 + a);
+                // two rounds of 64 columns (register budget of 16 warps); the accumulator is
+                // released once the last columns are in registers
 #pragma unroll
                 for (int x = 0; x < 4; ++x) {
                     if (x >= ngrp) break;
+                    uint32_t ov[1][32];
+                    tmem_ld32(trow + 32 * x, ov[0]);
+                    tmem_wait_ld();
+                    if (x == ngrp - 1) {
+                        tc_fence_before();
+                        warp_arrive(o_empty);
+                    }
                     uint8_t* sb = mystg + (sidx % NSTG) * STG;
                     if (lane == 0 && sidx >= NSTG) tma_store_wait_read<NSTG - 1>();
                     __syncwarp();
 #pragma unroll
                     for (int g = 0; g < 8; ++g) {
                         uint4 val;
-                        val.x = __float_as_uint(__uint_as_float(ov[x][4 * g + 0]) * scale);
-                        val.y = __float_as_uint(__uint_as_float(ov[x][4 * g + 1]) * scale);
-                        val.z = __float_as_uint(__uint_as_float(ov[x][4 * g + 2]) * scale);
-                        val.w = __float_as_uint(__uint_as_float(ov[x][4 * g + 3]) * scale);
+                        val.x = __float_as_uint(__uint_as_float(ov[0][4 * g + 0]) * scale);
+                        val.y = __float_as_uint(__uint_as_float(ov[0][4 * g + 1]) * scale);
+                        val.z = __float_as_uint(__uint_as_float(ov[0][4 * g + 2]) * scale);
+                        val.w = __float_as_uint(__uint_as_float(ov[0][4 * g + 3]) * scale);
                         *reinterpret_cast<uint4*>(sb + lane * 128 + ((g ^ (lane & 7)) << 4)) = val;
                     }
                     fence_proxy_async_smem();
@@ -634,12 +705,12 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         for (int i = 0; i < nr; ++i) {
             const int64_t r = r0 + i;
             Maps& m = p.maps[i];
-            bool ok = make_residue_map_f32(&m.a1, a1, L, d, units, dil, r, BM) &&
-                      make_residue_map_f32(&m.b1, b1, L, d, units, dil, r, NK) &&
+            bool ok = make_residue_map_f32(&m.a1, a1, L, d, units, dil, r, BM, 16) &&
+                      make_residue_map_f32(&m.b1, b1, L, d, units, dil, r, NK, 16) &&
                       make_residue_map_f32(&m.ob1, ob1, L, d, units, dil, r, KB) &&
                       make_residue_map_f32(&m.o1, o1, L, d, units, dil, r, 32);
-            if (ok && a2) ok = make_residue_map_f32(&m.a2, a2, L, d, units, dil, r, BM);
-            if (ok && b2) ok = make_residue_map_f32(&m.b2, b2, L, d, units, dil, r, NK);
+            if (ok && a2) ok = make_residue_map_f32(&m.a2, a2, L, d, units, dil, r, BM, 16);
+            if (ok && b2) ok = make_residue_map_f32(&m.b2, b2, L, d, units, dil, r, NK, 16);
             if (ok && ob2) ok = make_residue_map_f32(&m.ob2, ob2, L, d, units, dil, r, KB);
             if (ok && o2) ok = make_residue_map_f32(&m.o2, o2, L, d, units, dil, r, 32);
             if (!ok) return cudaErrorInvalidValue;
@@ -651,8 +722,9 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         p.w = (int)wc;
         p.dil = (int)dil;
         p.NK = NK;
-        p.nsl = (int)(d / 64);
+        p.nsl = (int)(d / 32);
         p.dpoll = MODE != FWD && dpoll_enabled();   // BWDQ marks its D rows, BWDKV polls them
+        p.trace = (unsigned long long*)trace_buffer(MODE);
         const int64_t Lr0 = ceil_div(L - r0, dil);
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;

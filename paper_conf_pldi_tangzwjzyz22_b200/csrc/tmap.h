@@ -48,20 +48,22 @@ inline bool make_residue_map(CUtensorMap* m, const void* tensor, int64_t L, int6
     return res == CUDA_SUCCESS;
 }
 
-// fp32 residue view with a {32 x box_rows} SWIZZLE_128B box (128-byte rows), for tc_band32.cu.
+// fp32 residue view with a {box_cols x box_rows} box, for tc_band32.cu: 32 columns (128-byte rows,
+// SWIZZLE_128B) or 16 columns (64-byte rows, SWIZZLE_64B).
 inline bool make_residue_map_f32(CUtensorMap* m, const void* tensor, int64_t L, int64_t d,
-                                 int64_t units, int64_t dil, int64_t r, int box_rows) {
+                                 int64_t units, int64_t dil, int64_t r, int box_rows, int box_cols = 32) {
     auto enc = tmap_encoder();
     if (!enc) return false;
     const int64_t Lr = (L - r + dil - 1) / dil;
     const char* base = static_cast<const char*>(tensor) + r * d * 4;
     cuuint64_t dims[3] = {(cuuint64_t)d, (cuuint64_t)Lr, (cuuint64_t)units};
     cuuint64_t strides[2] = {(cuuint64_t)(dil * d * 4), (cuuint64_t)(L * d * 4)};
-    cuuint32_t box[3] = {32u, (cuuint32_t)box_rows, 1u};
+    cuuint32_t box[3] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows, 1u};
     cuuint32_t estr[3] = {1u, 1u, 1u};
     CUresult res = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<char*>(base), dims,
                        strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                       CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                       box_cols == 16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return res == CUDA_SUCCESS;
 }
