@@ -1,19 +1,23 @@
 #!/usr/bin/env python
 """bench.py -- fwd+bwd banded window-attention throughput on B200 (one JSON line).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2a] [--dtype bf16]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2a] [--dtype f32|bf16]
     python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N
     python bench.py --impl reference ...      # the fp64 CPU oracle as the reference arm
 
 A step is one pass of the whole hot path (SURVEY.md §8(a) F0-F6 + B0-B5): ft_winattn_fwd
 then ft_winattn_bwd over one batch of synthetic inputs resident in HBM.  Default workload
 is BASELINE.json configs[2] "same shape forward+backward" at reading A14(a) of the
-paper's Longformer shape: B=1, H=8, L=10000, d=512, w=32 (C2a), bf16.
+paper's Longformer shape: B=1, H=8, L=10000, d=512, w=32 (C2a), in fp32 -- the paper's
+precision ("f32"), computed on the tensor cores as bf16 hi / lo planes
+within the north_star's 1e-4 bound (csrc/tc_band32.cu).  --dtype bf16 measures bf16 storage.
 
 Multi-GPU: (batch, head) units are independent, so the job is sharded
 with NO collective on the data path: every rank runs its own batch element (weak scaling,
 global_batch = N), timed between a barrier + synchronize on both sides, and the elapsed
-time is the max over ranks.
+time is the max over ranks.  The "strong_scaling" record splits the fixed --strong-workload
+(64 heads of 32K tokens by default) into per-rank head slabs; "e2e_nccl_scatter_gather" adds
+the NCCL scatter of the inputs and gather of the outputs from rank 0.
 
 Keys beyond the base contract: "roofline" (dominant kernel, CUDA events on the launching
 stream via the ft_winattn_profile_events hook, recorded in a second pass of the same steps:
@@ -21,7 +25,8 @@ an event between two launches would stop the BWDQ -> BWDKV programmatic dependen
 overlap inside the timed region), "hbm_step" (whole step vs SURVEY.md §8(d)
 algorithmic bytes), "cpu_baseline" (the fp64 oracle on a bounded sample, rank 0, N=1),
 "e2e" (pinned host buffers, H2D + fwd + bwd + D2H inside the timed region), "clocks"
-(NVML samples during the timed region) and "gpu_launches".
+(NVML samples during the timed region), "gpu_launches", and the sub-records "bf16" / "f32"
+(the other storage dtype), "fwd_bwd_call" (the one-call API) and "strong_scaling".
 """
 from __future__ import annotations
 
@@ -292,6 +297,46 @@ def scatter_gather_e2e(args, rank, world, dev, tdt, e, shape):
             "what": "rank 0 scatters q/k/v/dout (NCCL), per-rank fwd+bwd, gathers out/lse/dq/dk/dv"}
 
 
+def quick_time(ft, torch, dev, shape, dtype, steps, warmup, hd=None, api="separate", units=None):
+    """ms per fwd+bwd step of `shape` (B, H, L, d, w, dil) on this rank: inputs generated on the
+    device, L2 flushed between steps when they fit in it, CUDA events around the K steps.
+    api: "separate" = ft_winattn_fwd + ft_winattn_bwd, "fwd_bwd" = the one-call ft_winattn_fwd_bwd.
+    units: heads of this rank's slab (strong scaling), default H."""
+    B, H, L, d, w, dil = shape
+    H = H if units is None else units
+    tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
+    e = 2 if dtype == "bf16" else 4
+    gen = torch.Generator(device=dev)
+    gen.manual_seed(4321)
+    q, k, v, g = ((torch.rand((B, H, L, d), device=dev, generator=gen) * 2 - 1).to(tdt) for _ in range(4))
+    out, dq, dk, dv = (torch.empty_like(q) for _ in range(4))
+    lse = torch.empty((B, H, L), device=dev, dtype=torch.float32)
+    ws = torch.empty(max(ft.workspace_bytes(q, w, dil), 16), device=dev, dtype=torch.uint8)
+    flush = torch.empty(2 * L2_BYTES, device=dev, dtype=torch.uint8) if 4 * q.numel() * e <= L2_BYTES else None
+
+    def step():
+        if api == "fwd_bwd":
+            ft.fwd_bwd(q, k, v, g, w, dil, out=out, lse=lse, dq=dq, dk=dk, dv=dv, workspace=ws)
+        else:
+            ft.fwd(q, k, v, w, dil, out=out, lse=lse, dilated_heads=hd)
+            ft.bwd(q, k, v, out, lse, g, w, dil, dq=dq, dk=dk, dv=dv, workspace=ws, dilated_heads=hd)
+
+    for _ in range(warmup):
+        step()
+    torch.cuda.synchronize()
+    tot = 0.0
+    for _ in range(steps):
+        if flush is not None:
+            flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        step()
+        b.record()
+        b.synchronize()
+        tot += a.elapsed_time(b)
+    return tot / steps
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -299,7 +344,12 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="C2a", choices=sorted(WORKLOADS))
-    ap.add_argument("--dtype", default="bf16", choices=["bf16", "f32"])
+    ap.add_argument("--dtype", default="f32", choices=["bf16", "f32"],
+                    help="f32: the paper's precision (PAPER.md:147, 217), the headline; bf16: faster storage")
+    ap.add_argument("--strong-workload", default="C5_w32",
+                    help="fixed-work (batch, head)-sharded strong-scaling record (configs[4] corner)")
+    ap.add_argument("--extra-steps", type=int, default=50, help="steps of each sub-record")
+    ap.add_argument("--no-extras", action="store_true", help="skip the sub-records")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work (cpu_baseline)")
     ap.add_argument("--ref-rows", type=int, default=0, help="oracle rows per reference step (0 = full L)")
@@ -451,7 +501,7 @@ def main():
     mean_k = {n: sum(x) / len(x) for n, x in kdur.items()}
     dom = max(mean_k, key=mean_k.get)
     rows_per_launch = krows[dom]
-    if args.dtype == "bf16":
+    if path_b == ft.PATH_TC:   # tensor-core kernels (bf16, or fp32 as bf16 hi / lo planes): HBM bound
         by = kernel_bytes_per_row(kinds[dom], d, e) * rows_per_launch
         ach = by / (mean_k[dom] / 1e3) / 1e9
         roof = {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
@@ -488,15 +538,20 @@ def main():
     flops = 12.0 * d * nsum
     exps = 2.0 * nsum
     sm_mhz = sm_max
-    comp_peak = bf16_peak * 1e12 if args.dtype == "bf16" else 148 * 128 * 2 * sm_mhz * 1e6
+    # the tensor ceiling: bf16 products at the measured bf16 peak; the fp32 tensor-core path issues
+    # three bf16 products (hi.hi + hi.lo + lo.hi) per fp32 product; the CUDA-core path: FMA
+    tc_path = path_b == ft.PATH_TC
+    comp_peak = bf16_peak * 1e12 if tc_path else 148 * 128 * 2 * sm_mhz * 1e6
+    comp_work = flops * (3.0 if (tc_path and args.dtype == "f32") else 1.0)
     mufu_peak = 148 * 16 * sm_mhz * 1e6
-    bounds = {"hbm": step_alg / world / (hbm_peak * 1e9), "tensor" if args.dtype == "bf16" else "fma": flops / comp_peak,
+    bounds = {"hbm": step_alg / world / (hbm_peak * 1e9), "tensor" if tc_path else "fma": comp_work / comp_peak,
               "mufu": exps / mufu_peak}
     ceilings = {k: {"lower_bound_us": v * 1e6, "frac": v / step_s} for k, v in bounds.items()}
     ceilings["binding"] = max(bounds, key=bounds.get)
     ceilings["peaks"] = {"hbm_gbs": hbm_peak, "compute_tflops": comp_peak / 1e12, "mufu_gops": mufu_peak / 1e9,
                          "note": "HBM and bf16 measured (MEASURED_PEAKS.json); FMA and MUFU derived from "
-                                 "148 SMs x 128 lanes x 2 / 16 ex2 per clock at sm_max_mhz"}
+                                 "148 SMs x 128 lanes x 2 / 16 ex2 per clock at sm_max_mhz; fp32 on the "
+                                 "tensor cores counts 3 bf16 products per fp32 product"}
     ceilings["step_ms"] = {"mean": elapsed_ms / args.steps, "min": min(step_ms),
                            "median": sorted(step_ms)[len(step_ms) // 2]}
 
@@ -572,6 +627,59 @@ def main():
         except Exception as ex:   # the main line must survive; report why this extra is missing
             sg = {"error": f"{type(ex).__name__}: {ex}"[:300]}
 
+    # ---------------------------------------------------------------- sub-records
+    # (a) the other storage dtype on the same workload; (b) the one-call ft_winattn_fwd_bwd (the
+    # forward -> dQ-kernel lse hand-off); (c) fixed-work strong scaling: the --strong-workload's
+    # (batch, head) units split into contiguous slabs over the N ranks (rank r
+    # owns [r U / N, (r + 1) U / N)), compute only, max over ranks; the NCCL scatter / gather
+    # variant of the same job is e2e_nccl_scatter_gather.
+    extras = {}
+    if not args.no_extras and args.extra_steps > 0:
+        other = "bf16" if args.dtype == "f32" else "f32"
+        o_ms = quick_time(ft, torch, dev, shape, other, args.extra_steps, 3, hd=hd)
+        oe = 2 if other == "bf16" else 4
+        o_ms_t = torch.tensor([o_ms], dtype=torch.float64, device="cpu" if one_gpu else dev)
+        if world > 1:
+            dist.all_reduce(o_ms_t, op=dist.ReduceOp.MAX)
+        o_ms = float(o_ms_t.item())
+        extras[other] = {"ms_per_step": o_ms, "tokens_per_s": B * L * world / (o_ms / 1e3),
+                         "hbm_frac": step_bytes_per_row(d, oe) * rows / (o_ms / 1e3) / 1e9 / hbm_peak,
+                         "paths": dict(zip(("fwd", "bwd"), ("tc" if ft.plan(b_, B, H, L, d, w, dil,
+                                                                      ft.FT_BF16 if other == "bf16" else ft.FT_F32)[0]
+                                                   == ft.PATH_TC else "simt" for b_ in (False, True))))}
+        if hd is None:
+            fb_ms = quick_time(ft, torch, dev, shape, args.dtype, args.extra_steps, 3, api="fwd_bwd")
+            fb_t = torch.tensor([fb_ms], dtype=torch.float64, device="cpu" if one_gpu else dev)
+            if world > 1:
+                dist.all_reduce(fb_t, op=dist.ReduceOp.MAX)
+            fb_ms = float(fb_t.item())
+            extras["fwd_bwd_call"] = {"ms_per_step": fb_ms, "tokens_per_s": B * L * world / (fb_ms / 1e3),
+                                      "what": "ft_winattn_fwd_bwd: one call, the dQ kernel reads lse rows as "
+                                              "the forward stores them"}
+        sw = WORKLOADS[args.strong_workload]
+        sB, sH, sL, sd, sw_, sdil = sw[:6]
+        U = sB * sH
+        u0, u1 = (rank * U) // world, ((rank + 1) * U) // world
+        if sB == 1 and u1 > u0:
+            s_ms = quick_time(ft, torch, dev, (1, sH, sL, sd, sw_, sdil), args.dtype, args.extra_steps, 3,
+                              units=u1 - u0)
+        else:
+            s_ms = 0.0
+        s_t = torch.tensor([s_ms], dtype=torch.float64, device="cpu" if one_gpu else dev)
+        if world > 1:
+            dist.barrier()
+            dist.all_reduce(s_t, op=dist.ReduceOp.MAX)
+        s_ms = float(s_t.item())
+        se = 2 if args.dtype == "bf16" else 4
+        extras["strong_scaling"] = {
+            "workload": args.strong_workload, "units": U, "units_per_rank": [(r * U) // world for r in range(world + 1)],
+            "seq_len": sL, "d": sd, "w": sw_, "dtype": args.dtype, "ms_per_step": s_ms,
+            "tokens_per_s": sB * sL / (s_ms / 1e3) if s_ms > 0 else None,
+            "head_tokens_per_s": U * sL / (s_ms / 1e3) if s_ms > 0 else None,
+            "hbm_frac_per_gpu": step_bytes_per_row(sd, se) * U * sL / world / (s_ms / 1e3) / 1e9 / hbm_peak
+            if s_ms > 0 else None,
+            "scaling": "strong", "timing": "compute only (slab resident on its GPU), CUDA events, max over ranks"}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(shape, args.cpu_budget)
@@ -582,6 +690,9 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": args.dtype, "data": "synthetic: U(-1,1) q/k/v/dout generated on device",
+            **({"dtype_note": "fp32 storage and fp32 accuracy (north_star 1e-4 bound, parity-tested); the "
+                              "tensor-core products are bf16 hi + lo splits, 3 per fp32 product, fp32 "
+                              "accumulation (csrc/tc_band32.cu)"} if args.dtype == "f32" and path_b == ft.PATH_TC else {}),
             "config": cfg,
             "per_gpu_tokens_per_s": value / world,
             "paths": {"fwd": "tc" if path_f == ft.PATH_TC else "simt",
@@ -593,6 +704,7 @@ def main():
             "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": args.steps * (nf + nb),
             **({"e2e_nccl_scatter_gather": sg} if sg is not None else {}),
+            **extras,
             "clocks": sampler.summary(),
         }
         print(json.dumps(line), flush=True)
