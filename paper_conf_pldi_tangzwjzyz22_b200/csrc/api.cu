@@ -200,6 +200,24 @@ ft_status check_fwd(const void* q, const void* k, const void* v, void* out, floa
     return choose_path(0, batch * heads, seq_len, d, w, dilation, dtype, &path);
 }
 
+// Errors this call's launches report must be this call's: a non-sticky error another library
+// left pending on the calling thread (e.g. on PyTorch's autograd worker thread) would otherwise be
+// returned by the cudaGetLastError after our first launch.  Sticky errors persist and are reported.
+void clear_stale_error() { (void)cudaGetLastError(); }
+
+// The TMA descriptors are encoded with the driver API (cuTensorMapEncodeTiled), which needs the
+// device's context current on the calling thread.  A thread whose runtime calls so far did not
+// bind it -- PyTorch's autograd worker thread running a backward -- would get every encode
+// rejected; cudaSetDevice binds the primary context of the caller's current device.
+void bind_context() {
+    thread_local int bound = -1;
+    int dev = 0;
+    if (cudaGetDevice(&dev) == cudaSuccess && dev != bound) {
+        cudaSetDevice(dev);
+        bound = dev;
+    }
+}
+
 // Enqueue a validated forward.
 ft_status run_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t batch,
                   int64_t heads, int64_t seq_len, int64_t d, int64_t w, int64_t dilation, ft_dtype dtype,
@@ -209,6 +227,8 @@ ft_status run_fwd(const void* q, const void* k, const void* v, void* out, float*
     if (s != FT_OK) return s;
     cudaStream_t st = (cudaStream_t)stream;
     cudaError_t e;
+    bind_context();
+    clear_stale_error();
     if (path == FT_PATH_TC && dtype == FT_F32) {
         int n = 0;
         e = ftw::tc32_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, st, &n);
@@ -263,6 +283,8 @@ ft_status run_bwd(const void* q, const void* k, const void* v, const void* out, 
     cudaStream_t st = (cudaStream_t)stream;
     float* Dws = (float*)workspace;
     cudaError_t e;
+    bind_context();
+    clear_stale_error();
     if (path == FT_PATH_TC && dtype == FT_F32) {
         int n = 0;
         e = ftw::tc32_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w, dilation, st, &n);
@@ -458,6 +480,7 @@ ft_status ft_winattn_fwd_tape(const void* q, const void* k, const void* v, void*
     if (!tape) return FT_ERR_INVALID_VALUE;
     if (!aligned16(tape)) return FT_ERR_MISALIGNED;
     ftw::prof_reset();
+    clear_stale_error();
     const cudaError_t e = ftw::simt_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype,
                                         (cudaStream_t)stream, tape);
     return e == cudaSuccess ? FT_OK : cuda_fail(e);
@@ -474,6 +497,7 @@ ft_status ft_winattn_bwd_tape(const void* q, const void* k, const void* v, const
     if (!tape) return FT_ERR_INVALID_VALUE;
     if (!aligned16(tape)) return FT_ERR_MISALIGNED;
     ftw::prof_reset();
+    clear_stale_error();
     const cudaError_t e = ftw::simt_bwd(q, k, v, out, lse, dout, dq, dk, dv, (float*)workspace, batch,
                                         heads, seq_len, d, w, dilation, dtype, (cudaStream_t)stream, tape);
     return e == cudaSuccess ? FT_OK : cuda_fail(e);
