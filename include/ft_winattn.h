@@ -140,22 +140,23 @@ ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v,
 
 /* Tape vs recompute (the selective-materialization trade-off of PAPER.md:489-497 / Fig. 18,
  * SURVEY.md §8(f) item 2).  The plain entry points save only lse and RECOMPUTE the band
- * scores s_ij = q_i . k_j in the backward.  The _tape variants MATERIALIZE them instead:
- * ft_winattn_fwd_tape also writes tape, fp32 [batch*heads*seq_len][2*min(w, seq_len)+1] --
- * entry (row i, k + w) holds s_ij for key j = i + k*dilation (entries of keys outside the
- * sequence are left unwritten) -- and ft_winattn_bwd_tape reads it instead of recomputing
- * q_i . k_j.  Both always run the CUDA-core (SIMT) kernels, for either dtype; the tensor-core
- * path recomputes.  tape must hold ft_winattn_tape_bytes(...) bytes of device memory,
- * 16-byte aligned, not overlapping any other argument (not checked).  Errors: those of
- * ft_winattn_fwd / ft_winattn_bwd, plus FT_ERR_INVALID_VALUE for a NULL tape and
- * FT_ERR_MISALIGNED for a misaligned one. */
+ * scores in the backward.  The _tape variants MATERIALIZE them instead (Fig. 8's `dot`): the
+ * forward also writes tape, fp32 [batch*heads*seq_len][2*min(w, seq_len)+1] -- entry (row i, k + w)
+ * holds s_ij for key j = i + k*dilation (entries of keys outside the sequence are left unwritten)
+ * -- and the backward reads it instead of running the score GEMM q_i . k_j, computing
+ * P = exp(s - lse) from it.  bf16 calls the band tensor-core kernels can serve (w <= 64,
+ * d % 64 == 0, d <= 512) run on them; the rest on the CUDA-core kernels; forward and backward
+ * pick the same family for the same arguments (and FT_KNOB_PATH).  tape must hold
+ * ft_winattn_tape_bytes(...) bytes of device memory, 16-byte aligned, not overlapping any other
+ * argument (not checked).  Errors: those of ft_winattn_fwd / ft_winattn_bwd, plus
+ * FT_ERR_INVALID_VALUE for a NULL tape and FT_ERR_MISALIGNED for a misaligned one. */
 size_t    ft_winattn_tape_bytes(int64_t batch, int64_t heads, int64_t seq_len, int64_t w);
 ft_status ft_winattn_fwd_tape(const void* q, const void* k, const void* v,
-                              void* out, float* lse, float* tape,
+                              void* out, float* lse, void* tape,
                               int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
                               int64_t w, int64_t dilation, ft_dtype dtype, void* stream);
 ft_status ft_winattn_bwd_tape(const void* q, const void* k, const void* v,
-                              const void* out, const float* lse, const float* tape, const void* dout,
+                              const void* out, const float* lse, const void* tape, const void* dout,
                               void* dq, void* dk, void* dv,
                               int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
                               int64_t w, int64_t dilation, ft_dtype dtype,

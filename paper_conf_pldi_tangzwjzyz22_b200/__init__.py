@@ -272,8 +272,9 @@ def tape_bytes(q: torch.Tensor, w: int) -> int:
 
 
 def fwd_tape(q, k, v, w: int, dilation: int = 1):
-    """Forward that also materializes the band scores (ft_winattn_fwd_tape; CUDA-core kernels).
-    Returns (out, lse, tape) with tape fp32 [B, H, L, 2*min(w, L)+1]."""
+    """Forward that also materializes the band scores (ft_winattn_fwd_tape; band tensor-core
+    kernels for bf16 where they apply, else CUDA-core kernels).  Returns (out, lse, tape) with
+    tape fp32 [B, H, L, 2*min(w, L)+1]."""
     _check_inputs(q, k, v)
     B, H, L, d = q.shape
     out = torch.empty_like(q)

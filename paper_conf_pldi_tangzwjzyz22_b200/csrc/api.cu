@@ -472,22 +472,46 @@ size_t ft_winattn_tape_bytes(int64_t batch, int64_t heads, int64_t seq_len, int6
     return (size_t)(batch * heads * seq_len) * (size_t)(2 * wc + 1) * sizeof(float);
 }
 
+}  // extern "C"
+
+namespace {
+// Kernel family of a tape call (the same rule for the forward and the backward): the band
+// tensor-core kernels for bf16 where they apply, else the CUDA-core kernels.
+ft_status tape_path(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil, ft_dtype dt, int* path) {
+    const bool tc_ok = dt == FT_BF16 && ftw::tc_tape_supported(units, L, d, w, dil);
+    const int f = forced_path();
+    if (f == 2 && !tc_ok) return FT_ERR_NOT_SUPPORTED;
+    *path = (f != 1 && tc_ok) ? FT_PATH_TC : FT_PATH_SIMT;
+    return FT_OK;
+}
+}  // namespace
+
+extern "C" {
+
 ft_status ft_winattn_fwd_tape(const void* q, const void* k, const void* v, void* out, float* lse,
-                              float* tape, int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
+                              void* tape, int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
                               int64_t w, int64_t dilation, ft_dtype dtype, void* stream) {
     ft_status s = check_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype);
     if (s != FT_OK) return s;
     if (!tape) return FT_ERR_INVALID_VALUE;
     if (!aligned16(tape)) return FT_ERR_MISALIGNED;
+    int path = 0;
+    s = tape_path(batch * heads, seq_len, d, w, dilation, dtype, &path);
+    if (s != FT_OK) return s;
     ftw::prof_reset();
+    bind_context();
     clear_stale_error();
-    const cudaError_t e = ftw::simt_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype,
-                                        (cudaStream_t)stream, tape);
+    int n = 0;
+    const cudaError_t e =
+        path == FT_PATH_TC
+            ? ftw::tc_tape_fwd(q, k, v, out, lse, tape, batch, heads, seq_len, d, w, dilation, (cudaStream_t)stream, &n)
+            : ftw::simt_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype, (cudaStream_t)stream,
+                            static_cast<float*>(tape));
     return e == cudaSuccess ? FT_OK : cuda_fail(e);
 }
 
 ft_status ft_winattn_bwd_tape(const void* q, const void* k, const void* v, const void* out,
-                              const float* lse, const float* tape, const void* dout, void* dq, void* dk,
+                              const float* lse, const void* tape, const void* dout, void* dq, void* dk,
                               void* dv, int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
                               int64_t w, int64_t dilation, ft_dtype dtype, void* workspace,
                               size_t workspace_bytes, void* stream) {
@@ -496,13 +520,21 @@ ft_status ft_winattn_bwd_tape(const void* q, const void* k, const void* v, const
     if (s != FT_OK) return s;
     if (!tape) return FT_ERR_INVALID_VALUE;
     if (!aligned16(tape)) return FT_ERR_MISALIGNED;
+    int path = 0;
+    s = tape_path(batch * heads, seq_len, d, w, dilation, dtype, &path);
+    if (s != FT_OK) return s;
     ftw::prof_reset();
+    bind_context();
     clear_stale_error();
-    const cudaError_t e = ftw::simt_bwd(q, k, v, out, lse, dout, dq, dk, dv, (float*)workspace, batch,
-                                        heads, seq_len, d, w, dilation, dtype, (cudaStream_t)stream, tape);
+    int n = 0;
+    const cudaError_t e =
+        path == FT_PATH_TC
+            ? ftw::tc_tape_bwd(q, k, v, lse, tape, dout, dq, dk, dv, (float*)workspace, batch, heads, seq_len, d, w,
+                               dilation, (cudaStream_t)stream, &n)
+            : ftw::simt_bwd(q, k, v, out, lse, dout, dq, dk, dv, (float*)workspace, batch, heads, seq_len, d, w,
+                            dilation, dtype, (cudaStream_t)stream, static_cast<const float*>(tape));
     return e == cudaSuccess ? FT_OK : cuda_fail(e);
 }
-
 
 ft_status ft_winattn_fwd_bwd(const void* q, const void* k, const void* v, const void* dout, void* out,
                              float* lse, void* dq, void* dk, void* dv, int64_t batch, int64_t heads,

@@ -114,6 +114,17 @@ cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const float* l
                      void* dk, void* dv, float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
                      int64_t dil, cudaStream_t st, int* launches);
 
+// Score tape on the band kernels (bf16, w <= 64, d % 64 == 0): the forward also writes the band
+// scores (fp32 [rows][2w + 1], the CUDA-core kernels' format), the backward reads them and skips
+// the score GEMM -- tc_band.cu
+bool tc_tape_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
+cudaError_t tc_tape_fwd(const void* q, const void* k, const void* v, void* out, float* lse, void* tape,
+                        int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
+                        int* launches);
+cudaError_t tc_tape_bwd(const void* q, const void* k, const void* v, const float* lse, const void* tape,
+                        const void* dout, void* dq, void* dk, void* dv, float* Dws, int64_t B, int64_t H,
+                        int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches);
+
 // FT_ERR_CUDA with the CUDA error text recorded for ft_status_str (api.cu)
 ft_status cuda_error(cudaError_t e);
 

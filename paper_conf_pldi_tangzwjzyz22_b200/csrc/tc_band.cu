@@ -90,6 +90,12 @@ struct Params {
     int dpoll;                   // BWDKV: poll D row by row instead of waiting for all of BWDQ
     int lsepoll;                 // FWD -> BWDQ lse hand-off: FWD marks its lse rows unset and
                                  // triggers; BWDQ (PDL) and BWDKV poll lse rows
+    float* tape;                 // optional score tape (ft_winattn_fwd_tape / _bwd_tape): fp32
+                                 // [rows][2w + 1], entry (row i, k + w) = s_ij, key j = i + k dil
+                                 // (the materialized `dot` of Fig. 8).  FWD writes it; BWDQ / BWDKV
+                                 // read s from it and skip the score GEMM S = Q K^T (selective
+                                 // materialization)
+    int tstride;                 // tape row stride, elements (2w + 1)
 };
 
 
@@ -202,6 +208,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int NK = p.NK, nsl = p.nsl, w = p.w, NST = p.nst, d = p.d;
+    // backward with a P tape: only the dP GEMM runs in the score phase (one slot per slice)
+    const bool tp = MODE != FWD && p.tape != nullptr;
     // Programmatic dependent launch (BWDQ -> BWDKV, launch_pdl): BWDKV CTAs may take the SMs
     // BWDQ CTAs leave (its persistent CTAs finish 4 or 5 tiles apart) and stream their first
     // tiles' q/k/v/dout -- inputs of the whole backward call, complete before BWDQ started --
@@ -308,12 +316,15 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             auto adv = [&]() { if (++st == NST) { st = 0; ph ^= 1u; } };
             auto load_g_slice = [&](const Tile& T, int j, int s) {
                 const Maps& mp = p.maps[T.rl];
-                uint8_t* sp = take();
-                if (s == 0) trace_ev(p, j, 0);
-                mbar_arrive_expect_tx(&full[st], ABYTES + HB);
-                tma_load_3d(sp, &mp.a1, &full[st], s * 64, T.m0, T.u);
-                tma_load_3d(sp + ABYTES, &mp.b1, &full[st], s * 64, T.m0 - w, T.u);
-                adv();
+                uint8_t* sp;
+                if (!tp) {
+                    sp = take();
+                    if (s == 0) trace_ev(p, j, 0);
+                    mbar_arrive_expect_tx(&full[st], ABYTES + HB);
+                    tma_load_3d(sp, &mp.a1, &full[st], s * 64, T.m0, T.u);
+                    tma_load_3d(sp + ABYTES, &mp.b1, &full[st], s * 64, T.m0 - w, T.u);
+                    adv();
+                }
                 if (C::NA == 2) {
                     sp = take();
                     mbar_arrive_expect_tx(&full[st], ABYTES + HB);
@@ -396,16 +407,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 if (++st == NST) { st = 0; ph ^= 1u; }
             };
             auto g_slice = [&](int j, int s) {
-                const uint32_t a1 = wait_full();
-                if (s == 0 && h == 0) trace_ev(p, j, 2);
-                if (ownS) {
-                    const uint32_t b1 = a1 + ABYTES;
+                if (!tp) {
+                    const uint32_t a1 = wait_full();
+                    if (s == 0 && h == 0) trace_ev(p, j, 2);
+                    if (ownS) {
+                        const uint32_t b1 = a1 + ABYTES;
 #pragma unroll
-                    for (int kk = 0; kk < 4; ++kk)
-                        mma_ss(tbase, sdesc_sw128(a1 + kk * 32, 16, 1024),
-                               sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
+                        for (int kk = 0; kk < 4; ++kk)
+                            mma_ss(tbase, sdesc_sw128(a1 + kk * 32, 16, 1024),
+                                   sdesc_sw128(b1 + kk * 32, 16, 1024), idS, (s | kk) != 0);
+                    }
+                    release(ownS);
                 }
-                release(ownS);
                 if (C::NA == 2) {
                     const uint32_t a2 = wait_full();
                     if (ownDP) {
@@ -569,11 +582,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     for (int c = 0; c < nch; ++c)
                         if (c < c_lo || c > c_hi) st_p_chunk(sP, t, c, zero16);
                 float mx = -INFINITY;
+                // score tape: this row's band scores, entry n - t = k + w
+                float* ts = p.tape != nullptr && mrow < Lr ? p.tape + (rowbase + (int64_t)mrow * p.dil) * p.tstride : nullptr;
                 for (int c = c_lo; c <= c_hi; ++c) {
                     uint32_t rr[32];
                     tmem_ld32(trow + c * 32, rr);
                     tmem_wait_ld();
                     mx = chunk_max(rr, c * 32, t, w, kb, Lr, mx);
+                    if (ts) {
+#pragma unroll
+                        for (int e = 0; e < 32; ++e)
+                            if (band_ok(c * 32 + e, t, w, kb + c * 32 + e, Lr)) ts[c * 32 + e - t] = __uint_as_float(rr[e]);
+                    }
                 }
                 if (mx == -INFINITY) mx = 0.f;   // only rows beyond the sequence (never stored)
                 const float mxs = mx * LOG2E;
@@ -597,17 +617,20 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                                    : (p.lsepoll ? ld_lse_ready(p.lse + rowbase + (int64_t)mrow * p.dil, lse_settled)
                                                 : p.lse[rowbase + (int64_t)mrow * p.dil]) * LOG2E;
                 float D = 0.f;
+                // tape: this row's band scores read back (entry n - t); rows beyond the sequence get P = 0
+                const float* tq = tp && mrow < Lr ? p.tape + (rowbase + (int64_t)mrow * p.dil) * p.tstride : nullptr;
+                auto tape_p = [&](int n) -> float { return fast_exp2(fmaf(__ldg(tq + (n - t)), LOG2E, -lse2)); };
                 for (int c = c_lo; c <= c_hi; ++c) {   // pass 1: D = sum_j P_ij dP_ij
                     uint32_t rs[32], rd[32];
-                    tmem_ld32(trow + c * 32, rs);
+                    if (!tp) tmem_ld32(trow + c * 32, rs);
                     tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
 #pragma unroll
                     for (int e = 0; e < 32; ++e) {
                         const int n = c * 32 + e;
-                        const float pv = band_ok(n, t, w, kb + n, Lr)
-                                             ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2))
-                                             : 0.f;
+                        const bool ok = band_ok(n, t, w, kb + n, Lr);
+                        const float pv = tp ? (ok && tq ? tape_p(n) : 0.f)
+                                            : (ok ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f);
                         D = fmaf(pv, __uint_as_float(rd[e]), D);
                     }
                 }
@@ -626,7 +649,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         continue;
                     }
                     uint32_t rs[32], rd[32], pk[16], pl[16];
-                    tmem_ld32(trow + c * 32, rs);
+                    if (!tp) tmem_ld32(trow + c * 32, rs);
                     tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
 #pragma unroll
@@ -635,9 +658,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 #pragma unroll
                         for (int h = 0; h < 2; ++h) {
                             const int n = c * 32 + e + h;
-                            const float pv = band_ok(n, t, w, kb + n, Lr)
-                                                 ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -lse2))
-                                                 : 0.f;
+                            const bool ok = band_ok(n, t, w, kb + n, Lr);
+                            const float pv = tp ? (ok && tq ? tape_p(n) : 0.f)
+                                                : (ok ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -lse2)) : 0.f);
                             dv[h] = pv * (__uint_as_float(rd[e + h]) - D);
                         }
                         split_bf16x2(dv[0], dv[1], pk[e / 2], pl[e / 2]);
@@ -660,7 +683,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         continue;
                     }
                     uint32_t rs[32], rd[32], pk[16], dk[16], dl[16];
-                    tmem_ld32(trow + c * 32, rs);
+                    if (!tp) tmem_ld32(trow + c * 32, rs);
                     tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
 #pragma unroll
@@ -669,9 +692,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 #pragma unroll
                         for (int h = 0; h < 2; ++h) {
                             const int n = c * 32 + e + h;
-                            pv[h] = band_ok(n, t, w, kb + n, Lr)
-                                        ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -colLse[n]))
-                                        : 0.f;
+                            // tape: S^T[key t][query n] = tape[query kb + n][t - n + 2w] (offset of
+                            // key m0 + t from query kb + n is t - n + w); one 128-byte line per warp
+                            const bool ok = band_ok(n, t, w, kb + n, Lr) && (!tp || mrow < Lr);
+                            pv[h] = !ok ? 0.f
+                                    : fast_exp2(fmaf(tp ? __ldg(p.tape + (rowbase + (int64_t)(kb + n) * p.dil) * p.tstride + (t - n + 2 * w))
+                                                        : __uint_as_float(rs[e + h]),
+                                                     LOG2E, -colLse[n]));
                             dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
                         }
                         pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
@@ -775,6 +802,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     }
 }
 
+int tape_stride(int64_t wc);
+
 template <int MODE>
 void set_attr_once() {
     static std::once_flag once;
@@ -808,7 +837,8 @@ int halo_rows(int64_t L, int64_t w) {
 template <int MODE>
 cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b2, const void* ob1,
                    const void* ob2, void* o1, void* o2, float* lse, float* D, int64_t B, int64_t H,
-                   int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
+                   int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches,
+                   float* tape = nullptr) {
     const int64_t wc = w < L ? w : L;
     const int NK = halo_rows(L, w);
     const int64_t units = B * H;
@@ -849,7 +879,9 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         p.dpoll = MODE != FWD && dpoll_enabled();
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
-        p.lsepoll = lsepoll_enabled() && r0 == 0 && lsepoll_worth(total, num_sms());
+        p.lsepoll = lsepoll_enabled() && r0 == 0 && lsepoll_worth(total, num_sms()) && tape == nullptr;
+        p.tape = tape;
+        p.tstride = tape_stride(wc);
         dim3 grid((unsigned)(total < num_sms() ? total : num_sms()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_smem_bytes<MODE>(NK) + (size_t)nst * slot_bytes(NK);
@@ -886,6 +918,8 @@ bool band_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil)
            units * ((L + 127) / 128) < (1 << 30) && pick_nst<BWDKV>(NK) >= 2 &&
            pick_nst<FWD>(NK) >= 2 && pick_nst<BWDQ>(NK) >= 2;
 }
+
+int tape_stride(int64_t wc) { return (int)(2 * wc + 1); }
 
 int band_launches(int64_t L, int64_t dil) {
     const int64_t nres = dil < L ? dil : L;
@@ -946,6 +980,30 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
     // BWDKV accumulation order per chunk: dV (P^T dO, ob1 = dout) then dK (dS^T Q, ob2 = q)
     return launch<BWDKV>(k, q, v, dout, dout, q, dv, dk, const_cast<float*>(lse), Dws, B, H, L,
                          d, w, dil, st, launches);
+}
+
+bool tc_tape_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    return halo_rows(L, w) <= 256 && band_supported(units, L, d, w, dil);
+}
+
+cudaError_t tc_tape_fwd(const void* q, const void* k, const void* v, void* out, float* lse, void* tape,
+                        int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st,
+                        int* launches) {
+    if (launches) *launches = 0;
+    return launch<FWD>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, B, H, L, d, w, dil, st,
+                       launches, static_cast<float*>(tape));
+}
+
+cudaError_t tc_tape_bwd(const void* q, const void* k, const void* v, const float* lse, const void* tape,
+                        const void* dout, void* dq, void* dk, void* dv, float* Dws, int64_t B, int64_t H,
+                        int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
+    if (launches) *launches = 0;
+    float* t = const_cast<float*>(static_cast<const float*>(tape));
+    cudaError_t e = launch<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse), Dws, B, H, L, d,
+                                 w, dil, st, launches, t);
+    if (e != cudaSuccess) return e;
+    return launch<BWDKV>(k, q, v, dout, dout, q, dv, dk, const_cast<float*>(lse), Dws, B, H, L, d, w, dil, st,
+                         launches, t);
 }
 
 }  // namespace ftw

@@ -63,14 +63,26 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
 #endif
     return ok != 0;
 }
-// Watchdog: a protocol bug must end the kernel with an error, not hang the GPU.
+// Watchdog: a protocol bug must end the kernel with an error (cudaErrorLaunchFailure), not hang
+// the GPU.  No legitimate wait in these kernels lasts more than milliseconds; after
+// FT_WATCHDOG_NS of global time (checked every 256 polls) the waiting thread traps.
+#ifndef FT_WATCHDOG_NS
+#define FT_WATCHDOG_NS 4000000000ull
+#endif
 #ifndef FT_WATCHDOG_SPINS
 #define FT_WATCHDOG_SPINS (1u << 28)
 #endif
+__device__ __forceinline__ uint64_t global_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    if (mbar_try_wait(bar, parity)) return;
+    const uint64_t t0 = global_ns();
     uint32_t spins = 0;
     while (!mbar_try_wait(bar, parity)) {
-        if (++spins == FT_WATCHDOG_SPINS) __trap();
+        if ((++spins & 255u) == 0 && global_ns() - t0 > FT_WATCHDOG_NS) __trap();
     }
 }
 
@@ -89,9 +101,11 @@ __device__ __forceinline__ bool mbar_try_wait_spin(uint64_t* bar, uint32_t parit
     return ok != 0;
 }
 __device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
+    if (mbar_try_wait_spin(bar, parity)) return;
+    const uint64_t t0 = global_ns();
     uint32_t spins = 0;
     while (!mbar_try_wait_spin(bar, parity)) {
-        if (++spins == FT_WATCHDOG_SPINS) __trap();
+        if ((++spins & 1023u) == 0 && global_ns() - t0 > FT_WATCHDOG_NS) __trap();
     }
 }
 
@@ -365,11 +379,13 @@ constexpr uint32_t D_UNSET = 0xFFFFFFFFu;
 __device__ __forceinline__ float ld_D_ready(const float* ptr) {
     // D is stored by the dQ kernel of the same call, which is resident (the dependent grid
     // launches only after every dQ CTA triggered): a protocol bug traps instead of hanging
-    uint32_t x, spins = 0;
+    uint32_t x;
+    uint64_t t0 = 0;
     for (;;) {
         asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr) : "memory");
         if (x != D_UNSET) break;
-        if (++spins == FT_WATCHDOG_SPINS) __trap();
+        if (t0 == 0) t0 = global_ns();
+        else if (global_ns() - t0 > FT_WATCHDOG_NS) __trap();
         __nanosleep(128);
     }
     return __uint_as_float(x);

@@ -469,14 +469,21 @@ def test_mixed_dilation(ft, case):
 
 
 # Tape vs recompute (ft_winattn_fwd_tape / bwd_tape): the backward
-# reads the materialized band scores instead of recomputing them; same results as the oracle.
+# reads the materialized band scores instead of running the score GEMM -- on the band
+# tensor-core kernels for bf16 (w <= 64, d % 64 == 0), else on the CUDA-core kernels -- and must
+# give the oracle's results; the tape holds q_i . k_j.
 TAPE = [
     (1, 1, 64, 16, 4, 1, "f32"),
     (1, 2, 300, 64, 32, 3, "f32"),
-    (2, 1, 257, 128, 17, 2, "bf16"),
     (1, 1, 200, 512, 32, 1, "f32"),
     (1, 1, 50, 64, 100, 1, "f32"),     # w >= L
+    (2, 1, 257, 128, 17, 2, "bf16"),   # band kernels, dilation, ragged
     (1, 1, 130, 64, 0, 1, "bf16"),     # w = 0
+    (1, 2, 700, 512, 32, 1, "bf16"),   # the C2a shape
+    (1, 2, 900, 64, 32, 3, "bf16"),
+    (1, 2, 600, 256, 64, 1, "bf16"),   # widest band-kernel halo (256 rows)
+    (1, 2, 9000, 512, 32, 4, "bf16"),  # many tiles per CTA, residues
+    (1, 1, 300, 64, 100, 1, "bf16"),   # w > 64: CUDA-core tape
 ]
 
 

@@ -1,16 +1,20 @@
 """Tape vs recompute on B200 (Fig. 18): the paper's
 selective materialization decides per intermediate whether the gradient program reads it from a
-tape or recomputes it.  Here the intermediate is the band score s_ij = q_i . k_j:
+tape or recomputes it.  Here the intermediate is the band score s_ij = q_i . k_j (Fig. 8's `dot`):
 
-  recompute : ft_winattn_fwd + ft_winattn_bwd (saves lse only; bwd recomputes q_i . k_j)
-  tape      : ft_winattn_fwd_tape + ft_winattn_bwd_tape (fwd writes s, fp32 [rows][2w+1]; bwd reads it)
+  recompute : ft_winattn_fwd + ft_winattn_bwd (saves lse only; bwd reruns the score GEMM)
+  tape      : ft_winattn_fwd_tape + ft_winattn_bwd_tape (fwd also writes s, fp32 [rows][2w+1];
+              bwd reads it and skips the score GEMM)
 
-both on the CUDA-core kernels (FT_WINATTN_PATH=simt), plus the tensor-core recompute path for
-bf16.  Prints ms per fwd+bwd step (CUDA events, mean of 10 after 3 warm-ups) and the tape's
-extra HBM bytes per step (write + read).
+on the band tensor-core kernels (bf16; the d = 64, w <= 32 narrow kernels are switched off for
+the recompute leg so both legs use the same kernels) and on the CUDA-core kernels (fp32).  Both
+legs of one family run on the same inputs; one JSON line per case with ms per fwd+bwd step (CUDA
+events, mean of 20 after 3 warm-ups, L2 flushed between steps) and the tape's extra HBM bytes per
+step (one write + two reads, the dQ and dK/dV kernels each read it).
 
-    python tools/tape_ablation.py
+    python tools/tape_ablation.py [--quick]
 """
+import argparse
 import json
 import os
 import sys
@@ -21,53 +25,61 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 import paper_conf_pldi_tangzwjzyz22_b200 as ft  # noqa: E402
 
-CASES = [  # (name, B, H, L, d, w, dil)
-    ("C2a", 1, 8, 10000, 512, 32, 1),
-    ("C2b", 1, 12, 4096, 64, 256, 1),
-    ("d64_w32", 1, 16, 8192, 64, 32, 1),
-    ("d128_w64", 1, 8, 8192, 128, 64, 1),
-]
+# (name, B, H, L, d, w, dil): a (d, w) grid for the tensor-core family (w <= 64) and the C2 shapes
+TC_CASES = [(f"d{d}_w{w}", 1, max(1, 16 * 64 // d), 8192, d, w, 1)
+            for d in (64, 128, 256, 512) for w in (8, 32, 64)] + [("C2a", 1, 8, 10000, 512, 32, 1)]
+SIMT_CASES = [("C2a", 1, 8, 10000, 512, 32, 1), ("C2b", 1, 12, 4096, 64, 256, 1), ("d64_w32", 1, 16, 8192, 64, 32, 1)]
+FLUSH = None
 
 
-def timed(fn, n=10, warm=3):
+def timed(fn, n=20, warm=3):
     for _ in range(warm):
         fn()
     torch.cuda.synchronize()
-    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    a.record()
+    tot = 0.0
     for _ in range(n):
+        FLUSH.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
         fn()
-    b.record()
-    torch.cuda.synchronize()
-    return a.elapsed_time(b) / n
+        b.record()
+        b.synchronize()
+        tot += a.elapsed_time(b)
+    return tot / n
+
+
+def run(name, B, H, L, d, w, dil, dt, knobs):
+    dev = torch.device("cuda:0")
+    q, k, v, g = [(torch.rand(B, H, L, d, device=dev) * 2 - 1).to(dt) for _ in range(4)]
+    res = {"case": name, "dtype": "f32" if dt == torch.float32 else "bf16", "shape": [B, H, L, d, w, dil],
+           "family": "simt" if knobs.get("path") == "simt" else "tensor cores (band kernels)",
+           "tape_extra_bytes_per_step": 3 * ft.tape_bytes(q, w)}
+
+    def rec():
+        out, lse = ft.fwd(q, k, v, w, dil)
+        ft.bwd(q, k, v, out, lse, g, w, dil)
+
+    def tap():
+        out, lse, tape = ft.fwd_tape(q, k, v, w, dil)
+        ft.bwd_tape(q, k, v, out, lse, tape, g, w, dil)
+
+    with ft.knobs(**knobs):
+        res["recompute_ms"] = timed(rec)
+        res["tape_ms"] = timed(tap)
+    res["tape_speedup"] = res["recompute_ms"] / res["tape_ms"]
+    print(json.dumps(res), flush=True)
 
 
 def main():
-    dev = torch.device("cuda:0")
-    for name, B, H, L, d, w, dil in CASES:
-        for dt in (torch.float32, torch.bfloat16):
-            q, k, v, g = [(torch.rand(B, H, L, d, device=dev) * 2 - 1).to(dt) for _ in range(4)]
-            res = {"case": name, "dtype": "f32" if dt == torch.float32 else "bf16",
-                   "shape": [B, H, L, d, w, dil],
-                   "tape_extra_bytes_per_step": 2 * ft.tape_bytes(q, w)}
-
-            def rec():
-                out, lse = ft.fwd(q, k, v, w, dil)
-                ft.bwd(q, k, v, out, lse, g, w, dil)
-
-            def tap():
-                out, lse, tape = ft.fwd_tape(q, k, v, w, dil)
-                ft.bwd_tape(q, k, v, out, lse, tape, g, w, dil)
-
-            os.environ["FT_WINATTN_PATH"] = "simt"
-            res["simt_recompute_ms"] = timed(rec)
-            res["simt_tape_ms"] = timed(tap)
-            os.environ.pop("FT_WINATTN_PATH")
-            if dt == torch.bfloat16:
-                res["tc_recompute_ms"] = timed(rec)
-            print(json.dumps(res), flush=True)
-            del q, k, v, g
-            torch.cuda.empty_cache()
+    global FLUSH
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--quick", action="store_true")
+    a = ap.parse_args()
+    FLUSH = torch.empty(256 << 20, dtype=torch.uint8, device="cuda:0")
+    for c in TC_CASES[-4:] if a.quick else TC_CASES:
+        run(*c, torch.bfloat16, {"narrow": 0})
+    for c in SIMT_CASES[:1] if a.quick else SIMT_CASES:
+        run(*c, torch.float32, {"path": "simt"})
 
 
 if __name__ == "__main__":
