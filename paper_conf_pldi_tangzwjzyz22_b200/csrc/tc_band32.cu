@@ -342,8 +342,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             if (ct == 0) trace_slot(p, k, 1);
             uint8_t* sp = slots + (size_t)st * SLOT;
             if (kind == 0) {
-                convert_rows<64, 2>(sp, BM, ct);
-                convert_rows<64, 2>(sp + 2 * BM * 64, NK, ct);
+                convert_rows<64, 1>(sp, BM, ct);
+                convert_rows<64, 1>(sp + 2 * BM * 64, NK, ct);
             } else {
                 convert_rows<128, 1>(sp, KB, ct);
                 if (chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW) convert_rows<128, 1>(sp + 2 * KB * 128, KB, ct);
