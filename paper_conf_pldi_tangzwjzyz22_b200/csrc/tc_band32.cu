@@ -127,58 +127,57 @@ __device__ __forceinline__ bool band_ok(int n, int t, int w, int mcol, int Lr) {
     return (unsigned)(n - t) <= (unsigned)(2 * w) && mcol >= 0 && mcol < Lr;
 }
 
-// In-place fp32 -> bf16 hi / lo planes for the R rows of a box pair: box0 at p, box1 at p + R * RB,
+// In-place fp32 -> bf16 hi / lo planes of box pairs: a pair is box0 at p and box1 at p + R * RB,
 // RB-byte rows (RB = 128: 32 fp32 per box row, SWIZZLE_128B, 16-byte granule g of row r at
 // (g ^ (r & 7)) * 16; RB = 64: 16 fp32, SWIZZLE_64B, granule g at (g ^ ((r >> 1) & 3)) * 16).
-// The 2 * RB / 4 fp32 of row r (box0 columns first) become the bf16 hi row over box0 and the lo row
-// over box1 -- the K-major (score slices) or MN-major (output blocks) bf16 operand rows.  Four
-// threads per row (one warp holds whole rows): thread q reads fp32 columns [q, q + 1) * RB / 8 and
-// writes bf16 granule(s) of the same columns in both planes, after a __syncwarp separating every
-// read of the row from every write.  UNR row passes per iteration keep 2 UNR RB / 64 loads in
-// flight per thread (one pass per iteration was load-latency bound: ~4.2 kclk per 40 KB score
-// slot, tools/trace32.py).  ct: converter thread 0 .. 32 NCONV - 1.
+// The 2 RB / 4 fp32 of row r (box0 columns first) become the bf16 hi row over box0 and the lo row
+// over box1 -- the K-major (score slices) or MN-major (output blocks) bf16 operand rows.  One
+// thread converts a whole row: it reads every byte it writes, so no thread waits for another
+// (the earlier four-threads-per-row form needed a __syncwarp between reads and writes and ran
+// ~5.6 instructions per element; this one ~2, tools/trace32.py: 1.8 -> see DESIGN.md §7).  The
+// rows of two pairs (R0 rows at p0, R1 rows at p1) are dealt round robin to the 32 NCONV
+// converter threads; ct: converter thread 0 .. 32 NCONV - 1.
 template <int RB>
 __device__ __forceinline__ int swz(int g, int r) { return RB == 128 ? (g ^ (r & 7)) : (g ^ ((r >> 1) & 3)); }
 
-template <int RB, int UNR>
-__device__ __forceinline__ void convert_rows(uint8_t* p, int R, int ct) {
-    constexpr int NG = RB / 32;                  // 16-byte fp32 granules read per thread per row
-    const int q = ct & 3;
-    uint8_t* src = p + (q >> 1) * R * RB;        // box holding this thread's fp32 columns
-    constexpr int PASS = 8 * NCONV;              // rows per pass
-    for (int r0 = 0; r0 < R; r0 += UNR * PASS) {
-        uint4 v[UNR][NG];
+// (x0, x1) -> hi = bf16x2 RN, lo = bf16x2 RN of (x0, x1) - hi, with one packed fp32 subtraction
+__device__ __forceinline__ void split2p(float x0, float x1, uint32_t& hi, uint32_t& lo) {
+    asm("{\n\t.reg .b32 h0, h1, r0, r1;\n\t.reg .b64 xx, hh, rr;\n\t"
+        "cvt.rn.bf16x2.f32 %0, %3, %2;\n\t"
+        "shl.b32 h0, %0, 16;\n\tand.b32 h1, %0, 0xffff0000;\n\t"
+        "mov.b64 xx, {%2, %3};\n\tmov.b64 hh, {h0, h1};\n\t"
+        "sub.rn.f32x2 rr, xx, hh;\n\t"
+        "mov.b64 {r0, r1}, rr;\n\t"
+        "cvt.rn.bf16x2.f32 %1, r1, r0;\n\t}"
+        : "=r"(hi), "=r"(lo)
+        : "f"(x0), "f"(x1));
+}
+
+template <int RB>
+__device__ __forceinline__ void convert_rows2(uint8_t* p0, int R0, uint8_t* p1, int R1, int ct) {
+    constexpr int NX = RB / 16;   // 16-byte fp32 granules per box row
+    for (int vr = ct; vr < R0 + R1; vr += 32 * NCONV) {
+        const bool first = vr < R0;
+        uint8_t* p = first ? p0 : p1;
+        const int R = first ? R0 : R1, r = first ? vr : vr - R0;
+        uint4 v[2 * NX];
 #pragma unroll
-        for (int u = 0; u < UNR; ++u) {
-            const int r = r0 + u * PASS + (ct >> 2);
-            if (r < R) {
+        for (int b = 0; b < 2; ++b)
 #pragma unroll
-                for (int x = 0; x < NG; ++x)
-                    v[u][x] = *reinterpret_cast<const uint4*>(src + r * RB + (swz<RB>(NG * (q & 1) + x, r) << 4));
-            }
+            for (int g = 0; g < NX; ++g)
+                v[b * NX + g] = *reinterpret_cast<const uint4*>(p + b * R * RB + r * RB + (swz<RB>(g, r) << 4));
+#pragma unroll
+        for (int G = 0; G < NX; ++G) {   // output granule G: fp32 columns 8G .. 8G + 7
+            const uint4 a = v[2 * G], c = v[2 * G + 1];
+            uint32_t hi[4], lo[4];
+            split2p(__uint_as_float(a.x), __uint_as_float(a.y), hi[0], lo[0]);
+            split2p(__uint_as_float(a.z), __uint_as_float(a.w), hi[1], lo[1]);
+            split2p(__uint_as_float(c.x), __uint_as_float(c.y), hi[2], lo[2]);
+            split2p(__uint_as_float(c.z), __uint_as_float(c.w), hi[3], lo[3]);
+            const uint32_t off = r * RB + (swz<RB>(G, r) << 4);
+            *reinterpret_cast<uint4*>(p + off) = make_uint4(hi[0], hi[1], hi[2], hi[3]);
+            *reinterpret_cast<uint4*>(p + R * RB + off) = make_uint4(lo[0], lo[1], lo[2], lo[3]);
         }
-        __syncwarp();
-#pragma unroll
-        for (int u = 0; u < UNR; ++u) {
-            const int r = r0 + u * PASS + (ct >> 2);
-            if (r < R) {
-                uint32_t hi[2 * NG], lo[2 * NG];
-#pragma unroll
-                for (int x = 0; x < NG; ++x) {
-                    split2(__uint_as_float(v[u][x].x), __uint_as_float(v[u][x].y), hi[2 * x], lo[2 * x]);
-                    split2(__uint_as_float(v[u][x].z), __uint_as_float(v[u][x].w), hi[2 * x + 1], lo[2 * x + 1]);
-                }
-                // bf16 columns of this thread: granules NG / 2 * q .. of the plane rows
-#pragma unroll
-                for (int y = 0; y < NG / 2; ++y) {
-                    const uint32_t off = r * RB + (swz<RB>((NG / 2) * q + y, r) << 4);
-                    *reinterpret_cast<uint4*>(p + off) = make_uint4(hi[4 * y], hi[4 * y + 1], hi[4 * y + 2], hi[4 * y + 3]);
-                    *reinterpret_cast<uint4*>(p + R * RB + off) =
-                        make_uint4(lo[4 * y], lo[4 * y + 1], lo[4 * y + 2], lo[4 * y + 3]);
-                }
-            }
-        }
-        __syncwarp();
     }
 }
 
@@ -342,11 +341,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             if (ct == 0) trace_slot(p, k, 1);
             uint8_t* sp = slots + (size_t)st * SLOT;
             if (kind == 0) {
-                convert_rows<64, 1>(sp, BM, ct);
-                convert_rows<64, 1>(sp + 2 * BM * 64, NK, ct);
+                convert_rows2<64>(sp, BM, sp + 2 * BM * 64, NK, ct);
             } else {
-                convert_rows<128, 1>(sp, KB, ct);
-                if (chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW) convert_rows<128, 1>(sp + 2 * KB * 128, KB, ct);
+                const bool full_chunk = chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW;
+                convert_rows2<128>(sp, KB, sp + 2 * KB * 128, full_chunk ? KB : 0, ct);
             }
             fence_proxy_async_smem();
             warp_arrive(&conv[st]);
