@@ -5,15 +5,16 @@ cd "$(dirname "$0")/.."
 cat > /tmp/san_case.py <<'PY'
 import os, sys, torch
 sys.path.insert(0, ".")
-if len(sys.argv) > 1:   # "fused": the one-kernel d = 64 backward (tc_narrow_fused.cu) on every d = 64 case
-    os.environ["FT_WINATTN_FUSED"] = "2"
 import paper_conf_pldi_tangzwjzyz22_b200 as ft
+if len(sys.argv) > 1:   # "nopdl": every launch in plain stream order (FT_KNOB_PDL = 0)
+    ft.debug_set("pdl", 0)
 from synth import WinAttnShape, make_inputs
 dev = torch.device("cuda:0")
 for shape, dt in [((1, 2, 300, 64, 32, 3), "bf16"), ((1, 4, 1500, 64, 32, 1), "bf16"),
                   ((1, 2, 700, 64, 20, 5), "bf16"), ((1, 1, 200, 512, 32, 1), "bf16"),
                   ((1, 1, 600, 64, 100, 2), "bf16"), ((1, 1, 500, 128, 80, 1), "bf16"),
-                  ((1, 1, 130, 64, 8, 1), "f32")]:
+                  ((1, 1, 130, 64, 8, 1), "f32"), ((1, 2, 300, 512, 32, 1), "f32"),
+                  ((1, 2, 257, 128, 17, 3), "f32"), ((1, 1, 300, 192, 8, 1), "f32")]:
     s = WinAttnShape(*shape)
     x = make_inputs(s, 0, dt)
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
@@ -25,12 +26,19 @@ x = make_inputs(s, 0, "bf16")
 q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
 o, l = ft.fwd(q, k, v, s.w, s.dilation, dilated_heads=2)
 ft.bwd(q, k, v, o, l, g, s.w, s.dilation, dilated_heads=2)
-# tape path (SIMT kernels with the materialized scores)
-s = WinAttnShape(1, 2, 300, 64, 20, 3)
-x = make_inputs(s, 0, "f32")
-q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
-o, l, tp = ft.fwd_tape(q, k, v, s.w, s.dilation)
-ft.bwd_tape(q, k, v, o, l, tp, g, s.w, s.dilation)
+# tape path (materialized scores): CUDA-core (fp32) and band tensor-core (bf16) kernels
+for dt in ("f32", "bf16"):
+    s = WinAttnShape(1, 2, 300, 64, 20, 3)
+    x = make_inputs(s, 0, dt)
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    o, l, tp = ft.fwd_tape(q, k, v, s.w, s.dilation)
+    ft.bwd_tape(q, k, v, o, l, tp, g, s.w, s.dilation)
+# one-call forward + backward (lse hand-off)
+for shape in ((1, 2, 700, 512, 32, 1), (1, 4, 900, 64, 32, 1)):
+    s = WinAttnShape(*shape)
+    x = make_inputs(s, 0, "bf16")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    ft.fwd_bwd(q, k, v, g, s.w, s.dilation)
 # SubdivNet circular difference: vector / scalar, gather / scatter, fp32 / bf16
 import numpy as np
 from paper_conf_pldi_tangzwjzyz22_b200 import subdiv
@@ -45,10 +53,10 @@ for f, dt in ((64, "f32"), (13, "f32"), (64, "bf16")):
 torch.cuda.synchronize()
 print("cases ok")
 PY
-for variant in default fused; do
+for variant in default nopdl; do
   for tool in memcheck racecheck synccheck initcheck; do
     echo "== $tool ($variant)"
     timeout 600 compute-sanitizer --tool $tool --kernel-name kns=tc_ --kernel-name kns=simt --kernel-name kns=circdiff --kernel-name kns=f32_to_bf16 --kernel-name kns=zero_f32 --print-limit 10 \
-      python /tmp/san_case.py $([ $variant = fused ] && echo fused) 2>&1 | tail -4
+      python /tmp/san_case.py $([ $variant = nopdl ] && echo nopdl) 2>&1 | tail -4
   done
 done
