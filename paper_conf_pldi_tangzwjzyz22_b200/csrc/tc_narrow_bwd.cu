@@ -210,7 +210,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             for (int b = 0; b < 2; ++b) {
                 mbar_init(&acc_full[b], 1);
                 mbar_init(&acc_free[b], 8);
-                mbar_init(&hs_full[b], 1);
+                mbar_init(&hs_full[b], 32);
             }
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
@@ -274,8 +274,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 sc[q] = __uint_as_float((uint32_t)(127 + f) << 23);
                 tab[lane + 32 * q] = __uint_as_float((uint32_t)(127 - f) << 23);
             }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&hs_full[j & 1]);
+            mbar_arrive(&hs_full[j & 1]);   // every lane releases its own table entries
 #pragma unroll
             for (int q = 0; q < NK / 32; ++q) {
                 uint4* row = reinterpret_cast<uint4*>(hb + (lane + 32 * q) * 128);
