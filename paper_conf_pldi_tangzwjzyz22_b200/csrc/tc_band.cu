@@ -199,7 +199,9 @@ __device__ __forceinline__ float chunk_exp_store(uint8_t* sP, const uint32_t (&r
     return sum;
 }
 
-template <int MODE>
+// TAPE: score tape read (BWDQ / BWDKV) or written (FWD) -- a separate instantiation, so the plain
+// kernels carry no tape code in their softmax loops
+template <int MODE, bool TAPE>
 __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_constant__ Params p) {
     using C = Cfg<MODE>;
     extern __shared__ uint8_t smem_raw[];
@@ -209,7 +211,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int NK = p.NK, nsl = p.nsl, w = p.w, NST = p.nst, d = p.d;
     // backward with a P tape: only the dP GEMM runs in the score phase (one slot per slice)
-    const bool tp = MODE != FWD && p.tape != nullptr;
+    constexpr bool tp = TAPE && MODE != FWD;
     // Programmatic dependent launch (BWDQ -> BWDKV, launch_pdl): BWDKV CTAs may take the SMs
     // BWDQ CTAs leave (its persistent CTAs finish 4 or 5 tiles apart) and stream their first
     // tiles' q/k/v/dout -- inputs of the whole backward call, complete before BWDQ started --
@@ -583,7 +585,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         if (c < c_lo || c > c_hi) st_p_chunk(sP, t, c, zero16);
                 float mx = -INFINITY;
                 // score tape: this row's band scores, entry n - t = k + w
-                float* ts = p.tape != nullptr && mrow < Lr ? p.tape + (rowbase + (int64_t)mrow * p.dil) * p.tstride : nullptr;
+                float* ts = TAPE && mrow < Lr ? p.tape + (rowbase + (int64_t)mrow * p.dil) * p.tstride : nullptr;
                 for (int c = c_lo; c <= c_hi; ++c) {
                     uint32_t rr[32];
                     tmem_ld32(trow + c * 32, rr);
@@ -804,11 +806,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 
 int tape_stride(int64_t wc);
 
-template <int MODE>
+template <int MODE, bool TAPE>
 void set_attr_once() {
     static std::once_flag once;
     std::call_once(once, [] {
-        cudaFuncSetAttribute(tc_band_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaFuncSetAttribute(tc_band_kernel<MODE, TAPE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              227 * 1024);
     });
 }
@@ -845,7 +847,8 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
     const int64_t nres = dil < L ? dil : L;
     const int nst = pick_nst<MODE>(NK);
     if (nst < 2) return cudaErrorInvalidConfiguration;
-    set_attr_once<MODE>();
+    set_attr_once<MODE, false>();
+    set_attr_once<MODE, true>();
     int n = 0;
     for (int64_t r0 = 0; r0 < nres; r0 += RES_PER_LAUNCH) {
         Params p;
@@ -898,9 +901,10 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
             at[0].val.programmaticStreamSerializationAllowed = 1;
             cfg.attrs = at;
             cfg.numAttrs = 1;
-            cudaLaunchKernelEx(&cfg, tc_band_kernel<MODE>, p);
+            cudaLaunchKernelEx(&cfg, tape ? tc_band_kernel<MODE, true> : tc_band_kernel<MODE, false>, p);
         } else {
-            tc_band_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
+            if (tape) tc_band_kernel<MODE, true><<<grid, NTHREADS, smem, st>>>(p);
+            else tc_band_kernel<MODE, false><<<grid, NTHREADS, smem, st>>>(p);
         }
         prof_mark(st);
         cudaError_t e = cudaGetLastError();

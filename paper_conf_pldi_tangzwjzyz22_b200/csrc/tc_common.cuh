@@ -77,12 +77,38 @@ __device__ __forceinline__ uint64_t global_ns() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+// The timer is read only once a wait has polled 4096 times, so handoffs on the critical path
+// never pay for it.
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    if (mbar_try_wait(bar, parity)) return;
-    const uint64_t t0 = global_ns();
     uint32_t spins = 0;
+    uint64_t t0 = 0;
     while (!mbar_try_wait(bar, parity)) {
-        if ((++spins & 255u) == 0 && global_ns() - t0 > FT_WATCHDOG_NS) __trap();
+        if (++spins < 4096u || (spins & 255u) != 0) continue;
+        const uint64_t now = global_ns();
+        if (t0 == 0) t0 = now;
+        else if (now - t0 > FT_WATCHDOG_NS) __trap();
+    }
+}
+
+// Always-suspending wait (a suspend-time hint even where FT_MBAR_SUSPEND_NS is 0): for a warp
+// that would otherwise spin for thousands of cycles on an SM sub-partition another role needs
+// (the narrow backward's softmax waiting for the converter warps' scale table).
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
+    uint32_t ok = 0, spins = 0;
+    uint64_t t0 = 0;
+    for (;;) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(ok)
+            : "r"(smem_u32(bar)), "r"(parity), "r"(0x989680u)
+            : "memory");
+        if (ok) return;
+        if (++spins < 4096u || (spins & 255u) != 0) continue;
+        const uint64_t now = global_ns();
+        if (t0 == 0) t0 = now;
+        else if (now - t0 > FT_WATCHDOG_NS) __trap();
     }
 }
 
@@ -101,11 +127,13 @@ __device__ __forceinline__ bool mbar_try_wait_spin(uint64_t* bar, uint32_t parit
     return ok != 0;
 }
 __device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
-    if (mbar_try_wait_spin(bar, parity)) return;
-    const uint64_t t0 = global_ns();
     uint32_t spins = 0;
+    uint64_t t0 = 0;
     while (!mbar_try_wait_spin(bar, parity)) {
-        if ((++spins & 1023u) == 0 && global_ns() - t0 > FT_WATCHDOG_NS) __trap();
+        if (++spins < 65536u || (spins & 1023u) != 0) continue;
+        const uint64_t now = global_ns();
+        if (t0 == 0) t0 = now;
+        else if (now - t0 > FT_WATCHDOG_NS) __trap();
     }
 }
 

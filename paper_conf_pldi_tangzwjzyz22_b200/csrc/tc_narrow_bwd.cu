@@ -48,9 +48,6 @@
 #include <mutex>
 
 #include "internal.h"
-#ifndef FT_MBAR_SUSPEND_NS
-#define FT_MBAR_SUSPEND_NS 0   // latency-critical handoffs: no suspend-time hint
-#endif
 #include "tc_common.cuh"
 #include "tile_sched.cuh"
 #include "tmap.h"
@@ -66,7 +63,7 @@ constexpr int BM = 128;
 constexpr int D = 64;
 constexpr int NK = 192;
 constexpr int NSTAGE = 2;
-constexpr int NTHREADS = 352;
+constexpr int NTHREADS = 384;   // + converter warps 10, 11
 constexpr int RES_PER_LAUNCH = 8;
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t ABYTES = BM * D * 2;      // 16 KB: a 128-row tile
@@ -192,7 +189,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
     uint64_t* acc_full = s_full + 3;        // [2]
     uint64_t* acc_free = s_full + 5;        // [2]
     uint64_t* hs_full = s_full + 7;         // [2] halo row scales of tile j published
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 9);
+    uint64_t* s_full2 = s_full + 9;         // [2] S and dP of tile j done, for the converters (which
+                                            // may lag the softmax by a tile: a single-phase barrier
+                                            // would let its parity wrap)
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 11);
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int w = p.w;
@@ -206,11 +206,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             }
             mbar_init(s_full, 1);
             mbar_init(dp_free, 8);
-            mbar_init(p_done, 8 + 1);
+            mbar_init(p_done, 8 + 2);
             for (int b = 0; b < 2; ++b) {
                 mbar_init(&acc_full[b], 1);
                 mbar_init(&acc_free[b], 8);
-                mbar_init(&hs_full[b], 32);
+                mbar_init(&hs_full[b], 64);
+                mbar_init(&s_full2[b], 1);
             }
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
@@ -246,53 +247,64 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 tma_load_3d(st + 2 * ABYTES + HBYTES, &mp.b2, &full2[s], 0, T.m0 - w, T.u);
             }
         }
-    } else if (warp == 10) {   // ------------------------------------------ halo converter
-        // the halo of the dS GEMM (NQ: K_h, NKV: Q_h) to fp16 in place, once the score GEMM
-        // has read it as bf16 (s_full): pass 1 finds each row's largest |value| and publishes
-        // 2^-f (hs_full), pass 2 writes the row times 2^f as fp16; the output MMAs read it
-        // after p_done.  Lane l owns halo rows l, l + 32, ...
+    } else if (warp == 10 || warp == 11) {   // ----------------------------- halo converters
+        // the halo of the dS GEMM (NQ: K_h, NKV: Q_h) to fp16 in place.  Lane l of converter warp
+        // cw owns halo rows 64 i + 32 cw + l, i < 3 (whole 128-byte rows: no shuffles, no second
+        // read).  As soon as the TMA landed it loads its rows into registers, reduces each row's
+        // largest |value| and publishes 2^-f (hs_full); once the score GEMM has read the bf16 halo
+        // (s_full2) it writes the rows times 2^f as fp16; the output MMAs read them after p_done.
+        // (Two passes over shared memory, or eight lanes per row with shuffle reductions, left
+        // this warp pair on the tile's critical path: tools/trace_narrow.py.)
+        const int cw = warp - 10;
+        constexpr int NR = NK / 64;     // rows per lane
         TileCursor cur(p.sc);
         Tile T;
         for (int j = 0; cur.next(p.sc, T); ++j) {
-            mbar_wait(s_full, j & 1);
-            if (lane == 0) trace_ev(p, j, 14);
+            mbar_wait(&full1[j % NSTAGE], (j / NSTAGE) & 1);
+            if (lane == 0 && cw == 0) trace_ev(p, j, 14);
             uint8_t* hb = stages + (size_t)(j % NSTAGE) * STAGE + 2 * ABYTES;
             float* tab = hscale + (j & 1) * NK;
-            float sc[NK / 32];
+            uint4 v[NR][8];
+            float sc[NR];
 #pragma unroll
-            for (int q = 0; q < NK / 32; ++q) {
-                const uint4* row = reinterpret_cast<const uint4*>(hb + (lane + 32 * q) * 128);
+            for (int i = 0; i < NR; ++i) {
+                const int r = 64 * i + 32 * cw + lane;
+#pragma unroll
+                for (int x = 0; x < 8; ++x)
+                    v[i][x] = *reinterpret_cast<const uint4*>(hb + r * 128 + ((x ^ (r & 7)) << 4));
+            }
+#pragma unroll
+            for (int i = 0; i < NR; ++i) {
                 uint32_t m = 0;
 #pragma unroll
-                for (int g = 0; g < 8; ++g) {
-                    const uint4 v4 = row[g];
-                    m = __vmaxu2(m, __vmaxu2(__vmaxu2(v4.x & 0x7FFF7FFFu, v4.y & 0x7FFF7FFFu),
-                                             __vmaxu2(v4.z & 0x7FFF7FFFu, v4.w & 0x7FFF7FFFu)));
-                }
-                m = max(m & 0xFFFFu, m >> 16);                  // bf16 bits of the row's max |x|
+                for (int x = 0; x < 8; ++x)
+                    m = __vmaxu2(m, __vmaxu2(__vmaxu2(v[i][x].x & 0x7FFF7FFFu, v[i][x].y & 0x7FFF7FFFu),
+                                             __vmaxu2(v[i][x].z & 0x7FFF7FFFu, v[i][x].w & 0x7FFF7FFFu)));
+                m = max(m & 0xFFFFu, m >> 16);   // bf16 bits of the row's max |x|
                 const int f = m == 0 ? 0 : pow2_exp_fp16(int(m >> 7));
-                sc[q] = __uint_as_float((uint32_t)(127 + f) << 23);
-                tab[lane + 32 * q] = __uint_as_float((uint32_t)(127 - f) << 23);
+                sc[i] = __uint_as_float((uint32_t)(127 + f) << 23);
+                tab[64 * i + 32 * cw + lane] = __uint_as_float((uint32_t)(127 - f) << 23);
             }
             mbar_arrive(&hs_full[j & 1]);   // every lane releases its own table entries
+            if (lane == 0 && cw == 0) trace_ev(p, j, 17);
+            mbar_wait(&s_full2[j & 1], (j >> 1) & 1);   // the score GEMM has read the bf16 halo
 #pragma unroll
-            for (int q = 0; q < NK / 32; ++q) {
-                uint4* row = reinterpret_cast<uint4*>(hb + (lane + 32 * q) * 128);
+            for (int i = 0; i < NR; ++i) {
+                const int r = 64 * i + 32 * cw + lane;
 #pragma unroll
-                for (int g = 0; g < 8; ++g) {
-                    uint4 v4 = row[g];
-                    uint32_t* wv = reinterpret_cast<uint32_t*>(&v4);
+                for (int x = 0; x < 8; ++x) {
+                    uint32_t* wv = reinterpret_cast<uint32_t*>(&v[i][x]);
 #pragma unroll
-                    for (int x = 0; x < 4; ++x) {
-                        const float2 f2 = __bfloat1622float2(*reinterpret_cast<__nv_bfloat162*>(&wv[x]));
-                        wv[x] = pack_f16x2(f2.x * sc[q], f2.y * sc[q]);
+                    for (int y = 0; y < 4; ++y) {
+                        const float2 f2 = __bfloat1622float2(*reinterpret_cast<__nv_bfloat162*>(&wv[y]));
+                        wv[y] = pack_f16x2(f2.x * sc[i], f2.y * sc[i]);
                     }
-                    row[g] = v4;
+                    *reinterpret_cast<uint4*>(hb + r * 128 + ((x ^ (r & 7)) << 4)) = v[i][x];
                 }
             }
             fence_proxy_async_smem();
             warp_arrive(p_done);
-            if (lane == 0) trace_ev(p, j, 12);
+            if (lane == 0 && cw == 0) trace_ev(p, j, 12);
         }
     } else if (warp == 9) {
         if (lane == 0) {   // ------------------------------------------------------ MMA issuer
@@ -352,6 +364,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 mma_ss_x4<2, 2>(rP, sdesc_sw128(st + ABYTES, 16, 1024),
                                 sdesc_sw128(st + 2 * ABYTES + HBYTES, 16, 1024), idS, 0);
                 mma_commit(s_full);
+                mma_commit(&s_full2[j & 1]);
                 trace_ev(p, j, 3);
                 if (p.trace && j < 8) {   // debug only: when did the score GEMMs complete?
                     mbar_wait(s_full, j & 1);
@@ -539,7 +552,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 if (tr) trace_ev(p, j, 7);
                 const float Dv = dxb[t] + dxb[BM + t];
                 // dS' = P (dP - D) 2^-f_c (halo row scales), then this row's power of two
-                mbar_wait(&hs_full[j & 1], (j >> 1) & 1);
+                mbar_wait_sleep(&hs_full[j & 1], (j >> 1) & 1);
                 const float* tab = hscale + (j & 1) * NK + c0;
                 float mx = 0.f;
 #pragma unroll
@@ -569,7 +582,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             } else {
                 const float4* cL = reinterpret_cast<const float4*>(cl + c0);
                 const float4* cD = reinterpret_cast<const float4*>(cl + NK + c0);
-                mbar_wait(&hs_full[j & 1], (j >> 1) & 1);
+                mbar_wait_sleep(&hs_full[j & 1], (j >> 1) & 1);
                 const float* tab = hscale + (j & 1) * NK + c0;   // 2^-f of the Q_h rows (columns)
                 float mx = 0.f;
 #pragma unroll

@@ -20,7 +20,7 @@ import paper_conf_pldi_tangzwjzyz22_b200 as ft  # noqa: E402
 
 EV = ["mma iter start", "S(j) issued", "out(j-1) issued", "dP(j) issued", "sm s_full seen",
       "sm S/dP loaded", "sm operand buf free", "sm pair barrier", "sm p_done", "sm acc seen",
-      "sm drained", "prod loads issued", "halo converted", "mma sees s_full", "conv sees s_full", "sm setup done", "sm acc loaded"]
+      "sm drained", "prod loads issued", "halo converted", "mma sees s_full", "conv sees s_full", "sm setup done", "sm acc loaded", "conv table published"]
 
 
 def main():
@@ -47,8 +47,8 @@ def main():
     for m, name in ((1, "NQ"), (2, "NKV")):
         t = bufs[m].view(148, 8, 48).cpu().double()
         base = t[:, :, 0:1]
-        rel = t[:, 1:, :17] - base[:, 1:]
-        ok = (t[:, 1:, :17] > 0).all(dim=2)
+        rel = t[:, 1:, :len(EV)] - base[:, 1:]
+        ok = (t[:, 1:, :len(EV)] > 0).all(dim=2)
         print(f"== {name}")
         for e, nm in enumerate(EV):
             print(f"  {nm:22s} {float(rel[:, :, e][ok].median()):7.0f} clk")
@@ -57,7 +57,7 @@ def main():
                 t0 = t[c, 1, 0]
                 print(f"  CTA {c} raw (clk from tile 1 start):")
                 for jj in range(1, 8):
-                    print("   tile", jj, " ".join(f"{int(t[c, jj, e] - t0):6d}" for e in range(17)))
+                    print("   tile", jj, " ".join(f"{int(t[c, jj, e] - t0):6d}" for e in range(len(EV))))
         per = t[:, 2:, 0] - t[:, 1:-1, 0]
         print(f"  tile period            {float(per[(t[:, 2:, 0] > 0) & (t[:, 1:-1, 0] > 0)].median()):7.0f} clk")
 
