@@ -500,14 +500,25 @@ def main():
     krows.update({f"bwd{i}": r for i, (_, r) in enumerate(ltb)})
     mean_k = {n: sum(x) / len(x) for n, x in kdur.items()}
     dom = max(mean_k, key=mean_k.get)
-    rows_per_launch = krows[dom]
+    # The roofline is taken over the direction (forward or backward) whose launches take the most
+    # time, with SURVEY.md §8(d)'s algorithmic bytes of that direction -- fwd 4de + 4, bwd 8de + 4
+    # per row -- over the sum of its launches' CUDA-event durations.  (Round 1 booked the dominant
+    # launch's own I/O, e.g. the dK/dV kernel's 6de + 8, which flattered it.)  per_kernel adds each
+    # launch's own-I/O figure for detail.
+    t_dir = {"fwd": sum(v for n, v in mean_k.items() if n.startswith("fwd")),
+             "bwd": sum(v for n, v in mean_k.items() if n.startswith("bwd"))}
+    ddir = max(t_dir, key=t_dir.get)
+    per_kernel = {n: {"kind": kinds[n], "ms": mean_k[n],
+                      "own_io_gbs": kernel_bytes_per_row(kinds[n], d, e) * krows[n] / (mean_k[n] / 1e3) / 1e9}
+                  for n in mean_k}
     if path_b == ft.PATH_TC:   # tensor-core kernels (bf16, or fp32 as bf16 hi / lo planes): HBM bound
-        by = kernel_bytes_per_row(kinds[dom], d, e) * rows_per_launch
-        ach = by / (mean_k[dom] / 1e3) / 1e9
+        by = ((4 if ddir == "fwd" else 8) * d * e + 4) * rows
+        ach = by / (t_dir[ddir] / 1e3) / 1e9
         roof = {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
-                "frac": ach / hbm_peak, "traffic": None, "kernel": dom,
-                "kernel_kind": kinds[dom], "ms_per_launch": mean_k[dom],
-                "algorithmic_bytes_per_launch": by, "peak_source": peak_src}
+                "frac": ach / hbm_peak, "traffic": None, "kernel": f"{ddir} ({', '.join(n for n in mean_k if n.startswith(ddir))})",
+                "ms_per_launch": t_dir[ddir], "algorithmic_bytes_per_launch": by,
+                "algorithmic_bytes_rule": "SURVEY.md §8(d): fwd 4de+4, bwd 8de+4 per row",
+                "peak_source": peak_src, "per_kernel": per_kernel}
     else:
         nsum = float(window_sizes(L, w, dil).sum()) * B * H
         fl = {"fwd": 4, "bwdA": 6, "bwdB": 8}[kinds[dom]] * d * nsum
@@ -520,10 +531,18 @@ def main():
     tr_path = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tr_path):
         try:
-            tr = json.load(open(tr_path)).get(f"{args.workload}/{args.dtype}/{kinds[dom]}")
-            if tr:
-                roof["traffic"] = tr["bytes_per_launch"]
-                roof["traffic_source"] = tr.get("source")
+            trj = json.load(open(tr_path))
+            if path_b == ft.PATH_TC:   # DRAM bytes of the direction's launches (ncu --set full)
+                names = [n for n in mean_k if n.startswith(ddir)]
+                trs = [trj.get(f"{args.workload}/{args.dtype}/{kinds[n]}") for n in names]
+                if trs and all(trs):
+                    roof["traffic"] = sum(t["bytes_per_launch"] for t in trs)
+                    roof["traffic_source"] = trs[0].get("source")
+            else:
+                tr = trj.get(f"{args.workload}/{args.dtype}/{kinds[dom]}")
+                if tr:
+                    roof["traffic"] = tr["bytes_per_launch"]
+                    roof["traffic_source"] = tr.get("source")
         except Exception:
             pass
     step_alg = step_bytes_per_row(d, e) * rows * world
