@@ -199,9 +199,12 @@ ft_status ft_winattn_debug_trace(int kernel_mode, void* device_buffer);
  *   3 FT_KNOB_WIDE    1 the w > 64 wide kernels, 0 the chunked fallback  [FT_WINATTN_WIDE=0]
  *   4 FT_KNOB_SIDE    1 per-head-dilation calls use a side stream, 0 serial
  *                                                                [FT_WINATTN_MIXED_SERIAL=1]
+ *   5 FT_KNOB_DSTAPE  1 the fp32 tensor-core dK/dV kernel reads P and dS from the dQ kernel's
+ *                     tape (in the workspace), 0 it recomputes them  [FT_WINATTN_DSTAPE=0]
  * ft_winattn_debug_set returns FT_ERR_INVALID_VALUE for an unknown knob or value;
  * ft_winattn_debug_get returns the current value (-1 for an unknown knob). */
-enum { FT_KNOB_PATH = 0, FT_KNOB_PDL = 1, FT_KNOB_NARROW = 2, FT_KNOB_WIDE = 3, FT_KNOB_SIDE = 4 };
+enum { FT_KNOB_PATH = 0, FT_KNOB_PDL = 1, FT_KNOB_NARROW = 2, FT_KNOB_WIDE = 3, FT_KNOB_SIDE = 4,
+       FT_KNOB_DSTAPE = 5 };
 ft_status ft_winattn_debug_set(int knob, int value);
 int       ft_winattn_debug_get(int knob);
 

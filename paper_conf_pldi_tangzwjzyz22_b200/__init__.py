@@ -93,7 +93,7 @@ def load_library(build_if_missing: bool = False):
     return lib
 
 
-_KNOBS = {"path": 0, "pdl": 1, "narrow": 2, "wide": 3, "side": 4}
+_KNOBS = {"path": 0, "pdl": 1, "narrow": 2, "wide": 3, "side": 4, "dstape": 5}
 _PATHS = {"auto": 0, "simt": 1, "tc": 2}
 
 

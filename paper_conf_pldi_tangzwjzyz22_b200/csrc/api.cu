@@ -66,6 +66,7 @@ void knob_init() {
         g_knob[ftw::K_NARROW] = env_int("FT_WINATTN_NARROW", 1) != 0;
         g_knob[ftw::K_WIDE] = env_int("FT_WINATTN_WIDE", 1) != 0;
         g_knob[ftw::K_SIDE] = env_int("FT_WINATTN_MIXED_SERIAL", 0) != 1;
+        g_knob[ftw::K_DSTAPE] = env_int("FT_WINATTN_DSTAPE", 1) != 0;
     });
 }
 thread_local bool g_handoff = false;   // inside ft_winattn_fwd_bwd
@@ -86,6 +87,30 @@ ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w
     }
     *path = tc_ok ? FT_PATH_TC : FT_PATH_SIMT;
     return FT_OK;
+}
+
+// Backward workspace: D_i = dout_i . out_i per row (fp32), and -- for shapes the fp32 tensor-core
+// kernels serve -- the dS tape between the dQ and dK/dV kernels (ftw::DsTape): one flag word per
+// row and two fp32 planes of tsw floats per row.  Each region is 256-byte aligned; a slice of rows
+// [row0, ...) (per-head-dilation calls) uses the same offsets into every region.
+struct WsLayout {
+    size_t dB = 0, fB = 0, pB = 0;
+    int tsw = 0;
+    bool tape = false;
+    size_t total() const { return dB + fB + 2 * pB; }
+};
+size_t round256(size_t x) { return (x + 255) / 256 * 256; }
+WsLayout ws_layout(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, ft_dtype dt) {
+    WsLayout l;
+    const size_t rows = (size_t)(B * H * L);
+    l.dB = round256(rows * sizeof(float));
+    l.tape = dt == FT_F32 && ftw::tc32_supported(B * H, L, d, w, dil);
+    if (l.tape) {
+        l.tsw = ftw::dstape_tsw(w < L ? w : L);
+        l.fB = round256(rows * sizeof(uint32_t));
+        l.pB = round256(rows * (size_t)l.tsw * sizeof(float));
+    }
+    return l;
 }
 
 }  // namespace
@@ -150,9 +175,7 @@ const char* ft_status_str(ft_status s) {
 size_t ft_winattn_bwd_workspace_bytes(int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
                                       int64_t w, int64_t dilation, ft_dtype dtype) {
     if (check_scalars(batch, heads, seq_len, d, w, dilation, dtype) != FT_OK) return 0;
-    // D_i = dout_i . out_i for every row, fp32, rounded up to 256 bytes.
-    const size_t rows = (size_t)(batch * heads * seq_len);
-    return ((rows * sizeof(float) + 255) / 256) * 256;
+    return ws_layout(batch, heads, seq_len, d, w, dilation, dtype).total();
 }
 
 ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
@@ -273,21 +296,34 @@ ft_status check_bwd(const void* q, const void* k, const void* v, const void* out
     return choose_path(1, batch * heads, seq_len, d, w, dilation, dtype, &path);
 }
 
+// Enqueue a validated backward.  ws: the workspace of a call whose layout is `lay`; this backward
+// covers its rows [row0, row0 + batch * heads * seq_len).
 ft_status run_bwd(const void* q, const void* k, const void* v, const void* out, const float* lse,
                   const void* dout, void* dq, void* dk, void* dv, int64_t batch, int64_t heads,
                   int64_t seq_len, int64_t d, int64_t w, int64_t dilation, ft_dtype dtype,
-                  void* workspace, void* stream) {
+                  void* ws, const WsLayout& lay, int64_t row0, void* stream) {
     int path = 0;
     ft_status s = choose_path(1, batch * heads, seq_len, d, w, dilation, dtype, &path);
     if (s != FT_OK) return s;
     cudaStream_t st = (cudaStream_t)stream;
-    float* Dws = (float*)workspace;
+    char* base = static_cast<char*>(ws);
+    float* Dws = base ? (float*)(base + row0 * 4) : nullptr;
     cudaError_t e;
     bind_context();
     clear_stale_error();
     if (path == FT_PATH_TC && dtype == FT_F32) {
         int n = 0;
-        e = ftw::tc32_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w, dilation, st, &n);
+        ftw::DsTape tape;
+        const bool use_tape = lay.tape && base && ftw::knob(ftw::K_DSTAPE) && ftw::dstape_pays(d) &&
+                              ftw::tc32_supported(batch * heads, seq_len, d, w, dilation);
+        if (use_tape) {
+            tape.flags = (uint32_t*)(base + lay.dB + row0 * 4);
+            tape.P = (float*)(base + lay.dB + lay.fB + (size_t)row0 * lay.tsw * 4);
+            tape.S = (float*)(base + lay.dB + lay.fB + lay.pB + (size_t)row0 * lay.tsw * 4);
+            tape.tsw = lay.tsw;
+        }
+        e = ftw::tc32_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, use_tape ? &tape : nullptr, batch, heads,
+                          seq_len, d, w, dilation, st, &n);
     } else if (path == FT_PATH_TC) {
         int n = 0;
         e = ftw::tc_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w,
@@ -401,7 +437,7 @@ ft_status ft_winattn_bwd(const void* q, const void* k, const void* v, const void
     if (s != FT_OK) return s;
     ftw::prof_reset();
     return run_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, dilation, dtype,
-                   workspace, stream);
+                   workspace, ws_layout(batch, heads, seq_len, d, w, dilation, dtype), 0, stream);
 }
 
 ft_status ft_winattn_fwd_mixed(const void* q, const void* k, const void* v, void* out, float* lse,
@@ -448,6 +484,7 @@ ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v, cons
     const int ng = mixed_groups(heads, dilation, dilated_heads, g);
     const size_t e = elt_size(dtype);
     const int64_t nb = ng == 1 ? 1 : batch;
+    const WsLayout lay = ws_layout(batch, heads, seq_len, d, w, dilation, dtype);
     ftw::prof_reset();
     ForkJoin fj((cudaStream_t)stream, (int)(nb * ng));
     for (int64_t b = 0; b < nb; ++b) {
@@ -455,10 +492,10 @@ ft_status ft_winattn_bwd_mixed(const void* q, const void* k, const void* v, cons
             const int64_t B1 = ng == 1 ? batch : 1, H1 = ng == 1 ? heads : g[i].nh;
             const int64_t row0 = (b * heads + g[i].h0) * seq_len;
             const size_t off = (size_t)row0 * d * e;
-            // the workspace holds one fp32 per row: the slice's rows start at row0
+            // every workspace region is per row: the slice's rows start at row0
             s = run_bwd((const char*)q + off, (const char*)k + off, (const char*)v + off, (const char*)out + off,
                         lse + row0, (const char*)dout + off, (char*)dq + off, (char*)dk + off, (char*)dv + off,
-                        B1, H1, seq_len, d, w, g[i].dil, dtype, workspace ? (char*)workspace + row0 * 4 : nullptr,
+                        B1, H1, seq_len, d, w, g[i].dil, dtype, workspace, lay, row0,
                         fj.stream_of((int)(b * ng + i)));
             if (s != FT_OK) return fj.finish(s);
         }
@@ -558,7 +595,7 @@ ft_status ft_winattn_fwd_bwd(const void* q, const void* k, const void* v, const 
     s = run_fwd(q, k, v, out, lse, batch, heads, seq_len, d, w, dilation, dtype, stream);
     if (s == FT_OK)
         s = run_bwd(q, k, v, out, lse, dout, dq, dk, dv, batch, heads, seq_len, d, w, dilation, dtype,
-                    workspace, stream);
+                    workspace, ws_layout(batch, heads, seq_len, d, w, dilation, dtype), 0, stream);
     g_handoff = false;
     return s;
 }

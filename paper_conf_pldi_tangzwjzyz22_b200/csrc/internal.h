@@ -110,9 +110,25 @@ int tc32_fwd_launches(int64_t L, int64_t dil);
 int tc32_bwd_launches(int64_t L, int64_t dil);
 cudaError_t tc32_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B, int64_t H,
                      int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches);
+// The dS tape between the two backward kernels (selective materialization): the
+// dQ kernel stores every band entry's P_ij and dS_ij (fp32, row i of plane P / S holds entry
+// e = j - i + w at float offset (m & 3) + e, m = i's row in its residue, rows tsw floats apart)
+// and publishes flags[first row of each 128-row tile] = 1; the dK/dV kernel then reads its
+// P^T / dS^T from the tape instead of recomputing S^T and dP^T.  Workspace layout: api.cu.
+struct DsTape {
+    uint32_t* flags;   // one word per row (only tile-first rows used)
+    float* P;          // [rows][tsw]
+    float* S;          // [rows][tsw]
+    int tsw;
+};
+inline int dstape_tsw(int64_t wc) { return (int)((2 * wc + 4 + 3) / 4 * 4); }
+// The tape costs 2 tsw floats per row written and read; it replaces the dK/dV kernel's score phase
+// (K, V, Q, dO slices, two GEMMs, the operand conversion).  Measured (tools/tape_ablation.py,
+// DESIGN.md §10): slower at d = 64, even at d = 128, 1.1-1.26x faster at d >= 256.
+inline bool dstape_pays(int64_t d) { return d >= 256; }
 cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const float* lse, const void* dout, void* dq,
-                     void* dk, void* dv, float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
-                     int64_t dil, cudaStream_t st, int* launches);
+                     void* dk, void* dv, float* Dws, const DsTape* tape, int64_t B, int64_t H, int64_t L,
+                     int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches);
 
 // Score tape on the band kernels (bf16, w <= 64, d % 64 == 0): the forward also writes the band
 // scores (fp32 [rows][2w + 1], the CUDA-core kernels' format), the backward reads them and skips
@@ -136,7 +152,8 @@ enum Knob {
     K_NARROW = 2,   // 1: d = 64, w <= 32 narrow kernels; 0: band kernels (FT_WINATTN_NARROW=0)
     K_WIDE = 3,     // 1: w > 64 wide kernels; 0: the chunked fallback kernels (FT_WINATTN_WIDE=0)
     K_SIDE = 4,     // 1: per-head-dilation calls use a side stream; 0: serial (FT_WINATTN_MIXED_SERIAL=1)
-    K_NUM = 5
+    K_DSTAPE = 5,   // 1: fp32 tensor-core backward hands P / dS over on a tape; 0: recompute (FT_WINATTN_DSTAPE=0)
+    K_NUM = 6
 };
 int knob(Knob k);
 

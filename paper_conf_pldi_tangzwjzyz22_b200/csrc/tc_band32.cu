@@ -81,6 +81,7 @@ constexpr float LN2 = 0.6931471805599453f;
 // rows KB); o1/o2: outputs (box rows 32).  All fp32, 32-column SWIZZLE_128B boxes.
 struct Maps {
     CUtensorMap a1, b1, a2, b2, ob1, ob2, o1, o2;
+    CUtensorMap tp, ts;   // BWDKV with the dS tape: the P / dS planes, 64-row boxes
 };
 struct Params {
     Maps maps[RES_PER_LAUNCH];
@@ -90,6 +91,12 @@ struct Params {
     int d, w, dil, NK, nsl;
     SchedParams sc;
     int dpoll;    // BWDKV: poll D row by row (BWDQ marked its rows D_UNSET, PDL launch)
+    // dS tape (ftw::DsTape, internal.h): BWDQ stores P and dS of every band entry and sets the
+    // flag of each tile it finished; BWDKV (xt) loads them instead of recomputing S^T and dP^T.
+    int xt, tsw;
+    uint32_t* flags;
+    float* tP;
+    float* tS;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace), see trace32()
 };
 
@@ -201,6 +208,17 @@ struct Seq {
     static constexpr int NOUT = MODE == BWDKV ? 2 : 1;
 };
 
+// use counts of the three accumulator regions (registers, no dynamic indexing)
+struct AccUses {
+    int u0 = 0, u1 = 0, u2 = 0;
+    __device__ __forceinline__ int get(int r) const { return r == 0 ? u0 : r == 1 ? u1 : u2; }
+    __device__ __forceinline__ void inc(int r) {
+        if (r == 0) ++u0;
+        else if (r == 1) ++u1;
+        else ++u2;
+    }
+};
+
 template <int MODE>
 __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_constant__ Params p) {
     using C = Seq<MODE>;
@@ -213,7 +231,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     const int ncw = (d + CW - 1) / CW;      // output chunks per tensor (the last may be 64 wide)
     const int nacc = ncw * C::NOUT;         // accumulations per tile
 
-    if (MODE == BWDQ && p.dpoll) {   // mark this CTA's D rows unset before BWDKV may launch
+    if (MODE == BWDQ && p.xt) {   // clear this CTA's tile flags before BWDKV may launch
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T))
+            if (threadIdx.x == 0) p.flags[(int64_t)T.u * p.L + T.r + (int64_t)T.m0 * p.dil] = 0u;
+        __threadfence();
+        __syncthreads();
+    } else if (MODE == BWDQ && p.dpoll) {   // mark this CTA's D rows unset before BWDKV may launch
         TileCursor cr(p.sc);
         Tile T;
         while (cr.next(p.sc, T)) {
@@ -238,9 +263,26 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     uint64_t* empty = bars + 2 * NST;  // [NST] MMAs done with the slot
     uint64_t* s_full = bars + 3 * NST; // [2] score GEMMs of a tile done (FWD: region j & 1)
     uint64_t* p_full = s_full + 2;     // [2] softmax wrote the MMA operands of a tile (4 warps)
-    uint64_t* o_full = s_full + 4;     // accumulation done
-    uint64_t* o_empty = s_full + 5;    // accumulator drained (4 epilogue warps)
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 6);
+    uint64_t* o_full = s_full + 4;     // [3] accumulation done, per accumulator region (acc_rid)
+    uint64_t* o_empty = s_full + 7;    // [3] accumulator drained (4 epilogue warps)
+    // xt: [0] R1 free (the tile's last dK accumulation in R1 drained), [1] R0 free (last dV one in
+    // R0): one phase per tile each, so the softmax warps never lag two phases behind (o_empty
+    // completes u0 times per tile and is waited only by the MMA issuer, use by use)
+    uint64_t* xfree = s_full + 10;
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 12);
+    // Accumulator of accumulation a: RACC, except in BWDKV with the dS tape, where the dV (dK)
+    // chunks alternate between R0 (R1) and RACC, ending on RACC: during dV R1 holds the A operand
+    // P^T and R0 is free (dS^T is built into it after the last R0 drain), during dK R0 holds dS^T
+    // and R1 is free -- so an accumulation runs while the epilogue drains the previous one.
+    const bool xt = MODE == BWDKV && p.xt;
+    auto acc_rid = [&](int a) -> int {
+        if (!xt || ((ncw - 1 - a % ncw) & 1) == 0) return 0;
+        return a < ncw ? 1 : 2;
+    };
+    // (the R1 accumulator sits at column 256, 128-aligned like the others)
+    auto acc_col = [](int rid) -> uint32_t { return rid == 0 ? RACC : rid == 1 ? R0 : R1 + 64; };
+    const int npl = (NK + 127) / 128;   // tape slots per plane (128 rows each)
+    // (with ncw >= 2, the host's condition for xt, the last R0 / R1 accumulation is chunk ncw - 2)
 
     if (warp == 8) {
         if (lane == 0) {
@@ -253,8 +295,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 mbar_init(&s_full[i], 1);
                 mbar_init(&p_full[i], 4);
             }
-            mbar_init(o_full, 1);
-            mbar_init(o_empty, 4);
+            for (int i = 0; i < 3; ++i) {
+                mbar_init(&o_full[i], 1);
+                mbar_init(&o_empty[i], 4);
+            }
+            mbar_init(&xfree[0], 4);
+            mbar_init(&xfree[1], 4);
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
                 const Maps& mp = p.maps[i];
@@ -294,6 +340,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             }
         } else {
             while (co.next(p.sc, To)) {
+                if (xt) {   // P plane (slots of 128 tape rows), dV; dS plane, dK
+                    for (int h = 0; h < 2; ++h) {
+                        for (int b = 0; b < npl; ++b) fn(2, To, b, h);
+                        for (int a = h * ncw; a < (h + 1) * ncw; ++a)
+                            for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
+                    }
+                    continue;
+                }
                 for (int s = 0; s < nsl; ++s) {
                     fn(0, To, s, 0);
                     fn(0, To, s, 1);
@@ -313,7 +367,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 trace_slot(p, k++, 0);
                 uint8_t* sp = slots + (size_t)st * SLOT;
                 const Maps& mp = p.maps[T.rl];
-                if (kind == 0) {   // 32 columns: two 16-column boxes of each operand
+                if (kind == 2) {   // dS tape: query rows [128 a, 128 a + 128) of plane b (P, dS)
+                    if (a == 0 && b == 0 && p.dpoll) {   // BWDQ may still run: wait for these rows' tiles
+                        const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+                        const int lo = max(0, T.m0 - w) / BM, hi = min(T.Lr - 1, T.m0 + BM - 1 + w) / BM;
+                        for (int tq = lo; tq <= hi; ++tq) wait_flag(p.flags + rowbase + (int64_t)tq * BM * p.dil);
+                        asm volatile("fence.proxy.async.global;" ::: "memory");
+                    }
+                    const uint32_t box = 64u * (uint32_t)p.tsw * 4u;   // 64 rows
+                    const int nbx = NK - 128 * a > 64 ? 2 : 1;
+                    mbar_arrive_expect_tx(&full[st], nbx * box);
+                    for (int x = 0; x < nbx; ++x)
+                        tma_load_3d(sp + x * box, b ? &mp.ts : &mp.tp, &full[st], 0, T.m0 - w + 128 * a + 64 * x, T.u);
+                } else if (kind == 0) {   // 32 columns: two 16-column boxes of each operand
                     const CUtensorMap* ma = b ? &mp.a2 : &mp.a1;
                     const CUtensorMap* mb = b ? &mp.b2 : &mp.b1;
                     mbar_arrive_expect_tx(&full[st], (uint32_t)(2 * BM + 2 * NK) * 64u);
@@ -340,7 +406,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             mbar_wait(&full[st], ph);
             if (ct == 0) trace_slot(p, k, 1);
             uint8_t* sp = slots + (size_t)st * SLOT;
-            if (kind == 0) {
+            if (kind == 2) {
+                // tape slot: read as fp32 by the softmax warps (arrive only, keeping the phases)
+            } else if (kind == 0) {
                 convert_rows2<64>(sp, BM, sp + 2 * BM * 64, NK, ct);
             } else {
                 const bool full_chunk = chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW;
@@ -357,13 +425,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             const uint32_t idS = idesc_bf16(BM, NK, false, false);
             const uint32_t idO = idesc_bf16(BM, CW, false, true);
             const uint32_t idO64 = idesc_bf16(BM, 64, false, true);   // a 64-column last chunk
-            int st = 0, ga = 0, k = 0;
+            int st = 0, k = 0;
+            AccUses uses;   // accumulations per region so far
             uint32_t ph = 0;
             int jg = 0;          // score GEMMs: tile counter
             int jo = 0;          // output GEMMs: tile counter
             walk([&](int kind, const Tile&, int a, int b) {
                 const uint32_t sa = smem_u32(slots + (size_t)st * SLOT);
-                if (kind == 0) {
+                if (kind == 2) {   // tape slot: no MMA (the softmax warps free it)
+                    mbar_wait(&conv[st], ph);
+                } else if (kind == 0) {
                     // FWD: S(jg) into region jg & 1; BWD: S into R0, dP into R1
                     const uint32_t dst = tbase + (MODE == FWD ? ((jg & 1) ? R1 : R0) : (b ? R1 : R0));
                     if (MODE != FWD && a == 0 && b == 0 && jg > 0) {
@@ -392,14 +463,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 } else {
                     // output block b of accumulation a of tile jo.  A: packed hi | lo operand in TMEM
                     // (FWD: P over S(jo); BWDQ: dS over S; BWDKV: P^T over dP^T (dV), dS^T over S^T (dK))
-                    if (a == 0 && b == 0) {
-                        mbar_wait(&p_full[jo & 1], (jo >> 1) & 1);
+                    if (b == 0 && (a == 0 || (xt && a == ncw))) {   // xt: P^T (dV), dS^T (dK) built
+                        if (xt) mbar_wait(&p_full[a == 0 ? 0 : 1], (uint32_t)jo & 1u);
+                        else mbar_wait(&p_full[jo & 1], (jo >> 1) & 1);
                         tc_fence_after();
                     }
-                    if (b == 0 && ga > 0) {
-                        mbar_wait(o_empty, (ga - 1) & 1);
+                    const int rid = acc_rid(a);
+                    if (b == 0 && uses.get(rid) > 0) {
+                        mbar_wait(&o_empty[rid], (uint32_t)(uses.get(rid) - 1) & 1u);
                         tc_fence_after();
                     }
+                    const uint32_t Dacc = tbase + acc_col(rid);
                     const uint32_t Areg = tbase + (MODE == FWD ? ((jo & 1) ? R1 : R0)
                                                    : (MODE == BWDKV && a < ncw) ? R1 : R0);
                     const uint32_t id = chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW ? idO : idO64;
@@ -412,14 +486,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         const uint32_t tA = Areg + 16u * g;   // hi words; lo words at + 8
                         const uint64_t dbh = sdesc_sw128(sa + kk * 2048, 2 * KB * 128, 1024);
                         const uint64_t dbl = sdesc_sw128(sa + KB * 128 + kk * 2048, 2 * KB * 128, 1024);
-                        mma_ts(tbase + RACC, tA, dbh, id, g != 0);
-                        mma_ts(tbase + RACC, tA, dbl, id, 1);
-                        mma_ts(tbase + RACC, tA + 8, dbh, id, 1);
+                        mma_ts(Dacc, tA, dbh, id, g != 0);
+                        mma_ts(Dacc, tA, dbl, id, 1);
+                        mma_ts(Dacc, tA + 8, dbh, id, 1);
                     }
                     mma_commit(&empty[st]);
                     if (b == nkb - 1) {
-                        mma_commit(o_full);
-                        ++ga;
+                        mma_commit(&o_full[rid]);
+                        uses.inc(rid);
                         if (a == nacc - 1) ++jo;
                     }
                 }
@@ -442,7 +516,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         while (cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t, kb = m0 - w;
             const int64_t rowbase = (int64_t)T.u * p.L + T.r;
-            if (MODE == BWDKV) {
+            if (MODE == BWDKV && !p.xt) {
                 named_bar_sync(1, 128);   // everyone is done with the previous tile's columns
                 for (int n = t; n < NK; n += 128) {
                     const int mc = kb + n;
@@ -456,8 +530,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             }
             const int sidx = MODE == FWD ? (j & 1) : 0;
             const uint32_t sph = MODE == FWD ? ((j >> 1) & 1) : (j & 1);
-            mbar_wait(&s_full[sidx], sph);
-            tc_fence_after();
+            if (!xt) {
+                mbar_wait(&s_full[sidx], sph);
+                tc_fence_after();
+            }
             if (t == 0) trace_tile(p, j, 0);
             const uint32_t rS = tbase + lane_off + (MODE == FWD && (j & 1) ? R1 : R0);
             const uint32_t rP = tbase + lane_off + R1;
@@ -541,16 +617,26 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tmem_ld16(rS + n0, rs);
                         tmem_ld16(rP + n0, rd);
                         tmem_wait_ld();
+                        // tape entry e = n - t of row mrow sits at float (mrow & 3) + e = ob + (n - n0):
+                        // four entries per 16-byte store ((mrow & 3) == (t & 3), m0 % 128 == 0)
+                        const int ob = (t & 3) + n0 - t;
 #pragma unroll
-                        for (int e = 0; e < 16; e += 2) {
-                            float dv[2];
+                        for (int g4 = 0; g4 < 4; ++g4) {
+                            float pv[4], dv[4];
 #pragma unroll
-                            for (int h = 0; h < 2; ++h) {
-                                const int n = n0 + e + h;
-                                const float pv = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -lse2)) : 0.f;
-                                dv[h] = pv * (__uint_as_float(rd[e + h]) - D);
+                            for (int x = 0; x < 4; ++x) {
+                                const int n = n0 + 4 * g4 + x;
+                                pv[x] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[4 * g4 + x]), LOG2E, -lse2)) : 0.f;
+                                dv[x] = pv[x] * (__uint_as_float(rd[4 * g4 + x]) - D);
                             }
-                            split2(dv[0], dv[1], pk[e / 2], pl[e / 2]);
+                            split2(dv[0], dv[1], pk[2 * g4], pl[2 * g4]);
+                            split2(dv[2], dv[3], pk[2 * g4 + 1], pl[2 * g4 + 1]);
+                            const int o = ob + 4 * g4;
+                            if (p.xt && mrow < Lr && o >= 0 && o < p.tsw) {
+                                const size_t ro = (size_t)(rowbase + (int64_t)mrow * p.dil) * p.tsw + o;
+                                *reinterpret_cast<float4*>(p.tP + ro) = make_float4(pv[0], pv[1], pv[2], pv[3]);
+                                *reinterpret_cast<float4*>(p.tS + ro) = make_float4(dv[0], dv[1], dv[2], dv[3]);
+                            }
                         }
                         tmem_st8(rS + n0, pk);
                         tmem_st8(rS + n0 + 8, pl);
@@ -560,6 +646,57 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 tc_fence_before();
                 warp_arrive(&p_full[j & 1]);
                 if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
+                if (p.xt) {   // publish the tile's tape rows to BWDKV
+                    __threadfence();
+                    named_bar_sync(2, 128);
+                    if (t == 0) st_release_gpu(p.flags + rowbase + (int64_t)m0 * p.dil, 1u);
+                }
+            } else if (xt) {   // BWDKV from the dS tape: P^T -> R1 (hi | lo), then dS^T -> R0
+                const int per = 2 * npl + nacc * nkb;
+                for (int h = 0; h < 2; ++h) {
+                    // R1 once the previous tile's dK accumulations in it are drained; R0 once this
+                    // tile's dV accumulations in it are (the MMAs that read them as A came earlier)
+                    if (h == 1) mbar_wait(&xfree[1], (uint32_t)j & 1u);
+                    else if (j > 0) mbar_wait(&xfree[0], (uint32_t)(j - 1) & 1u);
+                    tc_fence_after();
+                    const uint32_t dst = h == 0 ? rP : rS;
+                    for (int b = 0; b < npl; ++b) {
+                        const int k = j * per + (h ? npl + ncw * nkb : 0) + b, st = k % NST;
+                        mbar_wait(&full[st], (uint32_t)(k / NST) & 1u);
+                        const float* sv = reinterpret_cast<const float*>(slots + (size_t)st * SLOT);
+                        for (int c = 4 * b; c < 4 * b + 4 && c < nch; ++c) {
+                            if (c < c_lo || c > c_hi) {
+                                tmem_st16(dst + c * 32, zero16);
+                                tmem_st16(dst + c * 32 + 16, zero16);
+                                continue;
+                            }
+#pragma unroll
+                            for (int hh = 0; hh < 2; ++hh) {
+                                const int n0 = c * 32 + 16 * hh;
+                                uint32_t pk[8], pl[8];
+#pragma unroll
+                                for (int e = 0; e < 16; e += 2) {
+                                    float x[2];
+#pragma unroll
+                                    for (int hx = 0; hx < 2; ++hx) {
+                                        // query column n (tape row kb + n), key t: entry t - n + 2w
+                                        const int n = n0 + e + hx, mq = kb + n;
+                                        x[hx] = band_ok(n, t, w, mq, Lr)
+                                                    ? sv[(n - 128 * b) * p.tsw + (mq & 3) + t - n + 2 * w] : 0.f;
+                                    }
+                                    split2(x[0], x[1], pk[e / 2], pl[e / 2]);
+                                }
+                                tmem_st8(dst + n0, pk);
+                                tmem_st8(dst + n0 + 8, pl);
+                            }
+                        }
+                        named_bar_sync(1, 128);   // all four warps are done with this slot
+                        if (t == 0) mbar_arrive(&empty[st]);
+                    }
+                    tmem_wait_st();
+                    tc_fence_before();
+                    warp_arrive(&p_full[h]);
+                }
             } else {   // BWDKV: rows are keys, columns halo queries
                 for (int c = 0; c < nch; ++c) {
                     if (c < c_lo || c > c_hi) {
@@ -602,11 +739,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         }
     } else if (warp < 8) {   // ----------------------------------------------- epilogue warps
         const int ew = warp - 4;   // TMEM lanes 32 ew ..
-        const uint32_t trow = tbase + ((uint32_t)(ew * 32) << 16) + RACC;
+        const uint32_t tlane = tbase + ((uint32_t)(ew * 32) << 16);
         uint8_t* mystg = stg + ew * NSTG * STG;
         TileCursor cur(p.sc);
         Tile T;
-        int j = 0, ga = 0, sidx = 0;
+        int j = 0, sidx = 0;
+        AccUses uses;
         while (cur.next(p.sc, T)) {
             const Maps& mp = p.maps[T.rl];
             float scale = 1.f;
@@ -614,11 +752,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 mbar_wait(&p_full[j & 1], (j >> 1) & 1);
                 scale = rowScale[(j % 3) * 128 + ew * 32 + lane];
             }
-            for (int a = 0; a < nacc; ++a, ++ga) {
+            for (int a = 0; a < nacc; ++a) {
                 const int c = C::NOUT == 2 ? a % ncw : a;
                 const CUtensorMap* om = (C::NOUT == 2 && a < ncw) ? &mp.o2 : &mp.o1;   // BWDKV: dV first
                 const int ngrp = chunk_w(d, c) / 32;
-                mbar_wait(o_full, ga & 1);
+                const int rid = acc_rid(a);
+                const uint32_t trow = tlane + acc_col(rid);
+                mbar_wait(&o_full[rid], (uint32_t)uses.get(rid) & 1u);
+                uses.inc(rid);
                 tc_fence_after();
                 if (ew == 0 && lane == 0) trace_tile(p, j, 2 + a);
                 // two rounds of 64 columns (register budget of 16 warps); the accumulator is
@@ -631,7 +772,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     tmem_wait_ld();
                     if (x == ngrp - 1) {
                         tc_fence_before();
-                        warp_arrive(o_empty);
+                        warp_arrive(&o_empty[rid]);
+                        if (xt && a % ncw == ncw - 2) warp_arrive(&xfree[a < ncw ? 1 : 0]);
                     }
                     uint8_t* sb = mystg + (sidx % NSTG) * STG;
                     if (lane == 0 && sidx >= NSTG) tma_store_wait_read<NSTG - 1>();
@@ -685,8 +827,8 @@ int halo_rows32(int64_t L, int64_t w) {
 
 template <int MODE>
 cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void* b2, const void* ob1,
-                     const void* ob2, void* o1, void* o2, float* lse, float* D, int64_t B, int64_t H,
-                     int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
+                     const void* ob2, void* o1, void* o2, float* lse, float* D, const DsTape* tape, int64_t B,
+                     int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
     static std::once_flag once;
     std::call_once(once, [] {
         cudaFuncSetAttribute(tc_band32_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES);
@@ -711,6 +853,10 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
             if (ok && b2) ok = make_residue_map_f32(&m.b2, b2, L, d, units, dil, r, NK, 16);
             if (ok && ob2) ok = make_residue_map_f32(&m.ob2, ob2, L, d, units, dil, r, KB);
             if (ok && o2) ok = make_residue_map_f32(&m.o2, o2, L, d, units, dil, r, 32);
+            if (ok && tape && MODE == BWDKV && d > CW) {
+                ok = make_residue_map_tape(&m.tp, tape->P, L, tape->tsw, units, dil, r, 64) &&
+                     make_residue_map_tape(&m.ts, tape->S, L, tape->tsw, units, dil, r, 64);
+            }
             if (!ok) return cudaErrorInvalidValue;
         }
         p.lse = lse;
@@ -722,6 +868,13 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         p.NK = NK;
         p.nsl = (int)(d / 32);
         p.dpoll = MODE != FWD && dpoll_enabled();   // BWDQ marks its D rows, BWDKV polls them
+        if (tape && MODE != FWD && d > CW) {   // xt needs two output chunks (acc_rid alternation)
+            p.xt = 1;
+            p.tsw = tape->tsw;
+            p.flags = tape->flags;
+            p.tP = tape->P;
+            p.tS = tape->S;
+        }
         p.trace = (unsigned long long*)trace_buffer(MODE);
         const int64_t Lr0 = ceil_div(L - r0, dil);
         const int tiles = (int)ceil_div(Lr0, BM);
@@ -769,22 +922,24 @@ int tc32_bwd_launches(int64_t L, int64_t dil) { return 2 * band32_launches(L, di
 cudaError_t tc32_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B, int64_t H,
                      int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
     if (launches) *launches = 0;
-    return launch32<FWD>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, B, H, L, d, w, dil, st,
-                         launches);
+    return launch32<FWD>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, nullptr, B, H, L, d, w,
+                         dil, st, launches);
 }
 
 cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const float* lse, const void* dout, void* dq,
-                     void* dk, void* dv, float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
-                     int64_t dil, cudaStream_t st, int* launches) {
+                     void* dk, void* dv, float* Dws, const DsTape* tape, int64_t B, int64_t H, int64_t L,
+                     int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
     if (launches) *launches = 0;
     // BWDQ: S = Q K_h^T (a1 = q, b1 = k), dP = dO V_h^T (a2 = dout, b2 = v), dQ = dS K_h (ob1 = k)
-    cudaError_t e = launch32<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse), Dws, B, H, L,
-                                   d, w, dil, st, launches);
+    cudaError_t e = launch32<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse), Dws, tape, B,
+                                   H, L, d, w, dil, st, launches);
     if (e != cudaSuccess) return e;
     // BWDKV: S^T = K Q_h^T, dP^T = V dO_h^T; dV = P^T dO_h (ob1 = dout -> o2 = dv), dK = dS^T Q_h
     // (ob2 = q -> o1 = dk).  Accumulations: dV chunks (a < ncw, o2), then dK chunks (o1).
-    return launch32<BWDKV>(k, q, v, dout, dout, q, dk, dv, const_cast<float*>(lse), Dws, B, H, L, d, w, dil, st,
-                           launches);
+    // With the dS tape (PAPER.md:489-497 selective materialization) BWDKV skips S^T and dP^T: it
+    // streams only the tape rows and the dO / Q blocks of its output GEMMs.
+    return launch32<BWDKV>(k, q, v, dout, dout, q, dk, dv, const_cast<float*>(lse), Dws, tape, B, H, L, d, w, dil,
+                           st, launches);
 }
 
 }  // namespace ftw

@@ -419,6 +419,23 @@ __device__ __forceinline__ float ld_D_ready(const float* ptr) {
     return __uint_as_float(x);
 }
 
+// Tile flags of the dS tape (tc_band32.cu): the dQ kernel clears them before triggering the dependent
+// launch and releases 1 once a tile's tape rows are stored; the dK/dV kernel acquires them.
+__device__ __forceinline__ void wait_flag(const uint32_t* ptr) {
+    uint32_t x;
+    uint64_t t0 = 0;
+    for (;;) {
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(x) : "l"(ptr) : "memory");
+        if (x != 0u) break;
+        if (t0 == 0) t0 = global_ns();
+        else if (global_ns() - t0 > FT_WATCHDOG_NS) __trap();
+        __nanosleep(256);
+    }
+}
+__device__ __forceinline__ void st_release_gpu(uint32_t* ptr, uint32_t v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(ptr), "r"(v) : "memory");
+}
+
 // one relaxed load (no memory clobber: a thread's loads of a halo issue back to back; the
 // few still D_UNSET are then re-read with ld_D_ready)
 __device__ __forceinline__ float ld_D_first(const float* ptr) {

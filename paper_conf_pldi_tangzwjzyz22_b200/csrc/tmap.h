@@ -68,4 +68,22 @@ inline bool make_residue_map_f32(CUtensorMap* m, const void* tensor, int64_t L, 
     return res == CUDA_SUCCESS;
 }
 
+// Residue view of a dS-tape plane (ftw::DsTape: fp32 rows of tsw floats, one per sequence row), a
+// {tsw x box_rows} box without swizzle (the softmax warps read it with plain shared loads).
+inline bool make_residue_map_tape(CUtensorMap* m, const void* plane, int64_t L, int64_t tsw,
+                                  int64_t units, int64_t dil, int64_t r, int box_rows) {
+    auto enc = tmap_encoder();
+    if (!enc) return false;
+    const int64_t Lr = (L - r + dil - 1) / dil;
+    const char* base = static_cast<const char*>(plane) + r * tsw * 4;
+    cuuint64_t dims[3] = {(cuuint64_t)tsw, (cuuint64_t)Lr, (cuuint64_t)units};
+    cuuint64_t strides[2] = {(cuuint64_t)(dil * tsw * 4), (cuuint64_t)(L * tsw * 4)};
+    cuuint32_t box[3] = {(cuuint32_t)tsw, (cuuint32_t)box_rows, 1u};
+    cuuint32_t estr[3] = {1u, 1u, 1u};
+    CUresult res = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<char*>(base), dims,
+                       strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return res == CUDA_SUCCESS;
+}
+
 }  // namespace ftw

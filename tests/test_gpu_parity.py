@@ -144,6 +144,22 @@ def test_tc32_parity(ft, shape):
     run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=16)
 
 
+# The dS tape between the fp32 backward kernels (FT_KNOB_DSTAPE): the dK/dV kernel
+# reads P and dS from the dQ kernel instead of recomputing them, with the per-tile flag hand-off
+# (PDL on) or plain stream order (PDL off); many tiles per CTA, ragged residues, several launches
+# of residues (dilation > 8), w = 0.
+# (d >= 256: where the library uses the tape; d = 320 has a 64-wide last output chunk.)
+DSTAPE = [(1, 4, 3000, 256, 32, 1), (2, 3, 1001, 256, 5, 3), (1, 1, 700, 512, 32, 1), (1, 2, 2000, 320, 32, 11),
+          (1, 2, 600, 256, 0, 1), (3, 1, 129, 384, 31, 1)]
+
+
+@pytest.mark.parametrize("tape,pdl", [(1, 1), (1, 0), (0, 1)])
+@pytest.mark.parametrize("shape", DSTAPE, ids=lambda s: "x".join(map(str, s)))
+def test_tc32_dstape(ft, shape, tape, pdl):
+    with ft.knobs(dstape=tape, pdl=pdl):
+        run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=21)
+
+
 @pytest.mark.parametrize("seed", [0, 1, 2])
 def test_default_path_seeds(ft, seed):
     run_case(ft, WinAttnShape(1, 2, 384, 64, 32, 1), "bf16", None, seed=seed)

@@ -12,7 +12,11 @@ legs of one family run on the same inputs; one JSON line per case with ms per fw
 events, mean of 20 after 3 warm-ups, L2 flushed between steps) and the tape's extra HBM bytes per
 step (one write + two reads, the dQ and dK/dV kernels each read it).
 
-    python tools/tape_ablation.py [--quick]
+The second table is the dS tape between the two fp32 tensor-core backward kernels
+(FT_KNOB_DSTAPE): the dQ kernel stores P and dS of every band entry and the dK/dV kernel reads them
+instead of recomputing S^T and dP^T (legs: dstape 0 / 1, ms per backward).
+
+    python tools/tape_ablation.py [--quick] [--dstape-only]
 """
 import argparse
 import json
@@ -70,12 +74,35 @@ def run(name, B, H, L, d, w, dil, dt, knobs):
     print(json.dumps(res), flush=True)
 
 
+DS_CASES = [(f"d{d}_w{w}", 1, max(1, 16 * 64 // d), 8192, d, w, 1)
+            for d in (64, 128, 256, 512) for w in (8, 16, 32)] + [("C2a", 8, 1, 10000, 512, 32, 1),
+                                                               ("C5_w32", 64, 1, 32768, 64, 32, 1)]
+
+
+def run_ds(name, B, H, L, d, w, dil):
+    dev = torch.device("cuda:0")
+    q, k, v, g = [torch.rand(B, H, L, d, device=dev) * 2 - 1 for _ in range(4)]
+    out, lse = ft.fwd(q, k, v, w, dil)
+    res = {"case": name, "dtype": "f32", "shape": [B, H, L, d, w, dil], "family": "dS tape (fp32 tensor cores)",
+           "tape_bytes_per_row": 2 * 4 * ((2 * min(w, L) + 4 + 3) // 4 * 4)}
+    for leg in (0, 1):
+        with ft.knobs(dstape=leg):
+            res[["recompute_bwd_ms", "dstape_bwd_ms"][leg]] = timed(lambda: ft.bwd(q, k, v, out, lse, g, w, dil))
+    res["dstape_speedup"] = res["recompute_bwd_ms"] / res["dstape_bwd_ms"]
+    print(json.dumps(res), flush=True)
+
+
 def main():
     global FLUSH
     ap = argparse.ArgumentParser()
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--dstape-only", action="store_true")
     a = ap.parse_args()
     FLUSH = torch.empty(256 << 20, dtype=torch.uint8, device="cuda:0")
+    for c in DS_CASES:
+        run_ds(*c)
+    if a.dstape_only:
+        return
     for c in TC_CASES[-4:] if a.quick else TC_CASES:
         run(*c, torch.bfloat16, {"narrow": 0})
     for c in SIMT_CASES[:1] if a.quick else SIMT_CASES:
