@@ -104,7 +104,8 @@ WsLayout ws_layout(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_
     WsLayout l;
     const size_t rows = (size_t)(B * H * L);
     l.dB = round256(rows * sizeof(float));
-    l.tape = dt == FT_F32 && ftw::tc32_supported(B * H, L, d, w, dil);
+    l.tape = ftw::dstape_pays(d) && (dt == FT_F32 ? ftw::tc32_supported(B * H, L, d, w, dil)
+                                                   : ftw::tc_band_dstape_ok(B * H, L, d, w, dil));
     if (l.tape) {
         l.tsw = ftw::dstape_tsw(w < L ? w : L);
         l.fB = round256(rows * sizeof(uint32_t));
@@ -308,26 +309,28 @@ ft_status run_bwd(const void* q, const void* k, const void* v, const void* out, 
     cudaStream_t st = (cudaStream_t)stream;
     char* base = static_cast<char*>(ws);
     float* Dws = base ? (float*)(base + row0 * 4) : nullptr;
+    // the dS tape regions of these rows (tensor-core families check that they can use it)
+    ftw::DsTape tape;
+    const bool use_tape = lay.tape && base && ftw::knob(ftw::K_DSTAPE);
+    if (use_tape) {
+        tape.flags = (uint32_t*)(base + lay.dB + row0 * 4);
+        tape.P = (float*)(base + lay.dB + lay.fB + (size_t)row0 * lay.tsw * 4);
+        tape.S = (float*)(base + lay.dB + lay.fB + lay.pB + (size_t)row0 * lay.tsw * 4);
+        tape.tsw = lay.tsw;
+    }
     cudaError_t e;
     bind_context();
     clear_stale_error();
     if (path == FT_PATH_TC && dtype == FT_F32) {
         int n = 0;
-        ftw::DsTape tape;
-        const bool use_tape = lay.tape && base && ftw::knob(ftw::K_DSTAPE) && ftw::dstape_pays(d) &&
-                              ftw::tc32_supported(batch * heads, seq_len, d, w, dilation);
-        if (use_tape) {
-            tape.flags = (uint32_t*)(base + lay.dB + row0 * 4);
-            tape.P = (float*)(base + lay.dB + lay.fB + (size_t)row0 * lay.tsw * 4);
-            tape.S = (float*)(base + lay.dB + lay.fB + lay.pB + (size_t)row0 * lay.tsw * 4);
-            tape.tsw = lay.tsw;
-        }
-        e = ftw::tc32_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, use_tape ? &tape : nullptr, batch, heads,
+        const bool ok = ftw::tc32_supported(batch * heads, seq_len, d, w, dilation);
+        e = ftw::tc32_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, use_tape && ok ? &tape : nullptr, batch, heads,
                           seq_len, d, w, dilation, st, &n);
     } else if (path == FT_PATH_TC) {
         int n = 0;
+        const bool ok = ftw::tc_band_dstape_ok(batch * heads, seq_len, d, w, dilation);
         e = ftw::tc_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w,
-                        dilation, st, &n);
+                        dilation, st, &n, use_tape && ok ? &tape : nullptr);
     } else {
         e = ftw::simt_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, batch, heads, seq_len, d, w,
                           dilation, dtype, st);

@@ -41,6 +41,23 @@ inline Geo make_geo(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64
 
 inline int64_t geo_blocks(const Geo& g) { return g.units * g.nres * g.tiles; }
 
+// The dS tape between the two backward kernels (selective materialization),
+// fp32 (tc_band32.cu) and bf16 band (tc_band.cu) tensor-core kernels: the dQ kernel stores every band entry's P_ij and dS_ij (fp32, row i of plane P / S holds entry
+// e = j - i + w at float offset (m & 3) + e, m = i's row in its residue, rows tsw floats apart)
+// and publishes flags[first row of each 128-row tile] = 1; the dK/dV kernel then reads its
+// P^T / dS^T from the tape instead of recomputing S^T and dP^T.  Workspace layout: api.cu.
+struct DsTape {
+    uint32_t* flags;   // one word per row (only tile-first rows used)
+    float* P;          // [rows][tsw]
+    float* S;          // [rows][tsw]
+    int tsw;
+};
+inline int dstape_tsw(int64_t wc) { return (int)((2 * wc + 4 + 3) / 4 * 4); }
+// The tape costs 2 tsw floats per row written and read; it replaces the dK/dV kernel's score phase
+// (K, V, Q, dO slices, two GEMMs, the operand conversion).  Measured (tools/tape_ablation.py,
+// DESIGN.md §10): slower at d = 64, even at d = 128, 1.1-1.26x faster at d >= 256.
+inline bool dstape_pays(int64_t d) { return d >= 256; }
+
 // SIMT (CUDA-core) kernels -- simt.cu
 // tape (optional): the raw band scores s_ij, fp32 [B*H*L][2w+1] (w clamped to L); the forward
 // writes it and the backward reads it instead of recomputing q_i . k_j (ft_winattn_*_tape).
@@ -63,7 +80,9 @@ cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float
 cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
                    const float* lse, const void* dout, void* dq, void* dk, void* dv,
                    float* Dws, int64_t B, int64_t H, int64_t L, int64_t d, int64_t w,
-                   int64_t dil, cudaStream_t st, int* launches);
+                   int64_t dil, cudaStream_t st, int* launches, const DsTape* ds = nullptr);
+// the bf16 backward of this shape runs on the band kernels, which can use the dS tape
+bool tc_band_dstape_ok(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
 int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil);
 int tc_bwd_launches(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
 
@@ -110,22 +129,6 @@ int tc32_fwd_launches(int64_t L, int64_t dil);
 int tc32_bwd_launches(int64_t L, int64_t dil);
 cudaError_t tc32_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B, int64_t H,
                      int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches);
-// The dS tape between the two backward kernels (selective materialization): the
-// dQ kernel stores every band entry's P_ij and dS_ij (fp32, row i of plane P / S holds entry
-// e = j - i + w at float offset (m & 3) + e, m = i's row in its residue, rows tsw floats apart)
-// and publishes flags[first row of each 128-row tile] = 1; the dK/dV kernel then reads its
-// P^T / dS^T from the tape instead of recomputing S^T and dP^T.  Workspace layout: api.cu.
-struct DsTape {
-    uint32_t* flags;   // one word per row (only tile-first rows used)
-    float* P;          // [rows][tsw]
-    float* S;          // [rows][tsw]
-    int tsw;
-};
-inline int dstape_tsw(int64_t wc) { return (int)((2 * wc + 4 + 3) / 4 * 4); }
-// The tape costs 2 tsw floats per row written and read; it replaces the dK/dV kernel's score phase
-// (K, V, Q, dO slices, two GEMMs, the operand conversion).  Measured (tools/tape_ablation.py,
-// DESIGN.md §10): slower at d = 64, even at d = 128, 1.1-1.26x faster at d >= 256.
-inline bool dstape_pays(int64_t d) { return d >= 256; }
 cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const float* lse, const void* dout, void* dq,
                      void* dk, void* dv, float* Dws, const DsTape* tape, int64_t B, int64_t H, int64_t L,
                      int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches);

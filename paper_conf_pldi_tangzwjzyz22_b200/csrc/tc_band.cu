@@ -77,6 +77,7 @@ template <int MODE> struct Cfg {
 // ob1/ob2: output-GEMM B operands (halo, box 64 rows); o1/o2: outputs (box 32 rows).
 struct Maps {
     CUtensorMap a1, b1, a2, b2, ob1, ob2, o1, o2;
+    CUtensorMap tp, ts;   // BWDKV with the dS tape (xt): P / dS planes, boxes of trows rows
 };
 struct Params {
     Maps maps[RES_PER_LAUNCH];
@@ -96,6 +97,13 @@ struct Params {
                                  // read s from it and skip the score GEMM S = Q K^T (selective
                                  // materialization)
     int tstride;                 // tape row stride, elements (2w + 1)
+    // dS tape between BWDQ and BWDKV (ftw::DsTape, internal.h; the fp32 kernels' scheme,
+    // tc_band32.cu): BWDQ stores P and dS of every band entry and releases a flag per tile;
+    // BWDKV (xt) loads them instead of running the S^T and dP^T GEMMs.
+    int xt, tsw, trows;          // trows: tape rows per ring slot (both planes)
+    uint32_t* flags;
+    float* tP;
+    float* tS;
 };
 
 
@@ -216,7 +224,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     // BWDQ CTAs leave (its persistent CTAs finish 4 or 5 tiles apart) and stream their first
     // tiles' q/k/v/dout -- inputs of the whole backward call, complete before BWDQ started --
     // while BWDQ drains; only BWDKV's softmax warps, which read BWDQ's D, wait for it.
-    if (MODE == BWDQ && p.dpoll) {
+    if (MODE == BWDQ && p.xt) {   // clear this CTA's tile flags before BWDKV may launch
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T))
+            if (threadIdx.x == 0) p.flags[(int64_t)T.u * p.L + T.r + (int64_t)T.m0 * p.dil] = 0u;
+        __threadfence();
+        __syncthreads();
+    } else if (MODE == BWDQ && p.dpoll) {
         // mark this CTA's D rows unset before BWDKV may launch (ld_D_ready); the CTA stores
         // the real values of the same rows later, ordered after this by the barrier
         TileCursor cr(p.sc);
@@ -275,7 +290,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     uint64_t* o_empty = s_full + 3;
     uint64_t* p_free = s_full + 4;   // P smem consumed by the tile's output MMAs
     uint64_t* p_blk = s_full + 5;    // [4] BWD: dS of 64-key block b written (per-block handoff)
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 9);
+    uint64_t* a_free = s_full + 9;   // xt: the tile's dK MMAs are done with dS^T in TMEM
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 10);
+    const bool xt = MODE == BWDKV && p.xt;
+    const int ntape = xt ? NK / p.trows : 0;   // tape slots per tile
 
     if (warp == 8) {
         if (lane == 0) {
@@ -288,6 +306,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             mbar_init(o_empty, 128);
             mbar_init(p_free, 1);
             for (int i = 0; i < 4; ++i) mbar_init(&p_blk[i], 128);
+            mbar_init(a_free, 1);
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
                 const Maps& mp = p.maps[i];
@@ -370,7 +389,26 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     }
                     if (hg) { ++jg; hg = cg.next(p.sc, Tg); }
                 } else {   // BWD: G(j) then O(j) (dS lives in the S columns)
-                    for (int s = 0; s < nsl; ++s) load_g_slice(To, jo, s);
+                    if (xt) {   // dS tape: trows query rows of both planes per slot
+                        const Maps& mp = p.maps[To.rl];
+                        if (p.dpoll) {   // BWDQ may still run: wait for the tiles of the halo rows
+                            const int64_t rowbase = (int64_t)To.u * p.L + To.r;
+                            const int lo = max(0, To.m0 - w) / BM, hi = min(To.Lr - 1, To.m0 + BM - 1 + w) / BM;
+                            for (int tq = lo; tq <= hi; ++tq) wait_flag(p.flags + rowbase + (int64_t)tq * BM * p.dil);
+                            asm volatile("fence.proxy.async.global;" ::: "memory");
+                        }
+                        const uint32_t pl = (uint32_t)p.trows * (uint32_t)p.tsw * 4u;
+                        for (int b = 0; b < ntape; ++b) {
+                            uint8_t* sp = take();
+                            if (b == 0) trace_ev(p, jo, 0);
+                            mbar_arrive_expect_tx(&full[st], 2 * pl);
+                            tma_load_3d(sp, &mp.tp, &full[st], 0, To.m0 - w + p.trows * b, To.u);
+                            tma_load_3d(sp + pl, &mp.ts, &full[st], 0, To.m0 - w + p.trows * b, To.u);
+                            adv();
+                        }
+                    }
+                    if (!xt)
+                        for (int s = 0; s < nsl; ++s) load_g_slice(To, jo, s);
                     for (int a = 0; a < nacc; ++a)
                         for (int kb = 0; kb < nkb; ++kb) load_o_block(To, a, kb);
                 }
@@ -495,7 +533,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             }
             while (co.next(p.sc, To)) {
                 jo_cur = jo;
-                if (MODE != FWD) {
+                if (xt) {   // tape slots: wait (phase order), the softmax warps release them
+                    for (int b = 0; b < ntape; ++b) {
+                        mbar_wait(&full[st], ph);
+                        if (b == 0 && h == 0) trace_ev(p, jo, 2);
+                        if (++st == NST) { st = 0; ph ^= 1u; }
+                    }
+                    if (h == 0) trace_ev(p, jo, 3);
+                } else if (MODE != FWD) {
                     // the score GEMMs write dP into the accumulator columns (unless early):
                     // the epilogue must have drained the previous tile's last accumulation
                     if (!early && ga > 0) {
@@ -524,6 +569,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         for (int kb = 0; kb < nkb; ++kb) o_block(a, kb);
                 }
                 if (C::PSMEM && ownSmemA) mma_commit(p_free);
+                if (xt && ownTmemA) mma_commit(a_free);
                 if (h == otr) trace_ev(p, jo, 5);
                 ++jo;
             }
@@ -551,7 +597,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             const int kb = m0 - w;   // residue index of halo column 0
             const int64_t rowbase = (int64_t)T.u * p.L + T.r;
 
-            if (MODE == BWDKV) {
+            if (MODE == BWDKV && !xt) {
                 named_bar_sync(1, 128);   // everyone is done with the previous tile's columns
                 for (int n = t; n < NK; n += 128) {
                     const int mc = kb + n;
@@ -574,8 +620,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 }
                 named_bar_sync(1, 128);
             }
-            mbar_wait(s_full, j & 1);
-            tc_fence_after();
+            if (!xt) {
+                mbar_wait(s_full, j & 1);
+                tc_fence_after();
+            }
             if (t == 0) trace_ev(p, j, 6);
 
             if (MODE == FWD) {
@@ -654,18 +702,28 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     if (!tp) tmem_ld32(trow + c * 32, rs);
                     tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
+                    // dS tape (xt): entry e = n - t of row mrow at float (mrow & 3) + e = ob + (n - 32 c),
+                    // four entries per 16-byte store ((mrow & 3) == (t & 3), m0 % 128 == 0)
+                    const int ob = (t & 3) + c * 32 - t;
 #pragma unroll
-                    for (int e = 0; e < 32; e += 2) {
-                        float dv[2];
+                    for (int g4 = 0; g4 < 8; ++g4) {
+                        float pv[4], dv[4];
 #pragma unroll
-                        for (int h = 0; h < 2; ++h) {
-                            const int n = c * 32 + e + h;
+                        for (int x = 0; x < 4; ++x) {
+                            const int n = c * 32 + 4 * g4 + x;
                             const bool ok = band_ok(n, t, w, kb + n, Lr);
-                            const float pv = tp ? (ok && tq ? tape_p(n) : 0.f)
-                                                : (ok ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -lse2)) : 0.f);
-                            dv[h] = pv * (__uint_as_float(rd[e + h]) - D);
+                            pv[x] = tp ? (ok && tq ? tape_p(n) : 0.f)
+                                       : (ok ? fast_exp2(fmaf(__uint_as_float(rs[4 * g4 + x]), LOG2E, -lse2)) : 0.f);
+                            dv[x] = pv[x] * (__uint_as_float(rd[4 * g4 + x]) - D);
                         }
-                        split_bf16x2(dv[0], dv[1], pk[e / 2], pl[e / 2]);
+                        split_bf16x2(dv[0], dv[1], pk[2 * g4], pl[2 * g4]);
+                        split_bf16x2(dv[2], dv[3], pk[2 * g4 + 1], pl[2 * g4 + 1]);
+                        const int o = ob + 4 * g4;
+                        if (!TAPE && p.xt && mrow < Lr && o >= 0 && o < p.tsw) {
+                            const size_t ro = (size_t)(rowbase + (int64_t)mrow * p.dil) * p.tsw + o;
+                            *reinterpret_cast<float4*>(p.tP + ro) = make_float4(pv[0], pv[1], pv[2], pv[3]);
+                            *reinterpret_cast<float4*>(p.tS + ro) = make_float4(dv[0], dv[1], dv[2], dv[3]);
+                        }
                     }
                     tmem_st16(trow + c * 32, pk);
                     tmem_st16(trow + c * 32 + 16, pl);
@@ -675,6 +733,65 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                 tc_fence_before();
                 mbar_arrive(p_full);
                 if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
+                if (!TAPE && p.xt) {   // publish the tile's tape rows to BWDKV
+                    __threadfence();
+                    named_bar_sync(2, 128);
+                    if (t == 0) st_release_gpu(p.flags + rowbase + (int64_t)m0 * p.dil, 1u);
+                }
+            } else if (xt) {   // BWDKV from the dS tape: P^T -> smem (bf16), dS^T -> TMEM (hi / lo)
+                if (j > 0) {   // the previous tile's dV / dK MMAs are done with P^T / dS^T
+                    mbar_wait(p_free, (j - 1) & 1);
+                    mbar_wait(a_free, (j - 1) & 1);
+                    tc_fence_after();
+                }
+                if (t == 0) trace_ev(p, j, 10);
+                const int per = ntape + nacc * nkb, cps = p.trows / 32;
+                for (int b = 0; b < ntape; ++b) {
+                    const int k = j * per + b, st = k % NST;
+                    mbar_wait(&full[st], (uint32_t)(k / NST) & 1u);
+                    if (t == 0) trace_ev(p, j, b == 0 ? 11 : 15);
+                    const float* sv = reinterpret_cast<const float*>(sslots + (size_t)st * SLOT);
+                    const float* sS = sv + p.trows * p.tsw;
+                    for (int c = b * cps; c < (b + 1) * cps; ++c) {
+                        if (c < c_lo || c > c_hi) {
+                            if (j == 0) st_p_chunk(sP, t, c, zero16);   // P^T zeros persist
+                            tmem_st16(trow + c * 32, zero16);
+                            tmem_st16(trow + c * 32 + 16, zero16);
+                            continue;
+                        }
+                        uint32_t pk[16], dk[16], dl[16];
+#pragma unroll
+                        for (int e = 0; e < 32; e += 2) {
+                            float pv[2], dv[2];
+#pragma unroll
+                            for (int h = 0; h < 2; ++h) {
+                                // query column n (tape row kb + n), key t: entry t - n + 2w
+                                const int n = c * 32 + e + h, mq = kb + n;
+                                // branch-free (all loads of a chunk issue back to back): an entry
+                                // outside the band reads offset 0 of the slot and is zeroed
+                                const bool ok = band_ok(n, t, w, mq, Lr);
+                                const int o = ok ? (n - b * p.trows) * p.tsw + (mq & 3) + t - n + 2 * w : 0;
+                                const float xp = sv[o], xs = sS[o];
+                                pv[h] = ok ? xp : 0.f;
+                                dv[h] = ok ? xs : 0.f;
+                            }
+                            pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
+                            split_bf16x2(dv[0], dv[1], dk[e / 2], dl[e / 2]);
+                        }
+                        st_p_chunk(sP, t, c, pk);
+                        tmem_st16(trow + c * 32, dk);
+                        tmem_st16(trow + c * 32 + 16, dl);
+                    }
+                    named_bar_sync(1, 128);   // all four warps are done with this slot
+                    if (t == 0) {
+                        mbar_arrive(&empty[st]);
+                        if (p.two) mbar_arrive(&empty[st]);
+                    }
+                }
+                fence_proxy_async_smem();
+                tmem_wait_st();
+                tc_fence_before();
+                mbar_arrive(p_full);
             } else {   // BWDKV: rows are keys, columns are halo queries
                 if (j > 0) mbar_wait(p_free, (j - 1) & 1);
                 for (int c = 0; c < nch; ++c) {
@@ -840,7 +957,7 @@ template <int MODE>
 cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b2, const void* ob1,
                    const void* ob2, void* o1, void* o2, float* lse, float* D, int64_t B, int64_t H,
                    int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches,
-                   float* tape = nullptr) {
+                   float* tape = nullptr, const DsTape* ds = nullptr) {
     const int64_t wc = w < L ? w : L;
     const int NK = halo_rows(L, w);
     const int64_t units = B * H;
@@ -865,6 +982,11 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
             if (ok && b2) ok = make_residue_map(&m.b2, b2, L, d, units, dil, r, NK);
             if (ok && ob2) ok = make_residue_map(&m.ob2, ob2, L, d, units, dil, r, KB);
             if (ok && o2) ok = make_residue_map(&m.o2, o2, L, d, units, dil, r, 32);
+            if (ok && ds && !tape && MODE == BWDKV) {
+                const int trows = 64u * (uint32_t)ds->tsw * 8u <= slot_bytes(NK) ? 64 : 32;
+                ok = make_residue_map_tape(&m.tp, ds->P, L, ds->tsw, units, dil, r, trows) &&
+                     make_residue_map_tape(&m.ts, ds->S, L, ds->tsw, units, dil, r, trows);
+            }
             if (!ok) return cudaErrorInvalidValue;
         }
         p.lse = lse;
@@ -885,6 +1007,14 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         p.lsepoll = lsepoll_enabled() && r0 == 0 && lsepoll_worth(total, num_sms()) && tape == nullptr;
         p.tape = tape;
         p.tstride = tape_stride(wc);
+        if (ds && !tape && MODE != FWD) {
+            p.xt = 1;
+            p.tsw = ds->tsw;
+            p.trows = 64u * (uint32_t)ds->tsw * 8u <= slot_bytes(NK) ? 64 : 32;
+            p.flags = ds->flags;
+            p.tP = ds->P;
+            p.tS = ds->S;
+        }
         dim3 grid((unsigned)(total < num_sms() ? total : num_sms()));
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         const size_t smem = fixed_smem_bytes<MODE>(NK) + (size_t)nst * slot_bytes(NK);
@@ -964,10 +1094,15 @@ cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float
                        d, w, dil, st, launches);
 }
 
+bool tc_band_dstape_ok(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    return halo_rows(L, w) <= 256 && !tc_narrow_bwd_supported(units, L, d, w, dil) &&
+           band_supported(units, L, d, w, dil);
+}
+
 cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
                    const float* lse, const void* dout, void* dq, void* dk, void* dv, float* Dws,
                    int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil,
-                   cudaStream_t st, int* launches) {
+                   cudaStream_t st, int* launches, const DsTape* ds) {
     // band kernels: D_i is recomputed exactly as sum_j P_ij dP_ij by BWDQ (reading R1); the
     // wide kernels also compute it exactly, and read out only for the first-guess D~
     if (launches) *launches = 0;
@@ -979,11 +1114,11 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
     if (tc_narrow_bwd_supported(B * H, L, d, w, dil))
         return tc_narrow_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     cudaError_t e = launch<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse),
-                                 Dws, B, H, L, d, w, dil, st, launches);
+                                 Dws, B, H, L, d, w, dil, st, launches, nullptr, ds);
     if (e != cudaSuccess) return e;
     // BWDKV accumulation order per chunk: dV (P^T dO, ob1 = dout) then dK (dS^T Q, ob2 = q)
     return launch<BWDKV>(k, q, v, dout, dout, q, dv, dk, const_cast<float*>(lse), Dws, B, H, L,
-                         d, w, dil, st, launches);
+                         d, w, dil, st, launches, nullptr, ds);
 }
 
 bool tc_tape_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {

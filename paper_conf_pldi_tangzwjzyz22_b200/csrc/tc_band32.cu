@@ -67,6 +67,11 @@ constexpr int KB = 64;                    // keys per output block
 constexpr int CW = 128;                   // output columns per accumulation
 constexpr int NST = 4;                    // ring slots
 constexpr uint32_t SLOT = 40 * 1024;      // fp32 score slice (128 + 192 rows x 32 cols) / 64 x 128 block
+// BWDKV with the dS tape streams no score slices: five smaller slots (a 128-row tape plane slice,
+// tsw <= 68, or a 32 KB output block), so the tape slots of the next operand and a whole output
+// chunk's key blocks fit in the ring together
+constexpr int NST_XT = 5;
+constexpr uint32_t SLOT_XT = 128 * 68 * 4;
 constexpr uint32_t STG = 32 * 128;        // one epilogue warp's 32-row x 32-col fp32 staging box
 constexpr int NSTG = 2;                   // staging boxes per epilogue warp
 constexpr int NTHREADS = 512;
@@ -102,19 +107,21 @@ struct Params {
 
 // Phase trace (profiling only): per CTA, clock64 stamps of its first TR_SLOTS slots --
 // [0] producer issued the TMA, [1] converter started, [2] converter done, [3] MMA issue start,
-// [4] MMA issue end -- and of its first TR_TILES tiles at [TR_SLOTS * 5 + tile * 8 + e]:
+// [4] MMA issue end -- and of its first TR_TILES tiles at [TR_SLOTS * 5 + tile * 16 + e]:
 // 0 softmax s_full seen, 1 softmax p_full arrived, 2.. epilogue o_full seen per accumulation.
-constexpr int TR_SLOTS = 96, TR_TILES = 4, TR_PER_CTA = TR_SLOTS * 5 + TR_TILES * 8;
+constexpr int TR_SLOTS = 96, TR_TILES = 4, TR_PER_CTA = TR_SLOTS * 5 + TR_TILES * 16;
 __device__ __forceinline__ void trace_slot(const Params& p, int k, int e) {
     if (p.trace && k < TR_SLOTS) p.trace[(size_t)blockIdx.x * TR_PER_CTA + k * 5 + e] = clock64();
 }
 __device__ __forceinline__ void trace_tile(const Params& p, int j, int e) {
-    if (p.trace && j < TR_TILES && e < 8) p.trace[(size_t)blockIdx.x * TR_PER_CTA + TR_SLOTS * 5 + j * 8 + e] = clock64();
+    if (p.trace && j < TR_TILES && e < 16) p.trace[(size_t)blockIdx.x * TR_PER_CTA + TR_SLOTS * 5 + j * 16 + e] = clock64();
 }
 
 constexpr size_t SCRATCH = 3 * 128 * 4 + 2 * 192 * 4;   // FWD row 1/l [3][128]; BWDKV column lse / D
 constexpr size_t SMEM_BYTES = 1024 + NST * SLOT + 4 * NSTG * STG + SCRATCH + 256;
-static_assert(SMEM_BYTES <= 227 * 1024, "shared memory plan");
+constexpr size_t SMEM_BYTES_XT = 1024 + NST_XT * SLOT_XT + 4 * NSTG * STG + SCRATCH + 256;
+static_assert(SMEM_BYTES <= 227 * 1024 && SMEM_BYTES_XT <= 227 * 1024, "shared memory plan");
+static_assert(3 * NST_XT * 8 + 12 * 8 + 4 <= 256, "barrier area");
 
 using Tile = SchedTile;
 using TileCursor = SchedCursor<BM>;
@@ -251,17 +258,20 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     }
     if (MODE == BWDQ) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 
+    const bool xt = MODE == BWDKV && p.xt;
+    const int nst = xt ? NST_XT : NST;
+    const uint32_t slotb = xt ? SLOT_XT : SLOT;
     uint8_t* slots = smem;
-    uint8_t* stg = smem + NST * SLOT;                                   // [4 warps][NSTG] fp32 boxes
+    uint8_t* stg = smem + nst * slotb;                                  // [4 warps][NSTG] fp32 boxes
     float* scratch = reinterpret_cast<float*>(stg + 4 * NSTG * STG);
     float* rowScale = scratch;                                          // FWD [3][128]
     float* colLse = scratch + 3 * 128;                                  // BWDKV [192] lse * log2e
     float* colD = colLse + 192;                                         // BWDKV [192]
     uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(scratch) + SCRATCH);
-    uint64_t* full = bars;             // [NST] TMA bytes landed
-    uint64_t* conv = bars + NST;       // [NST] planes written (4 converter warps)
-    uint64_t* empty = bars + 2 * NST;  // [NST] MMAs done with the slot
-    uint64_t* s_full = bars + 3 * NST; // [2] score GEMMs of a tile done (FWD: region j & 1)
+    uint64_t* full = bars;                // [nst] TMA bytes landed
+    uint64_t* conv = bars + NST_XT;       // [nst] planes written (4 converter warps)
+    uint64_t* empty = bars + 2 * NST_XT;  // [nst] MMAs done with the slot
+    uint64_t* s_full = bars + 3 * NST_XT; // [2] score GEMMs of a tile done (FWD: region j & 1)
     uint64_t* p_full = s_full + 2;     // [2] softmax wrote the MMA operands of a tile (4 warps)
     uint64_t* o_full = s_full + 4;     // [3] accumulation done, per accumulator region (acc_rid)
     uint64_t* o_empty = s_full + 7;    // [3] accumulator drained (4 epilogue warps)
@@ -274,7 +284,6 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     // chunks alternate between R0 (R1) and RACC, ending on RACC: during dV R1 holds the A operand
     // P^T and R0 is free (dS^T is built into it after the last R0 drain), during dK R0 holds dS^T
     // and R1 is free -- so an accumulation runs while the epilogue drains the previous one.
-    const bool xt = MODE == BWDKV && p.xt;
     auto acc_rid = [&](int a) -> int {
         if (!xt || ((ncw - 1 - a % ncw) & 1) == 0) return 0;
         return a < ncw ? 1 : 2;
@@ -286,7 +295,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
 
     if (warp == 8) {
         if (lane == 0) {
-            for (int i = 0; i < NST; ++i) {
+            for (int i = 0; i < nst; ++i) {
                 mbar_init(&full[i], 1);
                 mbar_init(&conv[i], NCONV);
                 mbar_init(&empty[i], 1);
@@ -338,16 +347,32 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 for (int a = 0; a < nacc; ++a)
                     for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
             }
+        } else if (xt) {
+            // Tape slots (npl of 128 rows per plane) sit one output chunk ahead of their use, so
+            // an operand is built while the last chunk of the other output accumulates:
+            //   P(0); per tile j: dV c0 .. c[ncw-2], dS(j), dV c[ncw-1], dK c0 .. c[ncw-2],
+            //   P(j+1) (if any), dK c[ncw-1].   Slot positions: xt_pos_P / xt_pos_S below.
+            bool has = co.next(p.sc, To);
+            if (has)
+                for (int b = 0; b < npl; ++b) fn(2, To, b, 0);
+            while (has) {
+                Tile Tnext;
+                const bool hnext = co.next(p.sc, Tnext);
+                auto blocks = [&](int a) {
+                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
+                };
+                for (int a = 0; a < ncw - 1; ++a) blocks(a);
+                for (int b = 0; b < npl; ++b) fn(2, To, b, 1);
+                blocks(ncw - 1);
+                for (int a = ncw; a < nacc - 1; ++a) blocks(a);
+                if (hnext)
+                    for (int b = 0; b < npl; ++b) fn(2, Tnext, b, 0);
+                blocks(nacc - 1);
+                To = Tnext;
+                has = hnext;
+            }
         } else {
             while (co.next(p.sc, To)) {
-                if (xt) {   // P plane (slots of 128 tape rows), dV; dS plane, dK
-                    for (int h = 0; h < 2; ++h) {
-                        for (int b = 0; b < npl; ++b) fn(2, To, b, h);
-                        for (int a = h * ncw; a < (h + 1) * ncw; ++a)
-                            for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
-                    }
-                    continue;
-                }
                 for (int s = 0; s < nsl; ++s) {
                     fn(0, To, s, 0);
                     fn(0, To, s, 1);
@@ -365,7 +390,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             walk([&](int kind, const Tile& T, int a, int b) {
                 mbar_wait(&empty[st], ph ^ 1u);
                 trace_slot(p, k++, 0);
-                uint8_t* sp = slots + (size_t)st * SLOT;
+                uint8_t* sp = slots + (size_t)st * slotb;
                 const Maps& mp = p.maps[T.rl];
                 if (kind == 2) {   // dS tape: query rows [128 a, 128 a + 128) of plane b (P, dS)
                     if (a == 0 && b == 0 && p.dpoll) {   // BWDQ may still run: wait for these rows' tiles
@@ -395,7 +420,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     for (int x = 0; x < nbox; ++x)
                         tma_load_3d(sp + x * KB * 128, m, &full[st], CW * c + 32 * x, T.m0 - w + KB * b, T.u);
                 }
-                if (++st == NST) { st = 0; ph ^= 1u; }
+                if (++st == nst) { st = 0; ph ^= 1u; }
             });
         }
     } else if (warp >= 10) {   // ------------------------------------------------- converters
@@ -405,7 +430,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         walk([&](int kind, const Tile&, int a, int) {
             mbar_wait(&full[st], ph);
             if (ct == 0) trace_slot(p, k, 1);
-            uint8_t* sp = slots + (size_t)st * SLOT;
+            uint8_t* sp = slots + (size_t)st * slotb;
             if (kind == 2) {
                 // tape slot: read as fp32 by the softmax warps (arrive only, keeping the phases)
             } else if (kind == 0) {
@@ -418,7 +443,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             warp_arrive(&conv[st]);
             if (ct == 0) trace_slot(p, k, 2);
             ++k;
-            if (++st == NST) { st = 0; ph ^= 1u; }
+            if (++st == nst) { st = 0; ph ^= 1u; }
         });
     } else if (warp == 9) {
         if (lane == 0) {   // ------------------------------------------------------ MMA issuer
@@ -431,7 +456,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             int jg = 0;          // score GEMMs: tile counter
             int jo = 0;          // output GEMMs: tile counter
             walk([&](int kind, const Tile&, int a, int b) {
-                const uint32_t sa = smem_u32(slots + (size_t)st * SLOT);
+                const uint32_t sa = smem_u32(slots + (size_t)st * slotb);
                 if (kind == 2) {   // tape slot: no MMA (the softmax warps free it)
                     mbar_wait(&conv[st], ph);
                 } else if (kind == 0) {
@@ -498,7 +523,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     }
                 }
                 trace_slot(p, k++, 4);
-                if (++st == NST) { st = 0; ph ^= 1u; }
+                if (++st == nst) { st = 0; ph ^= 1u; }
             });
         }
     } else if (warp < 4) {   // ------------------------------------------------ softmax warps
@@ -652,18 +677,26 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     if (t == 0) st_release_gpu(p.flags + rowbase + (int64_t)m0 * p.dil, 1u);
                 }
             } else if (xt) {   // BWDKV from the dS tape: P^T -> R1 (hi | lo), then dS^T -> R0
-                const int per = 2 * npl + nacc * nkb;
+                const int tsw = p.tsw;
+                // walk positions (see walk): every segment holds 2 ncw nkb output blocks and 2 npl tape slots, plus P(0) in
+                // segment 0; P(j > 0) is the npl slots before the last dK chunk of segment j - 1
+                const int seg = nacc * nkb + 2 * npl;
+                const int Sj = j * seg + (j > 0 ? npl : 0);
+                const int posP = j == 0 ? 0 : Sj - nkb - npl;
+                const int posS = Sj + (j == 0 ? npl : 0) + (ncw - 1) * nkb;
                 for (int h = 0; h < 2; ++h) {
                     // R1 once the previous tile's dK accumulations in it are drained; R0 once this
                     // tile's dV accumulations in it are (the MMAs that read them as A came earlier)
                     if (h == 1) mbar_wait(&xfree[1], (uint32_t)j & 1u);
                     else if (j > 0) mbar_wait(&xfree[0], (uint32_t)(j - 1) & 1u);
                     tc_fence_after();
+                    if (t == 0) trace_tile(p, j, 10 + 3 * h);   // operand region free
                     const uint32_t dst = h == 0 ? rP : rS;
                     for (int b = 0; b < npl; ++b) {
-                        const int k = j * per + (h ? npl + ncw * nkb : 0) + b, st = k % NST;
-                        mbar_wait(&full[st], (uint32_t)(k / NST) & 1u);
-                        const float* sv = reinterpret_cast<const float*>(slots + (size_t)st * SLOT);
+                        const int k = (h ? posS : posP) + b, st = k % nst;
+                        mbar_wait(&full[st], (uint32_t)(k / nst) & 1u);
+                        if (t == 0 && b == 0) trace_tile(p, j, 11 + 3 * h);   // first tape slot landed
+                        const float* sv = reinterpret_cast<const float*>(slots + (size_t)st * slotb);
                         for (int c = 4 * b; c < 4 * b + 4 && c < nch; ++c) {
                             if (c < c_lo || c > c_hi) {
                                 tmem_st16(dst + c * 32, zero16);
@@ -672,20 +705,23 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                             }
 #pragma unroll
                             for (int hh = 0; hh < 2; ++hh) {
+                                // column n = n0 + e (query kb + n, tape row n - 128 b of the slot),
+                                // key t: entry t - n + 2w at float (kb + n) & 3 + t - n + 2w; in the
+                                // band iff e in [lo, hi].  Branch-free, loads back to back.
                                 const int n0 = c * 32 + 16 * hh;
+                                const int a0 = (n0 - 128 * b) * tsw + t - n0 + 2 * w;
+                                const int lo = max(t - n0, -(kb + n0)), hi = min(t - n0 + 2 * w, Lr - 1 - (kb + n0));
+                                const int q3 = (kb + n0) & 3;
                                 uint32_t pk[8], pl[8];
+                                float x[16];
 #pragma unroll
-                                for (int e = 0; e < 16; e += 2) {
-                                    float x[2];
-#pragma unroll
-                                    for (int hx = 0; hx < 2; ++hx) {
-                                        // query column n (tape row kb + n), key t: entry t - n + 2w
-                                        const int n = n0 + e + hx, mq = kb + n;
-                                        x[hx] = band_ok(n, t, w, mq, Lr)
-                                                    ? sv[(n - 128 * b) * p.tsw + (mq & 3) + t - n + 2 * w] : 0.f;
-                                    }
-                                    split2(x[0], x[1], pk[e / 2], pl[e / 2]);
+                                for (int e = 0; e < 16; ++e) {
+                                    const bool ok = e >= lo && e <= hi;
+                                    const float xv = sv[ok ? a0 + e * (tsw - 1) + ((q3 + e) & 3) : 0];
+                                    x[e] = ok ? xv : 0.f;
                                 }
+#pragma unroll
+                                for (int e = 0; e < 16; e += 2) split2(x[e], x[e + 1], pk[e / 2], pl[e / 2]);
                                 tmem_st8(dst + n0, pk);
                                 tmem_st8(dst + n0 + 8, pl);
                             }
@@ -696,6 +732,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     tmem_wait_st();
                     tc_fence_before();
                     warp_arrive(&p_full[h]);
+                    if (t == 0) trace_tile(p, j, 12 + 3 * h);   // operand built
                 }
             } else {   // BWDKV: rows are keys, columns halo queries
                 for (int c = 0; c < nch; ++c) {
@@ -831,7 +868,8 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
                      int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
     static std::once_flag once;
     std::call_once(once, [] {
-        cudaFuncSetAttribute(tc_band32_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES);
+        cudaFuncSetAttribute(tc_band32_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)(SMEM_BYTES > SMEM_BYTES_XT ? SMEM_BYTES : SMEM_BYTES_XT));
     });
     const int64_t wc = w < L ? w : L;
     const int NK = halo_rows32(L, w);
@@ -880,12 +918,13 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         const int tiles = (int)ceil_div(Lr0, BM);
         const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms32() ? total : num_sms32()));
+        const size_t smem = MODE == BWDKV && p.xt ? SMEM_BYTES_XT : SMEM_BYTES;
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         if (MODE == BWDKV && r0 == 0 && p.dpoll) {   // directly after this call's last BWDQ launch
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = grid;
             cfg.blockDim = dim3(NTHREADS);
-            cfg.dynamicSmemBytes = SMEM_BYTES;
+            cfg.dynamicSmemBytes = smem;
             cfg.stream = st;
             cudaLaunchAttribute at[1];
             at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -894,7 +933,7 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
             cfg.numAttrs = 1;
             cudaLaunchKernelEx(&cfg, tc_band32_kernel<MODE>, p);
         } else {
-            tc_band32_kernel<MODE><<<grid, NTHREADS, SMEM_BYTES, st>>>(p);
+            tc_band32_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
         }
         prof_mark(st);
         cudaError_t e = cudaGetLastError();

@@ -144,7 +144,7 @@ def test_tc32_parity(ft, shape):
     run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=16)
 
 
-# The dS tape between the fp32 backward kernels (FT_KNOB_DSTAPE): the dK/dV kernel
+# The dS tape between the tensor-core backward kernels (FT_KNOB_DSTAPE): the dK/dV kernel
 # reads P and dS from the dQ kernel instead of recomputing them, with the per-tile flag hand-off
 # (PDL on) or plain stream order (PDL off); many tiles per CTA, ragged residues, several launches
 # of residues (dilation > 8), w = 0.
@@ -154,10 +154,11 @@ DSTAPE = [(1, 4, 3000, 256, 32, 1), (2, 3, 1001, 256, 5, 3), (1, 1, 700, 512, 32
 
 
 @pytest.mark.parametrize("tape,pdl", [(1, 1), (1, 0), (0, 1)])
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
 @pytest.mark.parametrize("shape", DSTAPE, ids=lambda s: "x".join(map(str, s)))
-def test_tc32_dstape(ft, shape, tape, pdl):
+def test_dstape(ft, shape, dtype, tape, pdl):
     with ft.knobs(dstape=tape, pdl=pdl):
-        run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=21)
+        run_case(ft, WinAttnShape(*shape), dtype, "tc", seed=21)
 
 
 @pytest.mark.parametrize("seed", [0, 1, 2])
@@ -460,6 +461,9 @@ MIXED = [
     (2, 2, 260, 64, 8, 5, 0, "bf16"),      # none dilated
     (1, 3, 200, 32, 6, 2, 1, "f32"),       # SIMT path
     (1, 4, 300, 512, 32, 4, 2, "bf16"),    # d = 512 band kernels
+    (2, 4, 300, 256, 32, 4, 2, "f32"),     # fp32 tensor cores with the dS tape: per-slice workspace rows
+    (1, 4, 700, 512, 32, 4, 2, "f32"),     # C2a_mix-like, fp32
+    (2, 4, 300, 256, 32, 4, 2, "bf16"),    # bf16 band kernels with the dS tape
 ]
 
 

@@ -21,7 +21,7 @@ import bench  # noqa: E402
 import paper_conf_pldi_tangzwjzyz22_b200 as ft  # noqa: E402
 
 TR_SLOTS, TR_TILES = 96, 4
-PER = TR_SLOTS * 5 + TR_TILES * 8
+PER = TR_SLOTS * 5 + TR_TILES * 16
 
 
 def main():
@@ -48,18 +48,19 @@ def main():
     for m, name in enumerate(["FWD", "BWDQ", "BWDKV"]):
         t = bufs[m].view(148, PER).cpu().double()
         s = t[:, :TR_SLOTS * 5].view(148, TR_SLOTS, 5)
-        tl = t[:, TR_SLOTS * 5:].view(148, TR_TILES, 8)
+        tl = t[:, TR_SLOTS * 5:].view(148, TR_TILES, 16)
         t0 = s[:, 0:1, 0:1]
         s = (s - t0) / 1e3
         tl = (tl - t0[:, :, :1]) / 1e3
         print(f"== {name} (CTA 0, kclk)   prod  cv0  cv1  mma0 mma1")
         for i in range(min(a.slots, TR_SLOTS)):
             r = s[0, i]
-            if (r <= -1e6).any() or (bufs[m].view(148, PER)[0, i * 5:(i + 1) * 5] == 0).any():
+            if int(bufs[m].view(148, PER)[0, i * 5]) == 0:
                 break
+            r = torch.where(bufs[m].view(148, PER)[0, i * 5:(i + 1) * 5].cpu() == 0, torch.full_like(r, float("nan")), r)
             print(f"  slot {i:3d} " + " ".join(f"{x:6.1f}" for x in r.tolist()))
         for j in range(TR_TILES):
-            print(f"  tile {j}: " + " ".join(f"{x:7.1f}" for x in tl[0, j].tolist()))
+            print(f"  tile {j}: " + " ".join("   -   " if x < -1e6 else f"{x:7.1f}" for x in tl[0, j].tolist()))
         ok = (bufs[m].view(148, PER)[:, :TR_SLOTS * 5].view(148, TR_SLOTS, 5) > 0).all(dim=2).cpu()
         def med(x):
             return float(x[ok].median()) if ok.any() else float("nan")

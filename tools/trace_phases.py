@@ -57,6 +57,11 @@ def main():
             print(f"    pass 1 (max)                    {med(t[:,:,10]-t[:,:,6]):7.2f}")
             print(f"    wait P buffer free              {med(t[:,:,11]-t[:,:,10]):7.2f}")
             print(f"    pass 2 (exp, P -> smem)         {med(t[:,:,7]-t[:,:,11]):7.2f}")
+        if name == "BWDKV" and float(t[:, :, 11].max()) > 0:   # dS tape: build phases
+            print(f"    xt: loop top -> A operands free {med(t[:,:,10]-t[:,:,6]):7.2f}")
+            print(f"    xt: -> first tape slot landed   {med(t[:,:,11]-t[:,:,10]):7.2f}")
+            print(f"    xt: -> last tape slot landed    {med(t[:,:,15]-t[:,:,11]):7.2f}")
+            print(f"    xt: -> p arrive (build)         {med(t[:,:,7]-t[:,:,15]):7.2f}")
         print(f"  p arrive -> mma sees p            {med(t[:,:,4]-t[:,:,7]):7.2f}")
         print(f"  output MMAs issued (p -> out end) {med(t[:,:,5]-t[:,:,4]):7.2f}")
         print(f"    p seen -> o_empty passed        {med(t[:,:,12]-t[:,:,4]):7.2f}")
