@@ -162,7 +162,12 @@ ft_status ft_winattn_bwd_tape(const void* q, const void* k, const void* v,
                               int64_t w, int64_t dilation, ft_dtype dtype,
                               void* workspace, size_t workspace_bytes, void* stream);
 
-/* Device workspace the backward needs (the per-row D_i, fp32). */
+/* Device workspace the backward needs: the per-row D_i (fp32), and, for shapes the tensor-core
+ * kernels serve with the dS tape (fp32 with d >= 256; bf16 band kernels with d > 256; or any they
+ * can serve while FT_KNOB_DSTAPE = 2), one flag word per row and two fp32 planes of
+ * 4 ceil((2w + 4) / 4) floats per row (P and dS of every band entry, written by the dQ kernel and
+ * read by the dK/dV kernel of the same call: selective materialization).  The
+ * size depends on FT_KNOB_DSTAPE; query it with the knobs the call will run under. */
 size_t ft_winattn_bwd_workspace_bytes(int64_t batch, int64_t heads, int64_t seq_len, int64_t d,
                                       int64_t w, int64_t dilation, ft_dtype dtype);
 
@@ -199,8 +204,9 @@ ft_status ft_winattn_debug_trace(int kernel_mode, void* device_buffer);
  *   3 FT_KNOB_WIDE    1 the w > 64 wide kernels, 0 the chunked fallback  [FT_WINATTN_WIDE=0]
  *   4 FT_KNOB_SIDE    1 per-head-dilation calls use a side stream, 0 serial
  *                                                                [FT_WINATTN_MIXED_SERIAL=1]
- *   5 FT_KNOB_DSTAPE  1 the fp32 tensor-core dK/dV kernel reads P and dS from the dQ kernel's
- *                     tape (in the workspace), 0 it recomputes them  [FT_WINATTN_DSTAPE=0]
+ *   5 FT_KNOB_DSTAPE  1 the tensor-core dK/dV kernel (fp32; bf16 band kernels) reads P and dS
+ *                     from the dQ kernel's tape in the workspace where that pays (d >= 256),
+ *                     2 wherever the kernels can, 0 it recomputes them  [FT_WINATTN_DSTAPE]
  * ft_winattn_debug_set returns FT_ERR_INVALID_VALUE for an unknown knob or value;
  * ft_winattn_debug_get returns the current value (-1 for an unknown knob). */
 enum { FT_KNOB_PATH = 0, FT_KNOB_PDL = 1, FT_KNOB_NARROW = 2, FT_KNOB_WIDE = 3, FT_KNOB_SIDE = 4,

@@ -66,7 +66,7 @@ void knob_init() {
         g_knob[ftw::K_NARROW] = env_int("FT_WINATTN_NARROW", 1) != 0;
         g_knob[ftw::K_WIDE] = env_int("FT_WINATTN_WIDE", 1) != 0;
         g_knob[ftw::K_SIDE] = env_int("FT_WINATTN_MIXED_SERIAL", 0) != 1;
-        g_knob[ftw::K_DSTAPE] = env_int("FT_WINATTN_DSTAPE", 1) != 0;
+        g_knob[ftw::K_DSTAPE] = env_int("FT_WINATTN_DSTAPE", 1) < 0 ? 0 : (env_int("FT_WINATTN_DSTAPE", 1) > 2 ? 2 : env_int("FT_WINATTN_DSTAPE", 1));
     });
 }
 thread_local bool g_handoff = false;   // inside ft_winattn_fwd_bwd
@@ -96,6 +96,7 @@ ft_status choose_path(int is_bwd, int64_t units, int64_t L, int64_t d, int64_t w
 struct WsLayout {
     size_t dB = 0, fB = 0, pB = 0;
     int tsw = 0;
+    int64_t rows = 0;
     bool tape = false;
     size_t total() const { return dB + fB + 2 * pB; }
 };
@@ -103,8 +104,9 @@ size_t round256(size_t x) { return (x + 255) / 256 * 256; }
 WsLayout ws_layout(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, ft_dtype dt) {
     WsLayout l;
     const size_t rows = (size_t)(B * H * L);
+    l.rows = (int64_t)rows;
     l.dB = round256(rows * sizeof(float));
-    l.tape = ftw::dstape_pays(d) && (dt == FT_F32 ? ftw::tc32_supported(B * H, L, d, w, dil)
+    l.tape = (ftw::dstape_pays(d, dt) || ftw::knob(ftw::K_DSTAPE) == 2) && (dt == FT_F32 ? ftw::tc32_supported(B * H, L, d, w, dil)
                                                    : ftw::tc_band_dstape_ok(B * H, L, d, w, dil));
     if (l.tape) {
         l.tsw = ftw::dstape_tsw(w < L ? w : L);
@@ -151,7 +153,8 @@ int ft_winattn_abi_version(void) { return FT_WINATTN_ABI_VERSION; }
 
 ft_status ft_winattn_debug_set(int which, int value) {
     if (which < 0 || which >= ftw::K_NUM) return FT_ERR_INVALID_VALUE;
-    if (which == ftw::K_PATH ? (value < 0 || value > 2) : (value < 0 || value > 1)) return FT_ERR_INVALID_VALUE;
+    const int vmax = (which == ftw::K_PATH || which == ftw::K_DSTAPE) ? 2 : 1;
+    if (value < 0 || value > vmax) return FT_ERR_INVALID_VALUE;
     knob_init();
     g_knob[which].store(value, std::memory_order_relaxed);
     return FT_OK;
@@ -314,9 +317,10 @@ ft_status run_bwd(const void* q, const void* k, const void* v, const void* out, 
     const bool use_tape = lay.tape && base && ftw::knob(ftw::K_DSTAPE);
     if (use_tape) {
         tape.flags = (uint32_t*)(base + lay.dB + row0 * 4);
-        tape.P = (float*)(base + lay.dB + lay.fB + (size_t)row0 * lay.tsw * 4);
-        tape.S = (float*)(base + lay.dB + lay.fB + lay.pB + (size_t)row0 * lay.tsw * 4);
+        tape.P = (float*)(base + lay.dB + lay.fB + (size_t)row0 * 16);   // granule-major planes
+        tape.S = (float*)(base + lay.dB + lay.fB + lay.pB + (size_t)row0 * 16);
         tape.tsw = lay.tsw;
+        tape.grows = lay.rows;
     }
     cudaError_t e;
     bind_context();

@@ -42,21 +42,26 @@ inline Geo make_geo(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64
 inline int64_t geo_blocks(const Geo& g) { return g.units * g.nres * g.tiles; }
 
 // The dS tape between the two backward kernels (selective materialization),
-// fp32 (tc_band32.cu) and bf16 band (tc_band.cu) tensor-core kernels: the dQ kernel stores every band entry's P_ij and dS_ij (fp32, row i of plane P / S holds entry
-// e = j - i + w at float offset (m & 3) + e, m = i's row in its residue, rows tsw floats apart)
-// and publishes flags[first row of each 128-row tile] = 1; the dK/dV kernel then reads its
-// P^T / dS^T from the tape instead of recomputing S^T and dP^T.  Workspace layout: api.cu.
+// fp32 (tc_band32.cu) and bf16 band (tc_band.cu) tensor-core kernels: the dQ kernel stores every
+// band entry's P_ij and dS_ij and publishes flags[first row of each 128-row tile] = 1; the dK/dV
+// kernel then reads its P^T / dS^T from the tape instead of recomputing S^T and dP^T.
+// Plane layout (fp32): entry e = j - i + w of row i sits at offset o = (m & 3) + e of that row
+// (m = i's row in its residue, so the dQ kernel's 16-byte stores are aligned), and the row's
+// offsets are grouped in 16-byte granules G = o / 4 stored granule-major: float (G grows + i) 4
+// + o % 4 -- a warp's stores of one granule index cover consecutive rows.  Workspace: api.cu.
 struct DsTape {
     uint32_t* flags;   // one word per row (only tile-first rows used)
-    float* P;          // [rows][tsw]
-    float* S;          // [rows][tsw]
-    int tsw;
+    float* P;          // [tsw / 4][grows][4]
+    float* S;          // [tsw / 4][grows][4]
+    int tsw;           // floats per row, a multiple of 4
+    int64_t grows;     // granule stride in rows (the rows of the whole call)
 };
 inline int dstape_tsw(int64_t wc) { return (int)((2 * wc + 4 + 3) / 4 * 4); }
 // The tape costs 2 tsw floats per row written and read; it replaces the dK/dV kernel's score phase
-// (K, V, Q, dO slices, two GEMMs, the operand conversion).  Measured (tools/tape_ablation.py,
-// DESIGN.md §10): slower at d = 64, even at d = 128, 1.1-1.26x faster at d >= 256.
-inline bool dstape_pays(int64_t d) { return d >= 256; }
+// (K, V, Q, dO slices, two GEMMs; in fp32 also their operand conversion).  Measured
+// (tools/tape_ablation.py): fp32 1.14-1.33x faster at d >= 256; bf16 0.91-0.95x at
+// d = 128, even at d = 256, 1.05-1.13x at d = 512.
+inline bool dstape_pays(int64_t d, ft_dtype dt) { return dt == FT_F32 ? d >= 256 : d > 256; }
 
 // SIMT (CUDA-core) kernels -- simt.cu
 // tape (optional): the raw band scores s_ij, fp32 [B*H*L][2w+1] (w clamped to L); the forward
@@ -155,7 +160,8 @@ enum Knob {
     K_NARROW = 2,   // 1: d = 64, w <= 32 narrow kernels; 0: band kernels (FT_WINATTN_NARROW=0)
     K_WIDE = 3,     // 1: w > 64 wide kernels; 0: the chunked fallback kernels (FT_WINATTN_WIDE=0)
     K_SIDE = 4,     // 1: per-head-dilation calls use a side stream; 0: serial (FT_WINATTN_MIXED_SERIAL=1)
-    K_DSTAPE = 5,   // 1: fp32 tensor-core backward hands P / dS over on a tape; 0: recompute (FT_WINATTN_DSTAPE=0)
+    K_DSTAPE = 5,   // 1: tensor-core backward hands P / dS over on a tape where it pays (d >= 256), 2: wherever
+                    // the kernels can, 0: recompute (FT_WINATTN_DSTAPE=0|1|2)
     K_NUM = 6
 };
 int knob(Knob k);

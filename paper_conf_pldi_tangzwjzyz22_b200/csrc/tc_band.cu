@@ -100,7 +100,8 @@ struct Params {
     // dS tape between BWDQ and BWDKV (ftw::DsTape, internal.h; the fp32 kernels' scheme,
     // tc_band32.cu): BWDQ stores P and dS of every band entry and releases a flag per tile;
     // BWDKV (xt) loads them instead of running the S^T and dP^T GEMMs.
-    int xt, tsw, trows;          // trows: tape rows per ring slot (both planes)
+    int xt, tsw, trows;          // trows: tape rows per ring slot (both planes; boxes of trows + 1)
+    int64_t grows;               // tape granule stride (rows)
     uint32_t* flags;
     float* tP;
     float* tS;
@@ -133,6 +134,11 @@ __device__ __forceinline__ bool band_ok(int n, int t, int w, int mcol, int Lr) {
     return (unsigned)(n - t) <= (unsigned)(2 * w) && mcol >= 0 && mcol < Lr;
 }
 
+// One tape plane's box in a ring slot ([tsw / 4][trows + 1][4] floats), padded so that the second
+// plane's TMA destination is 128-byte aligned.
+__host__ __device__ inline uint32_t tape_plane_bytes(int trows, int tsw) {
+    return ((uint32_t)(trows + 1) * (uint32_t)tsw * 4u + 127u) & ~127u;
+}
 __host__ __device__ inline int chunk_w(int d, int c) { return d - 256 * c < 256 ? d - 256 * c : 256; }
 
 __host__ __device__ inline uint32_t slot_bytes(int NK) {
@@ -291,8 +297,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
     uint64_t* p_free = s_full + 4;   // P smem consumed by the tile's output MMAs
     uint64_t* p_blk = s_full + 5;    // [4] BWD: dS of 64-key block b written (per-block handoff)
     uint64_t* a_free = s_full + 9;   // xt: the tile's dK MMAs are done with dS^T in TMEM
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 10);
+    uint64_t* tape_done = s_full + 10;   // xt3: BWDQ pass 3 read the tile's dS / P from TMEM
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 11);
     const bool xt = MODE == BWDKV && p.xt;
+    // BWDQ with the dS tape and free TMEM columns [XT3_COL, 256) beside S (NK <= 192): pass 3
+    constexpr uint32_t XT3_COL = 192;
+    const bool xt3 = !TAPE && MODE == BWDQ && p.xt && NK <= (int)XT3_COL && !early;
     const int ntape = xt ? NK / p.trows : 0;   // tape slots per tile
 
     if (warp == 8) {
@@ -307,6 +317,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
             mbar_init(p_free, 1);
             for (int i = 0; i < 4; ++i) mbar_init(&p_blk[i], 128);
             mbar_init(a_free, 1);
+            mbar_init(tape_done, 128);
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
                 const Maps& mp = p.maps[i];
@@ -397,13 +408,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                             for (int tq = lo; tq <= hi; ++tq) wait_flag(p.flags + rowbase + (int64_t)tq * BM * p.dil);
                             asm volatile("fence.proxy.async.global;" ::: "memory");
                         }
-                        const uint32_t pl = (uint32_t)p.trows * (uint32_t)p.tsw * 4u;
+                        const uint32_t pl = tape_plane_bytes(p.trows, p.tsw);
                         for (int b = 0; b < ntape; ++b) {
                             uint8_t* sp = take();
                             if (b == 0) trace_ev(p, jo, 0);
-                            mbar_arrive_expect_tx(&full[st], 2 * pl);
-                            tma_load_3d(sp, &mp.tp, &full[st], 0, To.m0 - w + p.trows * b, To.u);
-                            tma_load_3d(sp + pl, &mp.ts, &full[st], 0, To.m0 - w + p.trows * b, To.u);
+                            mbar_arrive_expect_tx(&full[st], 2u * (uint32_t)(p.trows + 1) * (uint32_t)p.tsw * 4u);
+                            tma_load_4d(sp, &mp.tp, &full[st], 0, To.m0 - w + p.trows * b, To.u, 0);
+                            tma_load_4d(sp + pl, &mp.ts, &full[st], 0, To.m0 - w + p.trows * b, To.u, 0);
                             adv();
                         }
                     }
@@ -545,6 +556,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     // the epilogue must have drained the previous tile's last accumulation
                     if (!early && ga > 0) {
                         mbar_wait(o_empty, (ga - 1) & 1);
+                        tc_fence_after();
+                    }
+                    if (xt3 && ownS && jo > 0) {   // pass 3 of the previous tile read its dS
+                        mbar_wait(tape_done, (jo - 1) & 1);
                         tc_fence_after();
                     }
                     for (int s = 0; s < nsl; ++s) g_slice(jo, s);
@@ -698,12 +713,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         block_done(c);
                         continue;
                     }
-                    uint32_t rs[32], rd[32], pk[16], pl[16];
+                    uint32_t rs[32], rd[32], pk[16], pl[16], pp[16];
                     if (!tp) tmem_ld32(trow + c * 32, rs);
                     tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
                     // dS tape (xt): entry e = n - t of row mrow at float (mrow & 3) + e = ob + (n - 32 c),
-                    // four entries per 16-byte store ((mrow & 3) == (t & 3), m0 % 128 == 0)
+                    // four entries per 16-byte store ((mrow & 3) == (t & 3), m0 % 128 == 0).  With
+                    // free TMEM columns (xt3) P goes there as bf16 and pass 3 stores the tape after
+                    // p_full, off the MMAs' critical path; else the stores are issued here.
                     const int ob = (t & 3) + c * 32 - t;
 #pragma unroll
                     for (int g4 = 0; g4 < 8; ++g4) {
@@ -718,21 +735,53 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                         }
                         split_bf16x2(dv[0], dv[1], pk[2 * g4], pl[2 * g4]);
                         split_bf16x2(dv[2], dv[3], pk[2 * g4 + 1], pl[2 * g4 + 1]);
+                        pp[2 * g4] = pack_bf16x2(pv[0], pv[1]);
+                        pp[2 * g4 + 1] = pack_bf16x2(pv[2], pv[3]);
                         const int o = ob + 4 * g4;
-                        if (!TAPE && p.xt && mrow < Lr && o >= 0 && o < p.tsw) {
-                            const size_t ro = (size_t)(rowbase + (int64_t)mrow * p.dil) * p.tsw + o;
+                        if (!TAPE && p.xt && !xt3 && mrow < Lr && o >= 0 && o < p.tsw) {
+                            const size_t ro = ((size_t)(o >> 2) * p.grows + rowbase + (int64_t)mrow * p.dil) * 4;
                             *reinterpret_cast<float4*>(p.tP + ro) = make_float4(pv[0], pv[1], pv[2], pv[3]);
                             *reinterpret_cast<float4*>(p.tS + ro) = make_float4(dv[0], dv[1], dv[2], dv[3]);
                         }
                     }
                     tmem_st16(trow + c * 32, pk);
                     tmem_st16(trow + c * 32 + 16, pl);
+                    if (xt3) tmem_st16(trow + XT3_COL + 16 * (c - c_lo), pp);
                     block_done(c);
                 }
                 tmem_wait_st();
                 tc_fence_before();
                 mbar_arrive(p_full);
                 if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
+                if (xt3) {   // pass 3: the tape from dS hi / lo and P (bf16) in TMEM
+                    for (int c = c_lo; c <= c_hi; ++c) {
+                        uint32_t hi[16], lo[16], pb[16];
+                        tmem_ld16(trow + c * 32, hi);
+                        tmem_ld16(trow + c * 32 + 16, lo);
+                        tmem_ld16(trow + XT3_COL + 16 * (c - c_lo), pb);
+                        tmem_wait_ld();
+                        if (c == c_hi) {   // the S columns may take the next tile's scores
+                            tc_fence_before();
+                            mbar_arrive(tape_done);
+                        }
+                        const int ob = (t & 3) + c * 32 - t;
+#pragma unroll
+                        for (int g4 = 0; g4 < 8; ++g4) {
+                            const int o = ob + 4 * g4;
+                            if (mrow < Lr && o >= 0 && o < p.tsw) {
+                                auto f0 = [](uint32_t x) { return __uint_as_float(x << 16); };
+                                auto f1 = [](uint32_t x) { return __uint_as_float(x & 0xFFFF0000u); };
+                                const uint32_t h0 = hi[2 * g4], h1 = hi[2 * g4 + 1];
+                                const uint32_t l0 = lo[2 * g4], l1 = lo[2 * g4 + 1];
+                                const uint32_t b0 = pb[2 * g4], b1 = pb[2 * g4 + 1];
+                                const size_t ro = ((size_t)(o >> 2) * p.grows + rowbase + (int64_t)mrow * p.dil) * 4;
+                                *reinterpret_cast<float4*>(p.tP + ro) = make_float4(f0(b0), f1(b0), f0(b1), f1(b1));
+                                *reinterpret_cast<float4*>(p.tS + ro) =
+                                    make_float4(f0(h0) + f0(l0), f1(h0) + f1(l0), f0(h1) + f0(l1), f1(h1) + f1(l1));
+                            }
+                        }
+                    }
+                }
                 if (!TAPE && p.xt) {   // publish the tile's tape rows to BWDKV
                     __threadfence();
                     named_bar_sync(2, 128);
@@ -751,7 +800,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     mbar_wait(&full[st], (uint32_t)(k / NST) & 1u);
                     if (t == 0) trace_ev(p, j, b == 0 ? 11 : 15);
                     const float* sv = reinterpret_cast<const float*>(sslots + (size_t)st * SLOT);
-                    const float* sS = sv + p.trows * p.tsw;
+                    const float* sS = sv + tape_plane_bytes(p.trows, p.tsw) / 4;
+                    const int gstr = 4 * (p.trows + 1);   // floats between granule rows of a plane
                     for (int c = b * cps; c < (b + 1) * cps; ++c) {
                         if (c < c_lo || c > c_hi) {
                             if (j == 0) st_p_chunk(sP, t, c, zero16);   // P^T zeros persist
@@ -770,7 +820,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                                 // branch-free (all loads of a chunk issue back to back): an entry
                                 // outside the band reads offset 0 of the slot and is zeroed
                                 const bool ok = band_ok(n, t, w, mq, Lr);
-                                const int o = ok ? (n - b * p.trows) * p.tsw + (mq & 3) + t - n + 2 * w : 0;
+                                const int oo = (mq & 3) + t - n + 2 * w;
+                                const int o = ok ? (oo >> 2) * gstr + (n - b * p.trows) * 4 + (oo & 3) : 0;
                                 const float xp = sv[o], xs = sS[o];
                                 pv[h] = ok ? xp : 0.f;
                                 dv[h] = ok ? xs : 0.f;
@@ -983,9 +1034,9 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
             if (ok && ob2) ok = make_residue_map(&m.ob2, ob2, L, d, units, dil, r, KB);
             if (ok && o2) ok = make_residue_map(&m.o2, o2, L, d, units, dil, r, 32);
             if (ok && ds && !tape && MODE == BWDKV) {
-                const int trows = 64u * (uint32_t)ds->tsw * 8u <= slot_bytes(NK) ? 64 : 32;
-                ok = make_residue_map_tape(&m.tp, ds->P, L, ds->tsw, units, dil, r, trows) &&
-                     make_residue_map_tape(&m.ts, ds->S, L, ds->tsw, units, dil, r, trows);
+                const int trows = 2 * tape_plane_bytes(64, ds->tsw) <= slot_bytes(NK) ? 64 : 32;
+                ok = make_residue_map_tape(&m.tp, ds->P, L, ds->tsw, units, dil, r, trows + 1, ds->grows) &&
+                     make_residue_map_tape(&m.ts, ds->S, L, ds->tsw, units, dil, r, trows + 1, ds->grows);
             }
             if (!ok) return cudaErrorInvalidValue;
         }
@@ -1010,7 +1061,8 @@ cudaError_t launch(const void* a1, const void* b1, const void* a2, const void* b
         if (ds && !tape && MODE != FWD) {
             p.xt = 1;
             p.tsw = ds->tsw;
-            p.trows = 64u * (uint32_t)ds->tsw * 8u <= slot_bytes(NK) ? 64 : 32;
+            p.trows = 2 * tape_plane_bytes(64, ds->tsw) <= slot_bytes(NK) ? 64 : 32;
+            p.grows = ds->grows;
             p.flags = ds->flags;
             p.tP = ds->P;
             p.tS = ds->S;

@@ -67,11 +67,13 @@ constexpr int KB = 64;                    // keys per output block
 constexpr int CW = 128;                   // output columns per accumulation
 constexpr int NST = 4;                    // ring slots
 constexpr uint32_t SLOT = 40 * 1024;      // fp32 score slice (128 + 192 rows x 32 cols) / 64 x 128 block
-// BWDKV with the dS tape streams no score slices: five smaller slots (a 128-row tape plane slice,
-// tsw <= 68, or a 32 KB output block), so the tape slots of the next operand and a whole output
-// chunk's key blocks fit in the ring together
-constexpr int NST_XT = 5;
-constexpr uint32_t SLOT_XT = 128 * 68 * 4;
+// BWDKV with the dS tape streams no score slices: six 32 KB slots (a 96-row slice of one tape
+// plane, [tsw / 4][97][4] floats with tsw <= 68, or a 64 x 128 output block), so the tape slots of
+// the next operand and a whole output chunk's key blocks fit in the ring together.  No scratch.
+constexpr int NST_XT = 6;
+constexpr uint32_t SLOT_XT = 32 * 1024;
+constexpr int TROWS = 96, TBOX = TROWS + 1;   // tape rows per slot; box rows (odd row stride: no bank conflicts)
+static_assert(TBOX * 68 * 4 <= (int)SLOT_XT, "tape slot");
 constexpr uint32_t STG = 32 * 128;        // one epilogue warp's 32-row x 32-col fp32 staging box
 constexpr int NSTG = 2;                   // staging boxes per epilogue warp
 constexpr int NTHREADS = 512;
@@ -99,6 +101,7 @@ struct Params {
     // dS tape (ftw::DsTape, internal.h): BWDQ stores P and dS of every band entry and sets the
     // flag of each tile it finished; BWDKV (xt) loads them instead of recomputing S^T and dP^T.
     int xt, tsw;
+    int64_t grows;   // tape granule stride (rows)
     uint32_t* flags;
     float* tP;
     float* tS;
@@ -119,7 +122,7 @@ __device__ __forceinline__ void trace_tile(const Params& p, int j, int e) {
 
 constexpr size_t SCRATCH = 3 * 128 * 4 + 2 * 192 * 4;   // FWD row 1/l [3][128]; BWDKV column lse / D
 constexpr size_t SMEM_BYTES = 1024 + NST * SLOT + 4 * NSTG * STG + SCRATCH + 256;
-constexpr size_t SMEM_BYTES_XT = 1024 + NST_XT * SLOT_XT + 4 * NSTG * STG + SCRATCH + 256;
+constexpr size_t SMEM_BYTES_XT = 1024 + NST_XT * SLOT_XT + 4 * NSTG * STG + 256;
 static_assert(SMEM_BYTES <= 227 * 1024 && SMEM_BYTES_XT <= 227 * 1024, "shared memory plan");
 static_assert(3 * NST_XT * 8 + 12 * 8 + 4 <= 256, "barrier area");
 
@@ -267,7 +270,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     float* rowScale = scratch;                                          // FWD [3][128]
     float* colLse = scratch + 3 * 128;                                  // BWDKV [192] lse * log2e
     float* colD = colLse + 192;                                         // BWDKV [192]
-    uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(scratch) + SCRATCH);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(scratch) + (xt ? 0 : SCRATCH));
     uint64_t* full = bars;                // [nst] TMA bytes landed
     uint64_t* conv = bars + NST_XT;       // [nst] planes written (4 converter warps)
     uint64_t* empty = bars + 2 * NST_XT;  // [nst] MMAs done with the slot
@@ -290,7 +293,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     };
     // (the R1 accumulator sits at column 256, 128-aligned like the others)
     auto acc_col = [](int rid) -> uint32_t { return rid == 0 ? RACC : rid == 1 ? R0 : R1 + 64; };
-    const int npl = (NK + 127) / 128;   // tape slots per plane (128 rows each)
+    const int npl = (NK + TROWS - 1) / TROWS;   // tape slots per plane
     // (with ncw >= 2, the host's condition for xt, the last R0 / R1 accumulation is chunk ncw - 2)
 
     if (warp == 8) {
@@ -392,18 +395,15 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 trace_slot(p, k++, 0);
                 uint8_t* sp = slots + (size_t)st * slotb;
                 const Maps& mp = p.maps[T.rl];
-                if (kind == 2) {   // dS tape: query rows [128 a, 128 a + 128) of plane b (P, dS)
+                if (kind == 2) {   // dS tape: query rows [96 a, 96 a + 97) of plane b (P, dS)
                     if (a == 0 && b == 0 && p.dpoll) {   // BWDQ may still run: wait for these rows' tiles
                         const int64_t rowbase = (int64_t)T.u * p.L + T.r;
                         const int lo = max(0, T.m0 - w) / BM, hi = min(T.Lr - 1, T.m0 + BM - 1 + w) / BM;
                         for (int tq = lo; tq <= hi; ++tq) wait_flag(p.flags + rowbase + (int64_t)tq * BM * p.dil);
                         asm volatile("fence.proxy.async.global;" ::: "memory");
                     }
-                    const uint32_t box = 64u * (uint32_t)p.tsw * 4u;   // 64 rows
-                    const int nbx = NK - 128 * a > 64 ? 2 : 1;
-                    mbar_arrive_expect_tx(&full[st], nbx * box);
-                    for (int x = 0; x < nbx; ++x)
-                        tma_load_3d(sp + x * box, b ? &mp.ts : &mp.tp, &full[st], 0, T.m0 - w + 128 * a + 64 * x, T.u);
+                    mbar_arrive_expect_tx(&full[st], (uint32_t)(TBOX * p.tsw * 4));
+                    tma_load_4d(sp, b ? &mp.ts : &mp.tp, &full[st], 0, T.m0 - w + TROWS * a, T.u, 0);
                 } else if (kind == 0) {   // 32 columns: two 16-column boxes of each operand
                     const CUtensorMap* ma = b ? &mp.a2 : &mp.a1;
                     const CUtensorMap* mb = b ? &mp.b2 : &mp.b1;
@@ -658,7 +658,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                             split2(dv[2], dv[3], pk[2 * g4 + 1], pl[2 * g4 + 1]);
                             const int o = ob + 4 * g4;
                             if (p.xt && mrow < Lr && o >= 0 && o < p.tsw) {
-                                const size_t ro = (size_t)(rowbase + (int64_t)mrow * p.dil) * p.tsw + o;
+                                const size_t ro = ((size_t)(o >> 2) * p.grows + rowbase + (int64_t)mrow * p.dil) * 4;
                                 *reinterpret_cast<float4*>(p.tP + ro) = make_float4(pv[0], pv[1], pv[2], pv[3]);
                                 *reinterpret_cast<float4*>(p.tS + ro) = make_float4(dv[0], dv[1], dv[2], dv[3]);
                             }
@@ -677,7 +677,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     if (t == 0) st_release_gpu(p.flags + rowbase + (int64_t)m0 * p.dil, 1u);
                 }
             } else if (xt) {   // BWDKV from the dS tape: P^T -> R1 (hi | lo), then dS^T -> R0
-                const int tsw = p.tsw;
+
                 // walk positions (see walk): every segment holds 2 ncw nkb output blocks and 2 npl tape slots, plus P(0) in
                 // segment 0; P(j > 0) is the npl slots before the last dK chunk of segment j - 1
                 const int seg = nacc * nkb + 2 * npl;
@@ -697,7 +697,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         mbar_wait(&full[st], (uint32_t)(k / nst) & 1u);
                         if (t == 0 && b == 0) trace_tile(p, j, 11 + 3 * h);   // first tape slot landed
                         const float* sv = reinterpret_cast<const float*>(slots + (size_t)st * slotb);
-                        for (int c = 4 * b; c < 4 * b + 4 && c < nch; ++c) {
+                        for (int c = 3 * b; c < 3 * b + 3 && c < nch; ++c) {
                             if (c < c_lo || c > c_hi) {
                                 tmem_st16(dst + c * 32, zero16);
                                 tmem_st16(dst + c * 32 + 16, zero16);
@@ -705,19 +705,20 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                             }
 #pragma unroll
                             for (int hh = 0; hh < 2; ++hh) {
-                                // column n = n0 + e (query kb + n, tape row n - 128 b of the slot),
-                                // key t: entry t - n + 2w at float (kb + n) & 3 + t - n + 2w; in the
-                                // band iff e in [lo, hi].  Branch-free, loads back to back.
+                                // column n = n0 + e (query kb + n, tape row n - 96 b of the slot), key
+                                // t: offset o = (kb + n) & 3 + t - n + 2w, at float (o / 4) 4 TBOX +
+                                // (n - 96 b) 4 + o % 4 of the slot; in the band iff e in [lo, hi].
+                                // Branch-free, loads back to back.
                                 const int n0 = c * 32 + 16 * hh;
-                                const int a0 = (n0 - 128 * b) * tsw + t - n0 + 2 * w;
                                 const int lo = max(t - n0, -(kb + n0)), hi = min(t - n0 + 2 * w, Lr - 1 - (kb + n0));
-                                const int q3 = (kb + n0) & 3;
                                 uint32_t pk[8], pl[8];
                                 float x[16];
 #pragma unroll
                                 for (int e = 0; e < 16; ++e) {
+                                    const int n = n0 + e;
+                                    const int o = ((kb + n) & 3) + t - n + 2 * w;
                                     const bool ok = e >= lo && e <= hi;
-                                    const float xv = sv[ok ? a0 + e * (tsw - 1) + ((q3 + e) & 3) : 0];
+                                    const float xv = sv[ok ? (o >> 2) * (4 * TBOX) + (n - TROWS * b) * 4 + (o & 3) : 0];
                                     x[e] = ok ? xv : 0.f;
                                 }
 #pragma unroll
@@ -892,8 +893,8 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
             if (ok && ob2) ok = make_residue_map_f32(&m.ob2, ob2, L, d, units, dil, r, KB);
             if (ok && o2) ok = make_residue_map_f32(&m.o2, o2, L, d, units, dil, r, 32);
             if (ok && tape && MODE == BWDKV && d > CW) {
-                ok = make_residue_map_tape(&m.tp, tape->P, L, tape->tsw, units, dil, r, 64) &&
-                     make_residue_map_tape(&m.ts, tape->S, L, tape->tsw, units, dil, r, 64);
+                ok = make_residue_map_tape(&m.tp, tape->P, L, tape->tsw, units, dil, r, TBOX, tape->grows) &&
+                     make_residue_map_tape(&m.ts, tape->S, L, tape->tsw, units, dil, r, TBOX, tape->grows);
             }
             if (!ok) return cudaErrorInvalidValue;
         }
@@ -909,6 +910,7 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         if (tape && MODE != FWD && d > CW) {   // xt needs two output chunks (acc_rid alternation)
             p.xt = 1;
             p.tsw = tape->tsw;
+            p.grows = tape->grows;
             p.flags = tape->flags;
             p.tP = tape->P;
             p.tS = tape->S;

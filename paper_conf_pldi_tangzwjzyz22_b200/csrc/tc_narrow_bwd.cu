@@ -414,6 +414,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
         bool hn = nxt.next(p.sc, Tn);
         bool lse_settled = false;   // ld_lse_ready fell back to griddepcontrol.wait
         bool first_store = true;    // NQ launched early: wait for the preceding grid first
+        // NKV with the D hand-off: D is stored by the NQ grid, which this grid does not wait for
+        // (no griddepcontrol.wait), so it is read with ld.relaxed.gpu (at the coherence point,
+        // never from a possibly stale L1 line) one tile ahead and kept in a register until setup
+        float dnext = 0.f, lnext = 0.f;   // (lse likewise while the forward may still run: lsepoll)
         auto prefetch = [&](const Tile& X, int jx) {
             const int64_t rb = (int64_t)X.u * p.L + X.r;
             if (MODE == NKV) {
@@ -422,14 +426,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                     const bool ok = mc >= 0 && mc < X.Lr;
                     const int64_t off = ok ? rb + (int64_t)mc * p.dil : 0;
                     float* cl = colv + (jx & 1) * 2 * NK;
-                    cp_async4(cl + threadIdx.x, p.lse + off, ok ? 4u : 0u);
-                    cp_async4(cl + NK + threadIdx.x, p.D + off, ok ? 4u : 0u);
+                    if (p.lsepoll) lnext = ok ? ld_D_first(p.lse + off) : 0.f;
+                    else cp_async4(cl + threadIdx.x, p.lse + off, ok ? 4u : 0u);
+                    if (p.dpoll) dnext = ok ? ld_D_first(p.D + off) : 0.f;
+                    else cp_async4(cl + NK + threadIdx.x, p.D + off, ok ? 4u : 0u);
                 }
             } else {
                 const int mrow = X.m0 + t;
                 const bool ok = mrow < X.Lr;
-                cp_async4(lpre + (jx & 1) * 256 + threadIdx.x, p.lse + (ok ? rb + (int64_t)mrow * p.dil : 0),
-                          ok ? 4u : 0u);
+                if (p.lsepoll) lnext = ok ? ld_D_first(p.lse + rb + (int64_t)mrow * p.dil) : 0.f;
+                else cp_async4(lpre + (jx & 1) * 256 + threadIdx.x, p.lse + (ok ? rb + (int64_t)mrow * p.dil : 0),
+                               ok ? 4u : 0u);
             }
             cp_async_commit();
         };
@@ -451,16 +458,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             if (p.lsepoll) {   // lse rows the forward had not stored yet
                 if (MODE == NQ) {
                     float* cl = lpre + (jx & 1) * 256 + threadIdx.x;
+                    *cl = lnext;
                     if (__float_as_uint(*cl) == D_UNSET)
                         *cl = ld_lse_ready(p.lse + c.rowbase + (int64_t)(c.m0 + t) * p.dil, lse_settled);
                 } else if (threadIdx.x < NK) {
                     float* cl = colv + (jx & 1) * 2 * NK + threadIdx.x;
+                    *cl = lnext;
                     if (__float_as_uint(*cl) == D_UNSET)
                         *cl = ld_lse_ready(p.lse + c.rowbase + (int64_t)(c.kb + (int)threadIdx.x) * p.dil, lse_settled);
                 }
             }
             if (MODE == NKV && p.dpoll && threadIdx.x < NK) {   // D rows NQ had not stored yet
                 float* cd = colv + (jx & 1) * 2 * NK + NK + threadIdx.x;
+                *cd = dnext;
                 if (__float_as_uint(*cd) == D_UNSET)
                     *cd = ld_D_ready(p.D + c.rowbase + (int64_t)(c.kb + (int)threadIdx.x) * p.dil);
             }

@@ -68,19 +68,22 @@ inline bool make_residue_map_f32(CUtensorMap* m, const void* tensor, int64_t L, 
     return res == CUDA_SUCCESS;
 }
 
-// Residue view of a dS-tape plane (ftw::DsTape: fp32 rows of tsw floats, one per sequence row), a
-// {tsw x box_rows} box without swizzle (the softmax warps read it with plain shared loads).
+// Residue view of a dS-tape plane (ftw::DsTape): 16-byte granules, element (row R, granule G) at
+// float (G grows + R) 4 of the plane.  4-D: {4 floats, residue row m (stride dil granules), unit
+// (stride L granules), G (stride grows granules)}; a {4, box_rows, 1, tsw / 4} box lands in shared
+// memory as [G][box_rows][4] (box_rows odd multiple of 1 beyond a power of two, so that a warp
+// reading one entry per key row hits distinct banks).
 inline bool make_residue_map_tape(CUtensorMap* m, const void* plane, int64_t L, int64_t tsw,
-                                  int64_t units, int64_t dil, int64_t r, int box_rows) {
+                                  int64_t units, int64_t dil, int64_t r, int box_rows, int64_t grows) {
     auto enc = tmap_encoder();
     if (!enc) return false;
     const int64_t Lr = (L - r + dil - 1) / dil;
-    const char* base = static_cast<const char*>(plane) + r * tsw * 4;
-    cuuint64_t dims[3] = {(cuuint64_t)tsw, (cuuint64_t)Lr, (cuuint64_t)units};
-    cuuint64_t strides[2] = {(cuuint64_t)(dil * tsw * 4), (cuuint64_t)(L * tsw * 4)};
-    cuuint32_t box[3] = {(cuuint32_t)tsw, (cuuint32_t)box_rows, 1u};
-    cuuint32_t estr[3] = {1u, 1u, 1u};
-    CUresult res = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<char*>(base), dims,
+    const char* base = static_cast<const char*>(plane) + r * 16;
+    cuuint64_t dims[4] = {4, (cuuint64_t)Lr, (cuuint64_t)units, (cuuint64_t)(tsw / 4)};
+    cuuint64_t strides[3] = {(cuuint64_t)(dil * 16), (cuuint64_t)(L * 16), (cuuint64_t)(grows * 16)};
+    cuuint32_t box[4] = {4u, (cuuint32_t)box_rows, 1u, (cuuint32_t)(tsw / 4)};
+    cuuint32_t estr[4] = {1u, 1u, 1u, 1u};
+    CUresult res = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<char*>(base), dims,
                        strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return res == CUDA_SUCCESS;

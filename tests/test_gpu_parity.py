@@ -161,6 +161,16 @@ def test_dstape(ft, shape, dtype, tape, pdl):
         run_case(ft, WinAttnShape(*shape), dtype, "tc", seed=21)
 
 
+# FT_KNOB_DSTAPE = 2 forces the tape below d = 256 (the crossover measurement of DESIGN.md §10):
+# the bf16 band kernels' dual-accumulator dK/dV mode (d <= 128) and d = 64 with the narrow kernels off
+@pytest.mark.parametrize("shape", [(1, 2, 1000, 128, 32, 1), (1, 2, 700, 64, 16, 1), (2, 1, 900, 192, 9, 2)],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_dstape_forced(ft, shape):
+    with ft.knobs(dstape=2, narrow=0):
+        run_case(ft, WinAttnShape(*shape), "bf16", "tc", seed=22)
+        run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=22)
+
+
 @pytest.mark.parametrize("seed", [0, 1, 2])
 def test_default_path_seeds(ft, seed):
     run_case(ft, WinAttnShape(1, 2, 384, 64, 32, 1), "bf16", None, seed=seed)
@@ -463,7 +473,7 @@ MIXED = [
     (1, 4, 300, 512, 32, 4, 2, "bf16"),    # d = 512 band kernels
     (2, 4, 300, 256, 32, 4, 2, "f32"),     # fp32 tensor cores with the dS tape: per-slice workspace rows
     (1, 4, 700, 512, 32, 4, 2, "f32"),     # C2a_mix-like, fp32
-    (2, 4, 300, 256, 32, 4, 2, "bf16"),    # bf16 band kernels with the dS tape
+    (2, 4, 300, 384, 32, 4, 2, "bf16"),    # bf16 band kernels with the dS tape (d > 256)
 ]
 
 

@@ -14,9 +14,17 @@ for shape, dt in [((1, 2, 300, 64, 32, 3), "bf16"), ((1, 4, 1500, 64, 32, 1), "b
                   ((1, 2, 700, 64, 20, 5), "bf16"), ((1, 1, 200, 512, 32, 1), "bf16"),
                   ((1, 1, 600, 64, 100, 2), "bf16"), ((1, 1, 500, 128, 80, 1), "bf16"),
                   ((1, 1, 130, 64, 8, 1), "f32"), ((1, 2, 300, 512, 32, 1), "f32"),
-                  ((1, 2, 257, 128, 17, 3), "f32"), ((1, 1, 300, 192, 8, 1), "f32")]:
+                  ((1, 2, 257, 128, 17, 3), "f32"), ((1, 1, 300, 192, 8, 1), "f32"),
+                  ((1, 1, 500, 384, 32, 1), "bf16"), ((1, 2, 400, 256, 16, 2), "f32")]:   # last two: dS tape
     s = WinAttnShape(*shape)
     x = make_inputs(s, 0, dt)
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    o, l = ft.fwd(q, k, v, s.w, s.dilation)
+    ft.bwd(q, k, v, o, l, g, s.w, s.dilation)
+# dS tape forced below its threshold: bf16 dual-accumulator dK/dV kernel, narrow kernels off
+with ft.knobs(dstape=2, narrow=0):
+    s = WinAttnShape(1, 2, 500, 128, 32, 1)
+    x = make_inputs(s, 0, "bf16")
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
     o, l = ft.fwd(q, k, v, s.w, s.dilation)
     ft.bwd(q, k, v, o, l, g, s.w, s.dilation)

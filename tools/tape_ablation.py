@@ -79,14 +79,16 @@ DS_CASES = [(f"d{d}_w{w}", 1, max(1, 16 * 64 // d), 8192, d, w, 1)
                                                                ("C5_w32", 64, 1, 32768, 64, 32, 1)]
 
 
-def run_ds(name, B, H, L, d, w, dil):
+def run_ds(name, B, H, L, d, w, dil, dt=torch.float32):
     dev = torch.device("cuda:0")
-    q, k, v, g = [torch.rand(B, H, L, d, device=dev) * 2 - 1 for _ in range(4)]
+    q, k, v, g = [(torch.rand(B, H, L, d, device=dev) * 2 - 1).to(dt) for _ in range(4)]
     out, lse = ft.fwd(q, k, v, w, dil)
-    res = {"case": name, "dtype": "f32", "shape": [B, H, L, d, w, dil], "family": "dS tape (fp32 tensor cores)",
+    res = {"case": name, "dtype": "f32" if dt == torch.float32 else "bf16", "shape": [B, H, L, d, w, dil],
+           "family": "dS tape (tensor cores)",
            "tape_bytes_per_row": 2 * 4 * ((2 * min(w, L) + 4 + 3) // 4 * 4)}
     for leg in (0, 1):
-        with ft.knobs(dstape=leg):
+        # leg 1 forces the tape (knob value 2) below the library's d >= 256 threshold too
+        with ft.knobs(dstape=2 * leg):
             res[["recompute_bwd_ms", "dstape_bwd_ms"][leg]] = timed(lambda: ft.bwd(q, k, v, out, lse, g, w, dil))
     res["dstape_speedup"] = res["recompute_bwd_ms"] / res["dstape_bwd_ms"]
     print(json.dumps(res), flush=True)
@@ -99,8 +101,11 @@ def main():
     ap.add_argument("--dstape-only", action="store_true")
     a = ap.parse_args()
     FLUSH = torch.empty(256 << 20, dtype=torch.uint8, device="cuda:0")
-    for c in DS_CASES:
-        run_ds(*c)
+    for dt in (torch.float32, torch.bfloat16):
+        for c in DS_CASES:
+            if dt == torch.bfloat16 and c[4] == 64 and c[5] <= 32:
+                continue   # d = 64, w <= 32 runs on the narrow kernels (no tape)
+            run_ds(*c, dt=dt)
     if a.dstape_only:
         return
     for c in TC_CASES[-4:] if a.quick else TC_CASES:
