@@ -151,6 +151,35 @@ def test_debug_knobs(lib):
     with ft.knobs(narrow=0, pdl=0):
         assert ft.debug_get("narrow") == 0 and ft.debug_get("pdl") == 0
     assert ft.debug_get("narrow") == 1 and ft.debug_get("pdl") == 1
+    # dS tape knob: 0 off, 1 where it pays (default), 2 forced; nothing else
+    assert lib.ft_winattn_debug_set(5, 3) == INVALID
+    assert ft.debug_get("dstape") == 1
+    with ft.knobs(dstape=2):
+        assert ft.debug_get("dstape") == 2
+
+
+def test_workspace_dstape_layout(lib):
+    """The backward workspace (include/ft_winattn.h): D (fp32 per row) always; the dS tape regions
+    -- a flag word per row and two fp32 planes of tsw = 4 ceil((2w + 4) / 4) floats per row, each
+    region rounded up to 256 bytes -- exactly where the tensor-core kernels use the tape (fp32
+    d >= 256, bf16 band kernels d > 256; any d they support with the knob at 2)."""
+    r256 = lambda x: (x + 255) // 256 * 256
+    def ws(B, H, L, d, w, dil, dt):
+        return lib.ft_winattn_bwd_workspace_bytes(B, H, L, d, w, dil, dt)
+    F32, BF16 = ft.FT_F32, ft.FT_BF16
+    rows = 2 * 3 * 1000
+    tape = lambda w: r256(rows * 4) + r256(rows * 4) + 2 * r256(rows * 4 * ((2 * w + 4 + 3) // 4 * 4))
+    assert ws(2, 3, 1000, 512, 32, 1, F32) == tape(32)        # fp32, d >= 256
+    assert ws(2, 3, 1000, 256, 5, 3, F32) == tape(5)
+    assert ws(2, 3, 1000, 128, 32, 1, F32) == r256(rows * 4)  # fp32 d = 128: recompute
+    assert ws(2, 3, 1000, 512, 32, 1, BF16) == tape(32)       # bf16 band kernels, d > 256
+    assert ws(2, 3, 1000, 256, 32, 1, BF16) == r256(rows * 4) # bf16 d = 256: recompute
+    assert ws(2, 3, 1000, 512, 100, 1, F32) == r256(rows * 4) # w > 32: CUDA-core fp32 path
+    assert ws(2, 3, 1000, 512, 100, 1, BF16) == r256(rows * 4) # w > 64: chunked kernels
+    with ft.knobs(dstape=2):
+        assert ws(2, 3, 1000, 256, 32, 1, BF16) == tape(32)
+    with ft.knobs(dstape=0):   # knob 0 keeps the size (the call then ignores the tape regions)
+        assert ws(2, 3, 1000, 512, 32, 1, F32) == tape(32)
 
 
 def test_workspace_and_plan(lib):
