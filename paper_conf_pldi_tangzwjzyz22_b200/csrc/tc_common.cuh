@@ -384,6 +384,22 @@ __host__ __device__ constexpr uint32_t idesc_f16(int M, int N, bool a_mn, bool b
     return (1u << 4) | ((a_mn ? 1u : 0u) << 15) | ((b_mn ? 1u : 0u) << 16) |
            ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
+// Blackwell packed fp32 pairs (one FFMA2 / FADD2 instruction for two lanes of work):
+// (r0, r1) = (a0 b + c, a1 b + c) and (s0, s1) += (a0, a1)
+__device__ __forceinline__ void ffma2_bc(float a0, float a1, float b, float c, float& r0, float& r1) {
+    asm("{\n\t.reg .b64 aa, bb, cc, rr;\n\t"
+        "mov.b64 aa, {%2, %3};\n\tmov.b64 bb, {%4, %4};\n\tmov.b64 cc, {%5, %5};\n\t"
+        "fma.rn.f32x2 rr, aa, bb, cc;\n\tmov.b64 {%0, %1}, rr;\n\t}"
+        : "=f"(r0), "=f"(r1)
+        : "f"(a0), "f"(a1), "f"(b), "f"(c));
+}
+__device__ __forceinline__ void fadd2_acc(float& s0, float& s1, float a0, float a1) {
+    asm("{\n\t.reg .b64 ss, aa;\n\t"
+        "mov.b64 ss, {%0, %1};\n\tmov.b64 aa, {%2, %3};\n\t"
+        "add.rn.f32x2 ss, ss, aa;\n\tmov.b64 {%0, %1}, ss;\n\t}"
+        : "+f"(s0), "+f"(s1)
+        : "f"(a0), "f"(a1));
+}
 __device__ __forceinline__ uint32_t pack_f16x2(float lo, float hi) {
     __half2 h = __floats2half2_rn(lo, hi);   // .x = lo (low 16 bits)
     return *reinterpret_cast<uint32_t*>(&h);

@@ -413,11 +413,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                     }
                     return fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * LOG2E;
                 };
-                // P = exp2(S - mref) for my half -> operand; returns my half's row sum and
-                // the max of my half's raw scores (log2 domain) in cmax
-                auto exp_sweep = [&](float mref, float& cmax) -> float {
+                // P = exp2(S - mref) for my half -> operand; returns my half's row sum.  Per pair
+                // of entries: one FFMA2 (s log2e - mref), two ex2, one FADD2 (the two partial
+                // sums), one pack -- no running max: the rescale test below uses the row sum
+                // (every P <= the sum of the chunk's P).
+                auto exp_sweep = [&](float mref) -> float {
                     float lc[2] = {0.f, 0.f};
-                    float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
                     if (!any_live) {
                         if (PSM) { st_p_sub(Pb, t, sp, zero16); st_p_sub(Pb, t, sp + 1, zero16); }
                         else { tmem_st16(tS + sp * 16, zero16); tmem_st16(tS + sp * 16 + 16, zero16); }
@@ -430,21 +431,25 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                             uint32_t pk[16];
 #pragma unroll
                             for (int e = 0; e < 32; e += 2) {
-                                const float s0 = __uint_as_float(rr[x][e]), s1 = __uint_as_float(rr[x][e + 1]);
-                                m4[e & 3] = fmaxf(m4[e & 3], s0);
-                                m4[(e + 1) & 3] = fmaxf(m4[(e + 1) & 3], s1);
-                                const float p0 = fast_exp2(fmaf(s0, LOG2E, -mref));
-                                const float p1 = fast_exp2(fmaf(s1, LOG2E, -mref));
-                                lc[0] += p0;
-                                lc[1] += p1;
+                                float a0, a1;
+                                ffma2_bc(__uint_as_float(rr[x][e]), __uint_as_float(rr[x][e + 1]), LOG2E, -mref, a0, a1);
+                                const float p0 = fast_exp2(a0), p1 = fast_exp2(a1);
+                                fadd2_acc(lc[0], lc[1], p0, p1);
                                 pk[e / 2] = pack_bf16x2(p0, p1);
                             }
                             if (PSM) st_p_sub(Pb, t, sp + x, pk);
                             else tmem_st16(tS + (sp + x) * 16, pk);
                         }
                     }
-                    cmax = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * LOG2E;
                     return lc[0] + lc[1];
+                };
+                // row sum of the whole chunk (both halves), exchanged with the partner warp
+                auto xsum = [&](float mine) -> float {
+                    float* slot = cmx + (xc & 1) * 256;
+                    slot[hf * 128 + t] = mine;
+                    named_bar_sync(1 + wq, 64);
+                    ++xc;
+                    return slot[t] + slot[128 + t];
                 };
                 // move the running max of rows whose chunk max exceeds it by more than the
                 // threshold; where such a row has already accumulated, the half-0 warp rescales
@@ -475,17 +480,22 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                 };
                 // rows without a running max yet (the first chunk): exact chunk max first
                 if (__any_sync(0xffffffffu, ms == -INFINITY)) move_max(xmax(half_max()));
-                // optimistic sweep at the running max; both warps redo the chunk in the rare
-                // case that some row's chunk max exceeds it by more than the threshold
-                float cmh, lc;
+                // optimistic sweep at the running max.  If some row's chunk sum exceeds
+                // 2^(RESCALE_LOG2 - 6) -- only then can one of its P exceed the threshold -- both
+                // warps take the chunk's exact max, move the running max where it exceeds it by
+                // more than the threshold, and redo the chunk (rare: m starts at the middle
+                // chunk's exact max)
+                float lc;
                 unsigned long long q1 = tr ? gtime() : 0, q2 = 0;
-#pragma unroll 1
-                for (;;) {
-                    lc = exp_sweep(ms == -INFINITY ? 0.f : ms, cmh);
-                    if (tr) q2 = gtime();
-                    const float cm = xmax(cmh);
-                    if (!__any_sync(0xffffffffu, cm > ms + RESCALE_LOG2)) break;
-                    move_max(cm);
+                lc = exp_sweep(ms == -INFINITY ? 0.f : ms);
+                if (tr) q2 = gtime();
+                const float rowsum = xsum(lc);
+                if (__any_sync(0xffffffffu, !(rowsum <= exp2f(RESCALE_LOG2 - 6.f)))) {   // (NaN: check)
+                    const float cm = xmax(half_max());
+                    if (__any_sync(0xffffffffu, cm > ms + RESCALE_LOG2)) {
+                        move_max(cm);
+                        lc = exp_sweep(ms == -INFINITY ? 0.f : ms);
+                    }
                 }
                 if (tr) { fine[1] += q2 - q1; fine[2] += gtime() - q2; }
                 l += lc;
