@@ -98,6 +98,9 @@ struct Params {
     int d, w, dil, NK, nsl;
     SchedParams sc;
     int dpoll;    // BWDKV: poll D row by row (BWDQ marked its rows D_UNSET, PDL launch)
+    // lse hand-off inside ft_winattn_fwd_bwd (tc_band.cu's scheme): FWD marks its lse rows
+    // D_UNSET and triggers, BWDQ (PDL) and a recomputing BWDKV read lse with ld_lse_ready
+    int lsepoll;
     // dS tape (ftw::DsTape, internal.h): BWDQ stores P and dS of every band entry and sets the
     // flag of each tile it finished; BWDKV (xt) loads them instead of recomputing S^T and dP^T.
     int xt, tsw;
@@ -259,7 +262,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         __threadfence();
         __syncthreads();
     }
-    if (MODE == BWDQ) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    if (MODE == FWD && p.lsepoll) {   // lse rows unset, then let the dQ kernel (PDL) launch
+        TileCursor cr(p.sc);
+        Tile T;
+        while (cr.next(p.sc, T)) {
+            const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+            for (int i = threadIdx.x; i < BM && T.m0 + i < T.Lr; i += NTHREADS)
+                reinterpret_cast<uint32_t*>(p.lse)[rowbase + (int64_t)(T.m0 + i) * p.dil] = D_UNSET;
+        }
+        __threadfence();
+        __syncthreads();
+    }
+    if (MODE == BWDQ || (MODE == FWD && p.lsepoll)) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 
     const bool xt = MODE == BWDKV && p.xt;
     const int nst = xt ? NST_XT : NST;
@@ -538,6 +552,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         Tile T;
         int j = 0;
         if (MODE == BWDKV && !p.dpoll) asm volatile("griddepcontrol.wait;" ::: "memory");
+        bool lse_settled = false;   // ld_lse_ready fell back to griddepcontrol.wait
         while (cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t, kb = m0 - w;
             const int64_t rowbase = (int64_t)T.u * p.L + T.r;
@@ -546,7 +561,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 for (int n = t; n < NK; n += 128) {
                     const int mc = kb + n;
                     const bool ok = mc >= 0 && mc < Lr;
-                    colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
+                    colLse[n] = !ok ? 0.f
+                                : (p.lsepoll ? ld_lse_ready(p.lse + rowbase + (int64_t)mc * p.dil, lse_settled)
+                                             : p.lse[rowbase + (int64_t)mc * p.dil]) * LOG2E;
                     float dv = 0.f;
                     if (ok) dv = p.dpoll ? ld_D_ready(p.D + rowbase + (int64_t)mc * p.dil) : p.D[rowbase + (int64_t)mc * p.dil];
                     colD[n] = dv;
@@ -611,7 +628,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 if (t == 0) trace_tile(p, j, 1);
                 if (mrow < Lr) p.lse[rowbase + (int64_t)mrow * p.dil] = (mxs + log2f(sum)) * LN2;
             } else if (MODE == BWDQ) {
-                const float lse2 = mrow < Lr ? p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E : 0.f;
+                const float lse2 = mrow >= Lr ? 0.f
+                                   : (p.lsepoll ? ld_lse_ready(p.lse + rowbase + (int64_t)mrow * p.dil, lse_settled)
+                                                : p.lse[rowbase + (int64_t)mrow * p.dil]) * LOG2E;
                 float D = 0.f;
                 for (int c = c_lo; c <= c_hi; ++c) {   // pass 1: D = sum_j P_ij dP_ij
 #pragma unroll
@@ -922,7 +941,12 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         dim3 grid((unsigned)(total < num_sms32() ? total : num_sms32()));
         const size_t smem = MODE == BWDKV && p.xt ? SMEM_BYTES_XT : SMEM_BYTES;
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
-        if (MODE == BWDKV && r0 == 0 && p.dpoll) {   // directly after this call's last BWDQ launch
+        // lse hand-off: one launch of residues on each side (nres <= RES_PER_LAUNCH) -- the
+        // dQ kernel's launch follows the forward's only launch
+        p.lsepoll = lsepoll_enabled() && nres <= RES_PER_LAUNCH && lsepoll_worth(total, num_sms32()) &&
+                    !(MODE == BWDKV && p.xt);   // the tape dK/dV kernel reads no lse
+        if ((MODE == BWDKV && r0 == 0 && p.dpoll) || (MODE == BWDQ && p.lsepoll)) {
+            // BWDKV directly after this call's last BWDQ launch; BWDQ after the forward
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = grid;
             cfg.blockDim = dim3(NTHREADS);

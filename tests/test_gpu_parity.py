@@ -620,15 +620,17 @@ def test_d_handoff_stale_workspace(ft, shape):
 @pytest.mark.parametrize("shape", [(1, 2, 700, 512, 32, 1), (1, 3, 900, 512, 20, 3), (1, 8, 10000, 512, 32, 1),
                                    (1, 2, 3000, 512, 32, 11), (2, 3, 1500, 128, 48, 1),
                                    (1, 8, 4096, 64, 32, 1), (1, 2, 700, 64, 32, 1), (1, 3, 5000, 64, 16, 3),
-                                   (1, 48, 2048, 64, 32, 1), (1, 2, 900, 64, 100, 1)],
+                                   (1, 48, 2048, 64, 32, 1), (1, 2, 900, 64, 100, 1), (1, 4, 2000, 128, 32, 1)],
                          ids=lambda s: "x".join(map(str, s)))
-def test_fwd_bwd_handoff(ft, shape):
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_fwd_bwd_handoff(ft, shape, dtype):
     """ft_winattn_fwd_bwd: its forward marks the lse rows and its dQ kernel (PDL) reads each row as
-    the forward stores it (tc_common.cuh ld_lse_ready).  The result
-    must be bit-identical to separate ft_winattn_fwd + ft_winattn_bwd calls and to the schedule
-    without programmatic dependent launch."""
+    the forward stores it (tc_common.cuh ld_lse_ready); in fp32 also
+    the recomputing dK/dV kernel (d < 256, no dS tape).  The result must be bit-identical to
+    separate ft_winattn_fwd + ft_winattn_bwd calls and to the schedule without programmatic
+    dependent launch."""
     sh = WinAttnShape(*shape)
-    x = make_inputs(sh, 41, "bf16")
+    x = make_inputs(sh, 41, dtype)
     dev = torch.device("cuda:0")
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
     o0, l0 = ft.fwd(q, k, v, sh.w, sh.dilation)
