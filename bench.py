@@ -353,7 +353,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work (cpu_baseline)")
     ap.add_argument("--ref-rows", type=int, default=0, help="oracle rows per reference step (0 = full L)")
-    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--sg-steps", type=int, default=3, help="N > 1: NCCL scatter/gather end-to-end steps")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
