@@ -65,7 +65,7 @@ enum { FWD = 0, BWDQ = 1, BWDKV = 2 };
 constexpr int BM = 128;
 constexpr int KB = 64;                    // keys per output block
 constexpr int CW = 128;                   // output columns per accumulation
-constexpr int NST = 4;                    // ring slots
+constexpr int NST = 5;                    // ring slots
 constexpr uint32_t SLOT = 40 * 1024;      // fp32 score slice (128 + 192 rows x 32 cols) / 64 x 128 block
 // BWDKV with the dS tape streams no score slices: six 32 KB slots (a 96-row slice of one tape
 // plane, [tsw / 4][97][4] floats with tsw <= 68, or a 64 x 128 output block), so the tape slots of
@@ -75,7 +75,8 @@ constexpr uint32_t SLOT_XT = 32 * 1024;
 constexpr int TROWS = 96, TBOX = TROWS + 1;   // tape rows per slot; box rows (odd row stride: no bank conflicts)
 static_assert(TBOX * 68 * 4 <= (int)SLOT_XT, "tape slot");
 constexpr uint32_t STG = 32 * 128;        // one epilogue warp's 32-row x 32-col fp32 staging box
-constexpr int NSTG = 2;                   // staging boxes per epilogue warp
+constexpr int NSTG = 1;                   // staging boxes per epilogue warp (five ring slots fit)
+constexpr int NSTG_XT = 2;                // in the tape dK/dV kernel (its eight drains per tile)
 constexpr int NTHREADS = 512;
 constexpr int NCONV = 6;                  // converter warps
 constexpr int RES_PER_LAUNCH = 8;
@@ -125,7 +126,7 @@ __device__ __forceinline__ void trace_tile(const Params& p, int j, int e) {
 
 constexpr size_t SCRATCH = 3 * 128 * 4 + 2 * 192 * 4;   // FWD row 1/l [3][128]; BWDKV column lse / D
 constexpr size_t SMEM_BYTES = 1024 + NST * SLOT + 4 * NSTG * STG + SCRATCH + 256;
-constexpr size_t SMEM_BYTES_XT = 1024 + NST_XT * SLOT_XT + 4 * NSTG * STG + 256;
+constexpr size_t SMEM_BYTES_XT = 1024 + NST_XT * SLOT_XT + 4 * NSTG_XT * STG + 256;
 static_assert(SMEM_BYTES <= 227 * 1024 && SMEM_BYTES_XT <= 227 * 1024, "shared memory plan");
 static_assert(3 * NST_XT * 8 + 12 * 8 + 4 <= 256, "barrier area");
 
@@ -279,8 +280,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     const int nst = xt ? NST_XT : NST;
     const uint32_t slotb = xt ? SLOT_XT : SLOT;
     uint8_t* slots = smem;
-    uint8_t* stg = smem + nst * slotb;                                  // [4 warps][NSTG] fp32 boxes
-    float* scratch = reinterpret_cast<float*>(stg + 4 * NSTG * STG);
+    const int nstg = xt ? NSTG_XT : NSTG;
+    uint8_t* stg = smem + nst * slotb;                                  // [4 warps][nstg] fp32 boxes
+    float* scratch = reinterpret_cast<float*>(stg + 4 * nstg * STG);
     float* rowScale = scratch;                                          // FWD [3][128]
     float* colLse = scratch + 3 * 128;                                  // BWDKV [192] lse * log2e
     float* colD = colLse + 192;                                         // BWDKV [192]
@@ -797,7 +799,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     } else if (warp < 8) {   // ----------------------------------------------- epilogue warps
         const int ew = warp - 4;   // TMEM lanes 32 ew ..
         const uint32_t tlane = tbase + ((uint32_t)(ew * 32) << 16);
-        uint8_t* mystg = stg + ew * NSTG * STG;
+        uint8_t* mystg = stg + ew * nstg * STG;
         TileCursor cur(p.sc);
         Tile T;
         int j = 0, sidx = 0;
@@ -832,8 +834,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         warp_arrive(&o_empty[rid]);
                         if (xt && a % ncw == ncw - 2) warp_arrive(&xfree[a < ncw ? 1 : 0]);
                     }
-                    uint8_t* sb = mystg + (sidx % NSTG) * STG;
-                    if (lane == 0 && sidx >= NSTG) tma_store_wait_read<NSTG - 1>();
+                    uint8_t* sb = mystg + (sidx % nstg) * STG;
+                    if (lane == 0 && sidx >= nstg) {
+                        if (nstg == 2) tma_store_wait_read<1>();
+                        else tma_store_wait_read<0>();
+                    }
                     __syncwarp();
 #pragma unroll
                     for (int g = 0; g < 8; ++g) {
