@@ -400,6 +400,22 @@ __device__ __forceinline__ void fadd2_acc(float& s0, float& s1, float a0, float 
         : "+f"(s0), "+f"(s1)
         : "f"(a0), "f"(a1));
 }
+// general packed pairs: (r0, r1) = (a0 b0 + c0, a1 b1 + c1), (a0 b0, a1 b1), (a0 + b0, a1 + b1)
+__device__ __forceinline__ void ffma2(float a0, float a1, float b0, float b1, float c0, float c1, float& r0,
+                                      float& r1) {
+    asm("{\n\t.reg .b64 aa, bb, cc, rr;\n\t"
+        "mov.b64 aa, {%2, %3};\n\tmov.b64 bb, {%4, %5};\n\tmov.b64 cc, {%6, %7};\n\t"
+        "fma.rn.f32x2 rr, aa, bb, cc;\n\tmov.b64 {%0, %1}, rr;\n\t}"
+        : "=f"(r0), "=f"(r1)
+        : "f"(a0), "f"(a1), "f"(b0), "f"(b1), "f"(c0), "f"(c1));
+}
+__device__ __forceinline__ void fmul2(float a0, float a1, float b0, float b1, float& r0, float& r1) {
+    asm("{\n\t.reg .b64 aa, bb, rr;\n\t"
+        "mov.b64 aa, {%2, %3};\n\tmov.b64 bb, {%4, %5};\n\t"
+        "mul.rn.f32x2 rr, aa, bb;\n\tmov.b64 {%0, %1}, rr;\n\t}"
+        : "=f"(r0), "=f"(r1)
+        : "f"(a0), "f"(a1), "f"(b0), "f"(b1));
+}
 __device__ __forceinline__ uint32_t pack_f16x2(float lo, float hi) {
     __half2 h = __floats2half2_rn(lo, hi);   // .x = lo (low 16 bits)
     return *reinterpret_cast<uint32_t*>(&h);

@@ -458,16 +458,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     uint32_t ph[16], pl[16], pp[16];
                     float dd[2] = {0.f, 0.f};
 #pragma unroll
-                    for (int e = 0; e < 32; e += 2) {
-                        const float p0 = fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2));
-                        const float p1 = fast_exp2(fmaf(__uint_as_float(rs[e + 1]), LOG2E, -lse2));
+                    for (int e = 0; e < 32; e += 2) {   // packed f32x2 pairs: FFMA2 / FMUL2
+                        const float dp0 = __uint_as_float(rd[e]), dp1 = __uint_as_float(rd[e + 1]);
+                        float a0, a1;
+                        ffma2_bc(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, -lse2, a0, a1);
+                        const float p0 = fast_exp2(a0), p1 = fast_exp2(a1);
                         if (wqc) {
-                            dd[0] = fmaf(p0, __uint_as_float(rd[e]), dd[0]);
-                            dd[1] = fmaf(p1, __uint_as_float(rd[e + 1]), dd[1]);
+                            ffma2(p0, p1, dp0, dp1, dd[0], dd[1], dd[0], dd[1]);
                             pp[e / 2] = pack_bf16x2(p0, p1);
                         }
-                        split_bf16x2(p0 * (__uint_as_float(rd[e]) - Dsub), p1 * (__uint_as_float(rd[e + 1]) - Dsub),
-                                     ph[e / 2], pl[e / 2]);
+                        float q0, q1, r0, r1;
+                        ffma2_bc(dp0, dp1, 1.f, -Dsub, q0, q1);   // dP - D (exact: a single rounding)
+                        fmul2(p0, p1, q0, q1, r0, r1);
+                        split_bf16x2(r0, r1, ph[e / 2], pl[e / 2]);
                     }
                     if (wqc) Dex += dd[0] + dd[1];
                     tmem_st16(xs, ph);
@@ -481,11 +484,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                         const float4 cd = *reinterpret_cast<const float4*>(&colD[h0 + (e & ~3)]);
                         const float l0 = (e & 2) ? cl.z : cl.x, l1 = (e & 2) ? cl.w : cl.y;
                         const float dd0 = (e & 2) ? cd.z : cd.x, dd1 = (e & 2) ? cd.w : cd.y;
-                        const float p0 = fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -l0));
-                        const float p1 = fast_exp2(fmaf(__uint_as_float(rs[e + 1]), LOG2E, -l1));
+                        float a0, a1, q0, q1, r0, r1;
+                        ffma2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, LOG2E, -l0, -l1, a0, a1);
+                        const float p0 = fast_exp2(a0), p1 = fast_exp2(a1);
                         pk[e / 2] = pack_bf16x2(p0, p1);
-                        split_bf16x2(p0 * (__uint_as_float(rd[e]) - dd0), p1 * (__uint_as_float(rd[e + 1]) - dd1),
-                                     ph[e / 2], pl[e / 2]);
+                        ffma2(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, 1.f, -dd0, -dd1, q0, q1);
+                        fmul2(p0, p1, q0, q1, r0, r1);
+                        split_bf16x2(r0, r1, ph[e / 2], pl[e / 2]);
                     }
                     tmem_st16(xs, pk);
                     tmem_st16(xd, ph);
