@@ -551,10 +551,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             if (MODE == NQ) {
                 float dpart[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-                for (int e = 0; e < 48; ++e) {
-                    const float pv = ((bits >> e) & 1ull) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f;
-                    rs[e] = __float_as_uint(pv);
-                    dpart[e & 3] = fmaf(pv, __uint_as_float(rd[e]), dpart[e & 3]);
+                for (int e = 0; e < 48; e += 2) {   // packed f32x2 pairs (FFMA2)
+                    float a0, a1;
+                    ffma2_bc(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, -lse2, a0, a1);
+                    const float p0 = ((bits >> e) & 1ull) ? fast_exp2(a0) : 0.f;
+                    const float p1 = ((bits >> (e + 1)) & 1ull) ? fast_exp2(a1) : 0.f;
+                    rs[e] = __float_as_uint(p0);
+                    rs[e + 1] = __float_as_uint(p1);
+                    const int q = e & 2;
+                    ffma2(p0, p1, __uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), dpart[q], dpart[q + 1],
+                          dpart[q], dpart[q + 1]);
                 }
                 float* dxb = dx + (j & 1) * 2 * BM;
                 dxb[h * BM + t] = (dpart[0] + dpart[1]) + (dpart[2] + dpart[3]);
@@ -566,10 +572,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 const float* tab = hscale + (j & 1) * NK + c0;
                 float mx = 0.f;
 #pragma unroll
-                for (int e = 0; e < 48; ++e) {
-                    const float dsv = __uint_as_float(rs[e]) * (__uint_as_float(rd[e]) - Dv) * tab[e];
-                    rs[e] = __float_as_uint(dsv);
-                    mx = fmaxf(mx, fabsf(dsv));
+                for (int e = 0; e < 48; e += 2) {
+                    float q0, q1, r0, r1;
+                    ffma2_bc(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, -Dv, q0, q1);
+                    fmul2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), q0, q1, r0, r1);
+                    fmul2(r0, r1, tab[e], tab[e + 1], r0, r1);
+                    rs[e] = __float_as_uint(r0);
+                    rs[e + 1] = __float_as_uint(r1);
+                    mx = fmaxf(mx, fmaxf(fabsf(r0), fabsf(r1)));
                 }
                 float* mxb = mxh + (j & 1) * 2 * BM;
                 mxb[h * BM + t] = mx;
@@ -578,8 +588,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 row_pow2(fmaxf(mxb[t], mxb[BM + t]), up, down);
                 cs.rsc = down;
 #pragma unroll
-                for (int e = 0; e < 48; e += 2)
-                    pk[e / 2] = pack_f16x2(__uint_as_float(rs[e]) * up, __uint_as_float(rs[e + 1]) * up);
+                for (int e = 0; e < 48; e += 2) {
+                    float r0, r1;
+                    fmul2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), up, up, r0, r1);
+                    pk[e / 2] = pack_f16x2(r0, r1);
+                }
                 // the dS buffer is free once out(j-1) completed
                 if (j >= 1) mbar_wait(&acc_full[(j - 1) & 1], ((j - 1) >> 1) & 1);
                 if (tr) trace_ev(p, j, 6);
@@ -602,12 +615,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                     const float dvv[4] = {d4.x, d4.y, d4.z, d4.w};
                     float pv[4];
 #pragma unroll
-                    for (int x = 0; x < 4; ++x) {
+                    for (int x = 0; x < 4; x += 2) {   // packed f32x2 pairs
                         const int e = 4 * e4 + x;
-                        pv[x] = ((bits >> e) & 1ull) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lv[x])) : 0.f;
-                        const float dsv = pv[x] * (__uint_as_float(rd[e]) - dvv[x]) * tab[e];
-                        rd[e] = __float_as_uint(dsv);
-                        mx = fmaxf(mx, fabsf(dsv));
+                        float a0, a1, q0, q1, r0, r1;
+                        ffma2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, LOG2E, -lv[x], -lv[x + 1], a0, a1);
+                        pv[x] = ((bits >> e) & 1ull) ? fast_exp2(a0) : 0.f;
+                        pv[x + 1] = ((bits >> (e + 1)) & 1ull) ? fast_exp2(a1) : 0.f;
+                        ffma2(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, 1.f, -dvv[x], -dvv[x + 1], q0, q1);
+                        fmul2(pv[x], pv[x + 1], q0, q1, r0, r1);
+                        fmul2(r0, r1, tab[e], tab[e + 1], r0, r1);
+                        rd[e] = __float_as_uint(r0);
+                        rd[e + 1] = __float_as_uint(r1);
+                        mx = fmaxf(mx, fmaxf(fabsf(r0), fabsf(r1)));
                     }
                     pk[2 * e4] = pack_bf16x2(pv[0], pv[1]);
                     pk[2 * e4 + 1] = pack_bf16x2(pv[2], pv[3]);
@@ -620,8 +639,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 row_pow2(fmaxf(mxb[t], mxb[BM + t]), up, down);
                 cs.rsc = down;
 #pragma unroll
-                for (int e = 0; e < 48; e += 2)
-                    pk2[e / 2] = pack_f16x2(__uint_as_float(rd[e]) * up, __uint_as_float(rd[e + 1]) * up);
+                for (int e = 0; e < 48; e += 2) {
+                    float r0, r1;
+                    fmul2(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), up, up, r0, r1);
+                    pk2[e / 2] = pack_f16x2(r0, r1);
+                }
                 // P^T (bf16) | dS^T (fp16) over S^T
                 st_operand(tS, pk);
                 st_operand(tS + 96, pk2);
