@@ -196,21 +196,19 @@ __device__ __forceinline__ float chunk_max(const uint32_t (&rr)[32], int n0, int
 __device__ __forceinline__ float chunk_exp_store(uint8_t* sP, const uint32_t (&rr)[32], int c,
                                                  int t, int w, int kb, int Lr, float mxs) {
     uint32_t pk[16];
-    float sum = 0.f;
+    float s0 = 0.f, s1 = 0.f;   // two partial sums, packed f32x2 pairs
 #pragma unroll
     for (int e = 0; e < 32; e += 2) {
-        float pv[2];
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            const int n = c * 32 + e + h;
-            pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rr[e + h]), LOG2E, -mxs))
-                                                 : 0.f;
-            sum += pv[h];
-        }
-        pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
+        const int n = c * 32 + e;
+        float a0, a1;
+        ffma2_bc(__uint_as_float(rr[e]), __uint_as_float(rr[e + 1]), LOG2E, -mxs, a0, a1);
+        const float p0 = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(a0) : 0.f;
+        const float p1 = band_ok(n + 1, t, w, kb + n + 1, Lr) ? fast_exp2(a1) : 0.f;
+        fadd2_acc(s0, s1, p0, p1);
+        pk[e / 2] = pack_bf16x2(p0, p1);
     }
     st_p_chunk(sP, t, c, pk);
-    return sum;
+    return s0 + s1;
 }
 
 // TAPE: score tape read (BWDQ / BWDKV) or written (FWD) -- a separate instantiation, so the plain
@@ -690,13 +688,26 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
                     if (!tp) tmem_ld32(trow + c * 32, rs);
                     tmem_ld32(trow + 256 + c * 32, rd);
                     tmem_wait_ld();
+                    if constexpr (tp) {
 #pragma unroll
-                    for (int e = 0; e < 32; ++e) {
-                        const int n = c * 32 + e;
-                        const bool ok = band_ok(n, t, w, kb + n, Lr);
-                        const float pv = tp ? (ok && tq ? tape_p(n) : 0.f)
-                                            : (ok ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f);
-                        D = fmaf(pv, __uint_as_float(rd[e]), D);
+                        for (int e = 0; e < 32; ++e) {
+                            const int n = c * 32 + e;
+                            const bool ok = band_ok(n, t, w, kb + n, Lr);
+                            const float pv = ok && tq ? tape_p(n) : 0.f;
+                            D = fmaf(pv, __uint_as_float(rd[e]), D);
+                        }
+                    } else {   // packed f32x2 pairs, four partial sums
+                        float Dp[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+                        for (int e = 0; e < 32; e += 2) {
+                            const int n = c * 32 + e, q = e & 2;
+                            float a0, a1;
+                            ffma2_bc(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, -lse2, a0, a1);
+                            const float p0 = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(a0) : 0.f;
+                            const float p1 = band_ok(n + 1, t, w, kb + n + 1, Lr) ? fast_exp2(a1) : 0.f;
+                            ffma2(p0, p1, __uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), Dp[q], Dp[q + 1], Dp[q], Dp[q + 1]);
+                        }
+                        D += (Dp[0] + Dp[1]) + (Dp[2] + Dp[3]);
                     }
                 }
                 auto block_done = [&](int c) {   // early: hand block c/2 to the MMA
@@ -725,13 +736,25 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 #pragma unroll
                     for (int g4 = 0; g4 < 8; ++g4) {
                         float pv[4], dv[4];
+                        if constexpr (tp) {
 #pragma unroll
-                        for (int x = 0; x < 4; ++x) {
-                            const int n = c * 32 + 4 * g4 + x;
-                            const bool ok = band_ok(n, t, w, kb + n, Lr);
-                            pv[x] = tp ? (ok && tq ? tape_p(n) : 0.f)
-                                       : (ok ? fast_exp2(fmaf(__uint_as_float(rs[4 * g4 + x]), LOG2E, -lse2)) : 0.f);
-                            dv[x] = pv[x] * (__uint_as_float(rd[4 * g4 + x]) - D);
+                            for (int x = 0; x < 4; ++x) {
+                                const int n = c * 32 + 4 * g4 + x;
+                                const bool ok = band_ok(n, t, w, kb + n, Lr);
+                                pv[x] = ok && tq ? tape_p(n) : 0.f;
+                                dv[x] = pv[x] * (__uint_as_float(rd[4 * g4 + x]) - D);
+                            }
+                        } else {   // packed f32x2 pairs
+#pragma unroll
+                            for (int x = 0; x < 4; x += 2) {
+                                const int n = c * 32 + 4 * g4 + x, i = 4 * g4 + x;
+                                float a0, a1, q0, q1;
+                                ffma2_bc(__uint_as_float(rs[i]), __uint_as_float(rs[i + 1]), LOG2E, -lse2, a0, a1);
+                                pv[x] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(a0) : 0.f;
+                                pv[x + 1] = band_ok(n + 1, t, w, kb + n + 1, Lr) ? fast_exp2(a1) : 0.f;
+                                ffma2_bc(__uint_as_float(rd[i]), __uint_as_float(rd[i + 1]), 1.f, -D, q0, q1);
+                                fmul2(pv[x], pv[x + 1], q0, q1, dv[x], dv[x + 1]);
+                            }
                         }
                         split_bf16x2(dv[0], dv[1], pk[2 * g4], pl[2 * g4]);
                         split_bf16x2(dv[2], dv[3], pk[2 * g4 + 1], pl[2 * g4 + 1]);
@@ -859,17 +882,26 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band_kernel(const __grid_const
 #pragma unroll
                     for (int e = 0; e < 32; e += 2) {
                         float pv[2], dv[2];
+                        if constexpr (tp) {
 #pragma unroll
-                        for (int h = 0; h < 2; ++h) {
-                            const int n = c * 32 + e + h;
-                            // tape: S^T[key t][query n] = tape[query kb + n][t - n + 2w] (offset of
-                            // key m0 + t from query kb + n is t - n + w); one 128-byte line per warp
-                            const bool ok = band_ok(n, t, w, kb + n, Lr) && (!tp || mrow < Lr);
-                            pv[h] = !ok ? 0.f
-                                    : fast_exp2(fmaf(tp ? __ldg(p.tape + (rowbase + (int64_t)(kb + n) * p.dil) * p.tstride + (t - n + 2 * w))
-                                                        : __uint_as_float(rs[e + h]),
-                                                     LOG2E, -colLse[n]));
-                            dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
+                            for (int h = 0; h < 2; ++h) {
+                                const int n = c * 32 + e + h;
+                                // tape: S^T[key t][query n] = tape[query kb + n][t - n + 2w] (offset of
+                                // key m0 + t from query kb + n is t - n + w); one 128-byte line per warp
+                                const bool ok = band_ok(n, t, w, kb + n, Lr) && mrow < Lr;
+                                pv[h] = !ok ? 0.f
+                                        : fast_exp2(fmaf(__ldg(p.tape + (rowbase + (int64_t)(kb + n) * p.dil) * p.tstride + (t - n + 2 * w)),
+                                                         LOG2E, -colLse[n]));
+                                dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
+                            }
+                        } else {   // packed f32x2 pairs
+                            const int n = c * 32 + e;
+                            float a0, a1, q0, q1;
+                            ffma2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, LOG2E, -colLse[n], -colLse[n + 1], a0, a1);
+                            pv[0] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(a0) : 0.f;
+                            pv[1] = band_ok(n + 1, t, w, kb + n + 1, Lr) ? fast_exp2(a1) : 0.f;
+                            ffma2(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, 1.f, -colD[n], -colD[n + 1], q0, q1);
+                            fmul2(pv[0], pv[1], q0, q1, dv[0], dv[1]);
                         }
                         pk[e / 2] = pack_bf16x2(pv[0], pv[1]);
                         split_bf16x2(dv[0], dv[1], dk[e / 2], dl[e / 2]);

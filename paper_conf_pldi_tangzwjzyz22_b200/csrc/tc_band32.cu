@@ -595,7 +595,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 }
                 if (mx == -INFINITY) mx = 0.f;   // rows beyond the sequence (never stored)
                 const float mxs = mx * LOG2E;
-                float sum = 0.f;
+                float sum2[2] = {0.f, 0.f};
                 for (int c = 0; c < nch; ++c) {
                     if (c < c_lo || c > c_hi) {
                         tmem_st16(rS + c * 32, zero16);
@@ -609,20 +609,20 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tmem_ld16(rS + n0, rr);
                         tmem_wait_ld();
 #pragma unroll
-                        for (int e = 0; e < 16; e += 2) {
-                            float pv[2];
-#pragma unroll
-                            for (int h = 0; h < 2; ++h) {
-                                const int n = n0 + e + h;
-                                pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rr[e + h]), LOG2E, -mxs)) : 0.f;
-                                sum += pv[h];
-                            }
-                            split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
+                        for (int e = 0; e < 16; e += 2) {   // packed f32x2 pairs, two partial sums
+                            float a0, a1;
+                            ffma2_bc(__uint_as_float(rr[e]), __uint_as_float(rr[e + 1]), LOG2E, -mxs, a0, a1);
+                            const int n = n0 + e;
+                            const float p0 = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(a0) : 0.f;
+                            const float p1 = band_ok(n + 1, t, w, kb + n + 1, Lr) ? fast_exp2(a1) : 0.f;
+                            fadd2_acc(sum2[0], sum2[1], p0, p1);
+                            split2(p0, p1, pk[e / 2], pl[e / 2]);
                         }
                         tmem_st8(rS + n0, pk);
                         tmem_st8(rS + n0 + 8, pl);
                     }
                 }
+                const float sum = sum2[0] + sum2[1];
                 rowScale[(j % 3) * 128 + t] = 1.f / sum;
                 tmem_wait_st();
                 tc_fence_before();
@@ -633,7 +633,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 const float lse2 = mrow >= Lr ? 0.f
                                    : (p.lsepoll ? ld_lse_ready(p.lse + rowbase + (int64_t)mrow * p.dil, lse_settled)
                                                 : p.lse[rowbase + (int64_t)mrow * p.dil]) * LOG2E;
-                float D = 0.f;
+                float Dp[4] = {0.f, 0.f, 0.f, 0.f};   // four partial sums (FFMA2 pairs)
                 for (int c = c_lo; c <= c_hi; ++c) {   // pass 1: D = sum_j P_ij dP_ij
 #pragma unroll
                     for (int hh = 0; hh < 2; ++hh) {
@@ -643,13 +643,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tmem_ld16(rP + n0, rd);
                         tmem_wait_ld();
 #pragma unroll
-                        for (int e = 0; e < 16; ++e) {
-                            const int n = n0 + e;
-                            const float pv = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e]), LOG2E, -lse2)) : 0.f;
-                            D = fmaf(pv, __uint_as_float(rd[e]), D);
+                        for (int e = 0; e < 16; e += 2) {
+                            float a0, a1;
+                            ffma2_bc(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, -lse2, a0, a1);
+                            const int n = n0 + e, q = e & 2;
+                            const float p0 = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(a0) : 0.f;
+                            const float p1 = band_ok(n + 1, t, w, kb + n + 1, Lr) ? fast_exp2(a1) : 0.f;
+                            ffma2(p0, p1, __uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), Dp[q], Dp[q + 1], Dp[q], Dp[q + 1]);
                         }
                     }
                 }
+                const float D = (Dp[0] + Dp[1]) + (Dp[2] + Dp[3]);
                 for (int c = 0; c < nch; ++c) {   // pass 2: dS = P (dP - D) -> hi | lo over S
                     if (c < c_lo || c > c_hi) {
                         tmem_st16(rS + c * 32, zero16);
@@ -670,10 +674,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         for (int g4 = 0; g4 < 4; ++g4) {
                             float pv[4], dv[4];
 #pragma unroll
-                            for (int x = 0; x < 4; ++x) {
-                                const int n = n0 + 4 * g4 + x;
-                                pv[x] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[4 * g4 + x]), LOG2E, -lse2)) : 0.f;
-                                dv[x] = pv[x] * (__uint_as_float(rd[4 * g4 + x]) - D);
+                            for (int x = 0; x < 4; x += 2) {   // packed f32x2 pairs
+                                const int n = n0 + 4 * g4 + x, i = 4 * g4 + x;
+                                float a0, a1, q0, q1;
+                                ffma2_bc(__uint_as_float(rs[i]), __uint_as_float(rs[i + 1]), LOG2E, -lse2, a0, a1);
+                                pv[x] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(a0) : 0.f;
+                                pv[x + 1] = band_ok(n + 1, t, w, kb + n + 1, Lr) ? fast_exp2(a1) : 0.f;
+                                ffma2_bc(__uint_as_float(rd[i]), __uint_as_float(rd[i + 1]), 1.f, -D, q0, q1);
+                                fmul2(pv[x], pv[x + 1], q0, q1, dv[x], dv[x + 1]);
                             }
                             split2(dv[0], dv[1], pk[2 * g4], pl[2 * g4]);
                             split2(dv[2], dv[3], pk[2 * g4 + 1], pl[2 * g4 + 1]);
@@ -774,13 +782,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tmem_wait_ld();
 #pragma unroll
                         for (int e = 0; e < 16; e += 2) {
-                            float pv[2], dv[2];
-#pragma unroll
-                            for (int h = 0; h < 2; ++h) {
-                                const int n = n0 + e + h;
-                                pv[h] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(fmaf(__uint_as_float(rs[e + h]), LOG2E, -colLse[n])) : 0.f;
-                                dv[h] = pv[h] * (__uint_as_float(rd[e + h]) - colD[n]);
-                            }
+                            float pv[2], dv[2], a0, a1, q0, q1;   // packed f32x2 pairs
+                            const int n = n0 + e;
+                            ffma2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, LOG2E, -colLse[n], -colLse[n + 1], a0, a1);
+                            pv[0] = band_ok(n, t, w, kb + n, Lr) ? fast_exp2(a0) : 0.f;
+                            pv[1] = band_ok(n + 1, t, w, kb + n + 1, Lr) ? fast_exp2(a1) : 0.f;
+                            ffma2(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, 1.f, -colD[n], -colD[n + 1], q0, q1);
+                            fmul2(pv[0], pv[1], q0, q1, dv[0], dv[1]);
                             split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
                             split2(dv[0], dv[1], dk[e / 2], dl[e / 2]);
                         }
