@@ -125,10 +125,7 @@ __device__ __forceinline__ float fast_exp2(float x) {
     return y;
 }
 __device__ __forceinline__ void split_bf16x2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
-    __nv_bfloat162 h = __floats2bfloat162_rn(x0, x1);
-    const float2 hf = __bfloat1622float2(h);
-    hi = *reinterpret_cast<uint32_t*>(&h);
-    lo = pack_bf16x2(x0 - hf.x, x1 - hf.y);
+    split_bf16x2_p(x0, x1, hi, lo);   // tc_common.cuh: one packed subtraction
 }
 __device__ __forceinline__ bool band_ok(int n, int t, int w, int mcol, int Lr) {
     return (unsigned)(n - t) <= (unsigned)(2 * w) && mcol >= 0 && mcol < Lr;

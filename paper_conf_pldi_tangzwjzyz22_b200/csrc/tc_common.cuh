@@ -416,6 +416,19 @@ __device__ __forceinline__ void fmul2(float a0, float a1, float b0, float b1, fl
         : "=f"(r0), "=f"(r1)
         : "f"(a0), "f"(a1), "f"(b0), "f"(b1));
 }
+// (x0, x1) -> hi = bf16x2 RN of (x0, x1), lo = bf16x2 RN of (x0, x1) - hi, the subtraction as one
+// packed f32x2 instruction (x0 in the low halves)
+__device__ __forceinline__ void split_bf16x2_p(float x0, float x1, uint32_t& hi, uint32_t& lo) {
+    asm("{\n\t.reg .b32 h0, h1, r0, r1;\n\t.reg .b64 xx, hh, rr;\n\t"
+        "cvt.rn.bf16x2.f32 %0, %3, %2;\n\t"
+        "shl.b32 h0, %0, 16;\n\tand.b32 h1, %0, 0xffff0000;\n\t"
+        "mov.b64 xx, {%2, %3};\n\tmov.b64 hh, {h0, h1};\n\t"
+        "sub.rn.f32x2 rr, xx, hh;\n\t"
+        "mov.b64 {r0, r1}, rr;\n\t"
+        "cvt.rn.bf16x2.f32 %1, r1, r0;\n\t}"
+        : "=r"(hi), "=r"(lo)
+        : "f"(x0), "f"(x1));
+}
 __device__ __forceinline__ uint32_t pack_f16x2(float lo, float hi) {
     __half2 h = __floats2half2_rn(lo, hi);   // .x = lo (low 16 bits)
     return *reinterpret_cast<uint32_t*>(&h);
