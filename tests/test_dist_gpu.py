@@ -79,7 +79,8 @@ def _shard_worker(rank, world, port, shape, dtype, result_q):
 
 
 @pytest.mark.parametrize("shape,dtype", [((1, 3, 700, 512, 32, 1), "bf16"), ((2, 3, 900, 64, 32, 2), "bf16"),
-                                         ((1, 4, 600, 64, 100, 1), "bf16"), ((1, 3, 300, 64, 16, 1), "f32")],
+                                         ((1, 4, 600, 64, 100, 1), "bf16"), ((1, 3, 300, 64, 16, 1), "f32"),
+                                         ((1, 2, 700, 512, 32, 1), "f32")],   # fp32 tensor cores + dS tape
                          ids=lambda s: "x".join(map(str, s)) if isinstance(s, tuple) else s)
 def test_sharded_fwd_bwd_cuda_world2(shape, dtype):
     ctx = mp.get_context("spawn")
@@ -126,7 +127,8 @@ def _cp_worker(rank, world, port, shape, dtype, result_q):
 @pytest.mark.parametrize("world,shape,dtype", [(2, (1, 2, 1000, 512, 32, 1), "bf16"),
                                                (3, (2, 2, 1500, 64, 32, 3), "bf16"),
                                                (2, (1, 2, 1200, 64, 100, 1), "bf16"),
-                                               (2, (1, 2, 500, 64, 16, 2), "f32")],
+                                               (2, (1, 2, 500, 64, 16, 2), "f32"),
+                                               (2, (1, 2, 800, 256, 32, 1), "f32")],   # fp32 tensor cores + dS tape
                          ids=lambda s: "x".join(map(str, s)) if isinstance(s, tuple) else str(s))
 def test_context_parallel_cuda(world, shape, dtype):
     ctx = mp.get_context("spawn")
