@@ -111,7 +111,7 @@ def launch_table(ft, B, H, L, d, w, dil, code):
             return [rows] * n_launch
         return [rows * sz / nres for sz in sizes]
 
-    res = 8 if min(w, L) <= 64 else 4
+    res = 8 if (min(w, L) <= 64 or code == 0) else 4   # fp32 tensor-core launches: 8 residues
     fwd = [("fwd", r) for r in (split(nf, res) if path_f == ft.PATH_TC else [rows] * nf)]
     if path_b == ft.PATH_TC:
         pre = nb % 2                                     # wide windows: optional rowdot pre-pass

@@ -106,7 +106,7 @@ WsLayout ws_layout(int64_t B, int64_t H, int64_t L, int64_t d, int64_t w, int64_
     const size_t rows = (size_t)(B * H * L);
     l.rows = (int64_t)rows;
     l.dB = round256(rows * sizeof(float));
-    l.tape = (ftw::dstape_pays(d, dt) || ftw::knob(ftw::K_DSTAPE) == 2) && (dt == FT_F32 ? ftw::tc32_supported(B * H, L, d, w, dil)
+    l.tape = (ftw::dstape_pays(d, dt) || ftw::knob(ftw::K_DSTAPE) == 2) && (dt == FT_F32 ? (w < L ? w : L) <= 32 && ftw::tc32_supported(B * H, L, d, w, dil)
                                                    : ftw::tc_band_dstape_ok(B * H, L, d, w, dil));
     if (l.tape) {
         l.tsw = ftw::dstape_tsw(w < L ? w : L);
@@ -192,7 +192,7 @@ ft_status ft_winattn_plan(int is_bwd, int64_t batch, int64_t heads, int64_t seq_
     if (s != FT_OK) return s;
     int n;
     if (p == FT_PATH_TC && dtype == FT_F32)
-        n = is_bwd ? ftw::tc32_bwd_launches(seq_len, dilation) : ftw::tc32_fwd_launches(seq_len, dilation);
+        n = is_bwd ? ftw::tc32_bwd_launches(seq_len, w, dilation) : ftw::tc32_fwd_launches(seq_len, w, dilation);
     else if (p == FT_PATH_TC)
         n = is_bwd ? ftw::tc_bwd_launches(batch * heads, seq_len, d, w, dilation)
                    : ftw::tc_fwd_launches(seq_len, d, w, dilation);
@@ -328,7 +328,7 @@ ft_status run_bwd(const void* q, const void* k, const void* v, const void* out, 
     if (path == FT_PATH_TC && dtype == FT_F32) {
         int n = 0;
         const bool ok = ftw::tc32_supported(batch * heads, seq_len, d, w, dilation);
-        e = ftw::tc32_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, use_tape && ok ? &tape : nullptr, batch, heads,
+        e = ftw::tc32_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, use_tape && ok ? &tape : nullptr, batch, heads,
                           seq_len, d, w, dilation, st, &n);
     } else if (path == FT_PATH_TC) {
         int n = 0;

@@ -130,11 +130,11 @@ cudaError_t tc_narrow_bwd(const void* q, const void* k, const void* v, const flo
 // fp32 tensor-core kernels (bf16 hi / lo planes, 3 products) for w <= 32, d % 64 == 0 --
 // tc_band32.cu
 bool tc32_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil);
-int tc32_fwd_launches(int64_t L, int64_t dil);
-int tc32_bwd_launches(int64_t L, int64_t dil);
+int tc32_fwd_launches(int64_t L, int64_t w, int64_t dil);
+int tc32_bwd_launches(int64_t L, int64_t w, int64_t dil);
 cudaError_t tc32_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B, int64_t H,
                      int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches);
-cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const float* lse, const void* dout, void* dq,
+cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const void* out, const float* lse, const void* dout, void* dq,
                      void* dk, void* dv, float* Dws, const DsTape* tape, int64_t B, int64_t H, int64_t L,
                      int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches);
 

@@ -82,6 +82,8 @@ constexpr int NCONV = 6;                  // converter warps
 constexpr int RES_PER_LAUNCH = 8;
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t R0 = 0, R1 = 192, RACC = 384;
+constexpr int WMAX_SB = 64;               // sub-bands of a WIDE launch (w <= 2079)
+constexpr float RESCALE_LOG2 = 20.f;      // WIDE FWD lazy rescaling: P <= 2^20 between max moves
 constexpr float LOG2E = 1.4426950408889634f;
 constexpr float LN2 = 0.6931471805599453f;
 
@@ -110,6 +112,12 @@ struct Params {
     float* tP;
     float* tS;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace), see trace32()
+    // WIDE (w > 32, d = 64): the band of offsets [-w, w] is cut into nsb sub-bands of <= 65
+    // offsets, [sb_lo[s], sb_lo[s] + sb_w2[s]], visited in this order (the one holding offset 0
+    // first); each (tile, sub-band) step is one pass of this kernel's normal work over a 192-row
+    // halo starting at m0 + sb_lo (keys; FWD, BWDQ) or m0 - sb_lo - sb_w2 (queries; BWDKV).
+    int nsb;
+    int sb_lo[WMAX_SB], sb_w2[WMAX_SB];
 };
 
 // Phase trace (profiling only): per CTA, clock64 stamps of its first TR_SLOTS slots --
@@ -125,10 +133,11 @@ __device__ __forceinline__ void trace_tile(const Params& p, int j, int e) {
 }
 
 constexpr size_t SCRATCH = 3 * 128 * 4 + 2 * 192 * 4;   // FWD row 1/l [3][128]; BWDKV column lse / D
-constexpr size_t SMEM_BYTES = 1024 + NST * SLOT + 4 * NSTG * STG + SCRATCH + 256;
-constexpr size_t SMEM_BYTES_XT = 1024 + NST_XT * SLOT_XT + 4 * NSTG_XT * STG + 256;
+constexpr size_t BAR_BYTES = 512;
+constexpr size_t SMEM_BYTES = 1024 + NST * SLOT + 4 * NSTG * STG + SCRATCH + BAR_BYTES;
+constexpr size_t SMEM_BYTES_XT = 1024 + NST_XT * SLOT_XT + 4 * NSTG_XT * STG + BAR_BYTES;
 static_assert(SMEM_BYTES <= 227 * 1024 && SMEM_BYTES_XT <= 227 * 1024, "shared memory plan");
-static_assert(3 * NST_XT * 8 + 12 * 8 + 4 <= 256, "barrier area");
+static_assert(3 * NST_XT * 8 + 16 * 8 + 4 <= BAR_BYTES, "barrier area");
 
 using Tile = SchedTile;
 using TileCursor = SchedCursor<BM>;
@@ -233,7 +242,7 @@ struct AccUses {
     }
 };
 
-template <int MODE>
+template <int MODE, bool WIDE>
 __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_constant__ Params p) {
     using C = Seq<MODE>;
     extern __shared__ uint8_t smem_raw[];
@@ -244,6 +253,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     const int nkb = NK / KB, nch = NK / 32;
     const int ncw = (d + CW - 1) / CW;      // output chunks per tensor (the last may be 64 wide)
     const int nacc = ncw * C::NOUT;         // accumulations per tile
+    const int nsb = WIDE ? p.nsb : 1;       // sub-bands per tile
+    // first halo row of sub-band sb relative to m0 (normal mode: -w)
+    auto koff = [&](int sb) -> int {
+        if (!WIDE) return -w;
+        return MODE == BWDKV ? -p.sb_lo[sb] - p.sb_w2[sb] : p.sb_lo[sb];
+    };
 
     if (MODE == BWDQ && p.xt) {   // clear this CTA's tile flags before BWDKV may launch
         TileCursor cr(p.sc);
@@ -298,17 +313,23 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     // R0): one phase per tile each, so the softmax warps never lag two phases behind (o_empty
     // completes u0 times per tile and is waited only by the MMA issuer, use by use)
     uint64_t* xfree = s_full + 10;
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 12);
+    uint64_t* pv_done = s_full + 12;  // WIDE FWD [2]: the output GEMMs of step k done (parity k & 1)
+    uint64_t* rs_full = s_full + 14;  // WIDE FWD [2]: 1/l and lse of tile j published (4 warps)
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 16);
     // Accumulator of accumulation a: RACC, except in BWDKV with the dS tape, where the dV (dK)
     // chunks alternate between R0 (R1) and RACC, ending on RACC: during dV R1 holds the A operand
     // P^T and R0 is free (dS^T is built into it after the last R0 drain), during dK R0 holds dS^T
     // and R1 is free -- so an accumulation runs while the epilogue drains the previous one.
     auto acc_rid = [&](int a) -> int {
+        if (WIDE) return a;   // FWD / BWDQ: one accumulation; BWDKV: dV (0), dK (1), both live across sub-bands
         if (!xt || ((ncw - 1 - a % ncw) & 1) == 0) return 0;
         return a < ncw ? 1 : 2;
     };
     // (the R1 accumulator sits at column 256, 128-aligned like the others)
-    auto acc_col = [](int rid) -> uint32_t { return rid == 0 ? RACC : rid == 1 ? R0 : R1 + 64; };
+    auto acc_col = [](int rid) -> uint32_t {
+        if (WIDE) return RACC + 64u * rid;
+        return rid == 0 ? RACC : rid == 1 ? R0 : R1 + 64;
+    };
     const int npl = (NK + TROWS - 1) / TROWS;   // tape slots per plane
     // (with ncw >= 2, the host's condition for xt, the last R0 / R1 accumulation is chunk ncw - 2)
 
@@ -329,6 +350,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             }
             mbar_init(&xfree[0], 4);
             mbar_init(&xfree[1], 4);
+            for (int i = 0; i < 2; ++i) {
+                mbar_init(&pv_done[i], 1);
+                mbar_init(&rs_full[i], 4);
+            }
             fence_barrier_init();
             for (int i = 0; i < p.sc.nr; ++i) {
                 const Maps& mp = p.maps[i];
@@ -353,18 +378,49 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         TileCursor cg(p.sc), co(p.sc);
         Tile Tg, To;
         bool hg = cg.next(p.sc, Tg);
+        if constexpr (WIDE) {
+            // steps (tile, sub-band); FWD: G(step 0), then per step G(step + 1), O(step); BWD: G, O
+            if (MODE == FWD) {
+                int sg = 0;
+                auto gnext = [&]() {
+                    for (int s = 0; s < nsl; ++s) fn(0, Tg, s, 0, sg);
+                    if (++sg == nsb) {
+                        sg = 0;
+                        hg = cg.next(p.sc, Tg);
+                    }
+                };
+                if (hg) gnext();
+                while (co.next(p.sc, To))
+                    for (int so = 0; so < nsb; ++so) {
+                        if (hg) gnext();
+                        for (int a = 0; a < nacc; ++a)
+                            for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb, so);
+                    }
+            } else {
+                while (co.next(p.sc, To))
+                    for (int so = 0; so < nsb; ++so) {
+                        for (int s = 0; s < nsl; ++s) {
+                            fn(0, To, s, 0, so);
+                            fn(0, To, s, 1, so);
+                        }
+                        for (int a = 0; a < nacc; ++a)
+                            for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb, so);
+                    }
+            }
+            return;
+        }
         if (MODE == FWD) {
             if (hg) {
-                for (int s = 0; s < nsl; ++s) fn(0, Tg, s, 0);
+                for (int s = 0; s < nsl; ++s) fn(0, Tg, s, 0, 0);
                 hg = cg.next(p.sc, Tg);
             }
             while (co.next(p.sc, To)) {
                 if (hg) {
-                    for (int s = 0; s < nsl; ++s) fn(0, Tg, s, 0);
+                    for (int s = 0; s < nsl; ++s) fn(0, Tg, s, 0, 0);
                     hg = cg.next(p.sc, Tg);
                 }
                 for (int a = 0; a < nacc; ++a)
-                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
+                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb, 0);
             }
         } else if (xt) {
             // Tape slots (npl of 128 rows per plane) sit one output chunk ahead of their use, so
@@ -373,19 +429,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             //   P(j+1) (if any), dK c[ncw-1].   Slot positions: xt_pos_P / xt_pos_S below.
             bool has = co.next(p.sc, To);
             if (has)
-                for (int b = 0; b < npl; ++b) fn(2, To, b, 0);
+                for (int b = 0; b < npl; ++b) fn(2, To, b, 0, 0);
             while (has) {
                 Tile Tnext;
                 const bool hnext = co.next(p.sc, Tnext);
                 auto blocks = [&](int a) {
-                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
+                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb, 0);
                 };
                 for (int a = 0; a < ncw - 1; ++a) blocks(a);
-                for (int b = 0; b < npl; ++b) fn(2, To, b, 1);
+                for (int b = 0; b < npl; ++b) fn(2, To, b, 1, 0);
                 blocks(ncw - 1);
                 for (int a = ncw; a < nacc - 1; ++a) blocks(a);
                 if (hnext)
-                    for (int b = 0; b < npl; ++b) fn(2, Tnext, b, 0);
+                    for (int b = 0; b < npl; ++b) fn(2, Tnext, b, 0, 0);
                 blocks(nacc - 1);
                 To = Tnext;
                 has = hnext;
@@ -393,11 +449,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         } else {
             while (co.next(p.sc, To)) {
                 for (int s = 0; s < nsl; ++s) {
-                    fn(0, To, s, 0);
-                    fn(0, To, s, 1);
+                    fn(0, To, s, 0, 0);
+                    fn(0, To, s, 1, 0);
                 }
                 for (int a = 0; a < nacc; ++a)
-                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb);
+                    for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb, 0);
             }
         }
     };
@@ -406,7 +462,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         if (lane == 0) {   // -------------------------------------------------- TMA producer
             int st = 0, k = 0;
             uint32_t ph = 0;
-            walk([&](int kind, const Tile& T, int a, int b) {
+            walk([&](int kind, const Tile& T, int a, int b, int sb) {
                 mbar_wait(&empty[st], ph ^ 1u);
                 trace_slot(p, k++, 0);
                 uint8_t* sp = slots + (size_t)st * slotb;
@@ -426,7 +482,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     mbar_arrive_expect_tx(&full[st], (uint32_t)(2 * BM + 2 * NK) * 64u);
                     for (int h = 0; h < 2; ++h) {
                         tma_load_3d(sp + h * BM * 64, ma, &full[st], 32 * a + 16 * h, T.m0, T.u);
-                        tma_load_3d(sp + 2 * BM * 64 + h * NK * 64, mb, &full[st], 32 * a + 16 * h, T.m0 - w, T.u);
+                        tma_load_3d(sp + 2 * BM * 64 + h * NK * 64, mb, &full[st], 32 * a + 16 * h, T.m0 + koff(sb), T.u);
                     }
                 } else {
                     const int c = C::NOUT == 2 ? a % ncw : a;
@@ -434,7 +490,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     const CUtensorMap* m = (C::NOUT == 2 && a >= ncw) ? &mp.ob2 : &mp.ob1;
                     mbar_arrive_expect_tx(&full[st], (uint32_t)nbox * KB * 128u);
                     for (int x = 0; x < nbox; ++x)
-                        tma_load_3d(sp + x * KB * 128, m, &full[st], CW * c + 32 * x, T.m0 - w + KB * b, T.u);
+                        tma_load_3d(sp + x * KB * 128, m, &full[st], CW * c + 32 * x, T.m0 + koff(sb) + KB * b, T.u);
                 }
                 if (++st == nst) { st = 0; ph ^= 1u; }
             });
@@ -443,7 +499,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         const int ct = threadIdx.x - 320;   // 0 .. 32 NCONV - 1
         int st = 0, k = 0;
         uint32_t ph = 0;
-        walk([&](int kind, const Tile&, int a, int) {
+        walk([&](int kind, const Tile&, int a, int, int) {
             mbar_wait(&full[st], ph);
             if (ct == 0) trace_slot(p, k, 1);
             uint8_t* sp = slots + (size_t)st * slotb;
@@ -469,9 +525,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             int st = 0, k = 0;
             AccUses uses;   // accumulations per region so far
             uint32_t ph = 0;
-            int jg = 0;          // score GEMMs: tile counter
-            int jo = 0;          // output GEMMs: tile counter
-            walk([&](int kind, const Tile&, int a, int b) {
+            int jg = 0;          // score GEMMs: tile (WIDE: step) counter
+            int jo = 0;          // output GEMMs: tile (WIDE: step) counter
+            walk([&](int kind, const Tile&, int a, int b, int sb) {
                 const uint32_t sa = smem_u32(slots + (size_t)st * slotb);
                 if (kind == 2) {   // tape slot: no MMA (the softmax warps free it)
                     mbar_wait(&conv[st], ph);
@@ -510,7 +566,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tc_fence_after();
                     }
                     const int rid = acc_rid(a);
-                    if (b == 0 && uses.get(rid) > 0) {
+                    // WIDE: the accumulators live across the sub-bands of a tile
+                    const bool first_sb = !WIDE || sb == 0, last_sb = !WIDE || sb == nsb - 1;
+                    if (b == 0 && first_sb && uses.get(rid) > 0) {
                         mbar_wait(&o_empty[rid], (uint32_t)(uses.get(rid) - 1) & 1u);
                         tc_fence_after();
                     }
@@ -527,14 +585,17 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         const uint32_t tA = Areg + 16u * g;   // hi words; lo words at + 8
                         const uint64_t dbh = sdesc_sw128(sa + kk * 2048, 2 * KB * 128, 1024);
                         const uint64_t dbl = sdesc_sw128(sa + KB * 128 + kk * 2048, 2 * KB * 128, 1024);
-                        mma_ts(Dacc, tA, dbh, id, g != 0);
+                        mma_ts(Dacc, tA, dbh, id, !first_sb || g != 0);
                         mma_ts(Dacc, tA, dbl, id, 1);
                         mma_ts(Dacc, tA + 8, dbh, id, 1);
                     }
                     mma_commit(&empty[st]);
                     if (b == nkb - 1) {
-                        mma_commit(&o_full[rid]);
-                        uses.inc(rid);
+                        if (last_sb) {
+                            mma_commit(&o_full[rid]);
+                            uses.inc(rid);
+                        }
+                        if (WIDE && MODE == FWD) mma_commit(&pv_done[jo & 1]);   // rescale hand-off
                         if (a == nacc - 1) ++jo;
                     }
                 }
@@ -554,8 +615,189 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         Tile T;
         int j = 0;
         if (MODE == BWDKV && !p.dpoll) asm volatile("griddepcontrol.wait;" ::: "memory");
+        if constexpr (WIDE) {
+            // One (tile, sub-band) step at a time.  FWD: online softmax over the sub-bands with
+            // lazy rescaling (the running max m only moves when a sub-band's max exceeds it by more
+            // than 2^RESCALE_LOG2; then this row's O partial in TMEM and l are scaled by 2^(m_old -
+            // m_new) after the previous step's output GEMMs completed).  BWDQ / BWDKV: the global lse
+            // and D (= dout . out, computed before the launch) make every step independent.
+            int k = 0;
+            float m_run = 0.f, l_run = 0.f;
+            while (cur.next(p.sc, T)) {
+                const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t;
+                const int64_t rowbase = (int64_t)T.u * p.L + T.r;
+                const bool rowv = mrow < Lr;
+                float lse2 = 0.f, Drow = 0.f;
+                if (MODE == BWDQ && rowv) {
+                    lse2 = p.lse[rowbase + (int64_t)mrow * p.dil] * LOG2E;
+                    Drow = p.D[rowbase + (int64_t)mrow * p.dil];
+                }
+                for (int sb = 0; sb < nsb; ++sb, ++k) {
+                    const int W2 = p.sb_w2[sb], kb = m0 + koff(sb);
+                    const int chi = min(nch - 1, (32 * warp + 31 + W2) / 32);
+                    if (MODE == BWDKV) {   // lse / D of this step's halo queries
+                        named_bar_sync(1, 128);
+                        for (int n = t; n < NK; n += 128) {
+                            const int mc = kb + n;
+                            const bool ok = mc >= 0 && mc < Lr;
+                            colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
+                            colD[n] = ok ? p.D[rowbase + (int64_t)mc * p.dil] : 0.f;
+                        }
+                        named_bar_sync(1, 128);
+                    }
+                    mbar_wait(&s_full[MODE == FWD ? (k & 1) : 0], MODE == FWD ? ((k >> 1) & 1) : (k & 1));
+                    tc_fence_after();
+                    const uint32_t rS = tbase + lane_off + (MODE == FWD && (k & 1) ? R1 : R0);
+                    const uint32_t rP = tbase + lane_off + R1;
+                    if (MODE == FWD) {
+                        float cm = -INFINITY;
+                        for (int c = c_lo; c <= chi; ++c) {
+                            uint32_t rr[32];
+                            tmem_ld32(rS + c * 32, rr);
+                            tmem_wait_ld();
+#pragma unroll
+                            for (int e = 0; e < 32; ++e)
+                                if ((unsigned)(c * 32 + e - t) <= (unsigned)W2 && kb + c * 32 + e >= 0 && kb + c * 32 + e < Lr)
+                                    cm = fmaxf(cm, __uint_as_float(rr[e]));
+                        }
+                        const float cms = cm * LOG2E;
+                        float fac = 1.f;
+                        bool need = false;
+                        if (sb == 0) {
+                            m_run = cm == -INFINITY ? 0.f : cms;
+                            l_run = 0.f;
+                        } else if (cm != -INFINITY && cms > m_run + RESCALE_LOG2) {
+                            need = true;
+                            fac = fast_exp2(m_run - cms);
+                            m_run = cms;
+                            l_run *= fac;
+                        }
+                        if (__any_sync(0xffffffffu, need)) {   // scale this warp's O rows (previous PV done)
+                            mbar_wait(&pv_done[(k - 1) & 1], ((k - 1) >> 1) & 1);
+                            tc_fence_after();
+#pragma unroll
+                            for (int h = 0; h < 2; ++h) {
+                                uint32_t ov[32];
+                                tmem_ld32(tbase + lane_off + RACC + 32 * h, ov);
+                                tmem_wait_ld();
+#pragma unroll
+                                for (int e = 0; e < 32; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * fac);
+                                tmem_st16(tbase + lane_off + RACC + 32 * h, *reinterpret_cast<const uint32_t(*)[16]>(&ov[0]));
+                                tmem_st16(tbase + lane_off + RACC + 32 * h + 16, *reinterpret_cast<const uint32_t(*)[16]>(&ov[16]));
+                            }
+                        }
+                        float sum2[2] = {0.f, 0.f};
+                        for (int c = 0; c < nch; ++c) {
+                            if (c < c_lo || c > chi) {
+                                tmem_st16(rS + c * 32, zero16);
+                                tmem_st16(rS + c * 32 + 16, zero16);
+                                continue;
+                            }
+#pragma unroll
+                            for (int hh = 0; hh < 2; ++hh) {
+                                const int n0 = c * 32 + 16 * hh;
+                                uint32_t rr[16], pk[8], pl[8];
+                                tmem_ld16(rS + n0, rr);
+                                tmem_wait_ld();
+#pragma unroll
+                                for (int e = 0; e < 16; e += 2) {
+                                    float a0, a1;
+                                    ffma2_bc(__uint_as_float(rr[e]), __uint_as_float(rr[e + 1]), LOG2E, -m_run, a0, a1);
+                                    const int n = n0 + e;
+                                    const float p0 = (unsigned)(n - t) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
+                                    const float p1 = (unsigned)(n + 1 - t) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
+                                    fadd2_acc(sum2[0], sum2[1], p0, p1);
+                                    split2(p0, p1, pk[e / 2], pl[e / 2]);
+                                }
+                                tmem_st8(rS + n0, pk);
+                                tmem_st8(rS + n0 + 8, pl);
+                            }
+                        }
+                        l_run += sum2[0] + sum2[1];
+                        tmem_wait_st();
+                        tc_fence_before();
+                        warp_arrive(&p_full[k & 1]);
+                        if (sb == nsb - 1) {   // 1/l and lse of the tile (the epilogue waits rs_full)
+                            rowScale[(j % 3) * 128 + t] = 1.f / l_run;
+                            if (rowv) p.lse[rowbase + (int64_t)mrow * p.dil] = (m_run + log2f(l_run)) * LN2;
+                            warp_arrive(&rs_full[j & 1]);
+                        }
+                    } else if (MODE == BWDQ) {   // dS = P (dP - D) -> hi | lo over S
+                        for (int c = 0; c < nch; ++c) {
+                            if (c < c_lo || c > chi) {
+                                tmem_st16(rS + c * 32, zero16);
+                                tmem_st16(rS + c * 32 + 16, zero16);
+                                continue;
+                            }
+#pragma unroll
+                            for (int hh = 0; hh < 2; ++hh) {
+                                const int n0 = c * 32 + 16 * hh;
+                                uint32_t rs[16], rd[16], pk[8], pl[8];
+                                tmem_ld16(rS + n0, rs);
+                                tmem_ld16(rP + n0, rd);
+                                tmem_wait_ld();
+#pragma unroll
+                                for (int e = 0; e < 16; e += 2) {
+                                    float a0, a1, q0, q1, d0, d1;
+                                    const int n = n0 + e;
+                                    ffma2_bc(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, -lse2, a0, a1);
+                                    const float p0 = (unsigned)(n - t) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
+                                    const float p1 = (unsigned)(n + 1 - t) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
+                                    ffma2_bc(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, -Drow, q0, q1);
+                                    fmul2(p0, p1, q0, q1, d0, d1);
+                                    split2(d0, d1, pk[e / 2], pl[e / 2]);
+                                }
+                                tmem_st8(rS + n0, pk);
+                                tmem_st8(rS + n0 + 8, pl);
+                            }
+                        }
+                        tmem_wait_st();
+                        tc_fence_before();
+                        warp_arrive(&p_full[k & 1]);
+                    } else {   // BWDKV: rows keys, columns halo queries; P^T over dP^T, dS^T over S^T
+                        for (int c = 0; c < nch; ++c) {
+                            if (c < c_lo || c > chi) {
+                                tmem_st16(rS + c * 32, zero16);
+                                tmem_st16(rS + c * 32 + 16, zero16);
+                                tmem_st16(rP + c * 32, zero16);
+                                tmem_st16(rP + c * 32 + 16, zero16);
+                                continue;
+                            }
+#pragma unroll
+                            for (int hh = 0; hh < 2; ++hh) {
+                                const int n0 = c * 32 + 16 * hh;
+                                uint32_t rs[16], rd[16], pk[8], pl[8], dk[8], dl[8];
+                                tmem_ld16(rS + n0, rs);
+                                tmem_ld16(rP + n0, rd);
+                                tmem_wait_ld();
+#pragma unroll
+                                for (int e = 0; e < 16; e += 2) {
+                                    float pv[2], dv[2], a0, a1, q0, q1;
+                                    const int n = n0 + e;
+                                    ffma2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, LOG2E, -colLse[n], -colLse[n + 1], a0, a1);
+                                    pv[0] = (unsigned)(n - t) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
+                                    pv[1] = (unsigned)(n + 1 - t) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
+                                    ffma2(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, 1.f, -colD[n], -colD[n + 1], q0, q1);
+                                    fmul2(pv[0], pv[1], q0, q1, dv[0], dv[1]);
+                                    split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
+                                    split2(dv[0], dv[1], dk[e / 2], dl[e / 2]);
+                                }
+                                tmem_st8(rS + n0, dk);          // dS^T over S^T
+                                tmem_st8(rS + n0 + 8, dl);
+                                tmem_st8(rP + n0, pk);          // P^T over dP^T
+                                tmem_st8(rP + n0 + 8, pl);
+                            }
+                        }
+                        tmem_wait_st();
+                        tc_fence_before();
+                        warp_arrive(&p_full[k & 1]);
+                    }
+                }
+                ++j;
+            }
+        }
         bool lse_settled = false;   // ld_lse_ready fell back to griddepcontrol.wait
-        while (cur.next(p.sc, T)) {
+        while (!WIDE && cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t, kb = m0 - w;
             const int64_t rowbase = (int64_t)T.u * p.L + T.r;
             if (MODE == BWDKV && !p.xt) {
@@ -815,8 +1057,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         while (cur.next(p.sc, T)) {
             const Maps& mp = p.maps[T.rl];
             float scale = 1.f;
-            if (MODE == FWD) {   // 1/l of this row, published before p_full
-                mbar_wait(&p_full[j & 1], (j >> 1) & 1);
+            if (MODE == FWD) {   // 1/l of this row, published before p_full (WIDE: rs_full)
+                if (WIDE) mbar_wait(&rs_full[j & 1], (j >> 1) & 1);
+                else mbar_wait(&p_full[j & 1], (j >> 1) & 1);
                 scale = rowScale[(j % 3) * 128 + ew * 32 + lane];
             }
             for (int a = 0; a < nacc; ++a) {
@@ -895,17 +1138,76 @@ int halo_rows32(int64_t L, int64_t w) {
     return (int)(((BM + 2 * wc) + 63) / 64 * 64);
 }
 
-template <int MODE>
+// WIDE sub-bands: the residue-space offsets [-wm, wm] (wm = min(w, longest residue - 1)) in
+// nsb <= WMAX_SB runs of <= 65 offsets, the run holding offset 0 first, then the others by their
+// distance from it (so the forward's first running max is a real row max estimate).
+struct SubBands {
+    int n = 0;
+    int lo[WMAX_SB], w2[WMAX_SB];
+};
+inline bool sub_bands(int64_t L, int64_t w, int64_t dil, SubBands& sb) {
+    const int64_t Lr = (L + dil - 1) / dil;
+    const int64_t wm = w < Lr - 1 ? w : Lr - 1;
+    const int64_t tot = 2 * wm + 1;
+    const int n = (int)((tot + 64) / 65);
+    if (n > WMAX_SB) return false;
+    int lo[WMAX_SB], w2[WMAX_SB], c = 0;
+    int64_t o = -wm;
+    for (int i = 0; i < n; ++i) {   // near-equal runs
+        const int64_t len = tot / n + (i < tot % n ? 1 : 0);
+        lo[i] = (int)o;
+        w2[i] = (int)(len - 1);
+        if (o <= 0 && 0 <= o + len - 1) c = i;
+        o += len;
+    }
+    sb.n = 0;
+    sb.lo[sb.n] = lo[c];
+    sb.w2[sb.n++] = w2[c];
+    for (int dd = 1; dd < n; ++dd)
+        for (int sgn = -1; sgn <= 1; sgn += 2) {
+            const int i = c + sgn * dd;
+            if (i >= 0 && i < n) {
+                sb.lo[sb.n] = lo[i];
+                sb.w2[sb.n++] = w2[i];
+            }
+        }
+    return true;
+}
+
+// D_i = dout_i . out_i (fp32; the WIDE backward's exact-to-rounding D, reading R1 for fp32 out):
+// one warp per row, d a multiple of 64.
+__global__ void __launch_bounds__(256) rowdot32_kernel(const float* __restrict__ out, const float* __restrict__ dout,
+                                                       float* __restrict__ D, int64_t rows, int d) {
+    const int64_t r = (int64_t)blockIdx.x * 8 + threadIdx.x / 32;
+    const int lane = threadIdx.x % 32;
+    if (r >= rows) return;
+    const float* o = out + r * d;
+    const float* g = dout + r * d;
+    float acc = 0.f;
+    for (int c = 2 * lane; c < d; c += 64) {
+        const float2 a = __ldg(reinterpret_cast<const float2*>(o + c));
+        const float2 b = __ldg(reinterpret_cast<const float2*>(g + c));
+        acc = fmaf(a.x, b.x, fmaf(a.y, b.y, acc));
+    }
+#pragma unroll
+    for (int x = 16; x >= 1; x >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, x);
+    if (lane == 0) D[r] = acc;
+}
+
+template <int MODE, bool WIDE>
 cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void* b2, const void* ob1,
                      const void* ob2, void* o1, void* o2, float* lse, float* D, const DsTape* tape, int64_t B,
                      int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
     static std::once_flag once;
     std::call_once(once, [] {
-        cudaFuncSetAttribute(tc_band32_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaFuncSetAttribute(tc_band32_kernel<MODE, WIDE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)(SMEM_BYTES > SMEM_BYTES_XT ? SMEM_BYTES : SMEM_BYTES_XT));
     });
     const int64_t wc = w < L ? w : L;
-    const int NK = halo_rows32(L, w);
+    const int NK = WIDE ? 192 : halo_rows32(L, w);
+    SubBands sbp;
+    if (WIDE && !sub_bands(L, w, dil, sbp)) return cudaErrorInvalidValue;
+    if (WIDE) tape = nullptr;
     const int64_t units = B * H;
     const int64_t nres = dil < L ? dil : L;
     int n = 0;
@@ -938,7 +1240,14 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         p.dil = (int)dil;
         p.NK = NK;
         p.nsl = (int)(d / 32);
-        p.dpoll = MODE != FWD && dpoll_enabled();   // BWDQ marks its D rows, BWDKV polls them
+        p.dpoll = MODE != FWD && dpoll_enabled() && !WIDE;   // BWDQ marks its D rows, BWDKV polls them
+        if (WIDE) {
+            p.nsb = sbp.n;
+            for (int i = 0; i < sbp.n; ++i) {
+                p.sb_lo[i] = sbp.lo[i];
+                p.sb_w2[i] = sbp.w2[i];
+            }
+        }
         if (tape && MODE != FWD && d > CW) {   // xt needs two output chunks (acc_rid alternation)
             p.xt = 1;
             p.tsw = tape->tsw;
@@ -957,7 +1266,7 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         // lse hand-off: one launch of residues on each side (nres <= RES_PER_LAUNCH) -- the
         // dQ kernel's launch follows the forward's only launch
         p.lsepoll = lsepoll_enabled() && nres <= RES_PER_LAUNCH && lsepoll_worth(total, num_sms32()) &&
-                    !(MODE == BWDKV && p.xt);   // the tape dK/dV kernel reads no lse
+                    !(MODE == BWDKV && p.xt) && !WIDE;   // the tape dK/dV kernel reads no lse
         if ((MODE == BWDKV && r0 == 0 && p.dpoll) || (MODE == BWDQ && p.lsepoll)) {
             // BWDKV directly after this call's last BWDQ launch; BWDQ after the forward
             cudaLaunchConfig_t cfg = {};
@@ -970,9 +1279,9 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
             at[0].val.programmaticStreamSerializationAllowed = 1;
             cfg.attrs = at;
             cfg.numAttrs = 1;
-            cudaLaunchKernelEx(&cfg, tc_band32_kernel<MODE>, p);
+            cudaLaunchKernelEx(&cfg, tc_band32_kernel<MODE, WIDE>, p);
         } else {
-            tc_band32_kernel<MODE><<<grid, NTHREADS, smem, st>>>(p);
+            tc_band32_kernel<MODE, WIDE><<<grid, NTHREADS, smem, st>>>(p);
         }
         prof_mark(st);
         cudaError_t e = cudaGetLastError();
@@ -990,34 +1299,56 @@ int band32_launches(int64_t L, int64_t dil) {
 
 }  // namespace
 
+// w > 32 runs the WIDE instantiation: d = 64 (its two accumulators, dV and dK, share the 128
+// accumulator columns across the sub-bands)
+static bool tc32_wide(int64_t L, int64_t w) { return (w < L ? w : L) > 32; }
 bool tc32_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
     const int64_t wc = w < L ? w : L;
-    return d % 64 == 0 && d <= 512 && wc <= 32 && dil <= 256 && units * ((L + 127) / 128) < (1 << 30);
+    if (!(dil <= 256 && units * ((L + 127) / 128) < (1 << 30))) return false;
+    if (wc <= 32) return d % 64 == 0 && d <= 512;
+    SubBands sb;
+    return d == 64 && sub_bands(L, w, dil, sb);
 }
-int tc32_fwd_launches(int64_t L, int64_t dil) { return band32_launches(L, dil); }
-int tc32_bwd_launches(int64_t L, int64_t dil) { return 2 * band32_launches(L, dil); }
+int tc32_fwd_launches(int64_t L, int64_t w, int64_t dil) { return band32_launches(L, dil); }
+int tc32_bwd_launches(int64_t L, int64_t w, int64_t dil) { return 2 * band32_launches(L, dil) + (tc32_wide(L, w) ? 1 : 0); }
 
 cudaError_t tc32_fwd(const void* q, const void* k, const void* v, void* out, float* lse, int64_t B, int64_t H,
                      int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
     if (launches) *launches = 0;
-    return launch32<FWD>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, nullptr, B, H, L, d, w,
-                         dil, st, launches);
+    if (tc32_wide(L, w))
+        return launch32<FWD, true>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, nullptr, B, H, L,
+                                   d, w, dil, st, launches);
+    return launch32<FWD, false>(q, k, nullptr, nullptr, v, nullptr, out, nullptr, lse, nullptr, nullptr, B, H, L, d, w,
+                                dil, st, launches);
 }
 
-cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const float* lse, const void* dout, void* dq,
-                     void* dk, void* dv, float* Dws, const DsTape* tape, int64_t B, int64_t H, int64_t L,
+cudaError_t tc32_bwd(const void* q, const void* k, const void* v, const void* out, const float* lse, const void* dout,
+                     void* dq, void* dk, void* dv, float* Dws, const DsTape* tape, int64_t B, int64_t H, int64_t L,
                      int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
     if (launches) *launches = 0;
+    if (tc32_wide(L, w)) {   // D = dout . out first; then the two kernels, independent of each other
+        const int64_t rows = B * H * L;
+        rowdot32_kernel<<<(unsigned)((rows + 7) / 8), 256, 0, st>>>((const float*)out, (const float*)dout, Dws, rows, (int)d);
+        prof_mark(st);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        if (launches) *launches += 1;
+        e = launch32<BWDQ, true>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse), Dws, nullptr, B, H,
+                                 L, d, w, dil, st, launches);
+        if (e != cudaSuccess) return e;
+        return launch32<BWDKV, true>(k, q, v, dout, dout, q, dk, dv, const_cast<float*>(lse), Dws, nullptr, B, H, L, d,
+                                     w, dil, st, launches);
+    }
     // BWDQ: S = Q K_h^T (a1 = q, b1 = k), dP = dO V_h^T (a2 = dout, b2 = v), dQ = dS K_h (ob1 = k)
-    cudaError_t e = launch32<BWDQ>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse), Dws, tape, B,
-                                   H, L, d, w, dil, st, launches);
+    cudaError_t e = launch32<BWDQ, false>(q, k, dout, v, k, nullptr, dq, nullptr, const_cast<float*>(lse), Dws, tape,
+                                          B, H, L, d, w, dil, st, launches);
     if (e != cudaSuccess) return e;
     // BWDKV: S^T = K Q_h^T, dP^T = V dO_h^T; dV = P^T dO_h (ob1 = dout -> o2 = dv), dK = dS^T Q_h
     // (ob2 = q -> o1 = dk).  Accumulations: dV chunks (a < ncw, o2), then dK chunks (o1).
     // With the dS tape (PAPER.md:489-497 selective materialization) BWDKV skips S^T and dP^T: it
     // streams only the tape rows and the dO / Q blocks of its output GEMMs.
-    return launch32<BWDKV>(k, q, v, dout, dout, q, dk, dv, const_cast<float*>(lse), Dws, tape, B, H, L, d, w, dil,
-                           st, launches);
+    return launch32<BWDKV, false>(k, q, v, dout, dout, q, dk, dv, const_cast<float*>(lse), Dws, tape, B, H, L, d, w,
+                                  dil, st, launches);
 }
 
 }  // namespace ftw

@@ -191,7 +191,11 @@ def test_workspace_and_plan(lib):
     assert path == ft.PATH_TC and n == 1
     path, n = ft.plan(True, 1, 8, 10000, 512, 32, 1, ft.FT_F32)
     assert path == ft.PATH_TC and n == 2
-    path, n = ft.plan(False, 1, 8, 4096, 64, 256, 1, ft.FT_F32)    # w > 32: CUDA cores
+    path, n = ft.plan(False, 1, 8, 4096, 64, 256, 1, ft.FT_F32)    # w > 32, d = 64: WIDE sub-bands
+    assert path == ft.PATH_TC and n == 1
+    path, n = ft.plan(True, 1, 8, 4096, 64, 256, 1, ft.FT_F32)     # D = dout . out, dQ, dK / dV
+    assert path == ft.PATH_TC and n == 3
+    path, n = ft.plan(False, 1, 8, 4096, 128, 256, 1, ft.FT_F32)   # w > 32, d != 64: CUDA cores
     assert path == ft.PATH_SIMT
     path, n = ft.plan(True, 1, 1, 64, 16, 4, 1, ft.FT_F32)
     assert path == ft.PATH_SIMT and n >= 1

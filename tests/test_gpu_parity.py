@@ -144,6 +144,62 @@ def test_tc32_parity(ft, shape):
     run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=16)
 
 
+# fp32 wide windows on the tensor cores (tc_band32.cu WIDE: the band cut into sub-bands of <= 65
+# offsets, one 192-row halo each, online softmax across them; d = 64): smallest wide window (two
+# sub-bands), w >= L, dilation with ragged residues and two launch groups, 31 sub-bands, many tiles
+TC32_WIDE = [(1, 1, 300, 64, 33, 1), (1, 2, 700, 64, 100, 1), (1, 1, 520, 64, 200, 2), (1, 1, 90, 64, 100, 1),
+             (1, 2, 1100, 64, 256, 3), (1, 2, 1300, 64, 40, 11), (1, 1, 2100, 64, 1000, 1),
+             (2, 3, 4096, 64, 256, 1)]
+
+
+@pytest.mark.parametrize("shape", TC32_WIDE, ids=lambda s: "x".join(map(str, s)))
+def test_tc32_wide_parity(ft, shape):
+    run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=17)
+
+
+@pytest.mark.parametrize("sign", [1, -1])
+def test_tc32_wide_rescale(ft, sign):
+    """fp32 wide forward with logits that grow along the keys (q = e_0, k_j0 = 0.15 j - 37, both
+    exact in bf16, so the hi / lo score products are exact): every later sub-band's max exceeds the
+    running one by more than the 2^20 lazy-rescale threshold (sign = 1), or never does (-1).  The
+    rescale lives in the forward; the backward of these |k| ~ 40 inputs is held to reading A10b's
+    error model instead of the plain 1e-4 bound (the hi / lo dS operand carries ~2^-17 of each
+    |dS_ij k_j| term, and dq cancels terms of size ~40 down to ~1e-2)."""
+    L, w, d = 500, 150, 64
+    shape = WinAttnShape(1, 2, L, d, w, 1)
+    x = make_inputs(shape, 10, "f32")
+    j = torch.arange(L, dtype=torch.float64)
+    q64 = torch.zeros(1, 2, L, d, dtype=torch.float64)
+    q64[..., 0] = 1.0
+    k64 = torch.zeros(1, 2, L, d, dtype=torch.float64)
+    k64[..., 0] = (sign * (0.15 * j - 37.0)).to(torch.bfloat16).double().view(1, 1, L)
+    dev = torch.device("cuda:0")
+    q, k = q64.float().to(dev), k64.float().to(dev)
+    v, g = x["v"].to(dev), x["dout"].to(dev)
+    out, lse = ft.fwd(q, k, v, w, 1)
+    dq, dk, dv = ft.bwd(q, k, v, out, lse, g, w, 1)
+    torch.cuda.synchronize()
+    ro, rl = oracle.fwd(q64.numpy(), k64.numpy(), x["v64"], w, 1)
+    r = oracle.bwd(q64.numpy(), k64.numpy(), x["v64"], ro, rl, x["dout64"], w, 1)
+    compare("out", out.double().cpu().numpy(), ro, "f32")
+    compare("lse", lse.double().cpu().numpy(), rl, "f32")
+    compare("dv", dv.double().cpu().numpy(), r[2], "f32")
+    # dq_i = sum_j dS_ij k_j: bound 2^-15 sum_j |dS_ij| |k_j| (4x the model) + 1e-4 max|dq|
+    P = np.zeros((2, L, L))
+    ii, jj = np.meshgrid(np.arange(L), np.arange(L), indexing="ij")
+    band = np.abs(ii - jj) <= w
+    for h in range(2):
+        S = np.where(band, np.outer(q64[0, h, :, 0].numpy(), k64[0, h, :, 0].numpy()), -np.inf)
+        Ph = np.exp(S - rl[0, h][:, None])
+        dP = x["dout64"][0, h] @ x["v64"][0, h].T
+        Dh = (x["dout64"][0, h] * ro[0, h]).sum(-1)
+        dS = np.where(band, Ph * (dP - Dh[:, None]), 0.0)
+        bound = 2.0 ** -15 * np.abs(dS) @ np.abs(k64[0, h].numpy()) + 1e-4 * np.abs(r[0]).max()
+        err = np.abs(dq[0, h].double().cpu().numpy() - r[0][0, h])
+        assert (err <= bound).all(), (h, float((err / bound).max()))
+    assert torch.isfinite(dk).all()
+
+
 # The dS tape between the tensor-core backward kernels (FT_KNOB_DSTAPE, DESIGN.md §10): the dK/dV kernel
 # reads P and dS from the dQ kernel instead of recomputing them, with the per-tile flag hand-off
 # (PDL on) or plain stream order (PDL off); many tiles per CTA, ragged residues, several launches
