@@ -82,7 +82,7 @@ constexpr int NCONV = 6;                  // converter warps
 constexpr int RES_PER_LAUNCH = 8;
 static_assert(RES_PER_LAUNCH <= SCHED_MAX_RES, "residue table of the tile cursor");
 constexpr uint32_t R0 = 0, R1 = 192, RACC = 384;
-constexpr int WMAX_SB = 64;               // sub-bands of a WIDE launch (w <= 2079)
+constexpr int WMAX_SB = 64;               // steps of a WIDE tile (w <= 6080)
 constexpr float RESCALE_LOG2 = 20.f;      // WIDE FWD lazy rescaling: P <= 2^20 between max moves
 constexpr float LOG2E = 1.4426950408889634f;
 constexpr float LN2 = 0.6931471805599453f;
@@ -112,12 +112,11 @@ struct Params {
     float* tP;
     float* tS;
     unsigned long long* trace;   // optional phase trace (ft_winattn_debug_trace), see trace32()
-    // WIDE (w > 32, d = 64): the band of offsets [-w, w] is cut into nsb sub-bands of <= 65
-    // offsets, [sb_lo[s], sb_lo[s] + sb_w2[s]], visited in this order (the one holding offset 0
-    // first); each (tile, sub-band) step is one pass of this kernel's normal work over a 192-row
-    // halo starting at m0 + sb_lo (keys; FWD, BWDQ) or m0 - sb_lo - sb_w2 (queries; BWDKV).
+    // WIDE (w > 32, d = 64): a tile's 128 + 2w halo rows are visited in nsb steps of NK = 192
+    // rows, step s covering halo rows [m0 - w + 192 s, m0 - w + 192 s + 192) (keys for FWD / BWDQ,
+    // queries for BWDKV); each (tile, step) is one pass of this kernel's normal work, masked by
+    // |i - j| <= w, with the accumulators live across the steps of a tile.
     int nsb;
-    int sb_lo[WMAX_SB], sb_w2[WMAX_SB];
 };
 
 // Phase trace (profiling only): per CTA, clock64 stamps of its first TR_SLOTS slots --
@@ -254,11 +253,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     const int ncw = (d + CW - 1) / CW;      // output chunks per tensor (the last may be 64 wide)
     const int nacc = ncw * C::NOUT;         // accumulations per tile
     const int nsb = WIDE ? p.nsb : 1;       // sub-bands per tile
-    // first halo row of sub-band sb relative to m0 (normal mode: -w)
-    auto koff = [&](int sb) -> int {
-        if (!WIDE) return -w;
-        return MODE == BWDKV ? -p.sb_lo[sb] - p.sb_w2[sb] : p.sb_lo[sb];
-    };
+    // first halo row of step sb relative to m0 (normal mode: -w)
+    auto koff = [&](int sb) -> int { return WIDE ? -w + (int)NK * sb : -w; };
 
     if (MODE == BWDQ && p.xt) {   // clear this CTA's tile flags before BWDKV may launch
         TileCursor cr(p.sc);
@@ -616,13 +612,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         int j = 0;
         if (MODE == BWDKV && !p.dpoll) asm volatile("griddepcontrol.wait;" ::: "memory");
         if constexpr (WIDE) {
-            // One (tile, sub-band) step at a time.  FWD: online softmax over the sub-bands with
-            // lazy rescaling (the running max m only moves when a sub-band's max exceeds it by more
+            // One (tile, step) at a time.  FWD: online softmax over the steps with
+            // lazy rescaling (the running max m only moves when a step's max exceeds it by more
             // than 2^RESCALE_LOG2; then this row's O partial in TMEM and l are scaled by 2^(m_old -
             // m_new) after the previous step's output GEMMs completed).  BWDQ / BWDKV: the global lse
             // and D (= dout . out, computed before the launch) make every step independent.
             int k = 0;
             float m_run = 0.f, l_run = 0.f;
+            bool m_set = false;   // FWD: the row has met a band entry (m_run is one of its scores)
             while (cur.next(p.sc, T)) {
                 const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t;
                 const int64_t rowbase = (int64_t)T.u * p.L + T.r;
@@ -633,8 +630,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     Drow = p.D[rowbase + (int64_t)mrow * p.dil];
                 }
                 for (int sb = 0; sb < nsb; ++sb, ++k) {
-                    const int W2 = p.sb_w2[sb], kb = m0 + koff(sb);
-                    const int chi = min(nch - 1, (32 * warp + 31 + W2) / 32);
+                    // column n of row t is in the band iff n - t + sh in [0, 2w] (halo row kb + n)
+                    const int sh = NK * sb, kb = m0 + koff(sb), W2 = 2 * w;
+                    const int nlo = 32 * warp - sh, nhi = 32 * warp + 31 - sh + W2;
+                    const int clo = nlo > 0 ? nlo / 32 : 0, chi = nhi < 0 ? -1 : min(nch - 1, nhi / 32);
                     if (MODE == BWDKV) {   // lse / D of this step's halo queries
                         named_bar_sync(1, 128);
                         for (int n = t; n < NK; n += 128) {
@@ -651,21 +650,28 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     const uint32_t rP = tbase + lane_off + R1;
                     if (MODE == FWD) {
                         float cm = -INFINITY;
-                        for (int c = c_lo; c <= chi; ++c) {
+                        for (int c = clo; c <= chi; ++c) {
                             uint32_t rr[32];
                             tmem_ld32(rS + c * 32, rr);
                             tmem_wait_ld();
 #pragma unroll
                             for (int e = 0; e < 32; ++e)
-                                if ((unsigned)(c * 32 + e - t) <= (unsigned)W2 && kb + c * 32 + e >= 0 && kb + c * 32 + e < Lr)
+                                if ((unsigned)(c * 32 + e - t + sh) <= (unsigned)W2 && kb + c * 32 + e >= 0 && kb + c * 32 + e < Lr)
                                     cm = fmaxf(cm, __uint_as_float(rr[e]));
                         }
                         const float cms = cm * LOG2E;
                         float fac = 1.f;
                         bool need = false;
                         if (sb == 0) {
-                            m_run = cm == -INFINITY ? 0.f : cms;
+                            m_set = false;
+                            m_run = 0.f;
                             l_run = 0.f;
+                        }
+                        if (!m_set) {   // O and l of this row are still 0: take this step's max
+                            if (cm != -INFINITY) {
+                                m_run = cms;
+                                m_set = true;
+                            }
                         } else if (cm != -INFINITY && cms > m_run + RESCALE_LOG2) {
                             need = true;
                             fac = fast_exp2(m_run - cms);
@@ -688,7 +694,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         }
                         float sum2[2] = {0.f, 0.f};
                         for (int c = 0; c < nch; ++c) {
-                            if (c < c_lo || c > chi) {
+                            if (c < clo || c > chi) {
                                 tmem_st16(rS + c * 32, zero16);
                                 tmem_st16(rS + c * 32 + 16, zero16);
                                 continue;
@@ -704,8 +710,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                                     float a0, a1;
                                     ffma2_bc(__uint_as_float(rr[e]), __uint_as_float(rr[e + 1]), LOG2E, -m_run, a0, a1);
                                     const int n = n0 + e;
-                                    const float p0 = (unsigned)(n - t) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
-                                    const float p1 = (unsigned)(n + 1 - t) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
+                                    const float p0 = (unsigned)(n - t + sh) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
+                                    const float p1 = (unsigned)(n + 1 - t + sh) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
                                     fadd2_acc(sum2[0], sum2[1], p0, p1);
                                     split2(p0, p1, pk[e / 2], pl[e / 2]);
                                 }
@@ -724,7 +730,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         }
                     } else if (MODE == BWDQ) {   // dS = P (dP - D) -> hi | lo over S
                         for (int c = 0; c < nch; ++c) {
-                            if (c < c_lo || c > chi) {
+                            if (c < clo || c > chi) {
                                 tmem_st16(rS + c * 32, zero16);
                                 tmem_st16(rS + c * 32 + 16, zero16);
                                 continue;
@@ -741,8 +747,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                                     float a0, a1, q0, q1, d0, d1;
                                     const int n = n0 + e;
                                     ffma2_bc(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, -lse2, a0, a1);
-                                    const float p0 = (unsigned)(n - t) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
-                                    const float p1 = (unsigned)(n + 1 - t) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
+                                    const float p0 = (unsigned)(n - t + sh) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
+                                    const float p1 = (unsigned)(n + 1 - t + sh) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
                                     ffma2_bc(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, -Drow, q0, q1);
                                     fmul2(p0, p1, q0, q1, d0, d1);
                                     split2(d0, d1, pk[e / 2], pl[e / 2]);
@@ -756,7 +762,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         warp_arrive(&p_full[k & 1]);
                     } else {   // BWDKV: rows keys, columns halo queries; P^T over dP^T, dS^T over S^T
                         for (int c = 0; c < nch; ++c) {
-                            if (c < c_lo || c > chi) {
+                            if (c < clo || c > chi) {
                                 tmem_st16(rS + c * 32, zero16);
                                 tmem_st16(rS + c * 32 + 16, zero16);
                                 tmem_st16(rP + c * 32, zero16);
@@ -775,8 +781,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                                     float pv[2], dv[2], a0, a1, q0, q1;
                                     const int n = n0 + e;
                                     ffma2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, LOG2E, -colLse[n], -colLse[n + 1], a0, a1);
-                                    pv[0] = (unsigned)(n - t) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
-                                    pv[1] = (unsigned)(n + 1 - t) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
+                                    pv[0] = (unsigned)(n - t + sh) <= (unsigned)W2 && kb + n >= 0 && kb + n < Lr ? fast_exp2(a0) : 0.f;
+                                    pv[1] = (unsigned)(n + 1 - t + sh) <= (unsigned)W2 && kb + n + 1 >= 0 && kb + n + 1 < Lr ? fast_exp2(a1) : 0.f;
                                     ffma2(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, 1.f, -colD[n], -colD[n + 1], q0, q1);
                                     fmul2(pv[0], pv[1], q0, q1, dv[0], dv[1]);
                                     split2(pv[0], pv[1], pk[e / 2], pl[e / 2]);
@@ -1138,40 +1144,13 @@ int halo_rows32(int64_t L, int64_t w) {
     return (int)(((BM + 2 * wc) + 63) / 64 * 64);
 }
 
-// WIDE sub-bands: the residue-space offsets [-wm, wm] (wm = min(w, longest residue - 1)) in
-// nsb <= WMAX_SB runs of <= 65 offsets, the run holding offset 0 first, then the others by their
-// distance from it (so the forward's first running max is a real row max estimate).
-struct SubBands {
-    int n = 0;
-    int lo[WMAX_SB], w2[WMAX_SB];
-};
-inline bool sub_bands(int64_t L, int64_t w, int64_t dil, SubBands& sb) {
+// WIDE steps: ceil((128 + 2w) / 192) halo windows of 192 rows per tile (w clamped to the longest
+// residue), at most WMAX_SB.
+inline int wide_steps(int64_t L, int64_t w, int64_t dil) {
     const int64_t Lr = (L + dil - 1) / dil;
-    const int64_t wm = w < Lr - 1 ? w : Lr - 1;
-    const int64_t tot = 2 * wm + 1;
-    const int n = (int)((tot + 64) / 65);
-    if (n > WMAX_SB) return false;
-    int lo[WMAX_SB], w2[WMAX_SB], c = 0;
-    int64_t o = -wm;
-    for (int i = 0; i < n; ++i) {   // near-equal runs
-        const int64_t len = tot / n + (i < tot % n ? 1 : 0);
-        lo[i] = (int)o;
-        w2[i] = (int)(len - 1);
-        if (o <= 0 && 0 <= o + len - 1) c = i;
-        o += len;
-    }
-    sb.n = 0;
-    sb.lo[sb.n] = lo[c];
-    sb.w2[sb.n++] = w2[c];
-    for (int dd = 1; dd < n; ++dd)
-        for (int sgn = -1; sgn <= 1; sgn += 2) {
-            const int i = c + sgn * dd;
-            if (i >= 0 && i < n) {
-                sb.lo[sb.n] = lo[i];
-                sb.w2[sb.n++] = w2[i];
-            }
-        }
-    return true;
+    const int64_t wm = w < Lr ? w : Lr;
+    const int64_t n = (BM + 2 * wm + 191) / 192;
+    return n <= WMAX_SB ? (int)n : 0;
 }
 
 // D_i = dout_i . out_i (fp32; the WIDE backward's exact-to-rounding D, reading R1 for fp32 out):
@@ -1205,8 +1184,8 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
     });
     const int64_t wc = w < L ? w : L;
     const int NK = WIDE ? 192 : halo_rows32(L, w);
-    SubBands sbp;
-    if (WIDE && !sub_bands(L, w, dil, sbp)) return cudaErrorInvalidValue;
+    const int nsteps = WIDE ? wide_steps(L, w, dil) : 1;
+    if (nsteps == 0) return cudaErrorInvalidValue;
     if (WIDE) tape = nullptr;
     const int64_t units = B * H;
     const int64_t nres = dil < L ? dil : L;
@@ -1236,18 +1215,12 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         p.D = D;
         p.L = L;
         p.d = (int)d;
-        p.w = (int)wc;
+        p.w = WIDE ? (int)(wc < ceil_div(L, dil) ? wc : ceil_div(L, dil)) : (int)wc;   // (wide_steps' clamp)
         p.dil = (int)dil;
         p.NK = NK;
         p.nsl = (int)(d / 32);
         p.dpoll = MODE != FWD && dpoll_enabled() && !WIDE;   // BWDQ marks its D rows, BWDKV polls them
-        if (WIDE) {
-            p.nsb = sbp.n;
-            for (int i = 0; i < sbp.n; ++i) {
-                p.sb_lo[i] = sbp.lo[i];
-                p.sb_w2[i] = sbp.w2[i];
-            }
-        }
+        if (WIDE) p.nsb = nsteps;
         if (tape && MODE != FWD && d > CW) {   // xt needs two output chunks (acc_rid alternation)
             p.xt = 1;
             p.tsw = tape->tsw;
@@ -1306,8 +1279,7 @@ bool tc32_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil)
     const int64_t wc = w < L ? w : L;
     if (!(dil <= 256 && units * ((L + 127) / 128) < (1 << 30))) return false;
     if (wc <= 32) return d % 64 == 0 && d <= 512;
-    SubBands sb;
-    return d == 64 && sub_bands(L, w, dil, sb);
+    return d == 64 && wide_steps(L, w, dil) > 0;
 }
 int tc32_fwd_launches(int64_t L, int64_t w, int64_t dil) { return band32_launches(L, dil); }
 int tc32_bwd_launches(int64_t L, int64_t w, int64_t dil) { return 2 * band32_launches(L, dil) + (tc32_wide(L, w) ? 1 : 0); }
