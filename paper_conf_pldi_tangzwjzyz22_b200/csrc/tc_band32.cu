@@ -117,6 +117,7 @@ struct Params {
     // queries for BWDKV); each (tile, step) is one pass of this kernel's normal work, masked by
     // |i - j| <= w, with the accumulators live across the steps of a tile.
     int nsb;
+    int pdl_free;   // WIDE BWDKV launched with PDL behind BWDQ: no data dependency, waits at exit
 };
 
 // Phase trace (profiling only): per CTA, clock64 stamps of its first TR_SLOTS slots --
@@ -610,7 +611,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         TileCursor cur(p.sc);
         Tile T;
         int j = 0;
-        if (MODE == BWDKV && !p.dpoll) asm volatile("griddepcontrol.wait;" ::: "memory");
+        if (MODE == BWDKV && !p.dpoll && !p.pdl_free) asm volatile("griddepcontrol.wait;" ::: "memory");
         if constexpr (WIDE) {
             // One (tile, step) at a time.  FWD: online softmax over the steps with
             // lazy rescaling (the running max m only moves when a step's max exceeds it by more
@@ -1120,6 +1121,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         if (lane == 0) tma_store_wait_all<0>();
     }
     tc_fence_before();
+    // (a PDL-launched grid that never waited must not complete before its primary: stream order
+    // for whatever follows it)
+    if (p.pdl_free) asm volatile("griddepcontrol.wait;" ::: "memory");
     __syncthreads();
     if (warp == 8) {
         tc_fence_after();
@@ -1221,6 +1225,9 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         p.nsl = (int)(d / 32);
         p.dpoll = MODE != FWD && dpoll_enabled() && !WIDE;   // BWDQ marks its D rows, BWDKV polls them
         if (WIDE) p.nsb = nsteps;
+        // WIDE: the dK/dV kernel needs only lse and D (both final before the dQ kernel starts), so it
+        // runs beside the dQ kernel as SMs free up
+        p.pdl_free = WIDE && MODE == BWDKV && r0 == 0 && dpoll_enabled();
         if (tape && MODE != FWD && d > CW) {   // xt needs two output chunks (acc_rid alternation)
             p.xt = 1;
             p.tsw = tape->tsw;
@@ -1240,7 +1247,7 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         // dQ kernel's launch follows the forward's only launch
         p.lsepoll = lsepoll_enabled() && nres <= RES_PER_LAUNCH && lsepoll_worth(total, num_sms32()) &&
                     !(MODE == BWDKV && p.xt) && !WIDE;   // the tape dK/dV kernel reads no lse
-        if ((MODE == BWDKV && r0 == 0 && p.dpoll) || (MODE == BWDQ && p.lsepoll)) {
+        if ((MODE == BWDKV && r0 == 0 && p.dpoll) || (MODE == BWDQ && p.lsepoll) || p.pdl_free) {
             // BWDKV directly after this call's last BWDQ launch; BWDQ after the forward
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = grid;
