@@ -622,6 +622,26 @@ def test_determinism_every_family(ft, shape):
             assert torch.equal(a, b)
 
 
+@pytest.mark.parametrize("shape", [(1, 4, 3000, 512, 32, 1), (1, 3, 2000, 64, 200, 2), (1, 8, 4096, 64, 32, 1)],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_determinism_fp32(ft, shape):
+    """fp32 tensor-core kernels (band, with its dS tape at d = 512; WIDE steps at w > 32; d = 64
+    band): bit-identical on repeated runs, with and without programmatic dependent launch (the
+    dK/dV kernel's tape flag hand-off, the WIDE dK/dV kernel launched beside the dQ kernel)."""
+    sh = WinAttnShape(*shape)
+    x = make_inputs(sh, 14, "f32")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    runs = []
+    for pdl in (1, 1, 1, 0):
+        with ft.knobs(pdl=pdl):
+            out, lse = ft.fwd(q, k, v, sh.w, sh.dilation)
+            runs.append((out, lse) + ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation))
+    for r in runs[1:]:
+        for a, b in zip(runs[0], r):
+            assert torch.equal(a, b)
+
+
 def test_autograd_mixed_dilation(ft):
     """win_attn with per-head dilation through torch.autograd against the oracle per head group."""
     B, H, L, d, w, dil, hd = 1, 3, 260, 64, 8, 3, 1

@@ -15,7 +15,8 @@ for shape, dt in [((1, 2, 300, 64, 32, 3), "bf16"), ((1, 4, 1500, 64, 32, 1), "b
                   ((1, 1, 600, 64, 100, 2), "bf16"), ((1, 1, 500, 128, 80, 1), "bf16"),
                   ((1, 1, 130, 64, 8, 1), "f32"), ((1, 2, 300, 512, 32, 1), "f32"),
                   ((1, 2, 257, 128, 17, 3), "f32"), ((1, 1, 300, 192, 8, 1), "f32"),
-                  ((1, 1, 500, 384, 32, 1), "bf16"), ((1, 2, 400, 256, 16, 2), "f32")]:   # last two: dS tape
+                  ((1, 1, 500, 384, 32, 1), "bf16"), ((1, 2, 400, 256, 16, 2), "f32"),   # these two: dS tape
+                  ((1, 1, 600, 64, 100, 2), "f32"), ((1, 2, 500, 64, 40, 1), "f32")]:     # fp32 WIDE steps
     s = WinAttnShape(*shape)
     x = make_inputs(s, 0, dt)
     q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
@@ -61,8 +62,9 @@ for f, dt in ((64, "f32"), (13, "f32"), (64, "bf16")):
 torch.cuda.synchronize()
 print("cases ok")
 PY
-for variant in default nopdl; do
-  for tool in memcheck racecheck synccheck initcheck; do
+# one tool per call is the safe pattern on this pool: TOOLS="memcheck" tools/sanitize.sh
+for variant in ${VARIANTS:-default nopdl}; do
+  for tool in ${TOOLS:-memcheck racecheck synccheck initcheck}; do
     echo "== $tool ($variant)"
     timeout 600 compute-sanitizer --tool $tool --kernel-name kns=tc_ --kernel-name kns=simt --kernel-name kns=circdiff --kernel-name kns=f32_to_bf16 --kernel-name kns=zero_f32 --print-limit 10 \
       python /tmp/san_case.py $([ $variant = nopdl ] && echo nopdl) 2>&1 | tail -4
