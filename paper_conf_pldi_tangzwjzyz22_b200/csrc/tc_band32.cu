@@ -254,6 +254,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     const int ncw = (d + CW - 1) / CW;      // output chunks per tensor (the last may be 64 wide)
     const int nacc = ncw * C::NOUT;         // accumulations per tile
     const int nsb = WIDE ? p.nsb : 1;       // sub-bands per tile
+    // WIDE backward: the epilogue warps also run the softmax (column halves; no row reduction
+    // there), so each step's softmax takes about half as long
+    constexpr bool SPLITSM = WIDE && MODE != FWD;
     // first halo row of step sb relative to m0 (normal mode: -w)
     auto koff = [&](int sb) -> int { return WIDE ? -w + (int)NK * sb : -w; };
 
@@ -339,7 +342,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             }
             for (int i = 0; i < 2; ++i) {
                 mbar_init(&s_full[i], 1);
-                mbar_init(&p_full[i], 4);
+                mbar_init(&p_full[i], SPLITSM ? 8 : 4);
             }
             for (int i = 0; i < 3; ++i) {
                 mbar_init(&o_full[i], 1);
@@ -451,6 +454,63 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 }
                 for (int a = 0; a < nacc; ++a)
                     for (int kb = 0; kb < nkb; ++kb) fn(1, To, a, kb, 0);
+            }
+        }
+    };
+
+    // ------------------------------------------------------------------ drain of one tile
+    // Epilogue warps 4-7 (TMEM lanes 32 (warp - 4) ..): every accumulation of tile T -> fp32 ->
+    // staging box -> TMA store, scaled by `scale` (FWD: 1/l of the row).
+    auto drain_tile = [&](const Tile& T, int j, int& sidx, AccUses& uses, float scale) {
+        const int ew = warp - 4;
+        const uint32_t tlane = tbase + ((uint32_t)(ew * 32) << 16);
+        uint8_t* mystg = stg + ew * nstg * STG;
+        const Maps& mp = p.maps[T.rl];
+        for (int a = 0; a < nacc; ++a) {
+            const int c = C::NOUT == 2 ? a % ncw : a;
+            const CUtensorMap* om = (C::NOUT == 2 && a < ncw) ? &mp.o2 : &mp.o1;   // BWDKV: dV first
+            const int ngrp = chunk_w(d, c) / 32;
+            const int rid = acc_rid(a);
+            const uint32_t trow = tlane + acc_col(rid);
+            mbar_wait(&o_full[rid], (uint32_t)uses.get(rid) & 1u);
+            uses.inc(rid);
+            tc_fence_after();
+            if (ew == 0 && lane == 0) trace_tile(p, j, 2 + a);
+            // two rounds of 64 columns (register budget of 16 warps); the accumulator is
+            // released once the last columns are in registers
+#pragma unroll
+            for (int x = 0; x < 4; ++x) {
+                if (x >= ngrp) break;
+                uint32_t ov[1][32];
+                tmem_ld32(trow + 32 * x, ov[0]);
+                tmem_wait_ld();
+                if (x == ngrp - 1) {
+                    tc_fence_before();
+                    warp_arrive(&o_empty[rid]);
+                    if (xt && a % ncw == ncw - 2) warp_arrive(&xfree[a < ncw ? 1 : 0]);
+                }
+                uint8_t* sb = mystg + (sidx % nstg) * STG;
+                if (lane == 0 && sidx >= nstg) {
+                    if (nstg == 2) tma_store_wait_read<1>();
+                    else tma_store_wait_read<0>();
+                }
+                __syncwarp();
+#pragma unroll
+                for (int g = 0; g < 8; ++g) {
+                    uint4 val;
+                    val.x = __float_as_uint(__uint_as_float(ov[0][4 * g + 0]) * scale);
+                    val.y = __float_as_uint(__uint_as_float(ov[0][4 * g + 1]) * scale);
+                    val.z = __float_as_uint(__uint_as_float(ov[0][4 * g + 2]) * scale);
+                    val.w = __float_as_uint(__uint_as_float(ov[0][4 * g + 3]) * scale);
+                    *reinterpret_cast<uint4*>(sb + lane * 128 + ((g ^ (lane & 7)) << 4)) = val;
+                }
+                fence_proxy_async_smem();
+                __syncwarp();
+                if (lane == 0) {
+                    tma_store_3d(om, sb, CW * c + 32 * x, T.m0 + 32 * ew, T.u);
+                    tma_store_commit();
+                }
+                ++sidx;
             }
         }
     };
@@ -600,11 +660,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 if (++st == nst) { st = 0; ph ^= 1u; }
             });
         }
-    } else if (warp < 4) {   // ------------------------------------------------ softmax warps
-        const int t = warp * 32 + lane;
-        const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+    } else if (warp < 4 || (SPLITSM && warp < 8)) {   // -------------------------- softmax warps
+        // SPLITSM: warps 4-7 take the upper half of every row's chunks and drain the tile after its
+        // last step (they are the epilogue warps)
+        const int hsm = SPLITSM ? warp / 4 : 0, wq = warp % 4;
+        const int t = wq * 32 + lane;
+        const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
         // chunks holding any band column of this warp's rows: [32 warp, 32 warp + 31 + 2w]
-        const int c_lo = warp, c_hi = min(nch - 1, (32 * warp + 31 + 2 * w) / 32);
+        const int c_lo = wq, c_hi = min(nch - 1, (32 * wq + 31 + 2 * w) / 32);
         uint32_t zero16[16];
 #pragma unroll
         for (int e = 0; e < 16; ++e) zero16[e] = 0u;
@@ -618,7 +681,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             // than 2^RESCALE_LOG2; then this row's O partial in TMEM and l are scaled by 2^(m_old -
             // m_new) after the previous step's output GEMMs completed).  BWDQ / BWDKV: the global lse
             // and D (= dout . out, computed before the launch) make every step independent.
-            int k = 0;
+            int k = 0, sidx = 0;
+            AccUses euses;   // SPLITSM drainers (warps 4-7)
             float m_run = 0.f, l_run = 0.f;
             bool m_set = false;   // FWD: the row has met a band entry (m_run is one of its scores)
             while (cur.next(p.sc, T)) {
@@ -633,17 +697,22 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 for (int sb = 0; sb < nsb; ++sb, ++k) {
                     // column n of row t is in the band iff n - t + sh in [0, 2w] (halo row kb + n)
                     const int sh = NK * sb, kb = m0 + koff(sb), W2 = 2 * w;
-                    const int nlo = 32 * warp - sh, nhi = 32 * warp + 31 - sh + W2;
+                    const int nlo = 32 * wq - sh, nhi = 32 * wq + 31 - sh + W2;
                     const int clo = nlo > 0 ? nlo / 32 : 0, chi = nhi < 0 ? -1 : min(nch - 1, nhi / 32);
+                    // chunks this warp handles: all (FWD), or its half of [clo, chi] plus the zero
+                    // chunks on its side (SPLITSM)
+                    const int cm = (clo + chi + 1) >> 1;
+                    auto mine = [&](int c) { return !SPLITSM || (hsm == 0 ? c < cm : c >= cm); };
                     if (MODE == BWDKV) {   // lse / D of this step's halo queries
-                        named_bar_sync(1, 128);
-                        for (int n = t; n < NK; n += 128) {
+                        constexpr int NSMT = SPLITSM ? 256 : 128;
+                        named_bar_sync(1, NSMT);
+                        for (int n = hsm * 128 + t; n < NK; n += NSMT) {
                             const int mc = kb + n;
                             const bool ok = mc >= 0 && mc < Lr;
                             colLse[n] = ok ? p.lse[rowbase + (int64_t)mc * p.dil] * LOG2E : 0.f;
                             colD[n] = ok ? p.D[rowbase + (int64_t)mc * p.dil] : 0.f;
                         }
-                        named_bar_sync(1, 128);
+                        named_bar_sync(1, NSMT);
                     }
                     mbar_wait(&s_full[MODE == FWD ? (k & 1) : 0], MODE == FWD ? ((k >> 1) & 1) : (k & 1));
                     tc_fence_after();
@@ -731,6 +800,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         }
                     } else if (MODE == BWDQ) {   // dS = P (dP - D) -> hi | lo over S
                         for (int c = 0; c < nch; ++c) {
+                            if (!mine(c)) continue;
                             if (c < clo || c > chi) {
                                 tmem_st16(rS + c * 32, zero16);
                                 tmem_st16(rS + c * 32 + 16, zero16);
@@ -763,6 +833,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         warp_arrive(&p_full[k & 1]);
                     } else {   // BWDKV: rows keys, columns halo queries; P^T over dP^T, dS^T over S^T
                         for (int c = 0; c < nch; ++c) {
+                            if (!mine(c)) continue;
                             if (c < clo || c > chi) {
                                 tmem_st16(rS + c * 32, zero16);
                                 tmem_st16(rS + c * 32 + 16, zero16);
@@ -800,8 +871,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         warp_arrive(&p_full[k & 1]);
                     }
                 }
+                if (SPLITSM && hsm == 1) drain_tile(T, j, sidx, euses, 1.f);
                 ++j;
             }
+            if (SPLITSM && hsm == 1 && lane == 0) tma_store_wait_all<0>();
         }
         bool lse_settled = false;   // ld_lse_ready fell back to griddepcontrol.wait
         while (!WIDE && cur.next(p.sc, T)) {
@@ -1054,68 +1127,18 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
             ++j;
         }
     } else if (warp < 8) {   // ----------------------------------------------- epilogue warps
-        const int ew = warp - 4;   // TMEM lanes 32 ew ..
-        const uint32_t tlane = tbase + ((uint32_t)(ew * 32) << 16);
-        uint8_t* mystg = stg + ew * nstg * STG;
         TileCursor cur(p.sc);
         Tile T;
         int j = 0, sidx = 0;
         AccUses uses;
         while (cur.next(p.sc, T)) {
-            const Maps& mp = p.maps[T.rl];
             float scale = 1.f;
             if (MODE == FWD) {   // 1/l of this row, published before p_full (WIDE: rs_full)
                 if (WIDE) mbar_wait(&rs_full[j & 1], (j >> 1) & 1);
                 else mbar_wait(&p_full[j & 1], (j >> 1) & 1);
-                scale = rowScale[(j % 3) * 128 + ew * 32 + lane];
+                scale = rowScale[(j % 3) * 128 + (warp - 4) * 32 + lane];
             }
-            for (int a = 0; a < nacc; ++a) {
-                const int c = C::NOUT == 2 ? a % ncw : a;
-                const CUtensorMap* om = (C::NOUT == 2 && a < ncw) ? &mp.o2 : &mp.o1;   // BWDKV: dV first
-                const int ngrp = chunk_w(d, c) / 32;
-                const int rid = acc_rid(a);
-                const uint32_t trow = tlane + acc_col(rid);
-                mbar_wait(&o_full[rid], (uint32_t)uses.get(rid) & 1u);
-                uses.inc(rid);
-                tc_fence_after();
-                if (ew == 0 && lane == 0) trace_tile(p, j, 2 + a);
-                // two rounds of 64 columns (register budget of 16 warps); the accumulator is
-                // released once the last columns are in registers
-#pragma unroll
-                for (int x = 0; x < 4; ++x) {
-                    if (x >= ngrp) break;
-                    uint32_t ov[1][32];
-                    tmem_ld32(trow + 32 * x, ov[0]);
-                    tmem_wait_ld();
-                    if (x == ngrp - 1) {
-                        tc_fence_before();
-                        warp_arrive(&o_empty[rid]);
-                        if (xt && a % ncw == ncw - 2) warp_arrive(&xfree[a < ncw ? 1 : 0]);
-                    }
-                    uint8_t* sb = mystg + (sidx % nstg) * STG;
-                    if (lane == 0 && sidx >= nstg) {
-                        if (nstg == 2) tma_store_wait_read<1>();
-                        else tma_store_wait_read<0>();
-                    }
-                    __syncwarp();
-#pragma unroll
-                    for (int g = 0; g < 8; ++g) {
-                        uint4 val;
-                        val.x = __float_as_uint(__uint_as_float(ov[0][4 * g + 0]) * scale);
-                        val.y = __float_as_uint(__uint_as_float(ov[0][4 * g + 1]) * scale);
-                        val.z = __float_as_uint(__uint_as_float(ov[0][4 * g + 2]) * scale);
-                        val.w = __float_as_uint(__uint_as_float(ov[0][4 * g + 3]) * scale);
-                        *reinterpret_cast<uint4*>(sb + lane * 128 + ((g ^ (lane & 7)) << 4)) = val;
-                    }
-                    fence_proxy_async_smem();
-                    __syncwarp();
-                    if (lane == 0) {
-                        tma_store_3d(om, sb, CW * c + 32 * x, T.m0 + 32 * ew, T.u);
-                        tma_store_commit();
-                    }
-                    ++sidx;
-                }
-            }
+            drain_tile(T, j, sidx, uses, scale);
             ++j;
         }
         if (lane == 0) tma_store_wait_all<0>();
