@@ -406,6 +406,28 @@ def test_full_size_whole_units(ft, name):
             compare(f"{n}[head {h}]", a[:, h:h + 1].double().cpu().numpy(), r, "bf16")
 
 
+@pytest.mark.parametrize("name", ["C4d2", "C5_big_w256"])
+def test_full_size_whole_units_f32(ft, name):
+    """fp32 wide windows at full size on the tensor cores (tc_band32.cu WIDE steps): the first and
+    last (batch, head) units element by element against the oracle at the fp32 bound."""
+    shape = CONFIGS[name]
+    x = make_inputs(shape, 0, "f32")
+    dev = torch.device("cuda:0")
+    for bwd in (False, True):
+        p, _ = ft.plan(bwd, shape.batch, shape.heads, shape.seq_len, shape.d, shape.w, shape.dilation, 0)
+        assert p == ft.PATH_TC
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    out, lse = ft.fwd(q, k, v, shape.w, shape.dilation)
+    dq, dk, dv = ft.bwd(q, k, v, out, lse, g, shape.w, shape.dilation)
+    torch.cuda.synchronize()
+    for h in sorted({0, shape.heads - 1}):
+        s = {n: np.ascontiguousarray(x[n + "64"][:, h:h + 1]) for n in ("q", "k", "v", "dout")}
+        ro, rl = oracle.fwd(s["q"], s["k"], s["v"], shape.w, shape.dilation)
+        rq, rk, rv = oracle.bwd(s["q"], s["k"], s["v"], ro, rl, s["dout"], shape.w, shape.dilation)
+        for n, a, r in (("out", out, ro), ("lse", lse, rl), ("dq", dq, rq), ("dk", dk, rk), ("dv", dv, rv)):
+            compare(f"{n}[head {h}]", a[:, h:h + 1].double().cpu().numpy(), r, "f32")
+
+
 @pytest.mark.parametrize("name,dtype", [("C2a_dil", "f32"), ("long_2M", "bf16")])
 def test_full_size_sampled(ft, name, dtype):
     shape = CONFIGS[name]
