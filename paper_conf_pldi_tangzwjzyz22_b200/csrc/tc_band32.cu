@@ -257,6 +257,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     // WIDE backward: the epilogue warps also run the softmax (column halves; no row reduction
     // there), so each step's softmax takes about half as long
     constexpr bool SPLITSM = WIDE && MODE != FWD;
+    // TMEM: R0 = [0, NK), R1 = [r1, r1 + NK), accumulators from racc.  WIDE d = 128 uses 128-row
+    // steps (R1 at 128, the accumulators at 256: BWDKV's dV and dK take 128 columns each).
+    const uint32_t r1 = (WIDE && d == 128) ? 128u : R1;
+    const uint32_t racc = (WIDE && d == 128) ? 256u : RACC;
     // first halo row of step sb relative to m0 (normal mode: -w)
     auto koff = [&](int sb) -> int { return WIDE ? -w + (int)NK * sb : -w; };
 
@@ -326,8 +330,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         return a < ncw ? 1 : 2;
     };
     // (the R1 accumulator sits at column 256, 128-aligned like the others)
-    auto acc_col = [](int rid) -> uint32_t {
-        if (WIDE) return RACC + 64u * rid;
+    auto acc_col = [&](int rid) -> uint32_t {
+        if (WIDE) return racc + (uint32_t)d * rid;
         return rid == 0 ? RACC : rid == 1 ? R0 : R1 + 64;
     };
     const int npl = (NK + TROWS - 1) / TROWS;   // tape slots per plane
@@ -590,7 +594,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     mbar_wait(&conv[st], ph);
                 } else if (kind == 0) {
                     // FWD: S(jg) into region jg & 1; BWD: S into R0, dP into R1
-                    const uint32_t dst = tbase + (MODE == FWD ? ((jg & 1) ? R1 : R0) : (b ? R1 : R0));
+                    const uint32_t dst = tbase + (MODE == FWD ? ((jg & 1) ? r1 : R0) : (b ? r1 : R0));
                     if (MODE != FWD && a == 0 && b == 0 && jg > 0) {
                         // R1 (dP) is free once the softmax of the previous tile read it (p_full);
                         // R0 (dS) once the previous tile's output MMAs read it (issue order)
@@ -630,8 +634,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         tc_fence_after();
                     }
                     const uint32_t Dacc = tbase + acc_col(rid);
-                    const uint32_t Areg = tbase + (MODE == FWD ? ((jo & 1) ? R1 : R0)
-                                                   : (MODE == BWDKV && a < ncw) ? R1 : R0);
+                    const uint32_t Areg = tbase + (MODE == FWD ? ((jo & 1) ? r1 : R0)
+                                                   : (MODE == BWDKV && a < ncw) ? r1 : R0);
                     const uint32_t id = chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW ? idO : idO64;
                     mbar_wait(&conv[st], ph);
                     tc_fence_after();
@@ -716,8 +720,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     }
                     mbar_wait(&s_full[MODE == FWD ? (k & 1) : 0], MODE == FWD ? ((k >> 1) & 1) : (k & 1));
                     tc_fence_after();
-                    const uint32_t rS = tbase + lane_off + (MODE == FWD && (k & 1) ? R1 : R0);
-                    const uint32_t rP = tbase + lane_off + R1;
+                    const uint32_t rS = tbase + lane_off + (MODE == FWD && (k & 1) ? r1 : R0);
+                    const uint32_t rP = tbase + lane_off + r1;
                     if (MODE == FWD) {
                         float cm = -INFINITY;
                         for (int c = clo; c <= chi; ++c) {
@@ -751,15 +755,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                         if (__any_sync(0xffffffffu, need)) {   // scale this warp's O rows (previous PV done)
                             mbar_wait(&pv_done[(k - 1) & 1], ((k - 1) >> 1) & 1);
                             tc_fence_after();
-#pragma unroll
-                            for (int h = 0; h < 2; ++h) {
+                            for (int h = 0; h < d / 32; ++h) {
                                 uint32_t ov[32];
-                                tmem_ld32(tbase + lane_off + RACC + 32 * h, ov);
+                                tmem_ld32(tbase + lane_off + racc + 32 * h, ov);
                                 tmem_wait_ld();
 #pragma unroll
                                 for (int e = 0; e < 32; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * fac);
-                                tmem_st16(tbase + lane_off + RACC + 32 * h, *reinterpret_cast<const uint32_t(*)[16]>(&ov[0]));
-                                tmem_st16(tbase + lane_off + RACC + 32 * h + 16, *reinterpret_cast<const uint32_t(*)[16]>(&ov[16]));
+                                tmem_st16(tbase + lane_off + racc + 32 * h, *reinterpret_cast<const uint32_t(*)[16]>(&ov[0]));
+                                tmem_st16(tbase + lane_off + racc + 32 * h + 16, *reinterpret_cast<const uint32_t(*)[16]>(&ov[16]));
                             }
                         }
                         float sum2[2] = {0.f, 0.f};
@@ -1171,12 +1174,14 @@ int halo_rows32(int64_t L, int64_t w) {
     return (int)(((BM + 2 * wc) + 63) / 64 * 64);
 }
 
-// WIDE steps: ceil((128 + 2w) / 192) halo windows of 192 rows per tile (w clamped to the longest
-// residue), at most WMAX_SB.
-inline int wide_steps(int64_t L, int64_t w, int64_t dil) {
+// WIDE steps: ceil((128 + 2w) / NK) halo windows of NK rows per tile (NK = 192 at d = 64, 128 at
+// d = 128; w clamped to the longest residue), at most WMAX_SB.
+inline int wide_nk(int64_t d) { return d == 128 ? 128 : 192; }
+inline int wide_steps(int64_t L, int64_t w, int64_t dil, int64_t d) {
     const int64_t Lr = (L + dil - 1) / dil;
     const int64_t wm = w < Lr ? w : Lr;
-    const int64_t n = (BM + 2 * wm + 191) / 192;
+    const int64_t nk = wide_nk(d);
+    const int64_t n = (BM + 2 * wm + nk - 1) / nk;
     return n <= WMAX_SB ? (int)n : 0;
 }
 
@@ -1210,8 +1215,8 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
                              (int)(SMEM_BYTES > SMEM_BYTES_XT ? SMEM_BYTES : SMEM_BYTES_XT));
     });
     const int64_t wc = w < L ? w : L;
-    const int NK = WIDE ? 192 : halo_rows32(L, w);
-    const int nsteps = WIDE ? wide_steps(L, w, dil) : 1;
+    const int NK = WIDE ? wide_nk(d) : halo_rows32(L, w);
+    const int nsteps = WIDE ? wide_steps(L, w, dil, d) : 1;
     if (nsteps == 0) return cudaErrorInvalidValue;
     if (WIDE) tape = nullptr;
     const int64_t units = B * H;
@@ -1302,14 +1307,14 @@ int band32_launches(int64_t L, int64_t dil) {
 
 }  // namespace
 
-// w > 32 runs the WIDE instantiation: d = 64 (its two accumulators, dV and dK, share the 128
-// accumulator columns across the sub-bands)
+// w > 32 runs the WIDE instantiation: d = 64 (192-row steps; dV and dK share the 128 accumulator
+// columns) or d = 128 (128-row steps; dV and dK take 128 columns each)
 static bool tc32_wide(int64_t L, int64_t w) { return (w < L ? w : L) > 32; }
 bool tc32_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
     const int64_t wc = w < L ? w : L;
     if (!(dil <= 256 && units * ((L + 127) / 128) < (1 << 30))) return false;
     if (wc <= 32) return d % 64 == 0 && d <= 512;
-    return d == 64 && wide_steps(L, w, dil) > 0;
+    return (d == 64 || d == 128) && wide_steps(L, w, dil, d) > 0;
 }
 int tc32_fwd_launches(int64_t L, int64_t w, int64_t dil) { return band32_launches(L, dil); }
 int tc32_bwd_launches(int64_t L, int64_t w, int64_t dil) { return 2 * band32_launches(L, dil) + (tc32_wide(L, w) ? 1 : 0); }

@@ -195,7 +195,9 @@ def test_workspace_and_plan(lib):
     assert path == ft.PATH_TC and n == 1
     path, n = ft.plan(True, 1, 8, 4096, 64, 256, 1, ft.FT_F32)     # D = dout . out, dQ, dK / dV
     assert path == ft.PATH_TC and n == 3
-    path, n = ft.plan(False, 1, 8, 4096, 128, 256, 1, ft.FT_F32)   # w > 32, d != 64: CUDA cores
+    path, n = ft.plan(False, 1, 8, 4096, 128, 256, 1, ft.FT_F32)   # w > 32, d = 128: 128-row steps
+    assert path == ft.PATH_TC
+    path, n = ft.plan(False, 1, 8, 4096, 192, 256, 1, ft.FT_F32)   # w > 32, d not in {64, 128}: CUDA cores
     assert path == ft.PATH_SIMT
     path, n = ft.plan(True, 1, 1, 64, 16, 4, 1, ft.FT_F32)
     assert path == ft.PATH_SIMT and n >= 1

@@ -144,12 +144,15 @@ def test_tc32_parity(ft, shape):
     run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=16)
 
 
-# fp32 wide windows on the tensor cores (tc_band32.cu WIDE: the band cut into sub-bands of <= 65
-# offsets, one 192-row halo each, online softmax across them; d = 64): smallest wide window (two
-# sub-bands), w >= L, dilation with ragged residues and two launch groups, 31 sub-bands, many tiles
+# fp32 wide windows on the tensor cores (tc_band32.cu WIDE: a tile's halo in steps of 192 rows at
+# d = 64, 128 rows at d = 128, online softmax across them): smallest wide window, w >= L, dilation
+# with ragged residues and two launch groups, many steps, many tiles
 TC32_WIDE = [(1, 1, 300, 64, 33, 1), (1, 2, 700, 64, 100, 1), (1, 1, 520, 64, 200, 2), (1, 1, 90, 64, 100, 1),
              (1, 2, 1100, 64, 256, 3), (1, 2, 1300, 64, 40, 11), (1, 1, 2100, 64, 1000, 1),
-             (2, 3, 4096, 64, 256, 1)]
+             (2, 3, 4096, 64, 256, 1),
+             # d = 128: 128-row steps
+             (1, 1, 300, 128, 33, 1), (1, 2, 700, 128, 100, 1), (1, 1, 520, 128, 200, 2), (1, 2, 1100, 128, 256, 3),
+             (1, 1, 90, 128, 100, 1)]
 
 
 @pytest.mark.parametrize("shape", TC32_WIDE, ids=lambda s: "x".join(map(str, s)))
