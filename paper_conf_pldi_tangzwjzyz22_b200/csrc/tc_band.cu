@@ -1143,12 +1143,21 @@ int band_launches(int64_t L, int64_t dil) {
 
 }  // namespace
 
+// Wide windows (halo > 256 rows): the one-pass wide kernels (d in {64, 128}), else the chunked
+// fallback kernels where their shared-memory plan fits.
+static bool wide_fwd_ok(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    return knob(K_WIDE) && tc_wide_supported(units, L, d, w, dil);
+}
+static bool wide_bwd_ok(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
+    return knob(K_WIDE) && tc_wide_bwd_supported(units, L, d, w, dil);
+}
 bool tc_fwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
     return halo_rows(L, w) <= 256 ? band_supported(units, L, d, w, dil)
-                                  : tc_chunk_supported(units, L, d, w, dil);
+                                  : (wide_fwd_ok(units, L, d, w, dil) || tc_chunk_supported(units, L, d, w, dil));
 }
 bool tc_bwd_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil) {
-    return tc_fwd_supported(units, L, d, w, dil);
+    return halo_rows(L, w) <= 256 ? band_supported(units, L, d, w, dil)
+                                  : (wide_bwd_ok(units, L, d, w, dil) || tc_chunk_supported(units, L, d, w, dil));
 }
 int tc_fwd_launches(int64_t L, int64_t d, int64_t w, int64_t dil) {
     if (tc_narrow_supported(1, L, d, w, dil)) return tc_narrow_launches(L, dil);
@@ -1165,7 +1174,7 @@ cudaError_t tc_fwd(const void* q, const void* k, const void* v, void* out, float
                    int* launches) {
     if (launches) *launches = 0;
     if (halo_rows(L, w) > 256) {
-        if (!knob(K_WIDE) || !tc_wide_supported(B * H, L, d, w, dil))
+        if (!wide_fwd_ok(B * H, L, d, w, dil))
             return tc_chunk_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
         return tc_wide_fwd(q, k, v, out, lse, B, H, L, d, w, dil, st, launches);
     }
@@ -1188,7 +1197,7 @@ cudaError_t tc_bwd(const void* q, const void* k, const void* v, const void* out,
     // wide kernels also compute it exactly, and read out only for the first-guess D~
     if (launches) *launches = 0;
     if (halo_rows(L, w) > 256) {
-        if (!knob(K_WIDE) || !tc_wide_bwd_supported(B * H, L, d, w, dil))
+        if (!wide_bwd_ok(B * H, L, d, w, dil))
             return tc_chunk_bwd(q, k, v, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
         return tc_wide_bwd(q, k, v, out, lse, dout, dq, dk, dv, Dws, B, H, L, d, w, dil, st, launches);
     }

@@ -402,10 +402,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                     }
                 };
                 // max of my half of S_c (log2 domain)
-                auto half_max = [&]() -> float {
+                // (reload = false: from the registers of the last load -- once P is packed over S in
+                // TMEM, d = 128, S can no longer be read back)
+                auto half_max = [&](bool reload) -> float {
                     float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
                     if (any_live) {
-                        load_half();
+                        if (reload) load_half();
 #pragma unroll
                         for (int x = 0; x < 2; ++x)
 #pragma unroll
@@ -417,14 +419,21 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                 // of entries: one FFMA2 (s log2e - mref), two ex2, one FADD2 (the two partial
                 // sums), one pack -- no running max: the rescale test below uses the row sum
                 // (every P <= the sum of the chunk's P).
-                auto exp_sweep = [&](float mref) -> float {
+                auto exp_sweep = [&](float mref, bool reload) -> float {
                     float lc[2] = {0.f, 0.f};
+                    if (!PSM && reload) {
+                        // P goes over S in TMEM, and this warp's packed P columns [16 sp, 16 sp + 32)
+                        // hold S of the partner warp's half when hf = 1: both warps must have read
+                        // their S halves before either stores
+                        if (any_live) load_half();
+                        named_bar_sync(1 + wq, 64);
+                    }
                     if (!any_live) {
                         if (PSM) { st_p_sub(Pb, t, sp, zero16); st_p_sub(Pb, t, sp + 1, zero16); }
                         else { tmem_st16(tS + sp * 16, zero16); tmem_st16(tS + sp * 16 + 16, zero16); }
                     } else {
                         unsigned long long q0 = tr ? gtime() : 0;
-                        load_half();
+                        if (PSM && reload) load_half();
                         if (tr) fine[0] += gtime() - q0;
 #pragma unroll
                         for (int x = 0; x < 2; ++x) {
@@ -479,7 +488,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                     if (mv) ms = cmf;
                 };
                 // rows without a running max yet (the first chunk): exact chunk max first
-                if (__any_sync(0xffffffffu, ms == -INFINITY)) move_max(xmax(half_max()));
+                if (__any_sync(0xffffffffu, ms == -INFINITY)) move_max(xmax(half_max(true)));
                 // optimistic sweep at the running max.  If some row's chunk sum exceeds
                 // 2^(RESCALE_LOG2 - 6) -- only then can one of its P exceed the threshold -- both
                 // warps take the chunk's exact max, move the running max where it exceeds it by
@@ -487,14 +496,14 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_fwd_kernel(const __grid_c
                 // chunk's exact max)
                 float lc;
                 unsigned long long q1 = tr ? gtime() : 0, q2 = 0;
-                lc = exp_sweep(ms == -INFINITY ? 0.f : ms);
+                lc = exp_sweep(ms == -INFINITY ? 0.f : ms, true);
                 if (tr) q2 = gtime();
                 const float rowsum = xsum(lc);
                 if (__any_sync(0xffffffffu, !(rowsum <= exp2f(RESCALE_LOG2 - 6.f)))) {   // (NaN: check)
-                    const float cm = xmax(half_max());
+                    const float cm = xmax(half_max(PSM));
                     if (__any_sync(0xffffffffu, cm > ms + RESCALE_LOG2)) {
                         move_max(cm);
-                        lc = exp_sweep(ms == -INFINITY ? 0.f : ms);
+                        lc = exp_sweep(ms == -INFINITY ? 0.f : ms, PSM);
                     }
                 }
                 if (tr) { fine[1] += q2 - q1; fine[2] += gtime() - q2; }

@@ -144,6 +144,34 @@ def test_tc32_parity(ft, shape):
     run_case(ft, WinAttnShape(*shape), "f32", "tc", seed=16)
 
 
+@pytest.mark.parametrize("shape", [(2, 1, 300, 128, 130, 1), (1, 3, 2000, 128, 256, 1), (1, 2, 1500, 128, 100, 3),
+                                   (1, 12, 4096, 128, 256, 1), (1, 1, 600, 128, 500, 1)],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_wide_d128(ft, shape):
+    """bf16, w > 64, d = 128 on the one-pass wide kernels (tc_wide.cu, tc_wide_bwd.cu): P packed
+    over S in TMEM, whose column halves belong to two warps (pair barrier before P is stored);
+    first and last heads element by element; three forward runs bit-identical."""
+    sh = WinAttnShape(*shape)
+    for bwd in (False, True):
+        assert ft.plan(bwd, sh.batch, sh.heads, sh.seq_len, sh.d, sh.w, sh.dilation, 1)[0] == ft.PATH_TC
+    x = make_inputs(sh, 18, "bf16")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    runs = [ft.fwd(q, k, v, sh.w, sh.dilation) for _ in range(3)]
+    torch.cuda.synchronize()
+    for o, l in runs[1:]:
+        assert torch.equal(o, runs[0][0]) and torch.equal(l, runs[0][1])
+    out, lse = runs[0]
+    dq, dk, dv = ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    hs = sorted({0, sh.heads - 1})
+    s64 = {n: np.ascontiguousarray(x[n + "64"][:, hs]) for n in ("q", "k", "v", "dout")}
+    ro, rl = oracle.fwd(s64["q"], s64["k"], s64["v"], sh.w, sh.dilation)
+    rq, rk, rv = oracle.bwd(s64["q"], s64["k"], s64["v"], ro, rl, s64["dout"], sh.w, sh.dilation)
+    for n, a, r in (("out", out, ro), ("lse", lse, rl), ("dq", dq, rq), ("dk", dk, rk), ("dv", dv, rv)):
+        compare(n, a[:, hs].double().cpu().numpy(), r, "bf16")
+
+
 # fp32 wide windows on the tensor cores (tc_band32.cu WIDE: a tile's halo in steps of 192 rows at
 # d = 64, 128 rows at d = 128, online softmax across them): smallest wide window, w >= L, dilation
 # with ragged residues and two launch groups, many steps, many tiles
