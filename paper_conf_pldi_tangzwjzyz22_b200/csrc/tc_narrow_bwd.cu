@@ -185,14 +185,20 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
     uint64_t* empty = bars + 2 * NSTAGE;    // [NSTAGE]
     uint64_t* s_full = bars + 3 * NSTAGE;   // S and dP of the tile done
     uint64_t* dp_free = s_full + 1;         // softmax holds S and dP in registers
-    uint64_t* p_done = s_full + 2;          // operands written and the dS halo converted
+    uint64_t* p_done = s_full + 2;          // the softmax warps wrote the tile's operands
     uint64_t* acc_full = s_full + 3;        // [2]
     uint64_t* acc_free = s_full + 5;        // [2]
     uint64_t* hs_full = s_full + 7;         // [2] halo row scales of tile j published
     uint64_t* s_full2 = s_full + 9;         // [2] S and dP of tile j done, for the converters (which
                                             // may lag the softmax by a tile: a single-phase barrier
                                             // would let its parity wrap)
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 11);
+    // [2] the converter warps converted tile j's dS halo.  Its own barrier, by tile parity: the
+    // converters may run a tile ahead of the softmax warps (they need only the tile's score GEMMs,
+    // which start once the softmax holds the previous tile's S and dP in registers), and sharing
+    // p_done let their arrivals for tile j+1 complete tile j's phase before the last softmax pair
+    // had written its rows of dS(j) -- 32 rows of dq / dk read a stale operand (~1-2 % of runs).
+    uint64_t* cv_done = s_full + 11;
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(s_full + 13);
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int w = p.w;
@@ -206,7 +212,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             }
             mbar_init(s_full, 1);
             mbar_init(dp_free, 8);
-            mbar_init(p_done, 8 + 2);
+            mbar_init(p_done, 8);
+            mbar_init(&cv_done[0], 2);
+            mbar_init(&cv_done[1], 2);
             for (int b = 0; b < 2; ++b) {
                 mbar_init(&acc_full[b], 1);
                 mbar_init(&acc_free[b], 8);
@@ -252,7 +260,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
         // cw owns halo rows 64 i + 32 cw + l, i < 3 (whole 128-byte rows: no shuffles, no second
         // read).  As soon as the TMA landed it loads its rows into registers, reduces each row's
         // largest |value| and publishes 2^-f (hs_full); once the score GEMM has read the bf16 halo
-        // (s_full2) it writes the rows times 2^f as fp16; the output MMAs read them after p_done.
+        // (s_full2) it writes the rows times 2^f as fp16; the output MMAs read them after cv_done.
         // (Two passes over shared memory, or eight lanes per row with shuffle reductions, left
         // this warp pair on the tile's critical path: tools/trace_narrow.py.)
         const int cw = warp - 10;
@@ -303,7 +311,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 }
             }
             fence_proxy_async_smem();
-            warp_arrive(p_done);
+            warp_arrive(&cv_done[j & 1]);
             if (lane == 0 && cw == 0) trace_ev(p, j, 12);
         }
     } else if (warp == 9) {
@@ -319,6 +327,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 const int s = i % NSTAGE, b = MODE == NQ ? (i & 1) : 0;
                 const uint32_t st = smem_u32(stages + (size_t)s * STAGE);
                 mbar_wait(p_done, i & 1);
+                mbar_wait(&cv_done[i & 1], (i >> 1) & 1);
                 if (MODE == NQ ? i >= 2 : i >= 1)
                     mbar_wait(&acc_free[b], (MODE == NQ ? (i - 2) >> 1 : i - 1) & 1);
                 tc_fence_after();

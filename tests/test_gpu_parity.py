@@ -695,6 +695,28 @@ def test_determinism_fp32(ft, shape):
             assert torch.equal(a, b)
 
 
+def test_narrow_backward_repeatable(ft):
+    """d = 64, w <= 32 backward (tc_narrow_bwd.cu): 40 repeated fwd + bwd calls give bit-identical
+    dq / dk / dv.  Its converter warps once arrived on the softmax warps' p_done barrier and,
+    running a tile ahead, could complete a tile's phase before the last softmax pair had written
+    its dS rows (32 rows of dq wrong in ~1-2 % of runs at this shape)."""
+    sh = WinAttnShape(1, 16, 8192, 64, 32, 1)
+    x = make_inputs(sh, 12, "bf16")
+    dev = torch.device("cuda:0")
+    q, k, v, g = (x[n].to(dev) for n in ("q", "k", "v", "dout"))
+    ref = None
+    for it in range(40):
+        with ft.knobs(pdl=it % 2):
+            out, lse = ft.fwd(q, k, v, sh.w, sh.dilation)
+            r = ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation)
+        torch.cuda.synchronize()
+        if ref is None:
+            ref = [t.clone() for t in r]
+            continue
+        for a, b in zip(r, ref):
+            assert torch.equal(a, b), it
+
+
 def test_autograd_mixed_dilation(ft):
     """win_attn with per-head dilation through torch.autograd against the oracle per head group."""
     B, H, L, d, w, dil, hd = 1, 3, 260, 64, 8, 3, 1
