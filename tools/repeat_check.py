@@ -1,0 +1,49 @@
+"""Repeatability sweep: every tensor-core family's fwd + bwd run N times on one input, every output
+compared bit for bit with the first run (the kernels own their output rows, no atomics, so any
+difference is a race).  Alternates the PDL knob.  Usage: python tools/repeat_check.py [N]"""
+import os
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_pldi_tangzwjzyz22_b200 as ft  # noqa: E402
+from synth import WinAttnShape, make_inputs  # noqa: E402
+
+CASES = [("narrow bf16 d64 w32", (1, 16, 8192, 64, 32, 1), "bf16"),
+         ("band bf16 d512 w32 (C2a)", (1, 8, 10000, 512, 32, 1), "bf16"),
+         ("band32 fp32 d512 w32 (C2a)", (1, 8, 10000, 512, 32, 1), "f32"),
+         ("band32 fp32 d64 w32", (1, 16, 8192, 64, 32, 1), "f32"),
+         ("wide bf16 d64 w256 d2", (1, 12, 16384, 64, 256, 2), "bf16"),
+         ("wide bf16 d128 w256", (1, 12, 4096, 128, 256, 1), "bf16"),
+         ("band32 WIDE fp32 d64 w256", (1, 12, 4096, 64, 256, 1), "f32"),
+         ("band32 WIDE fp32 d128 w100", (1, 8, 4096, 128, 100, 1), "f32"),
+         ("band bf16 d256 w16 d3", (1, 4, 6000, 256, 16, 3), "bf16")]
+
+
+def main():
+    n = int(sys.argv[1]) if len(sys.argv) > 1 else 50
+    dev = torch.device("cuda:0")
+    total_bad = 0
+    for name, shape, dt in CASES:
+        sh = WinAttnShape(*shape)
+        x = make_inputs(sh, 31, dt)
+        q, k, v, g = (x[t].to(dev) for t in ("q", "k", "v", "dout"))
+        ref, bad = None, 0
+        for it in range(n):
+            with ft.knobs(pdl=1 if it % 3 else 0):
+                out, lse = ft.fwd(q, k, v, sh.w, sh.dilation)
+                r = (out, lse) + ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation)
+            torch.cuda.synchronize()
+            if ref is None:
+                ref = [t.clone() for t in r]
+                continue
+            if not all(torch.equal(a, b) for a, b in zip(r, ref)):
+                bad += 1
+        total_bad += bad
+        print(f"{name:32s} {shape}: {bad} of {n - 1} repeats differ", flush=True)
+    print("total differing repeats:", total_bad)
+
+
+if __name__ == "__main__":
+    main()
