@@ -42,6 +42,35 @@ def main():
                 bad += 1
         total_bad += bad
         print(f"{name:32s} {shape}: {bad} of {n - 1} repeats differ", flush=True)
+    # one-call fwd + bwd (lse hand-off), per-head dilation (two streams), score tape
+    extra = [("fwd_bwd bf16 d512", (1, 8, 10000, 512, 32, 1), "bf16", "fwd_bwd"),
+             ("fwd_bwd fp32 d512", (1, 8, 10000, 512, 32, 1), "f32", "fwd_bwd"),
+             ("fwd_bwd narrow bf16", (1, 16, 8192, 64, 32, 1), "bf16", "fwd_bwd"),
+             ("mixed dilation bf16 d512", (1, 8, 10000, 512, 32, 4), "bf16", "mixed"),
+             ("mixed dilation fp32 d512", (1, 8, 10000, 512, 32, 4), "f32", "mixed"),
+             ("score tape bf16 d64", (1, 8, 4096, 64, 20, 1), "bf16", "tape")]
+    for name, shape, dt, kind in extra:
+        sh = WinAttnShape(*shape)
+        x = make_inputs(sh, 32, dt)
+        q, k, v, g = (x[t].to(dev) for t in ("q", "k", "v", "dout"))
+        ref, bad = None, 0
+        for it in range(n):
+            if kind == "fwd_bwd":
+                r = ft.fwd_bwd(q, k, v, g, sh.w, sh.dilation)
+            elif kind == "mixed":
+                out, lse = ft.fwd(q, k, v, sh.w, sh.dilation, dilated_heads=2)
+                r = (out, lse) + ft.bwd(q, k, v, out, lse, g, sh.w, sh.dilation, dilated_heads=2)
+            else:
+                out, lse, tp = ft.fwd_tape(q, k, v, sh.w, sh.dilation)
+                r = (out, lse) + ft.bwd_tape(q, k, v, out, lse, tp, g, sh.w, sh.dilation)
+            torch.cuda.synchronize()
+            if ref is None:
+                ref = [t.clone() for t in r]
+                continue
+            if not all(torch.equal(a, b) for a, b in zip(r, ref)):
+                bad += 1
+        total_bad += bad
+        print(f"{name:32s} {shape}: {bad} of {n - 1} repeats differ", flush=True)
     print("total differing repeats:", total_bad)
 
 
