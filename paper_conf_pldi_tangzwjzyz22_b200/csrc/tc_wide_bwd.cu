@@ -109,9 +109,11 @@ __device__ __forceinline__ void split_bf16x2(float x0, float x1, uint32_t& hi, u
     split_bf16x2_p(x0, x1, hi, lo);   // tc_common.cuh: one packed subtraction
 }
 
-// WQ: dQ (d = 64: hi and lo partials) + with wqc the PK = sum_j P_ij k_j accumulator
+// WQ: dQ + with wqc the PK = sum_j P_ij k_j accumulator (at column d); WKV: dV, dK (at d).  The
+// hi and lo products of dS share one accumulator (d = 64 had them in two partials, which cost a
+// 64-column TMEM region: 5 instead of 6 regions of score-GEMM lookahead)
 template <int MODE> __host__ __device__ inline int acc_cols(int d, int wqc) {
-    return MODE == WQ ? 128 + (wqc ? d : 0) : (d == 64 ? 192 : 256);
+    return MODE == WQ ? d + (wqc ? d : 0) : 2 * d;
 }
 template <int MODE> __host__ __device__ inline int n_regions(int d, int wqc) { return (512 - acc_cols<MODE>(d, wqc)) / 64; }
 __host__ __device__ inline uint32_t row_bytes(int d) { return (uint32_t)(d / 64) * ABOX; }
@@ -319,11 +321,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             int j = 0, gk = 0;
             TileCursor cur(p.sc);
             Tile T;
-            // dQ (WQ, dS hi/lo over S) or dK (WKV, dS^T hi/lo over dP^T): hi into column 0
-            // (+ d for dK), lo into the next d columns for d = 64 (separate partial: two
-            // 4-deep chains), into the same accumulator for d = 128.
+            // dQ (WQ, dS hi/lo over S) or dK (WKV, dS^T hi/lo over dP^T): hi and lo products
+            // into one accumulator at column 0 (+ d for dK)
             const uint32_t acc_hi = MODE == WQ ? 0u : (uint32_t)d;
-            const uint32_t acc_lo = d == 64 ? acc_hi + (uint32_t)d : acc_hi;
+            const uint32_t acc_lo = acc_hi;
             while (cur.next(p.sc, T)) {
                 int outk = 0;   // output steps issued in this tile
                 const bool tr = p.trace && j < 8;
@@ -353,9 +354,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                         const uint32_t ta = tbase + xa;
                         const uint32_t acc = outk == 0 ? 0u : 1u;
                         mma_ts_x4o<8, 32, 40, 128>(tbase + acc_hi, ta, bd, idO, acc);
-                        mma_ts_x4o<8, 32, 40, 128>(tbase + acc_lo, ta + 16, bd, idO, d == 64 ? acc : 1u);
+                        mma_ts_x4o<8, 32, 40, 128>(tbase + acc_lo, ta + 16, bd, idO, 1u);
                         if (wqc)   // PK += P K_c, P (bf16) packed over dP
-                            mma_ts_x4o<8, 32, 40, 128>(tbase + 128u, tbase + region_col(mD), bd, idO, acc);
+                            mma_ts_x4o<8, 32, 40, 128>(tbase + (uint32_t)d, tbase + region_col(mD), bd, idO, acc);
                     }
                     mma_commit(&rfree[(MODE == WQ ? mS : mD) % NREG]);
                     if (MODE == WQ) {
@@ -561,11 +562,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             if (ew == 0 && lane == 0) trace_put(p, j, 30, gtime());
             if (lane == 0) tma_store_wait_read<0>();   // staging of the previous tile read
             __syncwarp();
-            // WQ: dQ = [0, d) (+ [d, 2d) for d = 64);  WKV: dV = [0, d), dK = [d, 2d) (+ [2d, 3d))
+            // WQ: dQ = [0, d);  WKV: dV = [0, d), dK = [d, 2d)
             const int nout = MODE == WKV ? 2 : 1;
             for (int o = 0; o < nout; ++o) {
                 const uint32_t c0 = MODE == WQ ? 0u : (o == 0 ? 0u : (uint32_t)d);
-                const bool two = d == 64 && (MODE == WQ || o == 1);
+                const bool two = false;
                 const CUtensorMap* om = o == 0 ? &mp.o1 : &mp.o2;
                 for (int s = 0; s < nds; ++s) {
                     uint8_t* stg = mystg + s * STG;
@@ -579,7 +580,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                         const uint32_t col = c0 + (uint32_t)(s * 64 + hh * 32);
                         tmem_ld32(trow + col, v0);
                         if (two) tmem_ld32(trow + col + (uint32_t)d, v1);
-                        if (wqc) tmem_ld32(trow + 128u + col, v2);   // PK
+                        if (wqc) tmem_ld32(trow + (uint32_t)d + col, v2);   // PK
                         tmem_wait_ld();
                         float acc[32];
 #pragma unroll
