@@ -25,8 +25,9 @@
 //
 // Roles (512 threads): softmax warps 0-7 (warps w and w+4 share rows 32w.. -- TMEM lane
 // quarter w -- and take the two 32-column halves of every step); epilogue warps 8-11;
-// warp 12 TMA producer + TMEM allocator; issuers: warp 13 A (S / S^T), warp 14 B (dP / dP^T,
-// and dV), warp 15 C (dQ / dK, hi and lo).
+// warp 12 TMA producer + TMEM allocator; issuers: warp 13 A (S / S^T), warp 14 B (dP / dP^T),
+// warp 15 C (the output GEMMs once the softmax of a step is done: dQ, or dV and dK -- B issuing
+// dV(k-1) behind dP^T(k) held dV, and with it the S^T region, behind dP^T's region wait).
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -190,7 +191,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                 mbar_init(&p_full[i], 256);
             }
             for (int i = 0; i < 8; ++i) mbar_init(&rfree[i], 1);
-            mbar_init(o_full, MODE == WKV ? 2 : 1);
+            mbar_init(o_full, 1);
             mbar_init(o_empty, 128);
             mbar_init(&d_full[0], 256);
             mbar_init(&d_full[1], 256);
@@ -260,21 +261,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
         if (lane == 0) {   // ------------------------------- issuers A (S) and B (dP, dV)
             const bool isA = warp == 13;
             Ring rr;   // ring 1 (A) or ring 2 (B)
-            Ring rv;   // B, WKV: the ring-2 slot of the previous step (dV)
             int j = 0, gk = 0;
             TileCursor cur(p.sc);
             Tile T;
-            // WKV, issuer B: dV(step g) = P^T(g) dO_c(g), P^T packed bf16 in g's S region
-            auto issue_dv = [&](int g, bool first) {
-                mbar_wait(&p_full[g & 3], (g >> 2) & 1);
-                tc_fence_after();
-                const uint32_t xs = region_col(2 * g);
-                const uint32_t sb = smem_u32(sR2 + (size_t)rv.s * SB);
-                mma_ts_x4o<8, 32, 40, 128>(tbase, tbase + xs, sdesc_sw128(sb, HBOX, 1024), idO, first ? 0u : 1u);
-                mma_commit(&rfree[(2 * g) % NREG]);
-                mma_commit(&r2_empty[rv.s]);
-                rv.adv(p.n2);
-            };
             while (cur.next(p.sc, T)) {
                 const int ab = j % p.na;
                 mbar_wait(&a_full[ab], (j / p.na) & 1);
@@ -300,18 +289,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     if (isA) mma_commit(&r1_empty[rr.s]);
                     else if (MODE == WQ) mma_commit(&r2_empty[rr.s]);
                     rr.adv(isA ? p.n1 : p.n2);
-                    if (MODE == WKV && !isA && k > 0) {
-                        if (k == 1 && j > 0) { mbar_wait(o_empty, (j - 1) & 1); tc_fence_after(); }
-                        issue_dv(gk - 1, k == 1);
-                    }
                 }
                 mma_commit(&a_empty[ab]);
                 if (tr) { trace_put(p, j, isA ? 10 : 14, wr); trace_put(p, j, isA ? 11 : 15, wf); }
-                if (MODE == WKV && !isA) {   // the tile's last dV
-                    if (nsteps == 1 && j > 0) { mbar_wait(o_empty, (j - 1) & 1); tc_fence_after(); }
-                    issue_dv(gk - 1, nsteps == 1);
-                    mma_commit(o_full);
-                }
                 ++j;
             }
         }
@@ -325,6 +305,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
             // into one accumulator at column 0 (+ d for dK)
             const uint32_t acc_hi = MODE == WQ ? 0u : (uint32_t)d;
             const uint32_t acc_lo = acc_hi;
+            Ring rv;   // WKV: ring 2 (dO_c), read again here by dV = P^T dO_c after issuer B's dP^T
             while (cur.next(p.sc, T)) {
                 int outk = 0;   // output steps issued in this tile
                 const bool tr = p.trace && j < 8;
@@ -346,6 +327,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_wide_bwd_kernel(const __grid_c
                     if (tr) t0 = gtime();
                     if (outk == 0 && j > 0) { mbar_wait(o_empty, (j - 1) & 1); tc_fence_after(); }
                     if (tr) wo += gtime() - t0;
+                    if (MODE == WKV) {   // dV += P^T dO_c, P^T packed bf16 in the S region
+                        mbar_wait(&r2_full[rv.s], rv.ph);   // (landed long ago: issuer B's dP^T read it)
+                        tc_fence_after();
+                        const uint32_t sv = smem_u32(sR2 + (size_t)rv.s * SB);
+                        mma_ts_x4o<8, 32, 40, 128>(tbase, tbase + region_col(mS), sdesc_sw128(sv, HBOX, 1024), idO,
+                                                   outk == 0 ? 0u : 1u);
+                        mma_commit(&rfree[mS % NREG]);
+                        mma_commit(&r2_empty[rv.s]);
+                        rv.adv(p.n2);
+                    }
                     const uint32_t xa = region_col(MODE == WQ ? mS : mD);   // dS (hi/lo) region
                     const uint32_t sb = smem_u32(sR1 + (size_t)r1.s * SB);
                     {   // K-steps kk = 0..3 of the 64-key chunk: A columns 0, 8, 32, 40 (hi;
