@@ -26,7 +26,8 @@ overlap inside the timed region), "hbm_step" (whole step vs SURVEY.md §8(d)
 algorithmic bytes), "cpu_baseline" (the fp64 oracle on a bounded sample, rank 0, N=1),
 "e2e" (pinned host buffers, H2D + fwd + bwd + D2H inside the timed region), "clocks"
 (NVML samples during the timed region), "gpu_launches", and the sub-records "bf16" / "f32"
-(the other storage dtype), "fwd_bwd_call" (the one-call API) and "strong_scaling".
+(the other storage dtype), "fwd_bwd_call" (the one-call API), "strong_scaling" and, at N = 1,
+"other_configs" (every other BASELINE configuration timed in the same run).
 """
 from __future__ import annotations
 
@@ -698,6 +699,39 @@ def main():
             "hbm_frac_per_gpu": step_bytes_per_row(sd, se) * U * sL / world / (s_ms / 1e3) / 1e9 / hbm_peak
             if s_ms > 0 else None,
             "scaling": "strong", "timing": "compute only (slab resident on its GPU), CUDA events, max over ranks"}
+
+    # (d) the other BASELINE configurations on one GPU, so the driver's record carries every
+    # configs[] shape: C2b (Longformer-base, reading A14(b)) in both dtypes, C4 (configs[3],
+    # dilation 2 and 4), the C5 sweep corners (configs[4]) -- ms per fwd + bwd step, the path,
+    # and the step against its binding ceiling (HBM bytes of SURVEY.md §8(d) or tensor flops)
+    if not args.no_extras and args.extra_steps > 0 and world == 1:
+        others = {}
+        for wl, odt in (("C2b", "bf16"), ("C2b", "f32"), ("C4d2", "bf16"), ("C4d4", "bf16"), ("C4d2", "f32"),
+                        ("C5_w32", "bf16"), ("C5_w256", "bf16"), ("C5_small", "bf16")):
+            if wl == args.workload:
+                continue
+            oB, oH, oL, od, ow, odil = WORKLOADS[wl][:6]
+            oe = 2 if odt == "bf16" else 4
+            code = ft.FT_BF16 if odt == "bf16" else ft.FT_F32
+            try:
+                ms = quick_time(ft, torch, dev, (oB, oH, oL, od, ow, odil), odt, args.extra_steps, 3)
+            except Exception as ex:
+                others[f"{wl}/{odt}"] = {"error": f"{type(ex).__name__}: {ex}"[:200]}
+                continue
+            orows = oB * oH * oL
+            hbm_f = step_bytes_per_row(od, oe) * orows / (ms / 1e3) / 1e9 / hbm_peak
+            # band entries per row (exact), 12 d flops each for fwd + bwd; fp32 on the tensor cores
+            # counts its 3 bf16 products
+            n_i = float(window_sizes(oL, ow, odil).sum())
+            fl = 12.0 * od * n_i * oB * oH * (3 if odt == "f32" else 1)
+            ten_f = fl / (ms / 1e3) / (bf16_peak * 1e12)
+            pth = dict(zip(("fwd", "bwd"), ("tc" if ft.plan(b_, oB, oH, oL, od, ow, odil, code)[0] == ft.PATH_TC
+                                            else "simt" for b_ in (False, True))))
+            others[f"{wl}/{odt}"] = {"shape": {"heads": oH, "seq_len": oL, "d": od, "w": ow, "dilation": odil},
+                                     "ms_per_step": ms, "tokens_per_s": oB * oL / (ms / 1e3), "paths": pth,
+                                     "hbm_frac": hbm_f, "tensor_frac": ten_f,
+                                     "binding": "hbm" if hbm_f >= ten_f else "tensor"}
+        extras["other_configs"] = others
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
