@@ -18,7 +18,13 @@ CASES = [("narrow bf16 d64 w32", (1, 16, 8192, 64, 32, 1), "bf16"),
          ("wide bf16 d128 w256", (1, 12, 4096, 128, 256, 1), "bf16"),
          ("band32 WIDE fp32 d64 w256", (1, 12, 4096, 64, 256, 1), "f32"),
          ("band32 WIDE fp32 d128 w100", (1, 8, 4096, 128, 100, 1), "f32"),
-         ("band bf16 d256 w16 d3", (1, 4, 6000, 256, 16, 3), "bf16")]
+         ("band bf16 d256 w16 d3", (1, 4, 6000, 256, 16, 3), "bf16"),
+         ("narrow bf16 d64 w20 d3", (2, 6, 5001, 64, 20, 3), "bf16"),
+         ("wide bf16 d64 w100 d4", (1, 6, 9001, 64, 100, 4), "bf16"),
+         ("wide bf16 d128 w130 d2", (1, 4, 6001, 128, 130, 2), "bf16"),
+         ("band32 fp32 d256 w32 d5 (tape)", (1, 3, 7001, 256, 32, 5), "f32"),
+         ("band32 WIDE fp32 d64 w300 d3", (1, 4, 7001, 64, 300, 3), "f32"),
+         ("very wide bf16 d64 w2000 (chunk)", (1, 2, 5000, 64, 2000, 1), "bf16")]
 
 
 def main():
