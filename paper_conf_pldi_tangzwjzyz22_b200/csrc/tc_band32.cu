@@ -117,6 +117,7 @@ struct Params {
     // queries for BWDKV); each (tile, step) is one pass of this kernel's normal work, masked by
     // |i - j| <= w, with the accumulators live across the steps of a tile.
     int nsb;
+    int kbw;        // WIDE: keys per output block (NK itself when one block fits a slot, else KB)
     int pdl_free;   // WIDE BWDKV launched with PDL behind BWDQ: no data dependency, waits at exit
 };
 
@@ -250,7 +251,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     uint8_t* smem = smem_raw + (((raw_u32 + 1023u) & ~1023u) - raw_u32);
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int NK = p.NK, nsl = p.nsl, w = p.w, d = p.d;
-    const int nkb = NK / KB, nch = NK / 32;
+    const int kbw = WIDE ? p.kbw : KB;        // keys per output block
+    const int nkb = NK / kbw, nch = NK / 32;
     const int ncw = (d + CW - 1) / CW;      // output chunks per tensor (the last may be 64 wide)
     const int nacc = ncw * C::NOUT;         // accumulations per tile
     const int nsb = WIDE ? p.nsb : 1;       // sub-bands per tile
@@ -259,7 +261,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     constexpr bool SPLITSM = WIDE && MODE != FWD;
     // TMEM: R0 = [0, NK), R1 = [r1, r1 + NK), accumulators from racc.  WIDE d = 128 uses 128-row
     // steps (R1 at 128, the accumulators at 256: BWDKV's dV and dK take 128 columns each).
-    const uint32_t r1 = (WIDE && d == 128) ? 128u : R1;
+    const uint32_t r1 = WIDE ? (d == 128 ? 128u : (uint32_t)NK) : R1;
     const uint32_t racc = (WIDE && d == 128) ? 256u : RACC;
     // first halo row of step sb relative to m0 (normal mode: -w)
     auto koff = [&](int sb) -> int { return WIDE ? -w + (int)NK * sb : -w; };
@@ -549,9 +551,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     const int c = C::NOUT == 2 ? a % ncw : a;
                     const int nbox = chunk_w(d, c) / 32;
                     const CUtensorMap* m = (C::NOUT == 2 && a >= ncw) ? &mp.ob2 : &mp.ob1;
-                    mbar_arrive_expect_tx(&full[st], (uint32_t)nbox * KB * 128u);
+                    mbar_arrive_expect_tx(&full[st], (uint32_t)nbox * kbw * 128u);
                     for (int x = 0; x < nbox; ++x)
-                        tma_load_3d(sp + x * KB * 128, m, &full[st], CW * c + 32 * x, T.m0 + koff(sb) + KB * b, T.u);
+                        tma_load_3d(sp + x * kbw * 128, m, &full[st], CW * c + 32 * x, T.m0 + koff(sb) + kbw * b, T.u);
                 }
                 if (++st == nst) { st = 0; ph ^= 1u; }
             });
@@ -570,7 +572,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 convert_rows2<64>(sp, BM, sp + 2 * BM * 64, NK, ct);
             } else {
                 const bool full_chunk = chunk_w(d, C::NOUT == 2 ? a % ncw : a) == CW;
-                convert_rows2<128>(sp, KB, sp + 2 * KB * 128, full_chunk ? KB : 0, ct);
+                convert_rows2<128>(sp, kbw, sp + 2 * kbw * 128, full_chunk ? kbw : 0, ct);
             }
             fence_proxy_async_smem();
             warp_arrive(&conv[st]);
@@ -640,12 +642,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                     mbar_wait(&conv[st], ph);
                     tc_fence_after();
                     trace_slot(p, k, 3);
-#pragma unroll
-                    for (int kk = 0; kk < 4; ++kk) {
-                        const int g = 4 * b + kk;   // 16-key step over the halo
+                    const int kpb = kbw / 16;   // 16-key steps per output block
+#pragma unroll 4
+                    for (int kk = 0; kk < kpb; ++kk) {
+                        const int g = kpb * b + kk;   // 16-key step over the halo
                         const uint32_t tA = Areg + 16u * g;   // hi words; lo words at + 8
-                        const uint64_t dbh = sdesc_sw128(sa + kk * 2048, 2 * KB * 128, 1024);
-                        const uint64_t dbl = sdesc_sw128(sa + KB * 128 + kk * 2048, 2 * KB * 128, 1024);
+                        const uint64_t dbh = sdesc_sw128(sa + kk * 2048, 2 * kbw * 128, 1024);
+                        const uint64_t dbl = sdesc_sw128(sa + kbw * 128 + kk * 2048, 2 * kbw * 128, 1024);
                         mma_ts(Dacc, tA, dbh, id, !first_sb || g != 0);
                         mma_ts(Dacc, tA, dbl, id, 1);
                         mma_ts(Dacc, tA + 8, dbh, id, 1);
@@ -1176,13 +1179,30 @@ int halo_rows32(int64_t L, int64_t w) {
 
 // WIDE steps: ceil((128 + 2w) / NK) halo windows of NK rows per tile (NK = 192 at d = 64, 128 at
 // d = 128; w clamped to the longest residue), at most WMAX_SB.
-inline int wide_nk(int64_t d) { return d == 128 ? 128 : 192; }
-inline int wide_steps(int64_t L, int64_t w, int64_t dil, int64_t d) {
+// The steps are balanced: n = ceil(halo / NKmax) steps (NKmax = 192 at d = 64, 128 at d = 128) of
+// NK = halo / n rows rounded up to 32 -- e.g. 4 x 160 for w = 256 instead of 3 x 192 + a 64-row
+// remainder that costs a whole step.  At d = 64 with NK <= 160 a step's keys form one output
+// block (NK x 64 fp32 <= one 40 KB slot); otherwise blocks of KB = 64 keys (NK a multiple of 64).
+struct WideGeo {
+    int n, nk, kbw;
+};
+inline bool wide_geo(int64_t L, int64_t w, int64_t dil, int64_t d, WideGeo& g) {
     const int64_t Lr = (L + dil - 1) / dil;
     const int64_t wm = w < Lr ? w : Lr;
-    const int64_t nk = wide_nk(d);
-    const int64_t n = (BM + 2 * wm + nk - 1) / nk;
-    return n <= WMAX_SB ? (int)n : 0;
+    const int64_t halo = BM + 2 * wm, nkmax = d == 128 ? 128 : 192;
+    const int64_t n = (halo + nkmax - 1) / nkmax;
+    if (n > WMAX_SB) return false;
+    int64_t nk = ((halo + n - 1) / n + 31) / 32 * 32;
+    int kbw = (int)nk;
+    if (!(d == 64 && nk <= 160)) {
+        nk = (nk + 63) / 64 * 64;
+        kbw = KB;
+    }
+    if (nk > nkmax) return false;
+    g.n = (int)n;
+    g.nk = (int)nk;
+    g.kbw = kbw;
+    return true;
 }
 
 // D_i = dout_i . out_i (fp32; the WIDE backward's exact-to-rounding D, reading R1 for fp32 out):
@@ -1215,9 +1235,11 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
                              (int)(SMEM_BYTES > SMEM_BYTES_XT ? SMEM_BYTES : SMEM_BYTES_XT));
     });
     const int64_t wc = w < L ? w : L;
-    const int NK = WIDE ? wide_nk(d) : halo_rows32(L, w);
-    const int nsteps = WIDE ? wide_steps(L, w, dil, d) : 1;
-    if (nsteps == 0) return cudaErrorInvalidValue;
+    WideGeo wg = {1, 0, KB};
+    if (WIDE && !wide_geo(L, w, dil, d, wg)) return cudaErrorInvalidValue;
+    const int NK = WIDE ? wg.nk : halo_rows32(L, w);
+    const int nsteps = WIDE ? wg.n : 1;
+    const int kbw = WIDE ? wg.kbw : KB;
     if (WIDE) tape = nullptr;
     const int64_t units = B * H;
     const int64_t nres = dil < L ? dil : L;
@@ -1231,11 +1253,11 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
             Maps& m = p.maps[i];
             bool ok = make_residue_map_f32(&m.a1, a1, L, d, units, dil, r, BM, 16) &&
                       make_residue_map_f32(&m.b1, b1, L, d, units, dil, r, NK, 16) &&
-                      make_residue_map_f32(&m.ob1, ob1, L, d, units, dil, r, KB) &&
+                      make_residue_map_f32(&m.ob1, ob1, L, d, units, dil, r, kbw) &&
                       make_residue_map_f32(&m.o1, o1, L, d, units, dil, r, 32);
             if (ok && a2) ok = make_residue_map_f32(&m.a2, a2, L, d, units, dil, r, BM, 16);
             if (ok && b2) ok = make_residue_map_f32(&m.b2, b2, L, d, units, dil, r, NK, 16);
-            if (ok && ob2) ok = make_residue_map_f32(&m.ob2, ob2, L, d, units, dil, r, KB);
+            if (ok && ob2) ok = make_residue_map_f32(&m.ob2, ob2, L, d, units, dil, r, kbw);
             if (ok && o2) ok = make_residue_map_f32(&m.o2, o2, L, d, units, dil, r, 32);
             if (ok && tape && MODE == BWDKV && d > CW) {
                 ok = make_residue_map_tape(&m.tp, tape->P, L, tape->tsw, units, dil, r, TBOX, tape->grows) &&
@@ -1253,6 +1275,7 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         p.nsl = (int)(d / 32);
         p.dpoll = MODE != FWD && dpoll_enabled() && !WIDE;   // BWDQ marks its D rows, BWDKV polls them
         if (WIDE) p.nsb = nsteps;
+        p.kbw = kbw;
         // WIDE: the dK/dV kernel needs only lse and D (both final before the dQ kernel starts), so it
         // runs beside the dQ kernel as SMs free up
         p.pdl_free = WIDE && MODE == BWDKV && r0 == 0 && dpoll_enabled();
@@ -1314,7 +1337,8 @@ bool tc32_supported(int64_t units, int64_t L, int64_t d, int64_t w, int64_t dil)
     const int64_t wc = w < L ? w : L;
     if (!(dil <= 256 && units * ((L + 127) / 128) < (1 << 30))) return false;
     if (wc <= 32) return d % 64 == 0 && d <= 512;
-    return (d == 64 || d == 128) && wide_steps(L, w, dil, d) > 0;
+    WideGeo g;
+    return (d == 64 || d == 128) && wide_geo(L, w, dil, d, g);
 }
 int tc32_fwd_launches(int64_t L, int64_t w, int64_t dil) { return band32_launches(L, dil); }
 int tc32_bwd_launches(int64_t L, int64_t w, int64_t dil) { return 2 * band32_launches(L, dil) + (tc32_wide(L, w) ? 1 : 0); }
