@@ -707,7 +707,8 @@ def main():
     if not args.no_extras and args.extra_steps > 0 and world == 1:
         others = {}
         for wl, odt in (("C2b", "bf16"), ("C2b", "f32"), ("C4d2", "bf16"), ("C4d4", "bf16"), ("C4d2", "f32"),
-                        ("C5_w32", "bf16"), ("C5_w256", "bf16"), ("C5_small", "bf16")):
+                        ("C5_w32", "bf16"), ("C5_w256", "bf16"), ("C5_small", "bf16"), ("C5_w32", "f32"),
+                        ("C5_w256", "f32")):
             if wl == args.workload:
                 continue
             oB, oH, oL, od, ow, odil = WORKLOADS[wl][:6]
