@@ -128,7 +128,9 @@ def _cp_worker(rank, world, port, shape, dtype, result_q):
                                                (3, (2, 2, 1500, 64, 32, 3), "bf16"),
                                                (2, (1, 2, 1200, 64, 100, 1), "bf16"),
                                                (2, (1, 2, 500, 64, 16, 2), "f32"),
-                                               (2, (1, 2, 800, 256, 32, 1), "f32")],   # fp32 tensor cores + dS tape
+                                               (2, (1, 2, 800, 256, 32, 1), "f32"),    # fp32 tensor cores + dS tape
+                                               (2, (1, 2, 1400, 64, 150, 1), "f32"),   # fp32 WIDE steps
+                                               (2, (1, 1, 1000, 128, 100, 1), "bf16")],  # d = 128 wide kernels
                          ids=lambda s: "x".join(map(str, s)) if isinstance(s, tuple) else str(s))
 def test_context_parallel_cuda(world, shape, dtype):
     ctx = mp.get_context("spawn")
