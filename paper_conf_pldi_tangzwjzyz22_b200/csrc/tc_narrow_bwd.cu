@@ -257,12 +257,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
         }
     } else if (warp == 10 || warp == 11) {   // ----------------------------- halo converters
         // the halo of the dS GEMM (NQ: K_h, NKV: Q_h) to fp16 in place.  Lane l of converter warp
-        // cw owns halo rows 64 i + 32 cw + l, i < 3 (whole 128-byte rows: no shuffles, no second
-        // read).  As soon as the TMA landed it loads its rows into registers, reduces each row's
-        // largest |value| and publishes 2^-f (hs_full); once the score GEMM has read the bf16 halo
-        // (s_full2) it writes the rows times 2^f as fp16; the output MMAs read them after cv_done.
-        // (Two passes over shared memory, or eight lanes per row with shuffle reductions, left
-        // this warp pair on the tile's critical path: tools/trace_narrow.py.)
+        // cw owns halo rows 64 i + 32 cw + l, i < 3 (whole 128-byte rows: no shuffles).  As soon
+        // as the TMA landed it reduces each row's largest |value| and publishes 2^-f (hs_full);
+        // once the score GEMM has read the bf16 halo (s_full2) it rewrites the rows times 2^f as
+        // fp16; the output MMAs read them after cv_done.  The row loops stay rolled and the
+        // second pass re-reads its rows from shared memory: holding all three rows in registers
+        // unrolled this role to ~880 instructions, which pushed the kernel's steady-state code
+        // past the 32 KB instruction cache (ncu: no_inst the top stall reason of every role).
         const int cw = warp - 10;
         constexpr int NR = NK / 64;     // rows per lane
         TileCursor cur(p.sc);
@@ -272,42 +273,42 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             if (lane == 0 && cw == 0) trace_ev(p, j, 14);
             uint8_t* hb = stages + (size_t)(j % NSTAGE) * STAGE + 2 * ABYTES;
             float* tab = hscale + (j & 1) * NK;
-            uint4 v[NR][8];
-            float sc[NR];
-#pragma unroll
+#pragma unroll 1
             for (int i = 0; i < NR; ++i) {
                 const int r = 64 * i + 32 * cw + lane;
+                uint4 v[8];
 #pragma unroll
                 for (int x = 0; x < 8; ++x)
-                    v[i][x] = *reinterpret_cast<const uint4*>(hb + r * 128 + ((x ^ (r & 7)) << 4));
-            }
-#pragma unroll
-            for (int i = 0; i < NR; ++i) {
+                    v[x] = *reinterpret_cast<const uint4*>(hb + r * 128 + ((x ^ (r & 7)) << 4));
                 uint32_t m = 0;
 #pragma unroll
                 for (int x = 0; x < 8; ++x)
-                    m = __vmaxu2(m, __vmaxu2(__vmaxu2(v[i][x].x & 0x7FFF7FFFu, v[i][x].y & 0x7FFF7FFFu),
-                                             __vmaxu2(v[i][x].z & 0x7FFF7FFFu, v[i][x].w & 0x7FFF7FFFu)));
+                    m = __vmaxu2(m, __vmaxu2(__vmaxu2(v[x].x & 0x7FFF7FFFu, v[x].y & 0x7FFF7FFFu),
+                                             __vmaxu2(v[x].z & 0x7FFF7FFFu, v[x].w & 0x7FFF7FFFu)));
                 m = max(m & 0xFFFFu, m >> 16);   // bf16 bits of the row's max |x|
                 const int f = m == 0 ? 0 : pow2_exp_fp16(int(m >> 7));
-                sc[i] = __uint_as_float((uint32_t)(127 + f) << 23);
-                tab[64 * i + 32 * cw + lane] = __uint_as_float((uint32_t)(127 - f) << 23);
+                tab[r] = __uint_as_float((uint32_t)(127 - f) << 23);
             }
             mbar_arrive(&hs_full[j & 1]);   // every lane releases its own table entries
             if (lane == 0 && cw == 0) trace_ev(p, j, 17);
             mbar_wait(&s_full2[j & 1], (j >> 1) & 1);   // the score GEMM has read the bf16 halo
-#pragma unroll
+#pragma unroll 1
             for (int i = 0; i < NR; ++i) {
                 const int r = 64 * i + 32 * cw + lane;
+                const float sc = __uint_as_float((254u << 23) - __float_as_uint(tab[r]));   // 2^f
+                uint4 v[8];
+#pragma unroll
+                for (int x = 0; x < 8; ++x)
+                    v[x] = *reinterpret_cast<const uint4*>(hb + r * 128 + ((x ^ (r & 7)) << 4));
 #pragma unroll
                 for (int x = 0; x < 8; ++x) {
-                    uint32_t* wv = reinterpret_cast<uint32_t*>(&v[i][x]);
+                    uint32_t* wv = reinterpret_cast<uint32_t*>(&v[x]);
 #pragma unroll
                     for (int y = 0; y < 4; ++y) {
                         const float2 f2 = __bfloat1622float2(*reinterpret_cast<__nv_bfloat162*>(&wv[y]));
-                        wv[y] = pack_f16x2(f2.x * sc[i], f2.y * sc[i]);
+                        wv[y] = pack_f16x2(f2.x * sc, f2.y * sc);
                     }
-                    *reinterpret_cast<uint4*>(hb + r * 128 + ((x ^ (r & 7)) << 4)) = v[i][x];
+                    *reinterpret_cast<uint4*>(hb + r * 128 + ((x ^ (r & 7)) << 4)) = v[x];
                 }
             }
             fence_proxy_async_smem();
