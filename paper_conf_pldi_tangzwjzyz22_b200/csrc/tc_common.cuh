@@ -112,6 +112,20 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) 
     }
 }
 
+// Non-blocking probe (mbarrier.test_wait): for an issuer that polls several hand-offs and
+// serves whichever completes first.
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+
 // Spin variant (no suspend-time hint): for single-thread MMA issuers whose handoffs are on the
 // critical path -- the hinted wait compiles to NANOSLEEP.SYNCS, whose wake-up after the phase
 // completes cost the fused backward's issuers ~200 clk per wait (tools/trace_fused.py).

@@ -324,13 +324,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             //   NQ:  dQ = dS K_h, A = dS in smem (K-major SW128: 64-key atoms of 16 KB), -> acc[i&1]
             //   NKV: dV = P^T dO_h, dK = dS^T Q_h, A = packed operands over S^T in TMEM region
             //        i&1 (8 columns per step) -> acc (dV at 384, dK at 448)
-            auto out = [&](int i) {
+            auto acc_free_phase = [&](int i) -> int { return (MODE == NQ ? (i - 2) >> 1 : i - 1) & 1; };
+            auto acc_free_needed = [&](int i) -> bool { return MODE == NQ ? i >= 2 : i >= 1; };
+            // all of out(i)'s hand-offs complete (non-blocking)
+            auto out_ready = [&](int i) -> bool {
+                return mbar_test(p_done, i & 1) && mbar_test(&cv_done[i & 1], (i >> 1) & 1) &&
+                       (!acc_free_needed(i) || mbar_test(&acc_free[MODE == NQ ? (i & 1) : 0], acc_free_phase(i)));
+            };
+            auto out_issue = [&](int i) {
                 const int s = i % NSTAGE, b = MODE == NQ ? (i & 1) : 0;
                 const uint32_t st = smem_u32(stages + (size_t)s * STAGE);
-                mbar_wait(p_done, i & 1);
-                mbar_wait(&cv_done[i & 1], (i >> 1) & 1);
-                if (MODE == NQ ? i >= 2 : i >= 1)
-                    mbar_wait(&acc_free[b], (MODE == NQ ? (i - 2) >> 1 : i - 1) & 1);
                 tc_fence_after();
                 if (MODE == NQ) {
                     const uint32_t sb = st + 2 * ABYTES, sa = smem_u32(xbuf);
@@ -350,6 +353,12 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 mma_commit(&acc_full[b]);
                 mma_commit(&empty[s]);
             };
+            auto out = [&](int i) {
+                mbar_wait(p_done, i & 1);
+                mbar_wait(&cv_done[i & 1], (i >> 1) & 1);
+                if (acc_free_needed(i)) mbar_wait(&acc_free[MODE == NQ ? (i & 1) : 0], acc_free_phase(i));
+                out_issue(i);
+            };
             TileCursor cur(p.sc);
             Tile T;
             int j = 0;
@@ -364,11 +373,33 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                 const uint32_t rP = MODE == NQ ? tbase + 192u : tbase + 192u * ((j + 1) & 1);
                 trace_ev(p, j, 0);
                 if (j >= 1) mbar_wait(dp_free, (j - 1) & 1);
-                mbar_wait(&full1[s], ph);
-                tc_fence_after();
-                mma_ss_x4<2, 2>(rS, sdesc_sw128(st, 16, 1024), sdesc_sw128(st + 2 * ABYTES, 16, 1024), idS, 0);
-                trace_ev(p, j, 1);
-                if (MODE == NKV && j >= 1) out(j - 1);
+                // S(j) and out(j-1) in whichever order their inputs complete: out(j-1)'s
+                // completion frees the ring slot tile j+1 loads into, so it must not queue behind
+                // tile j's loads, and S(j) must not wait for the softmax of j-1 (dP(j) goes after
+                // both: in NKV it overwrites the operands out(j-1) reads)
+                {
+                    bool od = j == 0, sd = false;
+                    uint32_t spins = 0;
+                    uint64_t t0 = 0;
+                    while (!(od && sd)) {
+                        if (!od && out_ready(j - 1)) {
+                            out_issue(j - 1);
+                            od = true;
+                            trace_ev(p, j, 2);
+                        }
+                        if (!sd && mbar_test(&full1[s], ph)) {
+                            tc_fence_after();
+                            mma_ss_x4<2, 2>(rS, sdesc_sw128(st, 16, 1024), sdesc_sw128(st + 2 * ABYTES, 16, 1024),
+                                            idS, 0);
+                            sd = true;
+                            trace_ev(p, j, 1);
+                        }
+                        if (++spins < 4096u || (spins & 255u) != 0) continue;
+                        const uint64_t now = global_ns();
+                        if (t0 == 0) t0 = now;
+                        else if (now - t0 > FT_WATCHDOG_NS) __trap();
+                    }
+                }
                 mbar_wait(&full2[s], ph);
                 tc_fence_after();
                 mma_ss_x4<2, 2>(rP, sdesc_sw128(st + ABYTES, 16, 1024),
@@ -380,8 +411,6 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
                     mbar_wait(s_full, j & 1);
                     trace_ev(p, j, 13);
                 }
-                if (MODE == NQ && j >= 1) out(j - 1);
-                trace_ev(p, j, 2);
             }
             if (j >= 1) out(j - 1);
         }
