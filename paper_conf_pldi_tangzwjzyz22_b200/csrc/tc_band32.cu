@@ -243,8 +243,11 @@ struct AccUses {
     }
 };
 
-template <int MODE, bool WIDE>
+// XT: the dS tape (BWDQ writes it, BWDKV reads it) as its own instantiation, so neither kernel's
+// instruction working set carries the other path's code (p.xt is set iff XT)
+template <int MODE, bool WIDE, bool XT>
 __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_constant__ Params p) {
+    static_assert(!XT || (MODE != FWD && !WIDE), "tape instantiations: band BWDQ / BWDKV only");
     using C = Seq<MODE>;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw_u32 = smem_u32(smem_raw);
@@ -266,7 +269,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     // first halo row of step sb relative to m0 (normal mode: -w)
     auto koff = [&](int sb) -> int { return WIDE ? -w + (int)NK * sb : -w; };
 
-    if (MODE == BWDQ && p.xt) {   // clear this CTA's tile flags before BWDKV may launch
+    if (MODE == BWDQ && XT) {   // clear this CTA's tile flags before BWDKV may launch
         TileCursor cr(p.sc);
         Tile T;
         while (cr.next(p.sc, T))
@@ -297,7 +300,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
     }
     if (MODE == BWDQ || (MODE == FWD && p.lsepoll)) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 
-    const bool xt = MODE == BWDKV && p.xt;
+    constexpr bool xt = MODE == BWDKV && XT;
     const int nst = xt ? NST_XT : NST;
     const uint32_t slotb = xt ? SLOT_XT : SLOT;
     uint8_t* slots = smem;
@@ -886,7 +889,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
         while (!WIDE && cur.next(p.sc, T)) {
             const int Lr = T.Lr, m0 = T.m0, mrow = m0 + t, kb = m0 - w;
             const int64_t rowbase = (int64_t)T.u * p.L + T.r;
-            if (MODE == BWDKV && !p.xt) {
+            if (MODE == BWDKV && !XT) {
                 named_bar_sync(1, 128);   // everyone is done with the previous tile's columns
                 for (int n = t; n < NK; n += 128) {
                     const int mc = kb + n;
@@ -1014,7 +1017,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                             split2(dv[0], dv[1], pk[2 * g4], pl[2 * g4]);
                             split2(dv[2], dv[3], pk[2 * g4 + 1], pl[2 * g4 + 1]);
                             const int o = ob + 4 * g4;
-                            if (p.xt && mrow < Lr && o >= 0 && o < p.tsw) {
+                            if (XT && mrow < Lr && o >= 0 && o < p.tsw) {
                                 const size_t ro = ((size_t)(o >> 2) * p.grows + rowbase + (int64_t)mrow * p.dil) * 4;
                                 *reinterpret_cast<float4*>(p.tP + ro) = make_float4(pv[0], pv[1], pv[2], pv[3]);
                                 *reinterpret_cast<float4*>(p.tS + ro) = make_float4(dv[0], dv[1], dv[2], dv[3]);
@@ -1028,7 +1031,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_band32_kernel(const __grid_con
                 tc_fence_before();
                 warp_arrive(&p_full[j & 1]);
                 if (mrow < Lr) p.D[rowbase + (int64_t)mrow * p.dil] = D;
-                if (p.xt) {   // publish the tile's tape rows to BWDKV
+                if (XT) {   // publish the tile's tape rows to BWDKV
                     __threadfence();
                     named_bar_sync(2, 128);
                     if (t == 0) st_release_gpu(p.flags + rowbase + (int64_t)m0 * p.dil, 1u);
@@ -1229,10 +1232,14 @@ template <int MODE, bool WIDE>
 cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void* b2, const void* ob1,
                      const void* ob2, void* o1, void* o2, float* lse, float* D, const DsTape* tape, int64_t B,
                      int64_t H, int64_t L, int64_t d, int64_t w, int64_t dil, cudaStream_t st, int* launches) {
+    constexpr bool HAS_XT = MODE != FWD && !WIDE;
     static std::once_flag once;
     std::call_once(once, [] {
-        cudaFuncSetAttribute(tc_band32_kernel<MODE, WIDE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)(SMEM_BYTES > SMEM_BYTES_XT ? SMEM_BYTES : SMEM_BYTES_XT));
+        cudaFuncSetAttribute(tc_band32_kernel<MODE, WIDE, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)SMEM_BYTES);
+        if constexpr (HAS_XT)
+            cudaFuncSetAttribute(tc_band32_kernel<MODE, WIDE, HAS_XT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)(SMEM_BYTES > SMEM_BYTES_XT ? SMEM_BYTES : SMEM_BYTES_XT));
     });
     const int64_t wc = w < L ? w : L;
     WideGeo wg = {1, 0, KB};
@@ -1293,6 +1300,9 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
         const int64_t total = units * nr * tiles;
         dim3 grid((unsigned)(total < num_sms32() ? total : num_sms32()));
         const size_t smem = MODE == BWDKV && p.xt ? SMEM_BYTES_XT : SMEM_BYTES;
+        void (*kern)(Params) = tc_band32_kernel<MODE, WIDE, false>;
+        if constexpr (HAS_XT)
+            if (p.xt) kern = tc_band32_kernel<MODE, WIDE, HAS_XT>;
         sched_init(p.sc, L, dil, r0, nr, units, tiles, (int)grid.x);
         // lse hand-off: one launch of residues on each side (nres <= RES_PER_LAUNCH) -- the
         // dQ kernel's launch follows the forward's only launch
@@ -1310,9 +1320,9 @@ cudaError_t launch32(const void* a1, const void* b1, const void* a2, const void*
             at[0].val.programmaticStreamSerializationAllowed = 1;
             cfg.attrs = at;
             cfg.numAttrs = 1;
-            cudaLaunchKernelEx(&cfg, tc_band32_kernel<MODE, WIDE>, p);
+            cudaLaunchKernelEx(&cfg, kern, p);
         } else {
-            tc_band32_kernel<MODE, WIDE><<<grid, NTHREADS, smem, st>>>(p);
+            kern<<<grid, NTHREADS, smem, st>>>(p);
         }
         prof_mark(st);
         cudaError_t e = cudaGetLastError();
