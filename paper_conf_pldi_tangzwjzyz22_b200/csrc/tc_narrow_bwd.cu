@@ -25,7 +25,8 @@
 // turns the bf16 halo the dS GEMM multiplies (K_h for dQ, Q_h for dK) into fp16 row by row,
 // each row c scaled by 2^f_c so that its largest |value| lands in [2^14, 2^15), once the
 // score GEMM has read it, and publishes 2^-f_c; the softmax forms dS'_rc = dS_rc 2^-f_c,
-// scales its row r by 2^e_r (largest |dS'| in [2^14, 2^15)) and stores it as fp16.  The MMA
+// scales its row r by 2^e_r (largest |dS'| in [2^14, 2^15); NQ: an upper bound of it, so one
+// exchange between the row's column halves suffices) and stores it as fp16.  The MMA
 // then accumulates 2^e_r sum_c dS_rc x_c exactly up to fp16 rounding of the two operands, and
 // the drain multiplies the row by 2^-e_r.  Powers of two are exact, so a gradient scaled by
 // 2^16 (loss scaling) or 2^-24 gives the same relative error, with no overflow to inf and no
@@ -73,8 +74,9 @@ constexpr uint32_t STG = 32 * 128;
 constexpr uint32_t XBYTES = 3 * 16384;      // NQ: dS operand (fp16, 128 x 192); NKV: 8 x STG staging
 // per-tile scratch: NKV [2][2][NK] column lse / D; NQ [2][2][BM] D halves + [2][256] row lse
 constexpr int SCRATCH_FLOATS = 2 * 2 * BM + 2 * 256 > 2 * 2 * NK ? 2 * 2 * BM + 2 * 256 : 2 * 2 * NK;
-// halo row scales 2^-f_c [2][NK] and the two halves' row maxima of |dS'| [2][2][BM]
-constexpr int SCALE_FLOATS = 2 * NK + 2 * 2 * BM;
+// halo row scales 2^-f_c [2][NK] and the two halves' row maxima [2][2][BM] (NKV: of |dS'|; NQ:
+// of P 2^-f |dP|, then of P 2^-f [2][2][BM])
+constexpr int SCALE_FLOATS = 2 * NK + 2 * 2 * 2 * BM;
 constexpr size_t SMEM_BYTES = 1024 + (size_t)NSTAGE * STAGE + XBYTES + (SCRATCH_FLOATS + SCALE_FLOATS) * 4 + 256;
 static_assert(SMEM_BYTES <= 232448, "shared memory plan");
 constexpr float LOG2E = 1.4426950408889634f;
@@ -588,48 +590,49 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc_narrow_bwd_kernel(const __grid
             if (tr) trace_ev(p, j, 5);
             uint32_t pk[24], pk2[24];
             if (MODE == NQ) {
+                // One exchange between the row's two column halves: the D parts, and for the row
+                // scale the bound max_c |dS'_c| <= max_c P 2^-f_c |dP_c| + max_c P 2^-f_c |D| (dS' =
+                // P (dP - D) 2^-f_c).  The bound can exceed the true maximum (by cancellation in
+                // dP - D), which only moves the fp16 values down by powers of two: a normal fp16
+                // value keeps its 11 bits (a second exchange for the exact maximum cost more).
+                mbar_wait_sleep(&hs_full[j & 1], (j >> 1) & 1);
+                const float* tab = hscale + (j & 1) * NK + c0;
                 float dpart[4] = {0.f, 0.f, 0.f, 0.f};
+                float am = 0.f, bm = 0.f;
 #pragma unroll
                 for (int e = 0; e < 48; e += 2) {   // packed f32x2 pairs (FFMA2)
                     float a0, a1;
                     ffma2_bc(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), LOG2E, -lse2, a0, a1);
                     const float p0 = ((bits >> e) & 1ull) ? fast_exp2(a0) : 0.f;
                     const float p1 = ((bits >> (e + 1)) & 1ull) ? fast_exp2(a1) : 0.f;
-                    rs[e] = __float_as_uint(p0);
-                    rs[e + 1] = __float_as_uint(p1);
                     const int q = e & 2;
                     ffma2(p0, p1, __uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), dpart[q], dpart[q + 1],
                           dpart[q], dpart[q + 1]);
+                    float t0, t1;
+                    fmul2(p0, p1, tab[e], tab[e + 1], t0, t1);   // exact: 2^-f_c
+                    rs[e] = __float_as_uint(t0);
+                    rs[e + 1] = __float_as_uint(t1);
+                    am = fmaxf(am, fmaxf(t0 * fabsf(__uint_as_float(rd[e])), t1 * fabsf(__uint_as_float(rd[e + 1]))));
+                    bm = fmaxf(bm, fmaxf(t0, t1));
                 }
                 float* dxb = dx + (j & 1) * 2 * BM;
+                float* mxb = mxh + (j & 1) * 2 * BM;
+                float* mbb = mxh + 2 * 2 * BM + (j & 1) * 2 * BM;
                 dxb[h * BM + t] = (dpart[0] + dpart[1]) + (dpart[2] + dpart[3]);
-                named_bar_sync(1 + wq, 64);   // both halves posted their D part
+                mxb[h * BM + t] = am;
+                mbb[h * BM + t] = bm;
+                named_bar_sync(1 + wq, 64);   // both halves posted their parts
                 if (tr) trace_ev(p, j, 7);
                 const float Dv = dxb[t] + dxb[BM + t];
-                // dS' = P (dP - D) 2^-f_c (halo row scales), then this row's power of two
-                mbar_wait_sleep(&hs_full[j & 1], (j >> 1) & 1);
-                const float* tab = hscale + (j & 1) * NK + c0;
-                float mx = 0.f;
+                float up, down;
+                row_pow2(fmaxf(mxb[t], mxb[BM + t]) + fmaxf(mbb[t], mbb[BM + t]) * fabsf(Dv), up, down);
+                cs.rsc = down;
 #pragma unroll
-                for (int e = 0; e < 48; e += 2) {
+                for (int e = 0; e < 48; e += 2) {   // dS' 2^e = (P 2^-f_c) (dP - D) 2^e
                     float q0, q1, r0, r1;
                     ffma2_bc(__uint_as_float(rd[e]), __uint_as_float(rd[e + 1]), 1.f, -Dv, q0, q1);
                     fmul2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), q0, q1, r0, r1);
-                    fmul2(r0, r1, tab[e], tab[e + 1], r0, r1);
-                    rs[e] = __float_as_uint(r0);
-                    rs[e + 1] = __float_as_uint(r1);
-                    mx = fmaxf(mx, fmaxf(fabsf(r0), fabsf(r1)));
-                }
-                float* mxb = mxh + (j & 1) * 2 * BM;
-                mxb[h * BM + t] = mx;
-                named_bar_sync(1 + wq, 64);   // both halves posted their row max
-                float up, down;
-                row_pow2(fmaxf(mxb[t], mxb[BM + t]), up, down);
-                cs.rsc = down;
-#pragma unroll
-                for (int e = 0; e < 48; e += 2) {
-                    float r0, r1;
-                    fmul2(__uint_as_float(rs[e]), __uint_as_float(rs[e + 1]), up, up, r0, r1);
+                    fmul2(r0, r1, up, up, r0, r1);
                     pk[e / 2] = pack_f16x2(r0, r1);
                 }
                 // the dS buffer is free once out(j-1) completed
