@@ -899,3 +899,33 @@ def test_mixed_side_stream_and_graph(ft, shape):
     torch.cuda.synchronize()
     for a, b in zip((out, lse, dq, dk, dv), want):
         assert torch.equal(a, b)
+
+
+# Cancelling rows: every key's V row is the same vector, so dP_rc = dO_r . v for all c and
+# dS = P (dP - D) vanishes up to rounding (dq, dk ~ 0) while dv = sum P^T dO does not.  The
+# narrow dQ kernel's power-of-two row scale comes from an upper bound of max |dS'| (reading A10),
+# which here exceeds the true maximum by ~2^24: the result must stay finite and within tolerance.
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_cancelling_rows(ft, dtype):
+    sh = WinAttnShape(1, 4, 4096, 64, 32, 1)
+    x = make_inputs(sh, 21, dtype)
+    dev = torch.device("cuda:0")
+    v = x["v"][:, :, :1, :].expand_as(x["v"]).contiguous()
+    v64 = v.double().numpy()
+    ro, rl = oracle.fwd(x["q64"], x["k64"], v64, sh.w, sh.dilation)
+    rdq, rdk, rdv = oracle.bwd(x["q64"], x["k64"], v64, ro, rl, x["dout64"], sh.w, sh.dilation)
+    q, k, vd, g = x["q"].to(dev), x["k"].to(dev), v.to(dev), x["dout"].to(dev)
+    out, lse = ft.fwd(q, k, vd, sh.w, sh.dilation)
+    dq, dk, dv = ft.bwd(q, k, vd, out, lse, g, sh.w, sh.dilation)
+    torch.cuda.synchronize()
+    # dq, dk are rounding residues on both sides (the oracle's ~1e-16, fp32's ~1e-7 of the terms
+    # P |dP| |k| that cancel): bf16 takes its usual bound; fp32 an absolute 1e-4 of the terms' scale
+    # (a relative bound against the oracle's residue would be meaningless)
+    terms = float(np.abs(np.einsum("bhld,bhld->bhl", x["dout64"], v64)).max() * np.abs(x["k64"]).max())
+    for name, got, ref in (("out", out, ro), ("dq", dq, rdq), ("dk", dk, rdk), ("dv", dv, rdv)):
+        got = got.double().cpu().numpy()
+        assert np.isfinite(got).all(), name
+        if dtype == "f32" and name in ("dq", "dk"):
+            assert np.abs(got - ref).max() <= 1e-4 * terms, (name, np.abs(got - ref).max(), terms)
+        else:
+            compare(name, got, ref, dtype)
